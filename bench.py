@@ -1,0 +1,416 @@
+#!/usr/bin/env python
+"""bench.py -- ΣVP hot path on B200: VP-kernel jobs/s (+ HBM GB/s, speedup vs serial launch).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl svp|reference] [--config 5]
+
+A *step* is one pass of the whole hot path over one batch: every VP of the workload
+submits its job (svp_submit_batch -> Job Queue), then svp_flush runs Kernel Match ->
+Job Dispatcher -> Re-scheduler -> coalesced sm_100a kernels (interleaved streams) ->
+Profiler and returns when every output is in place.  Default workload = BASELINE.json
+config 5 (256 VPs: vecadd/SAXPY/hist256/Black-Scholes with ragged 64Ki-16Mi sizes +
+SGEMM 2048^3), the configuration the north-star target is stated on; at N GPUs the
+Job Dispatcher's LPT partition shards the 256 VPs over the ranks (no data-path
+collective: VPs share no data), so the scaling is strong (fixed total work).
+
+`value` is device-timed (CUDA events on the stream the library joins, max over ranks)
+with every VP's buffers resident in HBM; `e2e` is the same metric with pinned HOST
+buffers (H2D + D2H inside the timed region, Kernel Interleaving on).  The working set
+(~9 GB) is far larger than L2, so no L2 flush is needed between steps.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import workloads as W  # noqa: E402
+
+METRIC = "VP-kernel jobs/sec & HBM GB/s vs #VPs at 1/2/4/8 B200; speedup vs serial launch"
+CONFIG_NAMES = {
+    1: "cfg1: 2 VPs x vecadd 1Mi",
+    2: "cfg2: 16 VPs x SGEMM 512^3 fp32",
+    3: "cfg3: 64 VPs mixed vecadd/SAXPY/hist256/Black-Scholes 4Mi",
+    4: "cfg4: 64 VPs mixed, ragged 64Ki-16Mi + adversarial sizes",
+    5: "cfg5: 256 VPs mixed vecadd/SAXPY/hist256/Black-Scholes (ragged 64Ki-16Mi) + SGEMM 2048^3",
+}
+
+
+# ----------------------------------------------------------------------------- helpers
+def dist_setup():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if ws > 1:
+        import torch.distributed as dist
+        import torch
+        backend = "nccl" if torch.cuda.is_available() else "gloo"
+        if backend == "nccl":
+            torch.cuda.set_device(local)
+        dist.init_process_group(backend=backend)
+    return rank, ws, local
+
+
+def barrier(ws):
+    if ws > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def max_over_ranks(x: float, ws: int) -> float:
+    if ws == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def sum_over_ranks(x: float, ws: int) -> float:
+    if ws == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return float(t.item())
+
+
+def my_specs(specs, rank, ws):
+    """Job Dispatcher across ranks: the same kernel-stratified LPT every rank computes."""
+    if ws == 1:
+        return list(specs)
+    from paper_conf_dac_jungc15_b200 import svp
+    classes = [W.KERNELS.index(s.kernel) for s in specs]
+    costs = [s.algorithmic_bytes() / 6.5e12 + s.flops() / 60e12 for s in specs]
+    part = svp.lpt_partition(classes, costs, ws)
+    return [s for s, p in zip(specs, part) if p == rank]
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index: int):
+        self.p = None
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        try:
+            import torch
+            uuid = str(torch.cuda.get_device_properties(device_index).uuid)
+            ident = ["--id=GPU-" + uuid] if uuid and not uuid.startswith("GPU-") else (["--id=" + uuid] if uuid else [])
+        except Exception:
+            ident = []
+        try:
+            self.p = subprocess.Popen(["nvidia-smi"] + ident + ["--query-gpu=" + self.Q, "--format=csv,noheader,nounits",
+                                                                 "-lms", "50"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        time.sleep(0.06)
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        self.f.seek(0)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in self.f.read().splitlines():
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx.append(float(parts[2]))
+            except ValueError:
+                continue
+            for nm, val in zip(names, parts[5:9]):
+                if val.lower().startswith("active"):
+                    reasons.add(nm)
+        os.unlink(self.f.name)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "samples": len(sm),
+                "reasons": sorted(reasons)}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f), "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+def cpu_baseline(specs, inputs, label):
+    """The oracle as it stands on the host cores: a proportional sample of the workload
+    (the first min(#VPs, 5 x cores) VPs -- VP v runs kernel v % 5, so every class keeps
+    its share), each VP single-threaded, VPs spread over the cores."""
+    import oracle
+    cores = len(os.sched_getaffinity(0))
+    n = min(len(specs), 5 * cores)
+    sp, inp = specs[:n], inputs[:n]
+    oracle.build()
+    t0 = time.perf_counter()
+    oracle.run_jobs(sp, inp, threads=cores)
+    dt = time.perf_counter() - t0
+    kinds = {}
+    for s in sp:
+        kinds[s.kernel] = kinds.get(s.kernel, 0) + 1
+    return {"value": n / dt, "unit": "jobs/s", "cores": min(cores, n), "kind": "oracle",
+            "sample": f"{n} of {len(specs)} VPs of {label} ({', '.join(f'{v} {k}' for k, v in kinds.items())}), "
+                      f"one oracle pass, wall {dt:.2f} s"}
+
+
+# ----------------------------------------------------------------------------- arms
+def run_reference(args, rank, ws):
+    """--impl reference: the oracle (the paper's emulation baseline) on host cores."""
+    if rank != 0:
+        return
+    specs = W.config_specs(args.config, nvps=args.vps)
+    cores = len(os.sched_getaffinity(0))
+    n = min(len(specs), 5 * cores)
+    sample = specs[:n]
+    inputs = W.make_inputs_many(sample)
+    import oracle
+    oracle.build()
+    for _ in range(args.warmup):
+        oracle.run_jobs(sample, inputs, threads=cores)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.run_jobs(sample, inputs, threads=cores)
+    dt = time.perf_counter() - t0
+    value = n * args.steps / dt
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "jobs/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic",
+            "config": {"workload": CONFIG_NAMES[args.config], "vps": len(specs), "sample_vps": n,
+                       "parallelism": f"host threads x{min(cores, n)}"},
+            "cpu_baseline": {"value": value, "unit": "jobs/s", "cores": min(cores, n), "kind": "oracle",
+                             "sample": f"first {n} of {len(specs)} VPs (kernel = vp % 5) per step"},
+            "e2e": {"value": value, "unit": "jobs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def timed_steps(ctx, jobs, steps, stream):
+    import torch
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(steps):
+        ctx.submit_batch(jobs)
+        ctx.flush()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / 1e3
+
+
+def launches_per_flush(ctx):
+    n = 0
+    hist_id = ctx.kernel_ids.get("hist256")
+    for op in ctx.plan():
+        if op["kind"] == 1:
+            n += 1 + (1 if op["kernel"] == hist_id else 0)
+    return n
+
+
+def run_svp(args, rank, ws, local):
+    import torch
+    from paper_conf_dac_jungc15_b200 import svp
+    from paper_conf_dac_jungc15_b200.vpset import VPSet
+
+    torch.cuda.set_device(local)
+    stream = torch.cuda.current_stream()
+    all_specs = W.config_specs(args.config, nvps=args.vps)
+    specs = my_specs(all_specs, rank, ws)
+    t_gen = time.perf_counter()
+    inputs = W.make_inputs_many(specs)
+    t_gen = time.perf_counter() - t_gen
+
+    # ---------------- device-resident run (value)
+    ctx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, external_streams=[stream.cuda_stream],
+                      validate_ptrs=True)
+    vs = VPSet(ctx, specs, inputs, "device", device_ordinals=[local])
+    jobs = vs.job_list()
+    ctx.submit_batch(jobs)
+    ctx.flush()
+    torch.cuda.synchronize()
+    for _ in range(max(0, args.warmup - 1)):
+        ctx.submit_batch(jobs)
+        ctx.flush()
+    ctx.reset_profile()
+    barrier(ws)
+    clocks = Clocks(local)
+    dt = timed_steps(ctx, jobs, args.steps, stream)
+    clk = clocks.stop()
+    barrier(ws)
+    dt_max = max_over_ranks(dt, ws)
+    n_jobs_total = sum_over_ranks(len(specs), ws)
+    value = n_jobs_total * args.steps / dt_max
+    st = ctx.flush_stats()
+    kstats = {name: ctx.kernel_stats(kid) for name, kid in vs.kids.items()}
+    launches = launches_per_flush(ctx) * args.steps
+
+    # memory-bound kernels: algorithmic bytes / event-timed kernel time
+    mb_bytes = sum(k["bytes"] for n, k in kstats.items() if n != "sgemm")
+    mb_ns = sum(k["total_ns"] for n, k in kstats.items() if n != "sgemm")
+    hbm_gbs = mb_bytes / mb_ns if mb_ns else None
+    per_kernel = {}
+    for n, k in kstats.items():
+        if not k["launches"]:
+            continue
+        avg = k["total_ns"] / k["launches"]
+        if n == "sgemm":
+            per_kernel[n] = {"avg_launch_ms": avg / 1e6, "tflops": k["flops"] / k["total_ns"] / 1e3,
+                             "share_of_kernel_time": None}
+        else:
+            per_kernel[n] = {"avg_launch_ms": avg / 1e6, "gbs": k["bytes"] / k["total_ns"]}
+    tot_k = sum(k["total_ns"] for k in kstats.values())
+    for n in per_kernel:
+        per_kernel[n]["share_of_kernel_time"] = kstats[n]["total_ns"] / tot_k if tot_k else None
+    peaks, peak_src = measured_peaks()
+    dom = max(kstats, key=lambda n: kstats[n]["total_ns"])
+    dk = kstats[dom]
+    if dom == "sgemm":
+        sm_mhz = float(peaks.get("sm_max_mhz", 1965.0))
+        peak = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12
+        achieved = (dk["flops"] / dk["launches"]) / (dk["total_ns"] / dk["launches"]) / 1e3
+        roof = {"kernel": "sgemm_ffma (k_sgemm_ffma)", "bound": "alu", "achieved": achieved, "peak": peak,
+                "unit": "TFLOP/s", "frac": achieved / peak, "traffic": None,
+                "peak_source": f"derived: 148 SM x 128 FP32 lanes x 2 x {sm_mhz:.0f} MHz (sm_max_mhz, {peak_src})"}
+    else:
+        peak = float(peaks["hbm_gbs"])
+        achieved = (dk["bytes"] / dk["launches"]) / (dk["total_ns"] / dk["launches"])
+        roof = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": None, "peak_source": f"hbm_gbs ({peak_src})"}
+    prof_path = os.path.join(ROOT, "profiles", "traffic_r01.json")
+    if os.path.exists(prof_path):
+        try:
+            tr = json.load(open(prof_path))
+            if dom in tr:
+                roof["traffic"] = tr[dom]
+        except Exception:
+            pass
+
+    # ---------------- serial baselines on the same GPU, same buffers, same kernels
+    serial = {}
+    if not args.no_serial:
+        for name, kw in (("B1_serial_sync", dict(coalesce=False, interleave=False, sync_each_job=True)),
+                         ("B2_serial_async", dict(coalesce=False, interleave=False))):
+            sctx = svp.Context(num_gpus=1, device_ids=[local], external_streams=[stream.cuda_stream], **kw)
+            for k in vs.kids:
+                sctx.register_kernel(k)
+            ks = max(2, args.steps // 5)
+            sctx.submit_batch(jobs)
+            sctx.flush()
+            barrier(ws)
+            sdt = max_over_ranks(timed_steps(sctx, jobs, ks, stream), ws)
+            serial[name] = {"value": n_jobs_total * ks / sdt, "unit": "jobs/s", "steps": ks,
+                            "ms_per_step": sdt / ks * 1e3}
+            sctx.close()
+    ctx.close()
+    del vs
+    torch.cuda.empty_cache()
+
+    # ---------------- e2e: pinned host buffers, copies inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        hctx = svp.Context(num_gpus=1, device_ids=[local], external_streams=[stream.cuda_stream],
+                           arena_bytes=args.arena_gb << 30)
+        hvs = VPSet(hctx, specs, inputs, "host")
+        hjobs = hvs.job_list()
+        hctx.submit_batch(hjobs)
+        hctx.flush()
+        hst = hctx.flush_stats()
+        barrier(ws)
+        ks = args.e2e_steps or max(2, min(args.steps, 5))
+        edt = max_over_ranks(timed_steps(hctx, hjobs, ks, stream), ws)
+        e2e = {"value": n_jobs_total * ks / edt, "unit": "jobs/s",
+               "h2d_bytes_per_step": int(sum_over_ranks(hst["h2d_bytes"], ws)),
+               "d2h_bytes_per_step": int(sum_over_ranks(hst["d2h_bytes"], ws)),
+               "steps": ks, "ms_per_step": edt / ks * 1e3, "chunks": int(hst["chunks"]),
+               "api": "svp_submit_batch + svp_flush, HOST_PINNED buffers (H2D/D2H staged + interleaved)"}
+        hctx.close()
+        del hvs
+
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu:
+        cpu = cpu_baseline(specs, inputs, CONFIG_NAMES[args.config])
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "jobs/s", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": dt_max / args.steps * 1e3, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": CONFIG_NAMES[args.config], "vps": len(all_specs),
+                       "residency": "device (HBM)", "parallelism": f"dp{ws}: VPs sharded by the Job Dispatcher (LPT)",
+                       "l2": "inputs > L2: %.1f GB of VP buffers touched per step" %
+                             (sum(s.algorithmic_bytes() for s in all_specs) / 1e9)},
+            "clocks": clk, "e2e": e2e, "gpu_launches": int(sum_over_ranks(launches, ws)),
+            "roofline": roof, "cpu_baseline": cpu,
+            "hbm_gbs_membound": hbm_gbs,
+            "hbm_frac_membound": (hbm_gbs / float(peaks["hbm_gbs"])) if hbm_gbs else None,
+            "elements_per_s": sum(s.n for s in all_specs) * args.steps / dt_max,
+            "speedup_vs_serial": {k: value / v["value"] for k, v in serial.items()},
+            "serial": serial, "per_kernel": per_kernel,
+            "flush": {"host_plan_us": st["host_plan_ns"] / 1e3, "host_issue_us": st["host_issue_ns"] / 1e3,
+                      "host_total_us": st["host_total_ns"] / 1e3, "device_ms": st["device_ns"] / 1e6,
+                      "groups": int(st["groups"]), "launch_ops": int(st["launches"])},
+            "parity": "tests/test_gpu_parity.py (full-size configs vs oracle; not re-run here)",
+            "setup_s": {"input_generation": t_gen},
+        }
+        print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="svp", choices=["svp", "reference"])
+    ap.add_argument("--config", type=int, default=5)
+    ap.add_argument("--vps", type=int, default=None)
+    ap.add_argument("--e2e-steps", type=int, default=0)
+    ap.add_argument("--arena-gb", type=int, default=8)
+    ap.add_argument("--no-serial", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        print("warning: --warmup < 3 violates the timing rules; using 3", file=sys.stderr)
+        args.warmup = 3
+    if args.impl == "reference":
+        # rank 0 alone runs the oracle arm; other ranks exit without work or rendezvous
+        rank, ws = int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1"))
+        run_reference(args, rank, ws)
+        return
+    rank, ws, local = dist_setup()
+    run_svp(args, rank, ws, local)
+    if ws > 1:
+        import torch.distributed as dist
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,251 @@
+/*
+ * svp.h -- C-ABI of libsvp, the B200-native SigmaVP multiplexer.
+ *
+ * SigmaVP (Jung & Carloni, DAC'15) lets many virtual platforms (VPs) -- simulated
+ * embedded devices with virtual GPUs -- run their GPU kernels on the host GPUs
+ * ("multiplexes the host GPUs ... by using separate streams for each VP",
+ * PAPER.md L199-206, §2).  The host side (Fig 2, text L231-257) is
+ * a Job Queue fed by the VPs, a Kernel Match that finds identical kernel requests,
+ * a Re-scheduler that reorders jobs (Kernel Interleaving) and merges identical ones
+ * (Kernel Coalescing), a Job Dispatcher that invokes the physical GPUs, and a
+ * Profiler.  This header is that pipeline's boundary:
+ *
+ *   svp_init -> svp_register_kernel -> svp_submit* -> svp_flush -> svp_profile
+ *
+ * Conventions
+ *  - Every function returns svp_status (SVP_OK == 0, negative on error) unless noted.
+ *    No C++ exception crosses the ABI.  svp_last_error() returns a thread-local,
+ *    human-readable message for the last failing call on the calling thread.
+ *  - A CUDA failure inside svp_flush returns SVP_E_CUDA and makes the context
+ *    "sticky-errored": every later call except svp_finalize / svp_last_error /
+ *    svp_profile returns SVP_E_STATE.
+ *  - The library owns everything it creates (streams, events, tables, staging arena,
+ *    worker threads).  The caller owns every buffer passed in svp_buf.
+ *  - Pointers are plain host or device addresses; sizes are bytes unless noted.
+ *    No torch types appear here; PyTorch is only the caller's allocator.
+ */
+#ifndef SVP_H_
+#define SVP_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SVP_ABI_VERSION 1
+
+typedef int32_t svp_status;
+enum {
+    SVP_OK = 0,
+    SVP_E_INVAL = -1,       /* bad argument (null, size too small, wrong count/dir/residency) */
+    SVP_E_NOMEM = -2,       /* host/device/pinned allocation failed, or a job exceeds the arena */
+    SVP_E_CUDA = -3,        /* a CUDA runtime call failed; context becomes sticky-errored */
+    SVP_E_NOKERNEL = -4,    /* unknown kernel name or id */
+    SVP_E_STATE = -5,       /* context errored / finalized / flush re-entered */
+    SVP_E_TIMEOUT = -6,     /* flush watchdog expired (cfg.flush_timeout_ms) */
+    SVP_E_UNSUPPORTED = -7  /* valid request this build cannot run (e.g. sgemm K % 4 != 0) */
+};
+
+typedef struct svp_ctx svp_ctx; /* opaque */
+
+/* ------------------------------------------------------------------ configuration */
+enum { SVP_SGEMM_FFMA = 0, SVP_SGEMM_TF32 = 1 };
+
+typedef struct svp_config {
+    int32_t num_gpus;            /* GPUs to drive; 0 = all visible (dry_run: 0 -> 1)          */
+    const int32_t* device_ids;   /* optional [num_gpus] CUDA ordinals; NULL = 0..num_gpus-1   */
+    int32_t streams_per_gpu;     /* compute streams per GPU (>= 1); copies use 2 more streams */
+    int32_t coalesce;            /* 1: Kernel Coalescing; 0: one launch/job */
+    int32_t interleave;          /* 1: Kernel Interleaving: chunking,
+                                    Johnson order, H2D / compute / D2H on separate streams;
+                                    0: every op on one stream in submission order            */
+    int32_t max_chunks;          /* upper bound on chunks a group is split into (1..64)       */
+    uint64_t arena_bytes;        /* per-GPU device staging arena for host-resident buffers;
+                                    0 = 2 GiB.  Allocated lazily on first host-resident job.  */
+    int32_t profile_level;       /* 0: no events; 1: CUDA events around every op (per-VP
+                                    attribution, kernel stats)                                */
+    int32_t sync_each_job;       /* serial baseline B1: stream-synchronize after every job    */
+    int32_t dry_run;             /* 1: plan only -- no CUDA call at all, op times simulated
+                                    by the cost model (host-logic tests on CPU)               */
+    int32_t flush_timeout_ms;    /* 0 = wait forever; else watchdog -> SVP_E_TIMEOUT          */
+    int32_t validate_ptrs;       /* 1: svp_submit checks residency with cudaPointerGetAttributes
+                                    (device buffer on the VP's GPU, host buffer pinned)       */
+    void* const* external_streams; /* optional [num_gpus] caller cudaStream_t (e.g. torch's
+                                    current stream): flush work starts after the work already
+                                    queued on it, and it waits for the flush's last op.      */
+    /* cost model used for ordering/chunking before measurements exist (D8, PAPER.md
+       L272-275 "expected time for each invocation"); 0 = built-in B200 defaults      */
+    double hbm_gbps;             /* default 6552 (MEASURED_PEAKS.json hbm_gbs)                */
+    double pcie_gbps;            /* default 50 per direction                                  */
+    double ffma_tflops;          /* default 60                                                */
+    double launch_us;            /* default 4                                                 */
+} svp_config;
+
+/* Fill *cfg with defaults: num_gpus 0, 4 compute streams, coalesce 1, interleave 1,
+   max_chunks 8, profile_level 0, validate_ptrs 1, everything else 0. */
+void svp_config_default(svp_config* cfg);
+
+/* Create a context.  On success *out owns streams/events/threads for every GPU.
+   Errors: SVP_E_INVAL (null / bad values), SVP_E_CUDA (no device, bad ordinal). */
+svp_status svp_init(const svp_config* cfg, svp_ctx** out);
+
+/* Sync, free every library-owned resource, join worker threads.  Safe on an errored
+   context; ctx is invalid afterwards. */
+svp_status svp_finalize(svp_ctx* ctx);
+
+const char* svp_last_error(void);
+int32_t svp_abi_version(void);
+
+/* ------------------------------------------------------------------ kernels */
+/* Builtin guest kernels (BASELINE.json north_star):
+ *   "vecadd"        c = a + b                        args svp_args_vecadd   bufs [a IN f32, b IN f32, c OUT f32]
+ *   "saxpy"         y = fma(a, x, y)                 args svp_args_saxpy    bufs [x IN f32, y INOUT f32]
+ *   "hist256"       counts[b] = #{i: d[i]==b}        args svp_args_hist256  bufs [d IN u8, counts OUT u32[256]]
+ *                   (counts are overwritten)
+ *   "blackscholes"  call/put per option              args svp_args_bs       bufs [S IN, X IN, T IN, call OUT, put OUT] f32
+ *   "sgemm"         C = alpha A B + beta C, fp32 FFMA args svp_args_sgemm   bufs [A IN, B IN, C OUT (INOUT if beta != 0)]
+ *   "sgemm_tf32"    same, tcgen05 TF32 tensor cores  (own tolerance 2e-3)
+ * Registration is idempotent; the id is stable for the context's lifetime.
+ * Errors: SVP_E_NOKERNEL for an unknown name. */
+svp_status svp_register_kernel(svp_ctx* ctx, const char* name, int32_t* id_out);
+
+typedef struct svp_args_vecadd { uint64_t n; } svp_args_vecadd;
+typedef struct svp_args_saxpy { uint64_t n; float a; uint32_t _pad; } svp_args_saxpy;
+typedef struct svp_args_hist256 { uint64_t n; } svp_args_hist256;
+typedef struct svp_args_bs { uint64_t n; float R; float V; } svp_args_bs;
+typedef struct svp_args_sgemm { int32_t M, N, K; float alpha, beta; } svp_args_sgemm;
+
+/* ------------------------------------------------------------------ jobs */
+enum { SVP_DIR_IN = 1, SVP_DIR_OUT = 2, SVP_DIR_INOUT = 3 };
+enum { SVP_MEM_DEVICE = 0, SVP_MEM_HOST_PINNED = 1 };
+
+typedef struct svp_buf {
+    void* ptr;       /* device pointer (mem DEVICE, must be on svp_vp_device(vp)) or pinned host */
+    uint64_t bytes;  /* extent the caller guarantees valid; must cover what the kernel touches */
+    int32_t dir;     /* SVP_DIR_*; must match the kernel's buffer directions                     */
+    int32_t mem;     /* SVP_MEM_*                                                                 */
+} svp_buf;
+
+#define SVP_MAX_BUFS 5
+#define SVP_MAX_ARGS 64
+
+/* Queue one job of VP `vp` (0 <= vp < 2^20).  This is the in-process stand-in for the
+ * paper's VP -> IPC manager -> Job Queue path (Fig 2): it validates
+ * the job against the kernel descriptor, copies `args` and the buffer descriptors, and
+ * appends to the VP's FIFO (program order).  Asynchronous like cudaMemcpyAsync: the
+ * caller keeps every buffer valid and unmodified until svp_flush returns.  Pinned host
+ * buffers are staged through the device arena (the paper's physically-contiguous
+ * chunk, Fig 5); device buffers are used in place.  n = 0 is a legal no-op job.
+ * Thread-safe: many threads may submit concurrently.  *job_out (optional) gets a
+ * monotonically increasing job id.
+ * Errors: SVP_E_INVAL (bad vp/args/bufs/residency), SVP_E_NOKERNEL, SVP_E_UNSUPPORTED,
+ * SVP_E_STATE. */
+svp_status svp_submit(svp_ctx* ctx, int32_t vp, int32_t kernel, const void* args,
+                      size_t args_bytes, const svp_buf* bufs, int32_t nbufs, uint64_t* job_out);
+
+/* Batched submit (one lock, one validation pass) -- same semantics as n svp_submit
+ * calls in array order; on error nothing from the batch is queued. */
+typedef struct svp_job_desc {
+    int32_t vp;
+    int32_t kernel;
+    uint32_t args_bytes;
+    int32_t nbufs;
+    uint8_t args[SVP_MAX_ARGS];
+    svp_buf bufs[SVP_MAX_BUFS];
+} svp_job_desc;
+svp_status svp_submit_batch(svp_ctx* ctx, int32_t n, const svp_job_desc* jobs, uint64_t* job_ids_out);
+
+/* Drain every job submitted before the call: Kernel Match -> Job Dispatcher ->
+ * Re-scheduler -> per-GPU execution (coalesced launches over device segment tables,
+ * interleaved H2D/kernel/D2H streams) -> Profiler; blocks until every output is in
+ * the caller's buffers.  Not re-entrant (SVP_E_STATE if called concurrently).
+ * Errors: SVP_E_CUDA (sticky), SVP_E_TIMEOUT, SVP_E_NOMEM, SVP_E_STATE. */
+svp_status svp_flush(svp_ctx* ctx);
+
+/* ------------------------------------------------------------------ Job Dispatcher */
+/* The GPU (index into the context's device list, 0..num_gpus-1) that runs VP `vp`.
+ * Sticky: assigned on first use (least-loaded by estimated cost so far) or by
+ * svp_assign_vps, never moved afterwards -- the caller allocates device-resident VP
+ * buffers there. */
+svp_status svp_vp_device(svp_ctx* ctx, int32_t vp, int32_t* device_out);
+
+/* Pin n VPs to GPUs with kernel-stratified LPT: within each class
+ * (kernel id), VPs in decreasing cost go to the least-loaded GPU, so every GPU gets a
+ * share of every class.  Already-placed VPs keep their GPU.  devices_out[n] optional. */
+svp_status svp_assign_vps(svp_ctx* ctx, int32_t n, const int32_t* vps, const int32_t* classes,
+                          const double* costs, int32_t* devices_out);
+
+/* Pure function (no context, no CUDA): the same kernel-stratified LPT over G bins.
+ * Used by multi-process (one rank per GPU) runs so every rank computes the same
+ * partition without exchanging data.  out[n] receives the bin of each item. */
+svp_status svp_lpt_partition(int32_t n, const int32_t* classes, const double* costs, int32_t G,
+                             int32_t* out);
+
+/* ------------------------------------------------------------------ Profiler */
+/* Per-VP attribution of device-timed op durations (the profiler
+ * "acquires execution information such as ... the elapsed clock cycles"): an op's
+ * event-timed duration is split over its member VPs in proportion to their
+ * algorithmic bytes (FLOPs for SGEMM).  Needs profile_level >= 1.  vp = -1 returns
+ * device-wide totals (sum over VPs, plus op counts). */
+typedef struct svp_vp_profile {
+    uint64_t jobs;
+    double kernel_ns, h2d_ns, d2h_ns;
+    uint64_t bytes_kernel, bytes_h2d, bytes_d2h;
+    double flops;
+    uint64_t launches; /* vp = -1 only: kernel launches issued */
+} svp_vp_profile;
+svp_status svp_profile(svp_ctx* ctx, int32_t vp, svp_vp_profile* out);
+svp_status svp_reset_profile(svp_ctx* ctx);
+
+/* Aggregate per kernel id (profile_level >= 1): launches, summed event-timed kernel
+ * duration (ns), algorithmic bytes and FLOPs of those launches. */
+typedef struct svp_kernel_stats {
+    uint64_t launches;
+    double total_ns;
+    double bytes;
+    double flops;
+    double max_ns;
+} svp_kernel_stats;
+svp_status svp_kernel_stats_get(svp_ctx* ctx, int32_t kernel, svp_kernel_stats* out);
+
+/* Counters of the most recent flush. */
+typedef struct svp_flush_stats {
+    uint64_t jobs, groups, chunks, launches, levels;
+    uint64_t h2d_bytes, d2h_bytes, table_bytes, table_uploads;
+    double host_plan_ns;     /* match + dispatch + reschedule + table build      */
+    double host_issue_ns;    /* enqueueing copies/launches                        */
+    double host_total_ns;    /* whole svp_flush call                               */
+    double device_ns;        /* first-op start to last-op end (profile_level >= 1) */
+    double sim_makespan_ns;  /* cost-model makespan of the plan (always)           */
+    double sim_serial_ns;    /* cost-model time of the same ops run one at a time  */
+} svp_flush_stats;
+svp_status svp_flush_stats_get(svp_ctx* ctx, svp_flush_stats* out);
+
+/* ------------------------------------------------------------------ plan introspection */
+/* The last flush's plan, one entry per issued op in issue order (tests, tooling). */
+enum { SVP_OP_H2D = 0, SVP_OP_KERNEL = 1, SVP_OP_D2H = 2 };
+typedef struct svp_plan_op {
+    int32_t kind;       /* SVP_OP_* */
+    int32_t device;     /* GPU index                                      */
+    int32_t stream;     /* library stream index on that GPU               */
+    int32_t level;      /* program-order level (the level-th job of a VP)  */
+    int32_t kernel;     /* kernel id                                       */
+    int32_t group;      /* Kernel Match group index within the flush       */
+    int32_t chunk;      /* chunk index within the group                    */
+    int32_t nvps;       /* members (VPs) in this op                        */
+    uint64_t bytes;     /* copy bytes, or algorithmic kernel bytes          */
+    double flops;
+    double est_ns;      /* cost-model duration                              */
+    double sim_start_ns, sim_end_ns; /* cost-model schedule                */
+    double measured_ns; /* event-timed duration (profile_level >= 1), else -1 */
+} svp_plan_op;
+svp_status svp_plan_size(svp_ctx* ctx, int32_t* n_ops);
+/* vps_out (optional, capacity cap) receives the op's member VPs in segment order. */
+svp_status svp_plan_get(svp_ctx* ctx, int32_t i, svp_plan_op* op, int32_t* vps_out, int32_t cap);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SVP_H_ */

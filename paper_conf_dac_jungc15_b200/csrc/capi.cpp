@@ -1,0 +1,479 @@
+// capi.cpp -- the C-ABI entry points of libsvp (include/svp.h).
+//
+// This file is the boundary: argument checking, error codes, the thread-local error
+// message, context lifetime, and the Job Queue front end (svp_submit stands in for the
+// paper's VP -> IPC Manager -> Job Queue path, Fig 2).  The heavy
+// lifting is in scheduler.cpp (Kernel Match, Dispatcher, Re-scheduler) and
+// executor.cpp (per-GPU execution and the Profiler).
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <chrono>
+#include <new>
+
+#include "internal.h"
+
+namespace svp {
+
+static const bool kTf32Available = false;
+static thread_local std::string g_last_error;
+void set_error(const std::string& msg) { g_last_error = msg; }
+
+static const KernelDesc kKernels[] = {
+    {"", 0, 0, {0, 0, 0, 0, 0}, 0},
+    {"vecadd", K_VECADD, 3, {SVP_DIR_IN, SVP_DIR_IN, SVP_DIR_OUT, 0, 0}, sizeof(svp_args_vecadd)},
+    {"saxpy", K_SAXPY, 2, {SVP_DIR_IN, SVP_DIR_INOUT, 0, 0, 0}, sizeof(svp_args_saxpy) - 4},
+    {"hist256", K_HIST256, 2, {SVP_DIR_IN, SVP_DIR_OUT, 0, 0, 0}, sizeof(svp_args_hist256)},
+    {"blackscholes", K_BLACKSCHOLES, 5, {SVP_DIR_IN, SVP_DIR_IN, SVP_DIR_IN, SVP_DIR_OUT, SVP_DIR_OUT},
+     sizeof(svp_args_bs)},
+    {"sgemm", K_SGEMM, 3, {SVP_DIR_IN, SVP_DIR_IN, SVP_DIR_OUT, 0, 0}, sizeof(svp_args_sgemm)},
+    {"sgemm_tf32", K_SGEMM_TF32, 3, {SVP_DIR_IN, SVP_DIR_IN, SVP_DIR_OUT, 0, 0}, sizeof(svp_args_sgemm)},
+};
+
+const KernelDesc* kernel_desc(int32_t id) {
+    if (id <= 0 || id >= K_COUNT) return nullptr;
+    return &kKernels[id];
+}
+const KernelDesc* kernel_by_name(const char* name) {
+    if (!name) return nullptr;
+    for (int i = 1; i < K_COUNT; ++i)
+        if (strcmp(kKernels[i].name, name) == 0) return &kKernels[i];
+    return nullptr;
+}
+
+}  // namespace svp
+
+using namespace svp;
+
+#define SVP_TRY_BEGIN try {
+#define SVP_TRY_END                                  \
+    }                                                \
+    catch (const std::bad_alloc&) {                  \
+        set_error("out of host memory");             \
+        return SVP_E_NOMEM;                          \
+    }                                                \
+    catch (const std::exception& e) {                \
+        set_error(std::string("internal: ") + e.what()); \
+        return SVP_E_STATE;                          \
+    }                                                \
+    catch (...) {                                    \
+        set_error("internal: unknown exception");    \
+        return SVP_E_STATE;                          \
+    }
+
+static svp_status check_ctx(svp_ctx* h) {
+    if (!h) {
+        set_error("null context");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    if (c->sticky != SVP_OK) {
+        set_error("context is sticky-errored: " + c->sticky_msg);
+        return SVP_E_STATE;
+    }
+    return SVP_OK;
+}
+
+extern "C" {
+
+const char* svp_last_error(void) { return g_last_error.c_str(); }
+int32_t svp_abi_version(void) { return SVP_ABI_VERSION; }
+
+void svp_config_default(svp_config* cfg) {
+    if (!cfg) return;
+    memset(cfg, 0, sizeof(*cfg));
+    cfg->num_gpus = 0;
+    cfg->streams_per_gpu = 4;
+    cfg->coalesce = 1;
+    cfg->interleave = 1;
+    cfg->max_chunks = 8;
+    cfg->profile_level = 0;
+    cfg->validate_ptrs = 1;
+}
+
+svp_status svp_init(const svp_config* cfg, svp_ctx** out) {
+    SVP_TRY_BEGIN
+    if (!cfg || !out) {
+        set_error("svp_init: null cfg/out");
+        return SVP_E_INVAL;
+    }
+    *out = nullptr;
+    if (cfg->num_gpus < 0 || cfg->num_gpus > 64 || cfg->streams_per_gpu < 1 || cfg->streams_per_gpu > 32 ||
+        cfg->max_chunks < 1 || cfg->max_chunks > 64 || cfg->profile_level < 0 || cfg->profile_level > 2 ||
+        cfg->flush_timeout_ms < 0) {
+        set_error("svp_init: config value out of range");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = new Ctx();
+    c->cfg = *cfg;
+    c->cfg.device_ids = nullptr;
+    c->cfg.external_streams = nullptr;
+    if (cfg->hbm_gbps > 0) c->cost.hbm_Bps = cfg->hbm_gbps * 1e9;
+    if (cfg->pcie_gbps > 0) c->cost.pcie_Bps = cfg->pcie_gbps * 1e9;
+    if (cfg->ffma_tflops > 0) c->cost.ffma_flops = cfg->ffma_tflops * 1e12;
+    if (cfg->launch_us > 0) c->cost.launch_ns = cfg->launch_us * 1e3;
+    if (cfg->arena_bytes == 0) c->cfg.arena_bytes = 2ull << 30;
+
+    if (cfg->dry_run) {
+        c->ngpu = cfg->num_gpus > 0 ? cfg->num_gpus : 1;
+        for (int i = 0; i < c->ngpu; ++i) c->device_ids.push_back(cfg->device_ids ? cfg->device_ids[i] : i);
+    } else {
+        c->ngpu = cfg->num_gpus;  // 0 -> executor fills from cudaGetDeviceCount
+        if (cfg->device_ids)
+            for (int i = 0; i < cfg->num_gpus; ++i) c->device_ids.push_back(cfg->device_ids[i]);
+        // external streams are read by the executor at creation time
+        c->cfg.external_streams = cfg->external_streams;
+        svp_status st = SVP_OK;
+        c->exec = executor_create(c, &st);
+        c->cfg.external_streams = nullptr;
+        if (!c->exec) {
+            delete c;
+            return st == SVP_OK ? SVP_E_CUDA : st;
+        }
+    }
+    c->dev_load.assign(c->ngpu, 0.0);
+    *out = reinterpret_cast<svp_ctx*>(c);
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+svp_status svp_finalize(svp_ctx* h) {
+    SVP_TRY_BEGIN
+    if (!h) {
+        set_error("null context");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    if (c->exec) executor_destroy(c->exec);
+    delete c;
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+svp_status svp_register_kernel(svp_ctx* h, const char* name, int32_t* id_out) {
+    SVP_TRY_BEGIN
+    svp_status st = check_ctx(h);
+    if (st) return st;
+    const KernelDesc* d = kernel_by_name(name);
+    if (!d) {
+        set_error(std::string("unknown kernel '") + (name ? name : "(null)") + "'");
+        return SVP_E_NOKERNEL;
+    }
+    if (d->id == K_SGEMM_TF32 && !kTf32Available) {
+        set_error("sgemm_tf32: the tcgen05 TF32 kernel is not available in this build");
+        return SVP_E_UNSUPPORTED;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    c->registered[d->id] = true;
+    if (id_out) *id_out = d->id;
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+static svp_status submit_many(Ctx* c, int32_t n, const svp_job_desc* jd, const svp_job_desc* single_args_src,
+                              uint64_t* ids) {
+    (void)single_args_src;
+    std::vector<Job> jobs(n);
+    for (int i = 0; i < n; ++i) {
+        Job& j = jobs[i];
+        j.vp = jd[i].vp;
+        j.kernel = jd[i].kernel;
+        j.nbufs = jd[i].nbufs;
+        if (jd[i].args_bytes > SVP_MAX_ARGS || jd[i].nbufs < 0 || jd[i].nbufs > SVP_MAX_BUFS) {
+            set_error("svp_submit: args_bytes > 64 or nbufs out of range");
+            return SVP_E_INVAL;
+        }
+        memcpy(j.args, jd[i].args, jd[i].args_bytes);
+        const KernelDesc* d = kernel_desc(j.kernel);
+        if (d && jd[i].args_bytes < d->args_bytes) {
+            set_error(std::string("svp_submit: args too small for ") + d->name);
+            return SVP_E_INVAL;
+        }
+        for (int b = 0; b < j.nbufs; ++b) j.bufs[b] = jd[i].bufs[b];
+        svp_status st = validate_and_fill(c, &j);
+        if (st) return st;
+    }
+    std::lock_guard<std::mutex> lk(c->qmu);
+    for (int i = 0; i < n; ++i) {
+        jobs[i].id = c->next_job_id++;
+        if (ids) ids[i] = jobs[i].id;
+        c->queue.push_back(jobs[i]);
+    }
+    return SVP_OK;
+}
+
+svp_status svp_submit(svp_ctx* h, int32_t vp, int32_t kernel, const void* args, size_t args_bytes,
+                      const svp_buf* bufs, int32_t nbufs, uint64_t* job_out) {
+    SVP_TRY_BEGIN
+    svp_status st = check_ctx(h);
+    if (st) return st;
+    if ((!args && args_bytes) || args_bytes > SVP_MAX_ARGS || (!bufs && nbufs) || nbufs < 0 ||
+        nbufs > SVP_MAX_BUFS) {
+        set_error("svp_submit: bad args/bufs");
+        return SVP_E_INVAL;
+    }
+    svp_job_desc d;
+    memset(&d, 0, sizeof(d));
+    d.vp = vp;
+    d.kernel = kernel;
+    d.args_bytes = (uint32_t)args_bytes;
+    d.nbufs = nbufs;
+    if (args_bytes) memcpy(d.args, args, args_bytes);
+    for (int b = 0; b < nbufs; ++b) d.bufs[b] = bufs[b];
+    return submit_many(reinterpret_cast<Ctx*>(h), 1, &d, nullptr, job_out);
+    SVP_TRY_END
+}
+
+svp_status svp_submit_batch(svp_ctx* h, int32_t n, const svp_job_desc* jobs, uint64_t* ids) {
+    SVP_TRY_BEGIN
+    svp_status st = check_ctx(h);
+    if (st) return st;
+    if (n < 0 || (n && !jobs)) {
+        set_error("svp_submit_batch: bad n/jobs");
+        return SVP_E_INVAL;
+    }
+    return submit_many(reinterpret_cast<Ctx*>(h), n, jobs, nullptr, ids);
+    SVP_TRY_END
+}
+
+svp_status svp_flush(svp_ctx* h) {
+    SVP_TRY_BEGIN
+    svp_status st = check_ctx(h);
+    if (st) return st;
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    int expected = 0;
+    if (!c->flushing.compare_exchange_strong(expected, 1)) {
+        set_error("svp_flush: already flushing (not re-entrant)");
+        return SVP_E_STATE;
+    }
+    struct Guard {
+        Ctx* c;
+        ~Guard() { c->flushing.store(0); }
+    } guard{c};
+    auto t0 = std::chrono::steady_clock::now();
+    Flush f;
+    {
+        std::lock_guard<std::mutex> lk(c->qmu);
+        f.jobs.swap(c->queue);
+    }
+    memset(&c->fstats, 0, sizeof(c->fstats));
+    st = plan_flush(c, &f);
+    auto t1 = std::chrono::steady_clock::now();
+    if (st) {
+        c->last = std::move(f);
+        return st;
+    }
+    double makespan = 0, serial = 0;
+    simulate(c, &f, &makespan, &serial);
+    c->fstats.sim_makespan_ns = makespan;
+    c->fstats.sim_serial_ns = serial;
+    c->fstats.host_plan_ns = std::chrono::duration<double, std::nano>(t1 - t0).count();
+    if (c->exec && !f.ops.empty()) {
+        st = executor_run(c->exec, &f);
+        if (st == SVP_E_CUDA || st == SVP_E_TIMEOUT) {
+            c->sticky = st;
+            c->sticky_msg = executor_error(c->exec);
+            set_error(c->sticky_msg);
+        } else if (st) {
+            set_error(executor_error(c->exec));
+        }
+    }
+    auto t2 = std::chrono::steady_clock::now();
+    c->fstats.host_total_ns = std::chrono::duration<double, std::nano>(t2 - t0).count();
+    c->fstats.jobs = f.jobs.size();
+    c->fstats.groups = f.groups.size();
+    c->fstats.chunks = f.chunks.size();
+    c->fstats.levels = f.levels;
+    uint64_t launches = 0;
+    for (auto& op : f.ops) {
+        if (op.kind == SVP_OP_KERNEL) ++launches;
+        if (op.kind == SVP_OP_H2D) c->fstats.h2d_bytes += op.bytes;
+        if (op.kind == SVP_OP_D2H) c->fstats.d2h_bytes += op.bytes;
+    }
+    c->fstats.launches = launches;
+    c->last = std::move(f);
+    return st;
+    SVP_TRY_END
+}
+
+svp_status svp_vp_device(svp_ctx* h, int32_t vp, int32_t* device_out) {
+    SVP_TRY_BEGIN
+    svp_status st = check_ctx(h);
+    if (st) return st;
+    if (!device_out || vp < 0 || vp >= (1 << 20)) {
+        set_error("svp_vp_device: bad vp/out");
+        return SVP_E_INVAL;
+    }
+    *device_out = dispatch_vp(reinterpret_cast<Ctx*>(h), vp, 0.0);
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+svp_status svp_assign_vps(svp_ctx* h, int32_t n, const int32_t* vps, const int32_t* classes, const double* costs,
+                          int32_t* devices_out) {
+    SVP_TRY_BEGIN
+    svp_status st = check_ctx(h);
+    if (st) return st;
+    if (n < 0 || (n && (!vps || !classes || !costs))) {
+        set_error("svp_assign_vps: bad arguments");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    std::lock_guard<std::mutex> lk(c->dmu);
+    std::vector<int32_t> idx, cls;
+    std::vector<double> cst;
+    for (int i = 0; i < n; ++i) {
+        if (vps[i] < 0 || vps[i] >= (1 << 20)) {
+            set_error("svp_assign_vps: vp out of range");
+            return SVP_E_INVAL;
+        }
+        if (!c->vp_dev.count(vps[i])) {
+            idx.push_back(i);
+            cls.push_back(classes[i]);
+            cst.push_back(costs[i]);
+        }
+    }
+    std::vector<int32_t> out(idx.size());
+    lpt_stratified((int32_t)idx.size(), cls.data(), cst.data(), c->ngpu, c->dev_load.data(), out.data());
+    for (size_t k = 0; k < idx.size(); ++k) {
+        c->vp_dev[vps[idx[k]]] = out[k];
+        c->dev_load[out[k]] += cst[k];
+    }
+    if (devices_out)
+        for (int i = 0; i < n; ++i) devices_out[i] = c->vp_dev[vps[i]];
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+svp_status svp_lpt_partition(int32_t n, const int32_t* classes, const double* costs, int32_t G, int32_t* out) {
+    SVP_TRY_BEGIN
+    if (n < 0 || G < 1 || (n && (!classes || !costs || !out))) {
+        set_error("svp_lpt_partition: bad arguments");
+        return SVP_E_INVAL;
+    }
+    std::vector<double> load(G, 0.0);
+    lpt_stratified(n, classes, costs, G, load.data(), out);
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+svp_status svp_profile(svp_ctx* h, int32_t vp, svp_vp_profile* out) {
+    SVP_TRY_BEGIN
+    if (!h || !out) {
+        set_error("svp_profile: null argument");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    std::lock_guard<std::mutex> lk(c->pmu);
+    memset(out, 0, sizeof(*out));
+    const VpProfile* p = nullptr;
+    if (vp == -1) {
+        p = &c->prof_total;
+        out->launches = c->prof_launches;
+    } else {
+        auto it = c->prof.find(vp);
+        if (it == c->prof.end()) return SVP_OK;
+        p = &it->second;
+    }
+    out->jobs = p->jobs;
+    out->kernel_ns = p->kernel_ns;
+    out->h2d_ns = p->h2d_ns;
+    out->d2h_ns = p->d2h_ns;
+    out->bytes_kernel = p->bytes_kernel;
+    out->bytes_h2d = p->bytes_h2d;
+    out->bytes_d2h = p->bytes_d2h;
+    out->flops = p->flops;
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+svp_status svp_reset_profile(svp_ctx* h) {
+    SVP_TRY_BEGIN
+    if (!h) {
+        set_error("null context");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    std::lock_guard<std::mutex> lk(c->pmu);
+    c->prof.clear();
+    c->prof_total = VpProfile{};
+    c->prof_launches = 0;
+    for (auto& k : c->kstats) k = KStats{};
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+svp_status svp_kernel_stats_get(svp_ctx* h, int32_t kernel, svp_kernel_stats* out) {
+    SVP_TRY_BEGIN
+    if (!h || !out) {
+        set_error("null argument");
+        return SVP_E_INVAL;
+    }
+    if (!kernel_desc(kernel)) {
+        set_error("unknown kernel id");
+        return SVP_E_NOKERNEL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    std::lock_guard<std::mutex> lk(c->pmu);
+    const KStats& k = c->kstats[kernel];
+    out->launches = k.launches;
+    out->total_ns = k.total_ns;
+    out->bytes = k.bytes;
+    out->flops = k.flops;
+    out->max_ns = k.max_ns;
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+svp_status svp_flush_stats_get(svp_ctx* h, svp_flush_stats* out) {
+    if (!h || !out) {
+        set_error("null argument");
+        return SVP_E_INVAL;
+    }
+    *out = reinterpret_cast<Ctx*>(h)->fstats;
+    return SVP_OK;
+}
+
+svp_status svp_plan_size(svp_ctx* h, int32_t* n) {
+    if (!h || !n) {
+        set_error("null argument");
+        return SVP_E_INVAL;
+    }
+    *n = (int32_t)reinterpret_cast<Ctx*>(h)->last.ops.size();
+    return SVP_OK;
+}
+
+svp_status svp_plan_get(svp_ctx* h, int32_t i, svp_plan_op* op, int32_t* vps_out, int32_t cap) {
+    if (!h || !op) {
+        set_error("null argument");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    const Flush& f = c->last;
+    if (i < 0 || i >= (int32_t)f.ops.size()) {
+        set_error("svp_plan_get: index out of range");
+        return SVP_E_INVAL;
+    }
+    const Op& o = f.ops[i];
+    const Chunk& ch = f.chunks[o.chunk];
+    op->kind = o.kind;
+    op->device = o.device;
+    op->stream = o.stream;
+    op->level = ch.level;
+    op->kernel = ch.kernel;
+    op->group = ch.group;
+    op->chunk = ch.index;
+    op->nvps = (int32_t)ch.jobs.size();
+    op->bytes = o.bytes;
+    op->flops = o.flops;
+    op->est_ns = o.est_ns;
+    op->sim_start_ns = o.sim_start;
+    op->sim_end_ns = o.sim_end;
+    op->measured_ns = o.measured_ns;
+    if (vps_out)
+        for (int k = 0; k < (int)ch.jobs.size() && k < cap; ++k) vps_out[k] = f.jobs[ch.jobs[k]].vp;
+    return SVP_OK;
+}
+
+}  // extern "C"

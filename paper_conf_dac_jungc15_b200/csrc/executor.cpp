@@ -1,0 +1,636 @@
+// executor.cpp -- per-GPU execution of a flush plan, device tables, staging arena and
+// the Profiler.
+//
+//  * a5  segment / tile tables: built in pinned host memory, one H2D per GPU per flush
+//        (skipped when byte-identical to the table already resident on the device).
+//  * a6  H2D of host-resident inputs into the staging arena -- the paper's coalesced
+//        "physically-contiguous" chunk (Fig 5), 256-B aligned slots,
+//        element counts not padded.
+//  * a7  one coalesced launch per chunk (kernels/*.cu).
+//  * a8  D2H of each VP's outputs back to its own host buffer -- "the resulting data
+//        are properly divided to be copied ... back to the host memory addresses"
+//        (PAPER.md L303-306).
+//  * a9  Kernel Interleaving: H2D / compute / D2H ops on separate streams linked by
+//        events, so a chunk's copies overlap another chunk's kernel.
+//  * a10 Profiler: CUDA events bracket every op; an op's device time is attributed to
+//        its member VPs in proportion to algorithmic bytes (FLOPs for SGEMM).
+//        PAPER.md L253-257 (the profiler "acquires ... elapsed clock cycles").
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include <algorithm>
+#include <chrono>
+#include <thread>
+
+#include "internal.h"
+#include "launch.h"
+#include "tables.h"
+
+namespace svp {
+
+#define CK(call)                                                                              \
+    do {                                                                                      \
+        cudaError_t _e = (call);                                                              \
+        if (_e != cudaSuccess) {                                                              \
+            d.err = std::string(#call) + " -> " + cudaGetErrorName(_e) + ": " + cudaGetErrorString(_e); \
+            return SVP_E_CUDA;                                                                \
+        }                                                                                     \
+    } while (0)
+
+struct MapKey {
+    uint64_t a, b;
+    int32_t M, N, K, variant;
+    bool operator==(const MapKey& o) const {
+        return a == o.a && b == o.b && M == o.M && N == o.N && K == o.K && variant == o.variant;
+    }
+};
+struct MapKeyHash {
+    size_t operator()(const MapKey& k) const {
+        return std::hash<uint64_t>()(k.a * 1000003ull ^ k.b * 998244353ull ^ ((uint64_t)k.M << 40) ^
+                                     ((uint64_t)k.N << 20) ^ (uint64_t)k.K ^ ((uint64_t)k.variant << 62));
+    }
+};
+struct Maps2 {
+    alignas(64) uint8_t a[128];
+    alignas(64) uint8_t b[128];
+};
+
+struct Dev {
+    int ordinal = 0;
+    int idx = 0;
+    std::vector<cudaStream_t> streams;  // [0,S) compute, S = H2D, S+1 = D2H
+    cudaStream_t ext = nullptr;
+    std::vector<cudaEvent_t> dep_ev, t_ev;
+    cudaEvent_t ext_ev = nullptr, tbl_ev = nullptr;
+    std::vector<cudaEvent_t> end_ev;
+    uint8_t* arena = nullptr;
+    uint64_t arena_bytes = 0;
+    uint8_t* tbl_host = nullptr;
+    uint8_t* tbl_dev = nullptr;
+    size_t tbl_cap = 0;
+    std::vector<uint8_t> tbl_last;
+    LaunchLimits lim;
+    std::unordered_map<MapKey, Maps2, MapKeyHash> map_cache;
+    std::string err;
+    uint64_t table_uploads = 0;
+};
+
+struct Executor {
+    Ctx* c = nullptr;
+    std::vector<Dev> devs;
+    std::string err;
+};
+
+std::string executor_error(Executor* e) { return e->err; }
+
+static svp_status dev_setup(Dev& d, const svp_config& cfg, void* ext) {
+    CK(cudaSetDevice(d.ordinal));
+    CK(cudaFree(0));  // create / adopt the primary context
+    const int S = cfg.streams_per_gpu;
+    d.streams.resize(S + 2);
+    for (auto& s : d.streams) CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    d.ext = (cudaStream_t)ext;
+    CK(cudaEventCreateWithFlags(&d.ext_ev, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&d.tbl_ev, cudaEventDisableTiming));
+    d.end_ev.resize(S + 2);
+    for (auto& e : d.end_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    d.arena_bytes = cfg.arena_bytes;
+    CK(query_limits(&d.lim));
+    return SVP_OK;
+}
+
+static void dev_teardown(Dev& d) {
+    cudaSetDevice(d.ordinal);
+    for (auto& s : d.streams) if (s) cudaStreamSynchronize(s);
+    for (auto& s : d.streams) if (s) cudaStreamDestroy(s);
+    for (auto e : d.dep_ev) cudaEventDestroy(e);
+    for (auto e : d.t_ev) cudaEventDestroy(e);
+    for (auto e : d.end_ev) cudaEventDestroy(e);
+    if (d.ext_ev) cudaEventDestroy(d.ext_ev);
+    if (d.tbl_ev) cudaEventDestroy(d.tbl_ev);
+    if (d.arena) cudaFree(d.arena);
+    if (d.tbl_dev) cudaFree(d.tbl_dev);
+    if (d.tbl_host) cudaFreeHost(d.tbl_host);
+}
+
+Executor* executor_create(Ctx* c, svp_status* st) {
+    Executor* e = new Executor();
+    e->c = c;
+    int count = 0;
+    cudaError_t ce = cudaGetDeviceCount(&count);
+    if (ce != cudaSuccess || count == 0) {
+        e->err = std::string("no CUDA device: ") + cudaGetErrorString(ce);
+        set_error(e->err);
+        *st = SVP_E_CUDA;
+        delete e;
+        return nullptr;
+    }
+    if (c->ngpu == 0) c->ngpu = count;
+    if (c->device_ids.empty())
+        for (int i = 0; i < c->ngpu; ++i) c->device_ids.push_back(i);
+    e->devs.resize(c->ngpu);
+    for (int i = 0; i < c->ngpu; ++i) {
+        Dev& d = e->devs[i];
+        d.idx = i;
+        d.ordinal = c->device_ids[i];
+        if (d.ordinal < 0 || d.ordinal >= count) {
+            e->err = "device ordinal out of range";
+            set_error(e->err);
+            *st = SVP_E_INVAL;
+            executor_destroy(e);
+            return nullptr;
+        }
+        void* ext = c->cfg.external_streams ? c->cfg.external_streams[i] : nullptr;
+        if (dev_setup(d, c->cfg, ext) != SVP_OK) {
+            e->err = d.err;
+            set_error(e->err);
+            *st = SVP_E_CUDA;
+            executor_destroy(e);
+            return nullptr;
+        }
+    }
+    *st = SVP_OK;
+    return e;
+}
+
+void executor_destroy(Executor* e) {
+    if (!e) return;
+    for (auto& d : e->devs) dev_teardown(d);
+    delete e;
+}
+
+svp_status executor_check_ptr(Executor* e, const void* p, int32_t mem, int32_t device, std::string* why) {
+    cudaPointerAttributes at;
+    cudaError_t ce = cudaPointerGetAttributes(&at, p);
+    if (ce != cudaSuccess) {
+        cudaGetLastError();
+        *why = std::string("cudaPointerGetAttributes failed: ") + cudaGetErrorString(ce);
+        return SVP_E_INVAL;
+    }
+    if (mem == SVP_MEM_DEVICE) {
+        if (at.type != cudaMemoryTypeDevice && at.type != cudaMemoryTypeManaged) {
+            *why = "declared DEVICE but is not device memory";
+            return SVP_E_INVAL;
+        }
+        if (at.type == cudaMemoryTypeDevice && at.device != e->devs[device].ordinal) {
+            *why = "device buffer is on CUDA device " + std::to_string(at.device) + " but the VP runs on " +
+                   std::to_string(e->devs[device].ordinal) + " (see svp_vp_device)";
+            return SVP_E_INVAL;
+        }
+    } else {
+        if (at.type != cudaMemoryTypeHost) {
+            *why = "declared HOST_PINNED but is not page-locked host memory";
+            return SVP_E_INVAL;
+        }
+    }
+    return SVP_OK;
+}
+
+// ------------------------------------------------------------------ tables (a5)
+static int elem_size(int kernel, int b) { return (kernel == K_HIST256 && b == 0) ? 1 : 4; }
+static int tile_elems(int kernel) {
+    switch (kernel) {
+        case K_VECADD: return kVecaddTile;
+        case K_SAXPY: return kSaxpyTile;
+        case K_BLACKSCHOLES: return kBsTile;
+        case K_HIST256: return kHistTile;
+    }
+    return 0;
+}
+
+static size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+// Resolve the device address the kernel uses for every buffer of every job in the chunk.
+static void resolve_addresses(Dev& d, const Flush& f, Chunk& ch) {
+    ch.staged.clear();
+    uint64_t off = ch.arena_off;
+    for (int32_t ji : ch.jobs) {
+        const Job& j = f.jobs[ji];
+        for (int b = 0; b < SVP_MAX_BUFS; ++b) {
+            if (b >= j.nbufs) {
+                ch.staged.push_back(0);
+                continue;
+            }
+            if (j.bufs[b].mem == SVP_MEM_HOST_PINNED) {
+                ch.staged.push_back((uint64_t)(d.arena + off));
+                off += align_up(touched_bytes(j, b), 256);
+            } else {
+                ch.staged.push_back((uint64_t)j.bufs[b].ptr);
+            }
+        }
+    }
+}
+
+static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_t>& tbl) {
+    tbl.clear();
+    for (auto& ch : f.chunks) {
+        if (ch.device != d.idx) continue;
+        resolve_addresses(d, f, ch);
+        const bool gemm = ch.kernel == K_SGEMM || ch.kernel == K_SGEMM_TF32;
+        if (!gemm) {
+            ch.table_off = align_up(tbl.size(), 128);
+            tbl.resize(ch.table_off + ch.jobs.size() * sizeof(SegDesc));
+            SegDesc* seg = reinterpret_cast<SegDesc*>(tbl.data() + ch.table_off);
+            const int T = tile_elems(ch.kernel);
+            uint32_t tiles = 0;
+            for (size_t k = 0; k < ch.jobs.size(); ++k) {
+                const Job& j = f.jobs[ch.jobs[k]];
+                SegDesc s;
+                memset(&s, 0, sizeof(s));
+                int nalign = ch.kernel == K_HIST256 ? 1 : j.nbufs;  // counts need no alignment
+                uint64_t mis = ch.staged[k * SVP_MAX_BUFS] & 15;
+                bool co = true;
+                for (int b = 0; b < j.nbufs; ++b) {
+                    s.ptr[b] = ch.staged[k * SVP_MAX_BUFS + b];
+                    if (b < nalign && (s.ptr[b] & 15) != mis) co = false;
+                }
+                int es = elem_size(ch.kernel, 0);
+                if (mis % es) co = false;
+                s.n = j.n;
+                s.flags = co ? 0 : SEG_SCALAR;
+                s.shift = co ? (uint16_t)(mis / es) : 0;
+                s.f[0] = j.f0;
+                s.f[1] = j.f1;
+                s.tile_begin = tiles;
+                uint64_t nt = j.n ? (j.n + s.shift + T - 1) / T : 0;
+                if (tiles + nt >= (1ull << 31)) {
+                    d.err = "svp_flush: coalesced launch exceeds 2^31 tiles";
+                    return SVP_E_UNSUPPORTED;
+                }
+                tiles += (uint32_t)nt;
+                seg[k] = s;
+            }
+            ch.total_tiles = tiles;
+            ch.nsegs = (int32_t)ch.jobs.size();
+        } else {
+            const int variant = ch.kernel == K_SGEMM_TF32 ? 1 : 0;
+            const int BM = variant ? kTf32BM : kGemmBM, BN = variant ? kTf32BN : kGemmBN;
+            ch.maps_off = align_up(tbl.size(), 128);
+            size_t nj = ch.jobs.size();
+            ch.table_off = ch.maps_off + nj * 256;
+            tbl.resize(ch.table_off + nj * sizeof(GemmDesc));
+            uint32_t tiles = 0;
+            for (size_t k = 0; k < nj; ++k) {
+                const Job& j = f.jobs[ch.jobs[k]];
+                GemmDesc g;
+                memset(&g, 0, sizeof(g));
+                const float* A = (const float*)ch.staged[k * SVP_MAX_BUFS + 0];
+                const float* B = (const float*)ch.staged[k * SVP_MAX_BUFS + 1];
+                g.C = (float*)ch.staged[k * SVP_MAX_BUFS + 2];
+                g.M = j.M;
+                g.N = j.N;
+                g.K = j.K;
+                g.alpha = j.f0;
+                g.beta = j.f1;
+                g.tile_begin = tiles;
+                g.tiles_n = (uint32_t)((j.N + BN - 1) / BN);
+                uint64_t nt = (uint64_t)((j.M + BM - 1) / BM) * g.tiles_n;
+                if ((int64_t)j.M * j.N == 0) nt = 0;
+                tiles += (uint32_t)nt;
+                uint8_t* mp = tbl.data() + ch.maps_off + k * 256;
+                if (nt && j.K > 0) {
+                    MapKey key{(uint64_t)A, (uint64_t)B, j.M, j.N, j.K, variant};
+                    auto it = d.map_cache.find(key);
+                    if (it == d.map_cache.end()) {
+                        Maps2 m;
+                        if (encode_gemm_maps(m.a, m.b, A, B, j.M, j.N, j.K, variant) != 0) {
+                            d.err = "cuTensorMapEncodeTiled failed for an sgemm job";
+                            return SVP_E_CUDA;
+                        }
+                        if (d.map_cache.size() > 4096) d.map_cache.clear();
+                        it = d.map_cache.emplace(key, m).first;
+                    }
+                    memcpy(mp, it->second.a, 128);
+                    memcpy(mp + 128, it->second.b, 128);
+                } else {
+                    memset(mp, 0, 256);
+                }
+                memcpy(tbl.data() + ch.table_off + k * sizeof(GemmDesc), &g, sizeof(g));
+            }
+            ch.total_tiles = tiles;
+            ch.nsegs = (int32_t)nj;
+        }
+    }
+    (void)e;
+    return SVP_OK;
+}
+
+static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bool timing) {
+    while (pool.size() <= i) {
+        cudaEvent_t ev;
+        if (cudaEventCreateWithFlags(&ev, timing ? cudaEventDefault : cudaEventDisableTiming) != cudaSuccess)
+            return nullptr;
+        pool.push_back(ev);
+    }
+    (void)d;
+    return pool[i];
+}
+
+static cudaError_t launch_chunk(Dev& d, const Chunk& ch, cudaStream_t s) {
+    if (ch.total_tiles == 0) return cudaSuccess;
+    const uint8_t* base = d.tbl_dev;
+    auto grid_of = [&](int per_sm) { return (int)std::min<uint64_t>(ch.total_tiles, (uint64_t)d.lim.num_sms * per_sm); };
+    switch (ch.kernel) {
+        case K_VECADD:
+            return launch_vecadd((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
+                                 grid_of(d.lim.ew_blocks_per_sm), s);
+        case K_SAXPY:
+            return launch_saxpy((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
+                                grid_of(d.lim.ew_blocks_per_sm), s);
+        case K_BLACKSCHOLES:
+            return launch_blackscholes((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
+                                       grid_of(d.lim.bs_blocks_per_sm), s);
+        case K_HIST256:
+            return launch_hist256((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
+                                  grid_of(d.lim.hist_blocks_per_sm), s);
+        case K_SGEMM:
+            return launch_sgemm_ffma((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
+                                     ch.total_tiles, grid_of(d.lim.gemm_blocks_per_sm), s);
+        case K_SGEMM_TF32:
+            return launch_sgemm_tf32((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
+                                     ch.total_tiles, grid_of(1), s);
+    }
+    return cudaErrorInvalidValue;
+}
+
+// zero-work hist jobs still must overwrite counts: handled in the kernel launcher by
+// zeroing every segment (including n == 0 ones) before accumulating.
+static bool chunk_needs_launch(const Flush& f, const Chunk& ch) {
+    if (ch.total_tiles) return true;
+    for (int32_t ji : ch.jobs) {
+        const Job& j = f.jobs[ji];
+        if (j.kernel == K_HIST256) return true;
+        if ((j.kernel == K_SGEMM || j.kernel == K_SGEMM_TF32) && (int64_t)j.M * j.N > 0) return true;
+    }
+    return false;
+}
+
+static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
+    Ctx* c = e->c;
+    CK(cudaSetDevice(d.ordinal));
+    const bool prof = c->cfg.profile_level >= 1;
+    bool any = false;
+    uint64_t arena_need = 0;
+    for (auto& ch : f.chunks)
+        if (ch.device == d.idx) {
+            any = true;
+            arena_need = std::max(arena_need, ch.arena_off + ch.arena_len);
+        }
+    if (!any) return SVP_OK;
+    if (arena_need && !d.arena) {
+        cudaError_t ce = cudaMalloc(&d.arena, d.arena_bytes);
+        if (ce != cudaSuccess) {
+            cudaGetLastError();
+            d.err = "cannot allocate the staging arena (" + std::to_string(d.arena_bytes) + " B)";
+            d.arena = nullptr;
+            return SVP_E_NOMEM;
+        }
+    }
+    // ---- tables
+    std::vector<uint8_t> tbl;
+    svp_status st = build_tables(e, d, f, tbl);
+    if (st) return st;
+    auto t_issue0 = std::chrono::steady_clock::now();
+    if (d.ext) {
+        CK(cudaEventRecord(d.ext_ev, d.ext));
+        for (auto s : d.streams) CK(cudaStreamWaitEvent(s, d.ext_ev, 0));
+    }
+    bool upload = !tbl.empty() && (tbl.size() != d.tbl_last.size() || memcmp(tbl.data(), d.tbl_last.data(), tbl.size()));
+    if (upload) {
+        if (tbl.size() > d.tbl_cap) {
+            if (d.tbl_dev) CK(cudaFree(d.tbl_dev));
+            if (d.tbl_host) CK(cudaFreeHost(d.tbl_host));
+            d.tbl_dev = nullptr;
+            d.tbl_host = nullptr;
+            size_t cap = align_up(tbl.size() * 2, 1 << 16);
+            CK(cudaMalloc(&d.tbl_dev, cap));
+            CK(cudaHostAlloc(&d.tbl_host, cap, cudaHostAllocDefault));
+            d.tbl_cap = cap;
+        }
+        memcpy(d.tbl_host, tbl.data(), tbl.size());
+        CK(cudaMemcpyAsync(d.tbl_dev, d.tbl_host, tbl.size(), cudaMemcpyHostToDevice, d.streams[0]));
+        CK(cudaEventRecord(d.tbl_ev, d.streams[0]));
+        for (size_t s = 1; s < d.streams.size(); ++s) CK(cudaStreamWaitEvent(d.streams[s], d.tbl_ev, 0));
+        d.tbl_last.swap(tbl);
+        ++d.table_uploads;
+        c->fstats.table_uploads += 1;
+        c->fstats.table_bytes += d.tbl_last.size();
+    }
+    // ---- issue ops in plan order
+    size_t nt = 0;
+    std::vector<int> used(d.streams.size(), 0);
+    std::vector<int32_t> tstart(f.ops.size(), -1);
+    for (size_t i = 0; i < f.ops.size(); ++i) {
+        Op& o = f.ops[i];
+        if (o.device != d.idx) continue;
+        cudaStream_t s = d.streams[o.stream];
+        used[o.stream] = 1;
+        for (int32_t p : o.wait_ops) {
+            const Op& q = f.ops[p];
+            if (q.device != d.idx) continue;
+            CK(cudaStreamWaitEvent(s, d.dep_ev[p], 0));
+        }
+        if (prof) {
+            cudaEvent_t ev0 = pool_get(d, d.t_ev, 2 * nt, true), ev1 = pool_get(d, d.t_ev, 2 * nt + 1, true);
+            if (!ev0 || !ev1) {
+                d.err = "event allocation failed";
+                return SVP_E_CUDA;
+            }
+            CK(cudaEventRecord(ev0, s));
+            tstart[i] = (int32_t)nt;
+        }
+        Chunk& ch = f.chunks[o.chunk];
+        if (o.kind == SVP_OP_H2D || o.kind == SVP_OP_D2H) {
+            for (size_t k = 0; k < ch.jobs.size(); ++k) {
+                const Job& j = f.jobs[ch.jobs[k]];
+                for (int b = 0; b < j.nbufs; ++b) {
+                    if (j.bufs[b].mem != SVP_MEM_HOST_PINNED) continue;
+                    uint64_t bytes = touched_bytes(j, b);
+                    if (!bytes) continue;
+                    void* dev = (void*)ch.staged[k * SVP_MAX_BUFS + b];
+                    if (o.kind == SVP_OP_H2D && (j.bufs[b].dir & SVP_DIR_IN)) {
+                        // sgemm C with beta == 0 is OUT-only and not staged in
+                        CK(cudaMemcpyAsync(dev, j.bufs[b].ptr, bytes, cudaMemcpyHostToDevice, s));
+                    } else if (o.kind == SVP_OP_D2H && (j.bufs[b].dir & SVP_DIR_OUT)) {
+                        CK(cudaMemcpyAsync(j.bufs[b].ptr, dev, bytes, cudaMemcpyDeviceToHost, s));
+                    }
+                }
+            }
+        } else if (chunk_needs_launch(f, ch)) {
+            CK(launch_chunk(d, ch, s));
+        }
+        if (prof) {
+            CK(cudaEventRecord(d.t_ev[2 * nt + 1], s));
+            ++nt;
+        }
+        if (o.needs_event) {
+            cudaEvent_t ev = pool_get(d, d.dep_ev, i, false);
+            if (!ev) {
+                d.err = "event allocation failed";
+                return SVP_E_CUDA;
+            }
+            CK(cudaEventRecord(ev, s));
+        }
+        if (c->cfg.sync_each_job && o.last_of_job) CK(cudaStreamSynchronize(s));
+    }
+    // ---- join into the external stream, then wait (watchdog)
+    std::vector<cudaEvent_t> finals;
+    for (size_t s = 0; s < d.streams.size(); ++s) {
+        if (!used[s] && !(upload && s == 0)) continue;
+        CK(cudaEventRecord(d.end_ev[s], d.streams[s]));
+        finals.push_back(d.end_ev[s]);
+        if (d.ext) CK(cudaStreamWaitEvent(d.ext, d.end_ev[s], 0));
+    }
+    *issue_ns = std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t_issue0).count();
+    if (c->cfg.flush_timeout_ms > 0) {
+        auto deadline = std::chrono::steady_clock::now() + std::chrono::milliseconds(c->cfg.flush_timeout_ms);
+        for (auto ev : finals) {
+            for (;;) {
+                cudaError_t q = cudaEventQuery(ev);
+                if (q == cudaSuccess) break;
+                if (q != cudaErrorNotReady) CK(q);
+                if (std::chrono::steady_clock::now() > deadline) {
+                    d.err = "svp_flush: watchdog expired after " + std::to_string(c->cfg.flush_timeout_ms) + " ms";
+                    return SVP_E_TIMEOUT;
+                }
+                std::this_thread::sleep_for(std::chrono::microseconds(50));
+            }
+        }
+    } else {
+        for (auto ev : finals) CK(cudaEventSynchronize(ev));
+    }
+    CK(cudaGetLastError());
+    // ---- measured op durations
+    if (prof) {
+        for (size_t i = 0; i < f.ops.size(); ++i) {
+            if (tstart[i] < 0) continue;
+            float ms = 0;
+            CK(cudaEventElapsedTime(&ms, d.t_ev[2 * tstart[i]], d.t_ev[2 * tstart[i] + 1]));
+            f.ops[i].measured_ns = ms * 1e6;
+        }
+        // device span: earliest start to latest end
+        float span = 0;
+        int32_t first = -1, lastop = -1;
+        for (size_t i = 0; i < f.ops.size(); ++i)
+            if (tstart[i] >= 0) {
+                if (first < 0) first = (int32_t)i;
+                lastop = (int32_t)i;
+            }
+        if (first >= 0) {
+            float mx = 0;
+            for (size_t i = 0; i < f.ops.size(); ++i) {
+                if (tstart[i] < 0) continue;
+                float ms = 0;
+                CK(cudaEventElapsedTime(&ms, d.t_ev[2 * tstart[first]], d.t_ev[2 * tstart[i] + 1]));
+                mx = std::max(mx, ms);
+            }
+            span = mx;
+        }
+        (void)lastop;
+        c->fstats.device_ns = std::max(c->fstats.device_ns, (double)span * 1e6);
+    }
+    return SVP_OK;
+}
+
+// Profiler attribution (a10): w_v = algorithmic bytes (FLOPs for SGEMM) of the VP's job
+// in the op; T_v = T_op * w_v / sum w.  Conservation (sum_v T_v = T_op) holds exactly up
+// to fp64 rounding.
+static void attribute(Ctx* c, const Flush& f) {
+    std::lock_guard<std::mutex> lk(c->pmu);
+    for (const auto& j : f.jobs) {
+        c->prof[j.vp].jobs += 1;
+        c->prof_total.jobs += 1;
+    }
+    for (const auto& o : f.ops) {
+        const Chunk& ch = f.chunks[o.chunk];
+        if (o.kind == SVP_OP_KERNEL && o.measured_ns >= 0) {
+            c->prof_launches += chunk_needs_launch(f, ch) ? 1 : 0;
+            KStats& ks = c->kstats[ch.kernel];
+            ks.launches += 1;
+            ks.total_ns += o.measured_ns;
+            ks.max_ns = std::max(ks.max_ns, o.measured_ns);
+            ks.bytes += ch.alg_bytes;
+            ks.flops += ch.flops;
+        }
+        if (o.measured_ns < 0) continue;
+        double wsum = 0;
+        std::vector<double> w(ch.jobs.size());
+        for (size_t k = 0; k < ch.jobs.size(); ++k) {
+            const Job& j = f.jobs[ch.jobs[k]];
+            if (o.kind == SVP_OP_H2D) w[k] = (double)j.host_in_bytes;
+            else if (o.kind == SVP_OP_D2H) w[k] = (double)j.host_out_bytes;
+            else w[k] = j.flops > 0 ? j.flops : j.alg_bytes;
+            wsum += w[k];
+        }
+        for (size_t k = 0; k < ch.jobs.size(); ++k) {
+            const Job& j = f.jobs[ch.jobs[k]];
+            double share = wsum > 0 ? o.measured_ns * w[k] / wsum : o.measured_ns / ch.jobs.size();
+            VpProfile& p = c->prof[j.vp];
+            if (o.kind == SVP_OP_H2D) {
+                p.h2d_ns += share;
+                p.bytes_h2d += j.host_in_bytes;
+                c->prof_total.h2d_ns += share;
+                c->prof_total.bytes_h2d += j.host_in_bytes;
+            } else if (o.kind == SVP_OP_D2H) {
+                p.d2h_ns += share;
+                p.bytes_d2h += j.host_out_bytes;
+                c->prof_total.d2h_ns += share;
+                c->prof_total.bytes_d2h += j.host_out_bytes;
+            } else {
+                p.kernel_ns += share;
+                p.bytes_kernel += (uint64_t)j.alg_bytes;
+                p.flops += j.flops;
+                c->prof_total.kernel_ns += share;
+                c->prof_total.bytes_kernel += (uint64_t)j.alg_bytes;
+                c->prof_total.flops += j.flops;
+            }
+        }
+    }
+    // cost-model feedback (EMA of measured / predicted kernel time per kernel)
+    for (const auto& o : f.ops) {
+        if (o.kind != SVP_OP_KERNEL || o.measured_ns <= 0 || o.est_ns <= c->cost.launch_ns * 2) continue;
+        const Chunk& ch = f.chunks[o.chunk];
+        double pred = o.est_ns - c->cost.launch_ns;
+        double meas = std::max(1.0, o.measured_ns - c->cost.launch_ns);
+        double ratio = c->cost.kscale[ch.kernel] * meas / pred;
+        c->cost.kscale[ch.kernel] = 0.8 * c->cost.kscale[ch.kernel] + 0.2 * std::min(8.0, std::max(0.125, ratio));
+    }
+}
+
+svp_status executor_run(Executor* e, Flush* f) {
+    Ctx* c = e->c;
+    const int G = (int)e->devs.size();
+    std::vector<svp_status> st(G, SVP_OK);
+    std::vector<double> issue(G, 0.0);
+    // pre-size the dependency-event pools (event creation is not thread-safe per device
+    // pool vector growth, but each worker owns its Dev)
+    if (G == 1) {
+        st[0] = run_device(e, e->devs[0], *f, &issue[0]);
+    } else {
+        std::vector<std::thread> th;
+        for (int g = 0; g < G; ++g)
+            th.emplace_back([&, g] { st[g] = run_device(e, e->devs[g], *f, &issue[g]); });
+        for (auto& t : th) t.join();
+    }
+    c->fstats.host_issue_ns = *std::max_element(issue.begin(), issue.end());
+    for (int g = 0; g < G; ++g) {
+        if (st[g] != SVP_OK) {
+            e->err = "GPU " + std::to_string(g) + ": " + e->devs[g].err;
+            return st[g];
+        }
+    }
+    if (c->cfg.profile_level >= 1) attribute(c, *f);
+    else {
+        std::lock_guard<std::mutex> lk(c->pmu);
+        for (const auto& j : f->jobs) {
+            c->prof[j.vp].jobs += 1;
+            c->prof_total.jobs += 1;
+        }
+        for (const auto& o : f->ops)
+            if (o.kind == SVP_OP_KERNEL && chunk_needs_launch(*f, f->chunks[o.chunk])) c->prof_launches += 1;
+    }
+    return SVP_OK;
+}
+
+}  // namespace svp

@@ -1,0 +1,206 @@
+// internal.h -- core data structures of libsvp (host side).  Not part of the C-ABI.
+//
+// Layering: capi.cpp (L5 boundary) -> scheduler.cpp (L3: Job Queue,
+// Kernel Match, Job Dispatcher, Re-scheduler, cost model) -> executor.cpp (L2: per-GPU
+// streams/events/arena/tables, Profiler) -> kernels/*.cu (L0: sm_100a guest kernels).
+#pragma once
+#include <stdint.h>
+
+#include <atomic>
+#include <condition_variable>
+#include <functional>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <unordered_map>
+#include <vector>
+
+#include "../../include/svp.h"
+
+namespace svp {
+
+// ------------------------------------------------------------------ kernel registry
+enum KernelId : int32_t {
+    K_VECADD = 1,
+    K_SAXPY = 2,
+    K_HIST256 = 3,
+    K_BLACKSCHOLES = 4,
+    K_SGEMM = 5,
+    K_SGEMM_TF32 = 6,
+    K_COUNT = 7
+};
+
+struct KernelDesc {
+    const char* name;
+    int32_t id;
+    int32_t nbufs;
+    int32_t dirs[SVP_MAX_BUFS];   // required SVP_DIR_* (sgemm C may be OUT or INOUT)
+    uint32_t args_bytes;
+};
+const KernelDesc* kernel_desc(int32_t id);
+const KernelDesc* kernel_by_name(const char* name);
+
+// ------------------------------------------------------------------ jobs
+struct Job {
+    uint64_t id = 0;
+    int32_t vp = 0;
+    int32_t kernel = 0;
+    uint8_t args[SVP_MAX_ARGS] = {};
+    svp_buf bufs[SVP_MAX_BUFS] = {};
+    int32_t nbufs = 0;
+    // derived at submit
+    uint64_t n = 0;               // elements (memory-bound kernels)
+    int32_t M = 0, N = 0, K = 0;  // sgemm
+    float f0 = 0.f, f1 = 0.f;     // scalars
+    uint64_t shape_key = 0;       // Kernel Match key (with kernel id)
+    uint64_t in_bytes = 0;        // bytes of IN/INOUT buffers the kernel reads
+    uint64_t out_bytes = 0;       // bytes of OUT/INOUT buffers the kernel writes
+    uint64_t host_in_bytes = 0;   // of which host-resident (H2D staging)
+    uint64_t host_out_bytes = 0;  // of which host-resident (D2H)
+    double alg_bytes = 0;         // algorithmic bytes (roofline, profiler weights)
+    double flops = 0;
+    int32_t level = 0;            // program-order level within the flush
+    int32_t device = 0;           // assigned GPU
+};
+
+// Bytes the kernel touches in buffer b of job j (what must be staged / copied back).
+uint64_t touched_bytes(const Job& j, int b);
+
+// ------------------------------------------------------------------ plan
+struct Chunk {
+    int32_t group = 0;
+    int32_t index = 0;              // chunk index in group
+    int32_t device = 0;
+    int32_t level = 0;
+    int32_t kernel = 0;
+    std::vector<int32_t> jobs;      // indices into Flush::jobs, segment order (vp ascending)
+    double t_in = 0, t_k = 0, t_out = 0;  // cost-model estimates (ns)
+    uint64_t in_bytes = 0, out_bytes = 0;
+    double alg_bytes = 0, flops = 0;
+    // staging
+    uint64_t arena_off = 0, arena_len = 0;
+    std::vector<uint64_t> staged;   // per job per buffer: device address used by kernel
+    // table
+    uint64_t table_off = 0;         // offset of this chunk's table in the device table buffer
+    uint32_t total_tiles = 0;
+    int32_t nsegs = 0;
+    uint64_t maps_off = 0;          // sgemm: tensor maps offset
+};
+
+struct Op {
+    int32_t kind = SVP_OP_KERNEL;
+    int32_t chunk = 0;
+    int32_t device = 0;
+    int32_t stream = 0;
+    std::vector<int32_t> wait_ops;  // ops (global index) this op must wait for
+    bool needs_event = false;       // someone waits on this op -> record event after it
+    double est_ns = 0;
+    double sim_start = 0, sim_end = 0;
+    double measured_ns = -1;
+    uint64_t bytes = 0;
+    double flops = 0;
+    bool last_of_job = false;       // serial baseline: sync after this op
+};
+
+struct Group {
+    int32_t kernel = 0;
+    uint64_t shape_key = 0;
+    int32_t level = 0;
+    int32_t device = 0;
+    std::vector<int32_t> jobs;      // vp ascending
+};
+
+struct Flush {
+    std::vector<Job> jobs;
+    std::vector<Group> groups;
+    std::vector<Chunk> chunks;
+    std::vector<Op> ops;            // issue order (per device subsequence is that device's issue order)
+    int32_t levels = 0;
+};
+
+// ------------------------------------------------------------------ per-VP profile
+struct VpProfile {
+    uint64_t jobs = 0;
+    double kernel_ns = 0, h2d_ns = 0, d2h_ns = 0;
+    uint64_t bytes_kernel = 0, bytes_h2d = 0, bytes_d2h = 0;
+    double flops = 0;
+};
+
+struct KStats {
+    uint64_t launches = 0;
+    double total_ns = 0, bytes = 0, flops = 0, max_ns = 0;
+};
+
+// ------------------------------------------------------------------ cost model (D8)
+struct CostModel {
+    double hbm_Bps = 6552e9;
+    double pcie_Bps = 50e9;
+    double ffma_flops = 60e12;
+    double tf32_flops = 500e12;
+    double launch_ns = 4000;
+    double copy_ns = 2000;           // per-copy fixed overhead
+    // EMA of measured/predicted ratio per kernel (learned from the profiler)
+    double kscale[K_COUNT] = {1, 1, 1, 1, 1, 1, 1};
+    double kernel_ns(int32_t kernel, double alg_bytes, double flops) const;
+    double h2d_ns(uint64_t bytes, int ncopies) const;
+    double d2h_ns(uint64_t bytes, int ncopies) const;
+};
+
+class Executor;  // executor.cpp
+
+struct Ctx {
+    svp_config cfg{};
+    std::vector<int32_t> device_ids;
+    int32_t ngpu = 1;
+    CostModel cost;
+
+    // Job Queue (D2): per-VP FIFOs, program order = submission order
+    std::mutex qmu;
+    std::vector<Job> queue;          // appended in submission order; snapshot at flush
+    uint64_t next_job_id = 1;
+
+    // Job Dispatcher: sticky VP -> GPU
+    std::mutex dmu;
+    std::unordered_map<int32_t, int32_t> vp_dev;
+    std::vector<double> dev_load;
+
+    // state
+    std::atomic<int> flushing{0};
+    int32_t sticky = 0;              // SVP_OK or first fatal status
+    std::string sticky_msg;
+    bool registered[K_COUNT] = {};
+
+    // last flush
+    Flush last;
+    svp_flush_stats fstats{};
+
+    // Profiler
+    std::mutex pmu;
+    std::unordered_map<int32_t, VpProfile> prof;
+    VpProfile prof_total;
+    uint64_t prof_launches = 0;
+    KStats kstats[K_COUNT];
+
+    Executor* exec = nullptr;        // null in dry_run
+};
+
+// scheduler.cpp
+svp_status validate_and_fill(Ctx* c, Job* j);
+svp_status plan_flush(Ctx* c, Flush* f);             // match, dispatch, reschedule, simulate
+int32_t dispatch_vp(Ctx* c, int32_t vp, double cost);
+void lpt_stratified(int32_t n, const int32_t* classes, const double* costs, int32_t G,
+                    const double* init_load, int32_t* out);
+void simulate(Ctx* c, Flush* f, double* makespan, double* serial);
+
+// executor.cpp
+Executor* executor_create(Ctx* c, svp_status* st);
+void executor_destroy(Executor* e);
+svp_status executor_run(Executor* e, Flush* f);      // tables, staging, issue, wait, profile
+std::string executor_error(Executor* e);
+// residency check for svp_submit (validate_ptrs): returns SVP_OK or SVP_E_INVAL
+svp_status executor_check_ptr(Executor* e, const void* p, int32_t mem, int32_t device, std::string* why);
+
+// errors
+void set_error(const std::string& msg);
+
+}  // namespace svp

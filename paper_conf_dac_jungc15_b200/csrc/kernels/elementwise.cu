@@ -1,0 +1,196 @@
+// elementwise.cu -- coalesced vecadd, SAXPY and Black-Scholes for sm_100a.
+//
+// One launch serves every VP of a Kernel Match group (Kernel Coalescing, PAPER.md
+// L288-306, Fig 6b): the grid walks the launch's tile space persistently
+// (tile = blockIdx.x, += gridDim.x; grid = #SMs x resident CTAs, Eq 9's aligned
+// unit lambda), each tile is mapped to its VP segment by a binary search over the
+// segment table, interior tiles move 128-bit (float4) streaming loads/stores
+// (ld/st .cs -- evict-first, every byte is touched once), and a VP's ragged head/tail
+// tile runs a predicated scalar loop (no padding).
+//
+// Arithmetic per element (bit-exact with the oracle for vecadd / SAXPY):
+//   vecadd  c = a + b            (__fadd_rn: one rounding, never contracted)
+//   saxpy   y = fma(a_v, x, y)   (__fmaf_rn: single rounding, = C99 fmaf)
+//   BS      SDK formula with the A&S 26.2.17 CND, accurate expf/logf/sqrtf, IEEE div.
+#include "../launch.h"
+#include "common.cuh"
+
+namespace svp {
+
+// --------------------------------------------------------------------- vecadd
+__global__ void __launch_bounds__(kEwThreads) k_vecadd(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
+    constexpr int V = kVecaddVec, TILE = kVecaddTile;
+    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+        const int si = find_seg(segs, nsegs, t);
+        const SegDesc& sd = segs[si];
+        const float* __restrict__ a = reinterpret_cast<const float*>(sd.ptr[0]);
+        const float* __restrict__ b = reinterpret_cast<const float*>(sd.ptr[1]);
+        float* __restrict__ c = reinterpret_cast<float*>(sd.ptr[2]);
+        int64_t e0, e1;
+        bool vec;
+        tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, TILE, e0, e1, vec);
+        if (vec) {
+            const float4* a4 = reinterpret_cast<const float4*>(a + e0) + threadIdx.x;
+            const float4* b4 = reinterpret_cast<const float4*>(b + e0) + threadIdx.x;
+            float4* c4 = reinterpret_cast<float4*>(c + e0) + threadIdx.x;
+            float4 ra[V], rb[V];
+#pragma unroll
+            for (int i = 0; i < V; ++i) {
+                ra[i] = __ldcs(a4 + i * kEwThreads);
+                rb[i] = __ldcs(b4 + i * kEwThreads);
+            }
+#pragma unroll
+            for (int i = 0; i < V; ++i) {
+                float4 r;
+                r.x = __fadd_rn(ra[i].x, rb[i].x);
+                r.y = __fadd_rn(ra[i].y, rb[i].y);
+                r.z = __fadd_rn(ra[i].z, rb[i].z);
+                r.w = __fadd_rn(ra[i].w, rb[i].w);
+                __stcs(c4 + i * kEwThreads, r);
+            }
+        } else {
+            for (int64_t e = e0 + threadIdx.x; e < e1; e += kEwThreads) c[e] = __fadd_rn(a[e], b[e]);
+        }
+    }
+}
+
+// --------------------------------------------------------------------- SAXPY
+__global__ void __launch_bounds__(kEwThreads) k_saxpy(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
+    constexpr int V = kVecaddVec, TILE = kSaxpyTile;
+    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+        const int si = find_seg(segs, nsegs, t);
+        const SegDesc& sd = segs[si];
+        const float* __restrict__ x = reinterpret_cast<const float*>(sd.ptr[0]);
+        float* __restrict__ y = reinterpret_cast<float*>(sd.ptr[1]);
+        const float a = sd.f[0];
+        int64_t e0, e1;
+        bool vec;
+        tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, TILE, e0, e1, vec);
+        if (vec) {
+            const float4* x4 = reinterpret_cast<const float4*>(x + e0) + threadIdx.x;
+            float4* y4 = reinterpret_cast<float4*>(y + e0) + threadIdx.x;
+            float4 rx[V], ry[V];
+#pragma unroll
+            for (int i = 0; i < V; ++i) {
+                rx[i] = __ldcs(x4 + i * kEwThreads);
+                ry[i] = __ldcs(y4 + i * kEwThreads);
+            }
+#pragma unroll
+            for (int i = 0; i < V; ++i) {
+                float4 r;
+                r.x = __fmaf_rn(a, rx[i].x, ry[i].x);
+                r.y = __fmaf_rn(a, rx[i].y, ry[i].y);
+                r.z = __fmaf_rn(a, rx[i].z, ry[i].z);
+                r.w = __fmaf_rn(a, rx[i].w, ry[i].w);
+                __stcs(y4 + i * kEwThreads, r);
+            }
+        } else {
+            for (int64_t e = e0 + threadIdx.x; e < e1; e += kEwThreads) y[e] = __fmaf_rn(a, x[e], y[e]);
+        }
+    }
+}
+
+// --------------------------------------------------------------------- Black-Scholes
+__device__ __forceinline__ float cnd_as(float d) {
+    const float A1 = 0.31938153f, A2 = -0.356563782f, A3 = 1.781477937f, A4 = -1.821255978f,
+                A5 = 1.330274429f;
+    const float RSQRT2PI = 0.39894228040143267793994605993438f;
+    float K = 1.0f / (1.0f + 0.2316419f * fabsf(d));
+    float cnd = RSQRT2PI * expf(-0.5f * d * d) * (K * (A1 + K * (A2 + K * (A3 + K * (A4 + K * A5)))));
+    return d > 0.f ? 1.0f - cnd : cnd;
+}
+
+__device__ __forceinline__ void bs_one(float S, float X, float T, float R, float V, float& call, float& put) {
+    float sqrtT = sqrtf(T);
+    float d1 = (logf(S / X) + (R + 0.5f * V * V) * T) / (V * sqrtT);
+    float d2 = d1 - V * sqrtT;
+    float N1 = cnd_as(d1), N2 = cnd_as(d2);
+    float expRT = expf(-R * T);
+    call = S * N1 - X * expRT * N2;
+    put = X * expRT * (1.0f - N2) - S * (1.0f - N1);
+}
+
+__global__ void __launch_bounds__(kEwThreads) k_blackscholes(const SegDesc* __restrict__ segs, int nsegs,
+                                                             uint32_t total) {
+    constexpr int V = kBsVec, TILE = kBsTile;
+    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+        const int si = find_seg(segs, nsegs, t);
+        const SegDesc& sd = segs[si];
+        const float* __restrict__ S = reinterpret_cast<const float*>(sd.ptr[0]);
+        const float* __restrict__ X = reinterpret_cast<const float*>(sd.ptr[1]);
+        const float* __restrict__ T = reinterpret_cast<const float*>(sd.ptr[2]);
+        float* __restrict__ C = reinterpret_cast<float*>(sd.ptr[3]);
+        float* __restrict__ P = reinterpret_cast<float*>(sd.ptr[4]);
+        const float R = sd.f[0], Vol = sd.f[1];
+        int64_t e0, e1;
+        bool vec;
+        tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, TILE, e0, e1, vec);
+        if (vec) {
+            const int o = threadIdx.x;
+            float4 rs[V], rx[V], rt[V];
+#pragma unroll
+            for (int i = 0; i < V; ++i) {
+                rs[i] = __ldcs(reinterpret_cast<const float4*>(S + e0) + o + i * kEwThreads);
+                rx[i] = __ldcs(reinterpret_cast<const float4*>(X + e0) + o + i * kEwThreads);
+                rt[i] = __ldcs(reinterpret_cast<const float4*>(T + e0) + o + i * kEwThreads);
+            }
+#pragma unroll
+            for (int i = 0; i < V; ++i) {
+                float4 c, p;
+                bs_one(rs[i].x, rx[i].x, rt[i].x, R, Vol, c.x, p.x);
+                bs_one(rs[i].y, rx[i].y, rt[i].y, R, Vol, c.y, p.y);
+                bs_one(rs[i].z, rx[i].z, rt[i].z, R, Vol, c.z, p.z);
+                bs_one(rs[i].w, rx[i].w, rt[i].w, R, Vol, c.w, p.w);
+                __stcs(reinterpret_cast<float4*>(C + e0) + o + i * kEwThreads, c);
+                __stcs(reinterpret_cast<float4*>(P + e0) + o + i * kEwThreads, p);
+            }
+        } else {
+            for (int64_t e = e0 + threadIdx.x; e < e1; e += kEwThreads) {
+                float c, p;
+                bs_one(S[e], X[e], T[e], R, Vol, c, p);
+                C[e] = c;
+                P[e] = p;
+            }
+        }
+    }
+}
+
+// --------------------------------------------------------------------- launchers
+cudaError_t launch_vecadd(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+    k_vecadd<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
+    return cudaGetLastError();
+}
+cudaError_t launch_saxpy(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+    k_saxpy<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
+    return cudaGetLastError();
+}
+cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+    k_blackscholes<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
+    return cudaGetLastError();
+}
+
+cudaError_t query_limits_hist(int* per_sm);
+cudaError_t query_limits_gemm(int* per_sm);
+
+cudaError_t query_limits(LaunchLimits* out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e) return e;
+    e = cudaDeviceGetAttribute(&out->num_sms, cudaDevAttrMultiProcessorCount, dev);
+    if (e) return e;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&out->ew_blocks_per_sm, k_vecadd, kEwThreads, 0);
+    if (e) return e;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&out->bs_blocks_per_sm, k_blackscholes, kEwThreads, 0);
+    if (e) return e;
+    e = query_limits_hist(&out->hist_blocks_per_sm);
+    if (e) return e;
+    e = query_limits_gemm(&out->gemm_blocks_per_sm);
+    if (e) return e;
+    if (out->ew_blocks_per_sm < 1) out->ew_blocks_per_sm = 1;
+    if (out->bs_blocks_per_sm < 1) out->bs_blocks_per_sm = 1;
+    if (out->hist_blocks_per_sm < 1) out->hist_blocks_per_sm = 1;
+    if (out->gemm_blocks_per_sm < 1) out->gemm_blocks_per_sm = 1;
+    return cudaSuccess;
+}
+
+}  // namespace svp

@@ -1,0 +1,241 @@
+// sgemm_ffma.cu -- grouped (coalesced) fp32 SGEMM for sm_100a: TMA-staged tiles, fp32 FFMA.
+//
+// C_v = alpha_v A_v B_v + beta_v C_v for every VP v of a Kernel Match group (equal
+// M,N,K -- reading R1), all in ONE persistent launch: the paper's matmul guest
+// (Table 1) coalesced.  A single 512^3 job has
+// 16 output tiles and fills 16 of 148 SMs; 16 coalesced jobs give 256 tiles (the
+// "alignment" gain of PAPER.md L526-531 / Eq 9).
+//
+// Design (B200):
+//  * persistent grid = #SMs, 1 CTA/SM; static tile walk t = blockIdx.x + i*gridDim.x;
+//    tile -> (VP, tile_m, tile_n) through the GemmDesc table (binary search).
+//  * warp 8 = TMA producer: one elected lane issues cp.async.bulk.tensor for the A
+//    (128x32, 128-B swizzle) and B (32x128) tiles of each k-block into a 4-stage smem
+//    ring guarded by full/empty mbarriers; per-VP CUtensorMaps live in the table.
+//  * warps 0-7 = consumers: 8x8 fp32 register micro-tile per thread; per 4-k group a
+//    thread reads 8 float4 of A (k-vectorised, conflict-free thanks to the swizzle) and
+//    8 float4 of B, then issues 256 FFMA (16 FFMA per LDS.128).
+//  * epilogue: alpha*acc (+ beta*C) with 128-bit stores straight from registers.
+#include <cuda.h>
+#include <stdio.h>
+
+#include "../launch.h"
+#include "common.cuh"
+
+namespace svp {
+
+constexpr int GM = kGemmBM, GN = kGemmBN, GK = kGemmBK;
+constexpr int kStages = 4;
+constexpr int kConsumers = 256;
+constexpr int kGemmThreads = kConsumers + 32;
+constexpr int kStageA = GM * GK * 4;  // 16 KiB
+constexpr int kStageB = GK * GN * 4;  // 16 KiB
+constexpr size_t kGemmSmem = 1024 + kStages * (kStageA + kStageB) + 2 * kStages * sizeof(uint64_t);
+
+__device__ __forceinline__ int find_gemm(const GemmDesc* __restrict__ d, int n, uint32_t t) {
+    int lo = 0, hi = n;
+    while (lo < hi) {
+        int mid = (lo + hi) >> 1;
+        if (__ldg(&d[mid].tile_begin) <= t) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo - 1;
+}
+
+__global__ void __launch_bounds__(kGemmThreads, 1)
+    k_sgemm_ffma(const GemmDesc* __restrict__ descs, int n, const uint8_t* __restrict__ maps, uint32_t total) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    float* sA = reinterpret_cast<float*>(smem);
+    float* sB = reinterpret_cast<float*>(smem + kStages * kStageA);
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages * (kStageA + kStageB));
+    uint64_t* empty = full + kStages;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kStages; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kConsumers / 32);
+        }
+        mbar_fence_init();
+    }
+    __syncthreads();
+
+    if (warp == kConsumers / 32) {
+        // ------------------------------------------------------------ TMA producer
+        if (lane == 0) {
+            uint32_t it = 0;
+            int last = -1;
+            for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+                const int v = find_gemm(descs, n, t);
+                const GemmDesc& g = descs[v];
+                const void* mA = maps + (size_t)v * 256;
+                const void* mB = maps + (size_t)v * 256 + 128;
+                if (v != last) {
+                    prefetch_tmap(mA);
+                    prefetch_tmap(mB);
+                    last = v;
+                }
+                const uint32_t lt = t - g.tile_begin;
+                const int tm = lt / g.tiles_n, tn = lt % g.tiles_n;
+                const int KB = (g.K + GK - 1) / GK;
+                for (int kb = 0; kb < KB; ++kb, ++it) {
+                    const int s = it % kStages;
+                    const uint32_t ph = (it / kStages) & 1;
+                    mbar_wait(&empty[s], ph ^ 1);
+                    mbar_expect_tx(&full[s], kStageA + kStageB);
+                    tma_load_2d(sA + s * GM * GK, mA, kb * GK, tm * GM, &full[s]);
+                    tma_load_2d(sB + s * GK * GN, mB, tn * GN, kb * GK, &full[s]);
+                }
+            }
+        }
+        return;
+    }
+
+    // ---------------------------------------------------------------- consumers
+    const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+    uint32_t it = 0;
+    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+        const int v = find_gemm(descs, n, t);
+        const GemmDesc& g = descs[v];
+        const uint32_t lt = t - g.tile_begin;
+        const int tm = lt / g.tiles_n, tn = lt % g.tiles_n;
+        const int KB = (g.K + GK - 1) / GK;
+        float acc[8][8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+            for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+
+        for (int kb = 0; kb < KB; ++kb, ++it) {
+            const int s = it % kStages;
+            const uint32_t ph = (it / kStages) & 1;
+            mbar_wait(&full[s], ph);
+            const float* A = sA + s * GM * GK;
+            const float* B = sB + s * GK * GN;
+#pragma unroll
+            for (int kk = 0; kk < GK / 4; ++kk) {
+                float4 a[8];
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + (i - 4));
+                    const int chunk = kk ^ (r & 7);  // 128-B swizzle: 16-B chunk ^= row % 8
+                    a[i] = *reinterpret_cast<const float4*>(A + r * GK + chunk * 4);
+                }
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int k = kk * 4 + q;
+                    const float4 b0 = *reinterpret_cast<const float4*>(B + k * GN + tx * 4);
+                    const float4 b1 = *reinterpret_cast<const float4*>(B + k * GN + 64 + tx * 4);
+                    const float bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) {
+                        const float av = q == 0 ? a[i].x : q == 1 ? a[i].y : q == 2 ? a[i].z : a[i].w;
+#pragma unroll
+                        for (int j = 0; j < 8; ++j) acc[i][j] = __fmaf_rn(av, bv[j], acc[i][j]);
+                    }
+                }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+        }
+
+        // ------------------------------------------------------------ epilogue
+        const int M = g.M, N = g.N;
+        const float alpha = g.alpha, beta = g.beta;
+        float* __restrict__ C = g.C;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int r = tm * GM + ((i < 4) ? (ty * 4 + i) : (64 + ty * 4 + (i - 4)));
+            if (r >= M) continue;
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int c = tn * GN + h * 64 + tx * 4;
+                if (c >= N) continue;
+                float4* dst = reinterpret_cast<float4*>(C + (size_t)r * N + c);
+                float4 o;
+                o.x = alpha * acc[i][h * 4 + 0];
+                o.y = alpha * acc[i][h * 4 + 1];
+                o.z = alpha * acc[i][h * 4 + 2];
+                o.w = alpha * acc[i][h * 4 + 3];
+                if (beta != 0.f) {
+                    const float4 old = *dst;
+                    o.x = __fmaf_rn(beta, old.x, o.x);
+                    o.y = __fmaf_rn(beta, old.y, o.y);
+                    o.z = __fmaf_rn(beta, old.z, o.z);
+                    o.w = __fmaf_rn(beta, old.w, o.w);
+                }
+                *dst = o;
+            }
+        }
+    }
+}
+
+static bool g_smem_set[64] = {};
+
+cudaError_t launch_sgemm_ffma(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
+                              cudaStream_t s) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 64 && !g_smem_set[dev]) {
+        cudaError_t e = cudaFuncSetAttribute(k_sgemm_ffma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kGemmSmem);
+        if (e) return e;
+        g_smem_set[dev] = true;
+    }
+    k_sgemm_ffma<<<grid, kGemmThreads, kGemmSmem, s>>>(descs, n, reinterpret_cast<const uint8_t*>(maps), total);
+    return cudaGetLastError();
+}
+
+cudaError_t query_limits_gemm(int* per_sm) {
+    cudaError_t e = cudaFuncSetAttribute(k_sgemm_ffma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kGemmSmem);
+    if (e) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k_sgemm_ffma, kGemmThreads, kGemmSmem);
+}
+
+// ------------------------------------------------------------------ TMA descriptors
+typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                    const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static PFN_encodeTiled get_encode() {
+    static PFN_encodeTiled fn = nullptr;
+    if (!fn) {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_encodeTiled>(p);
+    }
+    return fn;
+}
+
+static int encode2d(void* out, const float* base, uint64_t inner, uint64_t outer, uint32_t box_inner,
+                    uint32_t box_outer, CUtensorMapSwizzle sw) {
+    PFN_encodeTiled enc = get_encode();
+    if (!enc) return -1;
+    cuuint64_t dims[2] = {inner, outer};
+    cuuint64_t strides[1] = {inner * 4};
+    cuuint32_t box[2] = {box_inner, box_outer};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(reinterpret_cast<CUtensorMap*>(out), CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)base, dims, strides,
+                     box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? 0 : (int)r;
+}
+
+int encode_gemm_maps(void* mapA, void* mapB, const float* A, const float* B, int M, int N, int K, int variant) {
+    static_assert(sizeof(CUtensorMap) == 128, "CUtensorMap is 128 B");
+    if (variant == 0) {
+        // A: M x K row-major -> box 32 (k) x 128 (m), 128-B swizzle; B: K x N -> box 128 (n) x 32 (k)
+        int r = encode2d(mapA, A, (uint64_t)K, (uint64_t)M, GK, GM, CU_TENSOR_MAP_SWIZZLE_128B);
+        if (r) return r;
+        return encode2d(mapB, B, (uint64_t)N, (uint64_t)K, GN, GK, CU_TENSOR_MAP_SWIZZLE_NONE);
+    }
+    // TF32 tcgen05 tiles: both operands K-major-in-smem is impossible for row-major B, so
+    // A is K-major (box 32 k x 128 m, SW128) and B is MN-major (box 32 n x 32 k, SW128).
+    int r = encode2d(mapA, A, (uint64_t)K, (uint64_t)M, kTf32BK, kTf32BM, CU_TENSOR_MAP_SWIZZLE_128B);
+    if (r) return r;
+    return encode2d(mapB, B, (uint64_t)N, (uint64_t)K, 32, kTf32BK, CU_TENSOR_MAP_SWIZZLE_128B);
+}
+
+}  // namespace svp

@@ -1,0 +1,44 @@
+// launch.h -- host-side launchers of the sm_100a guest kernels (internal to libsvp).
+// Every launcher enqueues ONE coalesced launch (plus hist256's output zeroing) on
+// `stream` and returns the launch error; none synchronizes.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "tables.h"
+
+namespace svp {
+
+struct LaunchLimits {
+    int num_sms = 148;
+    int ew_blocks_per_sm = 8;   // occupancy of the elementwise kernels
+    int bs_blocks_per_sm = 4;
+    int hist_blocks_per_sm = 4;
+    int gemm_blocks_per_sm = 1;
+};
+
+// Query occupancy / SM count for the current device (call once per device).
+cudaError_t query_limits(LaunchLimits* out);
+
+// Elementwise coalesced kernels: segs/nsegs describe the VPs, total_tiles is
+// segs[nsegs-1].tile_begin + tiles of the last segment.
+cudaError_t launch_vecadd(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
+cudaError_t launch_saxpy(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
+cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
+// hist256: zeroes each segment's 256 counters, then accumulates.
+cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
+
+// Grouped SGEMM (fp32 FFMA, TMA-staged).  maps = 2*n CUtensorMap (A_i, B_i), 64-B aligned.
+cudaError_t launch_sgemm_ffma(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
+                              int grid, cudaStream_t s);
+// Grouped SGEMM on tcgen05 TF32 tensor cores (TMEM accumulators).
+cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
+                              int grid, cudaStream_t s);
+
+// Host: encode the TMA descriptors an SGEMM entry needs (driver entry point fetched at
+// runtime, so libsvp does not link libcuda).  variant 0 = FFMA tiles, 1 = TF32 tiles.
+// Returns 0 on success.
+int encode_gemm_maps(void* mapA, void* mapB, const float* A, const float* B, int M, int N, int K,
+                     int variant);
+
+}  // namespace svp

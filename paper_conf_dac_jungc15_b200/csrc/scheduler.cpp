@@ -1,0 +1,507 @@
+// scheduler.cpp -- Job Queue validation, Kernel Match, Job Dispatcher, Re-scheduler
+// and the cost model (host side, no CUDA).  SURVEY.md §8(a) rows a1-a4.
+//
+//  * Job Queue (Fig 2): jobs arrive per VP in program
+//    order; at svp_flush the queue is snapshotted and the l-th pending job of a VP
+//    gets level l.  Reading R3: a VP's jobs are totally ordered (program order);
+//    jobs of different VPs are independent.
+//  * Kernel Match: within a level and a GPU, jobs with
+//    the same (kernel id, shape key) are "identical kernel requests" and form one
+//    group (reading R1: ragged n is allowed for the elementwise kernels, SGEMM needs
+//    equal M,N,K).  Groups are ordered by (kernel, shape key); members by VP id (R12).
+//  * Job Dispatcher ("multiplexes the host GPUs", L28-31): every VP
+//    is pinned to one GPU (sticky), placed by kernel-stratified LPT.
+//  * Re-scheduler (Fig 3/4a): splits each group into c
+//    chunks so copies of one chunk overlap the kernel of another, orders the chunks
+//    of a level with Johnson's rule on (Tin+Tk, Tk+Tout) using the expected time of
+//    each invocation (reading R4), assigns streams (one H2D, one
+//    D2H, a pool of compute streams -- the paper's Copy/Compute engines), and adds
+//    the event dependencies that keep every VP's program order.
+#include <math.h>
+#include <string.h>
+
+#include <algorithm>
+#include <map>
+#include <numeric>
+#include <tuple>
+
+#include "internal.h"
+#include "tables.h"
+
+namespace svp {
+
+// ------------------------------------------------------------------ cost model
+double CostModel::kernel_ns(int32_t kernel, double alg_bytes, double flops) const {
+    double body;
+    if (kernel == K_SGEMM) body = flops / ffma_flops * 1e9;
+    else if (kernel == K_SGEMM_TF32) body = flops / tf32_flops * 1e9;
+    else body = alg_bytes / hbm_Bps * 1e9;
+    return launch_ns + body * kscale[kernel];
+}
+double CostModel::h2d_ns(uint64_t bytes, int ncopies) const {
+    return bytes ? copy_ns * ncopies + (double)bytes / pcie_Bps * 1e9 : 0.0;
+}
+double CostModel::d2h_ns(uint64_t bytes, int ncopies) const {
+    return bytes ? copy_ns * ncopies + (double)bytes / pcie_Bps * 1e9 : 0.0;
+}
+
+// ------------------------------------------------------------------ validation (a1)
+uint64_t touched_bytes(const Job& j, int b) {
+    switch (j.kernel) {
+        case K_VECADD:
+        case K_SAXPY:
+        case K_BLACKSCHOLES: return 4ull * j.n;
+        case K_HIST256: return b == 0 ? j.n : 1024ull;
+        case K_SGEMM:
+        case K_SGEMM_TF32:
+            if (b == 0) return 4ull * j.M * j.K;
+            if (b == 1) return 4ull * j.K * j.N;
+            return 4ull * j.M * j.N;
+    }
+    return 0;
+}
+
+static svp_status fail(svp_status st, const std::string& msg) {
+    set_error(msg);
+    return st;
+}
+
+svp_status validate_and_fill(Ctx* c, Job* j) {
+    const KernelDesc* d = kernel_desc(j->kernel);
+    if (!d || !c->registered[j->kernel])
+        return fail(SVP_E_NOKERNEL, "svp_submit: kernel id " + std::to_string(j->kernel) + " not registered");
+    if (j->vp < 0 || j->vp >= (1 << 20)) return fail(SVP_E_INVAL, "svp_submit: vp out of range [0, 2^20)");
+    if (j->nbufs != d->nbufs)
+        return fail(SVP_E_INVAL, std::string("svp_submit: ") + d->name + " takes " + std::to_string(d->nbufs) +
+                                     " buffers");
+    switch (j->kernel) {
+        case K_VECADD:
+        case K_HIST256: memcpy(&j->n, j->args, 8); break;
+        case K_SAXPY:
+            memcpy(&j->n, j->args, 8);
+            memcpy(&j->f0, j->args + 8, 4);
+            break;
+        case K_BLACKSCHOLES:
+            memcpy(&j->n, j->args, 8);
+            memcpy(&j->f0, j->args + 8, 4);
+            memcpy(&j->f1, j->args + 12, 4);
+            break;
+        case K_SGEMM:
+        case K_SGEMM_TF32: {
+            svp_args_sgemm a;
+            memcpy(&a, j->args, sizeof(a));
+            if (a.M < 0 || a.N < 0 || a.K < 0 || a.M >= (1 << 20) || a.N >= (1 << 20) || a.K >= (1 << 20))
+                return fail(SVP_E_INVAL, "svp_submit: sgemm M,N,K must be in [0, 2^20)");
+            j->M = a.M;
+            j->N = a.N;
+            j->K = a.K;
+            j->f0 = a.alpha;
+            j->f1 = a.beta;
+            if ((int64_t)a.M * a.N * a.K > 0 && (a.K % 4 != 0 || a.N % 4 != 0))
+                return fail(SVP_E_UNSUPPORTED, "svp_submit: sgemm needs K % 4 == 0 and N % 4 == 0 (TMA row pitch)");
+            break;
+        }
+    }
+    if (j->n >= (1ull << 40)) return fail(SVP_E_INVAL, "svp_submit: n too large");
+    bool empty = (j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32) ? ((int64_t)j->M * j->N == 0) : (j->n == 0);
+    j->in_bytes = j->out_bytes = j->host_in_bytes = j->host_out_bytes = 0;
+    for (int b = 0; b < j->nbufs; ++b) {
+        const svp_buf& bf = j->bufs[b];
+        uint64_t need = touched_bytes(*j, b);
+        int want = d->dirs[b];
+        bool is_c = (j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32) && b == 2;
+        if (is_c) {
+            if (j->f1 != 0.f && bf.dir != SVP_DIR_INOUT)
+                return fail(SVP_E_INVAL, "svp_submit: sgemm with beta != 0 needs C as SVP_DIR_INOUT");
+            if (bf.dir != SVP_DIR_OUT && bf.dir != SVP_DIR_INOUT)
+                return fail(SVP_E_INVAL, "svp_submit: sgemm C must be OUT or INOUT");
+        } else if (bf.dir != want) {
+            return fail(SVP_E_INVAL, std::string("svp_submit: buffer ") + std::to_string(b) + " of " + d->name +
+                                         " has the wrong direction");
+        }
+        if (bf.mem != SVP_MEM_DEVICE && bf.mem != SVP_MEM_HOST_PINNED)
+            return fail(SVP_E_INVAL, "svp_submit: buffer mem must be DEVICE or HOST_PINNED");
+        if (empty) continue;
+        if (need && !bf.ptr) return fail(SVP_E_INVAL, "svp_submit: null buffer " + std::to_string(b));
+        if (bf.bytes < need)
+            return fail(SVP_E_INVAL, "svp_submit: buffer " + std::to_string(b) + " has " + std::to_string(bf.bytes) +
+                                         " bytes, kernel touches " + std::to_string(need));
+        if ((j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32) && bf.mem == SVP_MEM_DEVICE &&
+            ((uintptr_t)bf.ptr & 15))
+            return fail(SVP_E_UNSUPPORTED, "svp_submit: sgemm device buffers must be 16-B aligned (TMA)");
+        bool rd = bf.dir & SVP_DIR_IN, wr = bf.dir & SVP_DIR_OUT;
+        // sgemm C with beta == 0 is written only; hist counts are written only
+        if (rd) j->in_bytes += need;
+        if (wr) j->out_bytes += need;
+        if (bf.mem == SVP_MEM_HOST_PINNED) {
+            if (rd) j->host_in_bytes += need;
+            if (wr) j->host_out_bytes += need;
+        }
+    }
+    switch (j->kernel) {
+        case K_VECADD:
+        case K_SAXPY: j->alg_bytes = 12.0 * j->n; break;
+        case K_HIST256: j->alg_bytes = (double)j->n + (j->n ? 1024.0 : 0.0); break;
+        case K_BLACKSCHOLES: j->alg_bytes = 20.0 * j->n; break;
+        default:
+            j->alg_bytes = 4.0 * ((double)j->M * j->K + (double)j->K * j->N +
+                                  (double)j->M * j->N * (j->f1 != 0.f ? 2 : 1));
+            j->flops = 2.0 * j->M * j->N * (double)j->K;
+    }
+    j->shape_key = (j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32)
+                       ? (((uint64_t)j->M << 42) | ((uint64_t)j->N << 21) | (uint64_t)j->K)
+                       : 0;
+    double cost = c->cost.kernel_ns(j->kernel, j->alg_bytes, j->flops);
+    j->device = dispatch_vp(c, j->vp, cost);
+    if (c->exec && c->cfg.validate_ptrs && !empty) {
+        for (int b = 0; b < j->nbufs; ++b) {
+            std::string why;
+            if (executor_check_ptr(c->exec, j->bufs[b].ptr, j->bufs[b].mem, j->device, &why) != SVP_OK)
+                return fail(SVP_E_INVAL, "svp_submit: buffer " + std::to_string(b) + ": " + why);
+        }
+    }
+    return SVP_OK;
+}
+
+// ------------------------------------------------------------------ Job Dispatcher (a3)
+int32_t dispatch_vp(Ctx* c, int32_t vp, double cost) {
+    std::lock_guard<std::mutex> lk(c->dmu);
+    auto it = c->vp_dev.find(vp);
+    if (it != c->vp_dev.end()) return it->second;
+    int32_t best = 0;
+    for (int32_t g = 1; g < c->ngpu; ++g)
+        if (c->dev_load[g] < c->dev_load[best]) best = g;
+    c->vp_dev[vp] = best;
+    c->dev_load[best] += cost > 0 ? cost : 1.0;
+    return best;
+}
+
+void lpt_stratified(int32_t n, const int32_t* classes, const double* costs, int32_t G, const double* init_load,
+                    int32_t* out) {
+    std::vector<double> load(init_load, init_load + G);
+    std::map<int32_t, std::vector<int32_t>> by_class;
+    for (int32_t i = 0; i < n; ++i) by_class[classes[i]].push_back(i);
+    for (auto& kv : by_class) {
+        auto& items = kv.second;
+        std::stable_sort(items.begin(), items.end(), [&](int32_t a, int32_t b) {
+            if (costs[a] != costs[b]) return costs[a] > costs[b];
+            return a < b;
+        });
+        std::vector<double> cload(G, 0.0);
+        for (int32_t i : items) {
+            int32_t best = 0;
+            for (int32_t g = 1; g < G; ++g) {
+                if (std::tie(cload[g], load[g]) < std::tie(cload[best], load[best])) best = g;
+            }
+            out[i] = best;
+            cload[best] += costs[i];
+            load[best] += costs[i];
+        }
+    }
+}
+
+// ------------------------------------------------------------------ Re-scheduler (a4)
+static void split_group(const Ctx* c, const Flush& f, const Group& g, int nchunks, std::vector<std::vector<int32_t>>& out) {
+    // contiguous parts with balanced bytes (staged + algorithmic), members keep vp order
+    std::vector<double> w;
+    double tot = 0;
+    for (int32_t ji : g.jobs) {
+        const Job& j = f.jobs[ji];
+        double x = (double)j.host_in_bytes + (double)j.host_out_bytes + j.alg_bytes + j.flops * 0.05 + 1.0;
+        w.push_back(x);
+        tot += x;
+    }
+    (void)c;
+    out.clear();
+    size_t m = g.jobs.size();
+    nchunks = std::max(1, std::min<int>(nchunks, (int)m));
+    double target = tot / nchunks, acc = 0;
+    std::vector<int32_t> cur;
+    for (size_t k = 0; k < m; ++k) {
+        cur.push_back(g.jobs[k]);
+        acc += w[k];
+        size_t left_items = m - k - 1;
+        int left_chunks = nchunks - (int)out.size() - 1;
+        bool cut = acc >= target * (out.size() + 1) - 1e-9;
+        if ((cut && left_chunks > 0 && left_items >= (size_t)left_chunks) || (left_items == (size_t)left_chunks && left_chunks > 0)) {
+            out.push_back(cur);
+            cur.clear();
+        }
+    }
+    if (!cur.empty()) out.push_back(cur);
+}
+
+static void estimate_chunk(const Ctx* c, const Flush& f, Chunk& ch) {
+    int nin = 0, nout = 0;
+    ch.in_bytes = ch.out_bytes = 0;
+    ch.alg_bytes = ch.flops = 0;
+    for (int32_t ji : ch.jobs) {
+        const Job& j = f.jobs[ji];
+        ch.in_bytes += j.host_in_bytes;
+        ch.out_bytes += j.host_out_bytes;
+        ch.alg_bytes += j.alg_bytes;
+        ch.flops += j.flops;
+        for (int b = 0; b < j.nbufs; ++b) {
+            if (j.bufs[b].mem != SVP_MEM_HOST_PINNED) continue;
+            if (j.bufs[b].dir & SVP_DIR_IN) ++nin;
+            if (j.bufs[b].dir & SVP_DIR_OUT) ++nout;
+        }
+    }
+    ch.t_in = c->cost.h2d_ns(ch.in_bytes, nin);
+    ch.t_k = c->cost.kernel_ns(ch.kernel, ch.alg_bytes, ch.flops);
+    ch.t_out = c->cost.d2h_ns(ch.out_bytes, nout);
+}
+
+static uint64_t staged_bytes(const Flush& f, const std::vector<int32_t>& jobs) {
+    uint64_t s = 0;
+    for (int32_t ji : jobs) {
+        const Job& j = f.jobs[ji];
+        for (int b = 0; b < j.nbufs; ++b)
+            if (j.bufs[b].mem == SVP_MEM_HOST_PINNED) s += (touched_bytes(j, b) + 255) & ~255ull;
+    }
+    return s;
+}
+
+svp_status plan_flush(Ctx* c, Flush* f) {
+    // ---- levels (program order per VP)
+    std::unordered_map<int32_t, int32_t> next_level;
+    f->levels = 0;
+    for (auto& j : f->jobs) {
+        j.level = next_level[j.vp]++;
+        f->levels = std::max(f->levels, j.level + 1);
+    }
+    const int S = c->cfg.streams_per_gpu;
+    const bool inter = c->cfg.interleave != 0;
+    const bool coal = c->cfg.coalesce != 0;
+
+    // ---- Kernel Match (a2): groups per (level, device, kernel, shape)
+    typedef std::tuple<int32_t, int32_t, int32_t, uint64_t> Key;
+    std::map<Key, int32_t> gidx;
+    std::vector<int32_t> order(f->jobs.size());
+    std::iota(order.begin(), order.end(), 0);
+    if (coal) {
+        std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+            const Job &x = f->jobs[a], &y = f->jobs[b];
+            return std::tie(x.level, x.device, x.kernel, x.shape_key, x.vp) <
+                   std::tie(y.level, y.device, y.kernel, y.shape_key, y.vp);
+        });
+        for (int32_t ji : order) {
+            const Job& j = f->jobs[ji];
+            Key k{j.level, j.device, j.kernel, j.shape_key};
+            auto it = gidx.find(k);
+            if (it == gidx.end()) {
+                Group g;
+                g.kernel = j.kernel;
+                g.shape_key = j.shape_key;
+                g.level = j.level;
+                g.device = j.device;
+                gidx[k] = (int32_t)f->groups.size();
+                f->groups.push_back(g);
+                it = gidx.find(k);
+            }
+            f->groups[it->second].jobs.push_back(ji);
+        }
+    } else {
+        // no coalescing: one group per job, submission order within a level
+        std::stable_sort(order.begin(), order.end(),
+                         [&](int32_t a, int32_t b) { return f->jobs[a].level < f->jobs[b].level; });
+        for (int32_t ji : order) {
+            const Job& j = f->jobs[ji];
+            Group g;
+            g.kernel = j.kernel;
+            g.shape_key = j.shape_key;
+            g.level = j.level;
+            g.device = j.device;
+            g.jobs.push_back(ji);
+            f->groups.push_back(g);
+        }
+    }
+
+    // ---- chunking + estimates
+    const uint64_t arena = c->cfg.arena_bytes;
+    for (int32_t gi = 0; gi < (int32_t)f->groups.size(); ++gi) {
+        const Group& g = f->groups[gi];
+        Chunk whole;
+        whole.kernel = g.kernel;
+        whole.jobs = g.jobs;
+        estimate_chunk(c, *f, whole);
+        int nch = 1;
+        bool staged = whole.in_bytes + whole.out_bytes > 0;
+        if (staged && inter) {
+            // c* ~ sqrt((sum T - max T) / T_o)  (Eq 7 pipeline gain vs Eq 9 per-launch overhead)
+            double sum = whole.t_in + whole.t_k + whole.t_out;
+            double mx = std::max(whole.t_in, std::max(whole.t_k, whole.t_out));
+            double To = c->cost.launch_ns + 2 * c->cost.copy_ns;
+            nch = (int)lround(sqrt(std::max(0.0, sum - mx) / To));
+            nch = std::max(1, std::min(nch, c->cfg.max_chunks));
+        }
+        nch = std::min<int>(nch, (int)g.jobs.size());
+        std::vector<std::vector<int32_t>> parts;
+        for (;;) {
+            split_group(c, *f, g, nch, parts);
+            uint64_t mx = 0;
+            for (auto& p : parts) mx = std::max(mx, staged_bytes(*f, p));
+            if (mx <= arena / 2 || nch >= (int)g.jobs.size()) {
+                if (mx > arena) {
+                    set_error("svp_flush: a job's host-resident buffers exceed the staging arena");
+                    return SVP_E_NOMEM;
+                }
+                break;
+            }
+            nch = std::min<int>((int)g.jobs.size(), nch * 2);
+        }
+        for (size_t p = 0; p < parts.size(); ++p) {
+            Chunk ch;
+            ch.group = gi;
+            ch.index = (int32_t)p;
+            ch.device = g.device;
+            ch.level = g.level;
+            ch.kernel = g.kernel;
+            ch.jobs = parts[p];
+            estimate_chunk(c, *f, ch);
+            ch.arena_len = staged_bytes(*f, ch.jobs);
+            f->chunks.push_back(std::move(ch));
+        }
+    }
+
+    // ---- order per (level, device): Johnson's rule on (Tin+Tk, Tk+Tout) when interleaving
+    std::vector<int32_t> corder(f->chunks.size());
+    std::iota(corder.begin(), corder.end(), 0);
+    auto johnson_key = [&](int32_t ci) {
+        const Chunk& ch = f->chunks[ci];
+        double a = ch.t_in + ch.t_k, b = ch.t_k + ch.t_out;
+        bool first = a < b;
+        // first set: ascending a; second set: descending b; ties by (group, index)
+        return std::make_tuple(first ? 0 : 1, first ? a : -b, ch.group, ch.index);
+    };
+    std::stable_sort(corder.begin(), corder.end(), [&](int32_t x, int32_t y) {
+        const Chunk &a = f->chunks[x], &b = f->chunks[y];
+        if (a.level != b.level) return a.level < b.level;
+        if (!inter) return std::tie(a.group, a.index) < std::tie(b.group, b.index);
+        return johnson_key(x) < johnson_key(y);
+    });
+
+    // ---- ops, streams, dependencies, arena slots
+    std::unordered_map<int32_t, int32_t> vp_last_op;       // per VP: last op of its previous job
+    struct Slot { uint64_t off, len; int32_t release_op; };
+    std::vector<std::vector<Slot>> inflight(c->ngpu);
+    std::vector<uint64_t> arena_head(c->ngpu, 0);
+    std::vector<int32_t> rr(c->ngpu, 0);
+    for (int32_t ci : corder) {
+        Chunk& ch = f->chunks[ci];
+        const int dev = ch.device;
+        std::vector<int32_t> prev;
+        for (int32_t ji : ch.jobs) {
+            auto it = vp_last_op.find(f->jobs[ji].vp);
+            if (it != vp_last_op.end()) prev.push_back(it->second);
+        }
+        // arena slot (ring) -- waits for the ops that release overlapped regions
+        std::vector<int32_t> arena_waits;
+        if (ch.arena_len) {
+            uint64_t off = arena_head[dev];
+            if (off + ch.arena_len > arena) off = 0;
+            auto& fl = inflight[dev];
+            for (size_t k = 0; k < fl.size();) {
+                bool overlap = fl[k].off < off + ch.arena_len && off < fl[k].off + fl[k].len;
+                if (overlap) {
+                    arena_waits.push_back(fl[k].release_op);
+                    fl.erase(fl.begin() + k);
+                } else {
+                    ++k;
+                }
+            }
+            ch.arena_off = off;
+            arena_head[dev] = off + ch.arena_len;
+        }
+        int cs = inter ? (rr[dev]++ % S) : 0;
+        int sh2d = inter ? S : 0, sd2h = inter ? S + 1 : 0;
+        int32_t first_op = (int32_t)f->ops.size();
+        int32_t k_op = -1, last = -1;
+        if (ch.in_bytes) {
+            Op o;
+            o.kind = SVP_OP_H2D;
+            o.chunk = ci;
+            o.device = dev;
+            o.stream = sh2d;
+            o.wait_ops = prev;
+            o.wait_ops.insert(o.wait_ops.end(), arena_waits.begin(), arena_waits.end());
+            o.est_ns = ch.t_in;
+            o.bytes = ch.in_bytes;
+            f->ops.push_back(o);
+            last = (int32_t)f->ops.size() - 1;
+        }
+        {
+            Op o;
+            o.kind = SVP_OP_KERNEL;
+            o.chunk = ci;
+            o.device = dev;
+            o.stream = cs;
+            if (last >= 0) o.wait_ops.push_back(last);
+            else {
+                o.wait_ops = prev;
+                o.wait_ops.insert(o.wait_ops.end(), arena_waits.begin(), arena_waits.end());
+            }
+            o.est_ns = ch.t_k;
+            o.bytes = (uint64_t)ch.alg_bytes;
+            o.flops = ch.flops;
+            f->ops.push_back(o);
+            last = k_op = (int32_t)f->ops.size() - 1;
+        }
+        if (ch.out_bytes) {
+            Op o;
+            o.kind = SVP_OP_D2H;
+            o.chunk = ci;
+            o.device = dev;
+            o.stream = sd2h;
+            o.wait_ops.push_back(k_op);
+            o.est_ns = ch.t_out;
+            o.bytes = ch.out_bytes;
+            f->ops.push_back(o);
+            last = (int32_t)f->ops.size() - 1;
+        }
+        (void)first_op;
+        f->ops[last].last_of_job = true;
+        for (int32_t ji : ch.jobs) vp_last_op[f->jobs[ji].vp] = last;
+        if (ch.arena_len) inflight[dev].push_back(Slot{ch.arena_off, ch.arena_len, last});
+    }
+    // dependencies on the same stream that precede in issue order are implicit; keep
+    // only cross-stream waits, and mark the ops somebody waits on
+    for (size_t i = 0; i < f->ops.size(); ++i) {
+        Op& o = f->ops[i];
+        std::vector<int32_t> w;
+        for (int32_t p : o.wait_ops) {
+            if (p < 0 || p >= (int32_t)i) continue;
+            const Op& q = f->ops[p];
+            if (q.device == o.device && q.stream == o.stream) continue;
+            if (std::find(w.begin(), w.end(), p) == w.end()) w.push_back(p);
+        }
+        o.wait_ops.swap(w);
+        for (int32_t p : o.wait_ops) f->ops[p].needs_event = true;
+    }
+    return SVP_OK;
+}
+
+// ------------------------------------------------------------------ plan simulation
+// Engines per GPU (Fig 3): H2D copy engine, D2H copy engine, compute engine (coalesced
+// kernels that fill the GPU serialize).  An op starts when its engine, its stream and
+// every op it waits on are free.
+void simulate(Ctx* c, Flush* f, double* makespan, double* serial) {
+    const int S = c->cfg.streams_per_gpu + 2;
+    std::vector<double> eng(c->ngpu * 3, 0.0), strm(c->ngpu * S, 0.0);
+    double ms = 0, ser = 0;
+    for (auto& o : f->ops) {
+        int e = o.device * 3 + (o.kind == SVP_OP_H2D ? 0 : o.kind == SVP_OP_KERNEL ? 1 : 2);
+        double t = std::max(eng[e], strm[o.device * S + o.stream]);
+        for (int32_t p : o.wait_ops) t = std::max(t, f->ops[p].sim_end);
+        o.sim_start = t;
+        o.sim_end = t + o.est_ns;
+        eng[e] = strm[o.device * S + o.stream] = o.sim_end;
+        ms = std::max(ms, o.sim_end);
+        ser += o.est_ns;
+    }
+    // same-stream predecessors implicitly ordered (already via strm); done
+    *makespan = ms;
+    *serial = ser;
+}
+
+}  // namespace svp

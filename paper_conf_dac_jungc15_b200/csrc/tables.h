@@ -1,0 +1,53 @@
+// tables.h -- device-resident work tables shared by the executor (host) and the
+// guest kernels (device).  Internal to libsvp; not part of the C-ABI.
+//
+// Kernel Coalescing (Fig 5/6) merges the identical kernel calls of
+// several VPs into one launch over "one bigger piece of data".  Instead of physically
+// gathering every VP's chunk into contiguous memory, a coalesced launch reads a
+// segment table: segment i = one VP's job (its buffer bases, element count, scalar
+// args) and owns tiles [tile_begin_i, tile_begin_{i+1}) of the launch's tile space.
+// Ragged sizes need no padding: a VP's last tile is partial and predicated.
+#pragma once
+#include <stdint.h>
+
+namespace svp {
+
+// Elementwise / histogram segment: 64 bytes.
+struct SegDesc {
+    uint64_t ptr[5];      // buffer base addresses in kernel order (device)
+    uint64_t n;           // elements (bytes for hist256)
+    uint32_t tile_begin;  // first tile of this segment in the launch
+    uint16_t shift;       // virtual-index shift: elements between the previous 16-B
+                          // boundary and ptr[0] (tiles are aligned in address space)
+    uint16_t flags;       // SEG_SCALAR: buffers not co-aligned mod 16 -> scalar path only
+    float f[2];           // per-VP scalars (SAXPY a; Black-Scholes R, V)
+};
+static_assert(sizeof(SegDesc) == 64, "SegDesc must be 64 B");
+enum : uint16_t { SEG_SCALAR = 1 };
+
+// Grouped SGEMM: one entry per VP; tensor maps live in a separate 64-B aligned array
+// (2 per VP: A then B).
+struct GemmDesc {
+    float* C;
+    int32_t M, N, K;
+    float alpha, beta;
+    uint32_t tile_begin;  // first output tile of this VP
+    uint32_t tiles_n;     // tiles along N
+    uint32_t _pad[7];
+};
+static_assert(sizeof(GemmDesc) == 64, "GemmDesc must be 64 B");
+
+// Tile geometry (elements per tile) -- host planner and kernels must agree.
+constexpr int kEwThreads = 256;
+constexpr int kVecaddVec = 4;                                  // float4 per thread per array
+constexpr int kVecaddTile = kEwThreads * 4 * kVecaddVec;       // 4096 elements
+constexpr int kSaxpyTile = kVecaddTile;
+constexpr int kBsVec = 2;
+constexpr int kBsTile = kEwThreads * 4 * kBsVec;               // 2048 options
+constexpr int kHistThreads = 256;
+constexpr int kHistVec = 4;                                    // uint4 (16 B) per thread
+constexpr int kHistTile = kHistThreads * 16 * kHistVec;        // 16384 bytes
+constexpr int kGemmBM = 128, kGemmBN = 128, kGemmBK = 32;
+constexpr int kTf32BM = 128, kTf32BN = 256, kTf32BK = 32;
+
+}  // namespace svp

@@ -1,0 +1,163 @@
+"""libsvp C-ABI: the library loads, exports every symbol include/svp.h declares, and
+rejects bad requests with the documented status codes (CPU only: dry-run contexts)."""
+import os
+import re
+
+import pytest
+import torch
+
+from paper_conf_dac_jungc15_b200 import svp
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _header_functions():
+    src = open(os.path.join(ROOT, "include", "svp.h")).read()
+    decl = r"^\s*(?:svp_status|void|const char\s*\*|int32_t)\s*(svp_[a-z_]+)\s*\("
+    return sorted(set(re.findall(decl, src, flags=re.M)))
+
+
+def test_library_exports_every_declared_symbol():
+    L = svp.load()
+    declared = _header_functions()
+    assert set(declared) == set(svp.EXPORTS), (set(declared) ^ set(svp.EXPORTS))
+    for name in declared:
+        assert hasattr(L, name), name
+    assert L.svp_abi_version() == 1
+
+
+def test_lib_is_the_in_tree_build():
+    L = svp.load()
+    assert os.path.dirname(os.path.abspath(L._name)) == os.path.join(ROOT, "paper_conf_dac_jungc15_b200")
+
+
+def test_config_default():
+    cfg = svp.svp_config()
+    svp.load().svp_config_default(cfg)
+    assert cfg.streams_per_gpu == 4 and cfg.coalesce == 1 and cfg.interleave == 1 and cfg.max_chunks == 8
+    assert cfg.validate_ptrs == 1 and cfg.dry_run == 0
+
+
+@pytest.mark.skipif(torch.cuda.is_available(), reason="needs a host without GPUs")
+def test_init_without_gpu_fails_loudly():
+    with pytest.raises(svp.SvpError) as e:
+        svp.Context()
+    assert e.value.status == svp.SVP_E_CUDA
+
+
+def test_init_rejects_bad_config():
+    with pytest.raises(svp.SvpError) as e:
+        svp.Context(dry_run=True, streams_per_gpu=0)
+    assert e.value.status == svp.SVP_E_INVAL
+
+
+def test_register_kernels():
+    with svp.Context(dry_run=True) as c:
+        ids = [c.register_kernel(k) for k in ("vecadd", "saxpy", "hist256", "blackscholes", "sgemm")]
+        assert len(set(ids)) == 5
+        assert c.register_kernel("vecadd") == ids[0]  # idempotent
+        with pytest.raises(svp.SvpError) as e:
+            c.register_kernel("conv2d")
+        assert e.value.status == svp.SVP_E_NOKERNEL
+
+
+FAKE = 0x7F0000000000  # dry-run contexts never touch buffers
+
+
+def _vecadd_bufs(n, mem=svp.MEM_DEVICE, bytes_=None):
+    b = 4 * n if bytes_ is None else bytes_
+    return [(FAKE, b, svp.DIR_IN, mem), (FAKE + 2**30, b, svp.DIR_IN, mem), (FAKE + 2**31, b, svp.DIR_OUT, mem)]
+
+
+@pytest.mark.parametrize("case,status", [
+    ("wrong_nbufs", svp.SVP_E_INVAL), ("wrong_dir", svp.SVP_E_INVAL), ("too_small", svp.SVP_E_INVAL),
+    ("bad_vp", svp.SVP_E_INVAL), ("unregistered", svp.SVP_E_NOKERNEL), ("short_args", svp.SVP_E_INVAL),
+    ("null_ptr", svp.SVP_E_INVAL), ("bad_mem", svp.SVP_E_INVAL), ("sgemm_k", svp.SVP_E_UNSUPPORTED),
+    ("sgemm_beta_out", svp.SVP_E_INVAL), ("sgemm_misaligned", svp.SVP_E_UNSUPPORTED),
+])
+def test_submit_validation(case, status):
+    with svp.Context(dry_run=True) as c:
+        va = c.register_kernel("vecadd")
+        sg = c.register_kernel("sgemm")
+        n = 1000
+        vp, kid, args, bufs = 0, va, svp.args_vecadd(n), _vecadd_bufs(n)
+        if case == "wrong_nbufs":
+            bufs = bufs[:2]
+        elif case == "wrong_dir":
+            bufs[2] = (bufs[2][0], bufs[2][1], svp.DIR_IN, svp.MEM_DEVICE)
+        elif case == "too_small":
+            bufs = _vecadd_bufs(n, bytes_=4 * n - 4)
+        elif case == "bad_vp":
+            vp = 1 << 20
+        elif case == "unregistered":
+            kid = 3
+        elif case == "short_args":
+            args = b"\x01\x00"
+        elif case == "null_ptr":
+            bufs[0] = (0, 4 * n, svp.DIR_IN, svp.MEM_DEVICE)
+        elif case == "bad_mem":
+            bufs[1] = (bufs[1][0], bufs[1][1], svp.DIR_IN, 7)
+        elif case.startswith("sgemm"):
+            kid = sg
+            M, N, K = 64, 64, 64
+            beta = 0.0
+            dirc = svp.DIR_OUT
+            base = FAKE
+            if case == "sgemm_k":
+                K = 30
+            if case == "sgemm_beta_out":
+                beta = 1.0
+            if case == "sgemm_misaligned":
+                base = FAKE + 4
+            args = svp.args_sgemm(M, N, K, 1.0, beta)
+            bufs = [(base, 4 * M * K, svp.DIR_IN, 0), (FAKE + 2**30, 4 * K * N, svp.DIR_IN, 0),
+                    (FAKE + 2**31, 4 * M * N, dirc, 0)]
+        with pytest.raises(svp.SvpError) as e:
+            c.submit(vp, kid, args, bufs)
+        assert e.value.status == status, svp.last_error()
+        assert svp.last_error()
+
+
+def test_zero_sized_jobs_are_legal():
+    with svp.Context(dry_run=True) as c:
+        va = c.register_kernel("vecadd")
+        c.submit(0, va, svp.args_vecadd(0), [(0, 0, 1, 0), (0, 0, 1, 0), (0, 0, 2, 0)])
+        c.flush()
+        assert c.flush_stats()["jobs"] == 1
+
+
+def test_batch_is_all_or_nothing():
+    with svp.Context(dry_run=True) as c:
+        va = c.register_kernel("vecadd")
+        good = (0, va, svp.args_vecadd(10), _vecadd_bufs(10))
+        bad = (1, va, svp.args_vecadd(10), _vecadd_bufs(10)[:2])
+        with pytest.raises(svp.SvpError):
+            c.submit_batch([good, bad])
+        c.flush()
+        assert c.flush_stats()["jobs"] == 0
+        ids = c.submit_batch([good, (1, va, svp.args_vecadd(10), _vecadd_bufs(10))])
+        assert ids[1] == ids[0] + 1
+
+
+def test_thread_safe_concurrent_submit():
+    from concurrent.futures import ThreadPoolExecutor
+    with svp.Context(dry_run=True) as c:
+        va = c.register_kernel("vecadd")
+
+        def worker(vp):
+            for _ in range(50):
+                c.submit(vp, va, svp.args_vecadd(100), _vecadd_bufs(100))
+
+        with ThreadPoolExecutor(8) as ex:
+            list(ex.map(worker, range(16)))
+        c.flush()
+        st = c.flush_stats()
+        assert st["jobs"] == 800 and st["levels"] == 50
+        assert st["launches"] == 50  # one coalesced launch per level
+
+
+def test_lpt_partition_pure():
+    out = svp.lpt_partition([1, 1, 1, 1], [5.0, 5.0, 5.0, 5.0], 2)
+    assert out == [0, 1, 0, 1]
+    with pytest.raises(svp.SvpError):
+        svp.lpt_partition([1], [1.0], 0)

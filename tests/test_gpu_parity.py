@@ -1,0 +1,196 @@
+"""GPU parity: every VP's output from the coalesced / interleaved sm_100a path equals
+the oracle (bit-exact for integer-like kernels, stated tolerance for fp32), through
+the C-ABI, for device- and host-resident buffers, serial and coalesced modes."""
+import dataclasses
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import workloads as W
+from gpu_common import check_job, inputs_for, run_svp
+from paper_conf_dac_jungc15_b200 import svp
+from paper_conf_dac_jungc15_b200.vpset import VPSet
+
+pytestmark = pytest.mark.gpu
+
+MODES = {
+    "coalesced_interleaved": dict(coalesce=True, interleave=True),
+    "coalesced_1stream": dict(coalesce=True, interleave=False),
+    "serial_sync": dict(coalesce=False, interleave=False, sync_each_job=True),
+}
+
+
+@pytest.fixture(scope="module")
+def small():
+    specs = W.mixed_small(nvps=30, max_n=70000)
+    return specs, inputs_for(specs)
+
+
+@pytest.mark.parametrize("mode", list(MODES))
+@pytest.mark.parametrize("residency", ["device", "host"])
+def test_mixed_small(small, mode, residency):
+    specs, inputs = small
+    outs, prof, st = run_svp(specs, inputs, residency, **MODES[mode])
+    for s, inp, got in zip(specs, inputs, outs):
+        check_job(s, inp, got)
+    if mode == "serial_sync":
+        assert st["launches"] == len(specs)   # one launch op per job, no coalescing
+    else:
+        assert st["groups"] < len(specs)
+
+
+def test_coalesced_bit_identical_to_serial(small):
+    """T5: the same kernel code on one segment or many gives identical bits (per-element /
+    per-tile op order does not depend on coalescing)."""
+    specs, inputs = small
+    a, _, _ = run_svp(specs, inputs, "device", coalesce=True)
+    b, _, _ = run_svp(specs, inputs, "device", coalesce=False, interleave=False)
+    for s, x, y in zip(specs, a, b):
+        for k in x:
+            assert np.array_equal(x[k].view(np.uint32) if x[k].dtype == np.float32 else x[k],
+                                  y[k].view(np.uint32) if y[k].dtype == np.float32 else y[k]), (s.vp, s.kernel, k)
+
+
+@pytest.mark.parametrize("residency", ["device", "host"])
+def test_config4_ragged_full_size(residency):
+    """BASELINE config 4: 64 VPs, ragged 64Ki..16Mi + adversarial sizes, misaligned views."""
+    specs = W.config_specs(4)
+    for s in specs[8:16]:
+        s.misalign = 2 if s.vp % 2 else 1
+    inputs = inputs_for(specs)
+    outs, _, st = run_svp(specs, inputs, residency)
+    assert st["groups"] == 4
+    want = oracle.run_jobs(specs, inputs)
+    for s, inp, got, w in zip(specs, inputs, outs, want):
+        check_job(s, inp, got, w)
+
+
+def test_config3_interleaved_host():
+    specs = W.config_specs(3, scale=4)
+    inputs = inputs_for(specs)
+    outs, prof, st = run_svp(specs, inputs, "host", profile_level=1)
+    assert st["chunks"] > st["groups"]
+    want = oracle.run_jobs(specs, inputs)
+    for s, inp, got, w in zip(specs, inputs, outs, want):
+        check_job(s, inp, got, w)
+
+
+@pytest.mark.parametrize("int_inputs", [True, False])
+def test_config2_sgemm_512(int_inputs):
+    specs = W.config_specs(2, sgemm_int=int_inputs)
+    inputs = inputs_for(specs)
+    outs, _, st = run_svp(specs, inputs, "device")
+    assert st["launches"] == 1
+    want = oracle.run_jobs(specs, inputs)
+    for s, inp, got, w in zip(specs, inputs, outs, want):
+        check_job(s, inp, got, w)
+
+
+def test_sgemm_alpha_beta_ragged_edges():
+    specs = []
+    for v, (M, N, K) in enumerate([(200, 136, 40), (200, 136, 40), (1, 4, 4), (129, 260, 0), (64, 68, 1000)]):
+        specs.append(W.JobSpec(v, "sgemm", M=M, N=N, K=K, alpha=1.5, beta=-0.5))
+    inputs = inputs_for(specs)
+    outs, _, _ = run_svp(specs, inputs, "device")
+    for s, inp, got in zip(specs, inputs, outs):
+        check_job(s, inp, got)
+
+
+def test_program_order_chain():
+    """A VP's jobs run in program order: vecadd writes c, then SAXPY reads c as x and
+    updates y in place, then SAXPY again -- one flush."""
+    n = 100003
+    ctx = svp.Context(num_gpus=1)
+    va, sx = ctx.register_kernel("vecadd"), ctx.register_kernel("saxpy")
+    jobs, expect, bufs = [], [], []
+    for vp in range(6):
+        g = W.rng(9, vp, 1)
+        a, b, y = (W.uniform_f32(g, n, -1, 1) for _ in range(3))
+        ta, tb, ty = (torch.from_numpy(x).cuda() for x in (a, b, y))
+        tc = torch.empty_like(ta)
+        bufs.append((ta, tb, tc, ty))
+        c = oracle.vecadd(a, b)
+        y1 = oracle.saxpy(0.5 + vp, c, y)
+        y2 = oracle.saxpy(-2.0, c, y1)
+        expect.append((c, y2))
+        p = lambda t: t.data_ptr()
+        jobs.append((vp, va, svp.args_vecadd(n), [(p(ta), 4 * n, 1, 0), (p(tb), 4 * n, 1, 0), (p(tc), 4 * n, 2, 0)]))
+        jobs.append((vp, sx, svp.args_saxpy(n, 0.5 + vp), [(p(tc), 4 * n, 1, 0), (p(ty), 4 * n, 3, 0)]))
+        jobs.append((vp, sx, svp.args_saxpy(n, -2.0), [(p(tc), 4 * n, 1, 0), (p(ty), 4 * n, 3, 0)]))
+    ctx.submit_batch(jobs)
+    ctx.flush()
+    assert ctx.flush_stats()["levels"] == 3
+    for (ta, tb, tc, ty), (c, y2) in zip(bufs, expect):
+        assert np.array_equal(tc.cpu().numpy(), c)
+        assert np.array_equal(ty.cpu().numpy(), y2)
+    ctx.close()
+
+
+def test_profiler_conservation_and_kernel_stats(small):
+    specs, inputs = small
+    ctx = svp.Context(num_gpus=1, profile_level=1)
+    vs = VPSet(ctx, specs, inputs, "host")
+    vs.submit()
+    ctx.flush()
+    ops = ctx.plan()
+    tot = ctx.profile(-1)
+    per = [ctx.profile(s.vp) for s in specs]
+    k_meas = sum(op["measured_ns"] for op in ops if op["kind"] == svp.OP_KERNEL)
+    h_meas = sum(op["measured_ns"] for op in ops if op["kind"] == svp.OP_H2D)
+    assert all(op["measured_ns"] >= 0 for op in ops)
+    assert sum(p["kernel_ns"] for p in per) == pytest.approx(k_meas, rel=1e-9)
+    assert sum(p["h2d_ns"] for p in per) == pytest.approx(h_meas, rel=1e-9)
+    assert tot["kernel_ns"] == pytest.approx(k_meas, rel=1e-9)
+    assert sum(p["jobs"] for p in per) == len(specs)
+    n_launch = sum(ctx.kernel_stats(k)["launches"] for k in vs.kids.values())
+    assert n_launch == sum(1 for op in ops if op["kind"] == svp.OP_KERNEL)
+    st = ctx.flush_stats()
+    assert 0 < st["device_ns"] <= st["host_total_ns"]
+    ctx.close()
+
+
+def test_external_stream_join(small):
+    specs, inputs = small
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        ctx = svp.Context(num_gpus=1, external_streams=[s.cuda_stream])
+        vs = VPSet(ctx, specs[:10], inputs[:10], "device")
+        vs.submit()
+        ctx.flush()
+        s.synchronize()
+        for i, (sp, inp) in enumerate(zip(specs[:10], inputs[:10])):
+            check_job(sp, inp, vs.output(i))
+        ctx.close()
+
+
+def test_residency_validation():
+    ctx = svp.Context(num_gpus=1)
+    va = ctx.register_kernel("vecadd")
+    n = 1024
+    pageable = torch.empty(n, dtype=torch.float32)
+    dev = torch.empty(n, dtype=torch.float32, device="cuda")
+    with pytest.raises(svp.SvpError) as e:
+        ctx.submit(0, va, svp.args_vecadd(n), [(pageable.data_ptr(), 4 * n, 1, 1)] * 2 + [(dev.data_ptr(), 4 * n, 2, 0)])
+    assert e.value.status == svp.SVP_E_INVAL
+    with pytest.raises(svp.SvpError) as e:
+        ctx.submit(0, va, svp.args_vecadd(n), [(dev.data_ptr(), 4 * n, 1, 1)] * 2 + [(dev.data_ptr(), 4 * n, 2, 0)])
+    assert e.value.status == svp.SVP_E_INVAL
+    ctx.close()
+
+
+def test_repeated_flushes_reuse_tables(small):
+    specs, inputs = small
+    ctx = svp.Context(num_gpus=1)
+    vs = VPSet(ctx, specs, inputs, "device")
+    uploads = []
+    for r in range(3):
+        vs.load_inputs()
+        vs.submit()
+        ctx.flush()
+        uploads.append(ctx.flush_stats()["table_uploads"])
+        for i, (s, inp) in enumerate(zip(specs, inputs)):
+            check_job(s, inp, vs.output(i))
+    assert uploads[0] == 1 and uploads[1] == 0 and uploads[2] == 0
+    ctx.close()

@@ -1,0 +1,238 @@
+"""Host logic of the hot path on CPU (dry-run contexts: no CUDA call at all).
+
+Kernel Match, Job Dispatcher and Re-scheduler decisions are read back through
+svp_plan_get and checked against oracle.sched (Johnson's rule, flow-shop makespan,
+LPT) and against the invariants the paper states (identical kernels coalesced,
+per-VP order kept, results divided back per VP)."""
+import itertools
+from collections import defaultdict
+
+import numpy as np
+import pytest
+
+from oracle import sched
+from paper_conf_dac_jungc15_b200 import svp
+
+FAKE = 0x7F0000000000
+KIND = {"vecadd": 3, "saxpy": 2, "hist256": 2, "blackscholes": 5, "sgemm": 3}
+
+
+def fake_bufs(kernel, n=0, M=0, N=0, K=0, mem=svp.MEM_DEVICE, vp=0):
+    base = FAKE + vp * (1 << 34)
+    if kernel == "vecadd":
+        return [(base, 4 * n, 1, mem), (base + 2**32, 4 * n, 1, mem), (base + 2**33, 4 * n, 2, mem)]
+    if kernel == "saxpy":
+        return [(base, 4 * n, 1, mem), (base + 2**32, 4 * n, 3, mem)]
+    if kernel == "hist256":
+        return [(base, n, 1, mem), (base + 2**32, 1024, 2, mem)]
+    if kernel == "blackscholes":
+        return [(base + i * 2**31, 4 * n, 1 if i < 3 else 2, mem) for i in range(5)]
+    if kernel == "sgemm":
+        return [(base, 4 * M * K, 1, mem), (base + 2**32, 4 * K * N, 1, mem), (base + 2**33, 4 * M * N, 2, mem)]
+
+
+def args_for(kernel, n=0, M=0, N=0, K=0):
+    return {"vecadd": lambda: svp.args_vecadd(n), "saxpy": lambda: svp.args_saxpy(n, 2.0),
+            "hist256": lambda: svp.args_hist256(n), "blackscholes": lambda: svp.args_blackscholes(n, 0.02, 0.3),
+            "sgemm": lambda: svp.args_sgemm(M, N, K)}[kernel]()
+
+
+def submit(c, vp, kernel, n=0, M=0, N=0, K=0, mem=svp.MEM_DEVICE):
+    kid = c.kernel(kernel)
+    return c.submit(vp, kid, args_for(kernel, n, M, N, K), fake_bufs(kernel, n, M, N, K, mem, vp))
+
+
+MIX = ("vecadd", "saxpy", "hist256", "blackscholes")
+
+
+def test_kernel_match_groups_identical_kernels():
+    with svp.Context(dry_run=True) as c:
+        for vp in range(64):
+            submit(c, vp, MIX[vp % 4], n=1000 + 37 * vp)  # ragged sizes are still "identical"
+        c.flush()
+        ops = c.plan()
+        st = c.flush_stats()
+        assert st["groups"] == 4 and st["launches"] == 4
+        seen = set()
+        for op in ops:
+            assert op["kind"] == svp.OP_KERNEL and op["nvps"] == 16
+            assert op["vps"] == sorted(op["vps"])                    # members in VP order (R12)
+            kname = [k for k in MIX if c.kernel_ids[k] == op["kernel"]][0]
+            assert all(MIX[v % 4] == kname for v in op["vps"])
+            seen |= set(op["vps"])
+        assert seen == set(range(64))
+
+
+def test_sgemm_needs_equal_shapes():
+    with svp.Context(dry_run=True) as c:
+        for vp in range(6):
+            s = 128 if vp < 4 else 256
+            submit(c, vp, "sgemm", M=s, N=s, K=s)
+        c.flush()
+        sizes = sorted(op["nvps"] for op in c.plan())
+        assert sizes == [2, 4]
+
+
+def test_no_coalescing_is_one_launch_per_job_in_submission_order():
+    with svp.Context(dry_run=True, coalesce=False, interleave=False) as c:
+        order = [5, 3, 9, 1]
+        for vp in order:
+            submit(c, vp, "vecadd", n=100)
+        c.flush()
+        ops = c.plan()
+        assert [op["vps"] for op in ops] == [[v] for v in order]
+        assert all(op["stream"] == 0 for op in ops)
+
+
+def test_program_order_levels_and_dependencies():
+    with svp.Context(dry_run=True) as c:
+        for vp in range(8):
+            submit(c, vp, "vecadd", n=10000, mem=svp.MEM_HOST_PINNED)
+            submit(c, vp, "saxpy", n=20000, mem=svp.MEM_HOST_PINNED)
+            submit(c, vp, "hist256", n=30000, mem=svp.MEM_HOST_PINNED)
+        c.flush()
+        ops = c.plan()
+        assert c.flush_stats()["levels"] == 3
+        per_vp = defaultdict(list)
+        for i, op in enumerate(ops):
+            for v in op["vps"]:
+                per_vp[v].append((i, op))
+        for v, lst in per_vp.items():
+            levels = [op["level"] for _, op in lst]
+            assert levels == sorted(levels)
+            # every op of level l starts after every op of level l-1 of the same VP ends
+            for (_, a), (_, b) in itertools.combinations(lst, 2):
+                if b["level"] > a["level"]:
+                    assert b["sim_start_ns"] >= a["sim_end_ns"] - 1e-6
+
+
+def _host_cfg_plan(c, nvps=32, n=1 << 20):
+    for vp in range(nvps):
+        submit(c, vp, MIX[vp % 4], n=n + 4096 * vp, mem=svp.MEM_HOST_PINNED)
+    c.flush()
+    return c.plan()
+
+
+def test_interleaving_streams_and_chunks():
+    S = 4
+    with svp.Context(dry_run=True, streams_per_gpu=S) as c:
+        ops = _host_cfg_plan(c)
+        st = c.flush_stats()
+        assert st["chunks"] > st["groups"]          # groups split for copy/compute overlap
+        kinds = defaultdict(set)
+        for op in ops:
+            kinds[op["kind"]].add(op["stream"])
+        assert kinds[svp.OP_H2D] == {S} and kinds[svp.OP_D2H] == {S + 1}
+        assert kinds[svp.OP_KERNEL] <= set(range(S)) and len(kinds[svp.OP_KERNEL]) > 1
+        # chunks of a group partition its members, contiguous in VP order
+        by_group = defaultdict(list)
+        for op in ops:
+            if op["kind"] == svp.OP_KERNEL:
+                by_group[op["group"]].append((op["chunk"], op["vps"]))
+        for g, chunks in by_group.items():
+            members = [v for _, vs in sorted(chunks) for v in vs]
+            assert members == sorted(members) and len(set(members)) == len(members)
+        assert st["sim_makespan_ns"] < st["sim_serial_ns"]
+
+
+def _chunk_triples(ops):
+    t = {}
+    for op in ops:
+        key = (op["group"], op["chunk"])
+        t.setdefault(key, [0.0, 0.0, 0.0])
+        t[key][{svp.OP_H2D: 0, svp.OP_KERNEL: 1, svp.OP_D2H: 2}[op["kind"]]] = op["est_ns"]
+    return t
+
+
+def test_johnson_order_matches_oracle():
+    with svp.Context(dry_run=True) as c:
+        ops = _host_cfg_plan(c)
+        trip = _chunk_triples(ops)
+        canon = sorted(trip)                                   # (group, chunk) order = tie-break order
+        jobs = [tuple(trip[k]) for k in canon]
+        want = [canon[i] for i in sched.johnson_order(jobs)]
+        got = [(op["group"], op["chunk"]) for op in ops if op["kind"] == svp.OP_KERNEL]
+        assert got == want
+
+
+def test_simulated_makespan_is_flowshop_of_plan_order():
+    with svp.Context(dry_run=True) as c:
+        ops = _host_cfg_plan(c)
+        trip = _chunk_triples(ops)
+        order = [(op["group"], op["chunk"]) for op in ops if op["kind"] == svp.OP_KERNEL]
+        jobs = [tuple(trip[k]) for k in order]
+        assert all(a > 0 and b > 0 and cc > 0 for a, b, cc in jobs)
+        ms = c.flush_stats()["sim_makespan_ns"]
+        assert ms == pytest.approx(sched.flowshop_makespan(jobs), rel=1e-12)
+        assert c.flush_stats()["sim_serial_ns"] == pytest.approx(sched.serial_time(jobs), rel=1e-12)
+        if len(jobs) <= 7:
+            assert ms >= sched.best_makespan(jobs) - 1e-6
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_johnson_plan_optimal_when_copy_bound(seed):
+    """Small host-resident mixes (PCIe-bound: Tk << Tin, Tout) -- Johnson's 3-machine
+    condition holds, so the planned order is optimal (brute force over all orders)."""
+    g = np.random.default_rng(seed)
+    with svp.Context(dry_run=True, max_chunks=1) as c:
+        for vp in range(int(g.integers(2, 6))):
+            submit(c, vp, MIX[int(g.integers(0, 4))], n=int(g.integers(1, 40)) * 100000, mem=svp.MEM_HOST_PINNED)
+        c.flush()
+        ops = c.plan()
+        trip = _chunk_triples(ops)
+        jobs = [tuple(v) for v in trip.values()]
+        if min(j[0] for j in jobs) >= max(j[1] for j in jobs) or min(j[2] for j in jobs) >= max(j[1] for j in jobs):
+            assert c.flush_stats()["sim_makespan_ns"] == pytest.approx(sched.best_makespan(jobs), rel=1e-9)
+
+
+def test_dispatcher_shards_vps_across_gpus():
+    with svp.Context(dry_run=True, num_gpus=4) as c:
+        kids = [c.kernel(k) for k in MIX]
+        vps = list(range(64))
+        costs = [1000.0 + (v * 7919) % 97 for v in vps]
+        devs = c.assign_vps(vps, [kids[v % 4] for v in vps], costs)
+        for k in range(4):
+            cnt = np.bincount([devs[v] for v in vps if v % 4 == k], minlength=4)
+            assert cnt.max() - cnt.min() <= 1                 # every GPU gets its share of every class
+        assert all(c.vp_device(v) == devs[v] for v in vps)   # sticky
+        for vp in vps:
+            submit(c, vp, MIX[vp % 4], n=5000)
+        c.flush()
+        for op in c.plan():
+            assert all(devs[v] == op["device"] for v in op["vps"])
+        assert c.flush_stats()["launches"] == 16              # 4 kernels x 4 GPUs
+
+
+def test_lpt_single_class_matches_oracle_and_graham():
+    g = np.random.default_rng(3)
+    for G in (2, 3, 4, 8):
+        for _ in range(10):
+            costs = list(map(float, g.integers(1, 100, int(g.integers(1, 9)))))
+            got = svp.lpt_partition([7] * len(costs), costs, G)
+            assert got == sched.lpt_partition(costs, G)
+            if G <= 3:
+                opt = sched.best_partition_makespan(costs, G)
+                assert sched.partition_makespan(costs, got, G) <= sched.graham_bound(G) * opt + 1e-9
+
+
+def test_arena_ring_reuse_waits():
+    # host-resident jobs larger in total than the arena: slots must be reused, and the
+    # reusing H2D must start after the D2H that frees the slot
+    with svp.Context(dry_run=True, arena_bytes=64 << 20, max_chunks=4) as c:
+        for vp in range(16):
+            submit(c, vp, "vecadd", n=1 << 20, mem=svp.MEM_HOST_PINNED)  # 12 MiB staged per job
+        c.flush()
+        ops = c.plan()
+        assert c.flush_stats()["chunks"] >= 4
+        h2d = [op for op in ops if op["kind"] == svp.OP_H2D]
+        d2h = [op for op in ops if op["kind"] == svp.OP_D2H]
+        assert sum(op["bytes"] for op in h2d) == 16 * 8 * (1 << 20)
+        assert sum(op["bytes"] for op in d2h) == 16 * 4 * (1 << 20)
+
+
+def test_job_larger_than_arena_is_nomem():
+    with svp.Context(dry_run=True, arena_bytes=1 << 20) as c:
+        submit(c, 0, "vecadd", n=1 << 20, mem=svp.MEM_HOST_PINNED)
+        with pytest.raises(svp.SvpError) as e:
+            c.flush()
+        assert e.value.status == svp.SVP_E_NOMEM

@@ -155,16 +155,27 @@ def make_inputs(spec: JobSpec, seed: int = BASE_SEED) -> Dict[str, np.ndarray]:
         if spec.int_inputs:
             A = int_f32(rng(seed, vp, _S_A), M * K).reshape(M, K)
             B = int_f32(rng(seed, vp, _S_B), K * N).reshape(K, N)
-            C = int_f32(rng(seed, vp, _S_C), M * N).reshape(M, N)
         else:
             A = uniform_f32(rng(seed, vp, _S_A), M * K, -1, 1).reshape(M, K)
             B = uniform_f32(rng(seed, vp, _S_B), K * N, -1, 1).reshape(K, N)
-            C = uniform_f32(rng(seed, vp, _S_C), M * N, -1, 1).reshape(M, N)
-        return {"A": A, "B": B, "C": C}
+        out = {"A": A, "B": B}
+        if spec.beta != 0:  # C is an input only when beta != 0
+            gen = int_f32 if spec.int_inputs else (lambda g, n: uniform_f32(g, n, -1, 1))
+            out["C"] = gen(rng(seed, vp, _S_C), M * N).reshape(M, N)
+        return out
     raise ValueError(k)
 
 
 # --------------------------------------------------------------------------- configs
+def make_inputs_many(specs, seed: int = BASE_SEED, threads: int = 0) -> List[Dict[str, np.ndarray]]:
+    """make_inputs for many jobs on a thread pool (each job's streams are independent)."""
+    from concurrent.futures import ThreadPoolExecutor
+    import os
+    threads = threads or min(32, len(os.sched_getaffinity(0)))
+    with ThreadPoolExecutor(threads) as ex:
+        return list(ex.map(lambda s: make_inputs(s, seed), specs))
+
+
 def config_specs(cfg: int, seed: int = BASE_SEED, nvps: Optional[int] = None,
                  sgemm_int: bool = False, scale: int = 1) -> List[JobSpec]:
     """Job specs for BASELINE.json configs 1..5 (1-based, as listed there).
