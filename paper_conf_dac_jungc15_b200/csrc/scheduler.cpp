@@ -103,7 +103,10 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
         }
     }
     if (j->n >= (1ull << 40)) return fail(SVP_E_INVAL, "svp_submit: n too large");
-    bool empty = (j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32) ? ((int64_t)j->M * j->N == 0) : (j->n == 0);
+    // hist256 always writes its 256 counters (an empty input still overwrites them)
+    bool empty = (j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32) ? ((int64_t)j->M * j->N == 0)
+                 : j->kernel == K_HIST256                             ? false
+                                                                      : (j->n == 0);
     j->in_bytes = j->out_bytes = j->host_in_bytes = j->host_out_bytes = 0;
     for (int b = 0; b < j->nbufs; ++b) {
         const svp_buf& bf = j->bufs[b];
@@ -155,6 +158,7 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
     j->device = dispatch_vp(c, j->vp, cost);
     if (c->exec && c->cfg.validate_ptrs && !empty) {
         for (int b = 0; b < j->nbufs; ++b) {
+            if (touched_bytes(*j, b) == 0) continue;  // nothing is read or written there
             std::string why;
             if (executor_check_ptr(c->exec, j->bufs[b].ptr, j->bufs[b].mem, j->device, &why) != SVP_OK)
                 return fail(SVP_E_INVAL, "svp_submit: buffer " + std::to_string(b) + ": " + why);

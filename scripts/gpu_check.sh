@@ -1,0 +1,8 @@
+set -x
+nvidia-smi -L
+python -c "import torch;print(torch.cuda.get_device_name(0))"
+timeout 1200 python -m pytest tests -m gpu -q --timeout 300 --maxfail=30 -p no:cacheprovider > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"
+tail -5 gpurun_out/pytest_gpu.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"
+timeout 900 python bench.py --steps 10 --warmup 3 > gpurun_out/bench.log 2>&1; echo "bench rc=$?"
+tail -3 gpurun_out/bench.log
