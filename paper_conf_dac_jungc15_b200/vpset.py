@@ -109,6 +109,8 @@ class VPSet:
         for i, s in enumerate(self.specs):
             inp = self.inputs[i]
             for name, dt, d in BUFS[s.kernel]:
+                if s.kernel in ("sgemm", "sgemm_tf32") and name == "C" and s.beta != 0:
+                    d = svp.DIR_INOUT  # C is read when beta != 0
                 if d & svp.DIR_IN and name in inp:
                     src = torch.from_numpy(np.ascontiguousarray(inp[name]).reshape(-1).view(_NP[dt]))
                     if dt == "u32":
