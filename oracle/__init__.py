@@ -150,7 +150,7 @@ def run_job(spec, inputs: Dict[str, np.ndarray]) -> Dict[str, np.ndarray]:
     if k == "blackscholes":
         c, p = blackscholes(inputs["S"], inputs["X"], inputs["T"], spec.R, spec.V)
         return {"call": c, "put": p}
-    if k == "sgemm":
+    if k in ("sgemm", "sgemm_tf32"):  # same definition; the TF32 kernel has its own tolerance
         return {"C": sgemm(inputs["A"], inputs["B"], inputs.get("C") if spec.beta != 0 else None,
                            spec.alpha, spec.beta)}
     raise ValueError(k)

@@ -16,7 +16,7 @@
 
 namespace svp {
 
-static const bool kTf32Available = false;
+static const bool kTf32Available = true;
 static thread_local std::string g_last_error;
 void set_error(const std::string& msg) { g_last_error = msg; }
 
@@ -101,7 +101,7 @@ svp_status svp_init(const svp_config* cfg, svp_ctx** out) {
     *out = nullptr;
     if (cfg->num_gpus < 0 || cfg->num_gpus > 64 || cfg->streams_per_gpu < 1 || cfg->streams_per_gpu > 32 ||
         cfg->max_chunks < 1 || cfg->max_chunks > 64 || cfg->profile_level < 0 || cfg->profile_level > 2 ||
-        cfg->flush_timeout_ms < 0) {
+        cfg->flush_timeout_ms < 0 || cfg->sgemm_impl < 0 || cfg->sgemm_impl > 1) {
         set_error("svp_init: config value out of range");
         return SVP_E_INVAL;
     }
@@ -114,6 +114,7 @@ svp_status svp_init(const svp_config* cfg, svp_ctx** out) {
     if (cfg->ffma_tflops > 0) c->cost.ffma_flops = cfg->ffma_tflops * 1e12;
     if (cfg->launch_us > 0) c->cost.launch_ns = cfg->launch_us * 1e3;
     if (cfg->arena_bytes == 0) c->cfg.arena_bytes = 2ull << 30;
+    c->cost.sgemm_3xtf32 = cfg->sgemm_impl == SVP_SGEMM_3XTF32;
 
     if (cfg->dry_run) {
         c->ngpu = cfg->num_gpus > 0 ? cfg->num_gpus : 1;

@@ -264,7 +264,8 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             ch.total_tiles = tiles;
             ch.nsegs = (int32_t)ch.jobs.size();
         } else {
-            const int variant = ch.kernel == K_SGEMM_TF32 ? 1 : 0;
+            // tcgen05 tiles for sgemm_tf32 and for sgemm with the 3xTF32 implementation
+            const int variant = (ch.kernel == K_SGEMM_TF32 || e->c->cfg.sgemm_impl == SVP_SGEMM_3XTF32) ? 1 : 0;
             const int BM = variant ? kTf32BM : kGemmBM, BN = variant ? kTf32BN : kGemmBN;
             ch.maps_off = align_up(tbl.size(), 128);
             size_t nj = ch.jobs.size();
@@ -312,7 +313,6 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             ch.nsegs = (int32_t)nj;
         }
     }
-    (void)e;
     return SVP_OK;
 }
 
@@ -327,7 +327,7 @@ static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bo
     return pool[i];
 }
 
-static cudaError_t launch_chunk(Dev& d, const Chunk& ch, cudaStream_t s) {
+static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStream_t s) {
     if (ch.total_tiles == 0) return cudaSuccess;
     const uint8_t* base = d.tbl_dev;
     auto grid_of = [&](int per_sm) { return (int)std::min<uint64_t>(ch.total_tiles, (uint64_t)d.lim.num_sms * per_sm); };
@@ -345,6 +345,9 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, cudaStream_t s) {
             return launch_hist256((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
                                   grid_of(d.lim.hist_blocks_per_sm), s);
         case K_SGEMM:
+            if (sgemm_impl == SVP_SGEMM_3XTF32)
+                return launch_sgemm_3xtf32((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
+                                           ch.total_tiles, grid_of(1), s);
             return launch_sgemm_ffma((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
                                      ch.total_tiles, grid_of(d.lim.gemm_blocks_per_sm), s);
         case K_SGEMM_TF32:
@@ -458,7 +461,7 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
                 }
             }
         } else if (chunk_needs_launch(f, ch)) {
-            CK(launch_chunk(d, ch, s));
+            CK(launch_chunk(d, ch, c->cfg.sgemm_impl, s));
         }
         if (prof) {
             CK(cudaEventRecord(d.t_ev[2 * nt + 1], s));

@@ -138,6 +138,7 @@ struct CostModel {
     double ffma_flops = 60e12;
     double tf32_flops = 500e12;
     double launch_ns = 4000;
+    bool sgemm_3xtf32 = false;
     double copy_ns = 2000;           // per-copy fixed overhead
     // EMA of measured/predicted ratio per kernel (learned from the profiler)
     double kscale[K_COUNT] = {1, 1, 1, 1, 1, 1, 1};

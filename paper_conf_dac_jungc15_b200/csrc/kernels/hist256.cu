@@ -1,17 +1,18 @@
 // hist256.cu -- coalesced 256-bin byte histogram for sm_100a.
 //
 // counts_v[b] = #{i : d_v[i] == b} for every VP v of the group, in one launch.
-// Each tile lies in one VP; a CTA accumulates the bytes of its tiles into per-warp
-// shared-memory sub-histograms (one smem atomic per byte), and flushes them to the VP's
-// global counts with one atomicAdd per non-zero bin whenever it moves on to another VP.
-// A preceding tiny kernel zeroes every segment's counts, so the result overwrites the
-// output (the oracle's definition) and is bit-exact: integer adds commute.
+// Each tile lies in one VP.  A CTA keeps ONE shared histogram replicated per lane:
+// h[bin][lane] (256 x 32 u32 = 32 KiB), and lane l of every warp increments column l.
+// Within a warp instruction the 32 addresses therefore sit in 32 distinct banks
+// whatever the data (uniform or 90 % one value): one smem wavefront per ATOMS, no
+// same-address serialisation inside an instruction.  The CTA flushes the replicas to
+// the VP's global counts (one atomicAdd per non-zero bin) whenever it moves to another
+// VP; a preceding tiny kernel zeroes every segment's counts, so the result overwrites
+// the output and is bit-exact (integer adds commute).
 #include "../launch.h"
 #include "common.cuh"
 
 namespace svp {
-
-constexpr int kHistWarps = kHistThreads / 32;
 
 __global__ void __launch_bounds__(256) k_hist_zero(const SegDesc* __restrict__ segs, int nsegs) {
     for (int s = blockIdx.x; s < nsegs; s += gridDim.x) {
@@ -20,32 +21,36 @@ __global__ void __launch_bounds__(256) k_hist_zero(const SegDesc* __restrict__ s
     }
 }
 
+// h points at column `lane` of bin 0: h[b * 32] is this lane's counter for bin b.
 __device__ __forceinline__ void hist_add_word(uint32_t* h, uint32_t w) {
-    atomicAdd(&h[w & 0xFF], 1u);
-    atomicAdd(&h[(w >> 8) & 0xFF], 1u);
-    atomicAdd(&h[(w >> 16) & 0xFF], 1u);
-    atomicAdd(&h[w >> 24], 1u);
+    atomicAdd(h + ((w & 0xFFu) << 5), 1u);
+    atomicAdd(h + (((w >> 8) & 0xFFu) << 5), 1u);
+    atomicAdd(h + (((w >> 16) & 0xFFu) << 5), 1u);
+    atomicAdd(h + ((w >> 24) << 5), 1u);
 }
 
-__device__ __forceinline__ void hist_flush(uint32_t (*h)[256], uint32_t* counts) {
+// Sum the 32 replicas of each bin (thread t owns bin t; the column walk is rotated by
+// t so a warp's 32 reads hit 32 banks), zero them, and add to the VP's counts.
+__device__ __forceinline__ void hist_flush(uint32_t* h, uint32_t* counts) {
     __syncthreads();
-    for (int b = threadIdx.x; b < 256; b += kHistThreads) {
-        uint32_t s = 0;
-#pragma unroll
-        for (int w = 0; w < kHistWarps; ++w) {
-            s += h[w][b];
-            h[w][b] = 0;
-        }
-        if (s) atomicAdd(&counts[b], s);
+    const int b = threadIdx.x;  // kHistThreads == 256 == #bins
+    uint32_t s = 0;
+#pragma unroll 8
+    for (int j = 0; j < 32; ++j) {
+        const int c = (j + b) & 31;
+        s += h[b * 32 + c];
+        h[b * 32 + c] = 0;
     }
+    if (s) atomicAdd(&counts[b], s);
     __syncthreads();
 }
 
 __global__ void __launch_bounds__(kHistThreads) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
-    __shared__ uint32_t h[kHistWarps][256];
-    for (int i = threadIdx.x; i < kHistWarps * 256; i += kHistThreads) (&h[0][0])[i] = 0;
+    static_assert(kHistThreads == 256, "one flush thread per bin");
+    extern __shared__ uint32_t h[];  // [256][32]
+    for (int i = threadIdx.x; i < 256 * 32; i += kHistThreads) h[i] = 0;
     __syncthreads();
-    uint32_t* hw = h[threadIdx.x >> 5];
+    uint32_t* hl = h + (threadIdx.x & 31);
     int cur = -1;
     uint32_t* cur_counts = nullptr;
     for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
@@ -67,29 +72,31 @@ __global__ void __launch_bounds__(kHistThreads) k_hist256(const SegDesc* __restr
             for (int i = 0; i < kHistVec; ++i) r[i] = __ldcs(d4 + i * kHistThreads);
 #pragma unroll
             for (int i = 0; i < kHistVec; ++i) {
-                hist_add_word(hw, r[i].x);
-                hist_add_word(hw, r[i].y);
-                hist_add_word(hw, r[i].z);
-                hist_add_word(hw, r[i].w);
+                hist_add_word(hl, r[i].x);
+                hist_add_word(hl, r[i].y);
+                hist_add_word(hl, r[i].z);
+                hist_add_word(hl, r[i].w);
             }
         } else {
-            for (int64_t e = e0 + threadIdx.x; e < e1; e += kHistThreads) atomicAdd(&hw[d[e]], 1u);
+            for (int64_t e = e0 + threadIdx.x; e < e1; e += kHistThreads) atomicAdd(hl + ((uint32_t)d[e] << 5), 1u);
         }
     }
     if (cur >= 0) hist_flush(h, cur_counts);
 }
+
+constexpr int kHistSmem = 256 * 32 * 4;
 
 cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
     if (nsegs <= 0) return cudaSuccess;
     k_hist_zero<<<nsegs < 1024 ? nsegs : 1024, 256, 0, s>>>(segs, nsegs);
     cudaError_t e = cudaGetLastError();
     if (e || total == 0) return e;
-    k_hist256<<<grid, kHistThreads, 0, s>>>(segs, nsegs, total);
+    k_hist256<<<grid, kHistThreads, kHistSmem, s>>>(segs, nsegs, total);
     return cudaGetLastError();
 }
 
 cudaError_t query_limits_hist(int* per_sm) {
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k_hist256, kHistThreads, 0);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k_hist256, kHistThreads, kHistSmem);
 }
 
 }  // namespace svp

@@ -35,6 +35,10 @@ cudaError_t launch_sgemm_ffma(const GemmDesc* descs, int n, const void* maps, ui
 cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
                               int grid, cudaStream_t s);
 
+// fp32-accurate grouped SGEMM on tcgen05: 3xTF32 (hi/lo operand split, 3 MMAs per k-step).
+cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
+                                int grid, cudaStream_t s);
+
 // Host: encode the TMA descriptors an SGEMM entry needs (driver entry point fetched at
 // runtime, so libsvp does not link libcuda).  variant 0 = FFMA tiles, 1 = TF32 tiles.
 // Returns 0 on success.

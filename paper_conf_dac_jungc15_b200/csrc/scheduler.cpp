@@ -33,7 +33,7 @@ namespace svp {
 // ------------------------------------------------------------------ cost model
 double CostModel::kernel_ns(int32_t kernel, double alg_bytes, double flops) const {
     double body;
-    if (kernel == K_SGEMM) body = flops / ffma_flops * 1e9;
+    if (kernel == K_SGEMM) body = flops / (sgemm_3xtf32 ? tf32_flops / 3.0 : ffma_flops) * 1e9;
     else if (kernel == K_SGEMM_TF32) body = flops / tf32_flops * 1e9;
     else body = alg_bytes / hbm_Bps * 1e9;
     return launch_ns + body * kscale[kernel];

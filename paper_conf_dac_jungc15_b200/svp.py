@@ -23,6 +23,7 @@ STATUS_NAMES = {0: "SVP_OK", -1: "SVP_E_INVAL", -2: "SVP_E_NOMEM", -3: "SVP_E_CU
 DIR_IN, DIR_OUT, DIR_INOUT = 1, 2, 3
 MEM_DEVICE, MEM_HOST_PINNED = 0, 1
 OP_H2D, OP_KERNEL, OP_D2H = 0, 1, 2
+SGEMM_FFMA, SGEMM_3XTF32 = 0, 1
 MAX_BUFS, MAX_ARGS = 5, 64
 
 # ABI symbols declared in include/svp.h (tests check every one is exported)
@@ -37,6 +38,7 @@ class svp_config(C.Structure):
                 ("coalesce", C.c_int32), ("interleave", C.c_int32), ("max_chunks", C.c_int32),
                 ("arena_bytes", C.c_uint64), ("profile_level", C.c_int32), ("sync_each_job", C.c_int32),
                 ("dry_run", C.c_int32), ("flush_timeout_ms", C.c_int32), ("validate_ptrs", C.c_int32),
+                ("sgemm_impl", C.c_int32),
                 ("external_streams", C.POINTER(C.c_void_p)), ("hbm_gbps", C.c_double), ("pcie_gbps", C.c_double),
                 ("ffma_tflops", C.c_double), ("launch_us", C.c_double)]
 
@@ -180,7 +182,7 @@ class Context:
     def __init__(self, num_gpus: int = 0, device_ids: Optional[Sequence[int]] = None, streams_per_gpu: int = 4,
                  coalesce: bool = True, interleave: bool = True, max_chunks: int = 8, arena_bytes: int = 0,
                  profile_level: int = 0, sync_each_job: bool = False, dry_run: bool = False,
-                 flush_timeout_ms: int = 0, validate_ptrs: bool = True,
+                 flush_timeout_ms: int = 0, validate_ptrs: bool = True, sgemm_impl: int = SGEMM_FFMA,
                  external_streams: Optional[Sequence[int]] = None, hbm_gbps: float = 0.0, pcie_gbps: float = 0.0,
                  ffma_tflops: float = 0.0, launch_us: float = 0.0):
         L = load()
@@ -202,6 +204,7 @@ class Context:
         cfg.dry_run = int(dry_run)
         cfg.flush_timeout_ms = flush_timeout_ms
         cfg.validate_ptrs = int(validate_ptrs)
+        cfg.sgemm_impl = int(sgemm_impl)
         self._ext = None
         if external_streams is not None:
             self._ext = (C.c_void_p * len(external_streams))(*external_streams)

@@ -1,0 +1,63 @@
+"""tcgen05 SGEMM paths: "sgemm_tf32" (TF32 inputs, tolerance 2e-3) and "sgemm" with the
+3xTF32 implementation (fp32 contract, tolerance 1e-5), against the oracle."""
+import dataclasses
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+from gpu_common import check_job, inputs_for, run_svp
+from paper_conf_dac_jungc15_b200 import svp
+
+pytestmark = pytest.mark.gpu
+
+TF32_TOL = 2e-3
+
+
+def _as(kernel, specs):
+    return [dataclasses.replace(s, kernel=kernel) for s in specs]
+
+
+@pytest.mark.parametrize("int_inputs", [True, False])
+def test_tf32_config2(int_inputs):
+    specs = _as("sgemm_tf32", W.config_specs(2, sgemm_int=int_inputs))
+    inputs = inputs_for(specs)
+    outs, _, st = run_svp(specs, inputs, "device")
+    assert st["launches"] == 1
+    want = oracle.run_jobs(specs, inputs)
+    for s, inp, got, w in zip(specs, inputs, outs, want):
+        check_job(s, inp, got, w, sgemm_tol=TF32_TOL)
+
+
+@pytest.mark.parametrize("int_inputs", [True, False])
+def test_3xtf32_config2_fp32_tolerance(int_inputs):
+    specs = W.config_specs(2, sgemm_int=int_inputs)
+    inputs = inputs_for(specs)
+    outs, _, st = run_svp(specs, inputs, "device", sgemm_impl=svp.SGEMM_3XTF32)
+    want = oracle.run_jobs(specs, inputs)
+    for s, inp, got, w in zip(specs, inputs, outs, want):
+        check_job(s, inp, got, w)
+
+
+@pytest.mark.parametrize("kernel,impl,tol", [("sgemm_tf32", 0, TF32_TOL), ("sgemm", 1, 1e-5)])
+@pytest.mark.parametrize("residency", ["device", "host"])
+def test_tc_ragged_alpha_beta(kernel, impl, tol, residency):
+    dims = [(200, 136, 40), (200, 136, 40), (1, 4, 4), (129, 260, 0), (64, 68, 1000), (300, 516, 36)]
+    specs = [W.JobSpec(v, kernel, M=M, N=N, K=K, alpha=1.5, beta=-0.5) for v, (M, N, K) in enumerate(dims)]
+    inputs = inputs_for(specs)
+    outs, _, _ = run_svp(specs, inputs, residency, sgemm_impl=impl)
+    for s, inp, got in zip(specs, inputs, outs):
+        check_job(s, inp, got, sgemm_tol=tol)
+
+
+def test_3xtf32_2048_sampled():
+    """Full BASELINE cfg5 SGEMM shape (2048^3), 4 VPs coalesced, 64 sampled outputs each."""
+    specs = [W.JobSpec(v, "sgemm", M=2048, N=2048, K=2048) for v in range(4)]
+    inputs = inputs_for(specs)
+    outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=svp.SGEMM_3XTF32)
+    g = np.random.default_rng(1)
+    for s, inp, got in zip(specs, inputs, outs):
+        sample = [(int(g.integers(0, 2048)), int(g.integers(0, 2048))) for _ in range(64)]
+        sample += [(0, 0), (2047, 2047), (127, 255), (128, 256)]
+        check_job(s, inp, got, sample=sample)

@@ -97,7 +97,7 @@ class JobSpec:
             return self.n
         if self.kernel == "blackscholes":
             return 12 * self.n
-        if self.kernel == "sgemm":
+        if self.kernel in ("sgemm", "sgemm_tf32"):
             return 4 * (self.M * self.K + self.K * self.N + (self.M * self.N if self.beta != 0 else 0))
         raise ValueError(self.kernel)
 
@@ -108,7 +108,7 @@ class JobSpec:
             return 1024
         if self.kernel == "blackscholes":
             return 8 * self.n
-        if self.kernel == "sgemm":
+        if self.kernel in ("sgemm", "sgemm_tf32"):
             return 4 * self.M * self.N
         raise ValueError(self.kernel)
 
@@ -120,12 +120,12 @@ class JobSpec:
             return self.n + 1024
         if self.kernel == "blackscholes":
             return 20 * self.n
-        if self.kernel == "sgemm":
+        if self.kernel in ("sgemm", "sgemm_tf32"):
             return 4 * (self.M * self.K + self.K * self.N + self.M * self.N * (2 if self.beta != 0 else 1))
         raise ValueError(self.kernel)
 
     def flops(self) -> int:
-        return 2 * self.M * self.N * self.K if self.kernel == "sgemm" else 0
+        return 2 * self.M * self.N * self.K if self.kernel in ("sgemm", "sgemm_tf32") else 0
 
 
 def _scalar_for(seed: int, spec: JobSpec) -> None:
@@ -150,7 +150,7 @@ def make_inputs(spec: JobSpec, seed: int = BASE_SEED) -> Dict[str, np.ndarray]:
         return {"S": uniform_f32(rng(seed, vp, _S_A), n, 5.0, 30.0),
                 "X": uniform_f32(rng(seed, vp, _S_B), n, 1.0, 100.0),
                 "T": uniform_f32(rng(seed, vp, _S_C), n, 0.25, 10.0)}
-    if k == "sgemm":
+    if k in ("sgemm", "sgemm_tf32"):
         M, N, K = spec.M, spec.N, spec.K
         if spec.int_inputs:
             A = int_f32(rng(seed, vp, _S_A), M * K).reshape(M, K)
