@@ -3,27 +3,30 @@
 // C_v = alpha_v A_v B_v + beta_v C_v for every VP of a Kernel Match group, one persistent
 // launch (Kernel Coalescing; the paper's matmul guest, Table 1).
 //
-//  SPLIT = 1  "sgemm_tf32": one kind::tf32 MMA per k-step; the tensor core reads the fp32
+//  SPLIT = 1  "sgemm_tf32": one kind::tf32 MMA per k-step; the tensor core reads fp32
 //             operands as TF32 (low 13 mantissa bits ignored).  Own tolerance 2e-3.
-//  SPLIT = 3  "3xTF32": x = hi + lo with hi = x with the low 13 bits cleared (exactly what
-//             the tensor core sees when fed x) and lo = x - hi (exact in fp32); per k-step
-//             D += A_hi B_lo + A_lo B_hi + A_hi B_hi.  The dropped A_lo B_lo term and the
-//             truncation of lo are each < 2^-20 |a||b|, so the product error is
-//             < 3 * 2^-20 |a||b| ~ 2.9e-6 |a||b|: inside the fp32 SGEMM bound 1e-5 (|A||B|)_ij
-//             (R10) at tensor-core speed.
+//  SPLIT = 3  "3xTF32" (the fp32 "sgemm" on tensor cores): x = hi + lo, hi = x with the
+//             low 13 bits cleared (exactly what the tensor core reads from x) and
+//             lo = x - hi (exact in fp32); per k-step D += A_hi B_lo + A_lo B_hi + A_hi B_hi.
+//             The dropped A_lo B_lo and the truncation of lo are each < 2^-20 |a||b|, so
+//             the product error is < 3 * 2^-20 |a||b| ~ 2.9e-6 |a||b|, inside the fp32 bound
+//             1e-5 (|A||B|)_ij (R10).
 //
-// Structure (1 CTA per SM, persistent static tile walk, 256 threads):
-//   warp 0      TMA producer: A tile 128x32 (K-major, 128-B swizzle) + B tile 32x256 as 8
-//               boxes of 32x32 (MN-major, 128-B swizzle) per k-block into a smem ring.
-//   warp 1      TMEM allocator (512 columns = 2 fp32 accumulators of 128x256) and the MMA
-//               issuer: one elected lane issues tcgen05.mma.cta_group::1.kind::tf32
-//               (M=128, N=256, K=8) and tcgen05.commit's to the stage's empty barrier and,
-//               after the last k-block, to the accumulator's full barrier.
-//   warps 2-3   (SPLIT = 3) converters: lo = x - trunc_tf32(x) for the stage's A and B tiles
-//               (same swizzled layout), fence.proxy.async, arrive on the stage's conv barrier.
-//   warps 4-7   epilogue: tcgen05.ld 32x32b.x32 (warp w%4 owns TMEM lanes 32(w%4)..+31 =
-//               tile rows), alpha*acc (+ beta*C), 128-bit stores; double-buffered TMEM
-//               accumulators let tile i's epilogue overlap tile i+1's MMAs.
+// Both MMA operands are K-major with the 128-B swizzle (a kind::tf32 MMA with an MN-major
+// B operand returned zeros on B200 -- scripts/tc_probe.py, experiment E1 vs E2), so B
+// (row-major K x N, i.e. MN-major) is transposed in shared memory by converter warps.
+//
+// Roles (1 CTA per SM, persistent static tile walk, 320 threads):
+//   warp 0        TMA producer: A tile 128x32 (K-major, SW128) straight into the operand
+//                 stage; B tile 32x256 (row-major, no swizzle) into a raw staging ring.
+//   warp 1        TMEM allocator (512 cols = 2 accumulators of 128x256 fp32) + MMA issuer:
+//                 one lane issues tcgen05.mma.cta_group::1.kind::tf32 M128 N256 K8 and
+//                 tcgen05.commit's to the stage's empty barrier / the accumulator barrier.
+//   warps 2,3,8,9 converters: B^T (K-major SW128, hi = raw bits) [+ B_lo^T, A_lo for SPLIT 3]
+//                 from the staged tiles; fence.proxy.async; arrive on the stage's conv barrier.
+//   warps 4-7     epilogue: tcgen05.ld 32x32b.x32 (warp w%4 owns TMEM lanes = tile rows
+//                 32(w%4)..+31), alpha*acc (+ beta*C), 128-bit stores; the two TMEM
+//                 accumulators let tile i's epilogue overlap tile i+1's MMAs.
 #include <cuda.h>
 
 #include "../launch.h"
@@ -34,33 +37,34 @@ namespace svp {
 namespace tc {
 
 constexpr int BM = kTf32BM, BN = kTf32BN, BK = kTf32BK;  // 128 x 256 x 32
-constexpr int kThreads = 256;
-constexpr int kStageA = BM * BK * 4;  // 16 KiB
-constexpr int kStageB = BK * BN * 4;  // 32 KiB
+constexpr int kThreads = 320;
+constexpr int kConvThreads = 128;
+constexpr int kTileA = BM * BK * 4;   // 16 KiB
+constexpr int kTileB = BK * BN * 4;   // 32 KiB
 constexpr int kTmemCols = 512;
 
 template <int SPLIT>
 struct Cfg {
-    static constexpr int kStages = SPLIT == 1 ? 4 : 2;
-    static constexpr int kStageBytes = (kStageA + kStageB) * (SPLIT == 1 ? 1 : 2);
-    static constexpr size_t kSmem = 1024 + (size_t)kStages * kStageBytes + 256;
+    // operand stage: A_hi (TMA) | B_hi^T | [A_lo | B_lo^T]
+    static constexpr int kOpStageBytes = SPLIT == 1 ? kTileA + kTileB : 2 * (kTileA + kTileB);
+    static constexpr int kOpStages = SPLIT == 1 ? 3 : 2;
+    static constexpr int kRawStages = SPLIT == 1 ? 2 : 1;
+    static constexpr size_t kBarOff = (size_t)kOpStages * kOpStageBytes + (size_t)kRawStages * kTileB;
+    static constexpr size_t kSmem = 1024 + kBarOff + 256;
 };
 
-__device__ __forceinline__ uint64_t make_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
-    // SM100 shared-memory matrix descriptor: start>>4 [0,14), LBO>>4 [16,30), SBO>>4 [32,46),
-    // version 1 [46,48), base offset 0, layout SWIZZLE_128B (2) [61,64)
-    uint64_t d = 0;
-    d |= (uint64_t)((saddr >> 4) & 0x3FFF);
-    d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
-    d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;
-    d |= (uint64_t)1 << 46;
-    d |= (uint64_t)2 << 61;
-    return d;
+__device__ __forceinline__ uint64_t make_desc_kmajor_sw128(uint32_t saddr) {
+    // SM100 smem matrix descriptor: start>>4 [0,14), LBO>>4 [16,30) (=1, unused for
+    // swizzled K-major), SBO>>4 [32,46) (1024 B between 8-row groups), version 1 [46,48),
+    // layout SWIZZLE_128B (2) [61,64)
+    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
+           ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
 }
 
-// kind::tf32 instruction descriptor: D f32, A/B tf32, A K-major, B MN-major, N=256, M=128
-constexpr uint32_t kIdesc = (1u << 4) | (2u << 7) | (2u << 10) | (0u << 15) | (1u << 16) |
-                            ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+// kind::tf32 instruction descriptor: D f32 [4,6)=1, A tf32 [7,10)=2, B tf32 [10,13)=2,
+// A and B K-major (bits 15, 16 = 0), N>>3 at [17,23), M>>4 at [24,29)
+constexpr uint32_t kIdesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) |
+                            ((uint32_t)(BM >> 4) << 24);
 
 __device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accum) {
     asm volatile(
@@ -82,13 +86,14 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
     asm volatile(
         "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
         "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];\n\t"
+        "tcgen05.wait::ld.sync.aligned;"
         : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
           "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
           "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
           "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
-        : "r"(taddr));
-    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+        : "r"(taddr)
+        : "memory");
 }
 
 __device__ __forceinline__ int find_tile_owner(const GemmDesc* __restrict__ d, int n, uint32_t t) {
@@ -101,15 +106,7 @@ __device__ __forceinline__ int find_tile_owner(const GemmDesc* __restrict__ d, i
     return lo - 1;
 }
 
-// lo = x - (x with the low 13 mantissa bits cleared); exact in fp32
-__device__ __forceinline__ float4 split_lo(float4 x) {
-    float4 r;
-    r.x = x.x - __uint_as_float(__float_as_uint(x.x) & 0xFFFFE000u);
-    r.y = x.y - __uint_as_float(__float_as_uint(x.y) & 0xFFFFE000u);
-    r.z = x.z - __uint_as_float(__float_as_uint(x.z) & 0xFFFFE000u);
-    r.w = x.w - __uint_as_float(__float_as_uint(x.w) & 0xFFFFE000u);
-    return r;
-}
+__device__ __forceinline__ float lo_part(float x) { return x - __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
 
 }  // namespace tc
 
@@ -117,24 +114,31 @@ template <int SPLIT>
 __global__ void __launch_bounds__(tc::kThreads, 1)
     k_sgemm_tc(const GemmDesc* __restrict__ descs, int n, const uint8_t* __restrict__ maps, uint32_t total) {
     using namespace tc;
-    constexpr int ST = Cfg<SPLIT>::kStages;
-    constexpr int SB = Cfg<SPLIT>::kStageBytes;
+    using C = Cfg<SPLIT>;
+    constexpr int OS = C::kOpStages, RS = C::kRawStages, OB = C::kOpStageBytes;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + ST * SB);
-    uint64_t* full = bars;            // [ST]  TMA landed
-    uint64_t* empty = bars + ST;      // [ST]  MMAs done reading the stage
-    uint64_t* conv = bars + 2 * ST;   // [ST]  lo tiles written (SPLIT = 3)
-    uint64_t* acc_full = bars + 3 * ST;   // [2]
-    uint64_t* acc_empty = bars + 3 * ST + 2;  // [2]
-    uint32_t* tmem_base_slot = reinterpret_cast<uint32_t*>(bars + 3 * ST + 4);
+    uint8_t* raw_base = smem + (size_t)OS * OB;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::kBarOff);
+    uint64_t* a_full = bars;                 // [OS] TMA A landed
+    uint64_t* op_empty = bars + OS;          // [OS] MMAs done with the operand stage
+    uint64_t* conv_done = bars + 2 * OS;     // [OS] converters wrote the stage
+    uint64_t* raw_full = bars + 3 * OS;      // [RS] TMA B landed in the staging ring
+    uint64_t* raw_empty = raw_full + RS;     // [RS] converters done reading raw B
+    uint64_t* acc_full = raw_empty + RS;     // [2]
+    uint64_t* acc_empty = acc_full + 2;      // [2]
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_empty + 2);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
-        for (int s = 0; s < ST; ++s) {
-            mbar_init(&full[s], 1);
-            mbar_init(&empty[s], 1);
-            mbar_init(&conv[s], 2);
+        for (int s = 0; s < OS; ++s) {
+            mbar_init(&a_full[s], 1);
+            mbar_init(&op_empty[s], 1);
+            mbar_init(&conv_done[s], kConvThreads / 32);
+        }
+        for (int r = 0; r < RS; ++r) {
+            mbar_init(&raw_full[r], 1);
+            mbar_init(&raw_empty[r], kConvThreads / 32);
         }
         for (int a = 0; a < 2; ++a) {
             mbar_init(&acc_full[a], 1);
@@ -143,7 +147,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
         mbar_fence_init();
     }
     if (warp == 1) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_base_slot)),
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                      "n"(kTmemCols)
                      : "memory");
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
@@ -151,9 +155,10 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
-    const uint32_t tmem_base = *tmem_base_slot;
+    const uint32_t tmem_base = *tmem_slot;
 
-    auto stage_ptr = [&](int s) { return smem + (size_t)s * SB; };
+    auto op_stage = [&](int s) { return smem + (size_t)s * OB; };
+    auto raw_stage = [&](int r) { return raw_base + (size_t)r * kTileB; };
 
     if (warp == 0) {
         // ------------------------------------------------------------ TMA producer
@@ -174,15 +179,14 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                 const int tm = lt / g.tiles_n, tn = lt % g.tiles_n;
                 const int KB = (g.K + BK - 1) / BK;
                 for (int kb = 0; kb < KB; ++kb, ++it) {
-                    const int s = it % ST;
-                    const uint32_t ph = (it / ST) & 1;
-                    mbar_wait(&empty[s], ph ^ 1);
-                    uint8_t* sp = stage_ptr(s);
-                    mbar_expect_tx(&full[s], kStageA + kStageB);
-                    tma_load_2d(sp, mA, kb * BK, tm * BM, &full[s]);
-#pragma unroll
-                    for (int j = 0; j < BN / 32; ++j)
-                        tma_load_2d(sp + kStageA + j * (BK * 32 * 4), mB, tn * BN + j * 32, kb * BK, &full[s]);
+                    const int s = it % OS, r = it % RS;
+                    const uint32_t ph = (it / OS) & 1, rph = (it / RS) & 1;
+                    mbar_wait(&raw_empty[r], rph ^ 1);
+                    mbar_expect_tx(&raw_full[r], kTileB);
+                    tma_load_2d(raw_stage(r), mB, tn * BN, kb * BK, &raw_full[r]);
+                    mbar_wait(&op_empty[s], ph ^ 1);
+                    mbar_expect_tx(&a_full[s], kTileA);
+                    tma_load_2d(op_stage(s), mA, kb * BK, tm * BM, &a_full[s]);
                 }
             }
         }
@@ -198,26 +202,24 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
             tc_fence_after();
             const uint32_t tmem_d = tmem_base + (uint32_t)(a * BN);
             for (int kb = 0; kb < KB; ++kb, ++it) {
-                const int s = it % ST;
-                const uint32_t ph = (it / ST) & 1;
-                if (SPLIT == 1) mbar_wait(&full[s], ph);
-                else mbar_wait(&conv[s], ph);
+                const int s = it % OS;
+                const uint32_t ph = (it / OS) & 1;
+                mbar_wait(&a_full[s], ph);
+                mbar_wait(&conv_done[s], ph);
                 tc_fence_after();
                 if (lane == 0) {
-                    const uint32_t sa = smem_u32(stage_ptr(s));
-                    const uint32_t sbh = sa + kStageA;
+                    const uint32_t s_ah = smem_u32(op_stage(s));
+                    const uint32_t s_bh = s_ah + kTileA;
+                    const uint32_t s_al = s_bh + kTileB;
+                    const uint32_t s_bl = s_al + kTileA;
 #pragma unroll
                     for (int kk = 0; kk < BK / 8; ++kk) {
-                        // A: K-major SW128 rows of 128 B, 8-row groups 1024 B apart; K advance = 32 B
-                        const uint64_t ah = make_desc(sa + kk * 32, 16, 1024);
-                        // B: MN-major SW128, 32-col blocks of 32 k-rows (4 KiB); K advance = 8 rows
-                        const uint64_t bh = make_desc(sbh + kk * 1024, BK * 32 * 4, 1024);
+                        const uint64_t ah = make_desc_kmajor_sw128(s_ah + kk * 32);
+                        const uint64_t bh = make_desc_kmajor_sw128(s_bh + kk * 32);
                         const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
                         if (SPLIT == 3) {
-                            const uint32_t sal = sa + kStageA + kStageB;
-                            const uint32_t sbl = sal + kStageA;
-                            const uint64_t al = make_desc(sal + kk * 32, 16, 1024);
-                            const uint64_t bl = make_desc(sbl + kk * 1024, BK * 32 * 4, 1024);
+                            const uint64_t al = make_desc_kmajor_sw128(s_al + kk * 32);
+                            const uint64_t bl = make_desc_kmajor_sw128(s_bl + kk * 32);
                             mma_tf32(tmem_d, ah, bl, acc0);
                             mma_tf32(tmem_d, al, bh, 1u);
                             mma_tf32(tmem_d, ah, bh, 1u);
@@ -225,35 +227,69 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                             mma_tf32(tmem_d, ah, bh, acc0);
                         }
                     }
-                    mma_commit(&empty[s]);
+                    mma_commit(&op_empty[s]);
                     if (kb == KB - 1) mma_commit(&acc_full[a]);
                 }
                 __syncwarp();
             }
-            if (KB == 0 && lane == 0) mbar_arrive(&acc_full[a]);  // K == 0: nothing to wait for
+            if (KB == 0 && lane == 0) mbar_arrive(&acc_full[a]);  // K == 0: nothing accumulated
             __syncwarp();
         }
-    } else if (warp < 4) {
-        // ------------------------------------------------------------ lo converters (SPLIT 3)
-        if (SPLIT == 3) {
-            const int ct = threadIdx.x - 64;  // 0..63
-            uint32_t it = 0;
-            for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
-                const int v = find_tile_owner(descs, n, t);
-                const int KB = (descs[v].K + BK - 1) / BK;
-                for (int kb = 0; kb < KB; ++kb, ++it) {
-                    const int s = it % ST;
-                    const uint32_t ph = (it / ST) & 1;
-                    mbar_wait(&full[s], ph);
-                    const float4* src = reinterpret_cast<const float4*>(stage_ptr(s));
-                    float4* dst = reinterpret_cast<float4*>(stage_ptr(s) + kStageA + kStageB);
-                    constexpr int NV = (kStageA + kStageB) / 16;  // 3072 float4
+    } else if (warp < 4 || warp >= 8) {
+        // ------------------------------------------------------------ converters
+        const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;  // 0..127
+        uint32_t it = 0;
+        for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+            const int v = find_tile_owner(descs, n, t);
+            const int KB = (descs[v].K + BK - 1) / BK;
+            for (int kb = 0; kb < KB; ++kb, ++it) {
+                const int s = it % OS, r = it % RS;
+                const uint32_t ph = (it / OS) & 1, rph = (it / RS) & 1;
+                mbar_wait(&op_empty[s], ph ^ 1);  // previous MMAs on this stage are done
+                mbar_wait(&raw_full[r], rph);
+                const float* rawB = reinterpret_cast<const float*>(raw_stage(r));  // [k][n], row 1 KiB
+                uint8_t* bh = op_stage(s) + kTileA;
+                uint8_t* bl = bh + kTileB + kTileA;
+                // (n, 4-k chunk) pairs: a warp covers 32 consecutive n of one chunk ->
+                // conflict-free reads (one 128-B row segment per k) and swizzled 16-B writes
 #pragma unroll 4
-                    for (int i = ct; i < NV; i += 64) dst[i] = split_lo(src[i]);
-                    fence_proxy_async();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&conv[s]);
+                for (int p = ct; p < BN * (BK / 4); p += kConvThreads) {
+                    const int nn = p & (BN - 1), c = p / BN;
+                    float4 x;
+                    x.x = rawB[(4 * c + 0) * BN + nn];
+                    x.y = rawB[(4 * c + 1) * BN + nn];
+                    x.z = rawB[(4 * c + 2) * BN + nn];
+                    x.w = rawB[(4 * c + 3) * BN + nn];
+                    const int off = nn * 128 + ((c ^ (nn & 7)) << 4);
+                    *reinterpret_cast<float4*>(bh + off) = x;
+                    if (SPLIT == 3) {
+                        float4 y;
+                        y.x = lo_part(x.x);
+                        y.y = lo_part(x.y);
+                        y.z = lo_part(x.z);
+                        y.w = lo_part(x.w);
+                        *reinterpret_cast<float4*>(bl + off) = y;
+                    }
                 }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&raw_empty[r]);
+                if (SPLIT == 3) {
+                    mbar_wait(&a_full[s], ph);
+                    const float4* ah = reinterpret_cast<const float4*>(op_stage(s));
+                    float4* al = reinterpret_cast<float4*>(op_stage(s) + kTileA + kTileB);
+#pragma unroll 4
+                    for (int i = ct; i < kTileA / 16; i += kConvThreads) {
+                        float4 x = ah[i];
+                        x.x = lo_part(x.x);
+                        x.y = lo_part(x.y);
+                        x.z = lo_part(x.z);
+                        x.w = lo_part(x.w);
+                        al[i] = x;  // same swizzled position as the hi element
+                    }
+                }
+                fence_proxy_async();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&conv_done[s]);
             }
         }
     } else {
