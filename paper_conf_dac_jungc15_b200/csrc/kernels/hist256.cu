@@ -53,7 +53,11 @@ __global__ void __launch_bounds__(kHistThreads) k_hist256(const SegDesc* __restr
     uint32_t* hl = h + (threadIdx.x & 31);
     int cur = -1;
     uint32_t* cur_counts = nullptr;
-    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+    // blocked tile ranges: a CTA walks contiguous tiles, so it stays inside one VP for
+    // many tiles and flushes its replicas only at VP boundaries
+    const uint32_t per = (total + gridDim.x - 1) / gridDim.x;
+    const uint32_t t0 = blockIdx.x * per, t1 = min(total, t0 + per);
+    for (uint32_t t = t0; t < t1; ++t) {
         const int si = find_seg(segs, nsegs, t);
         const SegDesc& sd = segs[si];
         if (si != cur) {

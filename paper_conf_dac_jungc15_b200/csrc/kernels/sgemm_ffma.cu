@@ -45,7 +45,7 @@ __device__ __forceinline__ int find_gemm(const GemmDesc* __restrict__ d, int n, 
 __global__ void __launch_bounds__(kGemmThreads, 1)
     k_sgemm_ffma(const GemmDesc* __restrict__ descs, int n, const uint8_t* __restrict__ maps, uint32_t total) {
     extern __shared__ uint8_t smem_raw[];
-    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);  // keeps LDS (shared space)
     float* sA = reinterpret_cast<float*>(smem);
     float* sB = reinterpret_cast<float*>(smem + kStages * kStageA);
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages * (kStageA + kStageB));
@@ -159,13 +159,13 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 o.z = alpha * acc[i][h * 4 + 2];
                 o.w = alpha * acc[i][h * 4 + 3];
                 if (beta != 0.f) {
-                    const float4 old = *dst;
+                    const float4 old = __ldcs(dst);
                     o.x = __fmaf_rn(beta, old.x, o.x);
                     o.y = __fmaf_rn(beta, old.y, o.y);
                     o.z = __fmaf_rn(beta, old.z, o.z);
                     o.w = __fmaf_rn(beta, old.w, o.w);
                 }
-                *dst = o;
+                __stcs(dst, o);  // st.global.cs: C is written once
             }
         }
     }

@@ -117,7 +117,9 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
     using C = Cfg<SPLIT>;
     constexpr int OS = C::kOpStages, RS = C::kRawStages, OB = C::kOpStageBytes;
     extern __shared__ uint8_t smem_raw[];
-    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    // align to 1024 B (SW128 atoms) by offsetting smem_raw itself, so the compiler keeps
+    // the shared address space and emits LDS/STS (not generic LD/ST) for the converters
+    uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     uint8_t* raw_base = smem + (size_t)OS * OB;
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::kBarOff);
     uint64_t* a_full = bars;                 // [OS] TMA A landed
@@ -327,13 +329,13 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                     o.w = kzero ? 0.f : alpha * __uint_as_float(r[j + 3]);
                     float4* dst = reinterpret_cast<float4*>(crow + c);
                     if (beta != 0.f) {
-                        const float4 old = *dst;
+                        const float4 old = __ldcs(dst);
                         o.x = __fmaf_rn(beta, old.x, o.x);
                         o.y = __fmaf_rn(beta, old.y, o.y);
                         o.z = __fmaf_rn(beta, old.z, o.z);
                         o.w = __fmaf_rn(beta, old.w, o.w);
                     }
-                    *dst = o;
+                    __stcs(dst, o);  // st.global.cs: C is written once
                 }
             }
             tc_fence_before();
