@@ -1,11 +1,12 @@
 // hist256.cu -- coalesced 256-bin byte histogram for sm_100a.
 //
 // counts_v[b] = #{i : d_v[i] == b} for every VP v of the group, in one launch.
-// Each tile lies in one VP.  A CTA keeps ONE shared histogram replicated per lane:
-// h[bin][lane] (256 x 32 u32 = 32 KiB), and lane l of every warp increments column l.
-// Within a warp instruction the 32 addresses therefore sit in 32 distinct banks
-// whatever the data (uniform or 90 % one value): one smem wavefront per ATOMS, no
-// same-address serialisation inside an instruction.  The CTA flushes the replicas to
+// Each tile lies in one VP.  A CTA keeps ONE shared histogram replicated per lane
+// (lane l of every warp increments column l, two 16-bit bins per 32-bit word), so the 32
+// addresses of a warp instruction sit in 32 distinct banks whatever the data (uniform
+// or 90 % one value): one smem wavefront per ATOMS, no same-address serialisation
+// inside an instruction.  One smem atomic per byte caps this kernel at the measured
+// shared-atomic rate (tools/ubench.py: ~3.7e12 lanes/s = 3.7 TB/s of input bytes).  The CTA flushes the replicas to
 // the VP's global counts (one atomicAdd per non-zero bin) whenever it moves to another
 // VP; a preceding tiny kernel zeroes every segment's counts, so the result overwrites
 // the output and is bit-exact (integer adds commute).
@@ -21,50 +22,68 @@ __global__ void __launch_bounds__(256) k_hist_zero(const SegDesc* __restrict__ s
     }
 }
 
-// h points at column `lane` of bin 0: h[b * 32] is this lane's counter for bin b.
-__device__ __forceinline__ void hist_add_word(uint32_t* h, uint32_t w) {
-    atomicAdd(h + ((w & 0xFFu) << 5), 1u);
-    atomicAdd(h + (((w >> 8) & 0xFFu) << 5), 1u);
-    atomicAdd(h + (((w >> 16) & 0xFFu) << 5), 1u);
-    atomicAdd(h + ((w >> 24) << 5), 1u);
+// Shared table h[word][lane], word = bin & 127, 16-bit half = bin >> 7: 128 x 32 u32 =
+// 16 KiB per CTA, so 8 CTAs (2048 threads) fit an SM and keep enough loads in flight.
+// hl points at column `lane` of word 0.  A half-counter gains at most 8 warps x
+// kHistVec x 16 increments per tile, so flushing every kHistFlushTiles tiles keeps it
+// below 2^16.
+constexpr int kHistWords = 128;
+constexpr int kHistFlushTiles = 32;
+static_assert(kHistFlushTiles * (kHistThreads / 32) * kHistVec * 16 < 65536, "16-bit half-counters overflow");
+
+__device__ __forceinline__ void hist_add_byte(uint32_t* hl, uint32_t b) {
+    atomicAdd(hl + ((b & 127u) << 5), 1u << ((b >> 7) << 4));
+}
+__device__ __forceinline__ void hist_add_word(uint32_t* hl, uint32_t w) {
+    hist_add_byte(hl, w & 0xFFu);
+    hist_add_byte(hl, (w >> 8) & 0xFFu);
+    hist_add_byte(hl, (w >> 16) & 0xFFu);
+    hist_add_byte(hl, w >> 24);
 }
 
-// Sum the 32 replicas of each bin (thread t owns bin t; the column walk is rotated by
-// t so a warp's 32 reads hit 32 banks), zero them, and add to the VP's counts.
+// Sum the 32 lane replicas of each word (thread t < 128 owns word t; the column walk is
+// rotated by t so a warp's 32 reads hit 32 banks), zero them, and add both halves to the
+// VP's counts (bins t and t + 128).
 __device__ __forceinline__ void hist_flush(uint32_t* h, uint32_t* counts) {
     __syncthreads();
-    const int b = threadIdx.x;  // kHistThreads == 256 == #bins
-    uint32_t s = 0;
+    const int w = threadIdx.x;
+    if (w < kHistWords) {
+        uint32_t lo = 0, hi = 0;
 #pragma unroll 8
-    for (int j = 0; j < 32; ++j) {
-        const int c = (j + b) & 31;
-        s += h[b * 32 + c];
-        h[b * 32 + c] = 0;
+        for (int j = 0; j < 32; ++j) {
+            const int c = (j + w) & 31;
+            const uint32_t v = h[w * 32 + c];
+            lo += v & 0xFFFFu;
+            hi += v >> 16;
+            h[w * 32 + c] = 0;
+        }
+        if (lo) atomicAdd(&counts[w], lo);
+        if (hi) atomicAdd(&counts[w + 128], hi);
     }
-    if (s) atomicAdd(&counts[b], s);
     __syncthreads();
 }
 
 __global__ void __launch_bounds__(kHistThreads) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
-    static_assert(kHistThreads == 256, "one flush thread per bin");
-    extern __shared__ uint32_t h[];  // [256][32]
-    for (int i = threadIdx.x; i < 256 * 32; i += kHistThreads) h[i] = 0;
+    __shared__ uint32_t h[kHistWords * 32];
+    for (int i = threadIdx.x; i < kHistWords * 32; i += kHistThreads) h[i] = 0;
     __syncthreads();
     uint32_t* hl = h + (threadIdx.x & 31);
-    int cur = -1;
+    int cur = -1, since_flush = 0;
     uint32_t* cur_counts = nullptr;
     // blocked tile ranges: a CTA walks contiguous tiles, so it stays inside one VP for
-    // many tiles and flushes its replicas only at VP boundaries
+    // many tiles and flushes only at VP boundaries (or every kHistFlushTiles tiles)
     const uint32_t per = (total + gridDim.x - 1) / gridDim.x;
     const uint32_t t0 = blockIdx.x * per, t1 = min(total, t0 + per);
     for (uint32_t t = t0; t < t1; ++t) {
         const int si = find_seg(segs, nsegs, t);
         const SegDesc& sd = segs[si];
-        if (si != cur) {
+        if (si != cur || since_flush == kHistFlushTiles) {
             if (cur >= 0) hist_flush(h, cur_counts);
             cur = si;
+            since_flush = 0;
             cur_counts = reinterpret_cast<uint32_t*>(sd.ptr[1]);
         }
+        ++since_flush;
         const uint8_t* __restrict__ d = reinterpret_cast<const uint8_t*>(sd.ptr[0]);
         int64_t e0, e1;
         bool vec;
@@ -82,13 +101,13 @@ __global__ void __launch_bounds__(kHistThreads) k_hist256(const SegDesc* __restr
                 hist_add_word(hl, r[i].w);
             }
         } else {
-            for (int64_t e = e0 + threadIdx.x; e < e1; e += kHistThreads) atomicAdd(hl + ((uint32_t)d[e] << 5), 1u);
+            for (int64_t e = e0 + threadIdx.x; e < e1; e += kHistThreads) hist_add_byte(hl, d[e]);
         }
     }
     if (cur >= 0) hist_flush(h, cur_counts);
 }
 
-constexpr int kHistSmem = 256 * 32 * 4;
+constexpr int kHistSmem = 0;  // static shared table
 
 cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
     if (nsegs <= 0) return cudaSuccess;

@@ -231,10 +231,10 @@ int encode_gemm_maps(void* mapA, void* mapB, const float* A, const float* B, int
         if (r) return r;
         return encode2d(mapB, B, (uint64_t)N, (uint64_t)K, GN, GK, CU_TENSOR_MAP_SWIZZLE_NONE);
     }
-    // tcgen05 tiles: A lands K-major (box 32 k x 128 m, SW128) directly in the MMA operand
-    // stage; B (row-major K x N) lands raw (box 256 n x 32 k, no swizzle) in a staging ring
-    // and is transposed to K-major SW128 by the kernel's converter warps.
-    int r = encode2d(mapA, A, (uint64_t)K, (uint64_t)M, kTf32BK, kTf32BM, CU_TENSOR_MAP_SWIZZLE_128B);
+    // tcgen05 tiles: A lands K-major (box 16 k x 128 m, SW64) directly in the MMA operand
+    // stage; B (row-major K x N) lands raw (box 256 n x 16 k, no swizzle) in a staging ring
+    // and is transposed to K-major SW64 by the kernel's converter warps.
+    int r = encode2d(mapA, A, (uint64_t)K, (uint64_t)M, kTf32BK, kTf32BM, CU_TENSOR_MAP_SWIZZLE_64B);
     if (r) return r;
     return encode2d(mapB, B, (uint64_t)N, (uint64_t)K, kTf32BN, kTf32BK, CU_TENSOR_MAP_SWIZZLE_NONE);
 }

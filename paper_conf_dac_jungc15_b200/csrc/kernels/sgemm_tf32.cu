@@ -12,17 +12,18 @@
 //             the product error is < 3 * 2^-20 |a||b| ~ 2.9e-6 |a||b|, inside the fp32 bound
 //             1e-5 (|A||B|)_ij (R10).
 //
-// Both MMA operands are K-major with the 128-B swizzle (a kind::tf32 MMA with an MN-major
+// Both MMA operands are K-major with the 64-B swizzle (a kind::tf32 MMA with an MN-major
 // B operand returned zeros on B200 -- scripts/tc_probe.py, experiment E1 vs E2), so B
 // (row-major K x N, i.e. MN-major) is transposed in shared memory by converter warps.
 //
 // Roles (1 CTA per SM, persistent static tile walk, 320 threads):
-//   warp 0        TMA producer: A tile 128x32 (K-major, SW128) straight into the operand
-//                 stage; B tile 32x256 (row-major, no swizzle) into a raw staging ring.
+//   warp 0        TMA producer: A tile 128x16 (K-major, 64-B swizzle) straight into the
+//                 operand stage; B tile 16x256 (row-major, no swizzle) into a raw staging
+//                 ring (4 deep, so B's L2 latency hides behind 3 stages of MMAs).
 //   warp 1        TMEM allocator (512 cols = 2 accumulators of 128x256 fp32) + MMA issuer:
 //                 one lane issues tcgen05.mma.cta_group::1.kind::tf32 M128 N256 K8 and
 //                 tcgen05.commit's to the stage's empty barrier / the accumulator barrier.
-//   warps 2,3,8,9 converters: B^T (K-major SW128, hi = raw bits) [+ B_lo^T, A_lo for SPLIT 3]
+//   warps 2,3,8,9 converters: B^T (K-major SW64, hi = raw bits) [+ B_lo^T, A_lo for SPLIT 3]
 //                 from the staged tiles; fence.proxy.async; arrive on the stage's conv barrier.
 //   warps 4-7     epilogue: tcgen05.ld 32x32b.x32 (warp w%4 owns TMEM lanes = tile rows
 //                 32(w%4)..+31), alpha*acc (+ beta*C), 128-bit stores; the two TMEM
@@ -36,29 +37,31 @@ namespace svp {
 
 namespace tc {
 
-constexpr int BM = kTf32BM, BN = kTf32BN, BK = kTf32BK;  // 128 x 256 x 32
+constexpr int BM = kTf32BM, BN = kTf32BN, BK = kTf32BK;  // 128 x 256 x 16
+constexpr int kRowBytes = BK * 4;                          // 64-B K-major rows -> SWIZZLE_64B
+constexpr int kAtomBytes = 8 * kRowBytes;                  // 8-row swizzle atom (SBO)
 constexpr int kThreads = 320;
 constexpr int kConvThreads = 128;
-constexpr int kTileA = BM * BK * 4;   // 16 KiB
-constexpr int kTileB = BK * BN * 4;   // 32 KiB
+constexpr int kTileA = BM * BK * 4;   // 8 KiB
+constexpr int kTileB = BK * BN * 4;   // 16 KiB
 constexpr int kTmemCols = 512;
 
 template <int SPLIT>
 struct Cfg {
     // operand stage: A_hi (TMA) | B_hi^T | [A_lo | B_lo^T]
     static constexpr int kOpStageBytes = SPLIT == 1 ? kTileA + kTileB : 2 * (kTileA + kTileB);
-    static constexpr int kOpStages = SPLIT == 1 ? 3 : 2;
-    static constexpr int kRawStages = SPLIT == 1 ? 2 : 1;
+    static constexpr int kOpStages = SPLIT == 1 ? 4 : 3;
+    static constexpr int kRawStages = 4;
     static constexpr size_t kBarOff = (size_t)kOpStages * kOpStageBytes + (size_t)kRawStages * kTileB;
     static constexpr size_t kSmem = 1024 + kBarOff + 256;
 };
 
-__device__ __forceinline__ uint64_t make_desc_kmajor_sw128(uint32_t saddr) {
+__device__ __forceinline__ uint64_t make_desc_kmajor(uint32_t saddr) {
     // SM100 smem matrix descriptor: start>>4 [0,14), LBO>>4 [16,30) (=1, unused for
-    // swizzled K-major), SBO>>4 [32,46) (1024 B between 8-row groups), version 1 [46,48),
-    // layout SWIZZLE_128B (2) [61,64)
-    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
-           ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+    // swizzled K-major), SBO>>4 [32,46) (512 B between 8-row groups of 64-B rows),
+    // version 1 [46,48), layout SWIZZLE_64B (4) [61,64)
+    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)1 << 16) | ((uint64_t)(kAtomBytes >> 4) << 32) |
+           ((uint64_t)1 << 46) | ((uint64_t)4 << 61);
 }
 
 // kind::tf32 instruction descriptor: D f32 [4,6)=1, A tf32 [7,10)=2, B tf32 [10,13)=2,
@@ -216,12 +219,12 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                     const uint32_t s_bl = s_al + kTileA;
 #pragma unroll
                     for (int kk = 0; kk < BK / 8; ++kk) {
-                        const uint64_t ah = make_desc_kmajor_sw128(s_ah + kk * 32);
-                        const uint64_t bh = make_desc_kmajor_sw128(s_bh + kk * 32);
+                        const uint64_t ah = make_desc_kmajor(s_ah + kk * 32);
+                        const uint64_t bh = make_desc_kmajor(s_bh + kk * 32);
                         const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
                         if (SPLIT == 3) {
-                            const uint64_t al = make_desc_kmajor_sw128(s_al + kk * 32);
-                            const uint64_t bl = make_desc_kmajor_sw128(s_bl + kk * 32);
+                            const uint64_t al = make_desc_kmajor(s_al + kk * 32);
+                            const uint64_t bl = make_desc_kmajor(s_bl + kk * 32);
                             mma_tf32(tmem_d, ah, bl, acc0);
                             mma_tf32(tmem_d, al, bh, 1u);
                             mma_tf32(tmem_d, ah, bh, 1u);
@@ -253,7 +256,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                 uint8_t* bh = op_stage(s) + kTileA;
                 uint8_t* bl = bh + kTileB + kTileA;
                 // (n, 4-k chunk) pairs: a warp covers 32 consecutive n of one chunk ->
-                // conflict-free reads (one 128-B row segment per k) and swizzled 16-B writes
+                // conflict-free reads (one 128-B row segment per k) and 64-B-swizzled 16-B
+                // writes (8 lanes fill 8 distinct 16-B bank slots)
 #pragma unroll 4
                 for (int p = ct; p < BN * (BK / 4); p += kConvThreads) {
                     const int nn = p & (BN - 1), c = p / BN;
@@ -262,7 +266,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                     x.y = rawB[(4 * c + 1) * BN + nn];
                     x.z = rawB[(4 * c + 2) * BN + nn];
                     x.w = rawB[(4 * c + 3) * BN + nn];
-                    const int off = nn * 128 + ((c ^ (nn & 7)) << 4);
+                    const int off = nn * kRowBytes + ((c ^ ((nn >> 1) & 3)) << 4);
                     *reinterpret_cast<float4*>(bh + off) = x;
                     if (SPLIT == 3) {
                         float4 y;

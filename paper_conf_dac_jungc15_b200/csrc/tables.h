@@ -45,9 +45,9 @@ constexpr int kSaxpyTile = kVecaddTile;
 constexpr int kBsVec = 2;
 constexpr int kBsTile = kEwThreads * 4 * kBsVec;               // 2048 options
 constexpr int kHistThreads = 256;
-constexpr int kHistVec = 8;                                    // uint4 (16 B) per thread
-constexpr int kHistTile = kHistThreads * 16 * kHistVec;        // 32768 bytes
+constexpr int kHistVec = 4;                                    // uint4 (16 B) per thread
+constexpr int kHistTile = kHistThreads * 16 * kHistVec;        // 16384 bytes
 constexpr int kGemmBM = 128, kGemmBN = 128, kGemmBK = 32;
-constexpr int kTf32BM = 128, kTf32BN = 256, kTf32BK = 32;
+constexpr int kTf32BM = 128, kTf32BN = 256, kTf32BK = 16;
 
 }  // namespace svp
