@@ -16,14 +16,14 @@
 // B operand returned zeros on B200 -- scripts/tc_probe.py, experiment E1 vs E2), so B
 // (row-major K x N, i.e. MN-major) is transposed in shared memory by converter warps.
 //
-// Roles (1 CTA per SM, persistent static tile walk, 320 threads):
+// Roles (1 CTA per SM, persistent static tile walk, 448 threads):
 //   warp 0        TMA producer: A tile 128x16 (K-major, 64-B swizzle) straight into the
 //                 operand stage; B tile 16x256 (row-major, no swizzle) into a raw staging
 //                 ring (4 deep, so B's L2 latency hides behind 3 stages of MMAs).
 //   warp 1        TMEM allocator (512 cols = 2 accumulators of 128x256 fp32) + MMA issuer:
 //                 one lane issues tcgen05.mma.cta_group::1.kind::tf32 M128 N256 K8 and
 //                 tcgen05.commit's to the stage's empty barrier / the accumulator barrier.
-//   warps 2,3,8,9 converters: B^T (K-major SW64, hi = raw bits) [+ B_lo^T, A_lo for SPLIT 3]
+//   warps 2,3,8-13 converters: B^T (K-major SW64, hi = raw bits) [+ B_lo^T, A_lo for SPLIT 3]
 //                 from the staged tiles; fence.proxy.async; arrive on the stage's conv barrier.
 //   warps 4-7     epilogue: tcgen05.ld 32x32b.x32 (warp w%4 owns TMEM lanes = tile rows
 //                 32(w%4)..+31), alpha*acc (+ beta*C), 128-bit stores; the two TMEM
@@ -40,8 +40,9 @@ namespace tc {
 constexpr int BM = kTf32BM, BN = kTf32BN, BK = kTf32BK;  // 128 x 256 x 16
 constexpr int kRowBytes = BK * 4;                          // 64-B K-major rows -> SWIZZLE_64B
 constexpr int kAtomBytes = 8 * kRowBytes;                  // 8-row swizzle atom (SBO)
-constexpr int kThreads = 320;
-constexpr int kConvThreads = 128;
+constexpr int kConvWarps = 8;                  // warps 2,3 and 8..13
+constexpr int kConvThreads = kConvWarps * 32;
+constexpr int kThreads = (8 + kConvWarps - 2) * 32;  // 448
 constexpr int kTileA = BM * BK * 4;   // 8 KiB
 constexpr int kTileB = BK * BN * 4;   // 16 KiB
 constexpr int kTmemCols = 512;
@@ -242,7 +243,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
         }
     } else if (warp < 4 || warp >= 8) {
         // ------------------------------------------------------------ converters
-        const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;  // 0..127
+        const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;  // 0..kConvThreads-1
         uint32_t it = 0;
         for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
             const int v = find_tile_owner(descs, n, t);
