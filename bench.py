@@ -338,6 +338,25 @@ def run_svp(args, rank, ws, local):
         except Exception:
             pass
 
+    # ---------------- the other implementation of the fp32 "sgemm" kernel, same jobs
+    alt = None
+    if not args.no_alt:
+        alt_impl = svp.SGEMM_FFMA if impl == svp.SGEMM_3XTF32 else svp.SGEMM_3XTF32
+        actx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, external_streams=[stream.cuda_stream],
+                           sgemm_impl=alt_impl)
+        for k in vs.kids:
+            actx.register_kernel(k)
+        actx.submit_batch(jobs)
+        actx.flush()
+        actx.reset_profile()
+        ks = max(3, args.steps // 5)
+        adt = max_over_ranks(timed_steps(actx, jobs, ks, stream), ws)
+        sk = actx.kernel_stats(vs.kids["sgemm"]) if "sgemm" in vs.kids else None
+        alt = {"sgemm_impl": "ffma" if alt_impl == svp.SGEMM_FFMA else "3xtf32", "value": n_jobs_total * ks / adt,
+               "unit": "jobs/s", "ms_per_step": adt / ks * 1e3,
+               "sgemm_tflops_interleaved": (sk["flops"] / sk["total_ns"] / 1e3) if sk and sk["total_ns"] else None}
+        actx.close()
+
     # ---------------- serial baselines on the same GPU, same buffers, same kernels
     serial = {}
     if not args.no_serial:
@@ -398,7 +417,7 @@ def run_svp(args, rank, ws, local):
             "hbm_gbs_membound": hbm_gbs,
             "hbm_frac_membound": (hbm_gbs / float(peaks["hbm_gbs"])) if hbm_gbs else None,
             "elements_per_s": sum(s.n for s in all_specs) * args.steps / dt_max,
-            "sgemm_impl": args.sgemm_impl,
+            "sgemm_impl": args.sgemm_impl, "alt_sgemm_impl": alt,
             "speedup_vs_serial": {k: value / v["value"] for k, v in serial.items()},
             "serial": serial, "per_kernel": per_kernel,
             "one_stream": {"value": iso_value, "unit": "jobs/s",
@@ -422,9 +441,10 @@ def main():
     ap.add_argument("--vps", type=int, default=None)
     ap.add_argument("--e2e-steps", type=int, default=0)
     ap.add_argument("--arena-gb", type=int, default=8)
-    ap.add_argument("--sgemm-impl", default="ffma", choices=["ffma", "3xtf32"],
+    ap.add_argument("--sgemm-impl", default="3xtf32", choices=["ffma", "3xtf32"],
                     help="implementation of the fp32 'sgemm' kernel (both meet its 1e-5 contract)")
     ap.add_argument("--no-serial", action="store_true")
+    ap.add_argument("--no-alt", action="store_true", help="skip timing the other sgemm implementation")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     args = ap.parse_args()

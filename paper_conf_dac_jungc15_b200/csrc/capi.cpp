@@ -90,6 +90,7 @@ void svp_config_default(svp_config* cfg) {
     cfg->max_chunks = 8;
     cfg->profile_level = 0;
     cfg->validate_ptrs = 1;
+    cfg->sgemm_impl = SVP_SGEMM_3XTF32;
 }
 
 svp_status svp_init(const svp_config* cfg, svp_ctx** out) {

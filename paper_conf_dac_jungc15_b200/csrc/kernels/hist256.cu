@@ -1,19 +1,36 @@
 // hist256.cu -- coalesced 256-bin byte histogram for sm_100a.
 //
 // counts_v[b] = #{i : d_v[i] == b} for every VP v of the group, in one launch.
-// Each tile lies in one VP.  A CTA keeps ONE shared histogram replicated per lane
-// (lane l of every warp increments column l, two 16-bit bins per 32-bit word), so the 32
-// addresses of a warp instruction sit in 32 distinct banks whatever the data (uniform
-// or 90 % one value): one smem wavefront per ATOMS, no same-address serialisation
-// inside an instruction.  One smem atomic per byte caps this kernel at the measured
-// shared-atomic rate (tools/ubench.py: ~3.7e12 lanes/s = 3.7 TB/s of input bytes).  The CTA flushes the replicas to
-// the VP's global counts (one atomicAdd per non-zero bin) whenever it moves to another
-// VP; a preceding tiny kernel zeroes every segment's counts, so the result overwrites
-// the output and is bit-exact (integer adds commute).
+//
+// A histogram needs one increment per input byte; done with shared-memory atomics that
+// caps the kernel at the measured smem-atomic rate (tools/ubench.py: ~3.7e12 lanes/s =
+// 3.7 TB/s of input, ~56 % of HBM), so the design goal is to keep the atomics busy and
+// never let them wait on DRAM:
+//  * a producer warp streams each tile global -> shared with 1-D bulk copies
+//    (cp.async.bulk, mbarrier complete_tx) into a 3-stage ring, so DRAM latency is hidden
+//    behind the consumers' atomics;
+//  * 8 consumer warps read the staged tile (LDS.128, conflict-free) and increment a CTA
+//    histogram replicated per lane -- h[word][lane], two 16-bit bins per word -- so the
+//    32 addresses of every warp ATOMS sit in 32 distinct banks whatever the data
+//    (uniform or 90 % one value): one smem wavefront per instruction;
+//  * CTAs walk contiguous (blocked) tile ranges, so a CTA stays in one VP for many tiles
+//    and flushes its replicas to the VP's global counts (one atomicAdd per non-zero bin)
+//    only at VP boundaries or every kHistFlushTiles tiles (16-bit overflow guard).
+// A VP's ragged head/tail tiles (not 16-B aligned / partial) are read from global memory
+// directly.  A preceding tiny kernel zeroes every segment's counts, so the result
+// overwrites the output and is bit-exact (integer adds commute).
 #include "../launch.h"
 #include "common.cuh"
 
 namespace svp {
+
+constexpr int kHistConsumers = kHistThreads;          // 256 = 8 warps
+constexpr int kHistBlock = kHistConsumers + 32;       // + producer warp
+constexpr int kHistStages = 3;
+constexpr int kHistWords = 128;
+constexpr int kHistFlushTiles = 32;
+static_assert(kHistFlushTiles * (kHistConsumers / 32) * kHistVec * 16 < 65536, "16-bit half-counters overflow");
+constexpr int kHistSmem = kHistStages * kHistTile + kHistWords * 32 * 4 + 2 * kHistStages * 8 + 128;
 
 __global__ void __launch_bounds__(256) k_hist_zero(const SegDesc* __restrict__ segs, int nsegs) {
     for (int s = blockIdx.x; s < nsegs; s += gridDim.x) {
@@ -22,15 +39,17 @@ __global__ void __launch_bounds__(256) k_hist_zero(const SegDesc* __restrict__ s
     }
 }
 
-// Shared table h[word][lane], word = bin & 127, 16-bit half = bin >> 7: 128 x 32 u32 =
-// 16 KiB per CTA, so 8 CTAs (2048 threads) fit an SM and keep enough loads in flight.
-// hl points at column `lane` of word 0.  A half-counter gains at most 8 warps x
-// kHistVec x 16 increments per tile, so flushing every kHistFlushTiles tiles keeps it
-// below 2^16.
-constexpr int kHistWords = 128;
-constexpr int kHistFlushTiles = 32;
-static_assert(kHistFlushTiles * (kHistThreads / 32) * kHistVec * 16 < 65536, "16-bit half-counters overflow");
+__device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kHistConsumers) : "memory"); }
 
+__device__ __forceinline__ void bulk_g2s(void* smem_dst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(smem_dst)),
+        "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
+// hl points at column `lane` of word 0; bin b lives in word b & 127, half b >> 7.
 __device__ __forceinline__ void hist_add_byte(uint32_t* hl, uint32_t b) {
     atomicAdd(hl + ((b & 127u) << 5), 1u << ((b >> 7) << 4));
 }
@@ -43,9 +62,9 @@ __device__ __forceinline__ void hist_add_word(uint32_t* hl, uint32_t w) {
 
 // Sum the 32 lane replicas of each word (thread t < 128 owns word t; the column walk is
 // rotated by t so a warp's 32 reads hit 32 banks), zero them, and add both halves to the
-// VP's counts (bins t and t + 128).
+// VP's counts (bins t and t + 128).  Consumers only (named barrier 1).
 __device__ __forceinline__ void hist_flush(uint32_t* h, uint32_t* counts) {
-    __syncthreads();
+    consumers_sync();
     const int w = threadIdx.x;
     if (w < kHistWords) {
         uint32_t lo = 0, hi = 0;
@@ -60,21 +79,60 @@ __device__ __forceinline__ void hist_flush(uint32_t* h, uint32_t* counts) {
         if (lo) atomicAdd(&counts[w], lo);
         if (hi) atomicAdd(&counts[w + 128], hi);
     }
-    __syncthreads();
+    consumers_sync();
 }
 
-__global__ void __launch_bounds__(kHistThreads) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
-    __shared__ uint32_t h[kHistWords * 32];
-    for (int i = threadIdx.x; i < kHistWords * 32; i += kHistThreads) h[i] = 0;
+__global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
+    extern __shared__ __align__(128) uint8_t hsm[];
+    uint8_t* ring = hsm;                                                         // [stages][tile]
+    uint32_t* h = reinterpret_cast<uint32_t*>(hsm + kHistStages * kHistTile);     // [128][32]
+    uint64_t* full = reinterpret_cast<uint64_t*>(h + kHistWords * 32);
+    uint64_t* empty = full + kHistStages;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+    for (int i = threadIdx.x; i < kHistWords * 32; i += kHistBlock) h[i] = 0;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kHistStages; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kHistConsumers / 32);
+        }
+        mbar_fence_init();
+    }
     __syncthreads();
-    uint32_t* hl = h + (threadIdx.x & 31);
+
+    // blocked tile ranges
+    const uint32_t per = (total + gridDim.x - 1) / gridDim.x;
+    const uint32_t t0 = min(total, blockIdx.x * per), t1 = min(total, t0 + per);
+
+    if (warp == kHistConsumers / 32) {
+        // ------------------------------------------------------------ producer
+        if (lane == 0) {
+            uint32_t it = 0;
+            for (uint32_t t = t0; t < t1; ++t, ++it) {
+                const int s = it % kHistStages;
+                const uint32_t ph = (it / kHistStages) & 1;
+                const SegDesc& sd = segs[find_seg(segs, nsegs, t)];
+                int64_t e0, e1;
+                bool vec;
+                tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, kHistTile, e0, e1, vec);
+                mbar_wait(&empty[s], ph ^ 1);
+                if (vec) {
+                    mbar_expect_tx(&full[s], kHistTile);
+                    bulk_g2s(ring + s * kHistTile, reinterpret_cast<const uint8_t*>(sd.ptr[0]) + e0, kHistTile, &full[s]);
+                } else {
+                    mbar_arrive(&full[s]);  // consumers read this tile from global memory
+                }
+            }
+        }
+        return;  // no CTA-wide barrier after this point
+    }
+
+    // ---------------------------------------------------------------- consumers
+    uint32_t* hl = h + lane;
     int cur = -1, since_flush = 0;
     uint32_t* cur_counts = nullptr;
-    // blocked tile ranges: a CTA walks contiguous tiles, so it stays inside one VP for
-    // many tiles and flushes only at VP boundaries (or every kHistFlushTiles tiles)
-    const uint32_t per = (total + gridDim.x - 1) / gridDim.x;
-    const uint32_t t0 = blockIdx.x * per, t1 = min(total, t0 + per);
-    for (uint32_t t = t0; t < t1; ++t) {
+    uint32_t it = 0;
+    for (uint32_t t = t0; t < t1; ++t, ++it) {
         const int si = find_seg(segs, nsegs, t);
         const SegDesc& sd = segs[si];
         if (si != cur || since_flush == kHistFlushTiles) {
@@ -84,15 +142,19 @@ __global__ void __launch_bounds__(kHistThreads) k_hist256(const SegDesc* __restr
             cur_counts = reinterpret_cast<uint32_t*>(sd.ptr[1]);
         }
         ++since_flush;
-        const uint8_t* __restrict__ d = reinterpret_cast<const uint8_t*>(sd.ptr[0]);
         int64_t e0, e1;
         bool vec;
         tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, kHistTile, e0, e1, vec);
+        const int s = it % kHistStages;
+        const uint32_t ph = (it / kHistStages) & 1;
+        mbar_wait(&full[s], ph);
         if (vec) {
-            const uint4* d4 = reinterpret_cast<const uint4*>(d + e0) + threadIdx.x;
+            const uint4* st = reinterpret_cast<const uint4*>(ring + s * kHistTile) + threadIdx.x;
             uint4 r[kHistVec];
 #pragma unroll
-            for (int i = 0; i < kHistVec; ++i) r[i] = __ldcs(d4 + i * kHistThreads);
+            for (int i = 0; i < kHistVec; ++i) r[i] = st[i * kHistConsumers];
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);  // stage consumed (data now in registers)
 #pragma unroll
             for (int i = 0; i < kHistVec; ++i) {
                 hist_add_word(hl, r[i].x);
@@ -101,25 +163,36 @@ __global__ void __launch_bounds__(kHistThreads) k_hist256(const SegDesc* __restr
                 hist_add_word(hl, r[i].w);
             }
         } else {
-            for (int64_t e = e0 + threadIdx.x; e < e1; e += kHistThreads) hist_add_byte(hl, d[e]);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+            const uint8_t* __restrict__ d = reinterpret_cast<const uint8_t*>(sd.ptr[0]);
+            for (int64_t e = e0 + threadIdx.x; e < e1; e += kHistConsumers) hist_add_byte(hl, d[e]);
         }
     }
     if (cur >= 0) hist_flush(h, cur_counts);
 }
-
-constexpr int kHistSmem = 0;  // static shared table
 
 cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
     if (nsegs <= 0) return cudaSuccess;
     k_hist_zero<<<nsegs < 1024 ? nsegs : 1024, 256, 0, s>>>(segs, nsegs);
     cudaError_t e = cudaGetLastError();
     if (e || total == 0) return e;
-    k_hist256<<<grid, kHistThreads, kHistSmem, s>>>(segs, nsegs, total);
+    static bool attr[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 64 && !attr[dev]) {
+        e = cudaFuncSetAttribute(k_hist256, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmem);
+        if (e) return e;
+        attr[dev] = true;
+    }
+    k_hist256<<<grid, kHistBlock, kHistSmem, s>>>(segs, nsegs, total);
     return cudaGetLastError();
 }
 
 cudaError_t query_limits_hist(int* per_sm) {
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k_hist256, kHistThreads, kHistSmem);
+    cudaError_t e = cudaFuncSetAttribute(k_hist256, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmem);
+    if (e) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k_hist256, kHistBlock, kHistSmem);
 }
 
 }  // namespace svp

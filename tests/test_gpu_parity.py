@@ -77,23 +77,25 @@ def test_config3_interleaved_host():
         check_job(s, inp, got, w)
 
 
+@pytest.mark.parametrize("impl", [svp.SGEMM_FFMA, svp.SGEMM_3XTF32])
 @pytest.mark.parametrize("int_inputs", [True, False])
-def test_config2_sgemm_512(int_inputs):
+def test_config2_sgemm_512(int_inputs, impl):
     specs = W.config_specs(2, sgemm_int=int_inputs)
     inputs = inputs_for(specs)
-    outs, _, st = run_svp(specs, inputs, "device")
+    outs, _, st = run_svp(specs, inputs, "device", sgemm_impl=impl)
     assert st["launches"] == 1
     want = oracle.run_jobs(specs, inputs)
     for s, inp, got, w in zip(specs, inputs, outs, want):
         check_job(s, inp, got, w)
 
 
-def test_sgemm_alpha_beta_ragged_edges():
+@pytest.mark.parametrize("impl", [svp.SGEMM_FFMA, svp.SGEMM_3XTF32])
+def test_sgemm_alpha_beta_ragged_edges(impl):
     specs = []
     for v, (M, N, K) in enumerate([(200, 136, 40), (200, 136, 40), (1, 4, 4), (129, 260, 0), (64, 68, 1000)]):
         specs.append(W.JobSpec(v, "sgemm", M=M, N=N, K=K, alpha=1.5, beta=-0.5))
     inputs = inputs_for(specs)
-    outs, _, _ = run_svp(specs, inputs, "device")
+    outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl)
     for s, inp, got in zip(specs, inputs, outs):
         check_job(s, inp, got)
 
