@@ -10,12 +10,13 @@
 //    (cp.async.bulk, mbarrier complete_tx) into a 3-stage ring, so DRAM latency is hidden
 //    behind the consumers' atomics;
 //  * 8 consumer warps read the staged tile (LDS.128, conflict-free) and increment a CTA
-//    histogram replicated per lane -- h[word][lane], two 16-bit bins per word -- so the
-//    32 addresses of every warp ATOMS sit in 32 distinct banks whatever the data
-//    (uniform or 90 % one value): one smem wavefront per instruction;
+//    histogram replicated per lane -- h[bin][lane], 256 x 32 u32 = 32 KiB -- so the 32
+//    addresses of every warp ATOMS sit in 32 distinct banks whatever the data (uniform
+//    or 90 % one value): one smem wavefront per instruction.  (Packing two 16-bit bins
+//    per word halves the table but costs instructions: 2.5 vs 3.7 Tlanes/s measured.)
 //  * CTAs walk contiguous (blocked) tile ranges, so a CTA stays in one VP for many tiles
-//    and flushes its replicas to the VP's global counts (one atomicAdd per non-zero bin)
-//    only at VP boundaries or every kHistFlushTiles tiles (16-bit overflow guard).
+//    (segment lookups are cached) and flushes its replicas to the VP's global counts
+//    (one atomicAdd per non-zero bin) only at VP boundaries.
 // A VP's ragged head/tail tiles (not 16-B aligned / partial) are read from global memory
 // directly.  A preceding tiny kernel zeroes every segment's counts, so the result
 // overwrites the output and is bit-exact (integer adds commute).
@@ -27,10 +28,8 @@ namespace svp {
 constexpr int kHistConsumers = kHistThreads;          // 256 = 8 warps
 constexpr int kHistBlock = kHistConsumers + 32;       // + producer warp
 constexpr int kHistStages = 3;
-constexpr int kHistWords = 128;
-constexpr int kHistFlushTiles = 32;
-static_assert(kHistFlushTiles * (kHistConsumers / 32) * kHistVec * 16 < 65536, "16-bit half-counters overflow");
-constexpr int kHistSmem = kHistStages * kHistTile + kHistWords * 32 * 4 + 2 * kHistStages * 8 + 128;
+constexpr int kHistBins = 256;
+constexpr int kHistSmem = kHistStages * kHistTile + kHistBins * 32 * 4 + 2 * kHistStages * 8 + 128;
 
 __global__ void __launch_bounds__(256) k_hist_zero(const SegDesc* __restrict__ segs, int nsegs) {
     for (int s = blockIdx.x; s < nsegs; s += gridDim.x) {
@@ -49,10 +48,8 @@ __device__ __forceinline__ void bulk_g2s(void* smem_dst, const void* gsrc, uint3
         : "memory");
 }
 
-// hl points at column `lane` of word 0; bin b lives in word b & 127, half b >> 7.
-__device__ __forceinline__ void hist_add_byte(uint32_t* hl, uint32_t b) {
-    atomicAdd(hl + ((b & 127u) << 5), 1u << ((b >> 7) << 4));
-}
+// hl points at column `lane` of bin 0: hl[b * 32] is this lane's counter for bin b.
+__device__ __forceinline__ void hist_add_byte(uint32_t* hl, uint32_t b) { atomicAdd(hl + (b << 5), 1u); }
 __device__ __forceinline__ void hist_add_word(uint32_t* hl, uint32_t w) {
     hist_add_byte(hl, w & 0xFFu);
     hist_add_byte(hl, (w >> 8) & 0xFFu);
@@ -60,37 +57,48 @@ __device__ __forceinline__ void hist_add_word(uint32_t* hl, uint32_t w) {
     hist_add_byte(hl, w >> 24);
 }
 
-// Sum the 32 lane replicas of each word (thread t < 128 owns word t; the column walk is
-// rotated by t so a warp's 32 reads hit 32 banks), zero them, and add both halves to the
-// VP's counts (bins t and t + 128).  Consumers only (named barrier 1).
+// Sum the 32 lane replicas of each bin (thread t owns bin t; the column walk is rotated
+// by t so a warp's 32 reads hit 32 banks), zero them, and add to the VP's counts.
+// Consumers only (named barrier 1).
 __device__ __forceinline__ void hist_flush(uint32_t* h, uint32_t* counts) {
+    static_assert(kHistConsumers == kHistBins, "one flush thread per bin");
     consumers_sync();
-    const int w = threadIdx.x;
-    if (w < kHistWords) {
-        uint32_t lo = 0, hi = 0;
+    const int b = threadIdx.x;
+    uint32_t sum = 0;
 #pragma unroll 8
-        for (int j = 0; j < 32; ++j) {
-            const int c = (j + w) & 31;
-            const uint32_t v = h[w * 32 + c];
-            lo += v & 0xFFFFu;
-            hi += v >> 16;
-            h[w * 32 + c] = 0;
-        }
-        if (lo) atomicAdd(&counts[w], lo);
-        if (hi) atomicAdd(&counts[w + 128], hi);
+    for (int j = 0; j < 32; ++j) {
+        const int c = (j + b) & 31;
+        sum += h[b * 32 + c];
+        h[b * 32 + c] = 0;
     }
+    if (sum) atomicAdd(&counts[b], sum);
     consumers_sync();
 }
+
+// Segment of tile t with a one-entry cache (tiles of a CTA are contiguous): [lo, hi) is
+// the tile range the cached segment owns.
+struct SegCache {
+    int si = -1;
+    uint32_t lo = 1, hi = 0;
+    __device__ __forceinline__ int get(const SegDesc* __restrict__ segs, int nsegs, uint32_t total, uint32_t t) {
+        if (t < lo || t >= hi) {
+            si = find_seg(segs, nsegs, t);
+            lo = segs[si].tile_begin;
+            hi = si + 1 < nsegs ? segs[si + 1].tile_begin : total;
+        }
+        return si;
+    }
+};
 
 __global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
     extern __shared__ __align__(128) uint8_t hsm[];
     uint8_t* ring = hsm;                                                         // [stages][tile]
-    uint32_t* h = reinterpret_cast<uint32_t*>(hsm + kHistStages * kHistTile);     // [128][32]
-    uint64_t* full = reinterpret_cast<uint64_t*>(h + kHistWords * 32);
+    uint32_t* h = reinterpret_cast<uint32_t*>(hsm + kHistStages * kHistTile);     // [256][32]
+    uint64_t* full = reinterpret_cast<uint64_t*>(h + kHistBins * 32);
     uint64_t* empty = full + kHistStages;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
-    for (int i = threadIdx.x; i < kHistWords * 32; i += kHistBlock) h[i] = 0;
+    for (int i = threadIdx.x; i < kHistBins * 32; i += kHistBlock) h[i] = 0;
     if (threadIdx.x == 0) {
         for (int s = 0; s < kHistStages; ++s) {
             mbar_init(&full[s], 1);
@@ -108,10 +116,11 @@ __global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restric
         // ------------------------------------------------------------ producer
         if (lane == 0) {
             uint32_t it = 0;
+            SegCache sc;
             for (uint32_t t = t0; t < t1; ++t, ++it) {
                 const int s = it % kHistStages;
                 const uint32_t ph = (it / kHistStages) & 1;
-                const SegDesc& sd = segs[find_seg(segs, nsegs, t)];
+                const SegDesc& sd = segs[sc.get(segs, nsegs, total, t)];
                 int64_t e0, e1;
                 bool vec;
                 tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, kHistTile, e0, e1, vec);
@@ -129,19 +138,18 @@ __global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restric
 
     // ---------------------------------------------------------------- consumers
     uint32_t* hl = h + lane;
-    int cur = -1, since_flush = 0;
+    int cur = -1;
     uint32_t* cur_counts = nullptr;
     uint32_t it = 0;
+    SegCache sc;
     for (uint32_t t = t0; t < t1; ++t, ++it) {
-        const int si = find_seg(segs, nsegs, t);
+        const int si = sc.get(segs, nsegs, total, t);
         const SegDesc& sd = segs[si];
-        if (si != cur || since_flush == kHistFlushTiles) {
+        if (si != cur) {
             if (cur >= 0) hist_flush(h, cur_counts);
             cur = si;
-            since_flush = 0;
             cur_counts = reinterpret_cast<uint32_t*>(sd.ptr[1]);
         }
-        ++since_flush;
         int64_t e0, e1;
         bool vec;
         tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, kHistTile, e0, e1, vec);

@@ -46,6 +46,31 @@ __global__ void k_atoms(uint32_t* out, int iters) {
     }
 }
 
+// 16-bit packed variant: h[128][32] words, bin b -> word b & 127, half b >> 7
+__global__ void k_atoms16(uint32_t* out, int iters) {
+    __shared__ uint32_t h[128 * 32];
+    for (int i = threadIdx.x; i < 128 * 32; i += blockDim.x) h[i] = 0;
+    __syncthreads();
+    uint32_t x = 0x9E3779B9u * (threadIdx.x + 1) ^ blockIdx.x;
+    uint32_t* hl = h + (threadIdx.x & 31);
+    for (int it = 0; it < iters; ++it) {
+        x ^= x << 13;
+        x ^= x >> 17;
+        x ^= x << 5;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            uint32_t b = (x >> (8 * k)) & 0xFFu;
+            atomicAdd(hl + ((b & 127u) << 5), 1u << ((b >> 7) << 4));
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t s = 0;
+        for (int i = 0; i < 128 * 32; ++i) s += (h[i] & 0xFFFF) + (h[i] >> 16);
+        atomicAdd(out, s);
+    }
+}
+
 __global__ void k_ffma(float* out, int iters) {
     float a0 = threadIdx.x, a1 = a0 + 1, a2 = a0 + 2, a3 = a0 + 3, a4 = a0 + 4, a5 = a0 + 5, a6 = a0 + 6, a7 = a0 + 7;
     const float b = 0.999f, c = 0.001f;
@@ -66,6 +91,10 @@ int ub_copy(const void* a, void* b, size_t bytes, int grid, int block, void* str
 }
 int ub_atoms(uint32_t* out, int iters, int grid, int block, void* stream) {
     k_atoms<<<grid, block, 0, (cudaStream_t)stream>>>(out, iters);
+    return (int)cudaGetLastError();
+}
+int ub_atoms16(uint32_t* out, int iters, int grid, int block, void* stream) {
+    k_atoms16<<<grid, block, 0, (cudaStream_t)stream>>>(out, iters);
     return (int)cudaGetLastError();
 }
 int ub_ffma(float* out, int iters, int grid, int block, void* stream) {

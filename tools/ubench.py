@@ -49,6 +49,7 @@ def main():
     L.ub_copy.argtypes = [vp, vp, ctypes.c_size_t, ctypes.c_int, ctypes.c_int, vp]
     L.ub_atoms.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, vp]
     L.ub_ffma.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, vp]
+    L.ub_atoms16.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, vp]
     props = torch.cuda.get_device_properties(0)
     sms = props.multi_processor_count
     st = torch.cuda.current_stream().cuda_stream
@@ -72,6 +73,16 @@ def main():
         res[f"smem_atomic_lanes_per_clk_per_sm_{blocks_per_sm}cta"] = lanes / t / sms / (props.clock_rate * 1e3) \
             if hasattr(props, "clock_rate") else None
     res["hist256_ceiling_gbs_if_atomic_bound"] = res["smem_atomics_per_s_6cta"] / 1e9
+    sweep = {}
+    for fn, name in ((L.ub_atoms, "u32"), (L.ub_atoms16, "u16x2")):
+        for block in (256, 512):
+            for bps in (1, 2, 3, 4, 6, 8):
+                if block * bps > 2048:
+                    continue
+                grid = sms * bps
+                t = timed(lambda: fn(out.data_ptr(), iters, grid, block, st))
+                sweep[f"{name}_b{block}_x{bps}"] = round(grid * block * iters * 4 / t / 1e12, 3)
+    res["smem_atomics_Tlanes_per_s_sweep"] = sweep
 
     f = torch.zeros(1, device="cuda")
     fi = 2000
