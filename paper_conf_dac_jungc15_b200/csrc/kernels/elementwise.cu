@@ -17,6 +17,8 @@
 
 namespace svp {
 
+constexpr int kScalarU = 4;  // independent loads per thread in the scalar (ragged) path
+
 // --------------------------------------------------------------------- vecadd
 __global__ void __launch_bounds__(kEwThreads) k_vecadd(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
     constexpr int V = kVecaddVec, TILE = kVecaddTile;
@@ -49,7 +51,23 @@ __global__ void __launch_bounds__(kEwThreads) k_vecadd(const SegDesc* __restrict
                 __stcs(c4 + i * kEwThreads, r);
             }
         } else {
-            for (int64_t e = e0 + threadIdx.x; e < e1; e += kEwThreads) c[e] = __fadd_rn(a[e], b[e]);
+            // ragged head/tail: batch kScalarU independent loads before the stores
+            for (int64_t e = e0 + threadIdx.x; e < e1; e += kEwThreads * kScalarU) {
+                float ra[kScalarU], rb[kScalarU];
+#pragma unroll
+                for (int k = 0; k < kScalarU; ++k) {
+                    const int64_t i = e + k * kEwThreads;
+                    if (i < e1) {
+                        ra[k] = a[i];
+                        rb[k] = b[i];
+                    }
+                }
+#pragma unroll
+                for (int k = 0; k < kScalarU; ++k) {
+                    const int64_t i = e + k * kEwThreads;
+                    if (i < e1) c[i] = __fadd_rn(ra[k], rb[k]);
+                }
+            }
         }
     }
 }
@@ -85,7 +103,22 @@ __global__ void __launch_bounds__(kEwThreads) k_saxpy(const SegDesc* __restrict_
                 __stcs(y4 + i * kEwThreads, r);
             }
         } else {
-            for (int64_t e = e0 + threadIdx.x; e < e1; e += kEwThreads) y[e] = __fmaf_rn(a, x[e], y[e]);
+            for (int64_t e = e0 + threadIdx.x; e < e1; e += kEwThreads * kScalarU) {
+                float rx[kScalarU], ry[kScalarU];
+#pragma unroll
+                for (int k = 0; k < kScalarU; ++k) {
+                    const int64_t i = e + k * kEwThreads;
+                    if (i < e1) {
+                        rx[k] = x[i];
+                        ry[k] = y[i];
+                    }
+                }
+#pragma unroll
+                for (int k = 0; k < kScalarU; ++k) {
+                    const int64_t i = e + k * kEwThreads;
+                    if (i < e1) y[i] = __fmaf_rn(a, rx[k], ry[k]);
+                }
+            }
         }
     }
 }
@@ -151,11 +184,28 @@ __global__ void __launch_bounds__(kEwThreads) k_blackscholes(const SegDesc* __re
                 __stcs(reinterpret_cast<float4*>(P + e0) + o + i * kEwThreads, p);
             }
         } else {
-            for (int64_t e = e0 + threadIdx.x; e < e1; e += kEwThreads) {
-                float c, p;
-                bs_one(S[e], X[e], T[e], R, Vol, c, p);
-                C[e] = c;
-                P[e] = p;
+            for (int64_t e = e0 + threadIdx.x; e < e1; e += kEwThreads * kScalarU) {
+                float rs[kScalarU], rx[kScalarU], rt[kScalarU];
+#pragma unroll
+                for (int k = 0; k < kScalarU; ++k) {
+                    const int64_t i = e + k * kEwThreads;
+                    rs[k] = rx[k] = rt[k] = 1.f;
+                    if (i < e1) {
+                        rs[k] = S[i];
+                        rx[k] = X[i];
+                        rt[k] = T[i];
+                    }
+                }
+#pragma unroll
+                for (int k = 0; k < kScalarU; ++k) {
+                    const int64_t i = e + k * kEwThreads;
+                    if (i < e1) {
+                        float c, p;
+                        bs_one(rs[k], rx[k], rt[k], R, Vol, c, p);
+                        C[i] = c;
+                        P[i] = p;
+                    }
+                }
             }
         }
     }

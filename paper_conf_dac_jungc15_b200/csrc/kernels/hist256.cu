@@ -173,8 +173,19 @@ __global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restric
         } else {
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
+            // ragged head/tail tile: 8 independent byte loads in flight per thread
             const uint8_t* __restrict__ d = reinterpret_cast<const uint8_t*>(sd.ptr[0]);
-            for (int64_t e = e0 + threadIdx.x; e < e1; e += kHistConsumers) hist_add_byte(hl, d[e]);
+            for (int64_t e = e0 + threadIdx.x; e < e1; e += kHistConsumers * 8) {
+                uint32_t v[8];
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    const int64_t i = e + k * kHistConsumers;
+                    v[k] = i < e1 ? (uint32_t)d[i] : 256u;
+                }
+#pragma unroll
+                for (int k = 0; k < 8; ++k)
+                    if (v[k] < 256u) hist_add_byte(hl, v[k]);
+            }
         }
     }
     if (cur >= 0) hist_flush(h, cur_counts);
