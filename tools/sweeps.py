@@ -1,0 +1,173 @@
+"""Reproduce the paper's coalescing / interleaving experiments on B200 with libsvp.
+
+    python tools/sweeps.py [--out profiles/r01/sweeps.json] [--quick]
+
+S1 (Fig 10a): vectorAdd, constant total 2^26 elements split over N
+    VPs; one coalesced flush vs the same N jobs launched serially (B1: one launch per job,
+    sync after each; B2: no syncs).  Paper (Quadro 4000): 10.54x at N=16, 20.48x at N=64.
+S2 (Fig 10b + Eq 9): one vecadd VP of n = k tiles; kernel time vs k
+    is a staircase with step lambda = #SMs x resident CTAs (Eq 9's aligned unit).
+S3 (Fig 9 + Eq 7/8): N host-resident SGEMM jobs (H2D A,B -> kernel ->
+    D2H C) with Tk ~ Tm, interleaved on separate copy/compute streams vs one stream;
+    measured speedup next to Eq 7's prediction from the measured Tm, Tk.
+S4 (BASELINE metric): jobs/s of the cfg5 mix vs #VPs (1 GPU).
+Times are CUDA-event device times around whole flushes (median of reps).
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+from paper_conf_dac_jungc15_b200 import svp  # noqa: E402
+from paper_conf_dac_jungc15_b200.vpset import VPSet  # noqa: E402
+
+
+def flush_time(ctx, jobs, reps=5, warm=2):
+    s = torch.cuda.current_stream()
+    for _ in range(warm):
+        ctx.submit_batch(jobs)
+        ctx.flush()
+    ts = []
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record(s)
+        ctx.submit_batch(jobs)
+        ctx.flush()
+        e1.record(s)
+        torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1) / 1e3)
+    return statistics.median(ts)
+
+
+def ctx_for(**kw):
+    return svp.Context(num_gpus=1, external_streams=[torch.cuda.current_stream().cuda_stream], **kw)
+
+
+def s1_coalescing(quick):
+    total = 1 << 26
+    out = []
+    for N in ([1, 4, 16, 64] if quick else [1, 2, 4, 8, 16, 32, 64, 128, 256]):
+        specs = [W.JobSpec(v, "vecadd", n=total // N) for v in range(N)]
+        c = ctx_for()
+        vs = VPSet(c, specs, [W.make_inputs(s) for s in specs], "device")
+        jobs = vs.job_list()
+        t_coal = flush_time(c, jobs)
+        row = {"N": N, "coalesced_ms": t_coal * 1e3}
+        for name, kw in (("B1_serial_sync", dict(coalesce=False, interleave=False, sync_each_job=True)),
+                         ("B2_serial_async", dict(coalesce=False, interleave=False))):
+            sc = ctx_for(**kw)
+            sc.register_kernel("vecadd")
+            t = flush_time(sc, jobs)
+            row[name + "_ms"] = t * 1e3
+            row["speedup_vs_" + name] = t / t_coal
+            sc.close()
+        row["coalesced_gbs"] = 12 * total / t_coal / 1e9
+        out.append(row)
+        c.close()
+        del vs
+        torch.cuda.empty_cache()
+    return out
+
+
+def s2_staircase(quick):
+    c = ctx_for(profile_level=1, interleave=False)
+    kid = c.register_kernel("vecadd")
+    lim_tile = 4096
+    props = torch.cuda.get_device_properties(0)
+    rows = []
+    ks = list(range(148, 148 * 8 * 3 + 1, 148 if quick else 74))
+    nmax = max(ks) * lim_tile
+    a = torch.rand(nmax, device="cuda")
+    b = torch.rand(nmax, device="cuda")
+    cc = torch.empty(nmax, device="cuda")
+    for k in ks:
+        n = k * lim_tile
+        job = (0, kid, svp.args_vecadd(n), [(a.data_ptr(), 4 * n, 1, 0), (b.data_ptr(), 4 * n, 1, 0),
+                                            (cc.data_ptr(), 4 * n, 2, 0)])
+        c.reset_profile()
+        flush_time(c, [job], reps=7)
+        st = c.kernel_stats(kid)
+        rows.append({"tiles": k, "elements": n, "kernel_us": st["total_ns"] / st["launches"] / 1e3})
+    c.close()
+    return {"sms": props.multi_processor_count, "tile_elements": lim_tile, "rows": rows}
+
+
+def s3_interleaving(quick):
+    """N host-resident FFMA SGEMMs of n^3 with Tk ~ Tm (Fig 9b); no coalescing, so only the
+    Copy/Compute-engine interleaving differs between the two runs."""
+    n = 3072
+    rows = []
+    for N in ([2, 4, 8] if quick else [2, 4, 8, 16, 32]):
+        specs = [W.JobSpec(v, "sgemm", M=n, N=n, K=n) for v in range(N)]
+        inputs = [W.make_inputs(s) for s in specs]
+        res = {}
+        for name, kw in (("interleaved", dict(coalesce=False, interleave=True)),
+                         ("serial", dict(coalesce=False, interleave=False))):
+            c = ctx_for(sgemm_impl=svp.SGEMM_FFMA, profile_level=1, arena_bytes=8 << 30, **kw)
+            vs = VPSet(c, specs, inputs, "host")
+            t = flush_time(c, vs.job_list(), reps=3, warm=1)
+            res[name] = t
+            if name == "serial":
+                ops = c.plan()
+                tin = statistics.median([o["measured_ns"] for o in ops if o["kind"] == svp.OP_H2D]) / 1e6
+                tk = statistics.median([o["measured_ns"] for o in ops if o["kind"] == svp.OP_KERNEL]) / 1e6
+                tout = statistics.median([o["measured_ns"] for o in ops if o["kind"] == svp.OP_D2H]) / 1e6
+            c.close()
+            del vs
+            torch.cuda.empty_cache()
+        tm = tin
+        eq7 = 2 * tm + N * max(tm, tk)
+        rows.append({"N": N, "Tin_ms": tin, "Tk_ms": tk, "Tout_ms": tout, "serial_ms": res["serial"] * 1e3,
+                     "interleaved_ms": res["interleaved"] * 1e3, "speedup": res["serial"] / res["interleaved"],
+                     "eq7_pred_ms": eq7, "eq8_speedup_if_equal": 3 * N / (2 + N)})
+    return {"sgemm_n": n, "rows": rows}
+
+
+def s4_vps(quick):
+    rows = []
+    for nv in ([16, 64, 256] if quick else [2, 4, 8, 16, 32, 64, 128, 256]):
+        specs = W.config_specs(5, nvps=nv)
+        c = ctx_for()
+        vs = VPSet(c, specs, W.make_inputs_many(specs), "device")
+        t = flush_time(c, vs.job_list(), reps=5)
+        rows.append({"vps": nv, "ms": t * 1e3, "jobs_per_s": nv / t})
+        c.close()
+        del vs
+        torch.cuda.empty_cache()
+    return rows
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--out", default=None)
+    ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--only", default="1234")
+    args = ap.parse_args()
+    torch.cuda.set_device(0)
+    res = {"gpu": torch.cuda.get_device_name(0)}
+    if "1" in args.only:
+        res["S1_coalescing_fig10a"] = s1_coalescing(args.quick)
+    if "2" in args.only:
+        res["S2_staircase_fig10b"] = s2_staircase(args.quick)
+    if "3" in args.only:
+        res["S3_interleaving_fig9"] = s3_interleaving(args.quick)
+    if "4" in args.only:
+        res["S4_jobs_vs_vps"] = s4_vps(args.quick)
+    txt = json.dumps(res, indent=1)
+    print(txt)
+    if args.out:
+        with open(args.out, "w") as f:
+            f.write(txt + "\n")
+
+
+if __name__ == "__main__":
+    main()
