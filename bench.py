@@ -252,7 +252,7 @@ def run_svp(args, rank, ws, local):
     ctx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, external_streams=[stream.cuda_stream],
                       validate_ptrs=True, sgemm_impl=impl)
     vs = VPSet(ctx, specs, inputs, "device", device_ordinals=[local])
-    jobs = vs.job_list()
+    jobs = svp.JobBatch(vs.job_list())  # marshalled once; each step resubmits it
     ctx.submit_batch(jobs)
     ctx.flush()
     torch.cuda.synchronize()
@@ -384,7 +384,7 @@ def run_svp(args, rank, ws, local):
         hctx = svp.Context(num_gpus=1, device_ids=[local], external_streams=[stream.cuda_stream],
                            arena_bytes=args.arena_gb << 30, sgemm_impl=impl)
         hvs = VPSet(hctx, specs, inputs, "host")
-        hjobs = hvs.job_list()
+        hjobs = svp.JobBatch(hvs.job_list())
         hctx.submit_batch(hjobs)
         hctx.flush()
         hst = hctx.flush_stats()

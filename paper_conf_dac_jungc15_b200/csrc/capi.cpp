@@ -6,6 +6,7 @@
 // lifting is in scheduler.cpp (Kernel Match, Dispatcher, Re-scheduler) and
 // executor.cpp (per-GPU execution and the Profiler).
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -116,6 +117,7 @@ svp_status svp_init(const svp_config* cfg, svp_ctx** out) {
     if (cfg->launch_us > 0) c->cost.launch_ns = cfg->launch_us * 1e3;
     if (cfg->arena_bytes == 0) c->cfg.arena_bytes = 2ull << 30;
     c->cost.sgemm_3xtf32 = cfg->sgemm_impl == SVP_SGEMM_3XTF32;
+    if (const char* e = getenv("SVP_COSCHEDULE")) c->coschedule = atoi(e) != 0;
 
     if (cfg->dry_run) {
         c->ngpu = cfg->num_gpus > 0 ? cfg->num_gpus : 1;

@@ -330,7 +330,10 @@ static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bo
 static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStream_t s) {
     if (ch.total_tiles == 0) return cudaSuccess;
     const uint8_t* base = d.tbl_dev;
-    auto grid_of = [&](int per_sm) { return (int)std::min<uint64_t>(ch.total_tiles, (uint64_t)d.lim.num_sms * per_sm); };
+    auto grid_of = [&](int per_sm) {
+        if (ch.co_grid > 0) per_sm = std::min(per_sm, (int)ch.co_grid);
+        return (int)std::min<uint64_t>(ch.total_tiles, (uint64_t)d.lim.num_sms * per_sm);
+    };
     switch (ch.kernel) {
         case K_VECADD:
             return launch_vecadd((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,

@@ -85,6 +85,8 @@ struct Chunk {
     uint32_t total_tiles = 0;
     int32_t nsegs = 0;
     uint64_t maps_off = 0;          // sgemm: tensor maps offset
+    int32_t co_grid = 0;            // >0: launch with co_grid CTAs per SM so the kernel
+                                    // co-resides with a tensor-core SGEMM on the same SMs
 };
 
 struct Op {
@@ -183,6 +185,7 @@ struct Ctx {
     KStats kstats[K_COUNT];
 
     Executor* exec = nullptr;        // null in dry_run
+    bool coschedule = true;          // SVP_COSCHEDULE=0 disables memory/tensor co-residency
 };
 
 // scheduler.cpp

@@ -378,12 +378,40 @@ svp_status plan_flush(Ctx* c, Flush* f) {
         // first set: ascending a; second set: descending b; ties by (group, index)
         return std::make_tuple(first ? 0 : 1, first ? a : -b, ch.group, ch.index);
     };
+    // Device-resident chunks (no copies) have nothing for Johnson's rule to balance; the
+    // engines they interleave are the tensor cores and the HBM system instead: memory-bound
+    // launches go first with a small persistent grid (co_grid CTAs/SM, no shared memory),
+    // and the tensor-core SGEMM (1 CTA/SM) is then placed on the same SMs next to them,
+    // so the HBM-bound and tensor-bound coalesced kernels run concurrently.
+    auto tensor_kernel = [&](int32_t k) {
+        return k == K_SGEMM_TF32 || (k == K_SGEMM && c->cost.sgemm_3xtf32);
+    };
+    auto device_only = [&](const Chunk& ch) { return ch.t_in == 0 && ch.t_out == 0; };
     std::stable_sort(corder.begin(), corder.end(), [&](int32_t x, int32_t y) {
         const Chunk &a = f->chunks[x], &b = f->chunks[y];
         if (a.level != b.level) return a.level < b.level;
         if (!inter) return std::tie(a.group, a.index) < std::tie(b.group, b.index);
+        const bool da = device_only(a), db = device_only(b);
+        if (da != db) return da;  // device-only chunks first; copies are on their own streams
+        if (da && c->coschedule) {
+            const bool ta = tensor_kernel(a.kernel), tb = tensor_kernel(b.kernel);
+            if (ta != tb) return !ta;
+            return std::make_tuple(-a.t_k, a.group, a.index) < std::make_tuple(-b.t_k, b.group, b.index);
+        }
         return johnson_key(x) < johnson_key(y);
     });
+    if (inter && c->coschedule) {
+        // co_grid for memory-bound device-only chunks sharing a (level, device) with a
+        // tensor-core SGEMM chunk (hist256 keeps its default grid: it needs shared memory)
+        std::map<std::pair<int32_t, int32_t>, bool> has_tensor;
+        for (const auto& ch : f->chunks)
+            if (device_only(ch) && tensor_kernel(ch.kernel)) has_tensor[{ch.level, ch.device}] = true;
+        for (auto& ch : f->chunks) {
+            if (!device_only(ch) || !has_tensor.count({ch.level, ch.device})) continue;
+            if (ch.kernel == K_VECADD || ch.kernel == K_SAXPY) ch.co_grid = 2;
+            else if (ch.kernel == K_BLACKSCHOLES) ch.co_grid = 3;
+        }
+    }
 
     // ---- ops, streams, dependencies, arena slots
     std::unordered_map<int32_t, int32_t> vp_last_op;       // per VP: last op of its previous job

@@ -176,6 +176,22 @@ def lpt_partition(classes: Sequence[int], costs: Sequence[float], G: int) -> Lis
     return list(out)
 
 
+class JobBatch:
+    """A pre-marshalled svp_job_desc array: build once, submit many times (a VP that
+    resubmits the same kernel on the same buffers pays no Python marshalling)."""
+
+    def __init__(self, jobs: Sequence[Tuple[int, int, bytes, Sequence[Buf]]]):
+        self.n = len(jobs)
+        self.arr = (svp_job_desc * max(1, self.n))()
+        for i, (vp, kid, args, bufs) in enumerate(jobs):
+            d = self.arr[i]
+            d.vp, d.kernel, d.args_bytes, d.nbufs = vp, kid, len(args), len(bufs)
+            C.memmove(d.args, args, len(args))
+            for b, (p, nb, dr, m) in enumerate(bufs):
+                d.bufs[b] = svp_buf(p, nb, dr, m)
+        self.ids = (C.c_uint64 * max(1, self.n))()
+
+
 class Context:
     """Owns one svp_ctx.  Keyword arguments mirror svp_config fields."""
 
@@ -251,7 +267,11 @@ class Context:
         _check(self._L.svp_submit(self._h, vp, kernel, ab, len(args), arr, len(bufs), C.byref(jid)))
         return jid.value
 
-    def submit_batch(self, jobs: Sequence[Tuple[int, int, bytes, Sequence[Buf]]]) -> List[int]:
+    def submit_batch(self, jobs) -> List[int]:
+        """jobs: a JobBatch, or a sequence of (vp, kernel id, args, bufs)."""
+        if isinstance(jobs, JobBatch):
+            _check(self._L.svp_submit_batch(self._h, jobs.n, jobs.arr, jobs.ids))
+            return jobs.ids
         n = len(jobs)
         arr = (svp_job_desc * max(1, n))()
         for i, (vp, kid, args, bufs) in enumerate(jobs):

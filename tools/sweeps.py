@@ -32,6 +32,7 @@ from paper_conf_dac_jungc15_b200.vpset import VPSet  # noqa: E402
 
 def flush_time(ctx, jobs, reps=5, warm=2):
     s = torch.cuda.current_stream()
+    jobs = svp.JobBatch(jobs)
     for _ in range(warm):
         ctx.submit_batch(jobs)
         ctx.flush()
