@@ -185,7 +185,8 @@ struct Ctx {
     KStats kstats[K_COUNT];
 
     Executor* exec = nullptr;        // null in dry_run
-    bool coschedule = true;          // SVP_COSCHEDULE=0 disables memory/tensor co-residency
+    bool coschedule = false;         // SVP_COSCHEDULE=1: memory-first small-grid co-residency
+                                     // (measured slower than longest-first)
 };
 
 // scheduler.cpp

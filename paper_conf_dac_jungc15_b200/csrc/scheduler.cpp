@@ -378,11 +378,13 @@ svp_status plan_flush(Ctx* c, Flush* f) {
         // first set: ascending a; second set: descending b; ties by (group, index)
         return std::make_tuple(first ? 0 : 1, first ? a : -b, ch.group, ch.index);
     };
-    // Device-resident chunks (no copies) have nothing for Johnson's rule to balance; the
-    // engines they interleave are the tensor cores and the HBM system instead: memory-bound
-    // launches go first with a small persistent grid (co_grid CTAs/SM, no shared memory),
-    // and the tensor-core SGEMM (1 CTA/SM) is then placed on the same SMs next to them,
-    // so the HBM-bound and tensor-bound coalesced kernels run concurrently.
+    // Device-resident chunks (no copies): Johnson's key degenerates to longest-first, which
+    // launches the tensor-core SGEMM (1 CTA/SM, most of shared memory) before the HBM-bound
+    // kernels; their CTAs (no shared memory) then fill the SGEMM SMs' free thread and
+    // register slots, so tensor-bound and HBM-bound coalesced kernels run concurrently
+    // (cfg5: 44.1k jobs/s vs 42.7k on one stream).  SVP_COSCHEDULE=1 instead launches the
+    // memory-bound kernels first on a small grid (co_grid CTAs/SM) -- measured slower
+    // (41.3k), kept as an option for other mixes.
     auto tensor_kernel = [&](int32_t k) {
         return k == K_SGEMM_TF32 || (k == K_SGEMM && c->cost.sgemm_3xtf32);
     };
