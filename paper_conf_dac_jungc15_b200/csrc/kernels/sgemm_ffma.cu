@@ -231,12 +231,12 @@ int encode_gemm_maps(void* mapA, void* mapB, const float* A, const float* B, int
         if (r) return r;
         return encode2d(mapB, B, (uint64_t)N, (uint64_t)K, GN, GK, CU_TENSOR_MAP_SWIZZLE_NONE);
     }
-    // tcgen05 tiles: A lands K-major (box 16 k x 128 m, SW64) directly in the MMA operand
-    // stage; B (row-major K x N) lands raw (box 256 n x 16 k, no swizzle) in a staging ring
-    // and is transposed to K-major SW64 by the kernel's converter warps.
+    // tcgen05 tiles: A lands K-major (box 16 k x 128 m, SWIZZLE_64B); B (row-major K x N,
+    // MN-major for the MMA) lands as 32-n x 16-k boxes with the 32-B-atom 128-B swizzle
+    // (UMMA layout SWIZZLE_128B_BASE32B), 8 boxes per 256-wide tile.
     int r = encode2d(mapA, A, (uint64_t)K, (uint64_t)M, kTf32BK, kTf32BM, CU_TENSOR_MAP_SWIZZLE_64B);
     if (r) return r;
-    return encode2d(mapB, B, (uint64_t)N, (uint64_t)K, kTf32BN, kTf32BK, CU_TENSOR_MAP_SWIZZLE_NONE);
+    return encode2d(mapB, B, (uint64_t)N, (uint64_t)K, 32, kTf32BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B);
 }
 
 }  // namespace svp

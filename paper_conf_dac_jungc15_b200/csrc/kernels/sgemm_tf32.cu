@@ -12,19 +12,23 @@
 //             the product error is < 3 * 2^-20 |a||b| ~ 2.9e-6 |a||b|, inside the fp32 bound
 //             1e-5 (|A||B|)_ij (R10).
 //
-// Both MMA operands are K-major with the 64-B swizzle (a kind::tf32 MMA with an MN-major
-// B operand returned zeros on B200 -- scripts/tc_probe.py, experiment E1 vs E2), so B
-// (row-major K x N, i.e. MN-major) is transposed in shared memory by converter warps.
+// Operand layouts in shared memory (both written by TMA, no transposition):
+//   A (row-major M x K = K-major): 64-B rows of 16 k, SWIZZLE_64B (8-row atoms, SBO 512).
+//   B (row-major K x N = MN-major): 32-n x 16-k blocks of 128-B rows with the 32-B-atom
+//     128-B swizzle (TMA CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B = UMMA SWIZZLE_128B_BASE32B;
+//     LBO = 2 KiB between 32-n blocks, SBO = 512 B between 4-k groups).  A tf32 MMA with an
+//     MN-major B in the plain 16-B-atom SW128 layout reads zeros on B200 (scripts/
+//     tc_probe.py E1); the 32-B-atom layout is the one the hardware accepts (E6).
+// The lo parts (SPLIT 3) are element-wise, so they keep exactly the hi layouts.
 //
 // Roles (1 CTA per SM, persistent static tile walk, 448 threads):
-//   warp 0        TMA producer: A tile 128x16 (K-major, 64-B swizzle) straight into the
-//                 operand stage; B tile 16x256 (row-major, no swizzle) into a raw staging
-//                 ring (4 deep, so B's L2 latency hides behind 3 stages of MMAs).
+//   warp 0        TMA producer: A tile 128x16 + B tile 16x256 (8 boxes) per k-block into an
+//                 operand ring (8 stages for SPLIT 1, 4 for SPLIT 3).
 //   warp 1        TMEM allocator (512 cols = 2 accumulators of 128x256 fp32) + MMA issuer:
 //                 one lane issues tcgen05.mma.cta_group::1.kind::tf32 M128 N256 K8 and
 //                 tcgen05.commit's to the stage's empty barrier / the accumulator barrier.
-//   warps 2,3,8-13 converters: B^T (K-major SW64, hi = raw bits) [+ B_lo^T, A_lo for SPLIT 3]
-//                 from the staged tiles; fence.proxy.async; arrive on the stage's conv barrier.
+//   warps 2,3,8-13 converters (SPLIT 3): A_lo, B_lo element-wise, fence.proxy.async,
+//                 arrive on the stage's conv barrier.
 //   warps 4-7     epilogue: tcgen05.ld 32x32b.x32 (warp w%4 owns TMEM lanes = tile rows
 //                 32(w%4)..+31), alpha*acc (+ beta*C), 128-bit stores; the two TMEM
 //                 accumulators let tile i's epilogue overlap tile i+1's MMAs.
@@ -38,36 +42,37 @@ namespace svp {
 namespace tc {
 
 constexpr int BM = kTf32BM, BN = kTf32BN, BK = kTf32BK;  // 128 x 256 x 16
-constexpr int kRowBytes = BK * 4;                          // 64-B K-major rows -> SWIZZLE_64B
-constexpr int kAtomBytes = 8 * kRowBytes;                  // 8-row swizzle atom (SBO)
-constexpr int kConvWarps = 8;                  // warps 2,3 and 8..13
+constexpr int kConvWarps = 8;                              // warps 2,3 and 8..13
 constexpr int kConvThreads = kConvWarps * 32;
-constexpr int kThreads = (8 + kConvWarps - 2) * 32;  // 448
-constexpr int kTileA = BM * BK * 4;   // 8 KiB
-constexpr int kTileB = BK * BN * 4;   // 16 KiB
+constexpr int kThreads = (8 + kConvWarps - 2) * 32;        // 448
+constexpr int kTileA = BM * BK * 4;                        // 8 KiB
+constexpr int kTileB = BK * BN * 4;                        // 16 KiB
+constexpr int kBBlock = BK * 128;                          // one 32-n block of B: 2 KiB
 constexpr int kTmemCols = 512;
 
 template <int SPLIT>
 struct Cfg {
-    // operand stage: A_hi (TMA) | B_hi^T | [A_lo | B_lo^T]
-    static constexpr int kOpStageBytes = SPLIT == 1 ? kTileA + kTileB : 2 * (kTileA + kTileB);
-    static constexpr int kOpStages = SPLIT == 1 ? 4 : 3;
-    static constexpr int kRawStages = 4;
-    static constexpr size_t kBarOff = (size_t)kOpStages * kOpStageBytes + (size_t)kRawStages * kTileB;
+    // stage: A_hi | B_hi [| A_lo | B_lo]
+    static constexpr int kStageBytes = (kTileA + kTileB) * (SPLIT == 1 ? 1 : 2);
+    static constexpr int kStages = SPLIT == 1 ? 8 : 4;
+    static constexpr size_t kBarOff = (size_t)kStages * kStageBytes;
     static constexpr size_t kSmem = 1024 + kBarOff + 256;
 };
 
-__device__ __forceinline__ uint64_t make_desc_kmajor(uint32_t saddr) {
-    // SM100 smem matrix descriptor: start>>4 [0,14), LBO>>4 [16,30) (=1, unused for
-    // swizzled K-major), SBO>>4 [32,46) (512 B between 8-row groups of 64-B rows),
-    // version 1 [46,48), layout SWIZZLE_64B (4) [61,64)
-    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)1 << 16) | ((uint64_t)(kAtomBytes >> 4) << 32) |
-           ((uint64_t)1 << 46) | ((uint64_t)4 << 61);
+// SM100 shared-memory matrix descriptor: start>>4 [0,14), LBO>>4 [16,30), SBO>>4 [32,46),
+// version 1 [46,48), base offset 0, layout [61,64)
+__device__ __forceinline__ uint64_t make_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo, uint32_t layout) {
+    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+           ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | ((uint64_t)1 << 46) | ((uint64_t)layout << 61);
 }
+// A: K-major, SWIZZLE_64B (4): LBO unused (1), SBO 512 B
+__device__ __forceinline__ uint64_t desc_a(uint32_t saddr) { return make_desc(saddr, 16, 8 * BK * 4, 4); }
+// B: MN-major, SWIZZLE_128B_BASE32B (1): LBO = 32-n block stride, SBO = 4-k group stride
+__device__ __forceinline__ uint64_t desc_b(uint32_t saddr) { return make_desc(saddr, kBBlock, 512, 1); }
 
 // kind::tf32 instruction descriptor: D f32 [4,6)=1, A tf32 [7,10)=2, B tf32 [10,13)=2,
-// A and B K-major (bits 15, 16 = 0), N>>3 at [17,23), M>>4 at [24,29)
-constexpr uint32_t kIdesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) |
+// A K-major (bit 15 = 0), B MN-major (bit 16 = 1), N>>3 at [17,23), M>>4 at [24,29)
+constexpr uint32_t kIdesc = (1u << 4) | (2u << 7) | (2u << 10) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
                             ((uint32_t)(BM >> 4) << 24);
 
 __device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accum) {
@@ -111,6 +116,9 @@ __device__ __forceinline__ int find_tile_owner(const GemmDesc* __restrict__ d, i
 }
 
 __device__ __forceinline__ float lo_part(float x) { return x - __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
+__device__ __forceinline__ float4 lo_part4(float4 x) {
+    return make_float4(lo_part(x.x), lo_part(x.y), lo_part(x.z), lo_part(x.w));
+}
 
 }  // namespace tc
 
@@ -119,32 +127,25 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
     k_sgemm_tc(const GemmDesc* __restrict__ descs, int n, const uint8_t* __restrict__ maps, uint32_t total) {
     using namespace tc;
     using C = Cfg<SPLIT>;
-    constexpr int OS = C::kOpStages, RS = C::kRawStages, OB = C::kOpStageBytes;
+    constexpr int ST = C::kStages, SB = C::kStageBytes;
     extern __shared__ uint8_t smem_raw[];
-    // align to 1024 B (SW128 atoms) by offsetting smem_raw itself, so the compiler keeps
+    // align to 1024 B (swizzle atoms) by offsetting smem_raw itself, so the compiler keeps
     // the shared address space and emits LDS/STS (not generic LD/ST) for the converters
     uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-    uint8_t* raw_base = smem + (size_t)OS * OB;
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::kBarOff);
-    uint64_t* a_full = bars;                 // [OS] TMA A landed
-    uint64_t* op_empty = bars + OS;          // [OS] MMAs done with the operand stage
-    uint64_t* conv_done = bars + 2 * OS;     // [OS] converters wrote the stage
-    uint64_t* raw_full = bars + 3 * OS;      // [RS] TMA B landed in the staging ring
-    uint64_t* raw_empty = raw_full + RS;     // [RS] converters done reading raw B
-    uint64_t* acc_full = raw_empty + RS;     // [2]
-    uint64_t* acc_empty = acc_full + 2;      // [2]
+    uint64_t* full = bars;               // [ST] TMA A + B landed
+    uint64_t* empty = bars + ST;         // [ST] MMAs done with the stage
+    uint64_t* conv = bars + 2 * ST;      // [ST] lo parts written (SPLIT 3)
+    uint64_t* acc_full = bars + 3 * ST;  // [2]
+    uint64_t* acc_empty = acc_full + 2;  // [2]
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_empty + 2);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
-        for (int s = 0; s < OS; ++s) {
-            mbar_init(&a_full[s], 1);
-            mbar_init(&op_empty[s], 1);
-            mbar_init(&conv_done[s], kConvThreads / 32);
-        }
-        for (int r = 0; r < RS; ++r) {
-            mbar_init(&raw_full[r], 1);
-            mbar_init(&raw_empty[r], kConvThreads / 32);
+        for (int s = 0; s < ST; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 1);
+            mbar_init(&conv[s], kConvWarps);
         }
         for (int a = 0; a < 2; ++a) {
             mbar_init(&acc_full[a], 1);
@@ -163,8 +164,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
-    auto op_stage = [&](int s) { return smem + (size_t)s * OB; };
-    auto raw_stage = [&](int r) { return raw_base + (size_t)r * kTileB; };
+    auto stage = [&](int s) { return smem + (size_t)s * SB; };
 
     if (warp == 0) {
         // ------------------------------------------------------------ TMA producer
@@ -185,14 +185,15 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                 const int tm = lt / g.tiles_n, tn = lt % g.tiles_n;
                 const int KB = (g.K + BK - 1) / BK;
                 for (int kb = 0; kb < KB; ++kb, ++it) {
-                    const int s = it % OS, r = it % RS;
-                    const uint32_t ph = (it / OS) & 1, rph = (it / RS) & 1;
-                    mbar_wait(&raw_empty[r], rph ^ 1);
-                    mbar_expect_tx(&raw_full[r], kTileB);
-                    tma_load_2d(raw_stage(r), mB, tn * BN, kb * BK, &raw_full[r]);
-                    mbar_wait(&op_empty[s], ph ^ 1);
-                    mbar_expect_tx(&a_full[s], kTileA);
-                    tma_load_2d(op_stage(s), mA, kb * BK, tm * BM, &a_full[s]);
+                    const int s = it % ST;
+                    const uint32_t ph = (it / ST) & 1;
+                    mbar_wait(&empty[s], ph ^ 1);
+                    uint8_t* sp = stage(s);
+                    mbar_expect_tx(&full[s], kTileA + kTileB);
+                    tma_load_2d(sp, mA, kb * BK, tm * BM, &full[s]);
+#pragma unroll
+                    for (int j = 0; j < BN / 32; ++j)
+                        tma_load_2d(sp + kTileA + j * kBBlock, mB, tn * BN + j * 32, kb * BK, &full[s]);
                 }
             }
         }
@@ -208,32 +209,30 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
             tc_fence_after();
             const uint32_t tmem_d = tmem_base + (uint32_t)(a * BN);
             for (int kb = 0; kb < KB; ++kb, ++it) {
-                const int s = it % OS;
-                const uint32_t ph = (it / OS) & 1;
-                mbar_wait(&a_full[s], ph);
-                mbar_wait(&conv_done[s], ph);
+                const int s = it % ST;
+                const uint32_t ph = (it / ST) & 1;
+                mbar_wait(&full[s], ph);
+                if (SPLIT == 3) mbar_wait(&conv[s], ph);
                 tc_fence_after();
                 if (lane == 0) {
-                    const uint32_t s_ah = smem_u32(op_stage(s));
+                    const uint32_t s_ah = smem_u32(stage(s));
                     const uint32_t s_bh = s_ah + kTileA;
                     const uint32_t s_al = s_bh + kTileB;
                     const uint32_t s_bl = s_al + kTileA;
 #pragma unroll
                     for (int kk = 0; kk < BK / 8; ++kk) {
-                        const uint64_t ah = make_desc_kmajor(s_ah + kk * 32);
-                        const uint64_t bh = make_desc_kmajor(s_bh + kk * 32);
+                        const uint64_t ah = desc_a(s_ah + kk * 32);   // +8 k in a 64-B row
+                        const uint64_t bh = desc_b(s_bh + kk * 1024); // +8 k rows of 128 B
                         const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
                         if (SPLIT == 3) {
-                            const uint64_t al = make_desc_kmajor(s_al + kk * 32);
-                            const uint64_t bl = make_desc_kmajor(s_bl + kk * 32);
-                            mma_tf32(tmem_d, ah, bl, acc0);
-                            mma_tf32(tmem_d, al, bh, 1u);
+                            mma_tf32(tmem_d, ah, desc_b(s_bl + kk * 1024), acc0);
+                            mma_tf32(tmem_d, desc_a(s_al + kk * 32), bh, 1u);
                             mma_tf32(tmem_d, ah, bh, 1u);
                         } else {
                             mma_tf32(tmem_d, ah, bh, acc0);
                         }
                     }
-                    mma_commit(&op_empty[s]);
+                    mma_commit(&empty[s]);
                     if (kb == KB - 1) mma_commit(&acc_full[a]);
                 }
                 __syncwarp();
@@ -242,61 +241,26 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
             __syncwarp();
         }
     } else if (warp < 4 || warp >= 8) {
-        // ------------------------------------------------------------ converters
-        const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;  // 0..kConvThreads-1
-        uint32_t it = 0;
-        for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
-            const int v = find_tile_owner(descs, n, t);
-            const int KB = (descs[v].K + BK - 1) / BK;
-            for (int kb = 0; kb < KB; ++kb, ++it) {
-                const int s = it % OS, r = it % RS;
-                const uint32_t ph = (it / OS) & 1, rph = (it / RS) & 1;
-                mbar_wait(&op_empty[s], ph ^ 1);  // previous MMAs on this stage are done
-                mbar_wait(&raw_full[r], rph);
-                const float* rawB = reinterpret_cast<const float*>(raw_stage(r));  // [k][n], row 1 KiB
-                uint8_t* bh = op_stage(s) + kTileA;
-                uint8_t* bl = bh + kTileB + kTileA;
-                // (n, 4-k chunk) pairs: a warp covers 32 consecutive n of one chunk ->
-                // conflict-free reads (one 128-B row segment per k) and 64-B-swizzled 16-B
-                // writes (8 lanes fill 8 distinct 16-B bank slots)
-#pragma unroll 4
-                for (int p = ct; p < BN * (BK / 4); p += kConvThreads) {
-                    const int nn = p & (BN - 1), c = p / BN;
-                    float4 x;
-                    x.x = rawB[(4 * c + 0) * BN + nn];
-                    x.y = rawB[(4 * c + 1) * BN + nn];
-                    x.z = rawB[(4 * c + 2) * BN + nn];
-                    x.w = rawB[(4 * c + 3) * BN + nn];
-                    const int off = nn * kRowBytes + ((c ^ ((nn >> 1) & 3)) << 4);
-                    *reinterpret_cast<float4*>(bh + off) = x;
-                    if (SPLIT == 3) {
-                        float4 y;
-                        y.x = lo_part(x.x);
-                        y.y = lo_part(x.y);
-                        y.z = lo_part(x.z);
-                        y.w = lo_part(x.w);
-                        *reinterpret_cast<float4*>(bl + off) = y;
-                    }
+        // ------------------------------------------------------------ lo converters
+        if (SPLIT == 3) {
+            const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;  // 0..kConvThreads-1
+            uint32_t it = 0;
+            for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+                const int v = find_tile_owner(descs, n, t);
+                const int KB = (descs[v].K + BK - 1) / BK;
+                for (int kb = 0; kb < KB; ++kb, ++it) {
+                    const int s = it % ST;
+                    const uint32_t ph = (it / ST) & 1;
+                    mbar_wait(&full[s], ph);
+                    const float4* hi = reinterpret_cast<const float4*>(stage(s));
+                    float4* lo = reinterpret_cast<float4*>(stage(s) + kTileA + kTileB);
+                    constexpr int NV = (kTileA + kTileB) / 16;  // 1536 float4: A then B, same order
+#pragma unroll
+                    for (int i = ct; i < NV; i += kConvThreads) lo[i] = lo_part4(hi[i]);
+                    fence_proxy_async();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&conv[s]);
                 }
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&raw_empty[r]);
-                if (SPLIT == 3) {
-                    mbar_wait(&a_full[s], ph);
-                    const float4* ah = reinterpret_cast<const float4*>(op_stage(s));
-                    float4* al = reinterpret_cast<float4*>(op_stage(s) + kTileA + kTileB);
-#pragma unroll 4
-                    for (int i = ct; i < kTileA / 16; i += kConvThreads) {
-                        float4 x = ah[i];
-                        x.x = lo_part(x.x);
-                        x.y = lo_part(x.y);
-                        x.z = lo_part(x.z);
-                        x.w = lo_part(x.w);
-                        al[i] = x;  // same swizzled position as the hi element
-                    }
-                }
-                fence_proxy_async();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&conv_done[s]);
             }
         }
     } else {

@@ -112,6 +112,27 @@ for nk, R in ((1, R1), (4, R4)):
         d += [desc(kk * 256, sboA, 128, layout=0), desc(16384 + kk * 256, sboB, 128, layout=0)]
     report(f"E4' (lbo/sbo swapped) nk={nk}", *run(img, d, idesc("tf32", 0, 0), nk, 0), R)
 
+# E6: tf32 B MN-major with the 32-B-atom 128-B swizzle (LayoutType SWIZZLE_128B_BASE32B = 1)
+def put_mnmajor_sw128_32b(img, base, B):
+    K, N = B.shape
+    raw = B.view(np.uint8).reshape(K, N * 4)
+    for j in range(N // 32):
+        for k in range(K):
+            for g in range(4):
+                dst = base + j * (K * 128) + k * 128 + ((g ^ (k % 4)) * 32)
+                img[dst:dst + 32] = raw[k, j * 128 + g * 32: j * 128 + (g + 1) * 32]
+
+
+img = np.zeros(65536, np.uint8)
+put_kmajor_sw128(img, 0, A, 4)
+put_mnmajor_sw128_32b(img, 16384, B)
+for (lbo, sbo) in ((4096, 512), (512, 4096), (4096, 1024)):
+    for nk, R in ((1, R1), (4, R4)):
+        d = []
+        for kk in range(nk):
+            d += [desc(kk * 32, 16, 1024), desc(16384 + kk * 1024, lbo, sbo, layout=1)]
+        report(f"E6 tf32 A-K B-MN SW128_BASE32B lbo={lbo} sbo={sbo} nk={nk}", *run(img, d, idesc("tf32", 0, 1), nk, 0), R)
+
 # E5: bf16, both K-major SW128
 Ab = torch.from_numpy(g.integers(-3, 4, (128, 64)).astype(np.float32)).to(torch.bfloat16)
 Bb = torch.from_numpy(g.integers(-3, 4, (64, 256)).astype(np.float32)).to(torch.bfloat16)
