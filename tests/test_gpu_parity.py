@@ -196,3 +196,25 @@ def test_repeated_flushes_reuse_tables(small):
             check_job(s, inp, vs.output(i))
     assert uploads[0] == 1 and uploads[1] == 0 and uploads[2] == 0
     ctx.close()
+
+
+@pytest.mark.parametrize("residency", ["device", "host"])
+def test_two_logical_gpus_one_process(small, residency):
+    """Single-process multi-GPU path (one issuing thread per GPU, Job Dispatcher sharding)
+    on one physical B200: two logical devices mapped to CUDA ordinal 0."""
+    specs, inputs = small
+    ctx = svp.Context(num_gpus=2, device_ids=[0, 0], profile_level=1)
+    vs = VPSet(ctx, specs, inputs, residency, device_ordinals=[0, 0])
+    vs.submit()
+    ctx.flush()
+    ops = ctx.plan()
+    devs = {op["device"] for op in ops}
+    assert devs == {0, 1}
+    owner = {}
+    for op in ops:
+        for v in op["vps"]:
+            assert owner.setdefault(v, op["device"]) == op["device"]
+    for i, (s, inp) in enumerate(zip(specs, inputs)):
+        check_job(s, inp, vs.output(i))
+    assert vs.guards_intact()
+    ctx.close()
