@@ -163,9 +163,27 @@ svp_status svp_submit_batch(svp_ctx* ctx, int32_t n, const svp_job_desc* jobs, u
 /* Drain every job submitted before the call: Kernel Match -> Job Dispatcher ->
  * Re-scheduler -> per-GPU execution (coalesced launches over device segment tables,
  * interleaved H2D/kernel/D2H streams) -> Profiler; blocks until every output is in
- * the caller's buffers.  Not re-entrant (SVP_E_STATE if called concurrently).
+ * the caller's buffers.  Concurrent calls (other threads, the dispatcher) serialize.
+ * On an error the flushed jobs are dropped and reported failed to svp_wait.
  * Errors: SVP_E_CUDA (sticky), SVP_E_TIMEOUT, SVP_E_NOMEM, SVP_E_STATE. */
 svp_status svp_flush(svp_ctx* ctx);
+
+/* ------------------------------------------------------------------ VP Control */
+/* Block the calling VP until job `job` (an id returned by svp_submit*) has run and its
+ * outputs are in place -- the synchronous-call path of PAPER.md L276-286 / Fig 4(b):
+ * the VP is stopped while other VPs' jobs keep the GPU busy, and resumed when its job
+ * completes.  Somebody must flush (the caller from another thread, or the dispatcher).
+ * timeout_ms <= 0 waits forever.  Returns SVP_OK, the failing flush's status for a job
+ * that was dropped, SVP_E_TIMEOUT, SVP_E_STATE (context errored first) or SVP_E_INVAL
+ * (unknown id). */
+svp_status svp_wait(svp_ctx* ctx, uint64_t job, int32_t timeout_ms);
+
+/* Continuous dispatch (the paper's continuously fed Job Queue): a
+ * background thread flushes whenever jobs are queued, after letting more VPs join for up
+ * to window_us (or until max_jobs are queued, 0 = no cap) -- so concurrent VPs' identical
+ * synchronous calls still coalesce.  svp_stop_dispatcher drains the queue and joins. */
+svp_status svp_start_dispatcher(svp_ctx* ctx, int32_t window_us, int32_t max_jobs);
+svp_status svp_stop_dispatcher(svp_ctx* ctx);
 
 /* ------------------------------------------------------------------ Job Dispatcher */
 /* The GPU (index into the context's device list, 0..num_gpus-1) that runs VP `vp`.

@@ -78,6 +78,8 @@ static svp_status check_ctx(svp_ctx* h) {
 
 extern "C" {
 
+static void stop_dispatcher(Ctx* c);
+
 const char* svp_last_error(void) { return g_last_error.c_str(); }
 int32_t svp_abi_version(void) { return SVP_ABI_VERSION; }
 
@@ -149,6 +151,7 @@ svp_status svp_finalize(svp_ctx* h) {
         return SVP_E_INVAL;
     }
     Ctx* c = reinterpret_cast<Ctx*>(h);
+    stop_dispatcher(c);
     if (c->exec) executor_destroy(c->exec);
     delete c;
     return SVP_OK;
@@ -198,12 +201,15 @@ static svp_status submit_many(Ctx* c, int32_t n, const svp_job_desc* jd, const s
         svp_status st = validate_and_fill(c, &j);
         if (st) return st;
     }
-    std::lock_guard<std::mutex> lk(c->qmu);
-    for (int i = 0; i < n; ++i) {
-        jobs[i].id = c->next_job_id++;
-        if (ids) ids[i] = jobs[i].id;
-        c->queue.push_back(jobs[i]);
+    {
+        std::lock_guard<std::mutex> lk(c->qmu);
+        for (int i = 0; i < n; ++i) {
+            jobs[i].id = c->next_job_id++;
+            if (ids) ids[i] = jobs[i].id;
+            c->queue.push_back(jobs[i]);
+        }
     }
+    c->q_cv.notify_one();
     return SVP_OK;
 }
 
@@ -241,63 +247,179 @@ svp_status svp_submit_batch(svp_ctx* h, int32_t n, const svp_job_desc* jobs, uin
     SVP_TRY_END
 }
 
+// One flush of everything queued so far (serialized by flush_mu).  Marks every job id
+// below the snapshot's next id as completed (or failed with the flush's status) and
+// wakes svp_wait callers.
+static svp_status do_flush(Ctx* c) {
+    std::lock_guard<std::mutex> flk(c->flush_mu);
+    if (c->sticky != SVP_OK) {
+        set_error("context is sticky-errored: " + c->sticky_msg);
+        return SVP_E_STATE;
+    }
+    auto t0 = std::chrono::steady_clock::now();
+    Flush f;
+    uint64_t upto = 0;
+    {
+        std::lock_guard<std::mutex> lk(c->qmu);
+        f.jobs.swap(c->queue);
+        upto = c->next_job_id - 1;
+    }
+    memset(&c->fstats, 0, sizeof(c->fstats));
+    svp_status st = plan_flush(c, &f);
+    auto t1 = std::chrono::steady_clock::now();
+    if (st == SVP_OK) {
+        double makespan = 0, serial = 0;
+        simulate(c, &f, &makespan, &serial);
+        c->fstats.sim_makespan_ns = makespan;
+        c->fstats.sim_serial_ns = serial;
+        c->fstats.host_plan_ns = std::chrono::duration<double, std::nano>(t1 - t0).count();
+        if (c->exec && !f.ops.empty()) {
+            st = executor_run(c->exec, &f);
+            if (st == SVP_E_CUDA || st == SVP_E_TIMEOUT) {
+                c->sticky = st;
+                c->sticky_msg = executor_error(c->exec);
+                set_error(c->sticky_msg);
+            } else if (st) {
+                set_error(executor_error(c->exec));
+            }
+        }
+        auto t2 = std::chrono::steady_clock::now();
+        c->fstats.host_total_ns = std::chrono::duration<double, std::nano>(t2 - t0).count();
+        c->fstats.jobs = f.jobs.size();
+        c->fstats.groups = f.groups.size();
+        c->fstats.chunks = f.chunks.size();
+        c->fstats.levels = f.levels;
+        uint64_t launches = 0;
+        for (auto& op : f.ops) {
+            if (op.kind == SVP_OP_KERNEL) ++launches;
+            if (op.kind == SVP_OP_H2D) c->fstats.h2d_bytes += op.bytes;
+            if (op.kind == SVP_OP_D2H) c->fstats.d2h_bytes += op.bytes;
+        }
+        c->fstats.launches = launches;
+    }
+    c->last = std::move(f);
+    {
+        std::lock_guard<std::mutex> lk(c->done_mu);
+        if (st != SVP_OK && upto > c->completed_upto) c->failed.emplace_back(upto, st);
+        if (upto > c->completed_upto) c->completed_upto = upto;
+    }
+    c->done_cv.notify_all();
+    return st;
+}
+
 svp_status svp_flush(svp_ctx* h) {
     SVP_TRY_BEGIN
     svp_status st = check_ctx(h);
     if (st) return st;
-    Ctx* c = reinterpret_cast<Ctx*>(h);
-    int expected = 0;
-    if (!c->flushing.compare_exchange_strong(expected, 1)) {
-        set_error("svp_flush: already flushing (not re-entrant)");
-        return SVP_E_STATE;
+    return do_flush(reinterpret_cast<Ctx*>(h));
+    SVP_TRY_END
+}
+
+svp_status svp_wait(svp_ctx* h, uint64_t job, int32_t timeout_ms) {
+    SVP_TRY_BEGIN
+    if (!h) {
+        set_error("null context");
+        return SVP_E_INVAL;
     }
-    struct Guard {
-        Ctx* c;
-        ~Guard() { c->flushing.store(0); }
-    } guard{c};
-    auto t0 = std::chrono::steady_clock::now();
-    Flush f;
+    Ctx* c = reinterpret_cast<Ctx*>(h);
     {
         std::lock_guard<std::mutex> lk(c->qmu);
-        f.jobs.swap(c->queue);
-    }
-    memset(&c->fstats, 0, sizeof(c->fstats));
-    st = plan_flush(c, &f);
-    auto t1 = std::chrono::steady_clock::now();
-    if (st) {
-        c->last = std::move(f);
-        return st;
-    }
-    double makespan = 0, serial = 0;
-    simulate(c, &f, &makespan, &serial);
-    c->fstats.sim_makespan_ns = makespan;
-    c->fstats.sim_serial_ns = serial;
-    c->fstats.host_plan_ns = std::chrono::duration<double, std::nano>(t1 - t0).count();
-    if (c->exec && !f.ops.empty()) {
-        st = executor_run(c->exec, &f);
-        if (st == SVP_E_CUDA || st == SVP_E_TIMEOUT) {
-            c->sticky = st;
-            c->sticky_msg = executor_error(c->exec);
-            set_error(c->sticky_msg);
-        } else if (st) {
-            set_error(executor_error(c->exec));
+        if (job == 0 || job >= c->next_job_id) {
+            set_error("svp_wait: unknown job id");
+            return SVP_E_INVAL;
         }
     }
-    auto t2 = std::chrono::steady_clock::now();
-    c->fstats.host_total_ns = std::chrono::duration<double, std::nano>(t2 - t0).count();
-    c->fstats.jobs = f.jobs.size();
-    c->fstats.groups = f.groups.size();
-    c->fstats.chunks = f.chunks.size();
-    c->fstats.levels = f.levels;
-    uint64_t launches = 0;
-    for (auto& op : f.ops) {
-        if (op.kind == SVP_OP_KERNEL) ++launches;
-        if (op.kind == SVP_OP_H2D) c->fstats.h2d_bytes += op.bytes;
-        if (op.kind == SVP_OP_D2H) c->fstats.d2h_bytes += op.bytes;
+    std::unique_lock<std::mutex> lk(c->done_mu);
+    auto done = [&] { return c->completed_upto >= job || c->sticky != SVP_OK; };
+    if (timeout_ms > 0) {
+        if (!c->done_cv.wait_for(lk, std::chrono::milliseconds(timeout_ms), done)) {
+            set_error("svp_wait: timed out");
+            return SVP_E_TIMEOUT;
+        }
+    } else {
+        c->done_cv.wait(lk, done);
     }
-    c->fstats.launches = launches;
-    c->last = std::move(f);
-    return st;
+    if (c->completed_upto < job) {
+        set_error("svp_wait: context errored before the job ran: " + c->sticky_msg);
+        return SVP_E_STATE;
+    }
+    // the first failed flush whose range covers the job decides its status
+    uint64_t lo = 0;
+    for (const auto& fr : c->failed) {
+        if (job > lo && job <= fr.first) {
+            set_error("svp_wait: the flush that ran this job failed");
+            return fr.second;
+        }
+        lo = fr.first;
+    }
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+static void dispatcher_loop(Ctx* c) {
+    for (;;) {
+        {
+            std::unique_lock<std::mutex> lk(c->qmu);
+            c->q_cv.wait(lk, [&] { return c->disp_stop || !c->queue.empty(); });
+            if (c->queue.empty() && c->disp_stop) return;
+            // batching window: let more VPs join this flush (coalescing width)
+            if (c->disp_window_us > 0 && !c->disp_stop) {
+                auto deadline = std::chrono::steady_clock::now() + std::chrono::microseconds(c->disp_window_us);
+                c->q_cv.wait_until(lk, deadline, [&] {
+                    return c->disp_stop || (c->disp_max_jobs > 0 && (int64_t)c->queue.size() >= c->disp_max_jobs);
+                });
+            }
+        }
+        if (do_flush(c) == SVP_E_STATE && c->sticky != SVP_OK) {
+            c->done_cv.notify_all();
+            return;
+        }
+    }
+}
+
+svp_status svp_start_dispatcher(svp_ctx* h, int32_t window_us, int32_t max_jobs) {
+    SVP_TRY_BEGIN
+    svp_status st = check_ctx(h);
+    if (st) return st;
+    if (window_us < 0 || max_jobs < 0) {
+        set_error("svp_start_dispatcher: negative window/max_jobs");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    std::lock_guard<std::mutex> lk(c->qmu);
+    if (c->disp_running) {
+        set_error("svp_start_dispatcher: already running");
+        return SVP_E_STATE;
+    }
+    c->disp_window_us = window_us;
+    c->disp_max_jobs = max_jobs;
+    c->disp_stop = false;
+    c->disp_running = true;
+    c->disp = std::thread(dispatcher_loop, c);
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+static void stop_dispatcher(Ctx* c) {
+    {
+        std::lock_guard<std::mutex> lk(c->qmu);
+        if (!c->disp_running) return;
+        c->disp_stop = true;
+    }
+    c->q_cv.notify_all();
+    c->disp.join();
+    std::lock_guard<std::mutex> lk(c->qmu);
+    c->disp_running = false;
+}
+
+svp_status svp_stop_dispatcher(svp_ctx* h) {
+    SVP_TRY_BEGIN
+    if (!h) {
+        set_error("null context");
+        return SVP_E_INVAL;
+    }
+    stop_dispatcher(reinterpret_cast<Ctx*>(h));
+    return SVP_OK;
     SVP_TRY_END
 }
 

@@ -168,7 +168,20 @@ struct Ctx {
     std::vector<double> dev_load;
 
     // state
-    std::atomic<int> flushing{0};
+    std::mutex flush_mu;             // serializes flushes (user calls and the dispatcher)
+    // job completion (VP Control: svp_wait blocks a VP until its job is done)
+    std::mutex done_mu;
+    std::condition_variable done_cv;
+    uint64_t completed_upto = 0;     // every job id <= completed_upto has been flushed
+    std::vector<std::pair<uint64_t, int32_t>> failed;  // (last id of a failed flush, status), ascending
+    uint64_t failed_floor = 0;       // ids <= failed_floor that are not in `failed` succeeded
+    // continuous dispatcher (svp_start_dispatcher)
+    std::condition_variable q_cv;    // with qmu: a job was queued / stop requested
+    std::thread disp;
+    bool disp_running = false;
+    bool disp_stop = false;
+    int64_t disp_window_us = 0;
+    int32_t disp_max_jobs = 0;
     int32_t sticky = 0;              // SVP_OK or first fatal status
     std::string sticky_msg;
     bool registered[K_COUNT] = {};

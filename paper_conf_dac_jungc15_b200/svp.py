@@ -30,7 +30,8 @@ MAX_BUFS, MAX_ARGS = 5, 64
 EXPORTS = ("svp_config_default", "svp_init", "svp_finalize", "svp_last_error", "svp_abi_version",
            "svp_register_kernel", "svp_submit", "svp_submit_batch", "svp_flush", "svp_vp_device",
            "svp_assign_vps", "svp_lpt_partition", "svp_profile", "svp_reset_profile", "svp_kernel_stats_get",
-           "svp_flush_stats_get", "svp_plan_size", "svp_plan_get")
+           "svp_flush_stats_get", "svp_plan_size", "svp_plan_get", "svp_wait", "svp_start_dispatcher",
+           "svp_stop_dispatcher")
 
 
 class svp_config(C.Structure):
@@ -125,6 +126,9 @@ def load(build_if_stale: bool = True):
         L.svp_flush_stats_get.argtypes = [vp, P(svp_flush_stats)]
         L.svp_plan_size.argtypes = [vp, P(C.c_int32)]
         L.svp_plan_get.argtypes = [vp, C.c_int32, P(svp_plan_op), P(C.c_int32), C.c_int32]
+        L.svp_wait.argtypes = [vp, C.c_uint64, C.c_int32]
+        L.svp_start_dispatcher.argtypes = [vp, C.c_int32, C.c_int32]
+        L.svp_stop_dispatcher.argtypes = [vp]
         for name in EXPORTS:
             f = getattr(L, name)
             if name not in ("svp_config_default", "svp_last_error", "svp_abi_version"):
@@ -286,6 +290,16 @@ class Context:
 
     def flush(self):
         _check(self._L.svp_flush(self._h))
+
+    def wait(self, job: int, timeout_ms: int = 0):
+        """VP Control: block until `job` has run (svp_wait).  Releases the GIL."""
+        _check(self._L.svp_wait(self._h, job, timeout_ms))
+
+    def start_dispatcher(self, window_us: int = 50, max_jobs: int = 0):
+        _check(self._L.svp_start_dispatcher(self._h, window_us, max_jobs))
+
+    def stop_dispatcher(self):
+        _check(self._L.svp_stop_dispatcher(self._h))
 
     def vp_device(self, vp: int) -> int:
         d = C.c_int32()
