@@ -67,6 +67,8 @@ def lib():
             L.oracle_sgemm.argtypes = [i32, i32, i32, f32, _F32P, _F32P, f32, _F32P]
             L.oracle_sgemm_element.argtypes = [i32, i32, i32, f32, _F32P, _F32P, f32, f32, i32, i32]
             L.oracle_sgemm_element.restype = f32
+            L.oracle_dgemm.argtypes = [i32, i32, i32, f64, _F64P, _F64P, f64, _F64P]
+            L.oracle_dgemm.restype = None
             for f in ("oracle_vecadd", "oracle_saxpy", "oracle_hist256", "oracle_blackscholes",
                       "oracle_blackscholes_f64", "oracle_sgemm"):
                 getattr(L, f).restype = None
@@ -137,6 +139,18 @@ def sgemm_element(A, B, i: int, j: int, alpha: float = 1.0, beta: float = 0.0, c
                                             ctypes.c_float(beta), ctypes.c_float(c_old), i, j))
 
 
+def dgemm(A: np.ndarray, B: np.ndarray, C: np.ndarray | None = None, alpha: float = 1.0,
+          beta: float = 0.0) -> np.ndarray:
+    A = np.ascontiguousarray(A, dtype=np.float64)
+    B = np.ascontiguousarray(B, dtype=np.float64)
+    M, K = A.shape
+    K2, N = B.shape
+    assert K == K2
+    out = np.zeros((M, N), np.float64) if C is None else np.ascontiguousarray(C, dtype=np.float64).copy()
+    lib().oracle_dgemm(M, N, K, alpha, _p(A, _F64P), _p(B, _F64P), beta, _p(out, _F64P))
+    return out
+
+
 # ----------------------------------------------------------------- job-level runner
 def run_job(spec, inputs: Dict[str, np.ndarray]) -> Dict[str, np.ndarray]:
     """One VP job, plain definition; returns the job's outputs by name."""
@@ -150,6 +164,9 @@ def run_job(spec, inputs: Dict[str, np.ndarray]) -> Dict[str, np.ndarray]:
     if k == "blackscholes":
         c, p = blackscholes(inputs["S"], inputs["X"], inputs["T"], spec.R, spec.V)
         return {"call": c, "put": p}
+    if k == "dgemm":
+        return {"C": dgemm(inputs["A"], inputs["B"], inputs.get("C") if spec.beta != 0 else None,
+                           spec.alpha, spec.beta)}
     if k in ("sgemm", "sgemm_tf32"):  # same definition; the TF32 kernel has its own tolerance
         return {"C": sgemm(inputs["A"], inputs["B"], inputs.get("C") if spec.beta != 0 else None,
                            spec.alpha, spec.beta)}

@@ -137,3 +137,28 @@ float oracle_sgemm_element(int32_t M, int32_t N, int32_t K, float alpha, const f
     if (beta != 0.0f) r += (double)beta * (double)c_old;
     return (float)r;
 }
+
+/* DGEMM -- the paper's own matmul guest at its stated precision (Table 1: "multiplies
+ * 300 times two 320 x 320 matrices of double-precision numbers"):
+ *   C = alpha * A B + beta * C, fp64, row-major.  Plain i-k-j loop with an extended-
+ * precision (x87 long double, 64-bit mantissa) accumulator per output element, ascending
+ * k, then alpha*acc + beta*C in long double and one rounding to double. */
+void oracle_dgemm(int32_t M, int32_t N, int32_t K, double alpha, const double* A, const double* B,
+                  double beta, double* C) {
+    long double* acc = (long double*)malloc(sizeof(long double) * (size_t)(N > 0 ? N : 1));
+    for (int32_t i = 0; i < M; ++i) {
+        for (int32_t j = 0; j < N; ++j) acc[j] = 0.0L;
+        for (int32_t k = 0; k < K; ++k) {
+            long double a = (long double)A[(size_t)i * K + k];
+            const double* brow = B + (size_t)k * N;
+            for (int32_t j = 0; j < N; ++j) acc[j] += a * (long double)brow[j];
+        }
+        double* crow = C + (size_t)i * N;
+        for (int32_t j = 0; j < N; ++j) {
+            long double r = (long double)alpha * acc[j];
+            if (beta != 0.0) r += (long double)beta * (long double)crow[j];
+            crow[j] = (double)r;
+        }
+    }
+    free(acc);
+}

@@ -184,3 +184,29 @@ def test_run_jobs_independent_per_vp():
         single = oracle.run_job(s, inp)
         for k in single:
             assert np.array_equal(single[k], r[k])
+
+
+# ------------------------------------------------------------------ DGEMM (Table 1 guest)
+def test_dgemm_integer_exact_and_hand_case():
+    spec = W.JobSpec(0, "dgemm", M=37, N=29, K=65, int_inputs=True)
+    inp = W.make_inputs(spec, seed=9)
+    C = oracle.dgemm(inp["A"], inp["B"])
+    assert np.array_equal(C.astype(np.int64), inp["A"].astype(np.int64) @ inp["B"].astype(np.int64))
+    A = np.array([[1, 2, 3], [4, 5, 6]], np.float64)
+    B = np.array([[7, 8], [9, 10], [11, 12]], np.float64)
+    assert oracle.dgemm(A, B).tolist() == [[58, 64], [139, 154]]
+    Cin = np.array([[1, -1], [2, 0.5]])
+    assert oracle.dgemm(A, B, Cin, 2.0, -3.0).tolist() == [[113, 131], [272, 306.5]]
+
+
+def test_dgemm_identity_and_near_exact():
+    g = W.rng(8, 0, 2)
+    A = g.uniform(-1, 1, (40, 33))
+    assert np.array_equal(oracle.dgemm(A, np.eye(33)), A)
+    B = g.uniform(-1, 1, (33, 50))
+    # extended-precision accumulation: within 1 ulp of the correctly rounded product
+    from fractions import Fraction
+    C = oracle.dgemm(A, B)
+    for (i, j) in [(0, 0), (39, 49), (7, 21)]:
+        exact = sum(Fraction(float(A[i, k])) * Fraction(float(B[k, j])) for k in range(33))
+        assert abs(Fraction(float(C[i, j])) - exact) <= Fraction(np.spacing(abs(float(exact)))), (i, j)

@@ -97,8 +97,9 @@ class JobSpec:
             return self.n
         if self.kernel == "blackscholes":
             return 12 * self.n
-        if self.kernel in ("sgemm", "sgemm_tf32"):
-            return 4 * (self.M * self.K + self.K * self.N + (self.M * self.N if self.beta != 0 else 0))
+        if self.kernel in ("sgemm", "sgemm_tf32", "dgemm"):
+            es = 8 if self.kernel == "dgemm" else 4
+            return es * (self.M * self.K + self.K * self.N + (self.M * self.N if self.beta != 0 else 0))
         raise ValueError(self.kernel)
 
     def output_bytes(self) -> int:
@@ -108,8 +109,8 @@ class JobSpec:
             return 1024
         if self.kernel == "blackscholes":
             return 8 * self.n
-        if self.kernel in ("sgemm", "sgemm_tf32"):
-            return 4 * self.M * self.N
+        if self.kernel in ("sgemm", "sgemm_tf32", "dgemm"):
+            return (8 if self.kernel == "dgemm" else 4) * self.M * self.N
         raise ValueError(self.kernel)
 
     def algorithmic_bytes(self) -> int:
@@ -120,12 +121,13 @@ class JobSpec:
             return self.n + 1024
         if self.kernel == "blackscholes":
             return 20 * self.n
-        if self.kernel in ("sgemm", "sgemm_tf32"):
-            return 4 * (self.M * self.K + self.K * self.N + self.M * self.N * (2 if self.beta != 0 else 1))
+        if self.kernel in ("sgemm", "sgemm_tf32", "dgemm"):
+            es = 8 if self.kernel == "dgemm" else 4
+            return es * (self.M * self.K + self.K * self.N + self.M * self.N * (2 if self.beta != 0 else 1))
         raise ValueError(self.kernel)
 
     def flops(self) -> int:
-        return 2 * self.M * self.N * self.K if self.kernel in ("sgemm", "sgemm_tf32") else 0
+        return 2 * self.M * self.N * self.K if self.kernel in ("sgemm", "sgemm_tf32", "dgemm") else 0
 
 
 def _scalar_for(seed: int, spec: JobSpec) -> None:
@@ -150,6 +152,18 @@ def make_inputs(spec: JobSpec, seed: int = BASE_SEED) -> Dict[str, np.ndarray]:
         return {"S": uniform_f32(rng(seed, vp, _S_A), n, 5.0, 30.0),
                 "X": uniform_f32(rng(seed, vp, _S_B), n, 1.0, 100.0),
                 "T": uniform_f32(rng(seed, vp, _S_C), n, 0.25, 10.0)}
+    if k == "dgemm":
+        M, N, K = spec.M, spec.N, spec.K
+        if spec.int_inputs:
+            A = rng(seed, vp, _S_A).integers(-8, 9, M * K).astype(np.float64).reshape(M, K)
+            B = rng(seed, vp, _S_B).integers(-8, 9, K * N).astype(np.float64).reshape(K, N)
+        else:
+            A = rng(seed, vp, _S_A).uniform(-1.0, 1.0, M * K).reshape(M, K)
+            B = rng(seed, vp, _S_B).uniform(-1.0, 1.0, K * N).reshape(K, N)
+        out = {"A": A, "B": B}
+        if spec.beta != 0:
+            out["C"] = rng(seed, vp, _S_C).uniform(-1.0, 1.0, M * N).reshape(M, N)
+        return out
     if k in ("sgemm", "sgemm_tf32"):
         M, N, K = spec.M, spec.N, spec.K
         if spec.int_inputs:
@@ -218,6 +232,13 @@ def config_specs(cfg: int, seed: int = BASE_SEED, nvps: Optional[int] = None,
         if s.kernel == "hist256":
             s.skew = (s.vp // 4) % 2 == 1 if cfg in (3, 4, 5) else False
     return specs
+
+
+def table1_specs(nvps: int = 8, iters: int = 300, size: int = 320) -> List[JobSpec]:
+    """The paper's Table 1 program on each of nvps VPs: `iters` multiplications of two
+    size x size fp64 matrices, one job per multiplication in program
+    order (vp-major list: VP v's jobs are consecutive)."""
+    return [JobSpec(v, "dgemm", M=size, N=size, K=size) for v in range(nvps) for _ in range(iters)]
 
 
 def mixed_small(nvps: int = 24, seed: int = BASE_SEED, max_n: int = 70000) -> List[JobSpec]:
