@@ -110,6 +110,10 @@ int32_t svp_abi_version(void);
  *   "blackscholes"  call/put per option              args svp_args_bs       bufs [S IN, X IN, T IN, call OUT, put OUT] f32
  *   "sgemm"         C = alpha A B + beta C, fp32 FFMA args svp_args_sgemm   bufs [A IN, B IN, C OUT (INOUT if beta != 0)]
  *   "sgemm_tf32"    same, tcgen05 TF32 tensor cores  (own tolerance 2e-3)
+ *   "dgemm"         C = alpha A B + beta C, fp64     args svp_args_dgemm   bufs [A IN, B IN, C OUT (INOUT if beta != 0)] f64
+ *                   (the paper's Table 1 guest: 320x320 fp64 matmul)
+ * GEMM jobs of different shapes are "identical kernels" too: one grouped launch covers
+ * every VP's (M, N, K) (ragged grouped GEMM).
  * Registration is idempotent; the id is stable for the context's lifetime.
  * Errors: SVP_E_NOKERNEL for an unknown name. */
 svp_status svp_register_kernel(svp_ctx* ctx, const char* name, int32_t* id_out);
@@ -119,6 +123,7 @@ typedef struct svp_args_saxpy { uint64_t n; float a; uint32_t _pad; } svp_args_s
 typedef struct svp_args_hist256 { uint64_t n; } svp_args_hist256;
 typedef struct svp_args_bs { uint64_t n; float R; float V; } svp_args_bs;
 typedef struct svp_args_sgemm { int32_t M, N, K; float alpha, beta; } svp_args_sgemm;
+typedef struct svp_args_dgemm { int32_t M, N, K, _pad; double alpha, beta; } svp_args_dgemm;
 
 /* ------------------------------------------------------------------ jobs */
 enum { SVP_DIR_IN = 1, SVP_DIR_OUT = 2, SVP_DIR_INOUT = 3 };

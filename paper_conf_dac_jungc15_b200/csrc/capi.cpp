@@ -30,6 +30,7 @@ static const KernelDesc kKernels[] = {
      sizeof(svp_args_bs)},
     {"sgemm", K_SGEMM, 3, {SVP_DIR_IN, SVP_DIR_IN, SVP_DIR_OUT, 0, 0}, sizeof(svp_args_sgemm)},
     {"sgemm_tf32", K_SGEMM_TF32, 3, {SVP_DIR_IN, SVP_DIR_IN, SVP_DIR_OUT, 0, 0}, sizeof(svp_args_sgemm)},
+    {"dgemm", K_DGEMM, 3, {SVP_DIR_IN, SVP_DIR_IN, SVP_DIR_OUT, 0, 0}, sizeof(svp_args_dgemm)},
 };
 
 const KernelDesc* kernel_desc(int32_t id) {

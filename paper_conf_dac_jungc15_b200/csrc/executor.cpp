@@ -228,7 +228,31 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
         if (ch.device != d.idx) continue;
         resolve_addresses(d, f, ch);
         const bool gemm = ch.kernel == K_SGEMM || ch.kernel == K_SGEMM_TF32;
-        if (!gemm) {
+        if (ch.kernel == K_DGEMM) {
+            ch.table_off = align_up(tbl.size(), 128);
+            tbl.resize(ch.table_off + ch.jobs.size() * sizeof(DgemmDesc));
+            uint32_t tiles = 0;
+            for (size_t k = 0; k < ch.jobs.size(); ++k) {
+                const Job& j = f.jobs[ch.jobs[k]];
+                DgemmDesc g;
+                memset(&g, 0, sizeof(g));
+                g.A = (const double*)ch.staged[k * SVP_MAX_BUFS + 0];
+                g.B = (const double*)ch.staged[k * SVP_MAX_BUFS + 1];
+                g.C = (double*)ch.staged[k * SVP_MAX_BUFS + 2];
+                g.M = j.M;
+                g.N = j.N;
+                g.K = j.K;
+                g.alpha = j.d0;
+                g.beta = j.d1;
+                g.tile_begin = tiles;
+                g.tiles_n = (uint32_t)((j.N + kDgemmBN - 1) / kDgemmBN);
+                uint64_t nt = (int64_t)j.M * j.N == 0 ? 0 : (uint64_t)((j.M + kDgemmBM - 1) / kDgemmBM) * g.tiles_n;
+                tiles += (uint32_t)nt;
+                memcpy(tbl.data() + ch.table_off + k * sizeof(DgemmDesc), &g, sizeof(g));
+            }
+            ch.total_tiles = tiles;
+            ch.nsegs = (int32_t)ch.jobs.size();
+        } else if (!gemm) {
             ch.table_off = align_up(tbl.size(), 128);
             tbl.resize(ch.table_off + ch.jobs.size() * sizeof(SegDesc));
             SegDesc* seg = reinterpret_cast<SegDesc*>(tbl.data() + ch.table_off);
@@ -353,6 +377,9 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
                                            ch.total_tiles, grid_of(1), s);
             return launch_sgemm_ffma((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
                                      ch.total_tiles, grid_of(d.lim.gemm_blocks_per_sm), s);
+        case K_DGEMM:
+            return launch_dgemm((const DgemmDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
+                                grid_of(d.lim.dgemm_blocks_per_sm), s);
         case K_SGEMM_TF32:
             return launch_sgemm_tf32((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
                                      ch.total_tiles, grid_of(1), s);
@@ -367,7 +394,7 @@ static bool chunk_needs_launch(const Flush& f, const Chunk& ch) {
     for (int32_t ji : ch.jobs) {
         const Job& j = f.jobs[ji];
         if (j.kernel == K_HIST256) return true;
-        if ((j.kernel == K_SGEMM || j.kernel == K_SGEMM_TF32) && (int64_t)j.M * j.N > 0) return true;
+        if (is_gemm(j.kernel) && (int64_t)j.M * j.N > 0) return true;
     }
     return false;
 }

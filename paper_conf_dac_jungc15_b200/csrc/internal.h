@@ -27,7 +27,8 @@ enum KernelId : int32_t {
     K_BLACKSCHOLES = 4,
     K_SGEMM = 5,
     K_SGEMM_TF32 = 6,
-    K_COUNT = 7
+    K_DGEMM = 7,
+    K_COUNT = 8
 };
 
 struct KernelDesc {
@@ -38,6 +39,7 @@ struct KernelDesc {
     uint32_t args_bytes;
 };
 const KernelDesc* kernel_desc(int32_t id);
+inline bool is_gemm(int32_t k) { return k == K_SGEMM || k == K_SGEMM_TF32 || k == K_DGEMM; }
 const KernelDesc* kernel_by_name(const char* name);
 
 // ------------------------------------------------------------------ jobs
@@ -52,6 +54,7 @@ struct Job {
     uint64_t n = 0;               // elements (memory-bound kernels)
     int32_t M = 0, N = 0, K = 0;  // sgemm
     float f0 = 0.f, f1 = 0.f;     // scalars
+    double d0 = 1.0, d1 = 0.0;    // dgemm alpha, beta
     uint64_t shape_key = 0;       // Kernel Match key (with kernel id)
     uint64_t in_bytes = 0;        // bytes of IN/INOUT buffers the kernel reads
     uint64_t out_bytes = 0;       // bytes of OUT/INOUT buffers the kernel writes
@@ -143,7 +146,8 @@ struct CostModel {
     bool sgemm_3xtf32 = false;
     double copy_ns = 2000;           // per-copy fixed overhead
     // EMA of measured/predicted ratio per kernel (learned from the profiler)
-    double kscale[K_COUNT] = {1, 1, 1, 1, 1, 1, 1};
+    double fp64_flops = 30e12;
+    double kscale[K_COUNT] = {1, 1, 1, 1, 1, 1, 1, 1};
     double kernel_ns(int32_t kernel, double alg_bytes, double flops) const;
     double h2d_ns(uint64_t bytes, int ncopies) const;
     double d2h_ns(uint64_t bytes, int ncopies) const;

@@ -15,6 +15,7 @@ struct LaunchLimits {
     int bs_blocks_per_sm = 4;
     int hist_blocks_per_sm = 4;
     int gemm_blocks_per_sm = 1;
+    int dgemm_blocks_per_sm = 1;
 };
 
 // Query occupancy / SM count for the current device (call once per device).
@@ -38,6 +39,10 @@ cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, ui
 // fp32-accurate grouped SGEMM on tcgen05: 3xTF32 (hi/lo operand split, 3 MMAs per k-step).
 cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
                                 int grid, cudaStream_t s);
+
+// Grouped fp64 GEMM (the paper's Table 1 matmul), FP64 DFMA with smem tiles.
+cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total_tiles, int grid, cudaStream_t s);
+cudaError_t query_limits_dgemm(int* per_sm);
 
 // Host: encode the TMA descriptors an SGEMM entry needs (driver entry point fetched at
 // runtime, so libsvp does not link libcuda).  variant 0 = FFMA tiles, 1 = TF32 tiles.

@@ -34,6 +34,7 @@ namespace svp {
 double CostModel::kernel_ns(int32_t kernel, double alg_bytes, double flops) const {
     double body;
     if (kernel == K_SGEMM) body = flops / (sgemm_3xtf32 ? tf32_flops / 3.0 : ffma_flops) * 1e9;
+    else if (kernel == K_DGEMM) body = flops / fp64_flops * 1e9;
     else if (kernel == K_SGEMM_TF32) body = flops / tf32_flops * 1e9;
     else body = alg_bytes / hbm_Bps * 1e9;
     return launch_ns + body * kscale[kernel];
@@ -54,9 +55,12 @@ uint64_t touched_bytes(const Job& j, int b) {
         case K_HIST256: return b == 0 ? j.n : 1024ull;
         case K_SGEMM:
         case K_SGEMM_TF32:
-            if (b == 0) return 4ull * j.M * j.K;
-            if (b == 1) return 4ull * j.K * j.N;
-            return 4ull * j.M * j.N;
+        case K_DGEMM: {
+            const uint64_t es = j.kernel == K_DGEMM ? 8 : 4;
+            if (b == 0) return es * j.M * j.K;
+            if (b == 1) return es * j.K * j.N;
+            return es * j.M * j.N;
+        }
     }
     return 0;
 }
@@ -101,10 +105,22 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
                 return fail(SVP_E_UNSUPPORTED, "svp_submit: sgemm needs K % 4 == 0 and N % 4 == 0 (TMA row pitch)");
             break;
         }
+        case K_DGEMM: {
+            svp_args_dgemm a;
+            memcpy(&a, j->args, sizeof(a));
+            if (a.M < 0 || a.N < 0 || a.K < 0 || a.M >= (1 << 20) || a.N >= (1 << 20) || a.K >= (1 << 20))
+                return fail(SVP_E_INVAL, "svp_submit: dgemm M,N,K must be in [0, 2^20)");
+            j->M = a.M;
+            j->N = a.N;
+            j->K = a.K;
+            j->d0 = a.alpha;
+            j->d1 = a.beta;
+            break;
+        }
     }
     if (j->n >= (1ull << 40)) return fail(SVP_E_INVAL, "svp_submit: n too large");
     // hist256 always writes its 256 counters (an empty input still overwrites them)
-    bool empty = (j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32) ? ((int64_t)j->M * j->N == 0)
+    bool empty = is_gemm(j->kernel) ? ((int64_t)j->M * j->N == 0)
                  : j->kernel == K_HIST256                             ? false
                                                                       : (j->n == 0);
     j->in_bytes = j->out_bytes = j->host_in_bytes = j->host_out_bytes = 0;
@@ -112,9 +128,10 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
         const svp_buf& bf = j->bufs[b];
         uint64_t need = touched_bytes(*j, b);
         int want = d->dirs[b];
-        bool is_c = (j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32) && b == 2;
+        bool is_c = is_gemm(j->kernel) && b == 2;
+        const bool beta_nz = j->kernel == K_DGEMM ? j->d1 != 0.0 : j->f1 != 0.f;
         if (is_c) {
-            if (j->f1 != 0.f && bf.dir != SVP_DIR_INOUT)
+            if (beta_nz && bf.dir != SVP_DIR_INOUT)
                 return fail(SVP_E_INVAL, "svp_submit: sgemm with beta != 0 needs C as SVP_DIR_INOUT");
             if (bf.dir != SVP_DIR_OUT && bf.dir != SVP_DIR_INOUT)
                 return fail(SVP_E_INVAL, "svp_submit: sgemm C must be OUT or INOUT");
@@ -132,6 +149,8 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
         if ((j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32) && bf.mem == SVP_MEM_DEVICE &&
             ((uintptr_t)bf.ptr & 15))
             return fail(SVP_E_UNSUPPORTED, "svp_submit: sgemm device buffers must be 16-B aligned (TMA)");
+        if (j->kernel == K_DGEMM && ((uintptr_t)bf.ptr & 7))
+            return fail(SVP_E_INVAL, "svp_submit: dgemm buffers must be 8-B aligned");
         bool rd = bf.dir & SVP_DIR_IN, wr = bf.dir & SVP_DIR_OUT;
         // sgemm C with beta == 0 is written only; hist counts are written only
         if (rd) j->in_bytes += need;
@@ -146,14 +165,18 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
         case K_SAXPY: j->alg_bytes = 12.0 * j->n; break;
         case K_HIST256: j->alg_bytes = (double)j->n + (j->n ? 1024.0 : 0.0); break;
         case K_BLACKSCHOLES: j->alg_bytes = 20.0 * j->n; break;
-        default:
-            j->alg_bytes = 4.0 * ((double)j->M * j->K + (double)j->K * j->N +
-                                  (double)j->M * j->N * (j->f1 != 0.f ? 2 : 1));
+        default: {
+            const bool dbl = j->kernel == K_DGEMM;
+            const bool beta_nz2 = dbl ? j->d1 != 0.0 : j->f1 != 0.f;
+            j->alg_bytes = (dbl ? 8.0 : 4.0) * ((double)j->M * j->K + (double)j->K * j->N +
+                                                (double)j->M * j->N * (beta_nz2 ? 2 : 1));
             j->flops = 2.0 * j->M * j->N * (double)j->K;
+        }
     }
-    j->shape_key = (j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32)
-                       ? (((uint64_t)j->M << 42) | ((uint64_t)j->N << 21) | (uint64_t)j->K)
-                       : 0;
+    // Reading R1 (revised with f2): every job of a kernel is "identical" -- ragged element
+    // counts AND ragged GEMM shapes share one coalesced launch (per-VP M, N, K live in
+    // the tile table).
+    j->shape_key = 0;
     double cost = c->cost.kernel_ns(j->kernel, j->alg_bytes, j->flops);
     j->device = dispatch_vp(c, j->vp, cost);
     if (c->exec && c->cfg.validate_ptrs && !empty) {

@@ -37,6 +37,19 @@ struct GemmDesc {
 };
 static_assert(sizeof(GemmDesc) == 64, "GemmDesc must be 64 B");
 
+// Grouped DGEMM (fp64): one entry per VP, plain pointers (no TMA).
+struct DgemmDesc {
+    const double* A;
+    const double* B;
+    double* C;
+    int32_t M, N, K;
+    uint32_t tile_begin;
+    double alpha, beta;
+    uint32_t tiles_n;
+    uint32_t _pad;
+};
+static_assert(sizeof(DgemmDesc) == 64, "DgemmDesc must be 64 B");
+
 // Tile geometry (elements per tile) -- host planner and kernels must agree.
 constexpr int kEwThreads = 256;
 constexpr int kVecaddVec = 4;                                  // float4 per thread per array
@@ -49,5 +62,6 @@ constexpr int kHistVec = 4;                                    // uint4 (16 B) p
 constexpr int kHistTile = kHistThreads * 16 * kHistVec;        // 16384 bytes
 constexpr int kGemmBM = 128, kGemmBN = 128, kGemmBK = 32;
 constexpr int kTf32BM = 128, kTf32BN = 256, kTf32BK = 16;
+constexpr int kDgemmBM = 64, kDgemmBN = 64, kDgemmBK = 16;
 
 }  // namespace svp

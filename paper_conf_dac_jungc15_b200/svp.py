@@ -167,6 +167,10 @@ def args_sgemm(M: int, N: int, K: int, alpha: float = 1.0, beta: float = 0.0) ->
     return struct.pack("<iiiff", M, N, K, alpha, beta)
 
 
+def args_dgemm(M: int, N: int, K: int, alpha: float = 1.0, beta: float = 0.0) -> bytes:
+    return struct.pack("<iiiidd", M, N, K, 0, alpha, beta)
+
+
 Buf = Tuple[int, int, int, int]  # (ptr, bytes, dir, mem)
 
 

@@ -24,16 +24,18 @@ BUFS = {
                      ("call", "f32", svp.DIR_OUT), ("put", "f32", svp.DIR_OUT)],
     "sgemm": [("A", "f32", svp.DIR_IN), ("B", "f32", svp.DIR_IN), ("C", "f32", svp.DIR_OUT)],
     "sgemm_tf32": [("A", "f32", svp.DIR_IN), ("B", "f32", svp.DIR_IN), ("C", "f32", svp.DIR_OUT)],
+    "dgemm": [("A", "f64", svp.DIR_IN), ("B", "f64", svp.DIR_IN), ("C", "f64", svp.DIR_OUT)],
 }
-_TORCH = {"f32": torch.float32, "u8": torch.uint8, "u32": torch.int32}
-_NP = {"f32": np.float32, "u8": np.uint8, "u32": np.uint32}
-_ES = {"f32": 4, "u8": 1, "u32": 4}
+GEMMS = ("sgemm", "sgemm_tf32", "dgemm")
+_TORCH = {"f32": torch.float32, "u8": torch.uint8, "u32": torch.int32, "f64": torch.float64}
+_NP = {"f32": np.float32, "u8": np.uint8, "u32": np.uint32, "f64": np.float64}
+_ES = {"f32": 4, "u8": 1, "u32": 4, "f64": 8}
 GUARD = 64
 
 
 def buffer_elems(spec, name: str) -> int:
     k = spec.kernel
-    if k in ("sgemm", "sgemm_tf32"):
+    if k in GEMMS:
         return {"A": spec.M * spec.K, "B": spec.K * spec.N, "C": spec.M * spec.N}[name]
     if k == "hist256" and name == "counts":
         return 256
@@ -50,6 +52,8 @@ def job_args(spec) -> bytes:
         return svp.args_hist256(spec.n)
     if k == "blackscholes":
         return svp.args_blackscholes(spec.n, spec.R, spec.V)
+    if k == "dgemm":
+        return svp.args_dgemm(spec.M, spec.N, spec.K, spec.alpha, spec.beta)
     return svp.args_sgemm(spec.M, spec.N, spec.K, spec.alpha, spec.beta)
 
 
@@ -86,7 +90,7 @@ class VPSet:
                 # misalign 1: every buffer shifted by one element (co-aligned -> vector path
                 # with a head shift); misalign 2: only the first buffer (scalar path)
                 mis = m if (m == 1 or bi == 0) else 0
-                if s.kernel in ("sgemm", "sgemm_tf32") or (s.kernel == "hist256" and name == "counts"):
+                if s.kernel in GEMMS or (s.kernel == "hist256" and name == "counts"):
                     mis = 0
                 elif s.kernel == "hist256":
                     mis = 7 * m
@@ -109,7 +113,7 @@ class VPSet:
         for i, s in enumerate(self.specs):
             inp = self.inputs[i]
             for name, dt, d in BUFS[s.kernel]:
-                if s.kernel in ("sgemm", "sgemm_tf32") and name == "C" and s.beta != 0:
+                if s.kernel in GEMMS and name == "C" and s.beta != 0:
                     d = svp.DIR_INOUT  # C is read when beta != 0
                 if d & svp.DIR_IN and name in inp:
                     src = torch.from_numpy(np.ascontiguousarray(inp[name]).reshape(-1).view(_NP[dt]))
@@ -120,7 +124,7 @@ class VPSet:
                     # outputs start as NaN/garbage so a missing write is caught
                     v = self.bufs[i][name]
                     if v.numel():
-                        if v.dtype == torch.float32:
+                        if v.dtype in (torch.float32, torch.float64):
                             v.fill_(float("nan"))
                         else:
                             v.fill_(-1 if v.dtype == torch.int32 else 0x5A)
@@ -132,7 +136,7 @@ class VPSet:
             bl = []
             for name, dt, d in BUFS[s.kernel]:
                 t = self.bufs[i][name]
-                if s.kernel in ("sgemm", "sgemm_tf32") and name == "C" and s.beta != 0:
+                if s.kernel in GEMMS and name == "C" and s.beta != 0:
                     d = svp.DIR_INOUT
                 bl.append((t.data_ptr() if t.numel() else 0, t.numel() * t.element_size(), d, mem))
             jobs.append((s.vp, self.kids[s.kernel], job_args(s), bl))
@@ -145,12 +149,12 @@ class VPSet:
         s = self.specs[i]
         out = {}
         for name, dt, d in BUFS[s.kernel]:
-            if d & svp.DIR_OUT or (s.kernel in ("sgemm", "sgemm_tf32") and name == "C"):
+            if d & svp.DIR_OUT or (s.kernel in GEMMS and name == "C"):
                 t = self.bufs[i][name].cpu()
                 a = t.numpy()
                 if dt == "u32":
                     a = a.view(np.uint32)
-                if s.kernel in ("sgemm", "sgemm_tf32"):
+                if s.kernel in GEMMS:
                     a = a.reshape(s.M, s.N)
                 out[name] = a.copy()
         return out

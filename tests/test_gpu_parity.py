@@ -218,3 +218,43 @@ def test_two_logical_gpus_one_process(small, residency):
         check_job(s, inp, vs.output(i))
     assert vs.guards_intact()
     ctx.close()
+
+
+def test_ragged_grouped_sgemm_one_launch():
+    """Different (M, N, K) per VP in ONE coalesced launch (FFMA and 3xTF32)."""
+    dims = [(256, 512, 128), (128, 128, 512), (300, 260, 100), (64, 1024, 64), (1, 8, 8), (513, 132, 36)]
+    specs = [W.JobSpec(v, "sgemm", M=M, N=N, K=K) for v, (M, N, K) in enumerate(dims)]
+    inputs = inputs_for(specs)
+    for impl in (svp.SGEMM_FFMA, svp.SGEMM_3XTF32):
+        outs, _, st = run_svp(specs, inputs, "device", sgemm_impl=impl)
+        assert st["launches"] == 1
+        for s, inp, got in zip(specs, inputs, outs):
+            check_job(s, inp, got)
+
+
+@pytest.mark.parametrize("residency", ["device", "host"])
+def test_dgemm_ragged_and_alpha_beta(residency):
+    dims = [(320, 320, 320), (320, 320, 320), (65, 33, 129), (1, 1, 1), (100, 200, 0), (7, 130, 64)]
+    specs = [W.JobSpec(v, "dgemm", M=M, N=N, K=K, alpha=(1.0 if v % 2 else -0.75), beta=(0.0 if v % 3 else 0.5))
+             for v, (M, N, K) in enumerate(dims)]
+    specs.append(W.JobSpec(9, "dgemm", M=96, N=96, K=96, int_inputs=True))
+    inputs = inputs_for(specs)
+    outs, _, st = run_svp(specs, inputs, residency)
+    assert st["groups"] == 1
+    for s, inp, got in zip(specs, inputs, outs):
+        check_job(s, inp, got)
+
+
+def test_table1_program_8vps():
+    """The paper's Table 1 program on 8 VPs (fewer iterations): each VP multiplies two
+    320x320 fp64 matrices `iters` times in program order; every level is one coalesced
+    launch of 8 VPs."""
+    iters = 10
+    specs = W.table1_specs(nvps=8, iters=iters)
+    base = [W.make_inputs(s) for s in specs[::iters]]
+    inputs = [base[i // iters] for i in range(len(specs))]
+    outs, _, st = run_svp(specs, inputs, "device")
+    assert st["levels"] == iters and st["groups"] == iters
+    want = [oracle.run_job(specs[v * iters], base[v]) for v in range(8)]
+    for i, (s, got) in enumerate(zip(specs, outs)):
+        check_job(s, inputs[i], got, want[i // iters])

@@ -63,14 +63,17 @@ def test_kernel_match_groups_identical_kernels():
         assert seen == set(range(64))
 
 
-def test_sgemm_needs_equal_shapes():
+def test_ragged_gemm_shapes_share_one_launch():
+    """Reading R1 as revised for NEXT item f2: GEMMs of different (M, N, K) are identical
+    kernel requests too -- one grouped launch carries every VP's shape in its tile table."""
     with svp.Context(dry_run=True) as c:
         for vp in range(6):
             s = 128 if vp < 4 else 256
-            submit(c, vp, "sgemm", M=s, N=s, K=s)
+            submit(c, vp, "sgemm", M=s, N=s + 64, K=s // 2)
         c.flush()
-        sizes = sorted(op["nvps"] for op in c.plan())
-        assert sizes == [2, 4]
+        ops = c.plan()
+        assert [op["nvps"] for op in ops] == [6]
+        assert ops[0]["flops"] == sum(2.0 * s * (s + 64) * (s // 2) for s in [128] * 4 + [256] * 2)
 
 
 def test_no_coalescing_is_one_launch_per_job_in_submission_order():
