@@ -11,6 +11,9 @@ S3 (Fig 9 + Eq 7/8): N host-resident SGEMM jobs (H2D A,B -> 
     D2H C) with Tk ~ Tm, interleaved on separate copy/compute streams vs one stream;
     measured speedup next to Eq 7's prediction from the measured Tm, Tk.
 S4 (BASELINE metric): jobs/s of the cfg5 mix vs #VPs (1 GPU).
+S5 (Table 1): N VPs each running the paper's program -- 300
+    multiplications of two 320x320 fp64 matrices -- coalesced per program-order level vs
+    serial per-VP launches; DGEMM TFLOP/s.
 Times are CUDA-event device times around whole flushes (median of reps).
 """
 import argparse
@@ -147,11 +150,42 @@ def s4_vps(quick):
     return rows
 
 
+def s5_table1(quick):
+    iters = 100 if quick else 300
+    rows = []
+    for nv in ([1, 8] if quick else [1, 2, 4, 8, 16, 32]):
+        specs = W.table1_specs(nvps=nv, iters=iters)
+        base = [W.make_inputs(s) for s in specs[::iters]]
+        c = ctx_for(profile_level=1)
+        # every job of a VP reuses the VP's A, B, C buffers (the program's loop body)
+        vs = VPSet(c, specs[::iters], base, "device")
+        one = vs.job_list()
+        jobs = [one[i // iters] for i in range(len(specs))]
+        c.reset_profile()
+        t = flush_time(c, jobs, reps=3, warm=1)
+        ks = c.kernel_stats(c.kernel_ids["dgemm"])
+        row = {"vps": nv, "iters": iters, "coalesced_ms": t * 1e3, "jobs_per_s": len(jobs) / t,
+               "dgemm_tflops_kernel": ks["flops"] / ks["total_ns"] / 1e3 if ks["total_ns"] else None,
+               "launches_per_flush": c.flush_stats()["launches"]}
+        sc = ctx_for(coalesce=False, interleave=False, sync_each_job=True)
+        sc.register_kernel("dgemm")
+        ts = flush_time(sc, jobs, reps=1, warm=1)
+        sc.close()
+        row["serial_sync_ms"] = ts * 1e3
+        row["speedup_vs_serial_sync"] = ts / t
+        rows.append(row)
+        c.close()
+        del vs
+        torch.cuda.empty_cache()
+    return {"paper_table1_ms": {"native_gpu_quadro4000": 170.79, "sigma_vp": 568.12, "emul_on_cpu": 9141.51},
+            "rows": rows}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default=None)
     ap.add_argument("--quick", action="store_true")
-    ap.add_argument("--only", default="1234")
+    ap.add_argument("--only", default="12345")
     args = ap.parse_args()
     torch.cuda.set_device(0)
     res = {"gpu": torch.cuda.get_device_name(0)}
@@ -163,6 +197,8 @@ def main():
         res["S3_interleaving_fig9"] = s3_interleaving(args.quick)
     if "4" in args.only:
         res["S4_jobs_vs_vps"] = s4_vps(args.quick)
+    if "5" in args.only:
+        res["S5_table1_dgemm"] = s5_table1(args.quick)
     txt = json.dumps(res, indent=1)
     print(txt)
     if args.out:
