@@ -124,27 +124,54 @@ __global__ void __launch_bounds__(kEwThreads) k_saxpy(const SegDesc* __restrict_
 }
 
 // --------------------------------------------------------------------- Black-Scholes
-// Same formula as the oracle (CUDA-SDK form, A&S 26.2.17 CND), evaluated with the SFU
-// approximations the SDK sample uses (ex2/lg2/rcp/rsqrt based __expf, __logf,
-// __fdividef, rsqrtf): ~2-ulp-class errors, orders of magnitude inside the 1e-5
-// parity bound (R10), and ~3x fewer instructions than the libm-accurate
-// versions, which made the kernel ALU-bound at 53 % of HBM (profiles/r01).
+// Same formula as the oracle (CUDA-SDK form, A&S 26.2.17 CND) evaluated straight on the
+// SFU: rcp/rsqrt/lg2/ex2 .approx (2^-22-class relative errors), with the constants
+// folded so an option costs ~50 instructions (the libm-accurate form cost ~160 and made
+// the kernel ALU-bound at 53 % of HBM -- profiles/r01).  The resulting error is orders of
+// magnitude inside the 1e-5 parity bound (R10/R17): |d1 error| < ~2e-6 gives
+// |dN| < 1e-6 and |d price| < 1e-6 max(S, X).
+__device__ __forceinline__ float rcp_a(float x) {
+    float r;
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+    return r;
+}
+__device__ __forceinline__ float rsqrt_a(float x) {
+    float r;
+    asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+    return r;
+}
+__device__ __forceinline__ float lg2_a(float x) {
+    float r;
+    asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+    return r;
+}
+__device__ __forceinline__ float ex2_a(float x) {
+    float r;
+    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+    return r;
+}
+
 __device__ __forceinline__ float cnd_as(float d) {
     const float A1 = 0.31938153f, A2 = -0.356563782f, A3 = 1.781477937f, A4 = -1.821255978f,
                 A5 = 1.330274429f;
-    const float RSQRT2PI = 0.39894228040143267793994605993438f;
-    float K = __fdividef(1.0f, fmaf(0.2316419f, fabsf(d), 1.0f));
-    float cnd = RSQRT2PI * __expf(-0.5f * d * d) * (K * (A1 + K * (A2 + K * (A3 + K * (A4 + K * A5)))));
+    // RSQRT2PI * exp(-d^2/2) = 2^(d^2 * (-log2(e)/2) + log2(RSQRT2PI))
+    const float kE = -0.72134752044448170368f, kL = -1.32574806473616855f;
+    const float K = rcp_a(fmaf(0.2316419f, fabsf(d), 1.0f));
+    const float e = ex2_a(fmaf(d * d, kE, kL));
+    const float cnd = e * (K * (A1 + K * (A2 + K * (A3 + K * (A4 + K * A5)))));
     return d > 0.f ? 1.0f - cnd : cnd;
 }
 
-__device__ __forceinline__ void bs_one(float S, float X, float T, float R, float V, float& call, float& put) {
-    float sqrtT = T * rsqrtf(T);
-    float VsqrtT = V * sqrtT;
-    float d1 = __fdividef(__logf(__fdividef(S, X)) + (R + 0.5f * V * V) * T, VsqrtT);
-    float d2 = d1 - VsqrtT;
-    float N1 = cnd_as(d1), N2 = cnd_as(d2);
-    float XexpRT = X * __expf(-R * T);
+// mu = R + V^2/2 and mRlog2e = -R log2(e) are per-VP uniforms hoisted by the caller.
+__device__ __forceinline__ void bs_one(float S, float X, float T, float mu, float mRlog2e, float V, float& call,
+                                       float& put) {
+    const float LN2 = 0.69314718055994530942f;
+    const float sqrtT = T * rsqrt_a(T);
+    const float VsqrtT = V * sqrtT;
+    const float d1 = fmaf(lg2_a(S * rcp_a(X)), LN2, mu * T) * rcp_a(VsqrtT);
+    const float d2 = d1 - VsqrtT;
+    const float N1 = cnd_as(d1), N2 = cnd_as(d2);
+    const float XexpRT = X * ex2_a(mRlog2e * T);
     call = S * N1 - XexpRT * N2;
     put = XexpRT * (1.0f - N2) - S * (1.0f - N1);
 }
@@ -161,6 +188,7 @@ __global__ void __launch_bounds__(kEwThreads) k_blackscholes(const SegDesc* __re
         float* __restrict__ C = reinterpret_cast<float*>(sd.ptr[3]);
         float* __restrict__ P = reinterpret_cast<float*>(sd.ptr[4]);
         const float R = sd.f[0], Vol = sd.f[1];
+        const float mu = R + 0.5f * Vol * Vol, mRlog2e = -R * 1.44269504088896340736f;
         int64_t e0, e1;
         bool vec;
         tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, TILE, e0, e1, vec);
@@ -176,10 +204,10 @@ __global__ void __launch_bounds__(kEwThreads) k_blackscholes(const SegDesc* __re
 #pragma unroll
             for (int i = 0; i < V; ++i) {
                 float4 c, p;
-                bs_one(rs[i].x, rx[i].x, rt[i].x, R, Vol, c.x, p.x);
-                bs_one(rs[i].y, rx[i].y, rt[i].y, R, Vol, c.y, p.y);
-                bs_one(rs[i].z, rx[i].z, rt[i].z, R, Vol, c.z, p.z);
-                bs_one(rs[i].w, rx[i].w, rt[i].w, R, Vol, c.w, p.w);
+                bs_one(rs[i].x, rx[i].x, rt[i].x, mu, mRlog2e, Vol, c.x, p.x);
+                bs_one(rs[i].y, rx[i].y, rt[i].y, mu, mRlog2e, Vol, c.y, p.y);
+                bs_one(rs[i].z, rx[i].z, rt[i].z, mu, mRlog2e, Vol, c.z, p.z);
+                bs_one(rs[i].w, rx[i].w, rt[i].w, mu, mRlog2e, Vol, c.w, p.w);
                 __stcs(reinterpret_cast<float4*>(C + e0) + o + i * kEwThreads, c);
                 __stcs(reinterpret_cast<float4*>(P + e0) + o + i * kEwThreads, p);
             }
@@ -201,7 +229,7 @@ __global__ void __launch_bounds__(kEwThreads) k_blackscholes(const SegDesc* __re
                     const int64_t i = e + k * kEwThreads;
                     if (i < e1) {
                         float c, p;
-                        bs_one(rs[k], rx[k], rt[k], R, Vol, c, p);
+                        bs_one(rs[k], rx[k], rt[k], mu, mRlog2e, Vol, c, p);
                         C[i] = c;
                         P[i] = p;
                     }
