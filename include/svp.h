@@ -190,6 +190,40 @@ svp_status svp_wait(svp_ctx* ctx, uint64_t job, int32_t timeout_ms);
 svp_status svp_start_dispatcher(svp_ctx* ctx, int32_t window_us, int32_t max_jobs);
 svp_status svp_stop_dispatcher(svp_ctx* ctx);
 
+/* ------------------------------------------------------------------ IPC front end */
+/* The paper's IPC Manager (VPs reach the host "through an IPC method
+ * such as socket or shared memory"): VP *processes* submit jobs to a server process that
+ * owns the svp context.  svp_ipc_serve creates the POSIX shared-memory segment `name`
+ * (no '/'; shm_open("/name")) holding a ticketed ring of nslots job slots and a data
+ * arena of arena_bytes, registers the arena with CUDA (so jobs use it as HOST_PINNED
+ * memory -- staged, coalesced and interleaved like any host-resident job), starts the
+ * context's dispatcher if it is not running, and serves until svp_ipc_shutdown (which
+ * also unlinks the segment).  Clients need no CUDA: svp_ipc_connect maps the segment,
+ * svp_ipc_alloc bump-allocates 256-B aligned arena space (returns its offset and a
+ * pointer in the caller's mapping), svp_ipc_submit queues a job whose buffers are arena
+ * offsets (returns a ticket), svp_ipc_wait blocks until that job has run (its outputs
+ * are then in the arena) and returns the job's status.  Each ticket is waited once. */
+typedef struct svp_ipc_server svp_ipc_server;
+typedef struct svp_ipc_client svp_ipc_client;
+typedef struct svp_ipc_buf {
+    uint64_t offset; /* arena offset from svp_ipc_alloc */
+    uint64_t bytes;
+    int32_t dir;     /* SVP_DIR_* */
+    int32_t _pad;
+} svp_ipc_buf;
+svp_status svp_ipc_serve(svp_ctx* ctx, const char* name, uint64_t arena_bytes, int32_t nslots,
+                         svp_ipc_server** out);
+svp_status svp_ipc_server_stats(svp_ipc_server* s, uint64_t* jobs_served, uint64_t* tickets_issued);
+svp_status svp_ipc_shutdown(svp_ipc_server* s);
+svp_status svp_ipc_connect(const char* name, svp_ipc_client** out);
+svp_status svp_ipc_disconnect(svp_ipc_client* c);
+svp_status svp_ipc_alloc(svp_ipc_client* c, uint64_t bytes, uint64_t* offset_out, void** ptr_out);
+svp_status svp_ipc_submit(svp_ipc_client* c, int32_t vp, int32_t kernel, const void* args, size_t args_bytes,
+                          const svp_ipc_buf* bufs, int32_t nbufs, uint64_t* ticket_out);
+svp_status svp_ipc_wait(svp_ipc_client* c, uint64_t ticket, int32_t timeout_ms);
+/* Builtin kernel ids are stable; clients (which have no context) look them up by name. */
+svp_status svp_kernel_lookup(const char* name, int32_t* id_out);
+
 /* ------------------------------------------------------------------ Job Dispatcher */
 /* The GPU (index into the context's device list, 0..num_gpus-1) that runs VP `vp`.
  * Sticky: assigned on first use (least-loaded by estimated cost so far) or by

@@ -179,6 +179,26 @@ svp_status svp_register_kernel(svp_ctx* h, const char* name, int32_t* id_out) {
     SVP_TRY_END
 }
 
+}  // extern "C"
+
+// Status of a completed job: the failed flush whose id range covers it, else OK.
+svp_status svp::ctx_job_status(Ctx* c, uint64_t job) {
+    std::lock_guard<std::mutex> lk(c->done_mu);
+    uint64_t lo = 0;
+    for (const auto& fr : c->failed) {
+        if (job > lo && job <= fr.first) return fr.second;
+        lo = fr.first;
+    }
+    return SVP_OK;
+}
+
+uint64_t svp::ctx_completed_upto(Ctx* c, int32_t) {
+    std::lock_guard<std::mutex> lk(c->done_mu);
+    return c->completed_upto;
+}
+
+extern "C" {
+
 static svp_status submit_many(Ctx* c, int32_t n, const svp_job_desc* jd, const svp_job_desc* single_args_src,
                               uint64_t* ids) {
     (void)single_args_src;
@@ -344,16 +364,10 @@ svp_status svp_wait(svp_ctx* h, uint64_t job, int32_t timeout_ms) {
         set_error("svp_wait: context errored before the job ran: " + c->sticky_msg);
         return SVP_E_STATE;
     }
-    // the first failed flush whose range covers the job decides its status
-    uint64_t lo = 0;
-    for (const auto& fr : c->failed) {
-        if (job > lo && job <= fr.first) {
-            set_error("svp_wait: the flush that ran this job failed");
-            return fr.second;
-        }
-        lo = fr.first;
-    }
-    return SVP_OK;
+    lk.unlock();
+    svp_status js = ctx_job_status(c, job);
+    if (js) set_error("svp_wait: the flush that ran this job failed");
+    return js;
     SVP_TRY_END
 }
 
@@ -377,6 +391,15 @@ static void dispatcher_loop(Ctx* c) {
         }
     }
 }
+
+}  // extern "C"
+
+svp_status svp::ctx_submit_one(Ctx* c, const svp_job_desc& d, uint64_t* id) {
+    if (c->sticky != SVP_OK) return SVP_E_STATE;
+    return submit_many(c, 1, &d, nullptr, id);
+}
+
+extern "C" {
 
 svp_status svp_start_dispatcher(svp_ctx* h, int32_t window_us, int32_t max_jobs) {
     SVP_TRY_BEGIN

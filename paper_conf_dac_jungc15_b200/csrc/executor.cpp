@@ -160,6 +160,25 @@ void executor_destroy(Executor* e) {
     delete e;
 }
 
+svp_status executor_register_host(Executor* e, void* p, uint64_t bytes, std::string* why) {
+    if (e->devs.empty()) return SVP_OK;
+    cudaSetDevice(e->devs[0].ordinal);
+    cudaError_t ce = cudaHostRegister(p, bytes, cudaHostRegisterPortable);
+    if (ce != cudaSuccess) {
+        cudaGetLastError();
+        *why = cudaGetErrorString(ce);
+        return SVP_E_CUDA;
+    }
+    return SVP_OK;
+}
+
+void executor_unregister_host(Executor* e, void* p) {
+    if (e->devs.empty()) return;
+    cudaSetDevice(e->devs[0].ordinal);
+    cudaHostUnregister(p);
+    cudaGetLastError();
+}
+
 svp_status executor_check_ptr(Executor* e, const void* p, int32_t mem, int32_t device, std::string* why) {
     cudaPointerAttributes at;
     cudaError_t ce = cudaPointerGetAttributes(&at, p);

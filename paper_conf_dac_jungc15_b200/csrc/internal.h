@@ -225,4 +225,9 @@ svp_status executor_check_ptr(Executor* e, const void* p, int32_t mem, int32_t d
 // errors
 void set_error(const std::string& msg);
 
+// used by the IPC front end (ipc.cpp)
+svp_status ctx_submit_one(Ctx* c, const svp_job_desc& d, uint64_t* id);
+uint64_t ctx_completed_upto(Ctx* c, int32_t unused = 0);
+svp_status ctx_job_status(Ctx* c, uint64_t job);
+
 }  // namespace svp

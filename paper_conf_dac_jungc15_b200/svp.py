@@ -31,7 +31,8 @@ EXPORTS = ("svp_config_default", "svp_init", "svp_finalize", "svp_last_error", "
            "svp_register_kernel", "svp_submit", "svp_submit_batch", "svp_flush", "svp_vp_device",
            "svp_assign_vps", "svp_lpt_partition", "svp_profile", "svp_reset_profile", "svp_kernel_stats_get",
            "svp_flush_stats_get", "svp_plan_size", "svp_plan_get", "svp_wait", "svp_start_dispatcher",
-           "svp_stop_dispatcher")
+           "svp_stop_dispatcher", "svp_ipc_serve", "svp_ipc_server_stats", "svp_ipc_shutdown", "svp_ipc_connect",
+           "svp_ipc_disconnect", "svp_ipc_alloc", "svp_ipc_submit", "svp_ipc_wait", "svp_kernel_lookup")
 
 
 class svp_config(C.Structure):
@@ -51,6 +52,10 @@ class svp_buf(C.Structure):
 class svp_job_desc(C.Structure):
     _fields_ = [("vp", C.c_int32), ("kernel", C.c_int32), ("args_bytes", C.c_uint32), ("nbufs", C.c_int32),
                 ("args", C.c_uint8 * MAX_ARGS), ("bufs", svp_buf * MAX_BUFS)]
+
+
+class svp_ipc_buf(C.Structure):
+    _fields_ = [("offset", C.c_uint64), ("bytes", C.c_uint64), ("dir", C.c_int32), ("_pad", C.c_int32)]
 
 
 class svp_vp_profile(C.Structure):
@@ -129,6 +134,16 @@ def load(build_if_stale: bool = True):
         L.svp_wait.argtypes = [vp, C.c_uint64, C.c_int32]
         L.svp_start_dispatcher.argtypes = [vp, C.c_int32, C.c_int32]
         L.svp_stop_dispatcher.argtypes = [vp]
+        L.svp_ipc_serve.argtypes = [vp, C.c_char_p, C.c_uint64, C.c_int32, P(vp)]
+        L.svp_ipc_server_stats.argtypes = [vp, P(C.c_uint64), P(C.c_uint64)]
+        L.svp_ipc_shutdown.argtypes = [vp]
+        L.svp_ipc_connect.argtypes = [C.c_char_p, P(vp)]
+        L.svp_ipc_disconnect.argtypes = [vp]
+        L.svp_ipc_alloc.argtypes = [vp, C.c_uint64, P(C.c_uint64), P(vp)]
+        L.svp_ipc_submit.argtypes = [vp, C.c_int32, C.c_int32, C.c_void_p, C.c_size_t, P(svp_ipc_buf), C.c_int32,
+                                     P(C.c_uint64)]
+        L.svp_ipc_wait.argtypes = [vp, C.c_uint64, C.c_int32]
+        L.svp_kernel_lookup.argtypes = [C.c_char_p, P(C.c_int32)]
         for name in EXPORTS:
             f = getattr(L, name)
             if name not in ("svp_config_default", "svp_last_error", "svp_abi_version"):
@@ -347,3 +362,69 @@ class Context:
             d["vps"] = list(vps[: min(op.nvps, 4096)])
             out.append(d)
         return out
+
+
+# ----------------------------------------------------------------- IPC front end
+def kernel_lookup(name: str) -> int:
+    kid = C.c_int32()
+    _check(load().svp_kernel_lookup(name.encode(), C.byref(kid)))
+    return kid.value
+
+
+class IpcServer:
+    """svp_ipc_serve: serve VP processes through the shared-memory segment `name`."""
+
+    def __init__(self, ctx: "Context", name: str, arena_bytes: int = 1 << 28, nslots: int = 1024):
+        self._L = load()
+        h = C.c_void_p()
+        _check(self._L.svp_ipc_serve(ctx._h, name.encode(), arena_bytes, nslots, C.byref(h)))
+        self._h = h
+        self.ctx = ctx
+
+    def stats(self):
+        served, tickets = C.c_uint64(), C.c_uint64()
+        _check(self._L.svp_ipc_server_stats(self._h, C.byref(served), C.byref(tickets)))
+        return {"served": served.value, "tickets": tickets.value}
+
+    def shutdown(self):
+        if getattr(self, "_h", None):
+            _check(self._L.svp_ipc_shutdown(self._h))
+            self._h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.shutdown()
+
+
+class IpcClient:
+    """A VP process's view of an IpcServer (no CUDA needed in this process)."""
+
+    def __init__(self, name: str):
+        self._L = load(build_if_stale=False)
+        h = C.c_void_p()
+        _check(self._L.svp_ipc_connect(name.encode(), C.byref(h)))
+        self._h = h
+
+    def alloc(self, nbytes: int):
+        """Returns (offset, address) of nbytes in the shared arena."""
+        off, ptr = C.c_uint64(), C.c_void_p()
+        _check(self._L.svp_ipc_alloc(self._h, nbytes, C.byref(off), C.byref(ptr)))
+        return off.value, ptr.value
+
+    def submit(self, vp: int, kernel: int, args: bytes, bufs: Sequence[Tuple[int, int, int]]) -> int:
+        """bufs: (arena offset, bytes, dir).  Returns a ticket."""
+        arr = (svp_ipc_buf * max(1, len(bufs)))(*[svp_ipc_buf(o, b, d, 0) for (o, b, d) in bufs])
+        t = C.c_uint64()
+        ab = C.create_string_buffer(args, len(args))
+        _check(self._L.svp_ipc_submit(self._h, vp, kernel, ab, len(args), arr, len(bufs), C.byref(t)))
+        return t.value
+
+    def wait(self, ticket: int, timeout_ms: int = 0):
+        _check(self._L.svp_ipc_wait(self._h, ticket, timeout_ms))
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _check(self._L.svp_ipc_disconnect(self._h))
+            self._h = None
