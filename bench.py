@@ -359,9 +359,10 @@ def run_svp(args, rank, ws, local):
 
     # ---------------- serial baselines on the same GPU, same buffers, same kernels
     serial = {}
+    by_kernel = {}
     if not args.no_serial:
         for name, kw in (("B1_serial_sync", dict(coalesce=False, interleave=False, sync_each_job=True)),
-                         ("B2_serial_async", dict(coalesce=False, interleave=False))):
+                         ("B2_serial_async", dict(coalesce=False, interleave=False, profile_level=1))):
             sctx = svp.Context(num_gpus=1, device_ids=[local], external_streams=[stream.cuda_stream],
                                sgemm_impl=impl, **kw)
             for k in vs.kids:
@@ -369,10 +370,22 @@ def run_svp(args, rank, ws, local):
             ks = max(2, args.steps // 5)
             sctx.submit_batch(jobs)
             sctx.flush()
+            sctx.reset_profile()
             barrier(ws)
             sdt = max_over_ranks(timed_steps(sctx, jobs, ks, stream), ws)
             serial[name] = {"value": n_jobs_total * ks / sdt, "unit": "jobs/s", "steps": ks,
                             "ms_per_step": sdt / ks * 1e3}
+            if name == "B2_serial_async":
+                # Eq 9's alignment gain per kernel class: per-job launches vs one coalesced
+                # launch of the same jobs (event-timed kernel time per step, 1 stream each)
+                for kname, kid in vs.kids.items():
+                    st_ser = sctx.kernel_stats(kid)
+                    st_coal = kstats[kname]
+                    if st_ser["launches"] and st_coal["launches"]:
+                        ser_ms = st_ser["total_ns"] / ks / 1e6
+                        coal_ms = st_coal["total_ns"] / st_coal["launches"] / 1e6
+                        by_kernel[kname] = {"serial_kernel_ms": ser_ms, "coalesced_kernel_ms": coal_ms,
+                                            "speedup": ser_ms / coal_ms}
             sctx.close()
     ctx.close()
     del vs
@@ -419,7 +432,7 @@ def run_svp(args, rank, ws, local):
             "elements_per_s": sum(s.n for s in all_specs) * args.steps / dt_max,
             "sgemm_impl": args.sgemm_impl, "alt_sgemm_impl": alt,
             "speedup_vs_serial": {k: value / v["value"] for k, v in serial.items()},
-            "serial": serial, "per_kernel": per_kernel,
+            "serial": serial, "speedup_by_kernel_class": by_kernel, "per_kernel": per_kernel,
             "one_stream": {"value": iso_value, "unit": "jobs/s",
                            "note": "coalesced, 1 compute stream (no interleaving); per_kernel/roofline timed here"},
             "flush": {"host_plan_us": st["host_plan_ns"] / 1e3, "host_issue_us": st["host_issue_ns"] / 1e3,
