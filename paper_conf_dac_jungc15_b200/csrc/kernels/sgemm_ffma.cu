@@ -14,7 +14,8 @@
 //    ring guarded by full/empty mbarriers; per-VP CUtensorMaps live in the table.
 //  * warps 0-7 = consumers: 8x8 fp32 register micro-tile per thread; per 4-k group a
 //    thread reads 8 float4 of A (k-vectorised, conflict-free thanks to the swizzle) and
-//    8 float4 of B, then issues 256 FFMA (16 FFMA per LDS.128).
+//    8 float4 of B, then issues 128 FFMA2 (fma.rn.f32x2: a broadcast A value times a pair
+//    of B values, per-lane IEEE rounding) = 256 FMAs, half the issue slots of FFMA.
 //  * epilogue: alpha*acc (+ beta*C) with 128-bit stores straight from registers.
 #include <cuda.h>
 #include <stdio.h>
@@ -101,11 +102,14 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         const uint32_t lt = t - g.tile_begin;
         const int tm = lt / g.tiles_n, tn = lt % g.tiles_n;
         const int KB = (g.K + GK - 1) / GK;
-        float acc[8][8];
+        // accumulators as packed fp32 pairs: acc[i][p] = C(row i, cols 2p, 2p+1) of the
+        // thread's 8 columns; FFMA2 (fma.rn.f32x2) does both lanes with one instruction and
+        // per-lane IEEE rounding identical to FFMA
+        unsigned long long acc[8][4];
 #pragma unroll
         for (int i = 0; i < 8; ++i)
 #pragma unroll
-            for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+            for (int p = 0; p < 4; ++p) acc[i][p] = 0ull;
 
         for (int kb = 0; kb < KB; ++kb, ++it) {
             const int s = it % kStages;
@@ -125,14 +129,17 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
 #pragma unroll
                 for (int q = 0; q < 4; ++q) {
                     const int k = kk * 4 + q;
-                    const float4 b0 = *reinterpret_cast<const float4*>(B + k * GN + tx * 4);
-                    const float4 b1 = *reinterpret_cast<const float4*>(B + k * GN + 64 + tx * 4);
-                    const float bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+                    const ulonglong2 b0 = *reinterpret_cast<const ulonglong2*>(B + k * GN + tx * 4);
+                    const ulonglong2 b1 = *reinterpret_cast<const ulonglong2*>(B + k * GN + 64 + tx * 4);
+                    const unsigned long long bp[4] = {b0.x, b0.y, b1.x, b1.y};
 #pragma unroll
                     for (int i = 0; i < 8; ++i) {
                         const float av = q == 0 ? a[i].x : q == 1 ? a[i].y : q == 2 ? a[i].z : a[i].w;
+                        unsigned long long ap;
+                        asm("mov.b64 %0, {%1, %1};" : "=l"(ap) : "f"(av));
 #pragma unroll
-                        for (int j = 0; j < 8; ++j) acc[i][j] = __fmaf_rn(av, bv[j], acc[i][j]);
+                        for (int p = 0; p < 4; ++p)
+                            asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(acc[i][p]) : "l"(ap), "l"(bp[p]));
                     }
                 }
             }
@@ -154,10 +161,10 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                 if (c >= N) continue;
                 float4* dst = reinterpret_cast<float4*>(C + (size_t)r * N + c);
                 float4 o;
-                o.x = alpha * acc[i][h * 4 + 0];
-                o.y = alpha * acc[i][h * 4 + 1];
-                o.z = alpha * acc[i][h * 4 + 2];
-                o.w = alpha * acc[i][h * 4 + 3];
+                o.x = alpha * __uint_as_float((uint32_t)acc[i][h * 2 + 0]);
+                o.y = alpha * __uint_as_float((uint32_t)(acc[i][h * 2 + 0] >> 32));
+                o.z = alpha * __uint_as_float((uint32_t)acc[i][h * 2 + 1]);
+                o.w = alpha * __uint_as_float((uint32_t)(acc[i][h * 2 + 1] >> 32));
                 if (beta != 0.f) {
                     const float4 old = __ldcs(dst);
                     o.x = __fmaf_rn(beta, old.x, o.x);

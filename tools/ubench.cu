@@ -84,7 +84,33 @@ __global__ void k_ffma(float* out, int iters) {
     if (a0 + a1 + a2 + a3 + a4 + a5 + a6 + a7 == 12345.f) out[0] = a0;
 }
 
+// packed FP32 (sm_100: FFMA2 = fma.rn.f32x2): 2 FMAs per lane per instruction
+__global__ void k_ffma2(float* out, int iters) {
+    unsigned long long a0 = threadIdx.x, a1 = a0 + 1, a2 = a0 + 2, a3 = a0 + 3, a4 = a0 + 4, a5 = a0 + 5,
+                       a6 = a0 + 6, a7 = a0 + 7;
+    unsigned long long b = 0x3f7fbe773f7fbe77ull, c = 0x3a83126f3a83126full;
+    asm volatile("" : "+l"(b), "+l"(c));
+    for (int i = 0; i < iters; ++i) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            asm volatile("fma.rn.f32x2 %0, %0, %1, %2;" : "+l"(a0) : "l"(b), "l"(c));
+            asm volatile("fma.rn.f32x2 %0, %0, %1, %2;" : "+l"(a1) : "l"(b), "l"(c));
+            asm volatile("fma.rn.f32x2 %0, %0, %1, %2;" : "+l"(a2) : "l"(b), "l"(c));
+            asm volatile("fma.rn.f32x2 %0, %0, %1, %2;" : "+l"(a3) : "l"(b), "l"(c));
+            asm volatile("fma.rn.f32x2 %0, %0, %1, %2;" : "+l"(a4) : "l"(b), "l"(c));
+            asm volatile("fma.rn.f32x2 %0, %0, %1, %2;" : "+l"(a5) : "l"(b), "l"(c));
+            asm volatile("fma.rn.f32x2 %0, %0, %1, %2;" : "+l"(a6) : "l"(b), "l"(c));
+            asm volatile("fma.rn.f32x2 %0, %0, %1, %2;" : "+l"(a7) : "l"(b), "l"(c));
+        }
+    }
+    if ((a0 ^ a1 ^ a2 ^ a3 ^ a4 ^ a5 ^ a6 ^ a7) == 12345) out[0] = 1.f;
+}
+
 extern "C" {
+int ub_ffma2(float* out, int iters, int grid, int block, void* stream) {
+    k_ffma2<<<grid, block, 0, (cudaStream_t)stream>>>(out, iters);
+    return (int)cudaGetLastError();
+}
 int ub_copy(const void* a, void* b, size_t bytes, int grid, int block, void* stream) {
     k_copy<<<grid, block, 0, (cudaStream_t)stream>>>((const float4*)a, (float4*)b, bytes / 16);
     return (int)cudaGetLastError();
