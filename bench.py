@@ -47,14 +47,20 @@ CONFIG_NAMES = {
 
 # ----------------------------------------------------------------------------- helpers
 def dist_setup():
+    """One process per GPU (torchrun).  SVP_BENCH_DEVICE=<ordinal> pins every rank to one
+    GPU (tests the multi-rank path on a 1-GPU box; the barrier/max-over-ranks then run on
+    gloo because NCCL refuses two ranks on one device)."""
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    forced = os.environ.get("SVP_BENCH_DEVICE")
+    if forced is not None:
+        local = int(forced)
     if ws > 1:
         import torch.distributed as dist
         import torch
-        backend = "nccl" if torch.cuda.is_available() else "gloo"
-        if backend == "nccl":
+        backend = "nccl" if (torch.cuda.is_available() and forced is None) else "gloo"
+        if torch.cuda.is_available():
             torch.cuda.set_device(local)
         dist.init_process_group(backend=backend)
     return rank, ws, local

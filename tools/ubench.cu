@@ -84,6 +84,19 @@ __global__ void k_ffma(float* out, int iters) {
     if (a0 + a1 + a2 + a3 + a4 + a5 + a6 + a7 == 12345.f) out[0] = a0;
 }
 
+__global__ void k_dfma(double* out, int iters) {
+    double a0 = threadIdx.x, a1 = a0 + 1, a2 = a0 + 2, a3 = a0 + 3, a4 = a0 + 4, a5 = a0 + 5, a6 = a0 + 6, a7 = a0 + 7;
+    const double b = 0.999, c = 0.001;
+    for (int i = 0; i < iters; ++i) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            a0 = fma(a0, b, c); a1 = fma(a1, b, c); a2 = fma(a2, b, c); a3 = fma(a3, b, c);
+            a4 = fma(a4, b, c); a5 = fma(a5, b, c); a6 = fma(a6, b, c); a7 = fma(a7, b, c);
+        }
+    }
+    if (a0 + a1 + a2 + a3 + a4 + a5 + a6 + a7 == 12345.0) out[0] = a0;
+}
+
 // packed FP32 (sm_100: FFMA2 = fma.rn.f32x2): 2 FMAs per lane per instruction
 __global__ void k_ffma2(float* out, int iters) {
     unsigned long long a0 = threadIdx.x, a1 = a0 + 1, a2 = a0 + 2, a3 = a0 + 3, a4 = a0 + 4, a5 = a0 + 5,
@@ -107,6 +120,10 @@ __global__ void k_ffma2(float* out, int iters) {
 }
 
 extern "C" {
+int ub_dfma(double* out, int iters, int grid, int block, void* stream) {
+    k_dfma<<<grid, block, 0, (cudaStream_t)stream>>>(out, iters);
+    return (int)cudaGetLastError();
+}
 int ub_ffma2(float* out, int iters, int grid, int block, void* stream) {
     k_ffma2<<<grid, block, 0, (cudaStream_t)stream>>>(out, iters);
     return (int)cudaGetLastError();

@@ -51,6 +51,7 @@ def main():
     L.ub_ffma.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, vp]
     L.ub_atoms16.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, vp]
     L.ub_ffma2.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, vp]
+    L.ub_dfma.argtypes = [vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, vp]
     props = torch.cuda.get_device_properties(0)
     sms = props.multi_processor_count
     st = torch.cuda.current_stream().cuda_stream
@@ -91,6 +92,9 @@ def main():
     res["ffma_tflops"] = sms * 8 * 256 * fi * 64 * 2 / t / 1e12
     t = timed(lambda: L.ub_ffma2(f.data_ptr(), fi, sms * 8, 256, st))
     res["ffma2_tflops"] = sms * 8 * 256 * fi * 64 * 2 * 2 / t / 1e12
+    fd = torch.zeros(1, dtype=torch.float64, device="cuda")
+    t = timed(lambda: L.ub_dfma(fd.data_ptr(), fi // 4, sms * 8, 256, st))
+    res["dfma_tflops"] = sms * 8 * 256 * (fi // 4) * 64 * 2 / t / 1e12
 
     nb = 512 << 20
     h = torch.empty(nb, dtype=torch.uint8, pin_memory=True)
