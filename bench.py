@@ -46,6 +46,11 @@ CONFIG_NAMES = {
 
 
 # ----------------------------------------------------------------------------- helpers
+def trace(msg):
+    if os.environ.get("SVP_BENCH_TRACE"):
+        print(f"[rank {os.environ.get('RANK', '0')}] {time.strftime('%H:%M:%S')} {msg}", file=sys.stderr, flush=True)
+
+
 def dist_setup():
     """One process per GPU (torchrun).  SVP_BENCH_DEVICE=<ordinal> pins every rank to one
     GPU (tests the multi-rank path on a 1-GPU box; the barrier/max-over-ranks then run on
@@ -247,6 +252,7 @@ def run_svp(args, rank, ws, local):
 
     torch.cuda.set_device(local)
     stream = torch.cuda.current_stream()
+    trace("specs")
     all_specs = W.config_specs(args.config, nvps=args.vps)
     specs = my_specs(all_specs, rank, ws)
     t_gen = time.perf_counter()
@@ -255,6 +261,7 @@ def run_svp(args, rank, ws, local):
 
     # ---------------- device-resident run (value)
     impl = svp.SGEMM_3XTF32 if args.sgemm_impl == "3xtf32" else svp.SGEMM_FFMA
+    trace("inputs ready")
     ctx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, external_streams=[stream.cuda_stream],
                       validate_ptrs=True, sgemm_impl=impl)
     vs = VPSet(ctx, specs, inputs, "device", device_ordinals=[local])
@@ -267,6 +274,7 @@ def run_svp(args, rank, ws, local):
         ctx.flush()
     ctx.reset_profile()
     barrier(ws)
+    trace("warmup done, timing")
     clocks = Clocks(local)
     dt = timed_steps(ctx, jobs, args.steps, stream)
     clk = clocks.stop()
@@ -280,6 +288,7 @@ def run_svp(args, rank, ws, local):
     # coalesced launches of different kernels overlap on the compute streams (that is the
     # interleaving gain), so their events overlap too.  Re-run the same jobs on ONE stream
     # (profile_level 1: CUDA events around every launch on its stream) and read the stats.
+    trace("timed region done")
     ictx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, interleave=False,
                        external_streams=[stream.cuda_stream], sgemm_impl=impl)
     for k in vs.kids:
@@ -344,6 +353,7 @@ def run_svp(args, rank, ws, local):
         except Exception:
             pass
 
+    trace("one-stream pass done")
     # ---------------- the other implementation of the fp32 "sgemm" kernel, same jobs
     alt = None
     if not args.no_alt:
@@ -363,6 +373,7 @@ def run_svp(args, rank, ws, local):
                "sgemm_tflops_interleaved": (sk["flops"] / sk["total_ns"] / 1e3) if sk and sk["total_ns"] else None}
         actx.close()
 
+    trace("alt pass done")
     # ---------------- serial baselines on the same GPU, same buffers, same kernels
     serial = {}
     by_kernel = {}
@@ -399,6 +410,7 @@ def run_svp(args, rank, ws, local):
     del vs
     torch.cuda.empty_cache()
 
+    trace("serial passes done")
     # ---------------- e2e: pinned host buffers, copies inside the timed region
     e2e = None
     if not args.no_e2e:
