@@ -436,6 +436,7 @@ def run_svp(args, rank, ws, local):
     if rank == 0 and ws == 1 and not args.no_cpu:
         cpu = cpu_baseline(specs, inputs, CONFIG_NAMES[args.config])
 
+    total_launches = int(sum_over_ranks(launches, ws))  # collective: every rank calls it
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "jobs/s", "n_gpus": ws, "steps": args.steps,
@@ -445,7 +446,7 @@ def run_svp(args, rank, ws, local):
                        "residency": "device (HBM)", "parallelism": f"dp{ws}: VPs sharded by the Job Dispatcher (LPT)",
                        "l2": "inputs > L2: %.1f GB of VP buffers touched per step" %
                              (sum(s.algorithmic_bytes() for s in all_specs) / 1e9)},
-            "clocks": clk, "e2e": e2e, "gpu_launches": int(sum_over_ranks(launches, ws)),
+            "clocks": clk, "e2e": e2e, "gpu_launches": total_launches,
             "roofline": roof, "cpu_baseline": cpu,
             "hbm_gbs_membound": hbm_gbs,
             "hbm_frac_membound": (hbm_gbs / float(peaks["hbm_gbs"])) if hbm_gbs else None,
