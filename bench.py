@@ -262,8 +262,9 @@ def run_svp(args, rank, ws, local):
     # ---------------- device-resident run (value)
     impl = svp.SGEMM_3XTF32 if args.sgemm_impl == "3xtf32" else svp.SGEMM_FFMA
     trace("inputs ready")
+    f4 = dict(hetero=bool(args.hetero), graph=bool(args.graph))  # NEXT f4 options
     ctx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, external_streams=[stream.cuda_stream],
-                      validate_ptrs=True, sgemm_impl=impl)
+                      validate_ptrs=True, sgemm_impl=impl, **f4)
     vs = VPSet(ctx, specs, inputs, "device", device_ordinals=[local])
     jobs = svp.JobBatch(vs.job_list())  # marshalled once; each step resubmits it
     ctx.submit_batch(jobs)
@@ -284,6 +285,9 @@ def run_svp(args, rank, ws, local):
     value = n_jobs_total * args.steps / dt_max
     st = ctx.flush_stats()
     launches = launches_per_flush(ctx) * args.steps
+    main_kstats = {name: ctx.kernel_stats(kid) for name, kid in vs.kids.items()}
+    if args.hetero:
+        main_kstats["ew_mix"] = ctx.kernel_stats(svp.KERNEL_EW_MIX)
     # Per-kernel roofline numbers need each kernel's own duration: in the timed run the
     # coalesced launches of different kernels overlap on the compute streams (that is the
     # interleaving gain), so their events overlap too.  Re-run the same jobs on ONE stream
@@ -380,6 +384,7 @@ def run_svp(args, rank, ws, local):
     if not args.no_serial:
         for name, kw in (("B1_serial_sync", dict(coalesce=False, interleave=False, sync_each_job=True)),
                          ("B2_serial_async", dict(coalesce=False, interleave=False)),
+                         ("B3_serial_graph", dict(coalesce=False, interleave=False, graph=True)),
                          ("B2_profiled", dict(coalesce=False, interleave=False, profile_level=1))):
             sctx = svp.Context(num_gpus=1, device_ids=[local], external_streams=[stream.cuda_stream],
                                sgemm_impl=impl, **kw)
@@ -415,7 +420,7 @@ def run_svp(args, rank, ws, local):
     e2e = None
     if not args.no_e2e:
         hctx = svp.Context(num_gpus=1, device_ids=[local], external_streams=[stream.cuda_stream],
-                           arena_bytes=args.arena_gb << 30, sgemm_impl=impl)
+                           arena_bytes=args.arena_gb << 30, sgemm_impl=impl, **f4)
         hvs = VPSet(hctx, specs, inputs, "host")
         hjobs = svp.JobBatch(hvs.job_list())
         hctx.submit_batch(hjobs)
@@ -451,7 +456,10 @@ def run_svp(args, rank, ws, local):
             "hbm_gbs_membound": hbm_gbs,
             "hbm_frac_membound": (hbm_gbs / float(peaks["hbm_gbs"])) if hbm_gbs else None,
             "elements_per_s": sum(s.n for s in all_specs) * args.steps / dt_max,
-            "sgemm_impl": args.sgemm_impl, "alt_sgemm_impl": alt,
+            "sgemm_impl": args.sgemm_impl, "alt_sgemm_impl": alt, "hetero": args.hetero, "graph": args.graph,
+            "graph_replays_last_step": int(st["graph_replays"]),
+            "timed_kernel_ms_per_step": {n: k["total_ns"] / args.steps / 1e6 for n, k in main_kstats.items()
+                                         if k["launches"]},
             "speedup_vs_serial": {k: value / v["value"] for k, v in serial.items()},
             "serial": serial, "speedup_by_kernel_class": by_kernel, "per_kernel": per_kernel,
             "one_stream": {"value": iso_value, "unit": "jobs/s",
@@ -477,6 +485,10 @@ def main():
     ap.add_argument("--arena-gb", type=int, default=8)
     ap.add_argument("--sgemm-impl", default="3xtf32", choices=["ffma", "3xtf32"],
                     help="implementation of the fp32 'sgemm' kernel (both meet its 1e-5 contract)")
+    ap.add_argument("--hetero", type=int, default=0, choices=[0, 1],
+                    help="heterogeneous coalescing of vecadd/SAXPY/Black-Scholes (NEXT f4)")
+    ap.add_argument("--graph", type=int, default=0, choices=[0, 1],
+                    help="steady-state plan reuse + CUDA graph replay (NEXT f4)")
     ap.add_argument("--no-serial", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other sgemm implementation")
     ap.add_argument("--no-e2e", action="store_true")

@@ -34,7 +34,7 @@
 extern "C" {
 #endif
 
-#define SVP_ABI_VERSION 1
+#define SVP_ABI_VERSION 2
 
 typedef int32_t svp_status;
 enum {
@@ -84,10 +84,20 @@ typedef struct svp_config {
     double pcie_gbps;            /* default 50 per direction                                  */
     double ffma_tflops;          /* default 60                                                */
     double launch_us;            /* default 4                                                 */
+    /* NEXT item f4 (lifts "identical kernels only") */
+    int32_t hetero;              /* 1: heterogeneous coalescing -- the vecadd, SAXPY and
+                                    Black-Scholes groups of one (level, GPU) share ONE launch
+                                    whose segment table names each segment's kernel          */
+    int32_t graph;               /* 1: steady-state replay -- a flush whose requests (VP,
+                                    kernel, args, buffers, in order) equal the previous
+                                    flush's reuses its plan and tables, and from the second
+                                    repeat on replays the flush's device work as one CUDA
+                                    graph per GPU.  Ignored with sync_each_job.              */
 } svp_config;
 
 /* Fill *cfg with defaults: num_gpus 0, 4 compute streams, coalesce 1, interleave 1,
-   max_chunks 8, profile_level 0, validate_ptrs 1, sgemm_impl SVP_SGEMM_3XTF32, rest 0. */
+   max_chunks 8, profile_level 0, validate_ptrs 1, sgemm_impl SVP_SGEMM_3XTF32, rest 0
+   (hetero 0, graph 0). */
 void svp_config_default(svp_config* cfg);
 
 /* Create a context.  On success *out owns streams/events/threads for every GPU.
@@ -260,7 +270,11 @@ svp_status svp_profile(svp_ctx* ctx, int32_t vp, svp_vp_profile* out);
 svp_status svp_reset_profile(svp_ctx* ctx);
 
 /* Aggregate per kernel id (profile_level >= 1): launches, summed event-timed kernel
- * duration (ns), algorithmic bytes and FLOPs of those launches. */
+ * duration (ns), algorithmic bytes and FLOPs of those launches.  `kernel` is a
+ * registered id or SVP_KERNEL_EW_MIX, the heterogeneous elementwise launch that
+ * cfg.hetero forms (its vecadd/SAXPY/Black-Scholes members are counted there, not under
+ * their own ids); plan ops of such a launch also report SVP_KERNEL_EW_MIX. */
+#define SVP_KERNEL_EW_MIX 8
 typedef struct svp_kernel_stats {
     uint64_t launches;
     double total_ns;
@@ -280,6 +294,8 @@ typedef struct svp_flush_stats {
     double device_ns;        /* first-op start to last-op end (profile_level >= 1) */
     double sim_makespan_ns;  /* cost-model makespan of the plan (always)           */
     double sim_serial_ns;    /* cost-model time of the same ops run one at a time  */
+    uint64_t plan_reused;    /* cfg.graph: 1 if the previous flush's plan was reused */
+    uint64_t graph_replays;  /* cfg.graph: GPUs whose work ran as a replayed CUDA graph */
 } svp_flush_stats;
 svp_status svp_flush_stats_get(svp_ctx* ctx, svp_flush_stats* out);
 

@@ -34,12 +34,12 @@ static const KernelDesc kKernels[] = {
 };
 
 const KernelDesc* kernel_desc(int32_t id) {
-    if (id <= 0 || id >= K_COUNT) return nullptr;
+    if (id <= 0 || id >= K_EW_MIX) return nullptr;
     return &kKernels[id];
 }
 const KernelDesc* kernel_by_name(const char* name) {
     if (!name) return nullptr;
-    for (int i = 1; i < K_COUNT; ++i)
+    for (int i = 1; i < K_EW_MIX; ++i)
         if (strcmp(kKernels[i].name, name) == 0) return &kKernels[i];
     return nullptr;
 }
@@ -271,6 +271,22 @@ svp_status svp_submit_batch(svp_ctx* h, int32_t n, const svp_job_desc* jobs, uin
 // One flush of everything queued so far (serialized by flush_mu).  Marks every job id
 // below the snapshot's next id as completed (or failed with the flush's status) and
 // wakes svp_wait callers.
+// Same requests in the same order: VP, kernel, argument bytes and buffer descriptors.
+static bool same_requests(const std::vector<Job>& a, const std::vector<Job>& b) {
+    if (a.size() != b.size() || a.empty()) return false;
+    for (size_t i = 0; i < a.size(); ++i) {
+        const Job &x = a[i], &y = b[i];
+        if (x.vp != y.vp || x.kernel != y.kernel || x.nbufs != y.nbufs || x.device != y.device ||
+            memcmp(x.args, y.args, sizeof(x.args)) != 0)
+            return false;
+        for (int k = 0; k < x.nbufs; ++k)
+            if (x.bufs[k].ptr != y.bufs[k].ptr || x.bufs[k].bytes != y.bufs[k].bytes ||
+                x.bufs[k].dir != y.bufs[k].dir || x.bufs[k].mem != y.bufs[k].mem)
+                return false;
+    }
+    return true;
+}
+
 static svp_status do_flush(Ctx* c) {
     std::lock_guard<std::mutex> flk(c->flush_mu);
     if (c->sticky != SVP_OK) {
@@ -286,11 +302,30 @@ static svp_status do_flush(Ctx* c) {
         upto = c->next_job_id - 1;
     }
     memset(&c->fstats, 0, sizeof(c->fstats));
-    svp_status st = plan_flush(c, &f);
+    svp_status st = SVP_OK;
+    // Steady-state replay (cfg.graph, NEXT f4): the same requests as the previous flush
+    // get the same plan, so copy it (and, in the executor, its tables and CUDA graph).
+    const bool reuse = c->cfg.graph && !c->cfg.sync_each_job && c->last_ok && same_requests(f.jobs, c->last.jobs);
+    if (reuse) {
+        for (size_t i = 0; i < f.jobs.size(); ++i) f.jobs[i].level = c->last.jobs[i].level;
+        f.groups = c->last.groups;
+        f.chunks = c->last.chunks;
+        f.ops = c->last.ops;
+        for (auto& o : f.ops) o.measured_ns = -1;
+        f.levels = c->last.levels;
+        f.plan_gen = c->last.plan_gen;
+        f.reused = true;
+        c->fstats.plan_reused = 1;
+    } else {
+        st = plan_flush(c, &f);
+        f.plan_gen = ++c->plan_gen;
+    }
     auto t1 = std::chrono::steady_clock::now();
     if (st == SVP_OK) {
-        double makespan = 0, serial = 0;
-        simulate(c, &f, &makespan, &serial);
+        double makespan = c->last_sim_makespan, serial = c->last_sim_serial;
+        if (!reuse) simulate(c, &f, &makespan, &serial);
+        c->last_sim_makespan = makespan;
+        c->last_sim_serial = serial;
         c->fstats.sim_makespan_ns = makespan;
         c->fstats.sim_serial_ns = serial;
         c->fstats.host_plan_ns = std::chrono::duration<double, std::nano>(t1 - t0).count();
@@ -319,6 +354,7 @@ static svp_status do_flush(Ctx* c) {
         c->fstats.launches = launches;
     }
     c->last = std::move(f);
+    c->last_ok = st == SVP_OK;
     {
         std::lock_guard<std::mutex> lk(c->done_mu);
         if (st != SVP_OK && upto > c->completed_upto) c->failed.emplace_back(upto, st);
@@ -560,7 +596,7 @@ svp_status svp_kernel_stats_get(svp_ctx* h, int32_t kernel, svp_kernel_stats* ou
         set_error("null argument");
         return SVP_E_INVAL;
     }
-    if (!kernel_desc(kernel)) {
+    if (!kernel_desc(kernel) && kernel != K_EW_MIX) {
         set_error("unknown kernel id");
         return SVP_E_NOKERNEL;
     }

@@ -74,6 +74,12 @@ struct Dev {
     std::unordered_map<MapKey, Maps2, MapKeyHash> map_cache;
     std::string err;
     uint64_t table_uploads = 0;
+    // steady-state replay (cfg.graph): the device work of plan `gexec_gen` as one graph
+    cudaGraphExec_t gexec = nullptr;
+    uint64_t gexec_gen = 0;
+    std::vector<int32_t> g_tstart;      // profiling event slots of each op inside the graph
+    cudaEvent_t fork_ev = nullptr;
+    std::vector<cudaEvent_t> join_ev;
 };
 
 struct Executor {
@@ -95,6 +101,9 @@ static svp_status dev_setup(Dev& d, const svp_config& cfg, void* ext) {
     CK(cudaEventCreateWithFlags(&d.tbl_ev, cudaEventDisableTiming));
     d.end_ev.resize(S + 2);
     for (auto& e : d.end_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    d.join_ev.resize(S + 2);
+    for (auto& e : d.join_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&d.fork_ev, cudaEventDisableTiming));
     d.arena_bytes = cfg.arena_bytes;
     CK(query_limits(&d.lim));
     return SVP_OK;
@@ -107,6 +116,9 @@ static void dev_teardown(Dev& d) {
     for (auto e : d.dep_ev) cudaEventDestroy(e);
     for (auto e : d.t_ev) cudaEventDestroy(e);
     for (auto e : d.end_ev) cudaEventDestroy(e);
+    for (auto e : d.join_ev) cudaEventDestroy(e);
+    if (d.fork_ev) cudaEventDestroy(d.fork_ev);
+    if (d.gexec) cudaGraphExecDestroy(d.gexec);
     if (d.ext_ev) cudaEventDestroy(d.ext_ev);
     if (d.tbl_ev) cudaEventDestroy(d.tbl_ev);
     if (d.arena) cudaFree(d.arena);
@@ -275,23 +287,23 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             ch.table_off = align_up(tbl.size(), 128);
             tbl.resize(ch.table_off + ch.jobs.size() * sizeof(SegDesc));
             SegDesc* seg = reinterpret_cast<SegDesc*>(tbl.data() + ch.table_off);
-            const int T = tile_elems(ch.kernel);
             uint32_t tiles = 0;
             for (size_t k = 0; k < ch.jobs.size(); ++k) {
                 const Job& j = f.jobs[ch.jobs[k]];
+                const int T = tile_elems(j.kernel);  // per segment: K_EW_MIX mixes tile sizes
                 SegDesc s;
                 memset(&s, 0, sizeof(s));
-                int nalign = ch.kernel == K_HIST256 ? 1 : j.nbufs;  // counts need no alignment
+                int nalign = j.kernel == K_HIST256 ? 1 : j.nbufs;  // counts need no alignment
                 uint64_t mis = ch.staged[k * SVP_MAX_BUFS] & 15;
                 bool co = true;
                 for (int b = 0; b < j.nbufs; ++b) {
                     s.ptr[b] = ch.staged[k * SVP_MAX_BUFS + b];
                     if (b < nalign && (s.ptr[b] & 15) != mis) co = false;
                 }
-                int es = elem_size(ch.kernel, 0);
+                int es = elem_size(j.kernel, 0);
                 if (mis % es) co = false;
                 s.n = j.n;
-                s.flags = co ? 0 : SEG_SCALAR;
+                s.flags = (uint16_t)((co ? 0 : SEG_SCALAR) | (j.kernel << SEG_KIND_SHIFT));
                 s.shift = co ? (uint16_t)(mis / es) : 0;
                 s.f[0] = j.f0;
                 s.f[1] = j.f1;
@@ -387,6 +399,9 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
         case K_BLACKSCHOLES:
             return launch_blackscholes((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
                                        grid_of(d.lim.bs_blocks_per_sm), s);
+        case K_EW_MIX:
+            return launch_ew_mix((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
+                                 grid_of(d.lim.mix_blocks_per_sm), s);
         case K_HIST256:
             return launch_hist256((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
                                   grid_of(d.lim.hist_blocks_per_sm), s);
@@ -418,6 +433,12 @@ static bool chunk_needs_launch(const Flush& f, const Chunk& ch) {
     return false;
 }
 
+static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool capturing, std::vector<int>& used,
+                            std::vector<int32_t>& tstart);
+static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool upload, const std::vector<int>& used,
+                                const std::vector<int32_t>& tstart,
+                                std::chrono::steady_clock::time_point t_issue0, double* issue_ns);
+
 static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
     Ctx* c = e->c;
     CK(cudaSetDevice(d.ordinal));
@@ -439,16 +460,19 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             return SVP_E_NOMEM;
         }
     }
-    // ---- tables
+    // ---- tables (a reused plan's chunks already carry theirs, resident since last flush)
     std::vector<uint8_t> tbl;
-    svp_status st = build_tables(e, d, f, tbl);
-    if (st) return st;
+    if (!f.reused) {
+        svp_status st = build_tables(e, d, f, tbl);
+        if (st) return st;
+    }
     auto t_issue0 = std::chrono::steady_clock::now();
     if (d.ext) {
         CK(cudaEventRecord(d.ext_ev, d.ext));
         for (auto s : d.streams) CK(cudaStreamWaitEvent(s, d.ext_ev, 0));
     }
-    bool upload = !tbl.empty() && (tbl.size() != d.tbl_last.size() || memcmp(tbl.data(), d.tbl_last.data(), tbl.size()));
+    bool upload = !f.reused && !tbl.empty() &&
+                  (tbl.size() != d.tbl_last.size() || memcmp(tbl.data(), d.tbl_last.data(), tbl.size()));
     if (upload) {
         if (tbl.size() > d.tbl_cap) {
             if (d.tbl_dev) CK(cudaFree(d.tbl_dev));
@@ -469,10 +493,86 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
         c->fstats.table_uploads += 1;
         c->fstats.table_bytes += d.tbl_last.size();
     }
-    // ---- issue ops in plan order
-    size_t nt = 0;
+    // ---- steady-state replay: second sighting of a plan -> capture, later -> replay
     std::vector<int> used(d.streams.size(), 0);
     std::vector<int32_t> tstart(f.ops.size(), -1);
+    const bool graph = c->cfg.graph && f.reused && !c->cfg.sync_each_job;
+    bool replay = graph && d.gexec && d.gexec_gen == f.plan_gen;
+    bool capturing = false;
+    if (graph && !replay) {
+        if (d.gexec) {
+            CK(cudaGraphExecDestroy(d.gexec));
+            d.gexec = nullptr;
+        }
+        CK(cudaStreamBeginCapture(d.streams[0], cudaStreamCaptureModeThreadLocal));
+        capturing = true;
+        svp_status cs = [&]() -> svp_status {
+            CK(cudaEventRecord(d.fork_ev, d.streams[0]));
+            for (size_t s = 1; s < d.streams.size(); ++s) CK(cudaStreamWaitEvent(d.streams[s], d.fork_ev, 0));
+            return SVP_OK;
+        }();
+        if (cs) {
+            cudaGraph_t g = nullptr;
+            cudaStreamEndCapture(d.streams[0], &g);
+            if (g) cudaGraphDestroy(g);
+            return cs;
+        }
+    }
+    svp_status ist = replay ? SVP_OK : issue_ops(e, d, f, prof, capturing, used, tstart);
+    if (capturing) {
+        // join every stream back into stream 0, close the capture, instantiate
+        svp_status js = ist;
+        for (size_t s = 1; s < d.streams.size() && js == SVP_OK; ++s) {
+            cudaError_t ce = cudaEventRecord(d.join_ev[s], d.streams[s]);
+            if (ce == cudaSuccess) ce = cudaStreamWaitEvent(d.streams[0], d.join_ev[s], 0);
+            if (ce != cudaSuccess) {
+                d.err = std::string("graph join: ") + cudaGetErrorString(ce);
+                js = SVP_E_CUDA;
+            }
+        }
+        cudaGraph_t g = nullptr;
+        cudaError_t ce = cudaStreamEndCapture(d.streams[0], &g);
+        if (js) {
+            if (g) cudaGraphDestroy(g);
+            return js;
+        }
+        if (ce != cudaSuccess) {
+            d.err = std::string("cudaStreamEndCapture: ") + cudaGetErrorString(ce);
+            return SVP_E_CUDA;
+        }
+        ce = cudaGraphInstantiate(&d.gexec, g, 0);
+        cudaGraphDestroy(g);
+        if (ce != cudaSuccess) {
+            d.gexec = nullptr;
+            d.err = std::string("cudaGraphInstantiate: ") + cudaGetErrorString(ce);
+            return SVP_E_CUDA;
+        }
+        d.gexec_gen = f.plan_gen;
+        d.g_tstart = tstart;
+        replay = true;
+    } else if (ist) {
+        return ist;
+    }
+    if (replay) {
+        CK(cudaGraphLaunch(d.gexec, d.streams[0]));
+        tstart = d.g_tstart;
+        std::fill(used.begin(), used.end(), 0);
+        used[0] = 1;
+        std::lock_guard<std::mutex> lk(c->pmu);
+        c->fstats.graph_replays += 1;
+    }
+    return finish_device(e, d, f, prof, upload, used, tstart, t_issue0, issue_ns);
+}
+
+// Enqueue the device's ops in plan order (directly, or into an open stream capture).
+static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool capturing, std::vector<int>& used,
+                            std::vector<int32_t>& tstart) {
+    Ctx* c = e->c;
+    size_t nt = 0;
+    // inside a capture, timing events become event-record nodes of the graph
+    auto rec = [&](cudaEvent_t ev, cudaStream_t s) {
+        return capturing ? cudaEventRecordWithFlags(ev, s, cudaEventRecordExternal) : cudaEventRecord(ev, s);
+    };
     for (size_t i = 0; i < f.ops.size(); ++i) {
         Op& o = f.ops[i];
         if (o.device != d.idx) continue;
@@ -489,7 +589,7 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
                 d.err = "event allocation failed";
                 return SVP_E_CUDA;
             }
-            CK(cudaEventRecord(ev0, s));
+            CK(rec(ev0, s));
             tstart[i] = (int32_t)nt;
         }
         Chunk& ch = f.chunks[o.chunk];
@@ -513,7 +613,7 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             CK(launch_chunk(d, ch, c->cfg.sgemm_impl, s));
         }
         if (prof) {
-            CK(cudaEventRecord(d.t_ev[2 * nt + 1], s));
+            CK(rec(d.t_ev[2 * nt + 1], s));
             ++nt;
         }
         if (o.needs_event) {
@@ -526,6 +626,13 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
         }
         if (c->cfg.sync_each_job && o.last_of_job) CK(cudaStreamSynchronize(s));
     }
+    return SVP_OK;
+}
+
+static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool upload, const std::vector<int>& used,
+                                const std::vector<int32_t>& tstart,
+                                std::chrono::steady_clock::time_point t_issue0, double* issue_ns) {
+    Ctx* c = e->c;
     // ---- join into the external stream, then wait (watchdog)
     std::vector<cudaEvent_t> finals;
     for (size_t s = 0; s < d.streams.size(); ++s) {

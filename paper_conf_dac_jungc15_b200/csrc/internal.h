@@ -28,7 +28,9 @@ enum KernelId : int32_t {
     K_SGEMM = 5,
     K_SGEMM_TF32 = 6,
     K_DGEMM = 7,
-    K_COUNT = 8
+    K_EW_MIX = 8,   // heterogeneous elementwise launch (cfg.hetero, NEXT f4): not registrable,
+                    // appears only as a plan/kernel-stats id (SVP_KERNEL_EW_MIX)
+    K_COUNT = 9
 };
 
 struct KernelDesc {
@@ -40,6 +42,9 @@ struct KernelDesc {
 };
 const KernelDesc* kernel_desc(int32_t id);
 inline bool is_gemm(int32_t k) { return k == K_SGEMM || k == K_SGEMM_TF32 || k == K_DGEMM; }
+// kernels the heterogeneous launch can carry: same CTA shape (256 threads, no shared
+// memory) and the same SegDesc tile mapping
+inline bool is_ew(int32_t k) { return k == K_VECADD || k == K_SAXPY || k == K_BLACKSCHOLES; }
 const KernelDesc* kernel_by_name(const char* name);
 
 // ------------------------------------------------------------------ jobs
@@ -121,6 +126,10 @@ struct Flush {
     std::vector<Chunk> chunks;
     std::vector<Op> ops;            // issue order (per device subsequence is that device's issue order)
     int32_t levels = 0;
+    // steady-state replay (cfg.graph): plan_gen names the plan; reused = this flush's
+    // requests equal the previous flush's, so plan, chunks and tables were copied from it
+    uint64_t plan_gen = 0;
+    bool reused = false;
 };
 
 // ------------------------------------------------------------------ per-VP profile
@@ -147,7 +156,7 @@ struct CostModel {
     double copy_ns = 2000;           // per-copy fixed overhead
     // EMA of measured/predicted ratio per kernel (learned from the profiler)
     double fp64_flops = 30e12;
-    double kscale[K_COUNT] = {1, 1, 1, 1, 1, 1, 1, 1};
+    double kscale[K_COUNT] = {1, 1, 1, 1, 1, 1, 1, 1, 1};
     double kernel_ns(int32_t kernel, double alg_bytes, double flops) const;
     double h2d_ns(uint64_t bytes, int ncopies) const;
     double d2h_ns(uint64_t bytes, int ncopies) const;
@@ -192,6 +201,9 @@ struct Ctx {
 
     // last flush
     Flush last;
+    bool last_ok = false;            // the last flush completed with SVP_OK
+    uint64_t plan_gen = 0;           // bumped for every freshly planned flush
+    double last_sim_makespan = 0, last_sim_serial = 0;
     svp_flush_stats fstats{};
 
     // Profiler

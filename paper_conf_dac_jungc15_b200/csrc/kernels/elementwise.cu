@@ -20,17 +20,15 @@ namespace svp {
 constexpr int kScalarU = 4;  // independent loads per thread in the scalar (ragged) path
 
 // --------------------------------------------------------------------- vecadd
-__global__ void __launch_bounds__(kEwThreads) k_vecadd(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
+__device__ __forceinline__ void vecadd_tile(const SegDesc& sd, uint32_t lt) {
     constexpr int V = kVecaddVec, TILE = kVecaddTile;
-    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
-        const int si = find_seg(segs, nsegs, t);
-        const SegDesc& sd = segs[si];
+    {
         const float* __restrict__ a = reinterpret_cast<const float*>(sd.ptr[0]);
         const float* __restrict__ b = reinterpret_cast<const float*>(sd.ptr[1]);
         float* __restrict__ c = reinterpret_cast<float*>(sd.ptr[2]);
         int64_t e0, e1;
         bool vec;
-        tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, TILE, e0, e1, vec);
+        tile_range(sd.n, sd.shift, sd.flags, lt, TILE, e0, e1, vec);
         if (vec) {
             const float4* a4 = reinterpret_cast<const float4*>(a + e0) + threadIdx.x;
             const float4* b4 = reinterpret_cast<const float4*>(b + e0) + threadIdx.x;
@@ -73,17 +71,15 @@ __global__ void __launch_bounds__(kEwThreads) k_vecadd(const SegDesc* __restrict
 }
 
 // --------------------------------------------------------------------- SAXPY
-__global__ void __launch_bounds__(kEwThreads) k_saxpy(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
+__device__ __forceinline__ void saxpy_tile(const SegDesc& sd, uint32_t lt) {
     constexpr int V = kVecaddVec, TILE = kSaxpyTile;
-    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
-        const int si = find_seg(segs, nsegs, t);
-        const SegDesc& sd = segs[si];
+    {
         const float* __restrict__ x = reinterpret_cast<const float*>(sd.ptr[0]);
         float* __restrict__ y = reinterpret_cast<float*>(sd.ptr[1]);
         const float a = sd.f[0];
         int64_t e0, e1;
         bool vec;
-        tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, TILE, e0, e1, vec);
+        tile_range(sd.n, sd.shift, sd.flags, lt, TILE, e0, e1, vec);
         if (vec) {
             const float4* x4 = reinterpret_cast<const float4*>(x + e0) + threadIdx.x;
             float4* y4 = reinterpret_cast<float4*>(y + e0) + threadIdx.x;
@@ -176,12 +172,9 @@ __device__ __forceinline__ void bs_one(float S, float X, float T, float mu, floa
     put = XexpRT * (1.0f - N2) - S * (1.0f - N1);
 }
 
-__global__ void __launch_bounds__(kEwThreads) k_blackscholes(const SegDesc* __restrict__ segs, int nsegs,
-                                                             uint32_t total) {
+__device__ __forceinline__ void bs_tile(const SegDesc& sd, uint32_t lt) {
     constexpr int V = kBsVec, TILE = kBsTile;
-    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
-        const int si = find_seg(segs, nsegs, t);
-        const SegDesc& sd = segs[si];
+    {
         const float* __restrict__ S = reinterpret_cast<const float*>(sd.ptr[0]);
         const float* __restrict__ X = reinterpret_cast<const float*>(sd.ptr[1]);
         const float* __restrict__ T = reinterpret_cast<const float*>(sd.ptr[2]);
@@ -191,7 +184,7 @@ __global__ void __launch_bounds__(kEwThreads) k_blackscholes(const SegDesc* __re
         const float mu = R + 0.5f * Vol * Vol, mRlog2e = -R * 1.44269504088896340736f;
         int64_t e0, e1;
         bool vec;
-        tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, TILE, e0, e1, vec);
+        tile_range(sd.n, sd.shift, sd.flags, lt, TILE, e0, e1, vec);
         if (vec) {
             const int o = threadIdx.x;
             float4 rs[V], rx[V], rt[V];
@@ -239,6 +232,38 @@ __global__ void __launch_bounds__(kEwThreads) k_blackscholes(const SegDesc* __re
     }
 }
 
+// --------------------------------------------------------------------- kernels
+// Homogeneous coalesced launches: every segment runs the same tile body.
+#define SVP_EW_KERNEL(NAME, BODY)                                                               \
+    __global__ void __launch_bounds__(kEwThreads) NAME(const SegDesc* __restrict__ segs, int nsegs, \
+                                                       uint32_t total) {                        \
+        for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {                              \
+            const SegDesc& sd = segs[find_seg(segs, nsegs, t)];                                 \
+            BODY(sd, t - sd.tile_begin);                                                        \
+        }                                                                                       \
+    }
+SVP_EW_KERNEL(k_vecadd, vecadd_tile)
+SVP_EW_KERNEL(k_saxpy, saxpy_tile)
+SVP_EW_KERNEL(k_blackscholes, bs_tile)
+
+// Heterogeneous coalescing (NEXT f4, cfg.hetero): ONE launch carries the vecadd, SAXPY
+// and Black-Scholes segments of a (level, GPU); each segment's kernel id sits in its
+// flags, each segment keeps its own tile size, and the tile bodies are the ones above, so
+// every element is computed by exactly the same instructions as in its homogeneous launch
+// (results bit-identical).  The branch is uniform per CTA (a tile lies in one segment).
+__global__ void __launch_bounds__(kEwThreads) k_ew_mix(const SegDesc* __restrict__ segs, int nsegs,
+                                                       uint32_t total) {
+    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+        const SegDesc& sd = segs[find_seg(segs, nsegs, t)];
+        const uint32_t lt = t - sd.tile_begin;
+        switch (sd.flags >> SEG_KIND_SHIFT) {
+            case 1: vecadd_tile(sd, lt); break;  // K_VECADD
+            case 2: saxpy_tile(sd, lt); break;   // K_SAXPY
+            default: bs_tile(sd, lt); break;     // K_BLACKSCHOLES
+        }
+    }
+}
+
 // --------------------------------------------------------------------- launchers
 cudaError_t launch_vecadd(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
     k_vecadd<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
@@ -250,6 +275,11 @@ cudaError_t launch_saxpy(const SegDesc* segs, int nsegs, uint32_t total, int gri
 }
 cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
     k_blackscholes<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+    k_ew_mix<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
     return cudaGetLastError();
 }
 
@@ -266,6 +296,9 @@ cudaError_t query_limits(LaunchLimits* out) {
     if (e) return e;
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&out->bs_blocks_per_sm, k_blackscholes, kEwThreads, 0);
     if (e) return e;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&out->mix_blocks_per_sm, k_ew_mix, kEwThreads, 0);
+    if (e) return e;
+    if (out->mix_blocks_per_sm < 1) out->mix_blocks_per_sm = 1;
     e = query_limits_hist(&out->hist_blocks_per_sm);
     if (e) return e;
     e = query_limits_gemm(&out->gemm_blocks_per_sm);

@@ -13,6 +13,7 @@ struct LaunchLimits {
     int num_sms = 148;
     int ew_blocks_per_sm = 8;   // occupancy of the elementwise kernels
     int bs_blocks_per_sm = 4;
+    int mix_blocks_per_sm = 4;
     int hist_blocks_per_sm = 4;
     int gemm_blocks_per_sm = 1;
     int dgemm_blocks_per_sm = 1;
@@ -26,6 +27,8 @@ cudaError_t query_limits(LaunchLimits* out);
 cudaError_t launch_vecadd(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
 cudaError_t launch_saxpy(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
 cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
+// Heterogeneous elementwise launch: segment kernel id in flags >> SEG_KIND_SHIFT.
+cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
 // hist256: zeroes each segment's 256 counters, then accumulates.
 cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
 

@@ -306,19 +306,25 @@ svp_status plan_flush(Ctx* c, Flush* f) {
     std::map<Key, int32_t> gidx;
     std::vector<int32_t> order(f->jobs.size());
     std::iota(order.begin(), order.end(), 0);
+    // NEXT f4 (cfg.hetero): the elementwise kernels of one (level, GPU) match as ONE
+    // heterogeneous group -- "identical kernels only" lifted for the
+    // kernels that share a CTA shape and tile mapping; members stay in VP order.
+    const bool het = c->cfg.hetero != 0;
+    auto mkernel = [&](const Job& j) { return het && is_ew(j.kernel) ? (int32_t)K_EW_MIX : j.kernel; };
     if (coal) {
         std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
             const Job &x = f->jobs[a], &y = f->jobs[b];
-            return std::tie(x.level, x.device, x.kernel, x.shape_key, x.vp) <
-                   std::tie(y.level, y.device, y.kernel, y.shape_key, y.vp);
+            const int32_t kx = mkernel(x), ky = mkernel(y);
+            return std::tie(x.level, x.device, kx, x.shape_key, x.vp) <
+                   std::tie(y.level, y.device, ky, y.shape_key, y.vp);
         });
         for (int32_t ji : order) {
             const Job& j = f->jobs[ji];
-            Key k{j.level, j.device, j.kernel, j.shape_key};
+            Key k{j.level, j.device, mkernel(j), j.shape_key};
             auto it = gidx.find(k);
             if (it == gidx.end()) {
                 Group g;
-                g.kernel = j.kernel;
+                g.kernel = mkernel(j);
                 g.shape_key = j.shape_key;
                 g.level = j.level;
                 g.device = j.device;
@@ -433,7 +439,7 @@ svp_status plan_flush(Ctx* c, Flush* f) {
             if (device_only(ch) && tensor_kernel(ch.kernel)) has_tensor[{ch.level, ch.device}] = true;
         for (auto& ch : f->chunks) {
             if (!device_only(ch) || !has_tensor.count({ch.level, ch.device})) continue;
-            if (ch.kernel == K_VECADD || ch.kernel == K_SAXPY) ch.co_grid = 2;
+            if (ch.kernel == K_VECADD || ch.kernel == K_SAXPY || ch.kernel == K_EW_MIX) ch.co_grid = 2;
             else if (ch.kernel == K_BLACKSCHOLES) ch.co_grid = 3;
         }
     }

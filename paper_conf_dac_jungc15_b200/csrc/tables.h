@@ -19,11 +19,12 @@ struct SegDesc {
     uint32_t tile_begin;  // first tile of this segment in the launch
     uint16_t shift;       // virtual-index shift: elements between the previous 16-B
                           // boundary and ptr[0] (tiles are aligned in address space)
-    uint16_t flags;       // SEG_SCALAR: buffers not co-aligned mod 16 -> scalar path only
+    uint16_t flags;       // SEG_SCALAR: buffers not co-aligned mod 16 -> scalar path only;
+                          // bits 8..15: the segment's kernel id (heterogeneous launch)
     float f[2];           // per-VP scalars (SAXPY a; Black-Scholes R, V)
 };
 static_assert(sizeof(SegDesc) == 64, "SegDesc must be 64 B");
-enum : uint16_t { SEG_SCALAR = 1 };
+enum : uint16_t { SEG_SCALAR = 1, SEG_KIND_SHIFT = 8 };
 
 // Grouped SGEMM: one entry per VP; tensor maps live in a separate 64-B aligned array
 // (2 per VP: A then B).

@@ -24,6 +24,7 @@ DIR_IN, DIR_OUT, DIR_INOUT = 1, 2, 3
 MEM_DEVICE, MEM_HOST_PINNED = 0, 1
 OP_H2D, OP_KERNEL, OP_D2H = 0, 1, 2
 SGEMM_FFMA, SGEMM_3XTF32 = 0, 1
+KERNEL_EW_MIX = 8  # heterogeneous elementwise launch (cfg hetero): plan/kernel-stats id only
 MAX_BUFS, MAX_ARGS = 5, 64
 
 # ABI symbols declared in include/svp.h (tests check every one is exported)
@@ -42,7 +43,8 @@ class svp_config(C.Structure):
                 ("dry_run", C.c_int32), ("flush_timeout_ms", C.c_int32), ("validate_ptrs", C.c_int32),
                 ("sgemm_impl", C.c_int32),
                 ("external_streams", C.POINTER(C.c_void_p)), ("hbm_gbps", C.c_double), ("pcie_gbps", C.c_double),
-                ("ffma_tflops", C.c_double), ("launch_us", C.c_double)]
+                ("ffma_tflops", C.c_double), ("launch_us", C.c_double), ("hetero", C.c_int32),
+                ("graph", C.c_int32)]
 
 
 class svp_buf(C.Structure):
@@ -73,7 +75,8 @@ class svp_flush_stats(C.Structure):
     _fields_ = [(n, C.c_uint64) for n in ("jobs", "groups", "chunks", "launches", "levels", "h2d_bytes",
                                           "d2h_bytes", "table_bytes", "table_uploads")] + \
                [(n, C.c_double) for n in ("host_plan_ns", "host_issue_ns", "host_total_ns", "device_ns",
-                                          "sim_makespan_ns", "sim_serial_ns")]
+                                          "sim_makespan_ns", "sim_serial_ns")] + \
+               [(n, C.c_uint64) for n in ("plan_reused", "graph_replays")]
 
 
 class svp_plan_op(C.Structure):
@@ -223,7 +226,7 @@ class Context:
                  profile_level: int = 0, sync_each_job: bool = False, dry_run: bool = False,
                  flush_timeout_ms: int = 0, validate_ptrs: bool = True, sgemm_impl: int = SGEMM_3XTF32,
                  external_streams: Optional[Sequence[int]] = None, hbm_gbps: float = 0.0, pcie_gbps: float = 0.0,
-                 ffma_tflops: float = 0.0, launch_us: float = 0.0):
+                 ffma_tflops: float = 0.0, launch_us: float = 0.0, hetero: bool = False, graph: bool = False):
         L = load()
         cfg = svp_config()
         L.svp_config_default(C.byref(cfg))
@@ -249,6 +252,7 @@ class Context:
             self._ext = (C.c_void_p * len(external_streams))(*external_streams)
             cfg.external_streams = C.cast(self._ext, C.POINTER(C.c_void_p))
         cfg.hbm_gbps, cfg.pcie_gbps, cfg.ffma_tflops, cfg.launch_us = hbm_gbps, pcie_gbps, ffma_tflops, launch_us
+        cfg.hetero, cfg.graph = int(hetero), int(graph)
         h = C.c_void_p()
         _check(L.svp_init(C.byref(cfg), C.byref(h)))
         self._h = h

@@ -23,7 +23,7 @@ def test_library_exports_every_declared_symbol():
     assert set(declared) == set(svp.EXPORTS), (set(declared) ^ set(svp.EXPORTS))
     for name in declared:
         assert hasattr(L, name), name
-    assert L.svp_abi_version() == 1
+    assert L.svp_abi_version() == 2
 
 
 def test_lib_is_the_in_tree_build():
@@ -161,3 +161,42 @@ def test_lpt_partition_pure():
     assert out == [0, 1, 0, 1]
     with pytest.raises(svp.SvpError):
         svp.lpt_partition([1], [1.0], 0)
+
+
+_STRUCTS = ("svp_config", "svp_buf", "svp_job_desc", "svp_ipc_buf", "svp_vp_profile", "svp_kernel_stats",
+            "svp_flush_stats", "svp_plan_op")
+
+
+def test_ctypes_layouts_match_the_header(tmp_path):
+    """The binding's ctypes mirrors have the C compiler's size and field offsets (a field
+    added to the header but not to svp.py -- or vice versa -- fails here)."""
+    import ctypes
+    import shutil
+    import subprocess
+    if not shutil.which("gcc"):
+        pytest.skip("gcc not available")
+    lines = ["#include <stdio.h>", "#include <stddef.h>", '#include "svp.h"', "int main(void) {"]
+    for name in _STRUCTS:
+        py = getattr(svp, name)
+        lines.append(f'printf("{name} %zu\\n", sizeof({name}));')
+        for f, _ in py._fields_:
+            lines.append(f'printf("{name}.{f} %zu\\n", offsetof({name}, {f}));')
+    lines.append("return 0; }")
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)], check=True)
+    got = dict(l.split() for l in subprocess.run([str(exe)], check=True, capture_output=True, text=True).stdout.splitlines())
+    for name in _STRUCTS:
+        py = getattr(svp, name)
+        assert int(got[name]) == ctypes.sizeof(py), name
+        for f, _ in py._fields_:
+            assert int(got[f"{name}.{f}"]) == getattr(py, f).offset, f"{name}.{f}"
+
+
+def test_ew_mix_id_is_stats_only():
+    with svp.Context(dry_run=True) as c:
+        assert c.kernel_stats(svp.KERNEL_EW_MIX)["launches"] == 0
+        with pytest.raises(svp.SvpError) as e:
+            c.submit(0, svp.KERNEL_EW_MIX, svp.args_vecadd(4), _vecadd_bufs(4))
+        assert e.value.status == svp.SVP_E_NOKERNEL

@@ -239,3 +239,64 @@ def test_job_larger_than_arena_is_nomem():
         with pytest.raises(svp.SvpError) as e:
             c.flush()
         assert e.value.status == svp.SVP_E_NOMEM
+
+
+# ---------------------------------------------------------------- NEXT f4 (host side)
+def test_hetero_merges_elementwise_groups_only():
+    """cfg hetero: vecadd / SAXPY / Black-Scholes of one (level, GPU) form ONE group with
+    kernel id SVP_KERNEL_EW_MIX, members in VP order; hist256 and SGEMM keep their own."""
+    kinds = ("vecadd", "saxpy", "hist256", "blackscholes", "sgemm")
+    with svp.Context(dry_run=True, hetero=True) as c:
+        for vp in range(40):
+            k = kinds[vp % 5]
+            if k == "sgemm":
+                submit(c, vp, k, M=128, N=128, K=64)
+            else:
+                submit(c, vp, k, n=5000 + 911 * vp)
+        c.flush()
+        ops = c.plan()
+        st = c.flush_stats()
+        assert st["groups"] == 3 and st["launches"] == 3
+        by_kernel = {op["kernel"]: op for op in ops}
+        mix = by_kernel[svp.KERNEL_EW_MIX]
+        assert mix["vps"] == sorted(v for v in range(40) if kinds[v % 5] in ("vecadd", "saxpy", "blackscholes"))
+        assert by_kernel[c.kernel_ids["hist256"]]["nvps"] == 8
+        assert by_kernel[c.kernel_ids["sgemm"]]["nvps"] == 8
+
+
+def test_hetero_keeps_program_order_levels():
+    with svp.Context(dry_run=True, hetero=True) as c:
+        for vp in range(6):
+            submit(c, vp, "vecadd", n=1000)
+            submit(c, vp, "saxpy", n=1000)
+        c.flush()
+        ops = c.plan()
+        assert [op["level"] for op in ops] == [0, 1]
+        assert all(op["kernel"] == svp.KERNEL_EW_MIX and op["nvps"] == 6 for op in ops)
+
+
+def test_graph_mode_reuses_identical_plans():
+    """cfg graph: a flush with the same requests as the previous one reuses its plan
+    (same ops, streams, order); any change in the requests replans."""
+    with svp.Context(dry_run=True, graph=True) as c:
+        def round_(n0):
+            for vp in range(12):
+                submit(c, vp, MIX[vp % 4], n=n0 + 100 * vp, mem=svp.MEM_HOST_PINNED)
+            c.flush()
+            return c.plan(), c.flush_stats()
+        p1, s1 = round_(100000)
+        p2, s2 = round_(100000)
+        p3, s3 = round_(100001)
+        assert s1["plan_reused"] == 0 and s2["plan_reused"] == 1 and s3["plan_reused"] == 0
+        strip = lambda p: [{k: v for k, v in op.items() if k != "measured_ns"} for op in p]
+        assert strip(p1) == strip(p2)
+        assert s2["sim_makespan_ns"] == s1["sim_makespan_ns"]
+        assert strip(p3) != strip(p1)
+
+
+def test_graph_mode_off_never_reuses():
+    with svp.Context(dry_run=True) as c:
+        for _ in range(2):
+            submit(c, 0, "vecadd", n=1000)
+            c.flush()
+        assert c.flush_stats()["plan_reused"] == 0
