@@ -45,6 +45,10 @@ CONFIG_NAMES = {
 }
 
 
+IMPL_NAMES = ("ffma", "3xtf32", "tf32bf16")  # svp.SGEMM_FFMA, SGEMM_3XTF32, SGEMM_TF32BF16
+IMPLS = {n: i for i, n in enumerate(IMPL_NAMES)}
+
+
 # ----------------------------------------------------------------------------- helpers
 def trace(msg):
     if os.environ.get("SVP_BENCH_TRACE"):
@@ -260,7 +264,7 @@ def run_svp(args, rank, ws, local):
     t_gen = time.perf_counter() - t_gen
 
     # ---------------- device-resident run (value)
-    impl = svp.SGEMM_3XTF32 if args.sgemm_impl == "3xtf32" else svp.SGEMM_FFMA
+    impl = IMPLS[args.sgemm_impl]
     trace("inputs ready")
     f4 = dict(hetero=bool(args.hetero), graph=bool(args.graph))  # NEXT f4 options
     ctx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, external_streams=[stream.cuda_stream],
@@ -335,6 +339,14 @@ def run_svp(args, rank, ws, local):
                 "peak_source": f"bf16_tflops {bf16:.0f} ({peak_src} burst) x 0.5 (TF32/BF16 nominal) / 3 MMAs per "
                                f"product (3xTF32); achieved counts algorithmic 2MNK flops",
                 "tensor_pipe_tflops": 3 * achieved}
+    elif dom == "sgemm" and impl == svp.SGEMM_TF32BF16:
+        bf16 = float(peaks.get("bf16_tflops", 1590.0))
+        peak = bf16 / 4.0
+        achieved = (dk["flops"] / dk["launches"]) / (dk["total_ns"] / dk["launches"]) / 1e3
+        roof = {"kernel": "sgemm TF32+2xBF16 (k_sgemm_tc<2>, tcgen05 kind::tf32 + kind::f16)", "bound": "tensor",
+                "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak, "traffic": None,
+                "peak_source": f"bf16_tflops {bf16:.0f} ({peak_src} burst) / 4: per product one TF32 MMA (2 BF16 "
+                               f"slots at the nominal 1/2 ratio) + two BF16 MMAs; achieved counts 2MNK flops"}
     elif dom == "sgemm":
         sm_mhz = float(peaks.get("sm_max_mhz", 1965.0))
         peak = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12
@@ -351,7 +363,8 @@ def run_svp(args, rank, ws, local):
     if os.path.exists(prof_path):
         try:
             tr = json.load(open(prof_path))
-            key = dom + ("_3xtf32" if (dom == "sgemm" and impl == svp.SGEMM_3XTF32) else "")
+            key = dom + ({svp.SGEMM_3XTF32: "_3xtf32", svp.SGEMM_TF32BF16: "_tf32bf16"}.get(impl, "")
+                         if dom == "sgemm" else "")
             if key in tr:
                 roof["traffic"] = tr[key]
         except Exception:
@@ -361,7 +374,8 @@ def run_svp(args, rank, ws, local):
     # ---------------- the other implementation of the fp32 "sgemm" kernel, same jobs
     alt = None
     if not args.no_alt:
-        alt_impl = svp.SGEMM_FFMA if impl == svp.SGEMM_3XTF32 else svp.SGEMM_3XTF32
+        alt_impl = IMPLS[args.alt_impl] if args.alt_impl else (
+            svp.SGEMM_FFMA if impl != svp.SGEMM_FFMA else svp.SGEMM_3XTF32)
         actx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, external_streams=[stream.cuda_stream],
                            sgemm_impl=alt_impl)
         for k in vs.kids:
@@ -372,7 +386,7 @@ def run_svp(args, rank, ws, local):
         ks = max(3, args.steps // 5)
         adt = max_over_ranks(timed_steps(actx, jobs, ks, stream), ws)
         sk = actx.kernel_stats(vs.kids["sgemm"]) if "sgemm" in vs.kids else None
-        alt = {"sgemm_impl": "ffma" if alt_impl == svp.SGEMM_FFMA else "3xtf32", "value": n_jobs_total * ks / adt,
+        alt = {"sgemm_impl": {v: k for k, v in IMPLS.items()}[alt_impl], "value": n_jobs_total * ks / adt,
                "unit": "jobs/s", "ms_per_step": adt / ks * 1e3,
                "sgemm_tflops_interleaved": (sk["flops"] / sk["total_ns"] / 1e3) if sk and sk["total_ns"] else None}
         actx.close()
@@ -483,8 +497,10 @@ def main():
     ap.add_argument("--vps", type=int, default=None)
     ap.add_argument("--e2e-steps", type=int, default=0)
     ap.add_argument("--arena-gb", type=int, default=8)
-    ap.add_argument("--sgemm-impl", default="3xtf32", choices=["ffma", "3xtf32"],
-                    help="implementation of the fp32 'sgemm' kernel (both meet its 1e-5 contract)")
+    ap.add_argument("--sgemm-impl", default="3xtf32", choices=list(IMPL_NAMES),
+                    help="implementation of the fp32 'sgemm' kernel (all meet its 1e-5 contract)")
+    ap.add_argument("--alt-impl", default=None, choices=list(IMPL_NAMES),
+                    help="the other sgemm implementation timed beside (default: ffma, or 3xtf32 if --sgemm-impl ffma)")
     ap.add_argument("--hetero", type=int, default=0, choices=[0, 1],
                     help="heterogeneous coalescing of vecadd/SAXPY/Black-Scholes (NEXT f4)")
     ap.add_argument("--graph", type=int, default=0, choices=[0, 1],

@@ -51,9 +51,11 @@ enum {
 typedef struct svp_ctx svp_ctx; /* opaque */
 
 /* ------------------------------------------------------------------ configuration */
-/* Implementation of the fp32 "sgemm" kernel (both meet its 1e-5 fp32 contract). */
+/* Implementation of the fp32 "sgemm" kernel (all meet its 1e-5 fp32 contract). */
 enum { SVP_SGEMM_FFMA = 0,      /* TMA-staged tiles, fp32 FFMA on the CUDA cores          */
-       SVP_SGEMM_3XTF32 = 1 };  /* tcgen05 tensor cores, operands split hi+lo (3 MMAs)     */
+       SVP_SGEMM_3XTF32 = 1,    /* tcgen05 tensor cores, operands split hi+lo (3 TF32 MMAs) */
+       SVP_SGEMM_TF32BF16 = 2 };/* tcgen05: hi*hi as TF32 + the two cross corrections as
+                                   BF16 MMAs (1 TF32 + 2 BF16 MMAs = 2/3 of 3xTF32's time) */
 
 typedef struct svp_config {
     int32_t num_gpus;            /* GPUs to drive; 0 = all visible (dry_run: 0 -> 1)          */
@@ -74,7 +76,7 @@ typedef struct svp_config {
     int32_t flush_timeout_ms;    /* 0 = wait forever; else watchdog -> SVP_E_TIMEOUT          */
     int32_t validate_ptrs;       /* 1: svp_submit checks residency with cudaPointerGetAttributes
                                     (device buffer on the VP's GPU, host buffer pinned)       */
-    int32_t sgemm_impl;          /* SVP_SGEMM_3XTF32 (default, tensor cores) or SVP_SGEMM_FFMA */
+    int32_t sgemm_impl;          /* SVP_SGEMM_3XTF32 (default), SVP_SGEMM_TF32BF16 or SVP_SGEMM_FFMA */
     void* const* external_streams; /* optional [num_gpus] caller cudaStream_t (e.g. torch's
                                     current stream): flush work starts after the work already
                                     queued on it, and it waits for the flush's last op.      */

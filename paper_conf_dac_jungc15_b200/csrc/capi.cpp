@@ -106,7 +106,7 @@ svp_status svp_init(const svp_config* cfg, svp_ctx** out) {
     *out = nullptr;
     if (cfg->num_gpus < 0 || cfg->num_gpus > 64 || cfg->streams_per_gpu < 1 || cfg->streams_per_gpu > 32 ||
         cfg->max_chunks < 1 || cfg->max_chunks > 64 || cfg->profile_level < 0 || cfg->profile_level > 2 ||
-        cfg->flush_timeout_ms < 0 || cfg->sgemm_impl < 0 || cfg->sgemm_impl > 1) {
+        cfg->flush_timeout_ms < 0 || cfg->sgemm_impl < 0 || cfg->sgemm_impl > 2) {
         set_error("svp_init: config value out of range");
         return SVP_E_INVAL;
     }
@@ -119,7 +119,7 @@ svp_status svp_init(const svp_config* cfg, svp_ctx** out) {
     if (cfg->ffma_tflops > 0) c->cost.ffma_flops = cfg->ffma_tflops * 1e12;
     if (cfg->launch_us > 0) c->cost.launch_ns = cfg->launch_us * 1e3;
     if (cfg->arena_bytes == 0) c->cfg.arena_bytes = 2ull << 30;
-    c->cost.sgemm_3xtf32 = cfg->sgemm_impl == SVP_SGEMM_3XTF32;
+    c->cost.sgemm_tc_units = cfg->sgemm_impl == SVP_SGEMM_3XTF32 ? 3 : cfg->sgemm_impl == SVP_SGEMM_TF32BF16 ? 2 : 0;
     if (const char* e = getenv("SVP_COSCHEDULE")) c->coschedule = atoi(e) != 0;
 
     if (cfg->dry_run) {

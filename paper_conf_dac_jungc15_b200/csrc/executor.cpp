@@ -320,7 +320,7 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             ch.nsegs = (int32_t)ch.jobs.size();
         } else {
             // tcgen05 tiles for sgemm_tf32 and for sgemm with the 3xTF32 implementation
-            const int variant = (ch.kernel == K_SGEMM_TF32 || e->c->cfg.sgemm_impl == SVP_SGEMM_3XTF32) ? 1 : 0;
+            const int variant = (ch.kernel == K_SGEMM_TF32 || e->c->cfg.sgemm_impl != SVP_SGEMM_FFMA) ? 1 : 0;
             const int BM = variant ? kTf32BM : kGemmBM, BN = variant ? kTf32BN : kGemmBN;
             ch.maps_off = align_up(tbl.size(), 128);
             size_t nj = ch.jobs.size();
@@ -406,6 +406,9 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
             return launch_hist256((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
                                   grid_of(d.lim.hist_blocks_per_sm), s);
         case K_SGEMM:
+            if (sgemm_impl == SVP_SGEMM_TF32BF16)
+                return launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
+                                             ch.total_tiles, grid_of(1), s);
             if (sgemm_impl == SVP_SGEMM_3XTF32)
                 return launch_sgemm_3xtf32((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
                                            ch.total_tiles, grid_of(1), s);

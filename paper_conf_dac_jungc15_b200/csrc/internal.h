@@ -152,7 +152,8 @@ struct CostModel {
     double ffma_flops = 60e12;
     double tf32_flops = 500e12;
     double launch_ns = 4000;
-    bool sgemm_3xtf32 = false;
+    int sgemm_tc_units = 0;          // "sgemm" on tensor cores: TF32-MMA-equivalents per
+                                     // product (3xTF32: 3, TF32+2xBF16: 2); 0 = FFMA
     double copy_ns = 2000;           // per-copy fixed overhead
     // EMA of measured/predicted ratio per kernel (learned from the profiler)
     double fp64_flops = 30e12;

@@ -21,7 +21,21 @@
 //     tc_probe.py E1); the 32-B-atom layout is the one the hardware accepts (E6).
 // The lo parts (SPLIT 3) are element-wise, so they keep exactly the hi layouts.
 //
-// Roles (1 CTA per SM, persistent static tile walk, 448 threads):
+//  SPLIT = 2  "TF32 + 2xBF16" (sgemm_impl SVP_SGEMM_TF32BF16): the main product A_hi B_hi
+//             stays a kind::tf32 MMA on the raw TMA tiles; the two cross terms only need
+//             ~8 significant bits (they are 2^-10 smaller), so they run as kind::f16 BF16
+//             MMAs on converter-written bf16 tiles: D += bf(A_hi) bf(B_lo) + bf(A_lo) bf(B_hi).
+//             Per 16 k: 2 TF32 + 2 BF16 MMAs (a BF16 K16 MMA costs what a TF32 K8 one does)
+//             = 4 MMA slots instead of 6.  Error per product (|l| < 2^-10 |x|, bf16 rounding
+//             2^-9): 2 (2^-19 + 2^-19) + 2^-20 (dropped lo lo) = 4.5 * 2^-19 ~ 8.6e-6 |a||b|,
+//             inside the 1e-5 (|A||B|)_ij bound (R19); integer inputs stay exact
+//             (lo = 0).  bf16 tiles: A K-major SWIZZLE_NONE (8x16-B core matrices, LBO 128 B
+//             between the two k halves, SBO 256 B between 8-row groups); B MN-major
+//             SWIZZLE_128B (64-n x 8-k atoms, LBO 2 KiB between n atoms, SBO 1 KiB between
+//             k groups).  The converter lane mappings keep every LDS/STS.128 phase on 8
+//             distinct 16-B bank groups.
+//
+// Roles (1 CTA per SM, persistent static tile walk, 448 threads; SPLIT 2 like SPLIT 3):
 //   warp 0        TMA producer: A tile 128x16 + B tile 16x256 (8 boxes) per k-block into an
 //                 operand ring (8 stages for SPLIT 1, 4 for SPLIT 3).
 //   warp 1        TMEM allocator (512 cols = 2 accumulators of 128x256 fp32) + MMA issuer:
@@ -52,7 +66,7 @@ constexpr int kTmemCols = 512;
 
 template <int SPLIT>
 struct Cfg {
-    // stage: A_hi | B_hi [| A_lo | B_lo]
+    // stage: A_hi | B_hi [| A_lo | B_lo]   (SPLIT 2: A | B | bf A_hi | bf A_lo | bf B_hi | bf B_lo)
     static constexpr int kStageBytes = (kTileA + kTileB) * (SPLIT == 1 ? 1 : 2);
     static constexpr int kStages = SPLIT == 1 ? 8 : 4;
     static constexpr size_t kBarOff = (size_t)kStages * kStageBytes;
@@ -69,6 +83,26 @@ __device__ __forceinline__ uint64_t make_desc(uint32_t saddr, uint32_t lbo, uint
 __device__ __forceinline__ uint64_t desc_a(uint32_t saddr) { return make_desc(saddr, 16, 8 * BK * 4, 4); }
 // B: MN-major, SWIZZLE_128B_BASE32B (1): LBO = 32-n block stride, SBO = 4-k group stride
 __device__ __forceinline__ uint64_t desc_b(uint32_t saddr) { return make_desc(saddr, kBBlock, 512, 1); }
+
+// SPLIT 2 bf16 tiles.  A: K-major, no swizzle, [8-row group][k half][8 rows][16 B]
+__device__ __forceinline__ uint64_t desc_a16(uint32_t saddr) { return make_desc(saddr, 128, 256, 0); }
+// B: MN-major, SWIZZLE_128B (2), [64-n atom][8-k group][8 k rows][128 B]
+__device__ __forceinline__ uint64_t desc_b16(uint32_t saddr) { return make_desc(saddr, 2048, 1024, 2); }
+constexpr int kTileA16 = BM * BK * 2;  // 4 KiB
+constexpr int kTileB16 = BK * BN * 2;  // 8 KiB
+
+// kind::f16 instruction descriptor: D f32, A bf16 [7,10)=1, B bf16 [10,13)=1, A K-major,
+// B MN-major, N>>3, M>>4
+constexpr uint32_t kIdescBf16 = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
+                                ((uint32_t)(BM >> 4) << 24);
+__device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accum) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+        "l"(adesc), "l"(bdesc), "r"(kIdescBf16), "r"(accum)
+        : "memory");
+}
 
 // kind::tf32 instruction descriptor: D f32 [4,6)=1, A tf32 [7,10)=2, B tf32 [10,13)=2,
 // A K-major (bit 15 = 0), B MN-major (bit 16 = 1), N>>3 at [17,23), M>>4 at [24,29)
@@ -116,6 +150,27 @@ __device__ __forceinline__ int find_tile_owner(const GemmDesc* __restrict__ d, i
 }
 
 __device__ __forceinline__ float lo_part(float x) { return x - __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
+
+// bf16x2 of (a -> low half, b -> high half), round to nearest even
+__device__ __forceinline__ uint32_t bf2(float a, float b) {
+    uint32_t r;
+    asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
+    return r;
+}
+// 8 consecutive fp32 -> bf16(hi) and bf16(lo), hi = x with the low 13 mantissa bits cleared
+__device__ __forceinline__ void split8(const float4& p, const float4& q, uint4& hb, uint4& lb) {
+    const float x[8] = {p.x, p.y, p.z, p.w, q.x, q.y, q.z, q.w};
+    uint32_t h[4], l[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const float h0 = __uint_as_float(__float_as_uint(x[2 * i]) & 0xFFFFE000u);
+        const float h1 = __uint_as_float(__float_as_uint(x[2 * i + 1]) & 0xFFFFE000u);
+        h[i] = bf2(h0, h1);
+        l[i] = bf2(x[2 * i] - h0, x[2 * i + 1] - h1);
+    }
+    hb = make_uint4(h[0], h[1], h[2], h[3]);
+    lb = make_uint4(l[0], l[1], l[2], l[3]);
+}
 __device__ __forceinline__ float4 lo_part4(float4 x) {
     return make_float4(lo_part(x.x), lo_part(x.y), lo_part(x.z), lo_part(x.w));
 }
@@ -212,7 +267,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                 const int s = it % ST;
                 const uint32_t ph = (it / ST) & 1;
                 mbar_wait(&full[s], ph);
-                if (SPLIT == 3) mbar_wait(&conv[s], ph);
+                if (SPLIT != 1) mbar_wait(&conv[s], ph);
                 tc_fence_after();
                 if (lane == 0) {
                     const uint32_t s_ah = smem_u32(stage(s));
@@ -231,6 +286,13 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                         } else {
                             mma_tf32(tmem_d, ah, bh, acc0);
                         }
+                    }
+                    if (SPLIT == 2) {
+                        // cross terms on the bf16 tiles, K = 16 in one MMA each
+                        const uint32_t a16h = s_bh + kTileB, a16l = a16h + kTileA16;
+                        const uint32_t b16h = a16l + kTileA16, b16l = b16h + kTileB16;
+                        mma_bf16(tmem_d, desc_a16(a16h), desc_b16(b16l), 1u);
+                        mma_bf16(tmem_d, desc_a16(a16l), desc_b16(b16h), 1u);
                     }
                     mma_commit(&empty[s]);
                     if (kb == KB - 1) mma_commit(&acc_full[a]);
@@ -257,6 +319,63 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                     constexpr int NV = (kTileA + kTileB) / 16;  // 1536 float4: A then B, same order
 #pragma unroll
                     for (int i = ct; i < NV; i += kConvThreads) lo[i] = lo_part4(hi[i]);
+                    fence_proxy_async();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&conv[s]);
+                }
+            }
+        } else if (SPLIT == 2) {
+            const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;  // 0..255
+            // A unit (one per thread): row m, k half kc; a phase's 8 lanes = 8 rows, same kc
+            const int am = (ct >> 4) * 8 + (ct & 7), akc = (ct >> 3) & 1;
+            const int asw = (am >> 1) & 3;  // SWIZZLE_64B: 16-B chunk ^= bits [7,9) of the address
+            const int a_rd0 = am * 64 + (((2 * akc) ^ asw) << 4), a_rd1 = am * 64 + (((2 * akc + 1) ^ asw) << 4);
+            const int a_wr = (am >> 3) * 256 + akc * 128 + (am & 7) * 16;
+            // B units (two per thread): k row, 32-n block j, 32-B granule g (8 n); a phase's 8
+            // lanes = 4 granules x 2 adjacent blocks, the first 16-B half read alternates with j
+            int b_rd[2][2], b_wr[2];
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const int u = ct + 256 * r;
+                const int g = u & 3, j = ((u >> 2) & 1) + 2 * ((u >> 3) & 3), k = u >> 5;
+                const int base = j * kBBlock + k * 128 + ((g ^ (k & 3)) << 5);  // SWIZZLE_128B_BASE32B
+                const int h = j & 1;
+                b_rd[r][0] = base + 16 * h;
+                b_rd[r][1] = base + 16 * (h ^ 1);
+                const int c = 4 * (j & 1) + g, k8 = k & 7;  // bf16 SW128 MN-major
+                b_wr[r] = (j >> 1) * 2048 + (k >> 3) * 1024 + k8 * 128 + ((c ^ k8) << 4);
+            }
+            uint32_t it = 0;
+            for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+                const int v = find_tile_owner(descs, n, t);
+                const int KB = (descs[v].K + BK - 1) / BK;
+                for (int kb = 0; kb < KB; ++kb, ++it) {
+                    const int s = it % ST;
+                    const uint32_t ph = (it / ST) & 1;
+                    mbar_wait(&full[s], ph);
+                    uint8_t* sp = stage(s);
+                    uint8_t* a16h = sp + kTileA + kTileB;
+                    uint8_t* a16l = a16h + kTileA16;
+                    uint8_t* b16h = a16l + kTileA16;
+                    uint8_t* b16l = b16h + kTileB16;
+                    {
+                        const float4 p = *reinterpret_cast<const float4*>(sp + a_rd0);
+                        const float4 q = *reinterpret_cast<const float4*>(sp + a_rd1);
+                        uint4 hb, lb;
+                        split8(p, q, hb, lb);
+                        *reinterpret_cast<uint4*>(a16h + a_wr) = hb;
+                        *reinterpret_cast<uint4*>(a16l + a_wr) = lb;
+                    }
+#pragma unroll
+                    for (int r = 0; r < 2; ++r) {
+                        const float4 x0 = *reinterpret_cast<const float4*>(sp + kTileA + b_rd[r][0]);
+                        const float4 x1 = *reinterpret_cast<const float4*>(sp + kTileA + b_rd[r][1]);
+                        const bool sw = (b_rd[r][0] & 16) != 0;  // read the upper half first
+                        uint4 hb, lb;
+                        split8(sw ? x1 : x0, sw ? x0 : x1, hb, lb);
+                        *reinterpret_cast<uint4*>(b16h + b_wr[r]) = hb;
+                        *reinterpret_cast<uint4*>(b16l + b_wr[r]) = lb;
+                    }
                     fence_proxy_async();
                     __syncwarp();
                     if (lane == 0) mbar_arrive(&conv[s]);
@@ -322,14 +441,14 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
     }
 }
 
-static bool g_attr_set[2][64] = {};
+static bool g_attr_set[4][64] = {};
 
 template <int SPLIT>
 static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
                              cudaStream_t s) {
     int dev = 0;
     cudaGetDevice(&dev);
-    const int si = SPLIT == 1 ? 0 : 1;
+    const int si = SPLIT;
     if (dev < 64 && !g_attr_set[si][dev]) {
         cudaError_t e = cudaFuncSetAttribute(k_sgemm_tc<SPLIT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              (int)tc::Cfg<SPLIT>::kSmem);
@@ -344,6 +463,11 @@ static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uin
 cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
                               cudaStream_t s) {
     return launch_tc<1>(descs, n, maps, total, grid, s);
+}
+
+cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
+                                  cudaStream_t s) {
+    return launch_tc<2>(descs, n, maps, total, grid, s);
 }
 
 cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,

@@ -43,6 +43,11 @@ cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, ui
 cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
                                 int grid, cudaStream_t s);
 
+// fp32-accurate grouped SGEMM on tcgen05: A_hi B_hi as one kind::tf32 MMA per 8 k plus the
+// cross terms bf16(A_hi) bf16(B_lo) + bf16(A_lo) bf16(B_hi) as kind::f16 (BF16) MMAs.
+cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
+                                  int grid, cudaStream_t s);
+
 // Grouped fp64 GEMM (the paper's Table 1 matmul), FP64 DFMA with smem tiles.
 cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total_tiles, int grid, cudaStream_t s);
 cudaError_t query_limits_dgemm(int* per_sm);

@@ -33,7 +33,7 @@ namespace svp {
 // ------------------------------------------------------------------ cost model
 double CostModel::kernel_ns(int32_t kernel, double alg_bytes, double flops) const {
     double body;
-    if (kernel == K_SGEMM) body = flops / (sgemm_3xtf32 ? tf32_flops / 3.0 : ffma_flops) * 1e9;
+    if (kernel == K_SGEMM) body = flops / (sgemm_tc_units ? tf32_flops / sgemm_tc_units : ffma_flops) * 1e9;
     else if (kernel == K_DGEMM) body = flops / fp64_flops * 1e9;
     else if (kernel == K_SGEMM_TF32) body = flops / tf32_flops * 1e9;
     else body = alg_bytes / hbm_Bps * 1e9;
@@ -415,7 +415,7 @@ svp_status plan_flush(Ctx* c, Flush* f) {
     // memory-bound kernels first on a small grid (co_grid CTAs/SM) -- measured slower
     // (41.3k), kept as an option for other mixes.
     auto tensor_kernel = [&](int32_t k) {
-        return k == K_SGEMM_TF32 || (k == K_SGEMM && c->cost.sgemm_3xtf32);
+        return k == K_SGEMM_TF32 || (k == K_SGEMM && c->cost.sgemm_tc_units > 0);
     };
     auto device_only = [&](const Chunk& ch) { return ch.t_in == 0 && ch.t_out == 0; };
     std::stable_sort(corder.begin(), corder.end(), [&](int32_t x, int32_t y) {

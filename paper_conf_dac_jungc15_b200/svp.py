@@ -23,7 +23,7 @@ STATUS_NAMES = {0: "SVP_OK", -1: "SVP_E_INVAL", -2: "SVP_E_NOMEM", -3: "SVP_E_CU
 DIR_IN, DIR_OUT, DIR_INOUT = 1, 2, 3
 MEM_DEVICE, MEM_HOST_PINNED = 0, 1
 OP_H2D, OP_KERNEL, OP_D2H = 0, 1, 2
-SGEMM_FFMA, SGEMM_3XTF32 = 0, 1
+SGEMM_FFMA, SGEMM_3XTF32, SGEMM_TF32BF16 = 0, 1, 2
 KERNEL_EW_MIX = 8  # heterogeneous elementwise launch (cfg hetero): plan/kernel-stats id only
 MAX_BUFS, MAX_ARGS = 5, 64
 

@@ -1,5 +1,6 @@
 """tcgen05 SGEMM paths: "sgemm_tf32" (TF32 inputs, tolerance 2e-3) and "sgemm" with the
-3xTF32 implementation (fp32 contract, tolerance 1e-5), against the oracle."""
+3xTF32 and the TF32+2xBF16 implementations (fp32 contract, tolerance 1e-5), against the
+oracle."""
 import dataclasses
 
 import numpy as np
@@ -30,17 +31,21 @@ def test_tf32_config2(int_inputs):
         check_job(s, inp, got, w, sgemm_tol=TF32_TOL)
 
 
+TC_FP32 = [svp.SGEMM_3XTF32, svp.SGEMM_TF32BF16]
+
+
+@pytest.mark.parametrize("impl", TC_FP32)
 @pytest.mark.parametrize("int_inputs", [True, False])
-def test_3xtf32_config2_fp32_tolerance(int_inputs):
+def test_3xtf32_config2_fp32_tolerance(int_inputs, impl):
     specs = W.config_specs(2, sgemm_int=int_inputs)
     inputs = inputs_for(specs)
-    outs, _, st = run_svp(specs, inputs, "device", sgemm_impl=svp.SGEMM_3XTF32)
+    outs, _, st = run_svp(specs, inputs, "device", sgemm_impl=impl)
     want = oracle.run_jobs(specs, inputs)
     for s, inp, got, w in zip(specs, inputs, outs, want):
         check_job(s, inp, got, w)
 
 
-@pytest.mark.parametrize("kernel,impl,tol", [("sgemm_tf32", 0, TF32_TOL), ("sgemm", 1, 1e-5)])
+@pytest.mark.parametrize("kernel,impl,tol", [("sgemm_tf32", 0, TF32_TOL), ("sgemm", 1, 1e-5), ("sgemm", 2, 1e-5)])
 @pytest.mark.parametrize("residency", ["device", "host"])
 def test_tc_ragged_alpha_beta(kernel, impl, tol, residency):
     dims = [(200, 136, 40), (200, 136, 40), (1, 4, 4), (129, 260, 0), (64, 68, 1000), (300, 516, 36)]
@@ -51,13 +56,30 @@ def test_tc_ragged_alpha_beta(kernel, impl, tol, residency):
         check_job(s, inp, got, sgemm_tol=tol)
 
 
-def test_3xtf32_2048_sampled():
+@pytest.mark.parametrize("impl", TC_FP32)
+def test_3xtf32_2048_sampled(impl):
     """Full BASELINE cfg5 SGEMM shape (2048^3), 4 VPs coalesced, 64 sampled outputs each."""
     specs = [W.JobSpec(v, "sgemm", M=2048, N=2048, K=2048) for v in range(4)]
     inputs = inputs_for(specs)
-    outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=svp.SGEMM_3XTF32)
+    outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl)
     g = np.random.default_rng(1)
     for s, inp, got in zip(specs, inputs, outs):
         sample = [(int(g.integers(0, 2048)), int(g.integers(0, 2048))) for _ in range(64)]
         sample += [(0, 0), (2047, 2047), (127, 255), (128, 256)]
         check_job(s, inp, got, sample=sample)
+
+
+@pytest.mark.parametrize("impl", TC_FP32)
+def test_split_wide_dynamic_range(impl):
+    """Entries spread over 2^-40..2^40: the hi/lo splits are relative per element, so the
+    componentwise bound (|A||B|)_ij still holds (no shared exponent, no range scaling)."""
+    g = np.random.default_rng(7)
+    specs = [W.JobSpec(v, "sgemm", M=256, N=256, K=128) for v in range(2)]
+    inputs = inputs_for(specs)
+    for inp in inputs:
+        for k in ("A", "B"):
+            x = inp[k]
+            inp[k] = (x * np.exp2(g.integers(-40, 41, size=x.shape))).astype(np.float32)
+    outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl)
+    for s, inp, got in zip(specs, inputs, outs):
+        check_job(s, inp, got)
