@@ -321,7 +321,8 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
         } else {
             // tcgen05 tiles for sgemm_tf32 and for sgemm with the 3xTF32 implementation
             const int variant = (ch.kernel == K_SGEMM_TF32 || e->c->cfg.sgemm_impl != SVP_SGEMM_FFMA) ? 1 : 0;
-            const int BM = variant ? kTf32BM : kGemmBM, BN = variant ? kTf32BN : kGemmBN;
+            const bool pair = variant && ch.kernel == K_SGEMM && sgemm_tc_cta_pair();
+            const int BM = variant ? (pair ? 2 * kTf32BM : kTf32BM) : kGemmBM, BN = variant ? kTf32BN : kGemmBN;
             ch.maps_off = align_up(tbl.size(), 128);
             size_t nj = ch.jobs.size();
             ch.table_off = ch.maps_off + nj * 256;

@@ -5,22 +5,12 @@
 //
 //  SPLIT = 1  "sgemm_tf32": one kind::tf32 MMA per k-step; the tensor core reads fp32
 //             operands as TF32 (low 13 mantissa bits ignored).  Own tolerance 2e-3.
-//  SPLIT = 3  "3xTF32" (the fp32 "sgemm" on tensor cores): x = hi + lo, hi = x with the
-//             low 13 bits cleared (exactly what the tensor core reads from x) and
-//             lo = x - hi (exact in fp32); per k-step D += A_hi B_lo + A_lo B_hi + A_hi B_hi.
-//             The dropped A_lo B_lo and the truncation of lo are each < 2^-20 |a||b|, so
-//             the product error is < 3 * 2^-20 |a||b| ~ 2.9e-6 |a||b|, inside the fp32 bound
+//  SPLIT = 3  "3xTF32" (sgemm_impl SVP_SGEMM_3XTF32): x = hi + lo, hi = x with the low 13
+//             bits cleared (exactly what the tensor core reads from x) and lo = x - hi
+//             (exact in fp32); per k-step D += A_hi B_lo + A_lo B_hi + A_hi B_hi.  The
+//             dropped A_lo B_lo and the truncation of lo are each < 2^-20 |a||b|, so the
+//             product error is < 3 * 2^-20 |a||b| ~ 2.9e-6 |a||b|, inside the fp32 bound
 //             1e-5 (|A||B|)_ij (R10).
-//
-// Operand layouts in shared memory (both written by TMA, no transposition):
-//   A (row-major M x K = K-major): 64-B rows of 16 k, SWIZZLE_64B (8-row atoms, SBO 512).
-//   B (row-major K x N = MN-major): 32-n x 16-k blocks of 128-B rows with the 32-B-atom
-//     128-B swizzle (TMA CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B = UMMA SWIZZLE_128B_BASE32B;
-//     LBO = 2 KiB between 32-n blocks, SBO = 512 B between 4-k groups).  A tf32 MMA with an
-//     MN-major B in the plain 16-B-atom SW128 layout reads zeros on B200 (scripts/
-//     tc_probe.py E1); the 32-B-atom layout is the one the hardware accepts (E6).
-// The lo parts (SPLIT 3) are element-wise, so they keep exactly the hi layouts.
-//
 //  SPLIT = 2  "TF32 + 2xBF16" (sgemm_impl SVP_SGEMM_TF32BF16): the main product A_hi B_hi
 //             stays a kind::tf32 MMA on the raw TMA tiles; the two cross terms only need
 //             ~8 significant bits (they are 2^-10 smaller), so they run as kind::f16 BF16
@@ -29,24 +19,43 @@
 //             = 4 MMA slots instead of 6.  Error per product (|l| < 2^-10 |x|, bf16 rounding
 //             2^-9): 2 (2^-19 + 2^-19) + 2^-20 (dropped lo lo) = 4.5 * 2^-19 ~ 8.6e-6 |a||b|,
 //             inside the 1e-5 (|A||B|)_ij bound (R19); integer inputs stay exact
-//             (lo = 0).  bf16 tiles: A K-major SWIZZLE_NONE (8x16-B core matrices, LBO 128 B
-//             between the two k halves, SBO 256 B between 8-row groups); B MN-major
-//             SWIZZLE_128B (64-n x 8-k atoms, LBO 2 KiB between n atoms, SBO 1 KiB between
-//             k groups).  The converter lane mappings keep every LDS/STS.128 phase on 8
-//             distinct 16-B bank groups.
+//             (lo = 0).
 //
-// Roles (1 CTA per SM, persistent static tile walk, 448 threads; SPLIT 2 like SPLIT 3):
-//   warp 0        TMA producer: A tile 128x16 + B tile 16x256 (8 boxes) per k-block into an
-//                 operand ring (8 stages for SPLIT 1, 4 for SPLIT 3).
-//   warp 1        TMEM allocator (512 cols = 2 accumulators of 128x256 fp32) + MMA issuer:
-//                 one lane issues tcgen05.mma.cta_group::1.kind::tf32 M128 N256 K8 and
-//                 tcgen05.commit's to the stage's empty barrier / the accumulator barrier.
-//   warps 2,3,8-13 converters (SPLIT 3): A_lo, B_lo element-wise, fence.proxy.async,
-//                 arrive on the stage's conv barrier.
+// CG = 2 (CTA pair, cta_group::2; SPLIT 2 and 3): a cluster of 2 CTAs on one TPC computes a
+// 256 x 256 tile with M256 N256 MMAs issued by the leader CTA.  Each CTA stages its own
+// 128 rows of A and 128 columns of B (half the operand bytes per SM: the per-SM shared-
+// memory traffic -- TMA writes + converter reads/writes -- is what bounds the single-CTA
+// split kernels, profiles/r01), holds 128 rows x 256 columns of the accumulator in its
+// own TMEM, and runs its own converters and epilogue.  Cross-CTA signalling: converters
+// arrive on the leader's conv barrier (mbarrier.arrive.release.cluster), the leader's
+// commits multicast to both CTAs' empty / acc_full barriers, the peer's epilogue arrives on
+// the leader's acc_empty.
+//
+// Operand layouts in shared memory:
+//   A (row-major M x K = K-major, TMA): 64-B rows of 16 k, SWIZZLE_64B (SBO 512).
+//   B (row-major K x N = MN-major, TMA): 32-n x 16-k blocks of 128-B rows with the 32-B-atom
+//     128-B swizzle (TMA CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B = UMMA SWIZZLE_128B_BASE32B;
+//     LBO = 2 KiB between 32-n blocks, SBO = 512 B between 4-k groups).  A tf32 MMA with an
+//     MN-major B in the plain 16-B-atom SW128 layout reads zeros on B200 (scripts/
+//     tc_probe.py E1); the 32-B-atom layout is the one the hardware accepts (E6).
+//   SPLIT 3 lo tiles: element-wise, same layouts as hi.
+//   SPLIT 2 bf16 tiles: A K-major SWIZZLE_NONE (8x16-B core matrices, LBO 128 B between the
+//     two k halves, SBO 256 B between 8-row groups); B MN-major SWIZZLE_128B (64-n x 8-k
+//     atoms, LBO 2 KiB between n atoms, SBO 1 KiB between k groups).  The converter lane
+//     mappings keep every LDS/STS.128 on the minimum 4 wavefronts (ncu: 0 excessive).
+//
+// Roles (persistent static tile walk, 448 threads per CTA):
+//   warp 0        TMA producer: A 128x16 + B 16x(256/CG) per k-block into the operand ring.
+//   warp 1        TMEM allocator (512 cols = 2 accumulators of 128x256 fp32) + MMA issuer
+//                 (leader CTA only for CG 2): tcgen05.mma ... commit to empty / acc_full.
+//   warps 2,3,8-13 converters (SPLIT 2/3), fence.proxy.async, arrive on conv.
 //   warps 4-7     epilogue: tcgen05.ld 32x32b.x32 (warp w%4 owns TMEM lanes = tile rows
-//                 32(w%4)..+31), alpha*acc (+ beta*C), 128-bit stores; the two TMEM
+//                 32(w%4)..+31), alpha*acc (+ beta*C), 128-bit stores; two TMEM
 //                 accumulators let tile i's epilogue overlap tile i+1's MMAs.
 #include <cuda.h>
+#include <stdlib.h>
+
+#include <algorithm>
 
 #include "../launch.h"
 #include "common.cuh"
@@ -55,22 +64,27 @@ namespace svp {
 
 namespace tc {
 
-constexpr int BM = kTf32BM, BN = kTf32BN, BK = kTf32BK;  // 128 x 256 x 16
+constexpr int BM = kTf32BM, BN = kTf32BN, BK = kTf32BK;  // 128 x 256 x 16 per CTA
 constexpr int kConvWarps = 8;                              // warps 2,3 and 8..13
 constexpr int kConvThreads = kConvWarps * 32;
 constexpr int kThreads = (8 + kConvWarps - 2) * 32;        // 448
 constexpr int kTileA = BM * BK * 4;                        // 8 KiB
-constexpr int kTileB = BK * BN * 4;                        // 16 KiB
 constexpr int kBBlock = BK * 128;                          // one 32-n block of B: 2 KiB
 constexpr int kTmemCols = 512;
+constexpr int kTileA16 = BM * BK * 2;                      // 4 KiB
 
-template <int SPLIT>
+template <int SPLIT, int CG>
 struct Cfg {
-    // stage: A_hi | B_hi [| A_lo | B_lo]   (SPLIT 2: A | B | bf A_hi | bf A_lo | bf B_hi | bf B_lo)
+    static constexpr int kBN = BN / CG;                    // B columns staged per CTA
+    static constexpr int kTileB = BK * kBN * 4;            // 16 KiB (CG 1) / 8 KiB (CG 2)
+    static constexpr int kTileB16 = BK * kBN * 2;
+    // stage: A | B [| A_lo | B_lo]   (SPLIT 2: A | B | bf A_hi | bf A_lo | bf B_hi | bf B_lo)
     static constexpr int kStageBytes = (kTileA + kTileB) * (SPLIT == 1 ? 1 : 2);
-    static constexpr int kStages = SPLIT == 1 ? 8 : 4;
+    static constexpr int kStages = SPLIT == 1 ? 8 : (CG == 2 ? 6 : 4);
     static constexpr size_t kBarOff = (size_t)kStages * kStageBytes;
     static constexpr size_t kSmem = 1024 + kBarOff + 256;
+    static constexpr int kMmaM = BM * CG;
+    static_assert(kSmem <= 227 * 1024, "shared memory");
 };
 
 // SM100 shared-memory matrix descriptor: start>>4 [0,14), LBO>>4 [16,30), SBO>>4 [32,46),
@@ -83,47 +97,102 @@ __device__ __forceinline__ uint64_t make_desc(uint32_t saddr, uint32_t lbo, uint
 __device__ __forceinline__ uint64_t desc_a(uint32_t saddr) { return make_desc(saddr, 16, 8 * BK * 4, 4); }
 // B: MN-major, SWIZZLE_128B_BASE32B (1): LBO = 32-n block stride, SBO = 4-k group stride
 __device__ __forceinline__ uint64_t desc_b(uint32_t saddr) { return make_desc(saddr, kBBlock, 512, 1); }
-
 // SPLIT 2 bf16 tiles.  A: K-major, no swizzle, [8-row group][k half][8 rows][16 B]
 __device__ __forceinline__ uint64_t desc_a16(uint32_t saddr) { return make_desc(saddr, 128, 256, 0); }
 // B: MN-major, SWIZZLE_128B (2), [64-n atom][8-k group][8 k rows][128 B]
 __device__ __forceinline__ uint64_t desc_b16(uint32_t saddr) { return make_desc(saddr, 2048, 1024, 2); }
-constexpr int kTileA16 = BM * BK * 2;  // 4 KiB
-constexpr int kTileB16 = BK * BN * 2;  // 8 KiB
 
-// kind::f16 instruction descriptor: D f32, A bf16 [7,10)=1, B bf16 [10,13)=1, A K-major,
-// B MN-major, N>>3, M>>4
-constexpr uint32_t kIdescBf16 = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
-                                ((uint32_t)(BM >> 4) << 24);
-__device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accum) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "setp.ne.b32 p, %4, 0;\n\t"
-        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
-        "l"(adesc), "l"(bdesc), "r"(kIdescBf16), "r"(accum)
-        : "memory");
-}
+// instruction descriptors: D f32 [4,6)=1, A/B format [7,10)/[10,13) (kind::tf32: TF32 = 2;
+// kind::f16: BF16 = 1), A K-major (bit 15 = 0), B MN-major (bit 16 = 1), N>>3 at [17,23),
+// M>>4 at [24,29)
+template <int M>
+struct Idesc {
+    static constexpr uint32_t tf32 = (1u << 4) | (2u << 7) | (2u << 10) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
+                                     ((uint32_t)(M >> 4) << 24);
+    static constexpr uint32_t bf16 = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
+                                     ((uint32_t)(M >> 4) << 24);
+};
 
-// kind::tf32 instruction descriptor: D f32 [4,6)=1, A tf32 [7,10)=2, B tf32 [10,13)=2,
-// A K-major (bit 15 = 0), B MN-major (bit 16 = 1), N>>3 at [17,23), M>>4 at [24,29)
-constexpr uint32_t kIdesc = (1u << 4) | (2u << 7) | (2u << 10) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
-                            ((uint32_t)(BM >> 4) << 24);
-
+template <int CG>
 __device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accum) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "setp.ne.b32 p, %4, 0;\n\t"
-        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
-        "l"(adesc), "l"(bdesc), "r"(kIdesc), "r"(accum)
-        : "memory");
+    if constexpr (CG == 1)
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+            "l"(adesc), "l"(bdesc), "r"(Idesc<BM>::tf32), "r"(accum)
+            : "memory");
+    else
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+            "l"(adesc), "l"(bdesc), "r"(Idesc<2 * BM>::tf32), "r"(accum)
+            : "memory");
 }
+template <int CG>
+__device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accum) {
+    if constexpr (CG == 1)
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+            "l"(adesc), "l"(bdesc), "r"(Idesc<BM>::bf16), "r"(accum)
+            : "memory");
+    else
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+            "l"(adesc), "l"(bdesc), "r"(Idesc<2 * BM>::bf16), "r"(accum)
+            : "memory");
+}
+// MMA completion -> mbarrier (CG 2: the same barrier offset in both CTAs of the pair)
+template <int CG>
 __device__ __forceinline__ void mma_commit(uint64_t* bar) {
-    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
-                 : "memory");
+    if constexpr (CG == 1)
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                         smem_u32(bar))
+                     : "memory");
+    else
+        asm volatile(
+            "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+                smem_u32(bar)),
+            "h"((uint16_t)3)
+            : "memory");
 }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+// ---- cluster helpers (CTA pair)
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// shared::cluster address of `p` (a local shared variable) in CTA `rank` of the cluster
+__device__ __forceinline__ uint32_t map_to(const void* p, uint32_t rank) {
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(smem_u32(p)), "r"(rank));
+    return r;
+}
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+// wait that also acquires arrivals released by the peer CTA
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
+    const uint32_t a = smem_u32(bar);
+    uint32_t ok = 0;
+    while (!ok) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(ok)
+            : "r"(a), "r"(parity)
+            : "memory");
+    }
+}
 
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
     asm volatile(
@@ -150,6 +219,9 @@ __device__ __forceinline__ int find_tile_owner(const GemmDesc* __restrict__ d, i
 }
 
 __device__ __forceinline__ float lo_part(float x) { return x - __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
+__device__ __forceinline__ float4 lo_part4(float4 x) {
+    return make_float4(lo_part(x.x), lo_part(x.y), lo_part(x.z), lo_part(x.w));
+}
 
 // bf16x2 of (a -> low half, b -> high half), round to nearest even
 __device__ __forceinline__ uint32_t bf2(float a, float b) {
@@ -171,51 +243,62 @@ __device__ __forceinline__ void split8(const float4& p, const float4& q, uint4& 
     hb = make_uint4(h[0], h[1], h[2], h[3]);
     lb = make_uint4(l[0], l[1], l[2], l[3]);
 }
-__device__ __forceinline__ float4 lo_part4(float4 x) {
-    return make_float4(lo_part(x.x), lo_part(x.y), lo_part(x.z), lo_part(x.w));
-}
 
 }  // namespace tc
 
-template <int SPLIT>
+template <int SPLIT, int CG>
 __global__ void __launch_bounds__(tc::kThreads, 1)
     k_sgemm_tc(const GemmDesc* __restrict__ descs, int n, const uint8_t* __restrict__ maps, uint32_t total) {
     using namespace tc;
-    using C = Cfg<SPLIT>;
-    constexpr int ST = C::kStages, SB = C::kStageBytes;
+    using C = Cfg<SPLIT, CG>;
+    constexpr int ST = C::kStages, SB = C::kStageBytes, TB = C::kTileB, TB16 = C::kTileB16;
     extern __shared__ uint8_t smem_raw[];
     // align to 1024 B (swizzle atoms) by offsetting smem_raw itself, so the compiler keeps
-    // the shared address space and emits LDS/STS (not generic LD/ST) for the converters
+    // the shared address space and emits LDS/STS (not generic LD/ST) for the converters;
+    // both CTAs of a pair get the same offsets (the leader's descriptors address both)
     uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::kBarOff);
-    uint64_t* full = bars;               // [ST] TMA A + B landed
+    uint64_t* full = bars;               // [ST] this CTA's TMA A + B landed
     uint64_t* empty = bars + ST;         // [ST] MMAs done with the stage
-    uint64_t* conv = bars + 2 * ST;      // [ST] lo parts written (SPLIT 3)
+    uint64_t* conv = bars + 2 * ST;      // [ST] (leader) both CTAs' converted tiles written
     uint64_t* acc_full = bars + 3 * ST;  // [2]
-    uint64_t* acc_empty = acc_full + 2;  // [2]
+    uint64_t* acc_empty = acc_full + 2;  // [2] (leader) both CTAs' epilogues drained it
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_empty + 2);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t rank = CG == 2 ? cluster_rank() : 0;
+    const bool leader = rank == 0;
+    const uint32_t cl = blockIdx.x / CG, ncl = gridDim.x / CG;  // tile walk per CTA pair
     if (threadIdx.x == 0) {
         for (int s = 0; s < ST; ++s) {
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], 1);
-            mbar_init(&conv[s], kConvWarps);
+            mbar_init(&conv[s], kConvWarps * CG);
         }
         for (int a = 0; a < 2; ++a) {
             mbar_init(&acc_full[a], 1);
-            mbar_init(&acc_empty[a], 4);
+            mbar_init(&acc_empty[a], 4 * CG);
         }
         mbar_fence_init();
     }
     if (warp == 1) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                     "n"(kTmemCols)
-                     : "memory");
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+        if constexpr (CG == 1) {
+            asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                             smem_u32(tmem_slot)),
+                         "n"(kTmemCols)
+                         : "memory");
+            asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+        } else {
+            asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                             smem_u32(tmem_slot)),
+                         "n"(kTmemCols)
+                         : "memory");
+            asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+        }
     }
     tc_fence_before();
     __syncthreads();
+    if constexpr (CG == 2) cluster_sync_all();  // peer barriers initialised before any remote arrive
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
@@ -226,7 +309,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
         if (lane == 0) {
             uint32_t it = 0;
             int last = -1;
-            for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+            for (uint32_t t = cl; t < total; t += ncl) {
                 const int v = find_tile_owner(descs, n, t);
                 const GemmDesc& g = descs[v];
                 const void* mA = maps + (size_t)v * 256;
@@ -238,76 +321,100 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                 }
                 const uint32_t lt = t - g.tile_begin;
                 const int tm = lt / g.tiles_n, tn = lt % g.tiles_n;
+                const int m0 = tm * C::kMmaM + (int)rank * BM, n0 = tn * BN + (int)rank * C::kBN;
                 const int KB = (g.K + BK - 1) / BK;
                 for (int kb = 0; kb < KB; ++kb, ++it) {
                     const int s = it % ST;
                     const uint32_t ph = (it / ST) & 1;
                     mbar_wait(&empty[s], ph ^ 1);
                     uint8_t* sp = stage(s);
-                    mbar_expect_tx(&full[s], kTileA + kTileB);
-                    tma_load_2d(sp, mA, kb * BK, tm * BM, &full[s]);
+                    mbar_expect_tx(&full[s], kTileA + TB);
+                    tma_load_2d(sp, mA, kb * BK, m0, &full[s]);
 #pragma unroll
-                    for (int j = 0; j < BN / 32; ++j)
-                        tma_load_2d(sp + kTileA + j * kBBlock, mB, tn * BN + j * 32, kb * BK, &full[s]);
+                    for (int j = 0; j < C::kBN / 32; ++j)
+                        tma_load_2d(sp + kTileA + j * kBBlock, mB, n0 + j * 32, kb * BK, &full[s]);
                 }
             }
         }
     } else if (warp == 1) {
         // ------------------------------------------------------------ MMA issuer
-        uint32_t it = 0, tile_i = 0;
-        for (uint32_t t = blockIdx.x; t < total; t += gridDim.x, ++tile_i) {
-            const int v = find_tile_owner(descs, n, t);
-            const int KB = (descs[v].K + BK - 1) / BK;
-            const int a = tile_i & 1;
-            const uint32_t aph = (tile_i >> 1) & 1;
-            mbar_wait(&acc_empty[a], aph ^ 1);
-            tc_fence_after();
-            const uint32_t tmem_d = tmem_base + (uint32_t)(a * BN);
-            for (int kb = 0; kb < KB; ++kb, ++it) {
-                const int s = it % ST;
-                const uint32_t ph = (it / ST) & 1;
-                mbar_wait(&full[s], ph);
-                if (SPLIT != 1) mbar_wait(&conv[s], ph);
+        if (leader) {
+            uint32_t it = 0, tile_i = 0;
+            for (uint32_t t = cl; t < total; t += ncl, ++tile_i) {
+                const int v = find_tile_owner(descs, n, t);
+                const int KB = (descs[v].K + BK - 1) / BK;
+                const int a = tile_i & 1;
+                const uint32_t aph = (tile_i >> 1) & 1;
+                if constexpr (CG == 2) mbar_wait_cluster(&acc_empty[a], aph ^ 1);
+                else mbar_wait(&acc_empty[a], aph ^ 1);
                 tc_fence_after();
-                if (lane == 0) {
-                    const uint32_t s_ah = smem_u32(stage(s));
-                    const uint32_t s_bh = s_ah + kTileA;
-                    const uint32_t s_al = s_bh + kTileB;
-                    const uint32_t s_bl = s_al + kTileA;
+                const uint32_t tmem_d = tmem_base + (uint32_t)(a * BN);
+                for (int kb = 0; kb < KB; ++kb, ++it) {
+                    const int s = it % ST;
+                    const uint32_t ph = (it / ST) & 1;
+                    if constexpr (CG == 2) {
+                        mbar_wait_cluster(&conv[s], ph);  // implies both CTAs' TMA data landed
+                    } else {
+                        mbar_wait(&full[s], ph);
+                        if (SPLIT != 1) mbar_wait(&conv[s], ph);
+                    }
+                    tc_fence_after();
+                    if (lane == 0) {
+                        const uint32_t s_ah = smem_u32(stage(s));
+                        const uint32_t s_bh = s_ah + kTileA;
+                        const uint32_t s_al = s_bh + TB;
+                        const uint32_t s_bl = s_al + kTileA;
 #pragma unroll
-                    for (int kk = 0; kk < BK / 8; ++kk) {
-                        const uint64_t ah = desc_a(s_ah + kk * 32);   // +8 k in a 64-B row
-                        const uint64_t bh = desc_b(s_bh + kk * 1024); // +8 k rows of 128 B
-                        const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
-                        if (SPLIT == 3) {
-                            mma_tf32(tmem_d, ah, desc_b(s_bl + kk * 1024), acc0);
-                            mma_tf32(tmem_d, desc_a(s_al + kk * 32), bh, 1u);
-                            mma_tf32(tmem_d, ah, bh, 1u);
-                        } else {
-                            mma_tf32(tmem_d, ah, bh, acc0);
+                        for (int kk = 0; kk < BK / 8; ++kk) {
+                            const uint64_t ah = desc_a(s_ah + kk * 32);    // +8 k in a 64-B row
+                            const uint64_t bh = desc_b(s_bh + kk * 1024);  // +8 k rows of 128 B
+                            const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
+                            if (SPLIT == 3) {
+                                mma_tf32<CG>(tmem_d, ah, desc_b(s_bl + kk * 1024), acc0);
+                                mma_tf32<CG>(tmem_d, desc_a(s_al + kk * 32), bh, 1u);
+                                mma_tf32<CG>(tmem_d, ah, bh, 1u);
+                            } else {
+                                mma_tf32<CG>(tmem_d, ah, bh, acc0);
+                            }
                         }
+                        if (SPLIT == 2) {
+                            // cross terms on the bf16 tiles, K = 16 in one MMA each
+                            const uint32_t a16h = s_bh + TB, a16l = a16h + kTileA16;
+                            const uint32_t b16h = a16l + kTileA16, b16l = b16h + TB16;
+                            mma_bf16<CG>(tmem_d, desc_a16(a16h), desc_b16(b16l), 1u);
+                            mma_bf16<CG>(tmem_d, desc_a16(a16l), desc_b16(b16h), 1u);
+                        }
+                        mma_commit<CG>(&empty[s]);
+                        if (kb == KB - 1) mma_commit<CG>(&acc_full[a]);
                     }
-                    if (SPLIT == 2) {
-                        // cross terms on the bf16 tiles, K = 16 in one MMA each
-                        const uint32_t a16h = s_bh + kTileB, a16l = a16h + kTileA16;
-                        const uint32_t b16h = a16l + kTileA16, b16l = b16h + kTileB16;
-                        mma_bf16(tmem_d, desc_a16(a16h), desc_b16(b16l), 1u);
-                        mma_bf16(tmem_d, desc_a16(a16l), desc_b16(b16h), 1u);
+                    __syncwarp();
+                }
+                if (KB == 0 && lane == 0) {  // K == 0: nothing accumulated
+                    if constexpr (CG == 2) {
+                        mbar_arrive_cluster(map_to(&acc_full[a], 0));
+                        mbar_arrive_cluster(map_to(&acc_full[a], 1));
+                    } else {
+                        mbar_arrive(&acc_full[a]);
                     }
-                    mma_commit(&empty[s]);
-                    if (kb == KB - 1) mma_commit(&acc_full[a]);
                 }
                 __syncwarp();
             }
-            if (KB == 0 && lane == 0) mbar_arrive(&acc_full[a]);  // K == 0: nothing accumulated
-            __syncwarp();
         }
     } else if (warp < 4 || warp >= 8) {
-        // ------------------------------------------------------------ lo converters
-        if (SPLIT == 3) {
-            const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;  // 0..kConvThreads-1
+        // ------------------------------------------------------------ converters
+        const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;  // 0..255
+        const uint32_t conv_leader0 = CG == 2 ? map_to(&conv[0], 0) : 0;
+        auto conv_done = [&](int s) {
+            fence_proxy_async();
+            __syncwarp();
+            if (lane == 0) {
+                if constexpr (CG == 2) mbar_arrive_cluster(conv_leader0 + (uint32_t)s * 8u);
+                else mbar_arrive(&conv[s]);
+            }
+        };
+        if constexpr (SPLIT == 3) {
             uint32_t it = 0;
-            for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+            for (uint32_t t = cl; t < total; t += ncl) {
                 const int v = find_tile_owner(descs, n, t);
                 const int KB = (descs[v].K + BK - 1) / BK;
                 for (int kb = 0; kb < KB; ++kb, ++it) {
@@ -315,29 +422,29 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                     const uint32_t ph = (it / ST) & 1;
                     mbar_wait(&full[s], ph);
                     const float4* hi = reinterpret_cast<const float4*>(stage(s));
-                    float4* lo = reinterpret_cast<float4*>(stage(s) + kTileA + kTileB);
-                    constexpr int NV = (kTileA + kTileB) / 16;  // 1536 float4: A then B, same order
+                    float4* lo = reinterpret_cast<float4*>(stage(s) + kTileA + TB);
+                    constexpr int NV = (kTileA + TB) / 16;  // A then B, same order
 #pragma unroll
                     for (int i = ct; i < NV; i += kConvThreads) lo[i] = lo_part4(hi[i]);
-                    fence_proxy_async();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&conv[s]);
+                    conv_done(s);
                 }
             }
-        } else if (SPLIT == 2) {
-            const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;  // 0..255
+        } else if constexpr (SPLIT == 2) {
             // A unit (one per thread): row m, k half kc; a phase's 8 lanes = 8 rows, same kc
             const int am = (ct >> 4) * 8 + (ct & 7), akc = (ct >> 3) & 1;
             const int asw = (am >> 1) & 3;  // SWIZZLE_64B: 16-B chunk ^= bits [7,9) of the address
             const int a_rd0 = am * 64 + (((2 * akc) ^ asw) << 4), a_rd1 = am * 64 + (((2 * akc + 1) ^ asw) << 4);
             const int a_wr = (am >> 3) * 256 + akc * 128 + (am & 7) * 16;
-            // B units (two per thread): k row, 32-n block j, 32-B granule g (8 n); a phase's 8
-            // lanes = 4 granules x 2 adjacent blocks, the first 16-B half read alternates with j
-            int b_rd[2][2], b_wr[2];
+            // B units: k row, 32-n block j, 32-B granule g (8 n); a phase's 8 lanes = 4
+            // granules x 2 adjacent blocks, the first 16-B half read alternates with j
+            constexpr int NB = (BK * C::kBN / 8) / kConvThreads;  // 2 (CG 1) or 1 (CG 2)
+            constexpr int JB = C::kBN / 32;                       // 32-n blocks: 8 or 4
+            int b_rd[NB][2], b_wr[NB];
 #pragma unroll
-            for (int r = 0; r < 2; ++r) {
-                const int u = ct + 256 * r;
-                const int g = u & 3, j = ((u >> 2) & 1) + 2 * ((u >> 3) & 3), k = u >> 5;
+            for (int r = 0; r < NB; ++r) {
+                const int u = ct + kConvThreads * r;
+                const int g = u & 3, j = ((u >> 2) & 1) + 2 * ((u >> 3) & (JB / 2 - 1));
+                const int k = u / (4 * JB);
                 const int base = j * kBBlock + k * 128 + ((g ^ (k & 3)) << 5);  // SWIZZLE_128B_BASE32B
                 const int h = j & 1;
                 b_rd[r][0] = base + 16 * h;
@@ -346,7 +453,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                 b_wr[r] = (j >> 1) * 2048 + (k >> 3) * 1024 + k8 * 128 + ((c ^ k8) << 4);
             }
             uint32_t it = 0;
-            for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+            for (uint32_t t = cl; t < total; t += ncl) {
                 const int v = find_tile_owner(descs, n, t);
                 const int KB = (descs[v].K + BK - 1) / BK;
                 for (int kb = 0; kb < KB; ++kb, ++it) {
@@ -354,10 +461,10 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                     const uint32_t ph = (it / ST) & 1;
                     mbar_wait(&full[s], ph);
                     uint8_t* sp = stage(s);
-                    uint8_t* a16h = sp + kTileA + kTileB;
+                    uint8_t* a16h = sp + kTileA + TB;
                     uint8_t* a16l = a16h + kTileA16;
                     uint8_t* b16h = a16l + kTileA16;
-                    uint8_t* b16l = b16h + kTileB16;
+                    uint8_t* b16l = b16h + TB16;
                     {
                         const float4 p = *reinterpret_cast<const float4*>(sp + a_rd0);
                         const float4 q = *reinterpret_cast<const float4*>(sp + a_rd1);
@@ -367,7 +474,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                         *reinterpret_cast<uint4*>(a16l + a_wr) = lb;
                     }
 #pragma unroll
-                    for (int r = 0; r < 2; ++r) {
+                    for (int r = 0; r < NB; ++r) {
                         const float4 x0 = *reinterpret_cast<const float4*>(sp + kTileA + b_rd[r][0]);
                         const float4 x1 = *reinterpret_cast<const float4*>(sp + kTileA + b_rd[r][1]);
                         const bool sw = (b_rd[r][0] & 16) != 0;  // read the upper half first
@@ -376,17 +483,16 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                         *reinterpret_cast<uint4*>(b16h + b_wr[r]) = hb;
                         *reinterpret_cast<uint4*>(b16l + b_wr[r]) = lb;
                     }
-                    fence_proxy_async();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&conv[s]);
+                    conv_done(s);
                 }
             }
         }
     } else {
         // ------------------------------------------------------------ epilogue (warps 4-7)
         const int q = warp & 3;  // TMEM lane quarter
+        const uint32_t acc_empty_leader = CG == 2 ? map_to(&acc_empty[0], 0) : 0;
         uint32_t tile_i = 0;
-        for (uint32_t t = blockIdx.x; t < total; t += gridDim.x, ++tile_i) {
+        for (uint32_t t = cl; t < total; t += ncl, ++tile_i) {
             const int v = find_tile_owner(descs, n, t);
             const GemmDesc& g = descs[v];
             const uint32_t lt = t - g.tile_begin;
@@ -395,7 +501,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
             const uint32_t aph = (tile_i >> 1) & 1;
             mbar_wait(&acc_full[a], aph);
             tc_fence_after();
-            const int row = tm * BM + q * 32 + lane;
+            const int row = tm * C::kMmaM + (int)rank * BM + q * 32 + lane;
             const bool row_ok = row < g.M;
             float* crow = g.C + (size_t)(row_ok ? row : 0) * g.N;
             const float alpha = g.alpha, beta = g.beta;
@@ -428,51 +534,87 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
             }
             tc_fence_before();
             __syncwarp();
-            if (lane == 0) mbar_arrive(&acc_empty[a]);
+            if (lane == 0) {
+                if constexpr (CG == 2) mbar_arrive_cluster(acc_empty_leader + (uint32_t)a * 8u);
+                else mbar_arrive(&acc_empty[a]);
+            }
         }
     }
     // ---------------------------------------------------------------- teardown
     tc_fence_before();
     __syncthreads();
+    if constexpr (CG == 2) cluster_sync_all();  // neither CTA frees TMEM / exits under the peer
     tc_fence_after();
     if (warp == 1) {
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(kTmemCols)
-                     : "memory");
+        if constexpr (CG == 1)
+            asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(kTmemCols)
+                         : "memory");
+        else
+            asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(kTmemCols)
+                         : "memory");
     }
 }
 
-static bool g_attr_set[4][64] = {};
+static bool g_attr_set[8][64] = {};
 
-template <int SPLIT>
-static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
+template <int SPLIT, int CG>
+static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uint32_t total, int clusters,
                              cudaStream_t s) {
     int dev = 0;
     cudaGetDevice(&dev);
-    const int si = SPLIT;
+    const int si = SPLIT + 4 * (CG - 1);
+    auto kern = k_sgemm_tc<SPLIT, CG>;
     if (dev < 64 && !g_attr_set[si][dev]) {
-        cudaError_t e = cudaFuncSetAttribute(k_sgemm_tc<SPLIT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)tc::Cfg<SPLIT>::kSmem);
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)tc::Cfg<SPLIT, CG>::kSmem);
         if (e) return e;
         g_attr_set[si][dev] = true;
     }
-    k_sgemm_tc<SPLIT><<<grid, tc::kThreads, tc::Cfg<SPLIT>::kSmem, s>>>(descs, n, reinterpret_cast<const uint8_t*>(maps),
-                                                                       total);
-    return cudaGetLastError();
+    cudaLaunchConfig_t lc = {};
+    cudaLaunchAttribute attr[1];
+    lc.gridDim = dim3((unsigned)(clusters * CG));
+    lc.blockDim = dim3(tc::kThreads);
+    lc.dynamicSmemBytes = tc::Cfg<SPLIT, CG>::kSmem;
+    lc.stream = s;
+    if (CG == 2) {
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = 2;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        lc.attrs = attr;
+        lc.numAttrs = 1;
+    }
+    return cudaLaunchKernelEx(&lc, kern, descs, n, reinterpret_cast<const uint8_t*>(maps), total);
+}
+
+// CTA-pair kernels for the fp32-accurate splits unless SVP_TC_CTA_PAIR=0 (A/B switch)
+bool sgemm_tc_cta_pair() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("SVP_TC_CTA_PAIR");
+        v = (e && atoi(e) == 0) ? 0 : 1;
+    }
+    return v == 1;
 }
 
 cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
                               cudaStream_t s) {
-    return launch_tc<1>(descs, n, maps, total, grid, s);
+    return launch_tc<1, 1>(descs, n, maps, total, grid, s);
 }
 
+// `grid` counts SMs; with CTA pairs the grid of pairs is half of it
 cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
                                   cudaStream_t s) {
-    return launch_tc<2>(descs, n, maps, total, grid, s);
+    if (sgemm_tc_cta_pair())
+        return launch_tc<2, 2>(descs, n, maps, total, (int)std::min<uint32_t>(total, std::max(1, grid / 2)), s);
+    return launch_tc<2, 1>(descs, n, maps, total, grid, s);
 }
 
 cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
                                 cudaStream_t s) {
-    return launch_tc<3>(descs, n, maps, total, grid, s);
+    if (sgemm_tc_cta_pair())
+        return launch_tc<3, 2>(descs, n, maps, total, (int)std::min<uint32_t>(total, std::max(1, grid / 2)), s);
+    return launch_tc<3, 1>(descs, n, maps, total, grid, s);
 }
 
 }  // namespace svp

@@ -48,6 +48,10 @@ cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, 
 cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
                                   int grid, cudaStream_t s);
 
+// true: the fp32-accurate tcgen05 SGEMMs run as CTA pairs (cta_group::2, 256 x 256 tiles);
+// SVP_TC_CTA_PAIR=0 selects the single-CTA kernels (128 x 256 tiles)
+bool sgemm_tc_cta_pair();
+
 // Grouped fp64 GEMM (the paper's Table 1 matmul), FP64 DFMA with smem tiles.
 cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total_tiles, int grid, cudaStream_t s);
 cudaError_t query_limits_dgemm(int* per_sm);
