@@ -76,7 +76,7 @@ typedef struct svp_config {
     int32_t flush_timeout_ms;    /* 0 = wait forever; else watchdog -> SVP_E_TIMEOUT          */
     int32_t validate_ptrs;       /* 1: svp_submit checks residency with cudaPointerGetAttributes
                                     (device buffer on the VP's GPU, host buffer pinned)       */
-    int32_t sgemm_impl;          /* SVP_SGEMM_3XTF32 (default), SVP_SGEMM_TF32BF16 or SVP_SGEMM_FFMA */
+    int32_t sgemm_impl;          /* SVP_SGEMM_TF32BF16 (default), SVP_SGEMM_3XTF32 or SVP_SGEMM_FFMA */
     void* const* external_streams; /* optional [num_gpus] caller cudaStream_t (e.g. torch's
                                     current stream): flush work starts after the work already
                                     queued on it, and it waits for the flush's last op.      */
@@ -98,7 +98,7 @@ typedef struct svp_config {
 } svp_config;
 
 /* Fill *cfg with defaults: num_gpus 0, 4 compute streams, coalesce 1, interleave 1,
-   max_chunks 8, profile_level 0, validate_ptrs 1, sgemm_impl SVP_SGEMM_3XTF32, rest 0
+   max_chunks 8, profile_level 0, validate_ptrs 1, sgemm_impl SVP_SGEMM_TF32BF16, rest 0
    (hetero 0, graph 0). */
 void svp_config_default(svp_config* cfg);
 

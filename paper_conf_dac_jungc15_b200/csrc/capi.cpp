@@ -94,7 +94,7 @@ void svp_config_default(svp_config* cfg) {
     cfg->max_chunks = 8;
     cfg->profile_level = 0;
     cfg->validate_ptrs = 1;
-    cfg->sgemm_impl = SVP_SGEMM_3XTF32;
+    cfg->sgemm_impl = SVP_SGEMM_TF32BF16;
 }
 
 svp_status svp_init(const svp_config* cfg, svp_ctx** out) {

@@ -62,6 +62,10 @@
 
 namespace svp {
 
+#ifndef SVP_PAIR_STAGES
+#define SVP_PAIR_STAGES 6
+#endif
+
 namespace tc {
 
 constexpr int BM = kTf32BM, BN = kTf32BN, BK = kTf32BK;  // 128 x 256 x 16 per CTA
@@ -80,7 +84,7 @@ struct Cfg {
     static constexpr int kTileB16 = BK * kBN * 2;
     // stage: A | B [| A_lo | B_lo]   (SPLIT 2: A | B | bf A_hi | bf A_lo | bf B_hi | bf B_lo)
     static constexpr int kStageBytes = (kTileA + kTileB) * (SPLIT == 1 ? 1 : 2);
-    static constexpr int kStages = SPLIT == 1 ? 8 : (CG == 2 ? 6 : 4);
+    static constexpr int kStages = SPLIT == 1 ? 8 : (CG == 2 ? SVP_PAIR_STAGES : 4);
     static constexpr size_t kBarOff = (size_t)kStages * kStageBytes;
     static constexpr size_t kSmem = 1024 + kBarOff + 256;
     static constexpr int kMmaM = BM * CG;
