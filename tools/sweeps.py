@@ -13,7 +13,11 @@ S3 (Fig 9 + Eq 7/8): N host-resident SGEMM jobs (H2D A,B -> 
 S4 (BASELINE metric): jobs/s of the cfg5 mix vs #VPs (1 GPU).
 S5 (Table 1): N VPs each running the paper's program -- 300
     multiplications of two 320x320 fp64 matrices -- coalesced per program-order level vs
-    serial per-VP launches; DGEMM TFLOP/s.
+    serial per-VP launches; DGEMM TFLOP/s; the same program with steady-state graph replay.
+S6 (NEXT f4, launch-bound mixes): N VPs with small vecadd / SAXPY / Black-Scholes jobs
+    (16Ki-64Ki elements); wall time of submit + flush per round for the default path,
+    hetero (one mixed launch), graph (plan reuse + CUDA-graph replay), both, and the
+    serial baselines B2 / B3 (B2 as a graph).
 Times are CUDA-event device times around whole flushes (median of reps).
 """
 import argparse
@@ -171,6 +175,12 @@ def s5_table1(quick):
         sc.register_kernel("dgemm")
         ts = flush_time(sc, jobs, reps=1, warm=1)
         sc.close()
+        gc = ctx_for(graph=True)
+        gc.register_kernel("dgemm")
+        row["graph_ms"] = flush_time(gc, jobs, reps=3, warm=2) * 1e3
+        row["graph_wall_ms"] = wall_time(gc, jobs, reps=3, warm=1) * 1e3
+        row["coalesced_wall_ms"] = wall_time(c, jobs, reps=3, warm=1) * 1e3
+        gc.close()
         row["serial_sync_ms"] = ts * 1e3
         row["speedup_vs_serial_sync"] = ts / t
         rows.append(row)
@@ -181,11 +191,59 @@ def s5_table1(quick):
             "rows": rows}
 
 
+def wall_time(ctx, jobs, reps=50, warm=5):
+    """Host wall time of submit + flush (the flush returns when the outputs are in place)."""
+    import time
+    jobs = svp.JobBatch(jobs)
+    for _ in range(warm):
+        ctx.submit_batch(jobs)
+        ctx.flush()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        ctx.submit_batch(jobs)
+        ctx.flush()
+        ts.append(time.perf_counter() - t0)
+    return statistics.median(ts)
+
+
+def s6_f4(quick):
+    kinds = ("vecadd", "saxpy", "blackscholes")
+    rows = []
+    for nv in ([16, 256] if quick else [16, 64, 256, 1024]):
+        g = np.random.default_rng(nv)
+        specs = [W.JobSpec(v, kinds[v % 3], n=int(g.integers(1 << 14, 1 << 16)), R=0.02, V=0.3,
+                           a=float(g.uniform(-2, 2))) for v in range(nv)]
+        inputs = W.make_inputs_many(specs)
+        row = {"vps": nv, "elements": int(sum(s.n for s in specs))}
+        for name, kw in (("default", {}), ("hetero", dict(hetero=True)), ("graph", dict(graph=True)),
+                         ("hetero_graph", dict(hetero=True, graph=True)),
+                         ("B2_serial_async", dict(coalesce=False, interleave=False)),
+                         ("B3_serial_graph", dict(coalesce=False, interleave=False, graph=True))):
+            c = ctx_for(**kw)
+            vs = VPSet(c, specs, inputs, "device")
+            t = wall_time(c, vs.job_list())
+            st = c.flush_stats()
+            row[name + "_us"] = t * 1e6
+            row[name + "_launches"] = int(st["launches"])
+            row[name + "_host_plan_us"] = st["host_plan_ns"] / 1e3
+            row[name + "_host_issue_us"] = st["host_issue_ns"] / 1e3
+            c.close()
+            del vs
+        row["speedup_graph_vs_default"] = row["default_us"] / row["graph_us"]
+        row["speedup_hetero_graph_vs_default"] = row["default_us"] / row["hetero_graph_us"]
+        row["speedup_default_vs_B2"] = row["B2_serial_async_us"] / row["default_us"]
+        rows.append(row)
+        torch.cuda.empty_cache()
+    return rows
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default=None)
     ap.add_argument("--quick", action="store_true")
-    ap.add_argument("--only", default="12345")
+    ap.add_argument("--only", default="123456")
     args = ap.parse_args()
     torch.cuda.set_device(0)
     res = {"gpu": torch.cuda.get_device_name(0)}
@@ -199,6 +257,8 @@ def main():
         res["S4_jobs_vs_vps"] = s4_vps(args.quick)
     if "5" in args.only:
         res["S5_table1_dgemm"] = s5_table1(args.quick)
+    if "6" in args.only:
+        res["S6_f4_launch_bound"] = s6_f4(args.quick)
     txt = json.dumps(res, indent=1)
     print(txt)
     if args.out:
