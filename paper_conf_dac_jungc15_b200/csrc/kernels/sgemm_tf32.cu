@@ -21,7 +21,16 @@
 //             inside the 1e-5 (|A||B|)_ij bound (R19); integer inputs stay exact
 //             (lo = 0).
 //
-// CG = 2 (CTA pair, cta_group::2; SPLIT 2 and 3): a cluster of 2 CTAs on one TPC computes a
+//  SPLIT = 4  the SPLIT 2 arithmetic with the A-side bf16 operands in TMEM: converters
+//             tcgen05.st bf(A_hi) / bf(A_lo) (lane = row, column = k pair) into a TMEM ring
+//             next to the accumulator and the BF16 MMAs read A from TMEM ([a_tmem] form).
+//             Removes 8 KiB of converter smem writes and 8 KiB of MMA smem reads per stage
+//             (the pair kernel is shared-memory bound: LSU + tensor-core smem wavefronts ~96 %
+//             of the data pipe); the price is a single TMEM accumulator (2x256 + the ring
+//             would exceed 512 columns), so a tile's epilogue no longer overlaps the next
+//             tile's MMAs.
+//
+// CG = 2 (CTA pair, cta_group::2; SPLIT 2, 3, 4): a cluster of 2 CTAs on one TPC computes a
 // 256 x 256 tile with M256 N256 MMAs issued by the leader CTA.  Each CTA stages its own
 // 128 rows of A and 128 columns of B (half the operand bytes per SM: the per-SM shared-
 // memory traffic -- TMA writes + converter reads/writes -- is what bounds the single-CTA
@@ -82,9 +91,16 @@ struct Cfg {
     static constexpr int kBN = BN / CG;                    // B columns staged per CTA
     static constexpr int kTileB = BK * kBN * 4;            // 16 KiB (CG 1) / 8 KiB (CG 2)
     static constexpr int kTileB16 = BK * kBN * 2;
-    // stage: A | B [| A_lo | B_lo]   (SPLIT 2: A | B | bf A_hi | bf A_lo | bf B_hi | bf B_lo)
-    static constexpr int kStageBytes = (kTileA + kTileB) * (SPLIT == 1 ? 1 : 2);
-    static constexpr int kStages = SPLIT == 1 ? 8 : (CG == 2 ? SVP_PAIR_STAGES : 4);
+    // stage: A | B [| A_lo | B_lo]   (SPLIT 2: A | B | bf A_hi | bf A_lo | bf B_hi | bf B_lo;
+    // SPLIT 4: A | B | bf B_hi | bf B_lo, the A-side bf16 tiles live in TMEM)
+    static constexpr int kStageBytes = SPLIT == 4 ? kTileA + kTileB + 2 * kTileB16
+                                                  : (kTileA + kTileB) * (SPLIT == 1 ? 1 : 2);
+    static constexpr int kStages = SPLIT == 1 ? 8
+                                 : SPLIT == 4 ? (CG == 2 ? 8 : 5)
+                                              : (CG == 2 ? SVP_PAIR_STAGES : 4);
+    static constexpr int kAcc = SPLIT == 4 ? 1 : 2;        // TMEM accumulators (256 cols each)
+    static constexpr int kTaCol = 256;                     // SPLIT 4: A ring, 16 cols per stage
+    static_assert(SPLIT != 4 || kTaCol + 16 * kStages <= kTmemCols, "TMEM");
     static constexpr size_t kBarOff = (size_t)kStages * kStageBytes;
     static constexpr size_t kSmem = 1024 + kBarOff + 256;
     static constexpr int kMmaM = BM * CG;
@@ -132,6 +148,29 @@ __device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t adesc, uint64
             "l"(adesc), "l"(bdesc), "r"(Idesc<2 * BM>::tf32), "r"(accum)
             : "memory");
 }
+// kind::f16 with A from TMEM (lane = row, 32-bit column c = k pair {2c, 2c+1}, low half = even
+// k: scripts/tc_tmem_a.py)
+template <int CG>
+__device__ __forceinline__ void mma_bf16_ta(uint32_t tmem_d, uint32_t tmem_a, uint64_t bdesc, uint32_t accum) {
+    if constexpr (CG == 1)
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
+            "r"(tmem_a), "l"(bdesc), "r"(Idesc<BM>::bf16), "r"(accum)
+            : "memory");
+    else
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::2.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
+            "r"(tmem_a), "l"(bdesc), "r"(Idesc<2 * BM>::bf16), "r"(accum)
+            : "memory");
+}
+__device__ __forceinline__ void tmem_st4(uint32_t taddr, const uint4& v) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(v.x), "r"(v.y),
+                 "r"(v.z), "r"(v.w)
+                 : "memory");
+}
+
 template <int CG>
 __device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accum) {
     if constexpr (CG == 1)
@@ -339,8 +378,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
             for (uint32_t t = cl; t < total; t += ncl, ++tile_i) {
                 const int v = find_tile_owner(descs, n, t);
                 const int KB = (descs[v].K + BK - 1) / BK;
-                const int a = tile_i & 1;
-                const uint32_t aph = (tile_i >> 1) & 1;
+                const int a = tile_i % C::kAcc;
+                const uint32_t aph = (tile_i / C::kAcc) & 1;
                 if constexpr (CG == 2) mbar_wait_cluster(&acc_empty[a], aph ^ 1);
                 else mbar_wait(&acc_empty[a], aph ^ 1);
                 tc_fence_after();
@@ -379,6 +418,11 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                             const uint32_t b16h = a16l + kTileA16, b16l = b16h + TB16;
                             mma_bf16<CG>(tmem_d, desc_a16(a16h), desc_b16(b16l), 1u);
                             mma_bf16<CG>(tmem_d, desc_a16(a16l), desc_b16(b16h), 1u);
+                        } else if (SPLIT == 4) {
+                            const uint32_t ta = tmem_base + (uint32_t)(C::kTaCol + 16 * s);
+                            const uint32_t b16h = s_bh + TB, b16l = b16h + TB16;
+                            mma_bf16_ta<CG>(tmem_d, ta, desc_b16(b16l), 1u);       // bf(A_hi) bf(B_lo)
+                            mma_bf16_ta<CG>(tmem_d, ta + 8, desc_b16(b16h), 1u);   // bf(A_lo) bf(B_hi)
                         }
                         mma_commit<CG>(&empty[s]);
                         if (kb == KB - 1) mma_commit<CG>(&acc_full[a]);
@@ -425,8 +469,14 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                     conv_done(s);
                 }
             }
-        } else if constexpr (SPLIT == 2) {
-            // A unit (one per thread): row m, k half kc; a phase's 8 lanes = 8 rows, same kc
+        } else if constexpr (SPLIT == 2 || SPLIT == 4) {
+            // SPLIT 4: this warp's TMEM lane quarter q = warp % 4 holds rows 32q..32q+31; the two
+            // converter warps of a quarter split the 16 k into halves th (4 columns each)
+            const int tq = warp & 3, th = (warp == 2 || warp == 3 || warp == 8 || warp == 9) ? 0 : 1;
+            const int tm = tq * 32 + lane, tsw = (tm >> 1) & 3;
+            const int t_rd0 = tm * 64 + (((2 * th) ^ tsw) << 4), t_rd1 = tm * 64 + (((2 * th + 1) ^ tsw) << 4);
+            const uint32_t t_lane = tmem_base + ((uint32_t)(tq * 32) << 16) + (uint32_t)(C::kTaCol + 4 * th);
+            // SPLIT 2 A unit (one per thread): row m, k half kc; a phase's 8 lanes = 8 rows, same kc
             const int am = (ct >> 4) * 8 + (ct & 7), akc = (ct >> 3) & 1;
             const int asw = (am >> 1) & 3;  // SWIZZLE_64B: 16-B chunk ^= bits [7,9) of the address
             const int a_rd0 = am * 64 + (((2 * akc) ^ asw) << 4), a_rd1 = am * 64 + (((2 * akc + 1) ^ asw) << 4);
@@ -459,9 +509,16 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                     uint8_t* sp = stage(s);
                     uint8_t* a16h = sp + kTileA + TB;
                     uint8_t* a16l = a16h + kTileA16;
-                    uint8_t* b16h = a16l + kTileA16;
+                    uint8_t* b16h = SPLIT == 4 ? a16h : a16l + kTileA16;
                     uint8_t* b16l = b16h + TB16;
-                    {
+                    if constexpr (SPLIT == 4) {
+                        const float4 p = *reinterpret_cast<const float4*>(sp + t_rd0);
+                        const float4 q = *reinterpret_cast<const float4*>(sp + t_rd1);
+                        uint4 hb, lb;
+                        split8(p, q, hb, lb);
+                        tmem_st4(t_lane + 16 * s, hb);
+                        tmem_st4(t_lane + 16 * s + 8, lb);
+                    } else {
                         const float4 p = *reinterpret_cast<const float4*>(sp + a_rd0);
                         const float4 q = *reinterpret_cast<const float4*>(sp + a_rd1);
                         uint4 hb, lb;
@@ -479,6 +536,10 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                         *reinterpret_cast<uint4*>(b16h + b_wr[r]) = hb;
                         *reinterpret_cast<uint4*>(b16l + b_wr[r]) = lb;
                     }
+                    if constexpr (SPLIT == 4) {
+                        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+                        tc_fence_before();
+                    }
                     conv_done(s);
                 }
             }
@@ -493,8 +554,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
             const GemmDesc& g = descs[v];
             const uint32_t lt = t - g.tile_begin;
             const int tm = lt / g.tiles_n, tn = lt % g.tiles_n;
-            const int a = tile_i & 1;
-            const uint32_t aph = (tile_i >> 1) & 1;
+            const int a = tile_i % C::kAcc;
+            const uint32_t aph = (tile_i / C::kAcc) & 1;
             mbar_wait(&acc_full[a], aph);
             tc_fence_after();
             const int row = tm * C::kMmaM + (int)rank * BM + q * 32 + lane;
@@ -551,14 +612,14 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
     }
 }
 
-static bool g_attr_set[8][64] = {};
+static bool g_attr_set[10][64] = {};
 
 template <int SPLIT, int CG>
 static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uint32_t total, int clusters,
                              cudaStream_t s) {
     int dev = 0;
     cudaGetDevice(&dev);
-    const int si = SPLIT + 4 * (CG - 1);
+    const int si = SPLIT + 5 * (CG - 1);
     auto kern = k_sgemm_tc<SPLIT, CG>;
     if (dev < 64 && !g_attr_set[si][dev]) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -599,11 +660,22 @@ cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, ui
 }
 
 // `grid` counts SMs; with CTA pairs the grid of pairs is half of it
+// SVP_TC_TMEM_A=0 keeps the A-side bf16 operands in shared memory (SPLIT 2), else SPLIT 4
+static bool tmem_a() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("SVP_TC_TMEM_A");
+        v = (e && atoi(e) == 0) ? 0 : 1;
+    }
+    return v == 1;
+}
+
 cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
                                   cudaStream_t s) {
+    const int pairs = (int)std::min<uint32_t>(total, std::max(1, grid / 2));
     if (sgemm_tc_cta_pair())
-        return launch_tc<2, 2>(descs, n, maps, total, (int)std::min<uint32_t>(total, std::max(1, grid / 2)), s);
-    return launch_tc<2, 1>(descs, n, maps, total, grid, s);
+        return tmem_a() ? launch_tc<4, 2>(descs, n, maps, total, pairs, s) : launch_tc<2, 2>(descs, n, maps, total, pairs, s);
+    return tmem_a() ? launch_tc<4, 1>(descs, n, maps, total, grid, s) : launch_tc<2, 1>(descs, n, maps, total, grid, s);
 }
 
 cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
