@@ -443,7 +443,8 @@ def run_svp(args, rank, ws, local):
     e2e = None
     if not args.no_e2e:
         hctx = svp.Context(num_gpus=1, device_ids=[local], external_streams=[stream.cuda_stream],
-                           arena_bytes=args.arena_gb << 30, sgemm_impl=impl, **f4)
+                           arena_bytes=args.arena_gb << 30, sgemm_impl=impl,
+                           max_chunks=int(os.environ.get("SVP_BENCH_MAXCH", "8")), **f4)
         hvs = VPSet(hctx, specs, inputs, "host")
         hjobs = svp.JobBatch(hvs.job_list())
         hctx.submit_batch(hjobs)

@@ -660,12 +660,14 @@ cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, ui
 }
 
 // `grid` counts SMs; with CTA pairs the grid of pairs is half of it
-// SVP_TC_TMEM_A=0 keeps the A-side bf16 operands in shared memory (SPLIT 2), else SPLIT 4
+// SVP_TC_TMEM_A=1 selects SPLIT 4 (A-side bf16 operands in TMEM).  Measured on cfg5 it is
+// not faster (2.71 vs 2.64 ms per launch, profiles/r01/pair): the kernel runs under the
+// power cap, and the single accumulator costs the epilogue overlap; SPLIT 2 is the default.
 static bool tmem_a() {
     static int v = -1;
     if (v < 0) {
         const char* e = getenv("SVP_TC_TMEM_A");
-        v = (e && atoi(e) == 0) ? 0 : 1;
+        v = (e && atoi(e) == 1) ? 1 : 0;
     }
     return v == 1;
 }

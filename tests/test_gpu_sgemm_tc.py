@@ -83,3 +83,19 @@ def test_split_wide_dynamic_range(impl):
     outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl)
     for s, inp, got in zip(specs, inputs, outs):
         check_job(s, inp, got)
+
+
+@pytest.mark.parametrize("env", [{"SVP_TC_CTA_PAIR": "0"}, {"SVP_TC_TMEM_A": "1"},
+                                 {"SVP_TC_CTA_PAIR": "0", "SVP_TC_TMEM_A": "1"}])
+def test_kernel_variants_in_subprocess(env):
+    """The non-default tcgen05 variants (single-CTA kernels; A-side bf16 operands in TMEM)
+    are chosen once per process from the environment: run this file's fp32 parity tests
+    in a child process with the switch set."""
+    import os
+    import subprocess
+    import sys
+    here = os.path.dirname(os.path.abspath(__file__))
+    cmd = [sys.executable, "-m", "pytest", os.path.join(here, "test_gpu_sgemm_tc.py"), "-q", "-m", "gpu",
+           "-p", "no:cacheprovider", "-k", "(fp32_tolerance or ragged_alpha_beta or wide_dynamic) and not variants"]
+    r = subprocess.run(cmd, env={**os.environ, **env}, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
