@@ -262,6 +262,15 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
         if (ch.kernel == K_DGEMM) {
             ch.table_off = align_up(tbl.size(), 128);
             tbl.resize(ch.table_off + ch.jobs.size() * sizeof(DgemmDesc));
+            // 32x32 tiles when the launch has fewer than 2 waves of 64x64 tiles
+            uint64_t big = 0;
+            for (int32_t ji : ch.jobs) {
+                const Job& j = f.jobs[ji];
+                if ((int64_t)j.M * j.N > 0)
+                    big += (uint64_t)((j.M + kDgemmBM - 1) / kDgemmBM) * ((j.N + kDgemmBN - 1) / kDgemmBN);
+            }
+            ch.small_tiles = big < 2ull * d.lim.num_sms * d.lim.dgemm_blocks_per_sm;
+            const int TM = ch.small_tiles ? kDgemmSmall : kDgemmBM, TN = ch.small_tiles ? kDgemmSmall : kDgemmBN;
             uint32_t tiles = 0;
             for (size_t k = 0; k < ch.jobs.size(); ++k) {
                 const Job& j = f.jobs[ch.jobs[k]];
@@ -276,8 +285,8 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
                 g.alpha = j.d0;
                 g.beta = j.d1;
                 g.tile_begin = tiles;
-                g.tiles_n = (uint32_t)((j.N + kDgemmBN - 1) / kDgemmBN);
-                uint64_t nt = (int64_t)j.M * j.N == 0 ? 0 : (uint64_t)((j.M + kDgemmBM - 1) / kDgemmBM) * g.tiles_n;
+                g.tiles_n = (uint32_t)((j.N + TN - 1) / TN);
+                uint64_t nt = (int64_t)j.M * j.N == 0 ? 0 : (uint64_t)((j.M + TM - 1) / TM) * g.tiles_n;
                 tiles += (uint32_t)nt;
                 memcpy(tbl.data() + ch.table_off + k * sizeof(DgemmDesc), &g, sizeof(g));
             }
@@ -417,7 +426,8 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
                                      ch.total_tiles, grid_of(d.lim.gemm_blocks_per_sm), s);
         case K_DGEMM:
             return launch_dgemm((const DgemmDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
-                                grid_of(d.lim.dgemm_blocks_per_sm), s);
+                                grid_of(ch.small_tiles ? d.lim.dgemm_small_blocks_per_sm : d.lim.dgemm_blocks_per_sm),
+                                ch.small_tiles, s);
         case K_SGEMM_TF32:
             return launch_sgemm_tf32((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
                                      ch.total_tiles, grid_of(1), s);
@@ -494,8 +504,11 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
         for (size_t s = 1; s < d.streams.size(); ++s) CK(cudaStreamWaitEvent(d.streams[s], d.tbl_ev, 0));
         d.tbl_last.swap(tbl);
         ++d.table_uploads;
-        c->fstats.table_uploads += 1;
-        c->fstats.table_bytes += d.tbl_last.size();
+        {
+            std::lock_guard<std::mutex> lk(c->pmu);  // one worker thread per GPU updates fstats
+            c->fstats.table_uploads += 1;
+            c->fstats.table_bytes += d.tbl_last.size();
+        }
     }
     // ---- steady-state replay: second sighting of a plan -> capture, later -> replay
     std::vector<int> used(d.streams.size(), 0);
@@ -691,6 +704,7 @@ static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool u
             span = mx;
         }
         (void)lastop;
+        std::lock_guard<std::mutex> lk(c->pmu);
         c->fstats.device_ns = std::max(c->fstats.device_ns, (double)span * 1e6);
     }
     return SVP_OK;

@@ -93,6 +93,7 @@ struct Chunk {
     uint32_t total_tiles = 0;
     int32_t nsegs = 0;
     uint64_t maps_off = 0;          // sgemm: tensor maps offset
+    bool small_tiles = false;       // dgemm: 32x32 tile variant (launch under 2 waves of 64x64)
     int32_t co_grid = 0;            // >0: launch with co_grid CTAs per SM so the kernel
                                     // co-resides with a tensor-core SGEMM on the same SMs
 };

@@ -6,7 +6,10 @@
 // L526-531.  C_v = alpha_v A_v B_v + beta_v C_v, row-major, any M, N, K (ragged shapes
 // in one launch), fp64 DFMA:
 //  * persistent grid over the tiles of all VPs; tile -> (VP, tm, tn) via the DgemmDesc table;
-//  * 64x64 output tile, 16-deep k blocks, 256 threads with 4x4 accumulators each;
+//  * 64x64 output tile, 16-deep k blocks, 256 threads with 4x4 accumulators each; when a
+//    launch has fewer than 2 waves of 64x64 tiles (Table 1 with few VPs: 25 tiles per VP),
+//    32x32 tiles with 64 threads instead -- 4x the CTAs, so the dependent 320^3 GEMMs of
+//    the paper's program spread over the SMs instead of leaving 80 % of them idle;
 //  * A staged transposed in shared memory (k-major rows padded to 65 doubles: the 16
 //    k-rows of a warp's stores fall in distinct banks), B staged as is; two smem buffers
 //    with the next k block's global loads issued before the current block's DFMAs.
@@ -15,9 +18,7 @@
 
 namespace svp {
 
-constexpr int DM = kDgemmBM, DN = kDgemmBN, DK = kDgemmBK;
-constexpr int kDThreads = 256;
-constexpr int kApad = DM + 1;
+constexpr int DK = kDgemmBK;
 
 __device__ __forceinline__ int find_dgemm(const DgemmDesc* __restrict__ d, int n, uint32_t t) {
     int lo = 0, hi = n;
@@ -29,14 +30,20 @@ __device__ __forceinline__ int find_dgemm(const DgemmDesc* __restrict__ d, int n
     return lo - 1;
 }
 
-__global__ void __launch_bounds__(kDThreads) k_dgemm(const DgemmDesc* __restrict__ descs, int n, uint32_t total) {
+// TM x TN output tile, (TM/4) x (TN/4) threads with 4x4 accumulators each
+template <int TM, int TN>
+__global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* __restrict__ descs, int n,
+                                                               uint32_t total) {
+    constexpr int NT = (TM / 4) * (TN / 4);
+    constexpr int LA = TM * DK / NT, LB = DK * TN / NT;  // elements per thread per k block
+    constexpr int kApad = TM + 1;
     __shared__ double As[2][DK][kApad];
-    __shared__ __align__(16) double Bs[2][DK][DN];
-    const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+    __shared__ __align__(16) double Bs[2][DK][TN];
+    const int tid = threadIdx.x, tx = tid % (TN / 4), ty = tid / (TN / 4);
     for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
         const DgemmDesc& g = descs[find_dgemm(descs, n, t)];
         const uint32_t lt = t - g.tile_begin;
-        const int m0 = (lt / g.tiles_n) * DM, n0 = (lt % g.tiles_n) * DN;
+        const int m0 = (lt / g.tiles_n) * TM, n0 = (lt % g.tiles_n) * TN;
         const int M = g.M, N = g.N, K = g.K;
         const double* __restrict__ A = g.A;
         const double* __restrict__ B = g.B;
@@ -46,26 +53,33 @@ __global__ void __launch_bounds__(kDThreads) k_dgemm(const DgemmDesc* __restrict
 #pragma unroll
             for (int j = 0; j < 4; ++j) acc[i][j] = 0.0;
 
-        // each thread moves 4 A and 4 B elements per k block
-        double ra[4], rb[4];
+        double ra[LA], rb[LB];
         auto load = [&](int k0) {
 #pragma unroll
-            for (int i = 0; i < 4; ++i) {
-                const int idx = tid + i * kDThreads;   // A: 64 rows x 16 k, k fastest
+            for (int i = 0; i < LA; ++i) {
+                const int idx = tid + i * NT;  // A: TM rows x 16 k, k fastest
                 const int r = idx >> 4, c = idx & 15;
                 const int gm = m0 + r, gk = k0 + c;
                 ra[i] = (gm < M && gk < K) ? A[(size_t)gm * K + gk] : 0.0;
-                const int rr = idx >> 6, cc = idx & 63;  // B: 16 k x 64 cols, n fastest
+            }
+#pragma unroll
+            for (int i = 0; i < LB; ++i) {
+                const int idx = tid + i * NT;  // B: 16 k x TN cols, n fastest
+                const int rr = idx / TN, cc = idx % TN;
                 const int bk = k0 + rr, bn = n0 + cc;
                 rb[i] = (bk < K && bn < N) ? B[(size_t)bk * N + bn] : 0.0;
             }
         };
         auto store = [&](int buf) {
 #pragma unroll
-            for (int i = 0; i < 4; ++i) {
-                const int idx = tid + i * kDThreads;
+            for (int i = 0; i < LA; ++i) {
+                const int idx = tid + i * NT;
                 As[buf][idx & 15][idx >> 4] = ra[i];
-                Bs[buf][idx >> 6][idx & 63] = rb[i];
+            }
+#pragma unroll
+            for (int i = 0; i < LB; ++i) {
+                const int idx = tid + i * NT;
+                Bs[buf][idx / TN][idx % TN] = rb[i];
             }
         };
         const int KB = (K + DK - 1) / DK;
@@ -115,13 +129,18 @@ __global__ void __launch_bounds__(kDThreads) k_dgemm(const DgemmDesc* __restrict
     }
 }
 
-cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total, int grid, cudaStream_t s) {
-    k_dgemm<<<grid, kDThreads, 0, s>>>(descs, n, total);
+cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total, int grid, bool small, cudaStream_t s) {
+    if (small) k_dgemm<kDgemmSmall, kDgemmSmall><<<grid, (kDgemmSmall / 4) * (kDgemmSmall / 4), 0, s>>>(descs, n, total);
+    else k_dgemm<kDgemmBM, kDgemmBN><<<grid, (kDgemmBM / 4) * (kDgemmBN / 4), 0, s>>>(descs, n, total);
     return cudaGetLastError();
 }
 
-cudaError_t query_limits_dgemm(int* per_sm) {
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k_dgemm, kDThreads, 0);
+cudaError_t query_limits_dgemm(int* per_sm, int* per_sm_small) {
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k_dgemm<kDgemmBM, kDgemmBN>,
+                                                                  (kDgemmBM / 4) * (kDgemmBN / 4), 0);
+    if (e) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm_small, k_dgemm<kDgemmSmall, kDgemmSmall>,
+                                                         (kDgemmSmall / 4) * (kDgemmSmall / 4), 0);
 }
 
 }  // namespace svp

@@ -303,9 +303,10 @@ cudaError_t query_limits(LaunchLimits* out) {
     if (e) return e;
     e = query_limits_gemm(&out->gemm_blocks_per_sm);
     if (e) return e;
-    e = query_limits_dgemm(&out->dgemm_blocks_per_sm);
+    e = query_limits_dgemm(&out->dgemm_blocks_per_sm, &out->dgemm_small_blocks_per_sm);
     if (e) return e;
     if (out->dgemm_blocks_per_sm < 1) out->dgemm_blocks_per_sm = 1;
+    if (out->dgemm_small_blocks_per_sm < 1) out->dgemm_small_blocks_per_sm = 1;
     if (out->ew_blocks_per_sm < 1) out->ew_blocks_per_sm = 1;
     if (out->bs_blocks_per_sm < 1) out->bs_blocks_per_sm = 1;
     if (out->hist_blocks_per_sm < 1) out->hist_blocks_per_sm = 1;

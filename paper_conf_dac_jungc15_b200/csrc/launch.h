@@ -17,6 +17,7 @@ struct LaunchLimits {
     int hist_blocks_per_sm = 4;
     int gemm_blocks_per_sm = 1;
     int dgemm_blocks_per_sm = 1;
+    int dgemm_small_blocks_per_sm = 1;
 };
 
 // Query occupancy / SM count for the current device (call once per device).
@@ -52,9 +53,10 @@ cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps
 // SVP_TC_CTA_PAIR=0 selects the single-CTA kernels (128 x 256 tiles)
 bool sgemm_tc_cta_pair();
 
-// Grouped fp64 GEMM (the paper's Table 1 matmul), FP64 DFMA with smem tiles.
-cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total_tiles, int grid, cudaStream_t s);
-cudaError_t query_limits_dgemm(int* per_sm);
+// Grouped fp64 GEMM (the paper's Table 1 matmul), FP64 DFMA with smem tiles; `small`:
+// 32x32 tiles (the table was built with kDgemmSmall tiles).
+cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total_tiles, int grid, bool small, cudaStream_t s);
+cudaError_t query_limits_dgemm(int* per_sm, int* per_sm_small);
 
 // Host: encode the TMA descriptors an SGEMM entry needs (driver entry point fetched at
 // runtime, so libsvp does not link libcuda).  variant 0 = FFMA tiles, 1 = TF32 tiles.

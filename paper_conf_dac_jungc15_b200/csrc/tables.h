@@ -64,5 +64,6 @@ constexpr int kHistTile = kHistThreads * 16 * kHistVec;        // 16384 bytes
 constexpr int kGemmBM = 128, kGemmBN = 128, kGemmBK = 32;
 constexpr int kTf32BM = 128, kTf32BN = 256, kTf32BK = 16;
 constexpr int kDgemmBM = 64, kDgemmBN = 64, kDgemmBK = 16;
+constexpr int kDgemmSmall = 32;  // square tile of the small-launch DGEMM variant
 
 }  // namespace svp

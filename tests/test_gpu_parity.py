@@ -258,3 +258,16 @@ def test_table1_program_8vps():
     want = [oracle.run_job(specs[v * iters], base[v]) for v in range(8)]
     for i, (s, got) in enumerate(zip(specs, outs)):
         check_job(s, inputs[i], got, want[i // iters])
+
+
+def test_dgemm_both_tile_variants():
+    """A launch with >= 2 waves of 64x64 tiles uses the 64x64 kernel, a small one the 32x32
+    kernel (Table 1's 320^3 jobs); both against the oracle, ragged edges included."""
+    big = [W.JobSpec(v, "dgemm", M=1000, N=1030, K=72, alpha=1.25, beta=0.5 if v == 1 else 0.0) for v in range(2)]
+    big += [W.JobSpec(2 + v, "dgemm", M=640, N=640, K=40) for v in range(2)]  # 2*16*17 + 2*100 tiles
+    small = [W.JobSpec(10 + v, "dgemm", M=M, N=N, K=K) for v, (M, N, K) in enumerate([(320, 320, 320), (33, 65, 17)])]
+    for specs in (big, small):
+        inputs = inputs_for(specs)
+        outs, _, _ = run_svp(specs, inputs, "device")
+        for s, inp, got in zip(specs, inputs, outs):
+            check_job(s, inp, got)
