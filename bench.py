@@ -275,7 +275,7 @@ def run_svp(args, rank, ws, local):
     # ---------------- device-resident run (value)
     impl = IMPLS[args.sgemm_impl]
     trace("inputs ready")
-    f4 = dict(hetero=bool(args.hetero), graph=bool(args.graph))  # NEXT f4 options
+    f4 = dict(hetero=bool(args.hetero), graph=bool(args.graph), table_mode=args.table_mode)  # options
     ctx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, external_streams=[stream.cuda_stream],
                       validate_ptrs=True, sgemm_impl=impl, **f4)
     vs = VPSet(ctx, specs, inputs, "device", device_ordinals=[local])
@@ -489,7 +489,7 @@ def run_svp(args, rank, ws, local):
             "hbm_gbs_membound": hbm_gbs,
             "hbm_frac_membound": (hbm_gbs / float(peaks["hbm_gbs"])) if hbm_gbs else None,
             "elements_per_s": sum(s.n for s in all_specs) * args.steps / dt_max,
-            "sgemm_impl": args.sgemm_impl, "alt_sgemm_impls": alt, "hetero": args.hetero, "graph": args.graph,
+            "sgemm_impl": args.sgemm_impl, "alt_sgemm_impls": alt, "hetero": args.hetero, "graph": args.graph, "table_mode": args.table_mode,
             "graph_replays_last_step": int(st["graph_replays"]),
             "timed_kernel_ms_per_step": {n: k["total_ns"] / args.steps / 1e6 for n, k in main_kstats.items()
                                          if k["launches"]},
@@ -526,6 +526,8 @@ def main():
                     help="heterogeneous coalescing of vecadd/SAXPY/Black-Scholes (NEXT f4)")
     ap.add_argument("--graph", type=int, default=0, choices=[0, 1],
                     help="steady-state plan reuse + CUDA graph replay (NEXT f4)")
+    ap.add_argument("--table-mode", type=int, default=0, choices=[0, 1],
+                    help="segment tables: 0 global device buffer, 1 by-value kernel parameter")
     ap.add_argument("--no-serial", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other sgemm implementation")
     ap.add_argument("--no-e2e", action="store_true")

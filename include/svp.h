@@ -34,7 +34,7 @@
 extern "C" {
 #endif
 
-#define SVP_ABI_VERSION 2
+#define SVP_ABI_VERSION 3
 
 typedef int32_t svp_status;
 enum {
@@ -95,7 +95,15 @@ typedef struct svp_config {
                                     flush's reuses its plan and tables, and from the second
                                     repeat on replays the flush's device work as one CUDA
                                     graph per GPU.  Ignored with sync_each_job.              */
+    int32_t table_mode;          /* where a coalesced launch finds its segment table (SURVEY
+                                    §8(b)): SVP_TABLE_GLOBAL (default) -- one device table
+                                    buffer per GPU, uploaded once per flush when it changed;
+                                    SVP_TABLE_PARAM -- launches of elementwise / hist256
+                                    groups with <= 240 VPs receive it by value as a kernel
+                                    parameter (no upload; GEMM launches always use global) */
 } svp_config;
+
+enum { SVP_TABLE_GLOBAL = 0, SVP_TABLE_PARAM = 1 };
 
 /* Fill *cfg with defaults: num_gpus 0, 4 compute streams, coalesce 1, interleave 1,
    max_chunks 8, profile_level 0, validate_ptrs 1, sgemm_impl SVP_SGEMM_TF32BF16, rest 0

@@ -69,7 +69,8 @@ struct Dev {
     uint8_t* tbl_host = nullptr;
     uint8_t* tbl_dev = nullptr;
     size_t tbl_cap = 0;
-    std::vector<uint8_t> tbl_last;
+    std::vector<uint8_t> tbl_last;      // host copy of the current tables (param launches read it)
+    bool tbl_dev_valid = false;         // the device table buffer holds tbl_last
     LaunchLimits lim;
     std::unordered_map<MapKey, Maps2, MapKeyHash> map_cache;
     std::string err;
@@ -327,6 +328,7 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             }
             ch.total_tiles = tiles;
             ch.nsegs = (int32_t)ch.jobs.size();
+            ch.param = e->c->cfg.table_mode == SVP_TABLE_PARAM && ch.nsegs <= kParamSegs;
         } else {
             // tcgen05 tiles for sgemm_tf32 and for sgemm with the 3xTF32 implementation
             const int variant = (ch.kernel == K_SGEMM_TF32 || e->c->cfg.sgemm_impl != SVP_SGEMM_FFMA) ? 1 : 0;
@@ -393,12 +395,28 @@ static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bo
 }
 
 static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStream_t s) {
-    if (ch.total_tiles == 0) return cudaSuccess;
+    if (ch.total_tiles == 0 && ch.kernel != K_HIST256) return cudaSuccess;
     const uint8_t* base = d.tbl_dev;
     auto grid_of = [&](int per_sm) {
         if (ch.co_grid > 0) per_sm = std::min(per_sm, (int)ch.co_grid);
-        return (int)std::min<uint64_t>(ch.total_tiles, (uint64_t)d.lim.num_sms * per_sm);
+        return (int)std::max<uint64_t>(1, std::min<uint64_t>(ch.total_tiles, (uint64_t)d.lim.num_sms * per_sm));
     };
+    if (ch.param) {
+        // table by value: copied into the launch's parameter buffer at enqueue time
+        SegParam p;
+        memcpy(&p, d.tbl_last.data() + ch.table_off, (size_t)ch.nsegs * sizeof(SegDesc));
+        switch (ch.kernel) {
+            case K_VECADD:
+            case K_SAXPY: return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.ew_blocks_per_sm), s);
+            case K_BLACKSCHOLES:
+                return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.bs_blocks_per_sm), s);
+            case K_EW_MIX:
+                return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.mix_blocks_per_sm), s);
+            case K_HIST256:
+                return launch_hist256_param(p, ch.nsegs, ch.total_tiles, grid_of(d.lim.hist_blocks_per_sm), s);
+        }
+        return cudaErrorInvalidValue;
+    }
     switch (ch.kernel) {
         case K_VECADD:
             return launch_vecadd((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
@@ -485,29 +503,39 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
         CK(cudaEventRecord(d.ext_ev, d.ext));
         for (auto s : d.streams) CK(cudaStreamWaitEvent(s, d.ext_ev, 0));
     }
-    bool upload = !f.reused && !tbl.empty() &&
-                  (tbl.size() != d.tbl_last.size() || memcmp(tbl.data(), d.tbl_last.data(), tbl.size()));
+    // tables changed -> new host copy; the device copy is refreshed only if some launch on
+    // this GPU reads the global table (param-mode launches carry theirs by value)
+    if (!f.reused && !tbl.empty() &&
+        (tbl.size() != d.tbl_last.size() || memcmp(tbl.data(), d.tbl_last.data(), tbl.size()))) {
+        d.tbl_last.swap(tbl);
+        d.tbl_dev_valid = false;
+    }
+    bool need_dev = false;
+    for (const auto& ch : f.chunks)
+        if (ch.device == d.idx && !ch.param && chunk_needs_launch(f, ch)) need_dev = true;
+    const bool upload = need_dev && !d.tbl_dev_valid && !d.tbl_last.empty();
     if (upload) {
-        if (tbl.size() > d.tbl_cap) {
+        const size_t bytes = d.tbl_last.size();
+        if (bytes > d.tbl_cap) {
             if (d.tbl_dev) CK(cudaFree(d.tbl_dev));
             if (d.tbl_host) CK(cudaFreeHost(d.tbl_host));
             d.tbl_dev = nullptr;
             d.tbl_host = nullptr;
-            size_t cap = align_up(tbl.size() * 2, 1 << 16);
+            size_t cap = align_up(bytes * 2, 1 << 16);
             CK(cudaMalloc(&d.tbl_dev, cap));
             CK(cudaHostAlloc(&d.tbl_host, cap, cudaHostAllocDefault));
             d.tbl_cap = cap;
         }
-        memcpy(d.tbl_host, tbl.data(), tbl.size());
-        CK(cudaMemcpyAsync(d.tbl_dev, d.tbl_host, tbl.size(), cudaMemcpyHostToDevice, d.streams[0]));
+        memcpy(d.tbl_host, d.tbl_last.data(), bytes);
+        CK(cudaMemcpyAsync(d.tbl_dev, d.tbl_host, bytes, cudaMemcpyHostToDevice, d.streams[0]));
         CK(cudaEventRecord(d.tbl_ev, d.streams[0]));
         for (size_t s = 1; s < d.streams.size(); ++s) CK(cudaStreamWaitEvent(d.streams[s], d.tbl_ev, 0));
-        d.tbl_last.swap(tbl);
+        d.tbl_dev_valid = true;
         ++d.table_uploads;
         {
             std::lock_guard<std::mutex> lk(c->pmu);  // one worker thread per GPU updates fstats
             c->fstats.table_uploads += 1;
-            c->fstats.table_bytes += d.tbl_last.size();
+            c->fstats.table_bytes += bytes;
         }
     }
     // ---- steady-state replay: second sighting of a plan -> capture, later -> replay

@@ -9,12 +9,13 @@ namespace svp {
 
 // Segment owning launch tile t: the last segment with tile_begin <= t.  Empty
 // segments share their tile_begin with the next one, so upper_bound - 1 lands on the
-// segment that actually owns the tile.
+// segment that actually owns the tile.  Plain loads: `segs` is a global table or the
+// address of a __grid_constant__ SegParam (table_mode param).
 __device__ __forceinline__ int find_seg(const SegDesc* __restrict__ segs, int nsegs, uint32_t t) {
     int lo = 0, hi = nsegs;
     while (lo < hi) {
         int mid = (lo + hi) >> 1;
-        if (__ldg(&segs[mid].tile_begin) <= t) lo = mid + 1;
+        if (segs[mid].tile_begin <= t) lo = mid + 1;
         else hi = mid;
     }
     return lo - 1;

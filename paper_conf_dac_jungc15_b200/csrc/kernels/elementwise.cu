@@ -233,14 +233,22 @@ __device__ __forceinline__ void bs_tile(const SegDesc& sd, uint32_t lt) {
 }
 
 // --------------------------------------------------------------------- kernels
-// Homogeneous coalesced launches: every segment runs the same tile body.
+// Homogeneous coalesced launches: every segment runs the same tile body.  NAME reads a
+// global segment table, NAME##_p receives it by value (table_mode param).
 #define SVP_EW_KERNEL(NAME, BODY)                                                               \
-    __global__ void __launch_bounds__(kEwThreads) NAME(const SegDesc* __restrict__ segs, int nsegs, \
-                                                       uint32_t total) {                        \
+    __device__ __forceinline__ void NAME##_loop(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) { \
         for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {                              \
             const SegDesc& sd = segs[find_seg(segs, nsegs, t)];                                 \
             BODY(sd, t - sd.tile_begin);                                                        \
         }                                                                                       \
+    }                                                                                           \
+    __global__ void __launch_bounds__(kEwThreads) NAME(const SegDesc* __restrict__ segs, int nsegs, \
+                                                       uint32_t total) {                        \
+        NAME##_loop(segs, nsegs, total);                                                        \
+    }                                                                                           \
+    __global__ void __launch_bounds__(kEwThreads) NAME##_p(const __grid_constant__ SegParam p, int nsegs, \
+                                                           uint32_t total) {                    \
+        NAME##_loop(p.s, nsegs, total);                                                         \
     }
 SVP_EW_KERNEL(k_vecadd, vecadd_tile)
 SVP_EW_KERNEL(k_saxpy, saxpy_tile)
@@ -251,18 +259,14 @@ SVP_EW_KERNEL(k_blackscholes, bs_tile)
 // flags, each segment keeps its own tile size, and the tile bodies are the ones above, so
 // every element is computed by exactly the same instructions as in its homogeneous launch
 // (results bit-identical).  The branch is uniform per CTA (a tile lies in one segment).
-__global__ void __launch_bounds__(kEwThreads) k_ew_mix(const SegDesc* __restrict__ segs, int nsegs,
-                                                       uint32_t total) {
-    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
-        const SegDesc& sd = segs[find_seg(segs, nsegs, t)];
-        const uint32_t lt = t - sd.tile_begin;
-        switch (sd.flags >> SEG_KIND_SHIFT) {
-            case 1: vecadd_tile(sd, lt); break;  // K_VECADD
-            case 2: saxpy_tile(sd, lt); break;   // K_SAXPY
-            default: bs_tile(sd, lt); break;     // K_BLACKSCHOLES
-        }
+__device__ __forceinline__ void mix_tile(const SegDesc& sd, uint32_t lt) {
+    switch (sd.flags >> SEG_KIND_SHIFT) {
+        case 1: vecadd_tile(sd, lt); break;  // K_VECADD
+        case 2: saxpy_tile(sd, lt); break;   // K_SAXPY
+        default: bs_tile(sd, lt); break;     // K_BLACKSCHOLES
     }
 }
+SVP_EW_KERNEL(k_ew_mix, mix_tile)
 
 // --------------------------------------------------------------------- launchers
 cudaError_t launch_vecadd(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
@@ -280,6 +284,17 @@ cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total, 
 
 cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
     k_ew_mix<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_ew_param(int kind, const SegParam& p, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+    switch (kind) {
+        case 1: k_vecadd_p<<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
+        case 2: k_saxpy_p<<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
+        case 4: k_blackscholes_p<<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
+        case 8: k_ew_mix_p<<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
+        default: return cudaErrorInvalidValue;
+    }
     return cudaGetLastError();
 }
 

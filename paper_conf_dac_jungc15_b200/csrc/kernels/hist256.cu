@@ -31,11 +31,17 @@ constexpr int kHistStages = 3;
 constexpr int kHistBins = 256;
 constexpr int kHistSmem = kHistStages * kHistTile + kHistBins * 32 * 4 + 2 * kHistStages * 8 + 128;
 
-__global__ void __launch_bounds__(256) k_hist_zero(const SegDesc* __restrict__ segs, int nsegs) {
+__device__ __forceinline__ void hist_zero_body(const SegDesc* __restrict__ segs, int nsegs) {
     for (int s = blockIdx.x; s < nsegs; s += gridDim.x) {
         uint32_t* counts = reinterpret_cast<uint32_t*>(segs[s].ptr[1]);
         counts[threadIdx.x] = 0u;
     }
+}
+__global__ void __launch_bounds__(256) k_hist_zero(const SegDesc* __restrict__ segs, int nsegs) {
+    hist_zero_body(segs, nsegs);
+}
+__global__ void __launch_bounds__(256) k_hist_zero_p(const __grid_constant__ SegParam p, int nsegs) {
+    hist_zero_body(p.s, nsegs);
 }
 
 __device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kHistConsumers) : "memory"); }
@@ -90,7 +96,7 @@ struct SegCache {
     }
 };
 
-__global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
+__device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
     extern __shared__ __align__(128) uint8_t hsm[];
     uint8_t* ring = hsm;                                                         // [stages][tile]
     uint32_t* h = reinterpret_cast<uint32_t*>(hsm + kHistStages * kHistTile);     // [256][32]
@@ -191,20 +197,45 @@ __global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restric
     if (cur >= 0) hist_flush(h, cur_counts);
 }
 
+__global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
+    hist_body(segs, nsegs, total);
+}
+__global__ void __launch_bounds__(kHistBlock) k_hist256_p(const __grid_constant__ SegParam p, int nsegs,
+                                                          uint32_t total) {
+    hist_body(p.s, nsegs, total);
+}
+
+static cudaError_t hist_attr() {
+    static bool attr[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 64 && !attr[dev]) {
+        cudaError_t e = cudaFuncSetAttribute(k_hist256, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmem);
+        if (e) return e;
+        e = cudaFuncSetAttribute(k_hist256_p, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmem);
+        if (e) return e;
+        attr[dev] = true;
+    }
+    return cudaSuccess;
+}
+
 cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
     if (nsegs <= 0) return cudaSuccess;
     k_hist_zero<<<nsegs < 1024 ? nsegs : 1024, 256, 0, s>>>(segs, nsegs);
     cudaError_t e = cudaGetLastError();
     if (e || total == 0) return e;
-    static bool attr[64] = {};
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (dev < 64 && !attr[dev]) {
-        e = cudaFuncSetAttribute(k_hist256, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmem);
-        if (e) return e;
-        attr[dev] = true;
-    }
+    if ((e = hist_attr())) return e;
     k_hist256<<<grid, kHistBlock, kHistSmem, s>>>(segs, nsegs, total);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_hist256_param(const SegParam& p, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+    if (nsegs <= 0) return cudaSuccess;
+    k_hist_zero_p<<<nsegs < 1024 ? nsegs : 1024, 256, 0, s>>>(p, nsegs);
+    cudaError_t e = cudaGetLastError();
+    if (e || total == 0) return e;
+    if ((e = hist_attr())) return e;
+    k_hist256_p<<<grid, kHistBlock, kHistSmem, s>>>(p, nsegs, total);
     return cudaGetLastError();
 }
 

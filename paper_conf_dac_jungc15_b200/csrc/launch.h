@@ -30,6 +30,10 @@ cudaError_t launch_saxpy(const SegDesc* segs, int nsegs, uint32_t total_tiles, i
 cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
 // Heterogeneous elementwise launch: segment kernel id in flags >> SEG_KIND_SHIFT.
 cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
+// table_mode param: the same kernels with the segment table passed by value; kind = kernel
+// id (1 vecadd, 2 SAXPY, 4 Black-Scholes, 8 mixed), nsegs <= kParamSegs.
+cudaError_t launch_ew_param(int kind, const SegParam& p, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
+cudaError_t launch_hist256_param(const SegParam& p, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
 // hist256: zeroes each segment's 256 counters, then accumulates.
 cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
 

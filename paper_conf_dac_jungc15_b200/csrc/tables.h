@@ -26,6 +26,14 @@ struct SegDesc {
 static_assert(sizeof(SegDesc) == 64, "SegDesc must be 64 B");
 enum : uint16_t { SEG_SCALAR = 1, SEG_KIND_SHIFT = 8 };
 
+// table_mode = SVP_TABLE_PARAM: a launch of at most kParamSegs segments receives its table
+// by value as a __grid_constant__ kernel parameter (15 KiB of the 32 KiB parameter space):
+// no table upload and segment reads served from the constant cache.
+constexpr int kParamSegs = 240;
+struct SegParam {
+    SegDesc s[kParamSegs];
+};
+
 // Grouped SGEMM: one entry per VP; tensor maps live in a separate 64-B aligned array
 // (2 per VP: A then B).
 struct GemmDesc {

@@ -25,6 +25,7 @@ MEM_DEVICE, MEM_HOST_PINNED = 0, 1
 OP_H2D, OP_KERNEL, OP_D2H = 0, 1, 2
 SGEMM_FFMA, SGEMM_3XTF32, SGEMM_TF32BF16 = 0, 1, 2
 KERNEL_EW_MIX = 8  # heterogeneous elementwise launch (cfg hetero): plan/kernel-stats id only
+TABLE_GLOBAL, TABLE_PARAM = 0, 1
 MAX_BUFS, MAX_ARGS = 5, 64
 
 # ABI symbols declared in include/svp.h (tests check every one is exported)
@@ -44,7 +45,7 @@ class svp_config(C.Structure):
                 ("sgemm_impl", C.c_int32),
                 ("external_streams", C.POINTER(C.c_void_p)), ("hbm_gbps", C.c_double), ("pcie_gbps", C.c_double),
                 ("ffma_tflops", C.c_double), ("launch_us", C.c_double), ("hetero", C.c_int32),
-                ("graph", C.c_int32)]
+                ("graph", C.c_int32), ("table_mode", C.c_int32)]
 
 
 class svp_buf(C.Structure):
@@ -226,7 +227,8 @@ class Context:
                  profile_level: int = 0, sync_each_job: bool = False, dry_run: bool = False,
                  flush_timeout_ms: int = 0, validate_ptrs: bool = True, sgemm_impl: int = SGEMM_TF32BF16,
                  external_streams: Optional[Sequence[int]] = None, hbm_gbps: float = 0.0, pcie_gbps: float = 0.0,
-                 ffma_tflops: float = 0.0, launch_us: float = 0.0, hetero: bool = False, graph: bool = False):
+                 ffma_tflops: float = 0.0, launch_us: float = 0.0, hetero: bool = False, graph: bool = False,
+                 table_mode: int = TABLE_GLOBAL):
         L = load()
         cfg = svp_config()
         L.svp_config_default(C.byref(cfg))
@@ -252,7 +254,7 @@ class Context:
             self._ext = (C.c_void_p * len(external_streams))(*external_streams)
             cfg.external_streams = C.cast(self._ext, C.POINTER(C.c_void_p))
         cfg.hbm_gbps, cfg.pcie_gbps, cfg.ffma_tflops, cfg.launch_us = hbm_gbps, pcie_gbps, ffma_tflops, launch_us
-        cfg.hetero, cfg.graph = int(hetero), int(graph)
+        cfg.hetero, cfg.graph, cfg.table_mode = int(hetero), int(graph), int(table_mode)
         h = C.c_void_p()
         _check(L.svp_init(C.byref(cfg), C.byref(h)))
         self._h = h

@@ -23,7 +23,7 @@ def test_library_exports_every_declared_symbol():
     assert set(declared) == set(svp.EXPORTS), (set(declared) ^ set(svp.EXPORTS))
     for name in declared:
         assert hasattr(L, name), name
-    assert L.svp_abi_version() == 2
+    assert L.svp_abi_version() == 3
 
 
 def test_lib_is_the_in_tree_build():
@@ -200,3 +200,11 @@ def test_ew_mix_id_is_stats_only():
         with pytest.raises(svp.SvpError) as e:
             c.submit(0, svp.KERNEL_EW_MIX, svp.args_vecadd(4), _vecadd_bufs(4))
         assert e.value.status == svp.SVP_E_NOKERNEL
+
+
+def test_table_mode_values():
+    with svp.Context(dry_run=True, table_mode=svp.TABLE_PARAM):
+        pass
+    with pytest.raises(svp.SvpError) as e:
+        svp.Context(dry_run=True, table_mode=2)
+    assert e.value.status == svp.SVP_E_INVAL

@@ -124,3 +124,50 @@ def test_serial_graph_baseline_b3(small):
             check_job(s, inp, vs.output(i))
     finally:
         ctx.close()
+
+
+@pytest.mark.parametrize("residency", ["device", "host"])
+@pytest.mark.parametrize("hetero", [False, True])
+def test_table_mode_param(small, residency, hetero):
+    """SURVEY §8(b) table_mode: segment tables passed by value (kernel parameter) give the
+    same bits as the global table; GEMM launches keep the global table."""
+    specs, inputs = small
+    a, _, sa = run_svp(specs, inputs, residency, table_mode=svp.TABLE_PARAM, hetero=hetero)
+    b, _, _ = run_svp(specs, inputs, residency, table_mode=svp.TABLE_GLOBAL, hetero=hetero)
+    for s, inp, x, y in zip(specs, inputs, a, b):
+        check_job(s, inp, x)
+        for k in x:
+            assert np.array_equal(_bits(x[k]), _bits(y[k])), (s.vp, s.kernel, k)
+
+
+def test_table_mode_param_no_upload_and_fallback():
+    """Elementwise-only flushes in param mode upload no table; a group larger than the
+    parameter table (240 VPs) falls back to the global table and stays correct."""
+    few = [W.JobSpec(v, ("vecadd", "saxpy", "hist256", "blackscholes")[v % 4], n=5000 + 77 * v) for v in range(40)]
+    many = [W.JobSpec(v, "vecadd", n=1000 + 13 * v) for v in range(300)]
+    for specs, uploads in ((few, 0), (many, 1)):
+        inputs = inputs_for(specs)
+        outs, _, st = run_svp(specs, inputs, "device", table_mode=svp.TABLE_PARAM)
+        assert st["table_uploads"] == uploads
+        for s, inp, got in zip(specs, inputs, outs):
+            check_job(s, inp, got)
+
+
+def test_table_mode_param_with_graph(small):
+    specs, _ = small
+    ctx = svp.Context(num_gpus=1, graph=True, table_mode=svp.TABLE_PARAM)
+    try:
+        vs = VPSet(ctx, specs, None, "device")
+        jb = svp.JobBatch(vs.job_list())
+        for r in range(3):
+            inputs = inputs_for(specs, seed=W.BASE_SEED + 5 * r)
+            vs.inputs = inputs
+            vs.load_inputs()
+            ctx.submit_batch(jb)
+            ctx.flush()
+            torch.cuda.synchronize()
+            for i, (s, inp) in enumerate(zip(specs, inputs)):
+                check_job(s, inp, vs.output(i))
+        assert ctx.flush_stats()["graph_replays"] == 1
+    finally:
+        ctx.close()
