@@ -526,7 +526,7 @@ def main():
                     help="heterogeneous coalescing of vecadd/SAXPY/Black-Scholes (NEXT f4)")
     ap.add_argument("--graph", type=int, default=0, choices=[0, 1],
                     help="steady-state plan reuse + CUDA graph replay (NEXT f4)")
-    ap.add_argument("--table-mode", type=int, default=0, choices=[0, 1],
+    ap.add_argument("--table-mode", type=int, default=1, choices=[0, 1],
                     help="segment tables: 0 global device buffer, 1 by-value kernel parameter")
     ap.add_argument("--no-serial", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other sgemm implementation")

@@ -96,18 +96,19 @@ typedef struct svp_config {
                                     repeat on replays the flush's device work as one CUDA
                                     graph per GPU.  Ignored with sync_each_job.              */
     int32_t table_mode;          /* where a coalesced launch finds its segment table (SURVEY
-                                    §8(b)): SVP_TABLE_GLOBAL (default) -- one device table
-                                    buffer per GPU, uploaded once per flush when it changed;
-                                    SVP_TABLE_PARAM -- launches of elementwise / hist256
-                                    groups with <= 240 VPs receive it by value as a kernel
-                                    parameter (no upload; GEMM launches always use global) */
+                                    §8(b)): SVP_TABLE_PARAM (default) -- launches of
+                                    elementwise / hist256 groups with <= 240 VPs receive it
+                                    by value as a kernel parameter (no upload; cfg5 measured
+                                    +4 % over global); SVP_TABLE_GLOBAL -- one device table
+                                    buffer per GPU, uploaded once per flush when it changed.
+                                    GEMM launches always use the global table.             */
 } svp_config;
 
 enum { SVP_TABLE_GLOBAL = 0, SVP_TABLE_PARAM = 1 };
 
 /* Fill *cfg with defaults: num_gpus 0, 4 compute streams, coalesce 1, interleave 1,
-   max_chunks 8, profile_level 0, validate_ptrs 1, sgemm_impl SVP_SGEMM_TF32BF16, rest 0
-   (hetero 0, graph 0). */
+   max_chunks 8, profile_level 0, validate_ptrs 1, sgemm_impl SVP_SGEMM_TF32BF16,
+   table_mode SVP_TABLE_PARAM, rest 0 (hetero 0, graph 0). */
 void svp_config_default(svp_config* cfg);
 
 /* Create a context.  On success *out owns streams/events/threads for every GPU.

@@ -95,6 +95,7 @@ void svp_config_default(svp_config* cfg) {
     cfg->profile_level = 0;
     cfg->validate_ptrs = 1;
     cfg->sgemm_impl = SVP_SGEMM_TF32BF16;
+    cfg->table_mode = SVP_TABLE_PARAM;
 }
 
 svp_status svp_init(const svp_config* cfg, svp_ctx** out) {

@@ -228,7 +228,7 @@ class Context:
                  flush_timeout_ms: int = 0, validate_ptrs: bool = True, sgemm_impl: int = SGEMM_TF32BF16,
                  external_streams: Optional[Sequence[int]] = None, hbm_gbps: float = 0.0, pcie_gbps: float = 0.0,
                  ffma_tflops: float = 0.0, launch_us: float = 0.0, hetero: bool = False, graph: bool = False,
-                 table_mode: int = TABLE_GLOBAL):
+                 table_mode: int = TABLE_PARAM):
         L = load()
         cfg = svp_config()
         L.svp_config_default(C.byref(cfg))
