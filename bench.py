@@ -116,14 +116,21 @@ def my_specs(specs, rank, ws):
 
 
 class Clocks:
-    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    """nvidia-smi sampling of the timed region (B200_PROFILING.md clocks line).
 
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+    The sampler starts before the warm-up (nvidia-smi takes ~0.1-0.3 s to emit its first
+    line, longer than a short timed region), stamps every sample, and `stop()` keeps the
+    samples whose timestamps fall inside [mark_start(), mark_end()]; if fewer than 3 do,
+    the nearest samples around the window are added and `in_window` says how many were
+    strictly inside."""
+
+    Q = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
     def __init__(self, device_index: int):
         self.p = None
+        self.t0 = self.t1 = None
         self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
         try:
             import torch
@@ -133,14 +140,31 @@ class Clocks:
             ident = []
         try:
             self.p = subprocess.Popen(["nvidia-smi"] + ident + ["--query-gpu=" + self.Q, "--format=csv,noheader,nounits",
-                                                                 "-lms", "50"], stdout=self.f, stderr=subprocess.DEVNULL)
+                                                                 "-lms", "20"], stdout=self.f, stderr=subprocess.DEVNULL)
+            deadline = time.time() + 5.0
+            while time.time() < deadline and os.path.getsize(self.f.name) == 0:
+                time.sleep(0.02)
         except Exception:
             self.p = None
+
+    def mark_start(self):
+        self.t0 = time.time()
+
+    def mark_end(self):
+        self.t1 = time.time()
+
+    @staticmethod
+    def _ts(text):
+        import datetime
+        try:
+            return datetime.datetime.strptime(text.strip(), "%Y/%m/%d %H:%M:%S.%f").timestamp()
+        except ValueError:
+            return None
 
     def stop(self):
         if self.p is None:
             return None
-        time.sleep(0.06)
+        time.sleep(0.1)
         self.p.terminate()
         try:
             self.p.wait(timeout=5)
@@ -148,24 +172,32 @@ class Clocks:
             self.p.kill()
         self.f.flush()
         self.f.seek(0)
-        sm, mx, reasons = [], [], set()
+        rows = []
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for line in self.f.read().splitlines():
             parts = [x.strip() for x in line.split(",")]
-            if len(parts) < 9:
+            if len(parts) < 10:
                 continue
             try:
-                sm.append(float(parts[1]))
-                mx.append(float(parts[2]))
+                rows.append((self._ts(parts[0]), float(parts[2]), float(parts[3]), parts[6:10]))
             except ValueError:
                 continue
-            for nm, val in zip(names, parts[5:9]):
+        os.unlink(self.f.name)
+        rows = [r for r in rows if r[0] is not None]
+        if not rows or self.t0 is None or self.t1 is None:
+            return None
+        inside = [r for r in rows if self.t0 <= r[0] <= self.t1]
+        sel = list(inside)
+        if len(sel) < 3:  # short window: add the samples nearest to it
+            mid = 0.5 * (self.t0 + self.t1)
+            sel = sorted(rows, key=lambda r: abs(r[0] - mid))[:3]
+        reasons = set()
+        for r in sel:
+            for nm, val in zip(names, r[3]):
                 if val.lower().startswith("active"):
                     reasons.add(nm)
-        os.unlink(self.f.name)
-        if not sm:
-            return None
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "samples": len(sm),
+        return {"sm_mhz": statistics.median(r[1] for r in sel), "sm_max_mhz": max(r[2] for r in sel),
+                "samples": len(sel), "in_window": len(inside), "window_ms": (self.t1 - self.t0) * 1e3,
                 "reasons": sorted(reasons)}
 
 
@@ -283,14 +315,17 @@ def run_svp(args, rank, ws, local):
     ctx.submit_batch(jobs)
     ctx.flush()
     torch.cuda.synchronize()
+    clocks = Clocks(local)  # sampling starts before the warm-up (nvidia-smi start-up latency)
     for _ in range(max(0, args.warmup - 1)):
         ctx.submit_batch(jobs)
         ctx.flush()
     ctx.reset_profile()
     barrier(ws)
     trace("warmup done, timing")
-    clocks = Clocks(local)
+    torch.cuda.synchronize()
+    clocks.mark_start()
     dt = timed_steps(ctx, jobs, args.steps, stream)
+    clocks.mark_end()
     clk = clocks.stop()
     barrier(ws)
     dt_max = max_over_ranks(dt, ws)
