@@ -271,3 +271,47 @@ def test_dgemm_both_tile_variants():
         outs, _, _ = run_svp(specs, inputs, "device")
         for s, inp, got in zip(specs, inputs, outs):
             check_job(s, inp, got)
+
+
+def test_config5_bench_launch_config():
+    """BASELINE config 5 at full size in exactly the configuration bench.py times (256 VPs,
+    device-resident, interleaved, by-value segment tables, TF32+2xBF16 SGEMM on CTA pairs,
+    pre-marshalled JobBatch resubmitted per step): every memory-bound VP compared in full,
+    every SGEMM VP on 24 sampled elements (oracle.sgemm_element), over two consecutive
+    steps (the second SAXPY step reads the first one's y; tables are reused)."""
+    specs = W.config_specs(5)
+    inputs = W.make_inputs_many(specs)
+    stream = torch.cuda.current_stream()
+    ctx = svp.Context(num_gpus=1, device_ids=[0], profile_level=1, external_streams=[stream.cuda_stream],
+                      validate_ptrs=True, sgemm_impl=svp.SGEMM_TF32BF16, hetero=False, graph=False,
+                      table_mode=svp.TABLE_PARAM)
+    try:
+        vs = VPSet(ctx, specs, inputs, "device", device_ordinals=[0])
+        jobs = svp.JobBatch(vs.job_list())
+        g = np.random.default_rng(5)
+        prev = [dict(inp) for inp in inputs]
+        for step in range(2):
+            ctx.submit_batch(jobs)
+            ctx.flush()
+            torch.cuda.synchronize()
+            st = ctx.flush_stats()
+            assert st["groups"] == 5, st
+            mb = [i for i, s in enumerate(specs) if s.kernel != "sgemm"]
+            want = oracle.run_jobs([specs[i] for i in mb], [prev[i] for i in mb])
+            outs = {}
+            for i, w in zip(mb, want):
+                got = vs.output(i)
+                check_job(specs[i], prev[i], got, w)
+                outs[i] = got
+            for i, s in enumerate(specs):
+                if s.kernel != "sgemm":
+                    continue
+                sample = [(int(g.integers(0, s.M)), int(g.integers(0, s.N))) for _ in range(20)]
+                sample += [(0, 0), (s.M - 1, s.N - 1), (255, 256), (256, 255)]
+                check_job(s, inputs[i], vs.output(i), sample=sample)
+            for i, s in enumerate(specs):  # the next step's SAXPY reads this step's y
+                if s.kernel == "saxpy":
+                    prev[i] = dict(prev[i], y=outs[i]["y"].copy())
+        assert vs.guards_intact()
+    finally:
+        ctx.close()
