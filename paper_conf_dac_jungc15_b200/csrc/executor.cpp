@@ -333,7 +333,22 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             // tcgen05 tiles for sgemm_tf32 and for sgemm with the 3xTF32 implementation
             const int variant = (ch.kernel == K_SGEMM_TF32 || e->c->cfg.sgemm_impl != SVP_SGEMM_FFMA) ? 1 : 0;
             const bool pair = variant && ch.kernel == K_SGEMM && sgemm_tc_cta_pair();
-            const int BM = variant ? (pair ? 2 * kTf32BM : kTf32BM) : kGemmBM, BN = variant ? kTf32BN : kGemmBN;
+            // wide (256 x 512) pair tiles halve the A-side conversion and L2 traffic per flop
+            // but halve the tile count: used when they still fill >= 2 waves of CTA pairs
+            bool wide = false;
+            if (pair && e->c->cfg.sgemm_impl == SVP_SGEMM_TF32BF16) {
+                const int mode = sgemm_tc_wide_mode();
+                uint64_t tw = 0;
+                for (int32_t ji : ch.jobs) {
+                    const Job& j = f.jobs[ji];
+                    if ((int64_t)j.M * j.N > 0)
+                        tw += (uint64_t)((j.M + 2 * kTf32BM - 1) / (2 * kTf32BM)) * ((j.N + 2 * kTf32BN - 1) / (2 * kTf32BN));
+                }
+                wide = mode == 2 || (mode == 1 && tw >= 2ull * (uint64_t)(d.lim.num_sms / 2));
+            }
+            ch.wide = wide;
+            const int BM = variant ? (pair ? 2 * kTf32BM : kTf32BM) : kGemmBM;
+            const int BN = variant ? (wide ? 2 * kTf32BN : kTf32BN) : kGemmBN;
             ch.maps_off = align_up(tbl.size(), 128);
             size_t nj = ch.jobs.size();
             ch.table_off = ch.maps_off + nj * 256;
@@ -436,7 +451,7 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
         case K_SGEMM:
             if (sgemm_impl == SVP_SGEMM_TF32BF16)
                 return launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
-                                             ch.total_tiles, grid_of(1), s);
+                                             ch.total_tiles, grid_of(1), ch.wide, s);
             if (sgemm_impl == SVP_SGEMM_3XTF32)
                 return launch_sgemm_3xtf32((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
                                            ch.total_tiles, grid_of(1), s);

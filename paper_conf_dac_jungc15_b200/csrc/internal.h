@@ -94,6 +94,7 @@ struct Chunk {
     int32_t nsegs = 0;
     uint64_t maps_off = 0;          // sgemm: tensor maps offset
     bool small_tiles = false;       // dgemm: 32x32 tile variant (launch under 2 waves of 64x64)
+    bool wide = false;              // sgemm TF32+2xBF16: 256x512 pair tiles (>= 2 waves of them)
     bool param = false;             // table_mode param: the SegDesc table goes by value
     int32_t co_grid = 0;            // >0: launch with co_grid CTAs per SM so the kernel
                                     // co-resides with a tensor-core SGEMM on the same SMs

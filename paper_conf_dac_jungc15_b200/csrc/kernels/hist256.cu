@@ -167,8 +167,6 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
             uint4 r[kHistVec];
 #pragma unroll
             for (int i = 0; i < kHistVec; ++i) r[i] = st[i * kHistConsumers];
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&empty[s]);  // stage consumed (data now in registers)
 #pragma unroll
             for (int i = 0; i < kHistVec; ++i) {
                 hist_add_word(hl, r[i].x);
@@ -176,6 +174,12 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
                 hist_add_word(hl, r[i].z);
                 hist_add_word(hl, r[i].w);
             }
+            // Release the stage only after every loaded word was consumed: the mbarrier
+            // arrive (SYNCS unit) does not wait for this warp's outstanding LDS, so an
+            // arrive issued right after them let the producer's next bulk copy overwrite
+            // bytes not yet read (wrong-but-conserved counts under heavy co-scheduling).
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
         } else {
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);

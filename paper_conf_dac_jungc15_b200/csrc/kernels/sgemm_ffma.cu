@@ -143,6 +143,10 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
                     }
                 }
             }
+            // the stage is released to the TMA producer only once this warp's last LDS of it
+            // returned: an mbarrier arrive does not wait for outstanding shared loads
+            // (hist256.cu), so a membar.cta (MEMBAR + scoreboard drain) precedes it
+            __threadfence_block();
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
         }

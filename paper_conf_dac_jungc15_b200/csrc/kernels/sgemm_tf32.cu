@@ -61,6 +61,19 @@
 //   warps 4-7     epilogue: tcgen05.ld 32x32b.x32 (warp w%4 owns TMEM lanes = tile rows
 //                 32(w%4)..+31), alpha*acc (+ beta*C), 128-bit stores; two TMEM
 //                 accumulators let tile i's epilogue overlap tile i+1's MMAs.
+//
+// NH = 2 (wide, SPLIT 2 pairs): 256 x 512 tiles, 576 threads.  Each CTA stages 256 B
+// columns (two 128-column halves); per k-step the leader issues the SPLIT 2 MMAs once per
+// 256-column half into TMEM columns [0,256) / [256,512) -- the A tiles (and their bf16
+// conversions) serve both halves, halving the A-side conversion and L2 -> SM traffic per
+// flop (profiles/r01/power: the split SGEMM runs at the power cap, so energy per flop sets
+// its speed).  Warps 4-7 drain half 0 and warps 14-17 half 1, each half with its own
+// acc_full / acc_empty barrier, so the next tile's half-0 MMAs start while half 1 drains.
+// The executor uses NH 2 when a launch has >= 2 waves of wide tiles (SVP_TC_WIDE).
+//
+// Teardown: the producer waits for the release of the last use of every stage before the
+// CTA exits (tcgen05.commit arrives land asynchronously and must not reach the shared
+// memory of the next CTA scheduled on this SM).
 #include <cuda.h>
 #include <stdlib.h>
 
@@ -80,15 +93,20 @@ namespace tc {
 constexpr int BM = kTf32BM, BN = kTf32BN, BK = kTf32BK;  // 128 x 256 x 16 per CTA
 constexpr int kConvWarps = 8;                              // warps 2,3 and 8..13
 constexpr int kConvThreads = kConvWarps * 32;
-constexpr int kThreads = (8 + kConvWarps - 2) * 32;        // 448
+constexpr int kThreads = (8 + kConvWarps - 2) * 32;        // 448 (+128 for NH 2)
 constexpr int kTileA = BM * BK * 4;                        // 8 KiB
 constexpr int kBBlock = BK * 128;                          // one 32-n block of B: 2 KiB
 constexpr int kTmemCols = 512;
 constexpr int kTileA16 = BM * BK * 2;                      // 4 KiB
 
-template <int SPLIT, int CG>
+template <int SPLIT, int CG, int NH = 1>
 struct Cfg {
-    static constexpr int kBN = BN / CG;                    // B columns staged per CTA
+    // NH = 2 ("wide", SPLIT 2 pairs only): a pair computes 256 x 512, two 256-column MMA
+    // halves per k-step on the same A tiles; the two TMEM accumulators are the two halves
+    // of ONE tile (no double buffer), each drained by its own 4 epilogue warps.
+    static_assert(NH == 1 || (SPLIT == 2 && CG == 2), "wide tiles: TF32+2xBF16 CTA pairs only");
+    static constexpr int kThreads = tc::kThreads + (NH - 1) * 128;
+    static constexpr int kBN = BN / CG * NH;               // B columns staged per CTA
     static constexpr int kTileB = BK * kBN * 4;            // 16 KiB (CG 1) / 8 KiB (CG 2)
     static constexpr int kTileB16 = BK * kBN * 2;
     // stage: A | B [| A_lo | B_lo]   (SPLIT 2: A | B | bf A_hi | bf A_lo | bf B_hi | bf B_lo;
@@ -97,8 +115,9 @@ struct Cfg {
                                                   : (kTileA + kTileB) * (SPLIT == 1 ? 1 : 2);
     static constexpr int kStages = SPLIT == 1 ? 8
                                  : SPLIT == 4 ? (CG == 2 ? 8 : 5)
+                                 : NH == 2    ? 4
                                               : (CG == 2 ? SVP_PAIR_STAGES : 4);
-    static constexpr int kAcc = SPLIT == 4 ? 1 : 2;        // TMEM accumulators (256 cols each)
+    static constexpr int kAcc = (SPLIT == 4 || NH == 2) ? 1 : 2;  // accumulator sets (NH x 256 cols each)
     static constexpr int kTaCol = 256;                     // SPLIT 4: A ring, 16 cols per stage
     static_assert(SPLIT != 4 || kTaCol + 16 * kStages <= kTmemCols, "TMEM");
     static constexpr size_t kBarOff = (size_t)kStages * kStageBytes;
@@ -281,11 +300,12 @@ __device__ __forceinline__ void split8(const float4& p, const float4& q, uint4& 
 
 }  // namespace tc
 
-template <int SPLIT, int CG>
-__global__ void __launch_bounds__(tc::kThreads, 1)
+template <int SPLIT, int CG, int NH>
+__global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
     k_sgemm_tc(const GemmDesc* __restrict__ descs, int n, const uint8_t* __restrict__ maps, uint32_t total) {
     using namespace tc;
-    using C = Cfg<SPLIT, CG>;
+    using C = Cfg<SPLIT, CG, NH>;
+    constexpr int TN = BN * NH;  // tile width in N per CTA pair (or CTA)
     constexpr int ST = C::kStages, SB = C::kStageBytes, TB = C::kTileB, TB16 = C::kTileB16;
     extern __shared__ uint8_t smem_raw[];
     // align to 1024 B (swizzle atoms) by offsetting smem_raw itself, so the compiler keeps
@@ -356,7 +376,9 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                 }
                 const uint32_t lt = t - g.tile_begin;
                 const int tm = lt / g.tiles_n, tn = lt % g.tiles_n;
-                const int m0 = tm * C::kMmaM + (int)rank * BM, n0 = tn * BN + (int)rank * C::kBN;
+                const int m0 = tm * C::kMmaM + (int)rank * BM;
+                // 32-n block j of this CTA: half h = j / 4 (NH 2) at columns h*256 + rank*128
+                const int n0 = NH == 1 ? tn * BN + (int)rank * C::kBN : tn * TN + (int)rank * (BN / CG);
                 const int KB = (g.K + BK - 1) / BK;
                 for (int kb = 0; kb < KB; ++kb, ++it) {
                     const int s = it % ST;
@@ -366,9 +388,21 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                     mbar_expect_tx(&full[s], kTileA + TB);
                     tma_load_2d(sp, mA, kb * BK, m0, &full[s]);
 #pragma unroll
-                    for (int j = 0; j < C::kBN / 32; ++j)
-                        tma_load_2d(sp + kTileA + j * kBBlock, mB, n0 + j * 32, kb * BK, &full[s]);
+                    for (int j = 0; j < C::kBN / 32; ++j) {
+                        const int col = NH == 1 ? n0 + j * 32 : n0 + (j >> 2) * BN + (j & 3) * 32;
+                        tma_load_2d(sp + kTileA + j * kBBlock, mB, col, kb * BK, &full[s]);
+                    }
                 }
+            }
+            // Producer tail: the MMA issuer frees stages with tcgen05.commit, whose mbarrier
+            // arrives land asynchronously when the MMAs complete (multicast into both CTAs
+            // of a pair) -- possibly after the epilogue saw the last acc_full.  Wait for the
+            // release of the last use of every stage, so no arrive can land in this SM's
+            // shared memory after the CTA exited (it would corrupt whichever CTA of another
+            // kernel got the memory next: seen as wrong hist256 counts in the cfg5 mix).
+            for (uint32_t i = 0; i < (uint32_t)ST && i < it; ++i) {
+                const uint32_t u = it - 1 - i;
+                mbar_wait(&empty[u % ST], (u / ST) & 1);
             }
         }
     } else if (warp == 1) {
@@ -400,47 +434,64 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
                         const uint32_t s_al = s_bh + TB;
                         const uint32_t s_bl = s_al + kTileA;
 #pragma unroll
-                        for (int kk = 0; kk < BK / 8; ++kk) {
-                            const uint64_t ah = desc_a(s_ah + kk * 32);    // +8 k in a 64-B row
-                            const uint64_t bh = desc_b(s_bh + kk * 1024);  // +8 k rows of 128 B
-                            const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
-                            if (SPLIT == 3) {
-                                mma_tf32<CG>(tmem_d, ah, desc_b(s_bl + kk * 1024), acc0);
-                                mma_tf32<CG>(tmem_d, desc_a(s_al + kk * 32), bh, 1u);
-                                mma_tf32<CG>(tmem_d, ah, bh, 1u);
-                            } else {
-                                mma_tf32<CG>(tmem_d, ah, bh, acc0);
+                        for (int h = 0; h < NH; ++h) {
+                            // NH 2: half h = TMEM columns h*256, B blocks 4h..4h+3 (raw) /
+                            // 64-n atoms 2h, 2h+1 (bf16); its accumulator is free once the
+                            // previous tile's half-h epilogue drained it
+                            const int ab = NH == 1 ? a : h;
+                            if (NH == 2 && h == 1 && kb == 0) {
+                                mbar_wait_cluster(&acc_empty[1], aph ^ 1);
+                                tc_fence_after();
                             }
-                        }
-                        if (SPLIT == 2) {
-                            // cross terms on the bf16 tiles, K = 16 in one MMA each
-                            const uint32_t a16h = s_bh + TB, a16l = a16h + kTileA16;
-                            const uint32_t b16h = a16l + kTileA16, b16l = b16h + TB16;
-                            mma_bf16<CG>(tmem_d, desc_a16(a16h), desc_b16(b16l), 1u);
-                            mma_bf16<CG>(tmem_d, desc_a16(a16l), desc_b16(b16h), 1u);
-                        } else if (SPLIT == 4) {
-                            const uint32_t ta = tmem_base + (uint32_t)(C::kTaCol + 16 * s);
-                            const uint32_t b16h = s_bh + TB, b16l = b16h + TB16;
-                            mma_bf16_ta<CG>(tmem_d, ta, desc_b16(b16l), 1u);       // bf(A_hi) bf(B_lo)
-                            mma_bf16_ta<CG>(tmem_d, ta + 8, desc_b16(b16h), 1u);   // bf(A_lo) bf(B_hi)
+                            const uint32_t td = NH == 1 ? tmem_d : tmem_base + (uint32_t)(h * BN);
+                            const uint32_t bo = (uint32_t)h * (4 * kBBlock), bo16 = (uint32_t)h * 4096u;
+#pragma unroll
+                            for (int kk = 0; kk < BK / 8; ++kk) {
+                                const uint64_t ah = desc_a(s_ah + kk * 32);         // +8 k in a 64-B row
+                                const uint64_t bh = desc_b(s_bh + bo + kk * 1024);  // +8 k rows of 128 B
+                                const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
+                                if (SPLIT == 3) {
+                                    mma_tf32<CG>(td, ah, desc_b(s_bl + kk * 1024), acc0);
+                                    mma_tf32<CG>(td, desc_a(s_al + kk * 32), bh, 1u);
+                                    mma_tf32<CG>(td, ah, bh, 1u);
+                                } else {
+                                    mma_tf32<CG>(td, ah, bh, acc0);
+                                }
+                            }
+                            if (SPLIT == 2) {
+                                // cross terms on the bf16 tiles, K = 16 in one MMA each
+                                const uint32_t a16h = s_bh + TB, a16l = a16h + kTileA16;
+                                const uint32_t b16h = a16l + kTileA16 + bo16, b16l = b16h + TB16;
+                                mma_bf16<CG>(td, desc_a16(a16h), desc_b16(b16l), 1u);
+                                mma_bf16<CG>(td, desc_a16(a16l), desc_b16(b16h), 1u);
+                            } else if (SPLIT == 4) {
+                                const uint32_t ta = tmem_base + (uint32_t)(C::kTaCol + 16 * s);
+                                const uint32_t b16h = s_bh + TB, b16l = b16h + TB16;
+                                mma_bf16_ta<CG>(td, ta, desc_b16(b16l), 1u);      // bf(A_hi) bf(B_lo)
+                                mma_bf16_ta<CG>(td, ta + 8, desc_b16(b16h), 1u);  // bf(A_lo) bf(B_hi)
+                            }
+                            if (kb == KB - 1) mma_commit<CG>(&acc_full[ab]);
                         }
                         mma_commit<CG>(&empty[s]);
-                        if (kb == KB - 1) mma_commit<CG>(&acc_full[a]);
                     }
                     __syncwarp();
                 }
                 if (KB == 0 && lane == 0) {  // K == 0: nothing accumulated
-                    if constexpr (CG == 2) {
-                        mbar_arrive_cluster(map_to(&acc_full[a], 0));
-                        mbar_arrive_cluster(map_to(&acc_full[a], 1));
-                    } else {
-                        mbar_arrive(&acc_full[a]);
+                    for (int h = 0; h < NH; ++h) {
+                        const int ab = NH == 1 ? a : h;
+                        if (NH == 2 && h == 1) mbar_wait_cluster(&acc_empty[1], aph ^ 1);
+                        if constexpr (CG == 2) {
+                            mbar_arrive_cluster(map_to(&acc_full[ab], 0));
+                            mbar_arrive_cluster(map_to(&acc_full[ab], 1));
+                        } else {
+                            mbar_arrive(&acc_full[ab]);
+                        }
                     }
                 }
                 __syncwarp();
             }
         }
-    } else if (warp < 4 || warp >= 8) {
+    } else if (warp < 4 || (warp >= 8 && warp < 14)) {
         // ------------------------------------------------------------ converters
         const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;  // 0..255
         const uint32_t conv_leader0 = CG == 2 ? map_to(&conv[0], 0) : 0;
@@ -545,8 +596,10 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
             }
         }
     } else {
-        // ------------------------------------------------------------ epilogue (warps 4-7)
+        // ------------------------------------------------------------ epilogue (warps 4-7;
+        // NH 2: warps 4-7 drain half 0, warps 14-17 half 1)
         const int q = warp & 3;  // TMEM lane quarter
+        const int eh = (NH == 2 && warp >= 14) ? 1 : 0;
         const uint32_t acc_empty_leader = CG == 2 ? map_to(&acc_empty[0], 0) : 0;
         uint32_t tile_i = 0;
         for (uint32_t t = cl; t < total; t += ncl, ++tile_i) {
@@ -554,8 +607,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
             const GemmDesc& g = descs[v];
             const uint32_t lt = t - g.tile_begin;
             const int tm = lt / g.tiles_n, tn = lt % g.tiles_n;
-            const int a = tile_i % C::kAcc;
-            const uint32_t aph = (tile_i / C::kAcc) & 1;
+            const int a = NH == 1 ? (int)(tile_i % C::kAcc) : eh;
+            const uint32_t aph = NH == 1 ? (tile_i / C::kAcc) & 1 : tile_i & 1;
             mbar_wait(&acc_full[a], aph);
             tc_fence_after();
             const int row = tm * C::kMmaM + (int)rank * BM + q * 32 + lane;
@@ -567,7 +620,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
             for (int c0 = 0; c0 < BN; c0 += 32) {
                 uint32_t r[32];
                 tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0), r);
-                const int col0 = tn * BN + c0;
+                const int col0 = tn * TN + eh * BN + c0;
                 if (!row_ok) continue;
 #pragma unroll
                 for (int j = 0; j < 32; j += 4) {
@@ -612,26 +665,27 @@ __global__ void __launch_bounds__(tc::kThreads, 1)
     }
 }
 
-static bool g_attr_set[10][64] = {};
+static bool g_attr_set[20][64] = {};
 
-template <int SPLIT, int CG>
+template <int SPLIT, int CG, int NH = 1>
 static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uint32_t total, int clusters,
                              cudaStream_t s) {
+    using Cf = tc::Cfg<SPLIT, CG, NH>;
     int dev = 0;
     cudaGetDevice(&dev);
-    const int si = SPLIT + 5 * (CG - 1);
-    auto kern = k_sgemm_tc<SPLIT, CG>;
+    const int si = SPLIT + 5 * (CG - 1) + 10 * (NH - 1);
+    auto kern = k_sgemm_tc<SPLIT, CG, NH>;
     if (dev < 64 && !g_attr_set[si][dev]) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)tc::Cfg<SPLIT, CG>::kSmem);
+                                             (int)Cf::kSmem);
         if (e) return e;
         g_attr_set[si][dev] = true;
     }
     cudaLaunchConfig_t lc = {};
     cudaLaunchAttribute attr[1];
     lc.gridDim = dim3((unsigned)(clusters * CG));
-    lc.blockDim = dim3(tc::kThreads);
-    lc.dynamicSmemBytes = tc::Cfg<SPLIT, CG>::kSmem;
+    lc.blockDim = dim3(Cf::kThreads);
+    lc.dynamicSmemBytes = Cf::kSmem;
     lc.stream = s;
     if (CG == 2) {
         attr[0].id = cudaLaunchAttributeClusterDimension;
@@ -672,9 +726,22 @@ static bool tmem_a() {
     return v == 1;
 }
 
+// SVP_TC_WIDE: 0 never use the 256 x 512 pair tiles, 1 (default) let the executor choose per
+// launch (>= 2 waves of wide tiles), 2 always (tests).  The executor builds the tile table
+// for the choice and passes it to the launcher.
+int sgemm_tc_wide_mode() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("SVP_TC_WIDE");
+        v = e ? std::min(2, std::max(0, atoi(e))) : 1;
+    }
+    return (sgemm_tc_cta_pair() && !tmem_a()) ? v : 0;
+}
+
 cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
-                                  cudaStream_t s) {
+                                  bool wide, cudaStream_t s) {
     const int pairs = (int)std::min<uint32_t>(total, std::max(1, grid / 2));
+    if (wide) return launch_tc<2, 2, 2>(descs, n, maps, total, pairs, s);
     if (sgemm_tc_cta_pair())
         return tmem_a() ? launch_tc<4, 2>(descs, n, maps, total, pairs, s) : launch_tc<2, 2>(descs, n, maps, total, pairs, s);
     return tmem_a() ? launch_tc<4, 1>(descs, n, maps, total, grid, s) : launch_tc<2, 1>(descs, n, maps, total, grid, s);

@@ -86,9 +86,11 @@ def test_split_wide_dynamic_range(impl):
 
 
 @pytest.mark.parametrize("env", [{"SVP_TC_CTA_PAIR": "0"}, {"SVP_TC_TMEM_A": "1"},
-                                 {"SVP_TC_CTA_PAIR": "0", "SVP_TC_TMEM_A": "1"}])
+                                 {"SVP_TC_CTA_PAIR": "0", "SVP_TC_TMEM_A": "1"}, {"SVP_TC_WIDE": "0"},
+                                 {"SVP_TC_WIDE": "2"}])
 def test_kernel_variants_in_subprocess(env):
-    """The non-default tcgen05 variants (single-CTA kernels; A-side bf16 operands in TMEM)
+    """The non-default tcgen05 variants (single-CTA kernels; A-side bf16 operands in TMEM;
+    256 x 512 pair tiles never / always instead of per launch)
     are chosen once per process from the environment: run this file's fp32 parity tests
     in a child process with the switch set."""
     import os
@@ -96,6 +98,6 @@ def test_kernel_variants_in_subprocess(env):
     import sys
     here = os.path.dirname(os.path.abspath(__file__))
     cmd = [sys.executable, "-m", "pytest", os.path.join(here, "test_gpu_sgemm_tc.py"), "-q", "-m", "gpu",
-           "-p", "no:cacheprovider", "-k", "(fp32_tolerance or ragged_alpha_beta or wide_dynamic) and not variants"]
+           "-p", "no:cacheprovider", "-k", "(fp32_tolerance or ragged_alpha_beta or wide_dynamic or 2048_sampled) and not variants"]
     r = subprocess.run(cmd, env={**os.environ, **env}, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
