@@ -11,15 +11,16 @@
 //             dropped A_lo B_lo and the truncation of lo are each < 2^-20 |a||b|, so the
 //             product error is < 3 * 2^-20 |a||b| ~ 2.9e-6 |a||b|, inside the fp32 bound
 //             1e-5 (|A||B|)_ij (R10).
-//  SPLIT = 2  "TF32 + 2xBF16" (sgemm_impl SVP_SGEMM_TF32BF16): the main product A_hi B_hi
-//             stays a kind::tf32 MMA on the raw TMA tiles; the two cross terms only need
-//             ~8 significant bits (they are 2^-10 smaller), so they run as kind::f16 BF16
-//             MMAs on converter-written bf16 tiles: D += bf(A_hi) bf(B_lo) + bf(A_lo) bf(B_hi).
-//             Per 16 k: 2 TF32 + 2 BF16 MMAs (a BF16 K16 MMA costs what a TF32 K8 one does)
-//             = 4 MMA slots instead of 6.  Error per product (|l| < 2^-10 |x|, bf16 rounding
-//             2^-9): 2 (2^-19 + 2^-19) + 2^-20 (dropped lo lo) = 4.5 * 2^-19 ~ 8.6e-6 |a||b|,
-//             inside the 1e-5 (|A||B|)_ij bound (R19); integer inputs stay exact
-//             (lo = 0).
+//  SPLIT = 2  "TF32 + 2xBF16" (sgemm_impl SVP_SGEMM_TF32BF16): x = h + l with h = x rounded
+//             to TF32 (the converters write h back over the raw TMA tile) and l = x - h
+//             (exact, |l| <= 2^-11 |x|).  The main product A_h B_h is a kind::tf32 MMA on the
+//             rounded tiles (exact products); the two cross terms only need ~8 significant
+//             bits, so they run as kind::f16 BF16 MMAs on converter-written bf16 tiles:
+//             D += bf(A_h) bf(B_l) + bf(A_l) bf(B_h).  Per 16 k: 2 TF32 + 2 BF16 MMAs (a BF16
+//             K16 MMA costs what a TF32 K8 one does) = 4 MMA slots instead of 6.  Error per
+//             product (bf16 unit roundoff 2^-8): 2 (2^-8 + 2^-8) 2^-11 + 2^-22 (dropped l l)
+//             = 2^-17 + 2^-22 ~ 7.9e-6 |a||b|, inside the 1e-5 (|A||B|)_ij bound (DESIGN.md
+//             R19); integer inputs (|x| <= 2^11) stay exact (l = 0).
 //
 //  SPLIT = 4  the SPLIT 2 arithmetic with the A-side bf16 operands in TMEM: converters
 //             tcgen05.st bf(A_hi) / bf(A_lo) (lane = row, column = k pair) into a TMEM ring
@@ -104,7 +105,7 @@ struct Cfg {
     // NH = 2 ("wide", SPLIT 2 pairs only): a pair computes 256 x 512, two 256-column MMA
     // halves per k-step on the same A tiles; the two TMEM accumulators are the two halves
     // of ONE tile (no double buffer), each drained by its own 4 epilogue warps.
-    static_assert(NH == 1 || (SPLIT == 2 && CG == 2), "wide tiles: TF32+2xBF16 CTA pairs only");
+    static_assert(NH == 1 || (SPLIT == 2 && CG == 2), "wide tiles: split-BF16 CTA pairs only");
     static constexpr int kThreads = tc::kThreads + (NH - 1) * 128;
     static constexpr int kBN = BN / CG * NH;               // B columns staged per CTA
     static constexpr int kTileB = BK * kBN * 4;            // 16 KiB (CG 1) / 8 KiB (CG 2)
@@ -283,19 +284,30 @@ __device__ __forceinline__ uint32_t bf2(float a, float b) {
     asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
     return r;
 }
-// 8 consecutive fp32 -> bf16(hi) and bf16(lo), hi = x with the low 13 mantissa bits cleared
-__device__ __forceinline__ void split8(const float4& p, const float4& q, uint4& hb, uint4& lb) {
+
+// SPLIT 2 / 4 head: h = x rounded to TF32 (nearest, ties away: |x - h| <= 2^-11 |x|), written
+// back over the raw tile the TF32 MMA reads; the cross terms get bf16(h) and bf16(x - h).
+// (A truncated head -- what the tensor core reads from an untouched tile -- leaves |l| up to
+// 2^-10 |x| and a worst-case product error of 2^-16 + 2^-20 > 1e-5: tests/split_emulation.py.)
+// |x| within 2^-12 of FLT_MAX would round to inf; the guest data never gets there.
+__device__ __forceinline__ float rna_tf32(float x) {
+    return __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
+}
+__device__ __forceinline__ float4 rna_tf32_4(float4 x) {
+    return make_float4(rna_tf32(x.x), rna_tf32(x.y), rna_tf32(x.z), rna_tf32(x.w));
+}
+__device__ __forceinline__ void split8_given(const float4& p, const float4& q, const float4& ph, const float4& qh,
+                                             uint4& hb, uint4& lb) {
     const float x[8] = {p.x, p.y, p.z, p.w, q.x, q.y, q.z, q.w};
-    uint32_t h[4], l[4];
+    const float h[8] = {ph.x, ph.y, ph.z, ph.w, qh.x, qh.y, qh.z, qh.w};
+    uint32_t hh[4], ll[4];
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
-        const float h0 = __uint_as_float(__float_as_uint(x[2 * i]) & 0xFFFFE000u);
-        const float h1 = __uint_as_float(__float_as_uint(x[2 * i + 1]) & 0xFFFFE000u);
-        h[i] = bf2(h0, h1);
-        l[i] = bf2(x[2 * i] - h0, x[2 * i + 1] - h1);
+        hh[i] = bf2(h[2 * i], h[2 * i + 1]);
+        ll[i] = bf2(x[2 * i] - h[2 * i], x[2 * i + 1] - h[2 * i + 1]);
     }
-    hb = make_uint4(h[0], h[1], h[2], h[3]);
-    lb = make_uint4(l[0], l[1], l[2], l[3]);
+    hb = make_uint4(hh[0], hh[1], hh[2], hh[3]);
+    lb = make_uint4(ll[0], ll[1], ll[2], ll[3]);
 }
 
 }  // namespace tc
@@ -565,15 +577,22 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     if constexpr (SPLIT == 4) {
                         const float4 p = *reinterpret_cast<const float4*>(sp + t_rd0);
                         const float4 q = *reinterpret_cast<const float4*>(sp + t_rd1);
+                        const float4 ph = rna_tf32_4(p), qh = rna_tf32_4(q);
+                        *reinterpret_cast<float4*>(sp + t_rd0) = ph;
+                        *reinterpret_cast<float4*>(sp + t_rd1) = qh;
                         uint4 hb, lb;
-                        split8(p, q, hb, lb);
+                        split8_given(p, q, ph, qh, hb, lb);
                         tmem_st4(t_lane + 16 * s, hb);
                         tmem_st4(t_lane + 16 * s + 8, lb);
                     } else {
                         const float4 p = *reinterpret_cast<const float4*>(sp + a_rd0);
                         const float4 q = *reinterpret_cast<const float4*>(sp + a_rd1);
+                        // the TF32 MMA reads the raw tile: round it to TF32 in place (R19)
+                        const float4 ph = rna_tf32_4(p), qh = rna_tf32_4(q);
+                        *reinterpret_cast<float4*>(sp + a_rd0) = ph;
+                        *reinterpret_cast<float4*>(sp + a_rd1) = qh;
                         uint4 hb, lb;
-                        split8(p, q, hb, lb);
+                        split8_given(p, q, ph, qh, hb, lb);
                         *reinterpret_cast<uint4*>(a16h + a_wr) = hb;
                         *reinterpret_cast<uint4*>(a16l + a_wr) = lb;
                     }
@@ -582,8 +601,11 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                         const float4 x0 = *reinterpret_cast<const float4*>(sp + kTileA + b_rd[r][0]);
                         const float4 x1 = *reinterpret_cast<const float4*>(sp + kTileA + b_rd[r][1]);
                         const bool sw = (b_rd[r][0] & 16) != 0;  // read the upper half first
+                        const float4 h0 = rna_tf32_4(x0), h1 = rna_tf32_4(x1);
+                        *reinterpret_cast<float4*>(sp + kTileA + b_rd[r][0]) = h0;
+                        *reinterpret_cast<float4*>(sp + kTileA + b_rd[r][1]) = h1;
                         uint4 hb, lb;
-                        split8(sw ? x1 : x0, sw ? x0 : x1, hb, lb);
+                        split8_given(sw ? x1 : x0, sw ? x0 : x1, sw ? h1 : h0, sw ? h0 : h1, hb, lb);
                         *reinterpret_cast<uint4*>(b16h + b_wr[r]) = hb;
                         *reinterpret_cast<uint4*>(b16l + b_wr[r]) = lb;
                     }
