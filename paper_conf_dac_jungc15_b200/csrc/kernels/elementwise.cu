@@ -12,6 +12,10 @@
 //   vecadd  c = a + b            (__fadd_rn: one rounding, never contracted)
 //   saxpy   y = fma(a_v, x, y)   (__fmaf_rn: single rounding, = C99 fmaf)
 //   BS      SDK formula with the A&S 26.2.17 CND, SFU-approximate exp/log/div (tolerance).
+#include <stdlib.h>
+
+#include <algorithm>
+
 #include "../launch.h"
 #include "common.cuh"
 
@@ -322,6 +326,10 @@ cudaError_t query_limits(LaunchLimits* out) {
     if (e) return e;
     if (out->dgemm_blocks_per_sm < 1) out->dgemm_blocks_per_sm = 1;
     if (out->dgemm_small_blocks_per_sm < 1) out->dgemm_small_blocks_per_sm = 1;
+    // experiment knobs (tools/grid_probe.py): cap the resident CTAs per SM of the
+    // elementwise / Black-Scholes launches
+    if (const char* e = getenv("SVP_EW_PER_SM")) out->ew_blocks_per_sm = std::min(out->ew_blocks_per_sm, atoi(e));
+    if (const char* e = getenv("SVP_BS_PER_SM")) out->bs_blocks_per_sm = std::min(out->bs_blocks_per_sm, atoi(e));
     if (out->ew_blocks_per_sm < 1) out->ew_blocks_per_sm = 1;
     if (out->bs_blocks_per_sm < 1) out->bs_blocks_per_sm = 1;
     if (out->hist_blocks_per_sm < 1) out->hist_blocks_per_sm = 1;
