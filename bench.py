@@ -179,7 +179,8 @@ class Clocks:
             if len(parts) < 10:
                 continue
             try:
-                rows.append((self._ts(parts[0]), float(parts[2]), float(parts[3]), parts[6:10]))
+                pw = float(parts[4]) if parts[4] not in ("", "[N/A]") else float("nan")
+                rows.append((self._ts(parts[0]), float(parts[2]), float(parts[3]), parts[6:10], pw))
             except ValueError:
                 continue
         os.unlink(self.f.name)
@@ -196,9 +197,10 @@ class Clocks:
             for nm, val in zip(names, r[3]):
                 if val.lower().startswith("active"):
                     reasons.add(nm)
+        pws = [r[4] for r in sel if r[4] == r[4]]
         return {"sm_mhz": statistics.median(r[1] for r in sel), "sm_max_mhz": max(r[2] for r in sel),
                 "samples": len(sel), "in_window": len(inside), "window_ms": (self.t1 - self.t0) * 1e3,
-                "reasons": sorted(reasons)}
+                "reasons": sorted(reasons), "power_w": statistics.median(pws) if pws else None}
 
 
 def measured_peaks():

@@ -64,8 +64,8 @@ constexpr int kEwThreads = 256;
 constexpr int kVecaddVec = 4;                                  // float4 per thread per array
 constexpr int kVecaddTile = kEwThreads * 4 * kVecaddVec;       // 4096 elements
 constexpr int kSaxpyTile = kVecaddTile;
-constexpr int kBsVec = 2;
-constexpr int kBsTile = kEwThreads * 4 * kBsVec;               // 2048 options
+constexpr int kBsVec = 4;
+constexpr int kBsTile = kEwThreads * 4 * kBsVec;               // 4096 options (kBsVec 4: +1.5 % cfg5, profiles/r01/bsvec)
 constexpr int kHistThreads = 256;
 constexpr int kHistVec = 4;                                    // uint4 (16 B) per thread
 constexpr int kHistTile = kHistThreads * 16 * kHistVec;        // 16384 bytes
