@@ -74,8 +74,15 @@ typedef struct svp_config {
     int32_t dry_run;             /* 1: plan only -- no CUDA call at all, op times simulated
                                     by the cost model (host-logic tests on CPU)               */
     int32_t flush_timeout_ms;    /* 0 = wait forever; else watchdog -> SVP_E_TIMEOUT          */
-    int32_t validate_ptrs;       /* 1: svp_submit checks residency with cudaPointerGetAttributes
-                                    (device buffer on the VP's GPU, host buffer pinned)       */
+    int32_t validate_ptrs;       /* svp_submit checks every buffer [ptr, ptr + touched bytes):
+                                    DEVICE -> device/managed memory on the VP's GPU, HOST_PINNED
+                                    -> page-locked host memory, and the range inside ONE
+                                    allocation (else SVP_E_INVAL).  0: no check; 1: allocation
+                                    ranges are resolved once (cudaPointerGetAttributes +
+                                    cuPointerGetAttribute RANGE_START/SIZE) and remembered for
+                                    the context's lifetime -- memory freed and re-allocated at
+                                    the same address with another residency is not re-detected;
+                                    2: query the driver on every submit                       */
     int32_t sgemm_impl;          /* SVP_SGEMM_TF32BF16 (default), SVP_SGEMM_3XTF32 or SVP_SGEMM_FFMA */
     void* const* external_streams; /* optional [num_gpus] caller cudaStream_t (e.g. torch's
                                     current stream): flush work starts after the work already
@@ -97,9 +104,10 @@ typedef struct svp_config {
                                     graph per GPU.  Ignored with sync_each_job.              */
     int32_t table_mode;          /* where a coalesced launch finds its segment table (SURVEY
                                     §8(b)): SVP_TABLE_PARAM (default) -- launches of
-                                    elementwise / hist256 groups with <= 240 VPs receive it
-                                    by value as a kernel parameter (no upload; cfg5 measured
-                                    +4 % over global); SVP_TABLE_GLOBAL -- one device table
+                                    elementwise / hist256 groups with <= 64 VPs receive it
+                                    by value as a kernel parameter of 1 or 4 KiB (no upload;
+                                    cfg5 measured +4 % over global); larger groups, and
+                                    SVP_TABLE_GLOBAL -- one device table
                                     buffer per GPU, uploaded once per flush when it changed.
                                     GEMM launches always use the global table.             */
 } svp_config;

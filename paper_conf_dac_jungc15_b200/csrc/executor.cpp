@@ -20,6 +20,8 @@
 #include <string.h>
 
 #include <algorithm>
+#include <map>
+#include <mutex>
 #include <chrono>
 #include <thread>
 
@@ -83,10 +85,19 @@ struct Dev {
     std::vector<cudaEvent_t> join_ev;
 };
 
+// An allocation range resolved by executor_check_ptr (validate_ptrs 1 keeps them).
+struct PtrRange {
+    uintptr_t end = 0;
+    int type = 0;    // cudaMemoryType
+    int device = -1;
+};
+
 struct Executor {
     Ctx* c = nullptr;
     std::vector<Dev> devs;
     std::string err;
+    std::mutex rmu;                          // submits validate from many threads
+    std::map<uintptr_t, PtrRange> ranges;    // allocation start -> range (validate_ptrs 1)
 };
 
 std::string executor_error(Executor* e) { return e->err; }
@@ -192,29 +203,86 @@ void executor_unregister_host(Executor* e, void* p) {
     cudaGetLastError();
 }
 
-svp_status executor_check_ptr(Executor* e, const void* p, int32_t mem, int32_t device, std::string* why) {
-    cudaPointerAttributes at;
-    cudaError_t ce = cudaPointerGetAttributes(&at, p);
-    if (ce != cudaSuccess) {
-        cudaGetLastError();
-        *why = std::string("cudaPointerGetAttributes failed: ") + cudaGetErrorString(ce);
-        return SVP_E_INVAL;
+// Allocation range of p through the driver (CU_POINTER_ATTRIBUTE_RANGE_START_ADDR / _SIZE);
+// the entry point is fetched at runtime, libsvp does not link libcuda.  false: unknown.
+typedef CUresult (*PFN_ptrAttr)(void*, CUpointer_attribute, CUdeviceptr);
+static bool alloc_range(const void* p, uintptr_t* start, uintptr_t* end) {
+    static PFN_ptrAttr fn = [] {
+        void* q = nullptr;
+        cudaDriverEntryPointQueryResult r;
+        if (cudaGetDriverEntryPoint("cuPointerGetAttribute", &q, cudaEnableDefault, &r) != cudaSuccess ||
+            r != cudaDriverEntryPointSuccess)
+            q = nullptr;
+        return reinterpret_cast<PFN_ptrAttr>(q);
+    }();
+    if (!fn) return false;
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    if (fn(&base, CU_POINTER_ATTRIBUTE_RANGE_START_ADDR, (CUdeviceptr)p) != CUDA_SUCCESS ||
+        fn(&size, CU_POINTER_ATTRIBUTE_RANGE_SIZE, (CUdeviceptr)p) != CUDA_SUCCESS || size == 0)
+        return false;
+    *start = (uintptr_t)base;
+    *end = (uintptr_t)base + size;
+    return true;
+}
+
+svp_status executor_check_ptr(Executor* e, const void* p, uint64_t bytes, int32_t mem, int32_t device,
+                              std::string* why) {
+    const uintptr_t a = (uintptr_t)p;
+    const bool cached = e->c->cfg.validate_ptrs == 1;
+    PtrRange r;
+    bool hit = false, known = false;
+    if (cached) {
+        std::lock_guard<std::mutex> lk(e->rmu);
+        auto it = e->ranges.upper_bound(a);
+        if (it != e->ranges.begin()) {
+            --it;
+            if (a < it->second.end) {
+                r = it->second;
+                hit = known = true;
+            }
+        }
+    }
+    if (!hit) {
+        cudaPointerAttributes at;
+        cudaError_t ce = cudaPointerGetAttributes(&at, p);
+        if (ce != cudaSuccess) {
+            cudaGetLastError();
+            *why = std::string("cudaPointerGetAttributes failed: ") + cudaGetErrorString(ce);
+            return SVP_E_INVAL;
+        }
+        r.type = (int)at.type;
+        r.device = at.device;
+        uintptr_t st = 0, en = 0;
+        if (at.type != cudaMemoryTypeUnregistered && alloc_range(p, &st, &en) && st <= a && a < en) {
+            r.end = en;
+            known = true;
+            if (cached) {
+                std::lock_guard<std::mutex> lk(e->rmu);
+                e->ranges[st] = r;
+            }
+        }
     }
     if (mem == SVP_MEM_DEVICE) {
-        if (at.type != cudaMemoryTypeDevice && at.type != cudaMemoryTypeManaged) {
+        if (r.type != cudaMemoryTypeDevice && r.type != cudaMemoryTypeManaged) {
             *why = "declared DEVICE but is not device memory";
             return SVP_E_INVAL;
         }
-        if (at.type == cudaMemoryTypeDevice && at.device != e->devs[device].ordinal) {
-            *why = "device buffer is on CUDA device " + std::to_string(at.device) + " but the VP runs on " +
+        if (r.type == cudaMemoryTypeDevice && r.device != e->devs[device].ordinal) {
+            *why = "device buffer is on CUDA device " + std::to_string(r.device) + " but the VP runs on " +
                    std::to_string(e->devs[device].ordinal) + " (see svp_vp_device)";
             return SVP_E_INVAL;
         }
     } else {
-        if (at.type != cudaMemoryTypeHost) {
+        if (r.type != cudaMemoryTypeHost) {
             *why = "declared HOST_PINNED but is not page-locked host memory";
             return SVP_E_INVAL;
         }
+    }
+    if (known && bytes > r.end - a) {
+        *why = "buffer of " + std::to_string(bytes) + " B extends " + std::to_string(bytes - (r.end - a)) +
+               " B past the end of its allocation";
+        return SVP_E_INVAL;
     }
     return SVP_OK;
 }
@@ -418,8 +486,7 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
     };
     if (ch.param) {
         // table by value: copied into the launch's parameter buffer at enqueue time
-        SegParam p;
-        memcpy(&p, d.tbl_last.data() + ch.table_off, (size_t)ch.nsegs * sizeof(SegDesc));
+        const SegDesc* p = reinterpret_cast<const SegDesc*>(d.tbl_last.data() + ch.table_off);
         switch (ch.kernel) {
             case K_VECADD:
             case K_SAXPY: return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.ew_blocks_per_sm), s);

@@ -236,7 +236,12 @@ void executor_destroy(Executor* e);
 svp_status executor_run(Executor* e, Flush* f);      // tables, staging, issue, wait, profile
 std::string executor_error(Executor* e);
 // residency check for svp_submit (validate_ptrs): returns SVP_OK or SVP_E_INVAL
-svp_status executor_check_ptr(Executor* e, const void* p, int32_t mem, int32_t device, std::string* why);
+// Residency check of one buffer [p, p + bytes) (cfg.validate_ptrs): declared DEVICE ->
+// device (or managed) memory on the VP's GPU; HOST_PINNED -> page-locked host memory; and
+// the whole range inside ONE allocation.  validate_ptrs 1 remembers every allocation range
+// it has resolved (one driver query per allocation, not per submit); 2 queries every time.
+svp_status executor_check_ptr(Executor* e, const void* p, uint64_t bytes, int32_t mem, int32_t device,
+                              std::string* why);
 
 // errors
 void set_error(const std::string& msg);

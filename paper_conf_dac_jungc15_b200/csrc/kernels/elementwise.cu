@@ -13,6 +13,7 @@
 //   saxpy   y = fma(a_v, x, y)   (__fmaf_rn: single rounding, = C99 fmaf)
 //   BS      SDK formula with the A&S 26.2.17 CND, SFU-approximate exp/log/div (tolerance).
 #include <stdlib.h>
+#include <string.h>
 
 #include <algorithm>
 
@@ -251,7 +252,8 @@ __device__ __forceinline__ void bs_tile(const SegDesc& sd, uint32_t lt) {
                                                        uint32_t total) {                        \
         NAME##_loop(segs, nsegs, total);                                                        \
     }                                                                                           \
-    __global__ void __launch_bounds__(kEwThreads) NAME##_p(const __grid_constant__ SegParam p, int nsegs, \
+    template <int CAP>                                                                          \
+    __global__ void __launch_bounds__(kEwThreads) NAME##_p(const __grid_constant__ SegParamT<CAP> p, int nsegs, \
                                                            uint32_t total) {                    \
         NAME##_loop(p.s, nsegs, total);                                                         \
     }
@@ -292,15 +294,33 @@ cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total, int gr
     return cudaGetLastError();
 }
 
-cudaError_t launch_ew_param(int kind, const SegParam& p, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+template <int CAP>
+static cudaError_t launch_ew_param_cap(int kind, const SegDesc* segs, int nsegs, uint32_t total, int grid,
+                                      cudaStream_t s) {
+    SegParamT<CAP> p;
+    memcpy(p.s, segs, (size_t)nsegs * sizeof(SegDesc));
     switch (kind) {
-        case 1: k_vecadd_p<<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
-        case 2: k_saxpy_p<<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
-        case 4: k_blackscholes_p<<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
-        case 8: k_ew_mix_p<<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
+        case 1: k_vecadd_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
+        case 2: k_saxpy_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
+        case 4: k_blackscholes_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
+        case 8: k_ew_mix_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
         default: return cudaErrorInvalidValue;
     }
     return cudaGetLastError();
+}
+
+// experiment knob: SVP_PARAM_FULL=1 always passes the full kParamSegs block (A/B)
+bool param_full_block() {
+    static const bool full = getenv("SVP_PARAM_FULL") && atoi(getenv("SVP_PARAM_FULL")) != 0;
+    return full;
+}
+
+cudaError_t launch_ew_param(int kind, const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+    if (param_full_block() && nsegs <= kParamSegs)
+        return launch_ew_param_cap<kParamSegs>(kind, segs, nsegs, total, grid, s);
+    if (nsegs <= 16) return launch_ew_param_cap<16>(kind, segs, nsegs, total, grid, s);
+    if (nsegs <= kParamSegs) return launch_ew_param_cap<kParamSegs>(kind, segs, nsegs, total, grid, s);
+    return cudaErrorInvalidValue;
 }
 
 cudaError_t query_limits_hist(int* per_sm);

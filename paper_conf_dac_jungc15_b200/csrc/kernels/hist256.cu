@@ -20,6 +20,8 @@
 // A VP's ragged head/tail tiles (not 16-B aligned / partial) are read from global memory
 // directly.  A preceding tiny kernel zeroes every segment's counts, so the result
 // overwrites the output and is bit-exact (integer adds commute).
+#include <string.h>
+
 #include "../launch.h"
 #include "common.cuh"
 
@@ -40,7 +42,8 @@ __device__ __forceinline__ void hist_zero_body(const SegDesc* __restrict__ segs,
 __global__ void __launch_bounds__(256) k_hist_zero(const SegDesc* __restrict__ segs, int nsegs) {
     hist_zero_body(segs, nsegs);
 }
-__global__ void __launch_bounds__(256) k_hist_zero_p(const __grid_constant__ SegParam p, int nsegs) {
+template <int CAP>
+__global__ void __launch_bounds__(256) k_hist_zero_p(const __grid_constant__ SegParamT<CAP> p, int nsegs) {
     hist_zero_body(p.s, nsegs);
 }
 
@@ -204,9 +207,23 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
 __global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
     hist_body(segs, nsegs, total);
 }
-__global__ void __launch_bounds__(kHistBlock) k_hist256_p(const __grid_constant__ SegParam p, int nsegs,
+template <int CAP>
+__global__ void __launch_bounds__(kHistBlock) k_hist256_p(const __grid_constant__ SegParamT<CAP> p, int nsegs,
                                                           uint32_t total) {
     hist_body(p.s, nsegs, total);
+}
+
+template <int CAP>
+static cudaError_t hist_attr_p() {
+    static bool attr[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 64 && !attr[dev]) {
+        cudaError_t e = cudaFuncSetAttribute(k_hist256_p<CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmem);
+        if (e) return e;
+        attr[dev] = true;
+    }
+    return cudaSuccess;
 }
 
 static cudaError_t hist_attr() {
@@ -215,8 +232,6 @@ static cudaError_t hist_attr() {
     cudaGetDevice(&dev);
     if (dev < 64 && !attr[dev]) {
         cudaError_t e = cudaFuncSetAttribute(k_hist256, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmem);
-        if (e) return e;
-        e = cudaFuncSetAttribute(k_hist256_p, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmem);
         if (e) return e;
         attr[dev] = true;
     }
@@ -233,14 +248,26 @@ cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int g
     return cudaGetLastError();
 }
 
-cudaError_t launch_hist256_param(const SegParam& p, int nsegs, uint32_t total, int grid, cudaStream_t s) {
-    if (nsegs <= 0) return cudaSuccess;
-    k_hist_zero_p<<<nsegs < 1024 ? nsegs : 1024, 256, 0, s>>>(p, nsegs);
+template <int CAP>
+static cudaError_t launch_hist256_param_cap(const SegDesc* segs, int nsegs, uint32_t total, int grid,
+                                            cudaStream_t s) {
+    SegParamT<CAP> p;
+    memcpy(p.s, segs, (size_t)nsegs * sizeof(SegDesc));
+    k_hist_zero_p<CAP><<<nsegs, 256, 0, s>>>(p, nsegs);
     cudaError_t e = cudaGetLastError();
     if (e || total == 0) return e;
-    if ((e = hist_attr())) return e;
-    k_hist256_p<<<grid, kHistBlock, kHistSmem, s>>>(p, nsegs, total);
+    if ((e = hist_attr_p<CAP>())) return e;
+    k_hist256_p<CAP><<<grid, kHistBlock, kHistSmem, s>>>(p, nsegs, total);
     return cudaGetLastError();
+}
+
+cudaError_t launch_hist256_param(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+    if (nsegs <= 0) return cudaSuccess;
+    if (param_full_block() && nsegs <= kParamSegs)
+        return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s);
+    if (nsegs <= 16) return launch_hist256_param_cap<16>(segs, nsegs, total, grid, s);
+    if (nsegs <= kParamSegs) return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s);
+    return cudaErrorInvalidValue;
 }
 
 cudaError_t query_limits_hist(int* per_sm) {

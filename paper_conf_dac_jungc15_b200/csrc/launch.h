@@ -32,8 +32,11 @@ cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total_t
 cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
 // table_mode param: the same kernels with the segment table passed by value; kind = kernel
 // id (1 vecadd, 2 SAXPY, 4 Black-Scholes, 8 mixed), nsegs <= kParamSegs.
-cudaError_t launch_ew_param(int kind, const SegParam& p, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
-cudaError_t launch_hist256_param(const SegParam& p, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
+// `segs` is the HOST copy of the table (nsegs <= kParamSegs); it is copied into a
+// parameter block of 16 or 64 segments, the smallest that holds it.
+cudaError_t launch_ew_param(int kind, const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
+bool param_full_block();  // SVP_PARAM_FULL=1: always the kParamSegs block (A/B knob)
+cudaError_t launch_hist256_param(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
 // hist256: zeroes each segment's 256 counters, then accumulates.
 cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s);
 

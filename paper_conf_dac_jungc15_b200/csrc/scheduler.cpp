@@ -181,9 +181,10 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
     j->device = dispatch_vp(c, j->vp, cost);
     if (c->exec && c->cfg.validate_ptrs && !empty) {
         for (int b = 0; b < j->nbufs; ++b) {
-            if (touched_bytes(*j, b) == 0) continue;  // nothing is read or written there
+            const uint64_t tb = touched_bytes(*j, b);
+            if (tb == 0) continue;  // nothing is read or written there
             std::string why;
-            if (executor_check_ptr(c->exec, j->bufs[b].ptr, j->bufs[b].mem, j->device, &why) != SVP_OK)
+            if (executor_check_ptr(c->exec, j->bufs[b].ptr, tb, j->bufs[b].mem, j->device, &why) != SVP_OK)
                 return fail(SVP_E_INVAL, "svp_submit: buffer " + std::to_string(b) + ": " + why);
         }
     }

@@ -29,9 +29,15 @@ enum : uint16_t { SEG_SCALAR = 1, SEG_KIND_SHIFT = 8 };
 // table_mode = SVP_TABLE_PARAM: a launch of at most kParamSegs segments receives its table
 // by value as a __grid_constant__ kernel parameter (15 KiB of the 32 KiB parameter space):
 // no table upload and segment reads served from the constant cache.
-constexpr int kParamSegs = 240;
-struct SegParam {
-    SegDesc s[kParamSegs];
+// The parameter block is sized to the launch: CAP in {16, 64} segments (1 or 4 KiB), the
+// smallest that holds the group.  A launch's parameters are pushed through the front end
+// with the launch; a 15-KiB block (the earlier 240-segment cap) cost ~9 us per launch on an
+// idle GPU against ~1 us for 1 KiB, and groups above 64 segments ran faster from the global
+// table (no upload in steady state) -- tools/s1_probe.py, profiles/r01/param_cap/.
+constexpr int kParamSegs = 64;
+template <int CAP>
+struct SegParamT {
+    SegDesc s[CAP];
 };
 
 // Grouped SGEMM: one entry per VP; tensor maps live in a separate 64-B aligned array

@@ -225,7 +225,7 @@ class Context:
     def __init__(self, num_gpus: int = 0, device_ids: Optional[Sequence[int]] = None, streams_per_gpu: int = 4,
                  coalesce: bool = True, interleave: bool = True, max_chunks: int = 8, arena_bytes: int = 0,
                  profile_level: int = 0, sync_each_job: bool = False, dry_run: bool = False,
-                 flush_timeout_ms: int = 0, validate_ptrs: bool = True, sgemm_impl: int = SGEMM_TF32BF16,
+                 flush_timeout_ms: int = 0, validate_ptrs: int = 1, sgemm_impl: int = SGEMM_TF32BF16,
                  external_streams: Optional[Sequence[int]] = None, hbm_gbps: float = 0.0, pcie_gbps: float = 0.0,
                  ffma_tflops: float = 0.0, launch_us: float = 0.0, hetero: bool = False, graph: bool = False,
                  table_mode: int = TABLE_PARAM):

@@ -46,9 +46,11 @@ def test_init_without_gpu_fails_loudly():
     assert e.value.status == svp.SVP_E_CUDA
 
 
-def test_init_rejects_bad_config():
+@pytest.mark.parametrize("kw", [dict(streams_per_gpu=0), dict(validate_ptrs=3), dict(validate_ptrs=-1),
+                                dict(table_mode=2), dict(profile_level=3)])
+def test_init_rejects_bad_config(kw):
     with pytest.raises(svp.SvpError) as e:
-        svp.Context(dry_run=True, streams_per_gpu=0)
+        svp.Context(dry_run=True, **kw)
     assert e.value.status == svp.SVP_E_INVAL
 
 

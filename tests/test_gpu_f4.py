@@ -141,11 +141,15 @@ def test_table_mode_param(small, residency, hetero):
 
 
 def test_table_mode_param_no_upload_and_fallback():
-    """Elementwise-only flushes in param mode upload no table; a group larger than the
-    parameter table (240 VPs) falls back to the global table and stays correct."""
+    """Elementwise-only flushes in param mode upload no table (groups of 16 and of 17..64
+    VPs use the 1-KiB and 4-KiB parameter blocks); a group larger than the parameter table
+    (64 VPs) falls back to the global table and stays correct."""
     few = [W.JobSpec(v, ("vecadd", "saxpy", "hist256", "blackscholes")[v % 4], n=5000 + 77 * v) for v in range(40)]
+    cap16 = [W.JobSpec(v, ("hist256", "saxpy")[v % 2], n=3000 + 91 * v) for v in range(32)]
+    cap64 = [W.JobSpec(v, ("vecadd", "hist256")[v % 2], n=2000 + 51 * v) for v in range(128)]
+    over = [W.JobSpec(v, "hist256", n=1000 + 29 * v) for v in range(65)]
     many = [W.JobSpec(v, "vecadd", n=1000 + 13 * v) for v in range(300)]
-    for specs, uploads in ((few, 0), (many, 1)):
+    for specs, uploads in ((few, 0), (cap16, 0), (cap64, 0), (over, 1), (many, 1)):
         inputs = inputs_for(specs)
         outs, _, st = run_svp(specs, inputs, "device", table_mode=svp.TABLE_PARAM)
         assert st["table_uploads"] == uploads

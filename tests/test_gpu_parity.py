@@ -182,6 +182,35 @@ def test_residency_validation():
     ctx.close()
 
 
+@pytest.mark.parametrize("level", [1, 2])
+def test_residency_validation_ranges(level):
+    """validate_ptrs 1 (allocation ranges remembered) and 2 (queried every submit) reject a
+    buffer running past the end of its allocation, and a remembered device range declared
+    HOST_PINNED; in-range buffers pass on repeated submits and compute correctly."""
+    ctx = svp.Context(num_gpus=1, validate_ptrs=level)
+    va = ctx.register_kernel("vecadd")
+    n = 1 << 18
+    a = torch.rand(n, device="cuda")
+    b = torch.rand(n, device="cuda")
+    c = torch.empty(n, device="cuda")
+    for _ in range(2):  # the second pass hits the remembered ranges (level 1)
+        ctx.submit(0, va, svp.args_vecadd(n), [(a.data_ptr(), 4 * n, 1, 0), (b.data_ptr(), 4 * n, 1, 0),
+                                               (c.data_ptr(), 4 * n, 2, 0)])
+        ctx.flush()
+        torch.cuda.synchronize()
+        assert torch.equal(c, a + b)
+    big = 1 << 31  # far past any allocation holding a 1-MiB tensor
+    with pytest.raises(svp.SvpError) as e:
+        ctx.submit(0, va, svp.args_vecadd(big), [(a.data_ptr(), 4 * big, 1, 0), (b.data_ptr(), 4 * big, 1, 0),
+                                                 (c.data_ptr(), 4 * big, 2, 0)])
+    assert e.value.status == svp.SVP_E_INVAL and "past the end" in str(e.value)
+    with pytest.raises(svp.SvpError) as e:
+        ctx.submit(0, va, svp.args_vecadd(n), [(a.data_ptr(), 4 * n, 1, 1), (b.data_ptr(), 4 * n, 1, 0),
+                                               (c.data_ptr(), 4 * n, 2, 0)])
+    assert e.value.status == svp.SVP_E_INVAL
+    ctx.close()
+
+
 def test_repeated_flushes_reuse_tables(small):
     specs, inputs = small
     ctx = svp.Context(num_gpus=1)

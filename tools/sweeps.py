@@ -57,6 +57,8 @@ def flush_time(ctx, jobs, reps=5, warm=2):
 
 
 def ctx_for(**kw):
+    # SVP_SWEEP_VALIDATE: validate_ptrs level of every context (A/B of the range cache)
+    kw.setdefault("validate_ptrs", int(os.environ.get("SVP_SWEEP_VALIDATE", "1")))
     return svp.Context(num_gpus=1, external_streams=[torch.cuda.current_stream().cuda_stream], **kw)
 
 
