@@ -229,7 +229,12 @@ static svp_status submit_many(Ctx* c, int32_t n, const svp_job_desc* jd, const s
         for (int i = 0; i < n; ++i) {
             jobs[i].id = c->next_job_id++;
             if (ids) ids[i] = jobs[i].id;
-            c->queue.push_back(jobs[i]);
+        }
+        if (c->queue.empty()) {
+            c->queue.swap(jobs);
+        } else {
+            c->queue.reserve(c->queue.size() + n);
+            c->queue.insert(c->queue.end(), jobs.begin(), jobs.end());
         }
     }
     c->q_cv.notify_one();

@@ -290,50 +290,81 @@ static uint64_t staged_bytes(const Flush& f, const std::vector<int32_t>& jobs) {
     return s;
 }
 
+// Dense per-VP slots for the planner's per-VP state: a flat array when the VP ids are
+// compact (the usual case), else a hash map (ids go up to 2^20).
+struct VpSlots {
+    std::vector<int32_t> flat;
+    std::unordered_map<int32_t, int32_t> sparse;
+    bool dense = true;
+    int32_t init = 0;
+    VpSlots(const std::vector<Job>& jobs, int32_t init_value) : init(init_value) {
+        int32_t mx = -1;
+        for (const auto& j : jobs) mx = std::max(mx, j.vp);
+        dense = (size_t)mx < 4 * jobs.size() + 4096;
+        if (dense) flat.assign((size_t)mx + 1, init_value);
+        else sparse.reserve(jobs.size() * 2);
+    }
+    int32_t& operator[](int32_t vp) {
+        if (dense) return flat[vp];
+        auto it = sparse.find(vp);
+        if (it == sparse.end()) it = sparse.emplace(vp, init).first;
+        return it->second;
+    }
+};
+
 svp_status plan_flush(Ctx* c, Flush* f) {
+    const size_t n = f->jobs.size();
     // ---- levels (program order per VP)
-    std::unordered_map<int32_t, int32_t> next_level;
-    f->levels = 0;
-    for (auto& j : f->jobs) {
-        j.level = next_level[j.vp]++;
-        f->levels = std::max(f->levels, j.level + 1);
+    {
+        VpSlots next_level(f->jobs, 0);
+        f->levels = 0;
+        for (auto& j : f->jobs) {
+            j.level = next_level[j.vp]++;
+            f->levels = std::max(f->levels, j.level + 1);
+        }
     }
     const int S = c->cfg.streams_per_gpu;
     const bool inter = c->cfg.interleave != 0;
     const bool coal = c->cfg.coalesce != 0;
 
     // ---- Kernel Match (a2): groups per (level, device, kernel, shape)
-    typedef std::tuple<int32_t, int32_t, int32_t, uint64_t> Key;
-    std::map<Key, int32_t> gidx;
-    std::vector<int32_t> order(f->jobs.size());
+    std::vector<int32_t> order(n);
     std::iota(order.begin(), order.end(), 0);
     // NEXT f4 (cfg.hetero): the elementwise kernels of one (level, GPU) match as ONE
     // heterogeneous group -- "identical kernels only" lifted for the
     // kernels that share a CTA shape and tile mapping; members stay in VP order.
     const bool het = c->cfg.hetero != 0;
     auto mkernel = [&](const Job& j) { return het && is_ew(j.kernel) ? (int32_t)K_EW_MIX : j.kernel; };
+    f->groups.reserve(coal ? 16 : n);
     if (coal) {
+        // sort by (level, device, match kernel, shape, vp); groups are the runs of equal
+        // (level, device, match kernel, shape)
+        struct MKey {
+            int32_t level, device, kernel, vp;
+            uint64_t shape;
+        };
+        std::vector<MKey> key(n);
+        for (size_t i = 0; i < n; ++i) {
+            const Job& j = f->jobs[i];
+            key[i] = MKey{j.level, j.device, mkernel(j), j.vp, j.shape_key};
+        }
         std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
-            const Job &x = f->jobs[a], &y = f->jobs[b];
-            const int32_t kx = mkernel(x), ky = mkernel(y);
-            return std::tie(x.level, x.device, kx, x.shape_key, x.vp) <
-                   std::tie(y.level, y.device, ky, y.shape_key, y.vp);
+            const MKey &x = key[a], &y = key[b];
+            return std::tie(x.level, x.device, x.kernel, x.shape, x.vp) <
+                   std::tie(y.level, y.device, y.kernel, y.shape, y.vp);
         });
-        for (int32_t ji : order) {
-            const Job& j = f->jobs[ji];
-            Key k{j.level, j.device, mkernel(j), j.shape_key};
-            auto it = gidx.find(k);
-            if (it == gidx.end()) {
-                Group g;
-                g.kernel = mkernel(j);
-                g.shape_key = j.shape_key;
-                g.level = j.level;
-                g.device = j.device;
-                gidx[k] = (int32_t)f->groups.size();
-                f->groups.push_back(g);
-                it = gidx.find(k);
+        for (size_t i = 0; i < n; ++i) {
+            const MKey& k = key[order[i]];
+            if (i == 0 || k.level != key[order[i - 1]].level || k.device != key[order[i - 1]].device ||
+                k.kernel != key[order[i - 1]].kernel || k.shape != key[order[i - 1]].shape) {
+                f->groups.emplace_back();
+                Group& g = f->groups.back();
+                g.kernel = k.kernel;
+                g.shape_key = k.shape;
+                g.level = k.level;
+                g.device = k.device;
             }
-            f->groups[it->second].jobs.push_back(ji);
+            f->groups.back().jobs.push_back(order[i]);
         }
     } else {
         // no coalescing: one group per job, submission order within a level
@@ -341,13 +372,13 @@ svp_status plan_flush(Ctx* c, Flush* f) {
                          [&](int32_t a, int32_t b) { return f->jobs[a].level < f->jobs[b].level; });
         for (int32_t ji : order) {
             const Job& j = f->jobs[ji];
-            Group g;
+            f->groups.emplace_back();
+            Group& g = f->groups.back();
             g.kernel = j.kernel;
             g.shape_key = j.shape_key;
             g.level = j.level;
             g.device = j.device;
             g.jobs.push_back(ji);
-            f->groups.push_back(g);
         }
     }
 
@@ -370,6 +401,17 @@ svp_status plan_flush(Ctx* c, Flush* f) {
             nch = std::max(1, std::min(nch, c->cfg.max_chunks));
         }
         nch = std::min<int>(nch, (int)g.jobs.size());
+        if (!staged) {
+            // device-resident group: one chunk, the whole group (nothing to pipeline)
+            Chunk ch = std::move(whole);
+            ch.group = gi;
+            ch.index = 0;
+            ch.device = g.device;
+            ch.level = g.level;
+            ch.arena_len = 0;
+            f->chunks.push_back(std::move(ch));
+            continue;
+        }
         std::vector<std::vector<int32_t>> parts;
         for (;;) {
             split_group(c, *f, g, nch, parts);
@@ -446,7 +488,7 @@ svp_status plan_flush(Ctx* c, Flush* f) {
     }
 
     // ---- ops, streams, dependencies, arena slots
-    std::unordered_map<int32_t, int32_t> vp_last_op;       // per VP: last op of its previous job
+    VpSlots vp_last_op(f->jobs, -1);                       // per VP: last op of its previous job
     struct Slot { uint64_t off, len; int32_t release_op; };
     std::vector<std::vector<Slot>> inflight(c->ngpu);
     std::vector<uint64_t> arena_head(c->ngpu, 0);
@@ -456,8 +498,8 @@ svp_status plan_flush(Ctx* c, Flush* f) {
         const int dev = ch.device;
         std::vector<int32_t> prev;
         for (int32_t ji : ch.jobs) {
-            auto it = vp_last_op.find(f->jobs[ji].vp);
-            if (it != vp_last_op.end()) prev.push_back(it->second);
+            const int32_t lo = vp_last_op[f->jobs[ji].vp];
+            if (lo >= 0) prev.push_back(lo);
         }
         // arena slot (ring) -- waits for the ops that release overlapped regions
         std::vector<int32_t> arena_waits;
