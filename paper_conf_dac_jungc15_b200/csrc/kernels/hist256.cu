@@ -17,8 +17,10 @@
 //  * CTAs walk contiguous (blocked) tile ranges, so a CTA stays in one VP for many tiles
 //    (segment lookups are cached) and flushes its replicas to the VP's global counts
 //    (one atomicAdd per non-zero bin) only at VP boundaries.
-// A VP's ragged head/tail tiles (not 16-B aligned / partial) are read from global memory
-// directly.  A preceding tiny kernel zeroes every segment's counts, so the result
+// A VP's ragged head/tail tiles (not 16-B aligned / partial) go through the ring too: the
+// producer bulk-copies their 16-B-aligned interior, and the consumers read the < 16-B ends
+// from global memory (byte loads of whole ragged tiles had made a CTA holding one ~8x
+// slower than its neighbours: cfg5's hist launch ran at 65 % SM-active, ncu).  A preceding tiny kernel zeroes every segment's counts, so the result
 // overwrites the output and is bit-exact (integer adds commute).
 #include <string.h>
 
@@ -84,6 +86,13 @@ __device__ __forceinline__ void hist_flush(uint32_t* h, uint32_t* counts) {
     consumers_sync();
 }
 
+// [a, b): the 16-B-aligned interior (in element = byte indices) of the byte range [e0, e1)
+// of the buffer at `base`; b <= a when the range holds no aligned 16-B block.
+__device__ __forceinline__ void aligned_interior(uint64_t base, int64_t e0, int64_t e1, int64_t& a, int64_t& b) {
+    a = (int64_t)(((base + (uint64_t)e0 + 15) & ~15ull) - base);
+    b = (int64_t)(((base + (uint64_t)e1) & ~15ull) - base);
+}
+
 // Segment of tile t with a one-entry cache (tiles of a CTA are contiguous): [lo, hi) is
 // the tile range the cached segment owns.
 struct SegCache {
@@ -138,7 +147,17 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
                     mbar_expect_tx(&full[s], kHistTile);
                     bulk_g2s(ring + s * kHistTile, reinterpret_cast<const uint8_t*>(sd.ptr[0]) + e0, kHistTile, &full[s]);
                 } else {
-                    mbar_arrive(&full[s]);  // consumers read this tile from global memory
+                    // ragged head/tail tile: bulk-copy its 16-B-aligned interior too; the
+                    // consumers read the < 16-B ends from global memory
+                    int64_t a, b;
+                    aligned_interior(sd.ptr[0], e0, e1, a, b);
+                    if (b > a) {
+                        mbar_expect_tx(&full[s], (uint32_t)(b - a));
+                        bulk_g2s(ring + s * kHistTile, reinterpret_cast<const uint8_t*>(sd.ptr[0]) + a, (uint32_t)(b - a),
+                                 &full[s]);
+                    } else {
+                        mbar_arrive(&full[s]);  // < 32 B: consumers read it from global memory
+                    }
                 }
             }
         }
@@ -184,21 +203,33 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
         } else {
+            // ragged head/tail tile: aligned interior from the stage, the ends (< 16 B each,
+            // or the whole tile when it holds no aligned 16 B) from global memory
+            const uint8_t* __restrict__ d = reinterpret_cast<const uint8_t*>(sd.ptr[0]);
+            int64_t a, b;
+            aligned_interior(sd.ptr[0], e0, e1, a, b);
+            if (b > a) {
+                const uint4* st = reinterpret_cast<const uint4*>(ring + s * kHistTile);
+                const int nv = (int)((b - a) >> 4);
+                for (int i = threadIdx.x; i < nv; i += kHistConsumers) {
+                    const uint4 r = st[i];
+                    hist_add_word(hl, r.x);
+                    hist_add_word(hl, r.y);
+                    hist_add_word(hl, r.z);
+                    hist_add_word(hl, r.w);
+                }
+                const int th = threadIdx.x;
+                if (th < 16) {
+                    if (e0 + th < a) hist_add_byte(hl, d[e0 + th]);
+                } else if (th < 32) {
+                    if (b + (th - 16) < e1) hist_add_byte(hl, d[b + (th - 16)]);
+                }
+            } else {
+                for (int64_t e = e0 + threadIdx.x; e < e1; e += kHistConsumers) hist_add_byte(hl, d[e]);
+            }
+            // release after the stage was consumed (see the vec path)
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
-            // ragged head/tail tile: 8 independent byte loads in flight per thread
-            const uint8_t* __restrict__ d = reinterpret_cast<const uint8_t*>(sd.ptr[0]);
-            for (int64_t e = e0 + threadIdx.x; e < e1; e += kHistConsumers * 8) {
-                uint32_t v[8];
-#pragma unroll
-                for (int k = 0; k < 8; ++k) {
-                    const int64_t i = e + k * kHistConsumers;
-                    v[k] = i < e1 ? (uint32_t)d[i] : 256u;
-                }
-#pragma unroll
-                for (int k = 0; k < 8; ++k)
-                    if (v[k] < 256u) hist_add_byte(hl, v[k]);
-            }
         }
     }
     if (cur >= 0) hist_flush(h, cur_counts);

@@ -211,6 +211,50 @@ def test_residency_validation_ranges(level):
     ctx.close()
 
 
+@pytest.mark.parametrize("table_mode", [0, 1])
+def test_hist256_ragged_tiles_every_alignment(table_mode):
+    """hist256 head/tail tiles: the producer bulk-copies their 16-B-aligned interior and
+    the consumers read the < 16-B ends from global memory.  Every start offset mod 16 and
+    sizes around 16 B, 32 B and the 16-KiB tile, uniform / skewed / constant data, in one
+    coalesced launch; counts must equal the oracle's exactly."""
+    ctx = svp.Context(num_gpus=1, table_mode=table_mode)
+    kh = ctx.register_kernel("hist256")
+    T = 16384
+    sizes = [1, 15, 16, 17, 31, 32, 33, 47, 100, T - 1, T, T + 1, T + 15, 2 * T + 7, 3 * T - 5, 5 * T + 333]
+    g = np.random.default_rng(1234)
+    jobs, host, bufs, counts = [], [], [], []
+    vp = 0
+    for off in range(16):
+        for n in sizes[off % 4::4] + [sizes[(off * 7) % len(sizes)]]:
+            kind = vp % 3
+            if kind == 0:
+                d = g.integers(0, 256, size=n, dtype=np.uint8)
+            elif kind == 1:
+                d = np.where(g.random(n) < 0.9, np.uint8(g.integers(0, 256)), g.integers(0, 256, size=n)).astype(np.uint8)
+            else:
+                d = np.full(n, 200 + off, dtype=np.uint8)
+            raw = torch.empty(n + 64, dtype=torch.uint8, device="cuda")
+            raw[off:off + n].copy_(torch.from_numpy(d))
+            cnt = torch.full((256,), 0xDEADBEEF & 0x7FFFFFFF, dtype=torch.int32, device="cuda")
+            jobs.append((vp, kh, svp.args_hist256(n), [(raw.data_ptr() + off, n, svp.DIR_IN, svp.MEM_DEVICE),
+                                                      (cnt.data_ptr(), 1024, svp.DIR_OUT, svp.MEM_DEVICE)]))
+            host.append(d)
+            bufs.append(raw)
+            counts.append(cnt)
+            vp += 1
+    try:
+        ctx.submit_batch(jobs)
+        ctx.flush()
+        torch.cuda.synchronize()
+        assert ctx.flush_stats()["launches"] == 1
+        for v, (d, cnt) in enumerate(zip(host, counts)):
+            want = oracle.hist256(d).astype(np.int64)
+            got = cnt.cpu().numpy().view(np.uint32).astype(np.int64)
+            assert np.array_equal(got, want), (v, len(d))
+    finally:
+        ctx.close()
+
+
 def test_repeated_flushes_reuse_tables(small):
     specs, inputs = small
     ctx = svp.Context(num_gpus=1)
