@@ -69,7 +69,12 @@ typedef struct svp_config {
     uint64_t arena_bytes;        /* per-GPU device staging arena for host-resident buffers;
                                     0 = 2 GiB.  Allocated lazily on first host-resident job.  */
     int32_t profile_level;       /* 0: no events; 1: CUDA events around every op (per-VP
-                                    attribution, kernel stats)                                */
+                                    attribution by algorithmic work, kernel stats); 2: as 1,
+                                    and every vecadd/SAXPY/Black-Scholes/hist256 launch also
+                                    counts the SM clock cycles thread 0 of each CTA spends in
+                                    each tile, per segment -- the launch's time is then split
+                                    over its VPs by those measured cycles (GEMM launches keep
+                                    the FLOP split)                                           */
     int32_t sync_each_job;       /* serial baseline B1: stream-synchronize after every job    */
     int32_t dry_run;             /* 1: plan only -- no CUDA call at all, op times simulated
                                     by the cost model (host-logic tests on CPU)               */
@@ -276,7 +281,8 @@ svp_status svp_lpt_partition(int32_t n, const int32_t* classes, const double* co
 /* Per-VP attribution of device-timed op durations (the profiler
  * "acquires execution information such as ... the elapsed clock cycles"): an op's
  * event-timed duration is split over its member VPs in proportion to their
- * algorithmic bytes (FLOPs for SGEMM).  Needs profile_level >= 1.  vp = -1 returns
+ * algorithmic bytes (FLOPs for SGEMM), or with profile_level 2 for segment launches in
+ * proportion to the measured SM cycles of each VP's tiles.  Needs profile_level >= 1.  vp = -1 returns
  * device-wide totals (sum over VPs, plus op counts). */
 typedef struct svp_vp_profile {
     uint64_t jobs;

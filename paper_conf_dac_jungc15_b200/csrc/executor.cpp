@@ -68,6 +68,9 @@ struct Dev {
     std::vector<cudaEvent_t> end_ev;
     uint8_t* arena = nullptr;
     uint64_t arena_bytes = 0;
+    // profile_level 2: per-segment busy-cycle counters of this flush's segment launches
+    uint64_t* busy_dev = nullptr;
+    size_t busy_cap = 0;  // counters
     uint8_t* tbl_host = nullptr;
     uint8_t* tbl_dev = nullptr;
     size_t tbl_cap = 0;
@@ -134,6 +137,7 @@ static void dev_teardown(Dev& d) {
     if (d.ext_ev) cudaEventDestroy(d.ext_ev);
     if (d.tbl_ev) cudaEventDestroy(d.tbl_ev);
     if (d.arena) cudaFree(d.arena);
+    if (d.busy_dev) cudaFree(d.busy_dev);
     if (d.tbl_dev) cudaFree(d.tbl_dev);
     if (d.tbl_host) cudaFreeHost(d.tbl_host);
 }
@@ -480,6 +484,11 @@ static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bo
 static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStream_t s) {
     if (ch.total_tiles == 0 && ch.kernel != K_HIST256) return cudaSuccess;
     const uint8_t* base = d.tbl_dev;
+    uint64_t* busy = ch.busy_off >= 0 ? d.busy_dev + ch.busy_off : nullptr;
+    if (busy) {
+        cudaError_t e = cudaMemsetAsync(busy, 0, (size_t)ch.nsegs * sizeof(uint64_t), s);
+        if (e) return e;
+    }
     auto grid_of = [&](int per_sm) {
         if (ch.co_grid > 0) per_sm = std::min(per_sm, (int)ch.co_grid);
         return (int)std::max<uint64_t>(1, std::min<uint64_t>(ch.total_tiles, (uint64_t)d.lim.num_sms * per_sm));
@@ -489,32 +498,32 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
         const SegDesc* p = reinterpret_cast<const SegDesc*>(d.tbl_last.data() + ch.table_off);
         switch (ch.kernel) {
             case K_VECADD:
-            case K_SAXPY: return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.ew_blocks_per_sm), s);
+            case K_SAXPY: return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.ew_blocks_per_sm), s, busy);
             case K_BLACKSCHOLES:
-                return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.bs_blocks_per_sm), s);
+                return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.bs_blocks_per_sm), s, busy);
             case K_EW_MIX:
-                return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.mix_blocks_per_sm), s);
+                return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.mix_blocks_per_sm), s, busy);
             case K_HIST256:
-                return launch_hist256_param(p, ch.nsegs, ch.total_tiles, grid_of(d.lim.hist_blocks_per_sm), s);
+                return launch_hist256_param(p, ch.nsegs, ch.total_tiles, grid_of(d.lim.hist_blocks_per_sm), s, busy);
         }
         return cudaErrorInvalidValue;
     }
     switch (ch.kernel) {
         case K_VECADD:
             return launch_vecadd((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
-                                 grid_of(d.lim.ew_blocks_per_sm), s);
+                                 grid_of(d.lim.ew_blocks_per_sm), s, busy);
         case K_SAXPY:
             return launch_saxpy((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
-                                grid_of(d.lim.ew_blocks_per_sm), s);
+                                grid_of(d.lim.ew_blocks_per_sm), s, busy);
         case K_BLACKSCHOLES:
             return launch_blackscholes((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
-                                       grid_of(d.lim.bs_blocks_per_sm), s);
+                                       grid_of(d.lim.bs_blocks_per_sm), s, busy);
         case K_EW_MIX:
             return launch_ew_mix((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
-                                 grid_of(d.lim.mix_blocks_per_sm), s);
+                                 grid_of(d.lim.mix_blocks_per_sm), s, busy);
         case K_HIST256:
             return launch_hist256((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
-                                  grid_of(d.lim.hist_blocks_per_sm), s);
+                                  grid_of(d.lim.hist_blocks_per_sm), s, busy);
         case K_SGEMM:
             if (sgemm_impl == SVP_SGEMM_TF32BF16)
                 return launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
@@ -618,6 +627,30 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             std::lock_guard<std::mutex> lk(c->pmu);  // one worker thread per GPU updates fstats
             c->fstats.table_uploads += 1;
             c->fstats.table_bytes += bytes;
+        }
+    }
+    // ---- profile_level 2: busy-cycle counters for every segment launch on this GPU
+    {
+        size_t nbusy = 0;
+        for (auto& ch : f.chunks) {
+            if (ch.device != d.idx) continue;
+            ch.busy_off = -1;
+            ch.busy.clear();
+            if (c->cfg.profile_level >= 2 && is_seg_kernel(ch.kernel) && ch.nsegs > 0 && chunk_needs_launch(f, ch)) {
+                ch.busy_off = (int64_t)nbusy;
+                nbusy += (size_t)ch.nsegs;
+            }
+        }
+        if (nbusy > d.busy_cap) {
+            if (d.gexec) {  // a captured graph holds the old counter addresses
+                CK(cudaGraphExecDestroy(d.gexec));
+                d.gexec = nullptr;
+            }
+            if (d.busy_dev) CK(cudaFree(d.busy_dev));
+            d.busy_dev = nullptr;
+            d.busy_cap = 0;
+            CK(cudaMalloc(&d.busy_dev, std::max<size_t>(nbusy, 256) * sizeof(uint64_t)));
+            d.busy_cap = std::max<size_t>(nbusy, 256);
         }
     }
     // ---- steady-state replay: second sighting of a plan -> capture, later -> replay
@@ -817,11 +850,23 @@ static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool u
         std::lock_guard<std::mutex> lk(c->pmu);
         c->fstats.device_ns = std::max(c->fstats.device_ns, (double)span * 1e6);
     }
+    // ---- profile_level 2: measured busy cycles per segment (the kernels are done)
+    size_t nbusy = 0;
+    for (const auto& ch : f.chunks)
+        if (ch.device == d.idx && ch.busy_off >= 0) nbusy = std::max(nbusy, (size_t)ch.busy_off + ch.nsegs);
+    if (nbusy) {
+        std::vector<uint64_t> hb(nbusy);
+        CK(cudaMemcpy(hb.data(), d.busy_dev, nbusy * sizeof(uint64_t), cudaMemcpyDeviceToHost));
+        for (auto& ch : f.chunks)
+            if (ch.device == d.idx && ch.busy_off >= 0)
+                ch.busy.assign(hb.begin() + ch.busy_off, hb.begin() + ch.busy_off + ch.nsegs);
+    }
     return SVP_OK;
 }
 
 // Profiler attribution (a10): w_v = algorithmic bytes (FLOPs for SGEMM) of the VP's job
-// in the op; T_v = T_op * w_v / sum w.  Conservation (sum_v T_v = T_op) holds exactly up
+// in the op -- or, with profile_level 2, the SM cycles measured on the VP's tiles of a
+// segment launch; T_v = T_op * w_v / sum w.  Conservation (sum_v T_v = T_op) holds exactly up
 // to fp64 rounding.
 static void attribute(Ctx* c, const Flush& f) {
     std::lock_guard<std::mutex> lk(c->pmu);
@@ -843,10 +888,17 @@ static void attribute(Ctx* c, const Flush& f) {
         if (o.measured_ns < 0) continue;
         double wsum = 0;
         std::vector<double> w(ch.jobs.size());
+        // profile_level 2: a segment launch is split by the measured SM cycles of each VP's
+        // tiles (when any were recorded), every other op by algorithmic work
+        double bsum = 0;
+        const bool measured = o.kind == SVP_OP_KERNEL && ch.busy.size() == ch.jobs.size();
+        if (measured)
+            for (uint64_t b : ch.busy) bsum += (double)b;
         for (size_t k = 0; k < ch.jobs.size(); ++k) {
             const Job& j = f.jobs[ch.jobs[k]];
             if (o.kind == SVP_OP_H2D) w[k] = (double)j.host_in_bytes;
             else if (o.kind == SVP_OP_D2H) w[k] = (double)j.host_out_bytes;
+            else if (measured && bsum > 0) w[k] = (double)ch.busy[k];
             else w[k] = j.flops > 0 ? j.flops : j.alg_bytes;
             wsum += w[k];
         }

@@ -45,6 +45,8 @@ inline bool is_gemm(int32_t k) { return k == K_SGEMM || k == K_SGEMM_TF32 || k =
 // kernels the heterogeneous launch can carry: same CTA shape (256 threads, no shared
 // memory) and the same SegDesc tile mapping
 inline bool is_ew(int32_t k) { return k == K_VECADD || k == K_SAXPY || k == K_BLACKSCHOLES; }
+// launches that read a SegDesc segment table (tile -> VP segment)
+inline bool is_seg_kernel(int32_t k) { return is_ew(k) || k == K_EW_MIX || k == K_HIST256; }
 const KernelDesc* kernel_by_name(const char* name);
 
 // ------------------------------------------------------------------ jobs
@@ -98,6 +100,10 @@ struct Chunk {
     bool param = false;             // table_mode param: the SegDesc table goes by value
     int32_t co_grid = 0;            // >0: launch with co_grid CTAs per SM so the kernel
                                     // co-resides with a tensor-core SGEMM on the same SMs
+    // profile_level 2 (segment launches): offset of this launch's per-segment busy-cycle
+    // counters in the GPU's counter buffer (-1: none), and their values after the flush
+    int64_t busy_off = -1;
+    std::vector<uint64_t> busy;
 };
 
 struct Op {

@@ -241,25 +241,36 @@ __device__ __forceinline__ void bs_tile(const SegDesc& sd, uint32_t lt) {
 // --------------------------------------------------------------------- kernels
 // Homogeneous coalesced launches: every segment runs the same tile body.  NAME reads a
 // global segment table, NAME##_p receives it by value (table_mode param).
-#define SVP_EW_KERNEL(NAME, BODY)                                                               \
-    __device__ __forceinline__ void NAME##_loop(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) { \
+// `busy` (profile_level 2, else null): thread 0 of every CTA adds the SM clock cycles it
+// spent in each tile to busy[segment] -- the measured per-VP split of the launch's time
+// (the Profiler's second opinion next to the algorithmic-byte split).  The tile's start
+// cycle goes through shared memory so no register stays live across the tile body.
+#define SVP_EW_KERNEL(NAME, BODY, MINB)                                                               \
+    __device__ __forceinline__ void NAME##_loop(const SegDesc* __restrict__ segs, int nsegs, uint32_t total, \
+                                                unsigned long long* __restrict__ busy) {        \
+        __shared__ long long tile_c0;                                                           \
         for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {                              \
-            const SegDesc& sd = segs[find_seg(segs, nsegs, t)];                                 \
+            const int si = find_seg(segs, nsegs, t);                                            \
+            const SegDesc& sd = segs[si];                                                       \
+            if (busy && threadIdx.x == 0) tile_c0 = clock64();                                  \
             BODY(sd, t - sd.tile_begin);                                                        \
+            if (busy && threadIdx.x == 0) atomicAdd(busy + si, (unsigned long long)(clock64() - tile_c0)); \
         }                                                                                       \
     }                                                                                           \
-    __global__ void __launch_bounds__(kEwThreads) NAME(const SegDesc* __restrict__ segs, int nsegs, \
-                                                       uint32_t total) {                        \
-        NAME##_loop(segs, nsegs, total);                                                        \
+    __global__ void __launch_bounds__(kEwThreads, MINB) NAME(const SegDesc* __restrict__ segs, int nsegs, \
+                                                       uint32_t total, unsigned long long* busy) { \
+        NAME##_loop(segs, nsegs, total, busy);                                                  \
     }                                                                                           \
     template <int CAP>                                                                          \
-    __global__ void __launch_bounds__(kEwThreads) NAME##_p(const __grid_constant__ SegParamT<CAP> p, int nsegs, \
-                                                           uint32_t total) {                    \
-        NAME##_loop(p.s, nsegs, total);                                                         \
+    __global__ void __launch_bounds__(kEwThreads, MINB) NAME##_p(const __grid_constant__ SegParamT<CAP> p, int nsegs, \
+                                                           uint32_t total, unsigned long long* busy) { \
+        NAME##_loop(p.s, nsegs, total, busy);                                                   \
     }
-SVP_EW_KERNEL(k_vecadd, vecadd_tile)
-SVP_EW_KERNEL(k_saxpy, saxpy_tile)
-SVP_EW_KERNEL(k_blackscholes, bs_tile)
+// MINB: vecadd / SAXPY keep 6 resident CTAs per SM (<= 40 registers; the grid is sized
+// from k_vecadd's occupancy), Black-Scholes 4
+SVP_EW_KERNEL(k_vecadd, vecadd_tile, 6)
+SVP_EW_KERNEL(k_saxpy, saxpy_tile, 6)
+SVP_EW_KERNEL(k_blackscholes, bs_tile, 4)
 
 // Heterogeneous coalescing (NEXT f4, cfg.hetero): ONE launch carries the vecadd, SAXPY
 // and Black-Scholes segments of a (level, GPU); each segment's kernel id sits in its
@@ -273,37 +284,38 @@ __device__ __forceinline__ void mix_tile(const SegDesc& sd, uint32_t lt) {
         default: bs_tile(sd, lt); break;     // K_BLACKSCHOLES
     }
 }
-SVP_EW_KERNEL(k_ew_mix, mix_tile)
+SVP_EW_KERNEL(k_ew_mix, mix_tile, 3)
 
 // --------------------------------------------------------------------- launchers
-cudaError_t launch_vecadd(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
-    k_vecadd<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
+cudaError_t launch_vecadd(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy) {
+    k_vecadd<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
     return cudaGetLastError();
 }
-cudaError_t launch_saxpy(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
-    k_saxpy<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
+cudaError_t launch_saxpy(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy) {
+    k_saxpy<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
     return cudaGetLastError();
 }
-cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
-    k_blackscholes<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
+cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy) {
+    k_blackscholes<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
     return cudaGetLastError();
 }
 
-cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
-    k_ew_mix<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total);
+cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy) {
+    k_ew_mix<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
     return cudaGetLastError();
 }
 
 template <int CAP>
 static cudaError_t launch_ew_param_cap(int kind, const SegDesc* segs, int nsegs, uint32_t total, int grid,
-                                      cudaStream_t s) {
+                                      cudaStream_t s, uint64_t* busy_) {
+    unsigned long long* busy = reinterpret_cast<unsigned long long*>(busy_);
     SegParamT<CAP> p;
     memcpy(p.s, segs, (size_t)nsegs * sizeof(SegDesc));
     switch (kind) {
-        case 1: k_vecadd_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
-        case 2: k_saxpy_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
-        case 4: k_blackscholes_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
-        case 8: k_ew_mix_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total); break;
+        case 1: k_vecadd_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy); break;
+        case 2: k_saxpy_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy); break;
+        case 4: k_blackscholes_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy); break;
+        case 8: k_ew_mix_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy); break;
         default: return cudaErrorInvalidValue;
     }
     return cudaGetLastError();
@@ -315,11 +327,12 @@ bool param_full_block() {
     return full;
 }
 
-cudaError_t launch_ew_param(int kind, const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+cudaError_t launch_ew_param(int kind, const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s,
+                            uint64_t* busy) {
     if (param_full_block() && nsegs <= kParamSegs)
-        return launch_ew_param_cap<kParamSegs>(kind, segs, nsegs, total, grid, s);
-    if (nsegs <= 16) return launch_ew_param_cap<16>(kind, segs, nsegs, total, grid, s);
-    if (nsegs <= kParamSegs) return launch_ew_param_cap<kParamSegs>(kind, segs, nsegs, total, grid, s);
+        return launch_ew_param_cap<kParamSegs>(kind, segs, nsegs, total, grid, s, busy);
+    if (nsegs <= 16) return launch_ew_param_cap<16>(kind, segs, nsegs, total, grid, s, busy);
+    if (nsegs <= kParamSegs) return launch_ew_param_cap<kParamSegs>(kind, segs, nsegs, total, grid, s, busy);
     return cudaErrorInvalidValue;
 }
 

@@ -108,7 +108,8 @@ struct SegCache {
     }
 };
 
-__device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
+__device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int nsegs, uint32_t total,
+                                          unsigned long long* __restrict__ busy) {
     extern __shared__ __align__(128) uint8_t hsm[];
     uint8_t* ring = hsm;                                                         // [stages][tile]
     uint32_t* h = reinterpret_cast<uint32_t*>(hsm + kHistStages * kHistTile);     // [256][32]
@@ -183,6 +184,9 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
         tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, kHistTile, e0, e1, vec);
         const int s = it % kHistStages;
         const uint32_t ph = (it / kHistStages) & 1;
+        // profile_level 2: thread 0's cycles per tile (from the wait for the stage to the
+        // release) -> busy[segment]
+        const long long c0 = (busy && threadIdx.x == 0) ? clock64() : 0;
         mbar_wait(&full[s], ph);
         if (vec) {
             const uint4* st = reinterpret_cast<const uint4*>(ring + s * kHistTile) + threadIdx.x;
@@ -231,17 +235,19 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
         }
+        if (busy && threadIdx.x == 0) atomicAdd(busy + si, (unsigned long long)(clock64() - c0));
     }
     if (cur >= 0) hist_flush(h, cur_counts);
 }
 
-__global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total) {
-    hist_body(segs, nsegs, total);
+__global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total,
+                                                        unsigned long long* busy) {
+    hist_body(segs, nsegs, total, busy);
 }
 template <int CAP>
 __global__ void __launch_bounds__(kHistBlock) k_hist256_p(const __grid_constant__ SegParamT<CAP> p, int nsegs,
-                                                          uint32_t total) {
-    hist_body(p.s, nsegs, total);
+                                                          uint32_t total, unsigned long long* busy) {
+    hist_body(p.s, nsegs, total, busy);
 }
 
 template <int CAP>
@@ -269,35 +275,36 @@ static cudaError_t hist_attr() {
     return cudaSuccess;
 }
 
-cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy) {
     if (nsegs <= 0) return cudaSuccess;
     k_hist_zero<<<nsegs < 1024 ? nsegs : 1024, 256, 0, s>>>(segs, nsegs);
     cudaError_t e = cudaGetLastError();
     if (e || total == 0) return e;
     if ((e = hist_attr())) return e;
-    k_hist256<<<grid, kHistBlock, kHistSmem, s>>>(segs, nsegs, total);
+    k_hist256<<<grid, kHistBlock, kHistSmem, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
     return cudaGetLastError();
 }
 
 template <int CAP>
 static cudaError_t launch_hist256_param_cap(const SegDesc* segs, int nsegs, uint32_t total, int grid,
-                                            cudaStream_t s) {
+                                            cudaStream_t s, uint64_t* busy) {
     SegParamT<CAP> p;
     memcpy(p.s, segs, (size_t)nsegs * sizeof(SegDesc));
     k_hist_zero_p<CAP><<<nsegs, 256, 0, s>>>(p, nsegs);
     cudaError_t e = cudaGetLastError();
     if (e || total == 0) return e;
     if ((e = hist_attr_p<CAP>())) return e;
-    k_hist256_p<CAP><<<grid, kHistBlock, kHistSmem, s>>>(p, nsegs, total);
+    k_hist256_p<CAP><<<grid, kHistBlock, kHistSmem, s>>>(p, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
     return cudaGetLastError();
 }
 
-cudaError_t launch_hist256_param(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s) {
+cudaError_t launch_hist256_param(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s,
+                                 uint64_t* busy) {
     if (nsegs <= 0) return cudaSuccess;
     if (param_full_block() && nsegs <= kParamSegs)
-        return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s);
-    if (nsegs <= 16) return launch_hist256_param_cap<16>(segs, nsegs, total, grid, s);
-    if (nsegs <= kParamSegs) return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s);
+        return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s, busy);
+    if (nsegs <= 16) return launch_hist256_param_cap<16>(segs, nsegs, total, grid, s, busy);
+    if (nsegs <= kParamSegs) return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s, busy);
     return cudaErrorInvalidValue;
 }
 

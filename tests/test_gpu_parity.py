@@ -153,6 +153,44 @@ def test_profiler_conservation_and_kernel_stats(small):
     ctx.close()
 
 
+def test_profiler_measured_split_level2():
+    """profile_level 2 (a10 second opinion): a segment launch's event-timed duration is
+    split over its VPs by the SM cycles measured on their tiles.  Outputs stay exact, the
+    split conserves the launch time, and for full-tile VPs it agrees with the algorithmic
+    byte split of level 1 (uniform work per tile) within 25 %."""
+    sizes = [1 << 22, 1 << 20, (1 << 20) + 12345, 3 << 20]
+    specs = [W.JobSpec(v, "vecadd", n=n) for v, n in enumerate(sizes)]
+    specs += [W.JobSpec(4 + v, "hist256", n=n) for v, n in enumerate(sizes)]
+    inputs = inputs_for(specs)
+    shares = {}
+    for level in (1, 2):
+        ctx = svp.Context(num_gpus=1, profile_level=level)
+        try:
+            vs = VPSet(ctx, specs, inputs, "device")
+            jb = svp.JobBatch(vs.job_list())
+            ctx.submit_batch(jb)
+            ctx.flush()
+            ctx.reset_profile()
+            for _ in range(3):
+                ctx.submit_batch(jb)
+                ctx.flush()
+            torch.cuda.synchronize()
+            for i, (sp, inp) in enumerate(zip(specs, inputs)):
+                check_job(sp, inp, vs.output(i))
+            per_vp = [ctx.profile(sp.vp)["kernel_ns"] for sp in specs]
+            tot = ctx.profile(-1)["kernel_ns"]
+            ks = sum(ctx.kernel_stats(ctx.kernel_ids[k])["total_ns"] for k in ("vecadd", "hist256"))
+            assert abs(sum(per_vp) - tot) <= 1e-6 * tot and abs(tot - ks) <= 1e-6 * ks
+            assert all(x > 0 for x in per_vp)
+            shares[level] = per_vp
+        finally:
+            ctx.close()
+    for lo, hi in ((0, 4), (4, 8)):
+        s1 = np.array(shares[1][lo:hi]) / sum(shares[1][lo:hi])
+        s2 = np.array(shares[2][lo:hi]) / sum(shares[2][lo:hi])
+        assert np.all(np.abs(s2 / s1 - 1) < 0.25), (lo, s1, s2)
+
+
 def test_external_stream_join(small):
     specs, inputs = small
     s = torch.cuda.Stream()
