@@ -17,6 +17,7 @@
 //        PAPER.md L253-257 (the profiler "acquires ... elapsed clock cycles").
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -71,6 +72,9 @@ struct Dev {
     // profile_level 2: per-segment busy-cycle counters of this flush's segment launches
     uint64_t* busy_dev = nullptr;
     size_t busy_cap = 0;  // counters
+    // dynamic tile order of Black-Scholes / mixed launches: 2 self-resetting u32 per launch
+    uint32_t* sched_dev = nullptr;
+    size_t sched_cap = 0;  // slots
     uint8_t* tbl_host = nullptr;
     uint8_t* tbl_dev = nullptr;
     size_t tbl_cap = 0;
@@ -138,6 +142,7 @@ static void dev_teardown(Dev& d) {
     if (d.tbl_ev) cudaEventDestroy(d.tbl_ev);
     if (d.arena) cudaFree(d.arena);
     if (d.busy_dev) cudaFree(d.busy_dev);
+    if (d.sched_dev) cudaFree(d.sched_dev);
     if (d.tbl_dev) cudaFree(d.tbl_dev);
     if (d.tbl_host) cudaFreeHost(d.tbl_host);
 }
@@ -481,10 +486,17 @@ static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bo
     return pool[i];
 }
 
+// Dynamic tile order for Black-Scholes / mixed launches (SVP_EW_DYN=0: static order).
+static bool ew_dynamic_order() {
+    static const bool on = !(getenv("SVP_EW_DYN") && atoi(getenv("SVP_EW_DYN")) == 0);
+    return on;
+}
+
 static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStream_t s) {
     if (ch.total_tiles == 0 && ch.kernel != K_HIST256) return cudaSuccess;
     const uint8_t* base = d.tbl_dev;
     uint64_t* busy = ch.busy_off >= 0 ? d.busy_dev + ch.busy_off : nullptr;
+    uint32_t* sched = ch.sched_slot >= 0 ? d.sched_dev + 2 * ch.sched_slot : nullptr;
     if (busy) {
         cudaError_t e = cudaMemsetAsync(busy, 0, (size_t)ch.nsegs * sizeof(uint64_t), s);
         if (e) return e;
@@ -500,9 +512,9 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
             case K_VECADD:
             case K_SAXPY: return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.ew_blocks_per_sm), s, busy);
             case K_BLACKSCHOLES:
-                return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.bs_blocks_per_sm), s, busy);
+                return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.bs_blocks_per_sm), s, busy, sched);
             case K_EW_MIX:
-                return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.mix_blocks_per_sm), s, busy);
+                return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.mix_blocks_per_sm), s, busy, sched);
             case K_HIST256:
                 return launch_hist256_param(p, ch.nsegs, ch.total_tiles, grid_of(d.lim.hist_blocks_per_sm), s, busy);
         }
@@ -517,10 +529,10 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
                                 grid_of(d.lim.ew_blocks_per_sm), s, busy);
         case K_BLACKSCHOLES:
             return launch_blackscholes((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
-                                       grid_of(d.lim.bs_blocks_per_sm), s, busy);
+                                       grid_of(d.lim.bs_blocks_per_sm), s, busy, sched);
         case K_EW_MIX:
             return launch_ew_mix((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
-                                 grid_of(d.lim.mix_blocks_per_sm), s, busy);
+                                 grid_of(d.lim.mix_blocks_per_sm), s, busy, sched);
         case K_HIST256:
             return launch_hist256((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
                                   grid_of(d.lim.hist_blocks_per_sm), s, busy);
@@ -651,6 +663,38 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             d.busy_cap = 0;
             CK(cudaMalloc(&d.busy_dev, std::max<size_t>(nbusy, 256) * sizeof(uint64_t)));
             d.busy_cap = std::max<size_t>(nbusy, 256);
+        }
+    }
+    // ---- dynamic tile order (Black-Scholes / mixed launches): one counter slot per launch.
+    // Only for a launch that has the GPU to itself: alone it balances the SMs (cfg5's BS
+    // launch 0.753 -> 0.668 ms, one-stream step +2 %), but co-running with the other
+    // kernels of an interleaved level it cost 0.7 % of the step (profiles/r01/ew_dyn/).
+    {
+        std::map<int32_t, int> kernels_in_level;
+        for (const auto& ch : f.chunks)
+            if (ch.device == d.idx && ch.total_tiles > 0) kernels_in_level[ch.level] += 1;
+        size_t nslot = 0;
+        for (auto& ch : f.chunks) {
+            if (ch.device != d.idx) continue;
+            ch.sched_slot = -1;
+            const bool alone = !c->cfg.interleave || kernels_in_level[ch.level] == 1;
+            if (ew_dynamic_order() && alone && (ch.kernel == K_BLACKSCHOLES || ch.kernel == K_EW_MIX) &&
+                ch.total_tiles > 0)
+                ch.sched_slot = (int32_t)nslot++;
+        }
+        if (nslot > d.sched_cap) {
+            if (d.gexec) {  // a captured graph holds the old counter addresses
+                CK(cudaGraphExecDestroy(d.gexec));
+                d.gexec = nullptr;
+            }
+            // the previous flush's launches have finished (svp_flush is synchronous)
+            if (d.sched_dev) CK(cudaFree(d.sched_dev));
+            d.sched_dev = nullptr;
+            d.sched_cap = 0;
+            const size_t cap = std::max<size_t>(nslot, 64);
+            CK(cudaMalloc(&d.sched_dev, cap * 2 * sizeof(uint32_t)));
+            CK(cudaMemset(d.sched_dev, 0, cap * 2 * sizeof(uint32_t)));
+            d.sched_cap = cap;
         }
     }
     // ---- steady-state replay: second sighting of a plan -> capture, later -> replay

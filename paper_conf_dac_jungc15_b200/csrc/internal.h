@@ -104,6 +104,7 @@ struct Chunk {
     // counters in the GPU's counter buffer (-1: none), and their values after the flush
     int64_t busy_off = -1;
     std::vector<uint64_t> busy;
+    int32_t sched_slot = -1;        // dynamic tile order: counter slot of this launch (-1: static)
 };
 
 struct Op {

@@ -245,32 +245,61 @@ __device__ __forceinline__ void bs_tile(const SegDesc& sd, uint32_t lt) {
 // spent in each tile to busy[segment] -- the measured per-VP split of the launch's time
 // (the Profiler's second opinion next to the algorithmic-byte split).  The tile's start
 // cycle goes through shared memory so no register stays live across the tile body.
-#define SVP_EW_KERNEL(NAME, BODY, MINB)                                                               \
+// `sched` (null: static t = blockIdx.x + i * gridDim.x): dynamic tile order -- each CTA
+// takes the next tile from sched[0] (fetched one tile ahead), so CTAs on SMs that get a
+// smaller share of the memory system do fewer tiles instead of finishing last; the last
+// CTA to leave resets sched[0..1] to 0 for the next launch on the same slot.
+#define SVP_EW_KERNEL(NAME, BODY, MINB, DYN)                                                       \
+    __device__ __forceinline__ void NAME##_tile_at(const SegDesc* __restrict__ segs, int nsegs, uint32_t t, \
+                                                   unsigned long long* __restrict__ busy, long long& c0) { \
+        const int si = find_seg(segs, nsegs, t);                                                \
+        const SegDesc& sd = segs[si];                                                           \
+        if (busy && threadIdx.x == 0) c0 = clock64();                                           \
+        BODY(sd, t - sd.tile_begin);                                                            \
+        if (busy && threadIdx.x == 0) atomicAdd(busy + si, (unsigned long long)(clock64() - c0)); \
+    }                                                                                           \
     __device__ __forceinline__ void NAME##_loop(const SegDesc* __restrict__ segs, int nsegs, uint32_t total, \
-                                                unsigned long long* __restrict__ busy) {        \
+                                                unsigned long long* __restrict__ busy, uint32_t* sched) { \
         __shared__ long long tile_c0;                                                           \
-        for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {                              \
-            const int si = find_seg(segs, nsegs, t);                                            \
-            const SegDesc& sd = segs[si];                                                       \
-            if (busy && threadIdx.x == 0) tile_c0 = clock64();                                  \
-            BODY(sd, t - sd.tile_begin);                                                        \
-            if (busy && threadIdx.x == 0) atomicAdd(busy + si, (unsigned long long)(clock64() - tile_c0)); \
+        __shared__ uint32_t next_t[2];                                                          \
+        if (!DYN || !sched) {                                                                   \
+            for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) NAME##_tile_at(segs, nsegs, t, busy, tile_c0); \
+            return;                                                                             \
+        }                                                                                       \
+        if (threadIdx.x == 0) next_t[0] = atomicAdd(sched, 1u);                                 \
+        __syncthreads();                                                                        \
+        uint32_t t = next_t[0];                                                                 \
+        for (int i = 0; t < total; ++i) {                                                       \
+            if (threadIdx.x == 0) next_t[(i + 1) & 1] = atomicAdd(sched, 1u);                   \
+            NAME##_tile_at(segs, nsegs, t, busy, tile_c0);                                      \
+            __syncthreads();                                                                    \
+            t = next_t[(i + 1) & 1];                                                            \
+        }                                                                                       \
+        if (threadIdx.x == 0) {                                                                 \
+            __threadfence();                                                                    \
+            if (atomicAdd(sched + 1, 1u) == gridDim.x - 1) {                                    \
+                sched[0] = 0;                                                                   \
+                sched[1] = 0;                                                                   \
+                __threadfence();                                                                \
+            }                                                                                   \
         }                                                                                       \
     }                                                                                           \
     __global__ void __launch_bounds__(kEwThreads, MINB) NAME(const SegDesc* __restrict__ segs, int nsegs, \
-                                                       uint32_t total, unsigned long long* busy) { \
-        NAME##_loop(segs, nsegs, total, busy);                                                  \
+                                                       uint32_t total, unsigned long long* busy, uint32_t* sched) { \
+        NAME##_loop(segs, nsegs, total, busy, sched);                                           \
     }                                                                                           \
     template <int CAP>                                                                          \
     __global__ void __launch_bounds__(kEwThreads, MINB) NAME##_p(const __grid_constant__ SegParamT<CAP> p, int nsegs, \
-                                                           uint32_t total, unsigned long long* busy) { \
-        NAME##_loop(p.s, nsegs, total, busy);                                                   \
+                                                           uint32_t total, unsigned long long* busy, uint32_t* sched) { \
+        NAME##_loop(p.s, nsegs, total, busy, sched);                                            \
     }
 // MINB: vecadd / SAXPY keep 6 resident CTAs per SM (<= 40 registers; the grid is sized
-// from k_vecadd's occupancy), Black-Scholes 4
-SVP_EW_KERNEL(k_vecadd, vecadd_tile, 6)
-SVP_EW_KERNEL(k_saxpy, saxpy_tile, 6)
-SVP_EW_KERNEL(k_blackscholes, bs_tile, 4)
+// from k_vecadd's occupancy), Black-Scholes 4.  DYN: the dynamic tile order is compiled
+// in (Black-Scholes and the mixed launch; vecadd / SAXPY already stream at the measured
+// copy bandwidth with the static order, and the extra path would spill SAXPY at 40 regs).
+SVP_EW_KERNEL(k_vecadd, vecadd_tile, 6, 0)
+SVP_EW_KERNEL(k_saxpy, saxpy_tile, 6, 0)
+SVP_EW_KERNEL(k_blackscholes, bs_tile, 4, 1)
 
 // Heterogeneous coalescing (NEXT f4, cfg.hetero): ONE launch carries the vecadd, SAXPY
 // and Black-Scholes segments of a (level, GPU); each segment's kernel id sits in its
@@ -284,38 +313,42 @@ __device__ __forceinline__ void mix_tile(const SegDesc& sd, uint32_t lt) {
         default: bs_tile(sd, lt); break;     // K_BLACKSCHOLES
     }
 }
-SVP_EW_KERNEL(k_ew_mix, mix_tile, 3)
+SVP_EW_KERNEL(k_ew_mix, mix_tile, 3, 1)
 
 // --------------------------------------------------------------------- launchers
-cudaError_t launch_vecadd(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy) {
-    k_vecadd<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
+cudaError_t launch_vecadd(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy,
+                          uint32_t* sched) {
+    k_vecadd<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy), sched);
     return cudaGetLastError();
 }
-cudaError_t launch_saxpy(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy) {
-    k_saxpy<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
+cudaError_t launch_saxpy(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy,
+                          uint32_t* sched) {
+    k_saxpy<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy), sched);
     return cudaGetLastError();
 }
-cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy) {
-    k_blackscholes<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
+cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy,
+                          uint32_t* sched) {
+    k_blackscholes<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy), sched);
     return cudaGetLastError();
 }
 
-cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy) {
-    k_ew_mix<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
+cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy,
+                          uint32_t* sched) {
+    k_ew_mix<<<grid, kEwThreads, 0, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy), sched);
     return cudaGetLastError();
 }
 
 template <int CAP>
 static cudaError_t launch_ew_param_cap(int kind, const SegDesc* segs, int nsegs, uint32_t total, int grid,
-                                      cudaStream_t s, uint64_t* busy_) {
+                                      cudaStream_t s, uint64_t* busy_, uint32_t* sched) {
     unsigned long long* busy = reinterpret_cast<unsigned long long*>(busy_);
     SegParamT<CAP> p;
     memcpy(p.s, segs, (size_t)nsegs * sizeof(SegDesc));
     switch (kind) {
-        case 1: k_vecadd_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy); break;
-        case 2: k_saxpy_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy); break;
-        case 4: k_blackscholes_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy); break;
-        case 8: k_ew_mix_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy); break;
+        case 1: k_vecadd_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy, sched); break;
+        case 2: k_saxpy_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy, sched); break;
+        case 4: k_blackscholes_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy, sched); break;
+        case 8: k_ew_mix_p<CAP><<<grid, kEwThreads, 0, s>>>(p, nsegs, total, busy, sched); break;
         default: return cudaErrorInvalidValue;
     }
     return cudaGetLastError();
@@ -328,11 +361,11 @@ bool param_full_block() {
 }
 
 cudaError_t launch_ew_param(int kind, const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s,
-                            uint64_t* busy) {
+                            uint64_t* busy, uint32_t* sched) {
     if (param_full_block() && nsegs <= kParamSegs)
-        return launch_ew_param_cap<kParamSegs>(kind, segs, nsegs, total, grid, s, busy);
-    if (nsegs <= 16) return launch_ew_param_cap<16>(kind, segs, nsegs, total, grid, s, busy);
-    if (nsegs <= kParamSegs) return launch_ew_param_cap<kParamSegs>(kind, segs, nsegs, total, grid, s, busy);
+        return launch_ew_param_cap<kParamSegs>(kind, segs, nsegs, total, grid, s, busy, sched);
+    if (nsegs <= 16) return launch_ew_param_cap<16>(kind, segs, nsegs, total, grid, s, busy, sched);
+    if (nsegs <= kParamSegs) return launch_ew_param_cap<kParamSegs>(kind, segs, nsegs, total, grid, s, busy, sched);
     return cudaErrorInvalidValue;
 }
 

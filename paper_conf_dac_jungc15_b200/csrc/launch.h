@@ -26,22 +26,23 @@ cudaError_t query_limits(LaunchLimits* out);
 // Elementwise coalesced kernels: segs/nsegs describe the VPs, total_tiles is
 // segs[nsegs-1].tile_begin + tiles of the last segment.  `busy` (profile_level 2, else
 // null): nsegs zeroed u64 counters; thread 0 of every CTA adds its clock64 cycles per tile
-// to the tile's segment (measured per-VP split of the launch).
+// to the tile's segment (measured per-VP split of the launch).  `sched` (null: static
+// tile order): 2 zeroed u32 -- dynamic tile order; the launch leaves them zeroed again.
 cudaError_t launch_vecadd(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s,
-                        uint64_t* busy = nullptr);
+                        uint64_t* busy = nullptr, uint32_t* sched = nullptr);
 cudaError_t launch_saxpy(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s,
-                        uint64_t* busy = nullptr);
+                        uint64_t* busy = nullptr, uint32_t* sched = nullptr);
 cudaError_t launch_blackscholes(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s,
-                        uint64_t* busy = nullptr);
+                        uint64_t* busy = nullptr, uint32_t* sched = nullptr);
 // Heterogeneous elementwise launch: segment kernel id in flags >> SEG_KIND_SHIFT.
 cudaError_t launch_ew_mix(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s,
-                        uint64_t* busy = nullptr);
+                        uint64_t* busy = nullptr, uint32_t* sched = nullptr);
 // table_mode param: the same kernels with the segment table passed by value; kind = kernel
 // id (1 vecadd, 2 SAXPY, 4 Black-Scholes, 8 mixed), nsegs <= kParamSegs.
 // `segs` is the HOST copy of the table (nsegs <= kParamSegs); it is copied into a
 // parameter block of 16 or 64 segments, the smallest that holds it.
 cudaError_t launch_ew_param(int kind, const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s,
-                            uint64_t* busy = nullptr);
+                            uint64_t* busy = nullptr, uint32_t* sched = nullptr);
 bool param_full_block();  // SVP_PARAM_FULL=1: always the kParamSegs block (A/B knob)
 cudaError_t launch_hist256_param(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s,
                                  uint64_t* busy = nullptr);

@@ -191,6 +191,35 @@ def test_profiler_measured_split_level2():
         assert np.all(np.abs(s2 / s1 - 1) < 0.25), (lo, s1, s2)
 
 
+@pytest.mark.parametrize("hetero", [False, True])
+def test_dynamic_tile_order_repeated(hetero):
+    """A Black-Scholes (or mixed) launch alone on the GPU takes its tiles in dynamic order
+    from a self-resetting counter pair: three flushes in a row, outputs poisoned with NaN
+    before each, must all be recomputed and match the oracle (a counter left non-zero
+    would make the next launch skip tiles)."""
+    kinds = ("blackscholes", "vecadd", "saxpy") if hetero else ("blackscholes",)
+    specs = [W.JobSpec(v, kinds[v % len(kinds)], n=(1 << 18) + 4097 * v, R=0.02, V=0.3, a=1.5) for v in range(9)]
+    inputs = inputs_for(specs)
+    ctx = svp.Context(num_gpus=1, hetero=hetero)
+    try:
+        vs = VPSet(ctx, specs, inputs, "device")
+        jb = svp.JobBatch(vs.job_list())
+        for r in range(3):
+            vs.load_inputs()
+            for i, sp in enumerate(specs):
+                for name in ("call", "put", "c"):
+                    if name in vs.bufs[i]:
+                        vs.bufs[i][name].fill_(float("nan"))
+            ctx.submit_batch(jb)
+            ctx.flush()
+            torch.cuda.synchronize()
+            assert ctx.flush_stats()["launches"] == 1
+            for i, (sp, inp) in enumerate(zip(specs, inputs)):
+                check_job(sp, inp, vs.output(i))
+    finally:
+        ctx.close()
+
+
 def test_external_stream_join(small):
     specs, inputs = small
     s = torch.cuda.Stream()
