@@ -280,11 +280,14 @@ def timed_steps(ctx, jobs, steps, stream):
 
 
 def launches_per_flush(ctx):
+    """Kernel launches per flush: one per plan kernel op, plus hist256's zeroing kernel
+    (absent with SVP_HIST_FUSED=1, the single-launch form)."""
     n = 0
     hist_id = ctx.kernel_ids.get("hist256")
+    zero_kernel = os.environ.get("SVP_HIST_FUSED", "0") in ("", "0")
     for op in ctx.plan():
         if op["kind"] == 1:
-            n += 1 + (1 if op["kernel"] == hist_id else 0)
+            n += 1 + (1 if zero_kernel and op["kernel"] == hist_id else 0)
     return n
 
 

@@ -75,6 +75,9 @@ struct Dev {
     // dynamic tile order of Black-Scholes / mixed launches: 2 self-resetting u32 per launch
     uint32_t* sched_dev = nullptr;
     size_t sched_cap = 0;  // slots
+    // single-launch hist256: per launch nsegs * 257 self-resetting u32 (partials + arrivals)
+    uint32_t* hscr_dev = nullptr;
+    size_t hscr_cap = 0;  // u32
     uint8_t* tbl_host = nullptr;
     uint8_t* tbl_dev = nullptr;
     size_t tbl_cap = 0;
@@ -143,6 +146,7 @@ static void dev_teardown(Dev& d) {
     if (d.arena) cudaFree(d.arena);
     if (d.busy_dev) cudaFree(d.busy_dev);
     if (d.sched_dev) cudaFree(d.sched_dev);
+    if (d.hscr_dev) cudaFree(d.hscr_dev);
     if (d.tbl_dev) cudaFree(d.tbl_dev);
     if (d.tbl_host) cudaFreeHost(d.tbl_host);
 }
@@ -492,11 +496,21 @@ static bool ew_dynamic_order() {
     return on;
 }
 
+// SVP_HIST_FUSED=1: hist256 as ONE launch with a self-resetting per-launch scratch (the
+// last CTA of each VP writes its counts) instead of a zeroing kernel + the accumulating
+// launch.  Off by default: alone it was 2 us (4 %) faster per cfg5 hist launch, but the
+// interleaved cfg5 step measured ~1 % slower with it (profiles/r01/hist_fused/).
+static bool hist_single_launch() {
+    static const bool on = getenv("SVP_HIST_FUSED") && atoi(getenv("SVP_HIST_FUSED")) != 0;
+    return on;
+}
+
 static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStream_t s) {
     if (ch.total_tiles == 0 && ch.kernel != K_HIST256) return cudaSuccess;
     const uint8_t* base = d.tbl_dev;
     uint64_t* busy = ch.busy_off >= 0 ? d.busy_dev + ch.busy_off : nullptr;
     uint32_t* sched = ch.sched_slot >= 0 ? d.sched_dev + 2 * ch.sched_slot : nullptr;
+    uint32_t* hscr = ch.hscr_off >= 0 ? d.hscr_dev + ch.hscr_off : nullptr;
     if (busy) {
         cudaError_t e = cudaMemsetAsync(busy, 0, (size_t)ch.nsegs * sizeof(uint64_t), s);
         if (e) return e;
@@ -516,7 +530,7 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
             case K_EW_MIX:
                 return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.mix_blocks_per_sm), s, busy, sched);
             case K_HIST256:
-                return launch_hist256_param(p, ch.nsegs, ch.total_tiles, grid_of(d.lim.hist_blocks_per_sm), s, busy);
+                return launch_hist256_param(p, ch.nsegs, ch.total_tiles, grid_of(d.lim.hist_blocks_per_sm), s, busy, hscr);
         }
         return cudaErrorInvalidValue;
     }
@@ -535,7 +549,7 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
                                  grid_of(d.lim.mix_blocks_per_sm), s, busy, sched);
         case K_HIST256:
             return launch_hist256((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
-                                  grid_of(d.lim.hist_blocks_per_sm), s, busy);
+                                  grid_of(d.lim.hist_blocks_per_sm), s, busy, hscr);
         case K_SGEMM:
             if (sgemm_impl == SVP_SGEMM_TF32BF16)
                 return launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
@@ -681,6 +695,29 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             if (ew_dynamic_order() && alone && (ch.kernel == K_BLACKSCHOLES || ch.kernel == K_EW_MIX) &&
                 ch.total_tiles > 0)
                 ch.sched_slot = (int32_t)nslot++;
+        }
+        // single-launch hist256 scratch (SVP_HIST_FUSED=0: zeroing kernel + launch)
+        size_t nh = 0;
+        for (auto& ch : f.chunks) {
+            if (ch.device != d.idx) continue;
+            ch.hscr_off = -1;
+            if (hist_single_launch() && ch.kernel == K_HIST256 && ch.nsegs > 0) {
+                ch.hscr_off = (int64_t)nh;
+                nh += (size_t)ch.nsegs * 257;
+            }
+        }
+        if (nh > d.hscr_cap) {
+            if (d.gexec) {
+                CK(cudaGraphExecDestroy(d.gexec));
+                d.gexec = nullptr;
+            }
+            if (d.hscr_dev) CK(cudaFree(d.hscr_dev));
+            d.hscr_dev = nullptr;
+            d.hscr_cap = 0;
+            const size_t cap = std::max<size_t>(nh, 64 * 257);
+            CK(cudaMalloc(&d.hscr_dev, cap * sizeof(uint32_t)));
+            CK(cudaMemset(d.hscr_dev, 0, cap * sizeof(uint32_t)));
+            d.hscr_cap = cap;
         }
         if (nslot > d.sched_cap) {
             if (d.gexec) {  // a captured graph holds the old counter addresses

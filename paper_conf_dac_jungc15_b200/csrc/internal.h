@@ -105,6 +105,7 @@ struct Chunk {
     int64_t busy_off = -1;
     std::vector<uint64_t> busy;
     int32_t sched_slot = -1;        // dynamic tile order: counter slot of this launch (-1: static)
+    int64_t hscr_off = -1;          // single-launch hist256: scratch offset (u32) of this launch
 };
 
 struct Op {

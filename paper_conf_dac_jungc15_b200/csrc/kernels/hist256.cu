@@ -21,7 +21,9 @@
 // producer bulk-copies their 16-B-aligned interior, and the consumers read the < 16-B ends
 // from global memory (byte loads of whole ragged tiles had made a CTA holding one ~8x
 // slower than its neighbours: cfg5's hist launch ran at 65 % SM-active, ncu).  A preceding tiny kernel zeroes every segment's counts, so the result
-// overwrites the output and is bit-exact (integer adds commute).
+// overwrites the output and is bit-exact (integer adds commute).  With a per-launch
+// scratch (the executor's default) there is no zeroing kernel: the last CTA of each VP
+// writes its counts (hist_flush_fused).
 #include <string.h>
 
 #include "../launch.h"
@@ -86,6 +88,41 @@ __device__ __forceinline__ void hist_flush(uint32_t* h, uint32_t* counts) {
     consumers_sync();
 }
 
+// Single-launch form (`scratch` non-null, no zeroing kernel): the CTAs that touch VP `si`
+// add their sums into a per-launch partial histogram scratch[si][256], then count in
+// scratch arrive[si]; the last of the VP's expected CTAs (known from the blocked tile
+// ranges) moves the partial histogram into the VP's counts with plain stores -- the
+// output is overwritten, never accumulated -- and leaves the scratch zeroed for the next
+// launch on the same slot (threadfence-reduction pattern).
+__device__ __forceinline__ uint32_t hist_expected_ctas(const SegDesc* __restrict__ segs, int nsegs, uint32_t total,
+                                                       uint32_t per, int si) {
+    const uint32_t tb = segs[si].tile_begin, te = si + 1 < nsegs ? segs[si + 1].tile_begin : total;
+    return (te - 1) / per - tb / per + 1;
+}
+__device__ __forceinline__ void hist_flush_fused(uint32_t* h, uint32_t* counts, uint32_t* partial, uint32_t* arrive,
+                                                 uint32_t expected, uint32_t* last_flag) {
+    consumers_sync();
+    const int b = threadIdx.x;
+    uint32_t sum = 0;
+#pragma unroll 8
+    for (int j = 0; j < 32; ++j) {
+        const int c = (j + b) & 31;
+        sum += h[b * 32 + c];
+        h[b * 32 + c] = 0;
+    }
+    if (sum) atomicAdd(&partial[b], sum);
+    __threadfence();
+    consumers_sync();
+    if (b == 0) *last_flag = atomicAdd(arrive, 1u) == expected - 1;
+    consumers_sync();
+    if (*last_flag) {
+        __threadfence();
+        counts[b] = atomicExch(&partial[b], 0u);
+        if (b == 0) *arrive = 0;
+    }
+    consumers_sync();
+}
+
 // [a, b): the 16-B-aligned interior (in element = byte indices) of the byte range [e0, e1)
 // of the buffer at `base`; b <= a when the range holds no aligned 16-B block.
 __device__ __forceinline__ void aligned_interior(uint64_t base, int64_t e0, int64_t e1, int64_t& a, int64_t& b) {
@@ -109,13 +146,20 @@ struct SegCache {
 };
 
 __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int nsegs, uint32_t total,
-                                          unsigned long long* __restrict__ busy) {
+                                          unsigned long long* __restrict__ busy, uint32_t* __restrict__ scratch) {
     extern __shared__ __align__(128) uint8_t hsm[];
     uint8_t* ring = hsm;                                                         // [stages][tile]
     uint32_t* h = reinterpret_cast<uint32_t*>(hsm + kHistStages * kHistTile);     // [256][32]
     uint64_t* full = reinterpret_cast<uint64_t*>(h + kHistBins * 32);
     uint64_t* empty = full + kHistStages;
+    __shared__ uint32_t last_flag;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    uint32_t* arrive = scratch ? scratch + (size_t)nsegs * kHistBins : nullptr;
+    if (scratch) {
+        // single-launch form: VPs without input still get their counts overwritten with 0
+        for (int si = blockIdx.x; si < nsegs; si += gridDim.x)
+            if (segs[si].n == 0 && threadIdx.x < kHistBins) reinterpret_cast<uint32_t*>(segs[si].ptr[1])[threadIdx.x] = 0u;
+    }
 
     for (int i = threadIdx.x; i < kHistBins * 32; i += kHistBlock) h[i] = 0;
     if (threadIdx.x == 0) {
@@ -175,7 +219,13 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
         const int si = sc.get(segs, nsegs, total, t);
         const SegDesc& sd = segs[si];
         if (si != cur) {
-            if (cur >= 0) hist_flush(h, cur_counts);
+            if (cur >= 0) {
+                if (scratch)
+                    hist_flush_fused(h, cur_counts, scratch + (size_t)cur * kHistBins, arrive + cur,
+                                     hist_expected_ctas(segs, nsegs, total, per, cur), &last_flag);
+                else
+                    hist_flush(h, cur_counts);
+            }
             cur = si;
             cur_counts = reinterpret_cast<uint32_t*>(sd.ptr[1]);
         }
@@ -237,17 +287,24 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
         }
         if (busy && threadIdx.x == 0) atomicAdd(busy + si, (unsigned long long)(clock64() - c0));
     }
-    if (cur >= 0) hist_flush(h, cur_counts);
+    if (cur >= 0) {
+        if (scratch)
+            hist_flush_fused(h, cur_counts, scratch + (size_t)cur * kHistBins, arrive + cur,
+                             hist_expected_ctas(segs, nsegs, total, per, cur), &last_flag);
+        else
+            hist_flush(h, cur_counts);
+    }
 }
 
 __global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total,
-                                                        unsigned long long* busy) {
-    hist_body(segs, nsegs, total, busy);
+                                                        unsigned long long* busy, uint32_t* scratch) {
+    hist_body(segs, nsegs, total, busy, scratch);
 }
 template <int CAP>
 __global__ void __launch_bounds__(kHistBlock) k_hist256_p(const __grid_constant__ SegParamT<CAP> p, int nsegs,
-                                                          uint32_t total, unsigned long long* busy) {
-    hist_body(p.s, nsegs, total, busy);
+                                                          uint32_t total, unsigned long long* busy,
+                                                          uint32_t* scratch) {
+    hist_body(p.s, nsegs, total, busy, scratch);
 }
 
 template <int CAP>
@@ -275,36 +332,45 @@ static cudaError_t hist_attr() {
     return cudaSuccess;
 }
 
-cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy) {
+cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy,
+                           uint32_t* scratch) {
     if (nsegs <= 0) return cudaSuccess;
-    k_hist_zero<<<nsegs < 1024 ? nsegs : 1024, 256, 0, s>>>(segs, nsegs);
-    cudaError_t e = cudaGetLastError();
-    if (e || total == 0) return e;
+    cudaError_t e;
+    if (!scratch) {
+        k_hist_zero<<<nsegs < 1024 ? nsegs : 1024, 256, 0, s>>>(segs, nsegs);
+        e = cudaGetLastError();
+        if (e || total == 0) return e;
+    }
     if ((e = hist_attr())) return e;
-    k_hist256<<<grid, kHistBlock, kHistSmem, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
+    k_hist256<<<grid, kHistBlock, kHistSmem, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy),
+                                                  scratch);
     return cudaGetLastError();
 }
 
 template <int CAP>
 static cudaError_t launch_hist256_param_cap(const SegDesc* segs, int nsegs, uint32_t total, int grid,
-                                            cudaStream_t s, uint64_t* busy) {
+                                            cudaStream_t s, uint64_t* busy, uint32_t* scratch) {
     SegParamT<CAP> p;
     memcpy(p.s, segs, (size_t)nsegs * sizeof(SegDesc));
-    k_hist_zero_p<CAP><<<nsegs, 256, 0, s>>>(p, nsegs);
-    cudaError_t e = cudaGetLastError();
-    if (e || total == 0) return e;
+    cudaError_t e;
+    if (!scratch) {
+        k_hist_zero_p<CAP><<<nsegs, 256, 0, s>>>(p, nsegs);
+        e = cudaGetLastError();
+        if (e || total == 0) return e;
+    }
     if ((e = hist_attr_p<CAP>())) return e;
-    k_hist256_p<CAP><<<grid, kHistBlock, kHistSmem, s>>>(p, nsegs, total, reinterpret_cast<unsigned long long*>(busy));
+    k_hist256_p<CAP><<<grid, kHistBlock, kHistSmem, s>>>(p, nsegs, total, reinterpret_cast<unsigned long long*>(busy),
+                                                         scratch);
     return cudaGetLastError();
 }
 
 cudaError_t launch_hist256_param(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s,
-                                 uint64_t* busy) {
+                                 uint64_t* busy, uint32_t* scratch) {
     if (nsegs <= 0) return cudaSuccess;
     if (param_full_block() && nsegs <= kParamSegs)
-        return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s, busy);
-    if (nsegs <= 16) return launch_hist256_param_cap<16>(segs, nsegs, total, grid, s, busy);
-    if (nsegs <= kParamSegs) return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s, busy);
+        return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s, busy, scratch);
+    if (nsegs <= 16) return launch_hist256_param_cap<16>(segs, nsegs, total, grid, s, busy, scratch);
+    if (nsegs <= kParamSegs) return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s, busy, scratch);
     return cudaErrorInvalidValue;
 }
 

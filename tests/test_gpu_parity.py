@@ -287,7 +287,7 @@ def test_hist256_ragged_tiles_every_alignment(table_mode):
     ctx = svp.Context(num_gpus=1, table_mode=table_mode)
     kh = ctx.register_kernel("hist256")
     T = 16384
-    sizes = [1, 15, 16, 17, 31, 32, 33, 47, 100, T - 1, T, T + 1, T + 15, 2 * T + 7, 3 * T - 5, 5 * T + 333]
+    sizes = [0, 1, 15, 16, 17, 31, 32, 33, 47, 100, T - 1, T, T + 1, T + 15, 2 * T + 7, 3 * T - 5, 5 * T + 333]
     g = np.random.default_rng(1234)
     jobs, host, bufs, counts = [], [], [], []
     vp = 0
@@ -320,6 +320,22 @@ def test_hist256_ragged_tiles_every_alignment(table_mode):
             assert np.array_equal(got, want), (v, len(d))
     finally:
         ctx.close()
+
+
+def test_hist256_single_launch_in_subprocess():
+    """SVP_HIST_FUSED=1 (hist256 as one launch: per-launch self-resetting scratch, the last
+    CTA of each VP writes its counts) is chosen once per process: run the hist parity
+    tests (alignment sweep incl. empty VPs, ragged full-size cfg4, mixed small, repeated
+    flushes) in a child process with the switch set."""
+    import os
+    import subprocess
+    import sys
+    here = os.path.dirname(os.path.abspath(__file__))
+    cmd = [sys.executable, "-m", "pytest", os.path.join(here, "test_gpu_parity.py"), "-q", "-m", "gpu",
+           "-p", "no:cacheprovider", "-k",
+           "(hist256_ragged or config4 or mixed_small or repeated_flushes or config5) and not subprocess"]
+    r = subprocess.run(cmd, env={**os.environ, "SVP_HIST_FUSED": "1"}, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
 
 
 def test_repeated_flushes_reuse_tables(small):
