@@ -124,7 +124,9 @@ class Clocks:
     the nearest samples around the window are added and `in_window` says how many were
     strictly inside."""
 
-    Q = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+    # power.draw.instant: plain power.draw is a 1-s average on Ampere and newer, which
+    # mostly shows the idle time before a ~0.1-s timed region
+    Q = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw.instant,clocks_event_reasons.active,"
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
@@ -200,7 +202,8 @@ class Clocks:
         pws = [r[4] for r in sel if r[4] == r[4]]
         return {"sm_mhz": statistics.median(r[1] for r in sel), "sm_max_mhz": max(r[2] for r in sel),
                 "samples": len(sel), "in_window": len(inside), "window_ms": (self.t1 - self.t0) * 1e3,
-                "reasons": sorted(reasons), "power_w": statistics.median(pws) if pws else None}
+                "reasons": sorted(reasons), "power_w": statistics.median(pws) if pws else None,
+                "power_field": "power.draw.instant (median of the samples)"}
 
 
 def measured_peaks():
