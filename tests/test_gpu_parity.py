@@ -210,6 +210,7 @@ def test_dynamic_tile_order_repeated(hetero):
                 for name in ("call", "put", "c"):
                     if name in vs.bufs[i]:
                         vs.bufs[i][name].fill_(float("nan"))
+            torch.cuda.synchronize()  # the fills run on torch's stream, the flush on libsvp's
             ctx.submit_batch(jb)
             ctx.flush()
             torch.cuda.synchronize()
@@ -260,6 +261,7 @@ def test_residency_validation_ranges(level):
     a = torch.rand(n, device="cuda")
     b = torch.rand(n, device="cuda")
     c = torch.empty(n, device="cuda")
+    torch.cuda.synchronize()  # filled on torch's stream; libsvp runs on its own streams
     for _ in range(2):  # the second pass hits the remembered ranges (level 1)
         ctx.submit(0, va, svp.args_vecadd(n), [(a.data_ptr(), 4 * n, 1, 0), (b.data_ptr(), 4 * n, 1, 0),
                                                (c.data_ptr(), 4 * n, 2, 0)])
@@ -310,6 +312,7 @@ def test_hist256_ragged_tiles_every_alignment(table_mode):
             counts.append(cnt)
             vp += 1
     try:
+        torch.cuda.synchronize()  # buffers were filled on torch's stream; libsvp uses its own
         ctx.submit_batch(jobs)
         ctx.flush()
         torch.cuda.synchronize()
