@@ -143,15 +143,39 @@ def s3_interleaving(quick):
 
 
 def s4_vps(quick):
+    """BJ metric vs #VPs at G = 1: jobs/s of the cfg5 prefix with nv VPs (all kernels), and
+    HBM GB/s of its memory-bound VPs flushed on their own (algorithmic bytes / device span
+    of the flush, profile_level 1 events)."""
     rows = []
     for nv in ([16, 64, 256] if quick else [2, 4, 8, 16, 32, 64, 128, 256]):
         specs = W.config_specs(5, nvps=nv)
         c = ctx_for()
         vs = VPSet(c, specs, W.make_inputs_many(specs), "device")
         t = flush_time(c, vs.job_list(), reps=5)
-        rows.append({"vps": nv, "ms": t * 1e3, "jobs_per_s": nv / t})
+        row = {"vps": nv, "ms": t * 1e3, "jobs_per_s": nv / t}
         c.close()
         del vs
+        mem = [s for s in specs if s.kernel in W.MEMBOUND]
+        if mem:
+            c = ctx_for(profile_level=1)
+            vs = VPSet(c, mem, W.make_inputs_many(mem), "device")
+            jobs = vs.job_list()
+            flush_time(c, jobs, reps=3)
+            dev = []
+            for _ in range(5):
+                c.submit_batch(svp.JobBatch(jobs))
+                c.flush()
+                dev.append(c.flush_stats()["device_ns"])
+            # algorithmic bytes (DESIGN.md §6): 12 B/elem vecadd, SAXPY; 20 B/option BS;
+            # 1 B/byte + the 1-KiB counts for hist256
+            nbytes = sum(12 * s.n if s.kernel in ("vecadd", "saxpy") else 20 * s.n if s.kernel == "blackscholes"
+                         else s.n + (1024 if s.n else 0) for s in mem)
+            row["membound_vps"] = len(mem)
+            row["membound_device_ms"] = statistics.median(dev) / 1e6
+            row["membound_hbm_gbs"] = nbytes / (statistics.median(dev) * 1e-9) / 1e9
+            c.close()
+            del vs
+        rows.append(row)
         torch.cuda.empty_cache()
     return rows
 
