@@ -214,6 +214,13 @@ void executor_unregister_host(Executor* e, void* p) {
     cudaSetDevice(e->devs[0].ordinal);
     cudaHostUnregister(p);
     cudaGetLastError();
+    // forget the remembered range (validate_ptrs 1): it is no longer page-locked
+    std::lock_guard<std::mutex> lk(e->rmu);
+    auto it = e->ranges.upper_bound((uintptr_t)p);
+    if (it != e->ranges.begin()) {
+        --it;
+        if ((uintptr_t)p < it->second.end) e->ranges.erase(it);
+    }
 }
 
 // Allocation range of p through the driver (CU_POINTER_ATTRIBUTE_RANGE_START_ADDR / _SIZE);
@@ -617,8 +624,14 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
     }
     auto t_issue0 = std::chrono::steady_clock::now();
     if (d.ext) {
+        // only the streams this flush uses on this GPU (and stream 0: table upload, capture)
+        std::vector<char> touch(d.streams.size(), 0);
+        touch[0] = 1;
+        for (const auto& o : f.ops)
+            if (o.device == d.idx) touch[o.stream] = 1;
         CK(cudaEventRecord(d.ext_ev, d.ext));
-        for (auto s : d.streams) CK(cudaStreamWaitEvent(s, d.ext_ev, 0));
+        for (size_t s = 0; s < d.streams.size(); ++s)
+            if (touch[s]) CK(cudaStreamWaitEvent(d.streams[s], d.ext_ev, 0));
     }
     // tables changed -> new host copy; the device copy is refreshed only if some launch on
     // this GPU reads the global table (param-mode launches carry theirs by value)
