@@ -1,7 +1,9 @@
 """Full-size cfg5 soak: the bench's launch configuration (plus the hetero / graph / table
 options) flushed for several steps, every memory-bound VP checked against the oracle after
 every step (SAXPY chained on its previous output), every SGEMM VP on 8 sampled elements.
-argv: steps, then option sets as hetero:graph:table (e.g. 0:0:1 1:1:1 0:1:0).  GPU tool."""
+argv: steps, then option sets as hetero:graph:table[:interleave] (e.g. 0:0:1 1:1:1 0:1:0:0;
+interleave 0 = one stream, where Black-Scholes / mixed launches take the dynamic tile
+order).  GPU tool."""
 import sys
 
 import numpy as np
@@ -16,15 +18,15 @@ from paper_conf_dac_jungc15_b200 import svp  # noqa: E402
 from paper_conf_dac_jungc15_b200.vpset import VPSet  # noqa: E402
 
 steps = int(sys.argv[1])
-combos = [tuple(int(x) for x in c.split(":")) for c in sys.argv[2:]] or [(0, 0, 1)]
+combos = [tuple(int(x) for x in (c + ":1").split(":")[:4]) for c in sys.argv[2:]] or [(0, 0, 1, 1)]
 specs = W.config_specs(5)
 inputs = W.make_inputs_many(specs)
 mb = [i for i, s in enumerate(specs) if s.kernel != "sgemm"]
 g = np.random.default_rng(11)
 stream = torch.cuda.current_stream()
-for hetero, graph, table in combos:
+for hetero, graph, table, inter in combos:
     ctx = svp.Context(num_gpus=1, device_ids=[0], profile_level=1, external_streams=[stream.cuda_stream],
-                      hetero=bool(hetero), graph=bool(graph), table_mode=table)
+                      hetero=bool(hetero), graph=bool(graph), table_mode=table, interleave=bool(inter))
     vs = VPSet(ctx, specs, inputs, "device", device_ordinals=[0])
     jobs = svp.JobBatch(vs.job_list())
     prev = [dict(inp) for inp in inputs]
@@ -52,7 +54,7 @@ for hetero, graph, table in combos:
                     bad += 1
                     print(f"combo {hetero}:{graph}:{table} step {step} vp {s.vp} sgemm: {e}", flush=True)
     st = ctx.flush_stats()
-    print(f"combo hetero={hetero} graph={graph} table={table}: {bad} bad over {steps} steps; "
+    print(f"combo hetero={hetero} graph={graph} table={table} interleave={inter}: {bad} bad over {steps} steps; "
           f"graph_replays {st['graph_replays']} guards {vs.guards_intact()}", flush=True)
     ctx.close()
     del vs
