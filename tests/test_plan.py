@@ -109,6 +109,26 @@ def test_program_order_levels_and_dependencies():
                     assert b["sim_start_ns"] >= a["sim_end_ns"] - 1e-6
 
 
+def test_sparse_vp_ids_plan_like_compact_ids():
+    """The planner keeps per-VP state in a flat array for compact VP ids and in a hash map
+    for sparse ones (ids up to 2^20): both must give the same plan for the same program."""
+    def plan_for(ids):
+        with svp.Context(dry_run=True) as c:
+            for rep in range(2):
+                for k, vp in enumerate(ids):
+                    submit(c, vp, MIX[(k + rep) % 4], n=5000 + 100 * k, mem=svp.MEM_HOST_PINNED)
+            c.flush()
+            inv = {v: i for i, v in enumerate(ids)}
+            return [(op["kind"], op["level"], op["kernel"], sorted(inv[v] for v in op["vps"]), op["stream"],
+                     round(op["sim_start_ns"], 3)) for op in c.plan()], c.flush_stats()["levels"]
+    sparse = [5, (1 << 20) - 1, 300000, 77, 123456, 999999]
+    compact = [0, 5, 3, 1, 2, 4]  # the ranks of the sparse ids (same relative order)
+    ps, ls = plan_for(sparse)
+    pc, lc = plan_for(compact)
+    assert ls == lc == 2
+    assert ps == pc
+
+
 def _host_cfg_plan(c, nvps=32, n=1 << 20):
     for vp in range(nvps):
         submit(c, vp, MIX[vp % 4], n=n + 4096 * vp, mem=svp.MEM_HOST_PINNED)
