@@ -34,7 +34,7 @@
 extern "C" {
 #endif
 
-#define SVP_ABI_VERSION 3
+#define SVP_ABI_VERSION 4
 
 typedef int32_t svp_status;
 enum {
@@ -321,6 +321,9 @@ typedef struct svp_flush_stats {
     double sim_serial_ns;    /* cost-model time of the same ops run one at a time  */
     uint64_t plan_reused;    /* cfg.graph: 1 if the previous flush's plan was reused */
     uint64_t graph_replays;  /* cfg.graph: GPUs whose work ran as a replayed CUDA graph */
+    uint64_t kernel_launches; /* kernels actually launched (`launches` counts coalesced
+                                 launch ops; hist256's zeroing kernel and the SGEMM tail
+                                 split's slice launch + reduction add to this one)     */
 } svp_flush_stats;
 svp_status svp_flush_stats_get(svp_ctx* ctx, svp_flush_stats* out);
 

@@ -354,7 +354,11 @@ static svp_status do_flush(Ctx* c) {
         c->fstats.levels = f.levels;
         uint64_t launches = 0;
         for (auto& op : f.ops) {
-            if (op.kind == SVP_OP_KERNEL) ++launches;
+            if (op.kind == SVP_OP_KERNEL) {
+                ++launches;
+                if (executor_chunk_launches(f, f.chunks[op.chunk]))
+                    c->fstats.kernel_launches += (uint64_t)f.chunks[op.chunk].kernel_launches;
+            }
             if (op.kind == SVP_OP_H2D) c->fstats.h2d_bytes += op.bytes;
             if (op.kind == SVP_OP_D2H) c->fstats.d2h_bytes += op.bytes;
         }

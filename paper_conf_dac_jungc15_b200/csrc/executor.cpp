@@ -78,6 +78,8 @@ struct Dev {
     // single-launch hist256: per launch nsegs * 257 self-resetting u32 (partials + arrivals)
     uint32_t* hscr_dev = nullptr;
     size_t hscr_cap = 0;  // u32
+    // SGEMM tail split workspace (partial products), allocated once on first use
+    float* tail_ws = nullptr;
     uint8_t* tbl_host = nullptr;
     uint8_t* tbl_dev = nullptr;
     size_t tbl_cap = 0;
@@ -147,6 +149,7 @@ static void dev_teardown(Dev& d) {
     if (d.busy_dev) cudaFree(d.busy_dev);
     if (d.sched_dev) cudaFree(d.sched_dev);
     if (d.hscr_dev) cudaFree(d.hscr_dev);
+    if (d.tail_ws) cudaFree(d.tail_ws);
     if (d.tbl_dev) cudaFree(d.tbl_dev);
     if (d.tbl_host) cudaFreeHost(d.tbl_host);
 }
@@ -342,8 +345,145 @@ static void resolve_addresses(Dev& d, const Flush& f, Chunk& ch) {
     }
 }
 
+// SGEMM tail split (SVP_SGEMM_TAIL=0: off): see plan_sgemm_tail.
+static bool sgemm_tail_split() {
+    static const bool on = !(getenv("SVP_SGEMM_TAIL") && atoi(getenv("SVP_SGEMM_TAIL")) == 0);
+    return on;
+}
+constexpr size_t kTailWsFloats = (size_t)8 << 20;  // 32 MiB: up to 128 pieces of 256 x 256
+
+// Dynamic tile order for Black-Scholes / mixed launches (SVP_EW_DYN=0: static order).
+static bool ew_dynamic_order() {
+    static const bool on = !(getenv("SVP_EW_DYN") && atoi(getenv("SVP_EW_DYN")) == 0);
+    return on;
+}
+
+// SVP_HIST_FUSED=1: hist256 as ONE launch with a self-resetting per-launch scratch (the
+// last CTA of each VP writes its counts) instead of a zeroing kernel + the accumulating
+// launch.  Off by default: alone it was 2 us (4 %) faster per cfg5 hist launch, but the
+// interleaved cfg5 step measured ~1 % slower with it (profiles/r01/hist_fused/).
+static bool hist_single_launch() {
+    static const bool on = getenv("SVP_HIST_FUSED") && atoi(getenv("SVP_HIST_FUSED")) != 0;
+    return on;
+}
+
+// SGEMM tail split.  A wide (256 x 512 pair tile) launch over T tiles and P CTA pairs runs
+// floor(T / P) full waves and a last wave of R = T mod P tiles, during which P - R pairs
+// idle (cfg5: 1632 tiles, 74 pairs -> R = 4: ~110 us at 4/74 occupancy,
+// profiles/r01/sgemm_waves.jsonl).  When R <= P / 2, the main launch stops after the full
+// waves and the R tail tiles become 256 x 256 sub-tiles split along K into S slices
+// (sub-tiles x S <= P): one wave of the narrow pair kernel writes the partial products to
+// a workspace, and a reduction kernel sums them in a fixed order into C (alpha, beta).
+// Same per-product arithmetic; the K sum is regrouped into S fp32 partial sums.
+static svp_status plan_sgemm_tail(Executor* e, Dev& d, Flush& f, Chunk& ch, std::vector<uint8_t>& tbl, int P) {
+    ch.main_tiles = ch.total_tiles;
+    ch.tail_n = ch.tail_nred = 0;
+    const uint32_t T = ch.total_tiles;
+    if (!sgemm_tail_split() || !ch.wide || P < 2 || T < (uint32_t)P) return SVP_OK;
+    const uint32_t R = T % (uint32_t)P;
+    if (R == 0 || R > (uint32_t)P / 2) return SVP_OK;
+    constexpr int WM = 2 * kTf32BM, WN = 2 * kTf32BN, SN = kTf32BN;  // wide tile, sub-tile width
+    struct Sub {
+        size_t k;  // job index in the chunk
+        int m0, n0, rows, cols;
+    };
+    std::vector<Sub> subs;
+    const GemmDesc* gd = reinterpret_cast<const GemmDesc*>(tbl.data() + ch.table_off);
+    for (uint32_t t = T - R; t < T; ++t) {
+        size_t k = 0;
+        while (k + 1 < ch.jobs.size() && gd[k + 1].tile_begin <= t) ++k;
+        const Job& j = f.jobs[ch.jobs[k]];
+        const uint32_t lt = t - gd[k].tile_begin;
+        const int tm = (int)(lt / gd[k].tiles_n), tn = (int)(lt % gd[k].tiles_n);
+        const int m0 = tm * WM, rows = std::min(WM, j.M - m0);
+        for (int h = 0; h < WN / SN; ++h) {
+            const int n0 = tn * WN + h * SN;
+            if (n0 < j.N) subs.push_back(Sub{k, m0, n0, rows, std::min(SN, j.N - n0)});
+        }
+    }
+    int K = 0;
+    for (const auto& sb : subs) K = std::max(K, f.jobs[ch.jobs[sb.k]].K);
+    int S = std::min<int>(P / (int)subs.size(), K / 64);
+    if (S < 2) return SVP_OK;
+    size_t ws_need = 0;
+    for (const auto& sb : subs) ws_need += (size_t)S * sb.rows * sb.cols;
+    if (ws_need > kTailWsFloats) return SVP_OK;
+    if (!d.tail_ws) {
+        cudaError_t ce = cudaMalloc(&d.tail_ws, kTailWsFloats * sizeof(float));
+        if (ce != cudaSuccess) {
+            cudaGetLastError();
+            d.tail_ws = nullptr;
+            return SVP_OK;  // no workspace: run the plain last wave
+        }
+    }
+    // pieces: per sub-tile, S K-slices of Kp (multiple of the 16-k block) each
+    std::vector<GemmDesc> pd;
+    std::vector<uint8_t> pm;
+    std::vector<TailRed> rd;
+    size_t ws_off = 0;
+    for (const auto& sb : subs) {
+        const Job& j = f.jobs[ch.jobs[sb.k]];
+        const float* A = (const float*)ch.staged[sb.k * SVP_MAX_BUFS + 0];
+        const float* B = (const float*)ch.staged[sb.k * SVP_MAX_BUFS + 1];
+        float* Cp = (float*)ch.staged[sb.k * SVP_MAX_BUFS + 2];
+        const int Kp = ((j.K + S - 1) / S + kTf32BK - 1) / kTf32BK * kTf32BK;
+        const int Se = (j.K + Kp - 1) / Kp;  // slices this sub-tile really has (<= S)
+        const size_t plane = (size_t)sb.rows * sb.cols;
+        TailRed r;
+        memset(&r, 0, sizeof(r));
+        r.C = Cp + (size_t)sb.m0 * j.N + sb.n0;
+        r.ws = d.tail_ws + ws_off;
+        r.ldc = j.N;
+        r.rows = sb.rows;
+        r.cols = sb.cols;
+        r.S = Se;
+        r.alpha = j.f0;
+        r.beta = j.f1;
+        rd.push_back(r);
+        for (int s = 0; s < Se; ++s) {
+            const int k0 = s * Kp, kl = std::min(Kp, j.K - k0);
+            GemmDesc g;
+            memset(&g, 0, sizeof(g));
+            g.C = d.tail_ws + ws_off + (size_t)s * plane;
+            g.M = sb.rows;
+            g.N = sb.cols;
+            g.K = kl;
+            g.alpha = 1.f;
+            g.beta = 0.f;
+            g.tile_begin = (uint32_t)pd.size();
+            g.tiles_n = 1;
+            pd.push_back(g);
+            uint8_t m[256];
+            if (encode_gemm_maps_view(m, m + 128, A + (size_t)sb.m0 * j.K + k0, B + (size_t)k0 * j.N + sb.n0, sb.rows,
+                                      sb.cols, kl, j.K, j.N) != 0) {
+                d.err = "cuTensorMapEncodeTiled failed for an sgemm tail slice";
+                return SVP_E_CUDA;
+            }
+            pm.insert(pm.end(), m, m + 256);
+        }
+        ws_off += (size_t)Se * plane;
+    }
+    ch.tail_maps_off = align_up(tbl.size(), 128);
+    ch.tail_table_off = ch.tail_maps_off + pm.size();
+    ch.tail_red_off = align_up(ch.tail_table_off + pd.size() * sizeof(GemmDesc), 128);
+    tbl.resize(ch.tail_red_off + rd.size() * sizeof(TailRed));
+    memcpy(tbl.data() + ch.tail_maps_off, pm.data(), pm.size());
+    memcpy(tbl.data() + ch.tail_table_off, pd.data(), pd.size() * sizeof(GemmDesc));
+    memcpy(tbl.data() + ch.tail_red_off, rd.data(), rd.size() * sizeof(TailRed));
+    ch.main_tiles = T - R;
+    ch.tail_n = (int32_t)pd.size();
+    ch.tail_nred = (int32_t)rd.size();
+    ch.kernel_launches = 3;
+    (void)e;
+    return SVP_OK;
+}
+
 static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_t>& tbl) {
     tbl.clear();
+    // launches that share their level with other kernel launches on this GPU co-run with them
+    std::map<int32_t, int> chunks_in_level;
+    for (const auto& ch : f.chunks)
+        if (ch.device == d.idx) chunks_in_level[ch.level] += 1;
     for (auto& ch : f.chunks) {
         if (ch.device != d.idx) continue;
         resolve_addresses(d, f, ch);
@@ -417,6 +557,8 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             ch.total_tiles = tiles;
             ch.nsegs = (int32_t)ch.jobs.size();
             ch.param = e->c->cfg.table_mode == SVP_TABLE_PARAM && ch.nsegs <= kParamSegs;
+            // hist256: the zeroing kernel precedes the accumulating launch (unless single-launch)
+            ch.kernel_launches = ch.kernel == K_HIST256 && !hist_single_launch() && tiles > 0 ? 2 : 1;
         } else {
             // tcgen05 tiles for sgemm_tf32 and for sgemm with the 3xTF32 implementation
             const int variant = (ch.kernel == K_SGEMM_TF32 || e->c->cfg.sgemm_impl != SVP_SGEMM_FFMA) ? 1 : 0;
@@ -481,6 +623,19 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             }
             ch.total_tiles = tiles;
             ch.nsegs = (int32_t)nj;
+            ch.kernel_launches = 1;
+            ch.main_tiles = tiles;
+            ch.tail_n = ch.tail_nred = 0;
+            // tail split only for a launch that has the GPU to itself: co-running with the
+            // memory-bound launches of an interleaved level, the last wave's idle pairs are
+            // not idle GPU time, and the power-capped step measured 0.7-2 % slower with the
+            // extra slice pass (profiles/r01/sgemm_tail/)
+            const bool alone = !e->c->cfg.interleave || chunks_in_level[ch.level] == 1;
+            if (alone && ch.kernel == K_SGEMM && e->c->cfg.sgemm_impl == SVP_SGEMM_TF32BF16) {
+                const int P = (int)std::min<uint64_t>(tiles, (uint64_t)d.lim.num_sms / 2);
+                svp_status st = plan_sgemm_tail(e, d, f, ch, tbl, P);
+                if (st) return st;
+            }
         }
     }
     return SVP_OK;
@@ -495,21 +650,6 @@ static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bo
     }
     (void)d;
     return pool[i];
-}
-
-// Dynamic tile order for Black-Scholes / mixed launches (SVP_EW_DYN=0: static order).
-static bool ew_dynamic_order() {
-    static const bool on = !(getenv("SVP_EW_DYN") && atoi(getenv("SVP_EW_DYN")) == 0);
-    return on;
-}
-
-// SVP_HIST_FUSED=1: hist256 as ONE launch with a self-resetting per-launch scratch (the
-// last CTA of each VP writes its counts) instead of a zeroing kernel + the accumulating
-// launch.  Off by default: alone it was 2 us (4 %) faster per cfg5 hist launch, but the
-// interleaved cfg5 step measured ~1 % slower with it (profiles/r01/hist_fused/).
-static bool hist_single_launch() {
-    static const bool on = getenv("SVP_HIST_FUSED") && atoi(getenv("SVP_HIST_FUSED")) != 0;
-    return on;
 }
 
 static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStream_t s) {
@@ -558,9 +698,17 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
             return launch_hist256((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
                                   grid_of(d.lim.hist_blocks_per_sm), s, busy, hscr);
         case K_SGEMM:
-            if (sgemm_impl == SVP_SGEMM_TF32BF16)
-                return launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
-                                             ch.total_tiles, grid_of(1), ch.wide, s);
+            if (sgemm_impl == SVP_SGEMM_TF32BF16) {
+                cudaError_t e = launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.table_off), ch.nsegs,
+                                                      base + ch.maps_off, ch.main_tiles, grid_of(1), ch.wide, s);
+                if (e || ch.tail_n == 0) return e;
+                // tail split: the last wave's tiles as K-slices, then the ordered reduction
+                e = launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.tail_table_off), ch.tail_n,
+                                          base + ch.tail_maps_off, (uint32_t)ch.tail_n,
+                                          2 * std::min<int>(ch.tail_n, d.lim.num_sms / 2), false, s);
+                if (e) return e;
+                return launch_sgemm_tail_reduce((const TailRed*)(base + ch.tail_red_off), ch.tail_nred, s);
+            }
             if (sgemm_impl == SVP_SGEMM_3XTF32)
                 return launch_sgemm_3xtf32((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
                                            ch.total_tiles, grid_of(1), s);
@@ -588,6 +736,8 @@ static bool chunk_needs_launch(const Flush& f, const Chunk& ch) {
     }
     return false;
 }
+
+bool executor_chunk_launches(const Flush& f, const Chunk& ch) { return chunk_needs_launch(f, ch); }
 
 static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool capturing, std::vector<int>& used,
                             std::vector<int32_t>& tstart);

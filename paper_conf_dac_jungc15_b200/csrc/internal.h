@@ -106,6 +106,14 @@ struct Chunk {
     std::vector<uint64_t> busy;
     int32_t sched_slot = -1;        // dynamic tile order: counter slot of this launch (-1: static)
     int64_t hscr_off = -1;          // single-launch hist256: scratch offset (u32) of this launch
+    // SGEMM tail split (wide launches whose last wave is at most half full): the main launch
+    // runs main_tiles tiles, the last wave's tiles run as tail_n K-slices (narrow pair
+    // kernel) into a workspace, then tail_nred sub-tile reductions write C
+    uint32_t main_tiles = 0;
+    int32_t tail_n = 0, tail_nred = 0;
+    uint64_t tail_maps_off = 0, tail_table_off = 0, tail_red_off = 0;
+    // kernel launches this op issues (hist256 zeroing kernel, tail split: 3)
+    int32_t kernel_launches = 1;
 };
 
 struct Op {
@@ -248,6 +256,8 @@ std::string executor_error(Executor* e);
 // device (or managed) memory on the VP's GPU; HOST_PINNED -> page-locked host memory; and
 // the whole range inside ONE allocation.  validate_ptrs 1 remembers every allocation range
 // it has resolved (one driver query per allocation, not per submit); 2 queries every time.
+// true if the chunk's kernel op really launches (chunk_needs_launch)
+bool executor_chunk_launches(const Flush& f, const Chunk& ch);
 svp_status executor_check_ptr(Executor* e, const void* p, uint64_t bytes, int32_t mem, int32_t device,
                               std::string* why);
 

@@ -220,12 +220,14 @@ static PFN_encodeTiled get_encode() {
     return fn;
 }
 
+// pitch: row stride in elements (0 = inner, a dense matrix); a sub-matrix view passes the
+// parent's row length
 static int encode2d(void* out, const float* base, uint64_t inner, uint64_t outer, uint32_t box_inner,
-                    uint32_t box_outer, CUtensorMapSwizzle sw) {
+                    uint32_t box_outer, CUtensorMapSwizzle sw, uint64_t pitch = 0) {
     PFN_encodeTiled enc = get_encode();
     if (!enc) return -1;
     cuuint64_t dims[2] = {inner, outer};
-    cuuint64_t strides[1] = {inner * 4};
+    cuuint64_t strides[1] = {(pitch ? pitch : inner) * 4};
     cuuint32_t box[2] = {box_inner, box_outer};
     cuuint32_t estr[2] = {1, 1};
     CUresult r = enc(reinterpret_cast<CUtensorMap*>(out), CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)base, dims, strides,
@@ -248,6 +250,14 @@ int encode_gemm_maps(void* mapA, void* mapB, const float* A, const float* B, int
     int r = encode2d(mapA, A, (uint64_t)K, (uint64_t)M, kTf32BK, kTf32BM, CU_TENSOR_MAP_SWIZZLE_64B);
     if (r) return r;
     return encode2d(mapB, B, (uint64_t)N, (uint64_t)K, 32, kTf32BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B);
+}
+
+int encode_gemm_maps_view(void* mapA, void* mapB, const float* A, const float* B, int M, int N, int K, int lda,
+                          int ldb) {
+    // a sub-matrix view for the tcgen05 tiles: A (M x K, row stride lda), B (K x N, row stride ldb)
+    int r = encode2d(mapA, A, (uint64_t)K, (uint64_t)M, kTf32BK, kTf32BM, CU_TENSOR_MAP_SWIZZLE_64B, (uint64_t)lda);
+    if (r) return r;
+    return encode2d(mapB, B, (uint64_t)N, (uint64_t)K, 32, kTf32BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B, (uint64_t)ldb);
 }
 
 }  // namespace svp

@@ -769,6 +769,41 @@ cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps
     return tmem_a() ? launch_tc<4, 1>(descs, n, maps, total, grid, s) : launch_tc<2, 1>(descs, n, maps, total, grid, s);
 }
 
+// ------------------------------------------------------------------ tail split reduction
+// One CTA per 4 rows of a sub-tile: thread (r, c4) sums the S partial products of one
+// float4 in order s = 0..S-1, then C = alpha * sum (+ beta * C).
+__global__ void __launch_bounds__(256) k_sgemm_tail_reduce(const TailRed* __restrict__ reds) {
+    const TailRed& rd = reds[blockIdx.y];
+    const int row = blockIdx.x * 4 + (threadIdx.x >> 6), c = (threadIdx.x & 63) * 4;
+    if (row >= rd.rows || c >= rd.cols) return;
+    const size_t plane = (size_t)rd.rows * rd.cols;
+    const float* p = rd.ws + (size_t)row * rd.cols + c;
+    float4 acc = *reinterpret_cast<const float4*>(p);
+    for (int s = 1; s < rd.S; ++s) {
+        const float4 v = *reinterpret_cast<const float4*>(p + s * plane);
+        acc.x += v.x;
+        acc.y += v.y;
+        acc.z += v.z;
+        acc.w += v.w;
+    }
+    float4* dst = reinterpret_cast<float4*>(rd.C + (size_t)row * rd.ldc + c);
+    float4 o = make_float4(rd.alpha * acc.x, rd.alpha * acc.y, rd.alpha * acc.z, rd.alpha * acc.w);
+    if (rd.beta != 0.f) {
+        const float4 old = *dst;
+        o.x = __fmaf_rn(rd.beta, old.x, o.x);
+        o.y = __fmaf_rn(rd.beta, old.y, o.y);
+        o.z = __fmaf_rn(rd.beta, old.z, o.z);
+        o.w = __fmaf_rn(rd.beta, old.w, o.w);
+    }
+    *dst = o;
+}
+
+cudaError_t launch_sgemm_tail_reduce(const TailRed* reds, int nred, cudaStream_t s) {
+    if (nred <= 0) return cudaSuccess;
+    k_sgemm_tail_reduce<<<dim3((2 * kTf32BM) / 4, nred), 256, 0, s>>>(reds);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
                                 cudaStream_t s) {
     if (sgemm_tc_cta_pair())

@@ -85,5 +85,11 @@ cudaError_t query_limits_dgemm(int* per_sm, int* per_sm_small);
 // Returns 0 on success.
 int encode_gemm_maps(void* mapA, void* mapB, const float* A, const float* B, int M, int N, int K,
                      int variant);
+// tcgen05 maps of a sub-matrix view: A (M x K, row stride lda), B (K x N, row stride ldb).
+int encode_gemm_maps_view(void* mapA, void* mapB, const float* A, const float* B, int M, int N, int K, int lda,
+                          int ldb);
+// SGEMM tail split: C = alpha * (sum of the S partial products) + beta * C per sub-tile
+// (fixed summation order: deterministic).
+cudaError_t launch_sgemm_tail_reduce(const TailRed* reds, int nred, cudaStream_t s);
 
 }  // namespace svp

@@ -52,6 +52,20 @@ struct GemmDesc {
 };
 static_assert(sizeof(GemmDesc) == 64, "GemmDesc must be 64 B");
 
+// SGEMM tail split (the partial last wave of a wide launch, split along K): one entry per
+// 256 x 256 output sub-tile; its S partial products sit back to back in the workspace
+// (piece s at ws + s * rows * cols), the reduction writes C = alpha * sum_s + beta * C.
+struct TailRed {
+    float* C;          // first element of the sub-tile in C
+    const float* ws;   // first partial product
+    int32_t ldc;       // row stride of C (elements)
+    int32_t rows, cols;
+    int32_t S;         // partial products
+    float alpha, beta;
+    uint32_t _pad[6];
+};
+static_assert(sizeof(TailRed) == 64, "TailRed must be 64 B");
+
 // Grouped DGEMM (fp64): one entry per VP, plain pointers (no TMA).
 struct DgemmDesc {
     const double* A;

@@ -77,7 +77,7 @@ class svp_flush_stats(C.Structure):
                                           "d2h_bytes", "table_bytes", "table_uploads")] + \
                [(n, C.c_double) for n in ("host_plan_ns", "host_issue_ns", "host_total_ns", "device_ns",
                                           "sim_makespan_ns", "sim_serial_ns")] + \
-               [(n, C.c_uint64) for n in ("plan_reused", "graph_replays")]
+               [(n, C.c_uint64) for n in ("plan_reused", "graph_replays", "kernel_launches")]
 
 
 class svp_plan_op(C.Structure):

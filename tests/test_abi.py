@@ -23,7 +23,7 @@ def test_library_exports_every_declared_symbol():
     assert set(declared) == set(svp.EXPORTS), (set(declared) ^ set(svp.EXPORTS))
     for name in declared:
         assert hasattr(L, name), name
-    assert L.svp_abi_version() == 3
+    assert L.svp_abi_version() == 4
 
 
 def test_lib_is_the_in_tree_build():

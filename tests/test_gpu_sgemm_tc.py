@@ -118,3 +118,31 @@ def test_split_adversarial_constant_inputs(impl):
     outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl)
     for s, inp, got in zip(specs, inputs, outs):
         check_job(s, inp, got)
+
+
+@pytest.mark.parametrize("int_inputs", [True, False])
+def test_tail_split_last_wave(int_inputs):
+    """SGEMM tail split: 19 VPs of ~1024^3 = 152 wide pair tiles over 74 pairs leave a last
+    wave of 4 tiles; they run as 256 x 256 sub-tiles split along K (narrow pair kernel into
+    a workspace) plus an ordered reduction with alpha / beta.  The last VP is ragged
+    (partial row / column sub-tiles, K not a multiple of the 16-k block, beta != 0 with C
+    INOUT), so the tail covers every edge.  Integer inputs must stay bit-exact."""
+    specs = [W.JobSpec(v, "sgemm", M=1024, N=1024, K=1024, int_inputs=int_inputs) for v in range(18)]
+    specs.append(W.JobSpec(18, "sgemm", M=1000, N=1012, K=1000, alpha=1.5, beta=0.5, int_inputs=int_inputs))
+    inputs = inputs_for(specs)
+    ctx = svp.Context(num_gpus=1, sgemm_impl=svp.SGEMM_TF32BF16)
+    try:
+        from paper_conf_dac_jungc15_b200.vpset import VPSet
+        import torch
+        vs = VPSet(ctx, specs, inputs, "device")
+        vs.submit()
+        ctx.flush()
+        torch.cuda.synchronize()
+        st = ctx.flush_stats()
+        assert st["launches"] == 1 and st["kernel_launches"] == 3, st  # main + tail slices + reduction
+        outs = [vs.output(i) for i in range(len(specs))]
+        assert vs.guards_intact()
+    finally:
+        ctx.close()
+    for s, inp, got in zip(specs, inputs, outs):
+        check_job(s, inp, got)
