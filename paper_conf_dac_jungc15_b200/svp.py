@@ -14,7 +14,9 @@ import threading
 from typing import Dict, Iterable, List, Optional, Sequence, Tuple
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libsvp.so")
+# SVP_LIB: load another build of the same library (the host-sanitizer builds of
+# scripts/host_sanitizers.sh); it is then used as is, never rebuilt.
+LIB_PATH = os.environ.get("SVP_LIB") or os.path.join(_PKG, "libsvp.so")
 
 SVP_OK, SVP_E_INVAL, SVP_E_NOMEM, SVP_E_CUDA, SVP_E_NOKERNEL, SVP_E_STATE, SVP_E_TIMEOUT, SVP_E_UNSUPPORTED = (
     0, -1, -2, -3, -4, -5, -6, -7)
@@ -103,7 +105,7 @@ def load(build_if_stale: bool = True):
     with _lock:
         if _lib is not None:
             return _lib
-        if build_if_stale:
+        if build_if_stale and not os.environ.get("SVP_LIB"):
             try:
                 from . import _build
                 if os.path.exists(_build.NVCC):
