@@ -35,3 +35,4 @@ for san in asan tsan; do
   echo "$san rc=$?"; tail -2 "$OUT/host_$san.log"
   grep -c "ERROR: AddressSanitizer\|runtime error:\|WARNING: ThreadSanitizer" "$OUT/host_$san.log"
 done
+rm -rf "$ROOT/build/asan" "$ROOT/build/tsan"  # keep the gpurun snapshot small
