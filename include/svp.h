@@ -74,7 +74,8 @@ typedef struct svp_config {
                                     counts the SM clock cycles thread 0 of each CTA spends in
                                     each tile, per segment -- the launch's time is then split
                                     over its VPs by those measured cycles (GEMM launches keep
-                                    the FLOP split)                                           */
+                                    the FLOP split).  A latency-weighted split: a tile costs
+                                    what its loads waited when it ran                         */
     int32_t sync_each_job;       /* serial baseline B1: stream-synchronize after every job    */
     int32_t dry_run;             /* 1: plan only -- no CUDA call at all, op times simulated
                                     by the cost model (host-logic tests on CPU)               */

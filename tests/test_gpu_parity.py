@@ -221,6 +221,55 @@ def test_dynamic_tile_order_repeated(hetero):
         ctx.close()
 
 
+def test_profiler_split_vs_serial_per_vp_launches():
+    """SURVEY §4 T9, against an independent measurement: the event-timed duration of each
+    VP's OWN launch when the same jobs run uncoalesced (serial mode).  A standalone launch
+    is not proportional to the VP's bytes -- it pays the launch and a partly filled last
+    round of tiles, Eq 9's T_o + T_e * ceil(xi / lambda): 4 Mi elements took
+    ~18 us against ~7 us of bandwidth -- which is exactly what coalescing amortises.  So the
+    checks are: serial times rise with the VP's size; the coalesced launch takes less than
+    the VP's serial launches together; and the level-1 shares (bytes) rank the VPs as their
+    serial launches do, each within a factor 2 of the serial share.  The level-2 split
+    (thread 0's cycles per tile) is only checked for conservation here: it weighs a tile by
+    its latency when it ran, which depends on what else was in flight."""
+    sizes = np.array([1 << 22, 2 << 22, 3 << 22, 4 << 22, 6 << 22])
+    kinds = ("vecadd", "saxpy")
+    nv = len(sizes)
+    specs = [W.JobSpec(v, kinds[v // nv], n=int(sizes[v % nv]), a=1.25) for v in range(2 * nv)]
+    inputs = inputs_for(specs)
+    reps = 5
+
+    def per_vp(**cfg):
+        ctx = svp.Context(num_gpus=1, **cfg)
+        try:
+            vs = VPSet(ctx, specs, inputs, "device")
+            jb = svp.JobBatch(vs.job_list())
+            ctx.submit_batch(jb)
+            ctx.flush()
+            ctx.reset_profile()
+            for _ in range(reps):
+                ctx.submit_batch(jb)
+                ctx.flush()
+            torch.cuda.synchronize()
+            return np.array([ctx.profile(sp.vp)["kernel_ns"] for sp in specs]) / reps
+        finally:
+            ctx.close()
+
+    serial = per_vp(coalesce=False, interleave=False, profile_level=1)
+    # one stream, so each coalesced launch's event-timed duration is its own
+    coal = {level: per_vp(profile_level=level, interleave=False) for level in (1, 2)}
+    for lo in (0, nv):  # per kernel class (one coalesced launch each)
+        t = serial[lo:lo + nv]
+        assert np.all(np.diff(t) > 0), (kinds[lo // nv], t)
+        c = coal[1][lo:lo + nv]
+        assert c.sum() < t.sum(), (kinds[lo // nv], c.sum(), t.sum())  # coalescing gain
+        assert np.all(np.diff(c) > 0), (kinds[lo // nv], c)              # same ranking
+        a, b = t / t.sum(), c / c.sum()
+        assert np.all((b / a > 0.5) & (b / a < 2.0)), (kinds[lo // nv], a, b)
+        # level 2: same launch time, split differently (conservation within timing noise)
+        assert coal[2][lo:lo + nv].sum() == pytest.approx(c.sum(), rel=0.25)
+
+
 def test_external_stream_join(small):
     specs, inputs = small
     s = torch.cuda.Stream()
