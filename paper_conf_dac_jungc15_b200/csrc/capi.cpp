@@ -205,6 +205,7 @@ static svp_status submit_many(Ctx* c, int32_t n, const svp_job_desc* jd, const s
                               uint64_t* ids) {
     (void)single_args_src;
     std::vector<Job> jobs(n);
+    RangeBatchLock batch(c->exec);  // one lock of the validation cache for the whole batch
     for (int i = 0; i < n; ++i) {
         Job& j = jobs[i];
         j.vp = jd[i].vp;

@@ -110,7 +110,30 @@ struct Executor {
     std::string err;
     std::mutex rmu;                          // submits validate from many threads
     std::map<uintptr_t, PtrRange> ranges;    // allocation start -> range (validate_ptrs 1)
+    // direct-mapped front of `ranges` by 2-MiB page (hits skip the tree walk)
+    struct Hot {
+        uintptr_t start = 0, end = 0;
+        PtrRange r;
+    };
+    Hot hot[256];
 };
+
+// the calling thread holds e->rmu through a RangeBatchLock
+static thread_local Executor* t_range_locked = nullptr;
+
+RangeBatchLock::RangeBatchLock(Executor* ex) {
+    if (ex && ex->c->cfg.validate_ptrs == 1) {
+        ex->rmu.lock();
+        e = ex;
+        t_range_locked = ex;
+    }
+}
+RangeBatchLock::~RangeBatchLock() {
+    if (e) {
+        t_range_locked = nullptr;
+        e->rmu.unlock();
+    }
+}
 
 std::string executor_error(Executor* e) { return e->err; }
 
@@ -224,6 +247,7 @@ void executor_unregister_host(Executor* e, void* p) {
         --it;
         if ((uintptr_t)p < it->second.end) e->ranges.erase(it);
     }
+    for (auto& h : e->hot) h = Executor::Hot();
 }
 
 // Allocation range of p through the driver (CU_POINTER_ATTRIBUTE_RANGE_START_ADDR / _SIZE);
@@ -255,14 +279,25 @@ svp_status executor_check_ptr(Executor* e, const void* p, uint64_t bytes, int32_
     const bool cached = e->c->cfg.validate_ptrs == 1;
     PtrRange r;
     bool hit = false, known = false;
+    // a RangeBatchLock of this thread already holds the lock
+    std::unique_lock<std::mutex> lk(e->rmu, std::defer_lock);
+    if (cached && t_range_locked != e) lk.lock();
+    Executor::Hot& hot = e->hot[(a >> 21) & 255];
     if (cached) {
-        std::lock_guard<std::mutex> lk(e->rmu);
-        auto it = e->ranges.upper_bound(a);
-        if (it != e->ranges.begin()) {
-            --it;
-            if (a < it->second.end) {
-                r = it->second;
-                hit = known = true;
+        if (hot.start <= a && a < hot.end) {
+            r = hot.r;
+            hit = known = true;
+        } else {
+            auto it = e->ranges.upper_bound(a);
+            if (it != e->ranges.begin()) {
+                --it;
+                if (a < it->second.end) {
+                    r = it->second;
+                    hit = known = true;
+                    hot.start = it->first;
+                    hot.end = it->second.end;
+                    hot.r = it->second;
+                }
             }
         }
     }
@@ -281,8 +316,10 @@ svp_status executor_check_ptr(Executor* e, const void* p, uint64_t bytes, int32_
             r.end = en;
             known = true;
             if (cached) {
-                std::lock_guard<std::mutex> lk(e->rmu);
-                e->ranges[st] = r;
+                e->ranges[st] = r;  // under lk or the batch lock
+                hot.start = st;
+                hot.end = en;
+                hot.r = r;
             }
         }
     }

@@ -258,6 +258,13 @@ std::string executor_error(Executor* e);
 // it has resolved (one driver query per allocation, not per submit); 2 queries every time.
 // true if the chunk's kernel op really launches (chunk_needs_launch)
 bool executor_chunk_launches(const Flush& f, const Chunk& ch);
+// A batch of submits validates under one acquisition of the range cache's lock (the
+// guard is a no-op without an executor or with validate_ptrs != 1).
+struct RangeBatchLock {
+    Executor* e = nullptr;
+    explicit RangeBatchLock(Executor* ex);
+    ~RangeBatchLock();
+};
 svp_status executor_check_ptr(Executor* e, const void* p, uint64_t bytes, int32_t mem, int32_t device,
                               std::string* why);
 
