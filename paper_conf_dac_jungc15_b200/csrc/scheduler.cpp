@@ -18,6 +18,7 @@
 //    D2H, a pool of compute streams -- the paper's Copy/Compute engines), and adds
 //    the event dependencies that keep every VP's program order.
 #include <math.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -493,6 +494,11 @@ svp_status plan_flush(Ctx* c, Flush* f) {
     std::vector<std::vector<Slot>> inflight(c->ngpu);
     std::vector<uint64_t> arena_head(c->ngpu, 0);
     std::vector<int32_t> rr(c->ngpu, 0);
+    // compute stream of a chunk: the one with the least estimated kernel time queued so far
+    // (list scheduling; ties -> lowest index).  Round-robin put cfg5's 5th launch (hist256)
+    // behind the SGEMM on stream 0, so it ran alone after it.  SVP_STREAM_RR=1: round-robin.
+    static const bool stream_rr = getenv("SVP_STREAM_RR") && atoi(getenv("SVP_STREAM_RR")) != 0;
+    std::vector<std::vector<double>> sload(c->ngpu, std::vector<double>(S, 0.0));
     for (int32_t ci : corder) {
         Chunk& ch = f->chunks[ci];
         const int dev = ch.device;
@@ -519,7 +525,16 @@ svp_status plan_flush(Ctx* c, Flush* f) {
             ch.arena_off = off;
             arena_head[dev] = off + ch.arena_len;
         }
-        int cs = inter ? (rr[dev]++ % S) : 0;
+        int cs = 0;
+        if (inter) {
+            if (stream_rr) {
+                cs = rr[dev]++ % S;
+            } else {
+                for (int k = 1; k < S; ++k)
+                    if (sload[dev][k] < sload[dev][cs]) cs = k;
+                sload[dev][cs] += std::max(ch.t_k, 1.0);
+            }
+        }
         int sh2d = inter ? S : 0, sd2h = inter ? S + 1 : 0;
         int32_t first_op = (int32_t)f->ops.size();
         int32_t k_op = -1, last = -1;
