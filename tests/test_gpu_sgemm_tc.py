@@ -120,21 +120,24 @@ def test_split_adversarial_constant_inputs(impl):
         check_job(s, inp, got)
 
 
+@pytest.mark.parametrize("residency,interleave", [("device", True), ("host", False)])
 @pytest.mark.parametrize("int_inputs", [True, False])
-def test_tail_split_last_wave(int_inputs):
+def test_tail_split_last_wave(int_inputs, residency, interleave):
     """SGEMM tail split: 19 VPs of ~1024^3 = 152 wide pair tiles over 74 pairs leave a last
     wave of 4 tiles; they run as 256 x 256 sub-tiles split along K (narrow pair kernel into
     a workspace) plus an ordered reduction with alpha / beta.  The last VP is ragged
     (partial row / column sub-tiles, K not a multiple of the 16-k block, beta != 0 with C
-    INOUT), so the tail covers every edge.  Integer inputs must stay bit-exact."""
+    INOUT), so the tail covers every edge.  Integer inputs must stay bit-exact.  Host-
+    resident on one stream (one chunk, so the launch is alone): the slices read the
+    staging arena."""
     specs = [W.JobSpec(v, "sgemm", M=1024, N=1024, K=1024, int_inputs=int_inputs) for v in range(18)]
     specs.append(W.JobSpec(18, "sgemm", M=1000, N=1012, K=1000, alpha=1.5, beta=0.5, int_inputs=int_inputs))
     inputs = inputs_for(specs)
-    ctx = svp.Context(num_gpus=1, sgemm_impl=svp.SGEMM_TF32BF16)
+    ctx = svp.Context(num_gpus=1, sgemm_impl=svp.SGEMM_TF32BF16, interleave=interleave, arena_bytes=1 << 31)
     try:
         from paper_conf_dac_jungc15_b200.vpset import VPSet
         import torch
-        vs = VPSet(ctx, specs, inputs, "device")
+        vs = VPSet(ctx, specs, inputs, residency)
         vs.submit()
         ctx.flush()
         torch.cuda.synchronize()
