@@ -210,3 +210,48 @@ def test_dgemm_identity_and_near_exact():
     for (i, j) in [(0, 0), (39, 49), (7, 21)]:
         exact = sum(Fraction(float(A[i, k])) * Fraction(float(B[k, j])) for k in range(33))
         assert abs(Fraction(float(C[i, j])) - exact) <= Fraction(np.spacing(abs(float(exact)))), (i, j)
+
+
+# ------------------------------------------------------------------ property tests
+from hypothesis import given, settings  # noqa: E402
+from hypothesis import strategies as st  # noqa: E402
+
+
+@settings(max_examples=60, deadline=None)
+@given(M=st.integers(0, 9), N=st.integers(0, 9), K=st.integers(0, 9), seed=st.integers(0, 2**31 - 1),
+       alpha=st.sampled_from([1.0, -2.0, 0.5]), beta=st.sampled_from([0.0, 1.0, -0.25]))
+def test_sgemm_random_tiny_shapes_exact(M, N, K, seed, alpha, beta):
+    """Random tiny shapes (incl. empty), integer operands in [-8, 8]: the oracle's SGEMM equals
+    alpha * (int64 matmul) + beta * C exactly (every intermediate is a small dyadic)."""
+    g = np.random.default_rng(seed)
+    A = g.integers(-8, 9, size=(M, K)).astype(np.float32)
+    B = g.integers(-8, 9, size=(K, N)).astype(np.float32)
+    C = g.integers(-8, 9, size=(M, N)).astype(np.float32)
+    want = alpha * (A.astype(np.int64) @ B.astype(np.int64)).astype(np.float64) + beta * C.astype(np.float64)
+    got = oracle.sgemm(A, B, C.copy(), alpha, beta)
+    assert got.shape == (M, N)
+    assert np.array_equal(got.astype(np.float64), want)
+
+
+@settings(max_examples=60, deadline=None)
+@given(data=st.binary(min_size=0, max_size=600))
+def test_hist_random_bytes_brute_force(data):
+    """Arbitrary byte strings (incl. empty): counts equal a pure-Python tally and sum to n."""
+    d = np.frombuffer(data, dtype=np.uint8)
+    want = [0] * 256
+    for x in data:
+        want[x] += 1
+    got = oracle.hist256(d)
+    assert list(got) == want and int(got.sum()) == len(data)
+
+
+@settings(max_examples=60, deadline=None)
+@given(n=st.integers(0, 300), seed=st.integers(0, 2**31 - 1), a=st.integers(-64, 64))
+def test_saxpy_random_integer_exact(n, seed, a):
+    """Integer-valued a, x, y (|.| <= 2^10): y' = a x + y is exact in fp32, so the oracle must
+    match the exact integer result for any length (incl. 0)."""
+    g = np.random.default_rng(seed)
+    x = g.integers(-1024, 1025, size=n).astype(np.float32)
+    y = g.integers(-1024, 1025, size=n).astype(np.float32)
+    want = a * x.astype(np.int64) + y.astype(np.int64)
+    assert np.array_equal(oracle.saxpy(float(a), x, y.copy()).astype(np.int64), want)
