@@ -569,21 +569,20 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
                 SegDesc s;
                 memset(&s, 0, sizeof(s));
                 int nalign = j.kernel == K_HIST256 ? 1 : j.nbufs;  // counts need no alignment
-                uint64_t mis = ch.staged[k * SVP_MAX_BUFS] & 15;
+                const uint64_t mis = ch.staged[k * SVP_MAX_BUFS] & 15;
                 bool co = true;
                 for (int b = 0; b < j.nbufs; ++b) {
                     s.ptr[b] = ch.staged[k * SVP_MAX_BUFS + b];
                     if (b < nalign && (s.ptr[b] & 15) != mis) co = false;
                 }
-                int es = elem_size(j.kernel, 0);
-                if (mis % es) co = false;
                 s.n = j.n;
-                s.flags = (uint16_t)((co ? 0 : SEG_SCALAR) | (j.kernel << SEG_KIND_SHIFT));
-                s.shift = co ? (uint16_t)(mis / es) : 0;
+                uint64_t nt = 0;
+                bool scalar = false;
+                seg_layout(s.ptr[0], co, elem_size(j.kernel, 0), T, j.n, &s.shift, &nt, &scalar);
+                s.flags = (uint16_t)((scalar ? SEG_SCALAR : 0) | (j.kernel << SEG_KIND_SHIFT));
                 s.f[0] = j.f0;
                 s.f[1] = j.f1;
                 s.tile_begin = tiles;
-                uint64_t nt = j.n ? (j.n + s.shift + T - 1) / T : 0;
                 if (tiles + nt >= (1ull << 31)) {
                     d.err = "svp_flush: coalesced launch exceeds 2^31 tiles";
                     return SVP_E_UNSUPPORTED;

@@ -21,17 +21,8 @@ __device__ __forceinline__ int find_seg(const SegDesc* __restrict__ segs, int ns
     return lo - 1;
 }
 
-// Element range [e0, e1) of local tile lt of a segment.  Tiles are laid out in a
-// virtual index space shifted by `shift` so that every interior tile starts on a 16-B
-// boundary of all the segment's buffers; `vec` says the whole tile is interior.
-__device__ __forceinline__ void tile_range(uint64_t n, uint32_t shift, uint32_t flags, uint32_t lt, int tile,
-                                           int64_t& e0, int64_t& e1, bool& vec) {
-    int64_t v0 = (int64_t)lt * tile - (int64_t)shift;
-    int64_t v1 = v0 + tile;
-    e0 = v0 > 0 ? v0 : 0;
-    e1 = v1 < (int64_t)n ? v1 : (int64_t)n;
-    vec = !(flags & SEG_SCALAR) && v0 >= 0 && v1 <= (int64_t)n;
-}
+// tile_range (element range of a segment's local tile) lives in tables.h: the host-side
+// layout (seg_layout) and the kernels share it, and tests/tile_check.cpp checks both on CPU.
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));

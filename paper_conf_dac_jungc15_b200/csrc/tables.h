@@ -10,6 +10,12 @@
 #pragma once
 #include <stdint.h>
 
+#ifdef __CUDACC__
+#define SVP_HD __host__ __device__ __forceinline__
+#else
+#define SVP_HD inline
+#endif
+
 namespace svp {
 
 // Elementwise / histogram segment: 64 bytes.
@@ -29,6 +35,33 @@ enum : uint16_t { SEG_SCALAR = 1, SEG_KIND_SHIFT = 8 };
 // table_mode = SVP_TABLE_PARAM: a launch of at most kParamSegs segments receives its table
 // by value as a __grid_constant__ kernel parameter (15 KiB of the 32 KiB parameter space):
 // no table upload and segment reads served from the constant cache.
+// Tile layout of one segment (host side of the segment table): ptr0 = address of the
+// first tiled buffer, co = every tiled buffer of the VP has the same address mod 16,
+// es = element size.  Tiles live in a virtual index space shifted by `shift` elements so
+// that every interior tile starts 16-B aligned in all buffers (the kernels' float4 /
+// uint4 path, tile_range below); a VP whose buffers are mutually misaligned (or
+// misaligned by a non-multiple of es) gets shift 0 and the scalar path (SEG_SCALAR).
+inline void seg_layout(uint64_t ptr0, bool co, int es, int tile, uint64_t n, uint16_t* shift, uint64_t* ntiles,
+                       bool* scalar) {
+    const uint64_t mis = ptr0 & 15;
+    const bool ok = co && mis % (uint64_t)es == 0;
+    *scalar = !ok;
+    *shift = ok ? (uint16_t)(mis / (uint64_t)es) : 0;
+    *ntiles = n ? (n + *shift + (uint64_t)tile - 1) / (uint64_t)tile : 0;
+}
+
+// Element range [e0, e1) of local tile lt of a segment.  Tiles are laid out in a
+// virtual index space shifted by `shift` so that every interior tile starts on a 16-B
+// boundary of all the segment's buffers; `vec` says the whole tile is interior.
+SVP_HD void tile_range(uint64_t n, uint32_t shift, uint32_t flags, uint32_t lt, int tile, int64_t& e0, int64_t& e1,
+                       bool& vec) {
+    int64_t v0 = (int64_t)lt * tile - (int64_t)shift;
+    int64_t v1 = v0 + tile;
+    e0 = v0 > 0 ? v0 : 0;
+    e1 = v1 < (int64_t)n ? v1 : (int64_t)n;
+    vec = !(flags & SEG_SCALAR) && v0 >= 0 && v1 <= (int64_t)n;
+}
+
 // The parameter block is sized to the launch: CAP in {16, 64} segments (1 or 4 KiB), the
 // smallest that holds the group.  A launch's parameters are pushed through the front end
 // with the launch; a 15-KiB block (the earlier 240-segment cap) cost ~9 us per launch on an
