@@ -18,7 +18,6 @@
 
 namespace svp {
 
-constexpr int DK = kDgemmBK;
 
 __device__ __forceinline__ int find_dgemm(const DgemmDesc* __restrict__ d, int n, uint32_t t) {
     int lo = 0, hi = n;
@@ -30,8 +29,8 @@ __device__ __forceinline__ int find_dgemm(const DgemmDesc* __restrict__ d, int n
     return lo - 1;
 }
 
-// TM x TN output tile, (TM/4) x (TN/4) threads with 4x4 accumulators each
-template <int TM, int TN>
+// TM x TN output tile, (TM/4) x (TN/4) threads with 4x4 accumulators each, DK-deep k blocks
+template <int TM, int TN, int DK>
 __global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* __restrict__ descs, int n,
                                                                uint32_t total) {
     constexpr int NT = (TM / 4) * (TN / 4);
@@ -57,14 +56,14 @@ __global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* 
         auto load = [&](int k0) {
 #pragma unroll
             for (int i = 0; i < LA; ++i) {
-                const int idx = tid + i * NT;  // A: TM rows x 16 k, k fastest
-                const int r = idx >> 4, c = idx & 15;
+                const int idx = tid + i * NT;  // A: TM rows x DK k, k fastest
+                const int r = idx / DK, c = idx % DK;
                 const int gm = m0 + r, gk = k0 + c;
                 ra[i] = (gm < M && gk < K) ? A[(size_t)gm * K + gk] : 0.0;
             }
 #pragma unroll
             for (int i = 0; i < LB; ++i) {
-                const int idx = tid + i * NT;  // B: 16 k x TN cols, n fastest
+                const int idx = tid + i * NT;  // B: DK k x TN cols, n fastest
                 const int rr = idx / TN, cc = idx % TN;
                 const int bk = k0 + rr, bn = n0 + cc;
                 rb[i] = (bk < K && bn < N) ? B[(size_t)bk * N + bn] : 0.0;
@@ -74,7 +73,7 @@ __global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* 
 #pragma unroll
             for (int i = 0; i < LA; ++i) {
                 const int idx = tid + i * NT;
-                As[buf][idx & 15][idx >> 4] = ra[i];
+                As[buf][idx % DK][idx / DK] = ra[i];
             }
 #pragma unroll
             for (int i = 0; i < LB; ++i) {
@@ -130,16 +129,33 @@ __global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* 
 }
 
 cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total, int grid, bool small, cudaStream_t s) {
-    if (small) k_dgemm<kDgemmSmall, kDgemmSmall><<<grid, (kDgemmSmall / 4) * (kDgemmSmall / 4), 0, s>>>(descs, n, total);
-    else k_dgemm<kDgemmBM, kDgemmBN><<<grid, (kDgemmBM / 4) * (kDgemmBN / 4), 0, s>>>(descs, n, total);
+    // small tiles: 32-deep k stages (fewer barriers per tile, 255 registers) when all tiles
+    // are resident at once at that occupancy -- the Table 1 program with 1-4 VPs (S5: 1 VP
+    // 14.9 -> 12.4 ms); otherwise the 16-deep variant's higher occupancy wins (8 VPs).
+    static const int deep_cap = [] {
+        int dev = 0, sms = 0, per = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_dgemm<kDgemmSmall, kDgemmSmall, kDgemmSmallDeepBK>,
+                                                      (kDgemmSmall / 4) * (kDgemmSmall / 4), 0);
+        cudaGetLastError();
+        return sms * per;
+    }();
+    if (small && total <= (uint32_t)deep_cap)
+        k_dgemm<kDgemmSmall, kDgemmSmall, kDgemmSmallDeepBK>
+            <<<grid, (kDgemmSmall / 4) * (kDgemmSmall / 4), 0, s>>>(descs, n, total);
+    else if (small)
+        k_dgemm<kDgemmSmall, kDgemmSmall, kDgemmSmallBK>
+            <<<grid, (kDgemmSmall / 4) * (kDgemmSmall / 4), 0, s>>>(descs, n, total);
+    else k_dgemm<kDgemmBM, kDgemmBN, kDgemmBK><<<grid, (kDgemmBM / 4) * (kDgemmBN / 4), 0, s>>>(descs, n, total);
     return cudaGetLastError();
 }
 
 cudaError_t query_limits_dgemm(int* per_sm, int* per_sm_small) {
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k_dgemm<kDgemmBM, kDgemmBN>,
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k_dgemm<kDgemmBM, kDgemmBN, kDgemmBK>,
                                                                   (kDgemmBM / 4) * (kDgemmBN / 4), 0);
     if (e) return e;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm_small, k_dgemm<kDgemmSmall, kDgemmSmall>,
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm_small, k_dgemm<kDgemmSmall, kDgemmSmall, kDgemmSmallBK>,
                                                          (kDgemmSmall / 4) * (kDgemmSmall / 4), 0);
 }
 

@@ -126,5 +126,7 @@ constexpr int kGemmBM = 128, kGemmBN = 128, kGemmBK = 32;
 constexpr int kTf32BM = 128, kTf32BN = 256, kTf32BK = 16;
 constexpr int kDgemmBM = 64, kDgemmBN = 64, kDgemmBK = 16;
 constexpr int kDgemmSmall = 32;  // square tile of the small-launch DGEMM variant
+constexpr int kDgemmSmallBK = 16;      // k depth per stage of the small variant
+constexpr int kDgemmSmallDeepBK = 32;  // ... when every tile fits in one wave at its occupancy
 
 }  // namespace svp
