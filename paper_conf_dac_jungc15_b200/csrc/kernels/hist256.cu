@@ -26,6 +26,8 @@
 // writes its counts (hist_flush_fused).
 #include <string.h>
 
+#include <atomic>
+
 #include "../launch.h"
 #include "common.cuh"
 
@@ -309,7 +311,7 @@ __global__ void __launch_bounds__(kHistBlock) k_hist256_p(const __grid_constant_
 
 template <int CAP>
 static cudaError_t hist_attr_p() {
-    static bool attr[64] = {};
+    static std::atomic<bool> attr[64] = {};  // per device; worker threads of several GPUs launch
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev < 64 && !attr[dev]) {
@@ -321,7 +323,7 @@ static cudaError_t hist_attr_p() {
 }
 
 static cudaError_t hist_attr() {
-    static bool attr[64] = {};
+    static std::atomic<bool> attr[64] = {};  // per device; worker threads of several GPUs launch
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev < 64 && !attr[dev]) {

@@ -20,6 +20,8 @@
 #include <cuda.h>
 #include <stdio.h>
 
+#include <atomic>
+
 #include "../launch.h"
 #include "common.cuh"
 
@@ -182,7 +184,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     }
 }
 
-static bool g_smem_set[64] = {};
+static std::atomic<bool> g_smem_set[64] = {};  // per device (one worker thread per GPU)
 
 cudaError_t launch_sgemm_ffma(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
                               cudaStream_t s) {

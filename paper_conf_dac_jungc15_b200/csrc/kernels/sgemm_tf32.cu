@@ -80,6 +80,8 @@
 
 #include <algorithm>
 
+#include <atomic>
+
 #include "../launch.h"
 #include "common.cuh"
 
@@ -687,7 +689,7 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
     }
 }
 
-static bool g_attr_set[20][64] = {};
+static std::atomic<bool> g_attr_set[20][64] = {};  // per kernel variant and device
 
 template <int SPLIT, int CG, int NH = 1>
 static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uint32_t total, int clusters,
