@@ -490,7 +490,7 @@ static svp_status plan_sgemm_tail(Executor* e, Dev& d, Flush& f, Chunk& ch, std:
             g.tile_begin = (uint32_t)pd.size();
             g.tiles_n = 1;
             pd.push_back(g);
-            uint8_t m[256];
+            alignas(64) uint8_t m[256];  // CUtensorMap is 64-B aligned
             if (encode_gemm_maps_view(m, m + 128, A + (size_t)sb.m0 * j.K + k0, B + (size_t)k0 * j.N + sb.n0, sb.rows,
                                       sb.cols, kl, j.K, j.N) != 0) {
                 d.err = "cuTensorMapEncodeTiled failed for an sgemm tail slice";
