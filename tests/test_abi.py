@@ -212,3 +212,21 @@ def test_table_mode_values():
     with pytest.raises(svp.SvpError) as e:
         svp.Context(dry_run=True, table_mode=2)
     assert e.value.status == svp.SVP_E_INVAL
+
+
+def test_use_after_finalize_and_null_context():
+    """after svp_finalize the binding holds no handle, and every entry point
+    answers a null context with SVP_E_INVAL (no crash, no CUDA call)."""
+    c = svp.Context(dry_run=True)
+    k = c.register_kernel("vecadd")
+    c.close()
+    c.close()  # idempotent
+    for call in (lambda: c.flush(), lambda: c.profile(-1), lambda: c.flush_stats(), lambda: c.reset_profile(),
+                 lambda: c.submit(0, k, svp.args_vecadd(0), [(0, 0, 1, 0)] * 2 + [(0, 0, 2, 0)]),
+                 lambda: c.register_kernel("saxpy"), lambda: c.vp_device(0)):
+        with pytest.raises(svp.SvpError) as e:
+            call()
+        assert e.value.status == svp.SVP_E_INVAL
+    L = svp.load()
+    assert L.svp_flush(None) == svp.SVP_E_INVAL
+    assert L.svp_finalize(None) in (svp.SVP_OK, svp.SVP_E_INVAL)
