@@ -48,6 +48,11 @@ CONFIG_NAMES = {
 
 IMPL_NAMES = ("ffma", "3xtf32", "tf32bf16")  # svp.SGEMM_FFMA, SGEMM_3XTF32, SGEMM_TF32BF16
 IMPLS = {n: i for i, n in enumerate(IMPL_NAMES)}
+# what the path computes in: the memory-bound kernels are fp32 (u8 -> u32 for hist256); the
+# fp32 "sgemm" contract (1e-5) is met by the selected implementation
+DTYPE_LABEL = {"tf32bf16": "f32 (sgemm: tf32 + 2x bf16 MMAs on an operand hi/lo split, f32 accumulate)",
+               "3xtf32": "f32 (sgemm: 3x tf32 MMAs on an operand hi/lo split, f32 accumulate)",
+               "ffma": "f32"}
 
 
 # ----------------------------------------------------------------------------- helpers
@@ -58,8 +63,9 @@ def trace(msg):
 
 def dist_setup():
     """One process per GPU (torchrun).  SVP_BENCH_DEVICE=<ordinal> pins every rank to one
-    GPU (tests the multi-rank path on a 1-GPU box; the barrier/max-over-ranks then run on
-    gloo because NCCL refuses two ranks on one device)."""
+    GPU (tests the multi-rank path on a 1-GPU box).  The process group is gloo: it only
+    carries the barrier and the max / sum of a few timing scalars -- the data path has no
+    collective (VPs share no data; BASELINE.json: "NCCL is not used")."""
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -69,10 +75,9 @@ def dist_setup():
     if ws > 1:
         import torch.distributed as dist
         import torch
-        backend = "nccl" if (torch.cuda.is_available() and forced is None) else "gloo"
         if torch.cuda.is_available():
             torch.cuda.set_device(local)
-        dist.init_process_group(backend=backend)
+        dist.init_process_group(backend="gloo")
     return rank, ws, local
 
 
@@ -87,8 +92,7 @@ def max_over_ranks(x: float, ws: int) -> float:
         return x
     import torch
     import torch.distributed as dist
-    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
-    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    t = torch.tensor([x], dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -98,8 +102,7 @@ def sum_over_ranks(x: float, ws: int) -> float:
         return x
     import torch
     import torch.distributed as dist
-    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
-    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    t = torch.tensor([x], dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.SUM)
     return float(t.item())
 
@@ -130,14 +133,19 @@ class Clocks:
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
-    def __init__(self, device_index: int):
+    def __init__(self, device_indices):
         self.p = None
         self.t0 = self.t1 = None
         self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        if isinstance(device_indices, int):
+            device_indices = [device_indices]
         try:
             import torch
-            uuid = str(torch.cuda.get_device_properties(device_index).uuid)
-            ident = ["--id=GPU-" + uuid] if uuid and not uuid.startswith("GPU-") else (["--id=" + uuid] if uuid else [])
+            uu = []
+            for d in device_indices:
+                u = str(torch.cuda.get_device_properties(d).uuid)
+                uu.append(u if u.startswith("GPU-") else "GPU-" + u)
+            ident = ["--id=" + ",".join(uu)] if uu else []
         except Exception:
             ident = []
         try:
@@ -259,9 +267,10 @@ def run_reference(args, rank, ws):
     value = n * args.steps / dt
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "jobs/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
-            "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f32",
-            "data": "synthetic",
-            "config": {"workload": CONFIG_NAMES[args.config], "vps": len(specs), "sample_vps": n,
+            "higher_is_better": True, "scaling": "strong" if args.gpus > 1 else "weak", "vs_baseline": None,
+            "dtype": "f64 accumulation for sgemm (oracle), f32 elsewhere", "data": "synthetic",
+            "config": {"workload": CONFIG_NAMES[args.config], "config_index": args.config, "vps": len(specs),
+                       "sample_vps": n,
                        "parallelism": f"host threads x{min(cores, n)}"},
             "cpu_baseline": {"value": value, "unit": "jobs/s", "cores": min(cores, n), "kind": "oracle",
                              "sample": f"first {n} of {len(specs)} VPs (kernel = vp % 5) per step"},
@@ -269,17 +278,78 @@ def run_reference(args, rank, ws):
     print(json.dumps(line), flush=True)
 
 
-def timed_steps(ctx, jobs, steps, stream):
-    import torch
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    torch.cuda.synchronize()
-    e0.record(stream)
-    for _ in range(steps):
-        ctx.submit_batch(jobs)
-        ctx.flush()
-    e1.record(stream)
-    torch.cuda.synchronize()
-    return e0.elapsed_time(e1) / 1e3
+L2_BYTES = 126 << 20  # B200 L2 (B200_PROFILING.md)
+
+
+def n_buffer_sets(specs):
+    """Rotating buffer sets so that consecutive steps never find their inputs in L2: one set
+    when a step's working set is already >= 4 x L2, else enough sets to cover 4 x L2
+    (cfg1: 24 MiB per step -> 24 sets; cfg2: 48 MiB -> 11 sets)."""
+    ws = sum(s.input_bytes() + s.output_bytes() for s in specs)
+    return 1 if ws >= 4 * L2_BYTES else -(-4 * L2_BYTES // max(1, ws))
+
+
+def l2_note(specs, nsets):
+    ws = sum(s.input_bytes() + s.output_bytes() for s in specs)
+    if nsets == 1:
+        return "inputs > L2: %.2f GB of VP buffers touched per step" % (ws / 1e9)
+    return ("step working set %.1f MiB < L2: %d rotating buffer sets (%.0f MiB > 4 x L2), step i uses set i mod %d"
+            % (ws / 2**20, nsets, nsets * ws / 2**20, nsets))
+
+
+class Arm:
+    """One svp.Context driving this process's GPUs, and the workload's VP buffers (one or
+    more rotating buffer sets) pre-marshalled as JobBatches."""
+
+    def __init__(self, specs, inputs, residency, ordinals, streams, nsets=1, kids=None, **cfg):
+        from paper_conf_dac_jungc15_b200 import svp
+        from paper_conf_dac_jungc15_b200.vpset import VPSet
+        self.svp = svp
+        self.ordinals = list(ordinals)
+        self.streams = streams
+        self.ctx = svp.Context(num_gpus=len(self.ordinals), device_ids=self.ordinals,
+                               external_streams=[st.cuda_stream for st in streams], **cfg)
+        self.sets = [VPSet(self.ctx, specs, inputs, residency,
+                           device_ordinals=self.ordinals if residency == "device" else None)
+                     for _ in range(nsets)]
+        self.kids = self.sets[0].kids
+        self.batches = [svp.JobBatch(vs.job_list()) for vs in self.sets]
+        self.i = 0
+
+    def step(self):
+        self.ctx.submit_batch(self.batches[self.i % len(self.batches)])
+        self.ctx.flush()
+        self.i += 1
+
+    def steps(self, k):
+        for _ in range(k):
+            self.step()
+
+    def timed(self, k):
+        """k steps bracketed by CUDA events on every GPU's stream (the stream the library
+        joins); returns (max over GPUs, per-GPU seconds)."""
+        import torch
+        evs = []
+        for d, st in zip(self.ordinals, self.streams):
+            torch.cuda.synchronize(d)
+        for st in self.streams:
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(st)
+            evs.append((e0, e1))
+        self.steps(k)
+        for (e0, e1), st in zip(evs, self.streams):
+            e1.record(st)
+        for d in set(self.ordinals):
+            torch.cuda.synchronize(d)
+        per = [e0.elapsed_time(e1) / 1e3 for e0, e1 in evs]
+        return max(per), per
+
+    def device_stats(self):
+        return [self.ctx.device_stats(g) for g in range(len(self.ordinals))]
+
+    def close(self):
+        self.ctx.close()
+        self.sets = []
 
 
 def launches_per_flush(ctx):
@@ -289,92 +359,32 @@ def launches_per_flush(ctx):
     return int(ctx.flush_stats()["kernel_launches"])
 
 
-def run_svp(args, rank, ws, local):
+def gpu_plan(args, ws, local):
+    """Which CUDA devices this process drives.  torchrun (WORLD_SIZE = N): one GPU per rank.
+    Otherwise one process drives all N GPUs through the library's own Job Dispatcher and
+    per-GPU workers; SVP_BENCH_DEVICES="0,0" maps N logical GPUs onto given ordinals (a
+    1-GPU box can then exercise the N-GPU path; the line says so)."""
     import torch
+    N = args.gpus
+    if ws > 1:
+        if ws != N:
+            raise SystemExit(f"--gpus {N} but WORLD_SIZE={ws}: launch one rank per GPU")
+        return [local], "process"
+    env = os.environ.get("SVP_BENCH_DEVICES")
+    if env:
+        ords = [int(x) for x in env.split(",") if x.strip()]
+        if len(ords) != N:
+            raise SystemExit(f"SVP_BENCH_DEVICES lists {len(ords)} devices, --gpus {N}")
+    else:
+        ords = list(range(N))
+    have = torch.cuda.device_count()
+    if max(ords) >= have:
+        raise SystemExit(f"--gpus {N} needs CUDA devices {ords}, this box has {have}")
+    return ords, "single"
+
+
+def roofline_of(kstats, impl, peaks, peak_src):
     from paper_conf_dac_jungc15_b200 import svp
-    from paper_conf_dac_jungc15_b200.vpset import VPSet
-
-    torch.cuda.set_device(local)
-    stream = torch.cuda.current_stream()
-    trace("specs")
-    # weak scaling (default): every GPU gets a full workload of its own -- N x 256 VPs for
-    # cfg5 -- sharded by the Job Dispatcher's LPT (VPs are independent units, no collective);
-    # strong: the config's fixed VP count split over the N GPUs
-    per_gpu = args.vps or len(W.config_specs(args.config))
-    all_specs = W.config_specs(args.config, nvps=per_gpu * (ws if args.scaling == "weak" else 1))
-    specs = my_specs(all_specs, rank, ws)
-    t_gen = time.perf_counter()
-    inputs = W.make_inputs_many(specs)
-    t_gen = time.perf_counter() - t_gen
-
-    # ---------------- device-resident run (value)
-    impl = IMPLS[args.sgemm_impl]
-    trace("inputs ready")
-    f4 = dict(hetero=bool(args.hetero), graph=bool(args.graph), table_mode=args.table_mode)  # options
-    ctx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, external_streams=[stream.cuda_stream],
-                      validate_ptrs=True, sgemm_impl=impl, **f4)
-    vs = VPSet(ctx, specs, inputs, "device", device_ordinals=[local])
-    jobs = svp.JobBatch(vs.job_list())  # marshalled once; each step resubmits it
-    ctx.submit_batch(jobs)
-    ctx.flush()
-    torch.cuda.synchronize()
-    clocks = Clocks(local)  # sampling starts before the warm-up (nvidia-smi start-up latency)
-    for _ in range(max(0, args.warmup - 1)):
-        ctx.submit_batch(jobs)
-        ctx.flush()
-    ctx.reset_profile()
-    barrier(ws)
-    trace("warmup done, timing")
-    torch.cuda.synchronize()
-    clocks.mark_start()
-    dt = timed_steps(ctx, jobs, args.steps, stream)
-    clocks.mark_end()
-    clk = clocks.stop()
-    barrier(ws)
-    dt_max = max_over_ranks(dt, ws)
-    n_jobs_total = sum_over_ranks(len(specs), ws)
-    value = n_jobs_total * args.steps / dt_max
-    st = ctx.flush_stats()
-    launches = launches_per_flush(ctx) * args.steps
-    main_kstats = {name: ctx.kernel_stats(kid) for name, kid in vs.kids.items()}
-    if args.hetero:
-        main_kstats["ew_mix"] = ctx.kernel_stats(svp.KERNEL_EW_MIX)
-    # Per-kernel roofline numbers need each kernel's own duration: in the timed run the
-    # coalesced launches of different kernels overlap on the compute streams (that is the
-    # interleaving gain), so their events overlap too.  Re-run the same jobs on ONE stream
-    # (profile_level 1: CUDA events around every launch on its stream) and read the stats.
-    trace("timed region done")
-    ictx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1, interleave=False,
-                       external_streams=[stream.cuda_stream], sgemm_impl=impl)
-    for k in vs.kids:
-        ictx.register_kernel(k)
-    ictx.submit_batch(jobs)
-    ictx.flush()
-    ictx.reset_profile()
-    iso_steps = max(3, args.steps // 5)
-    iso_dt = timed_steps(ictx, jobs, iso_steps, stream)
-    kstats = {name: ictx.kernel_stats(kid) for name, kid in vs.kids.items()}
-    ictx.close()
-    iso_value = n_jobs_total * iso_steps / max_over_ranks(iso_dt, ws)
-
-    # memory-bound kernels: algorithmic bytes / event-timed kernel time
-    mb_bytes = sum(k["bytes"] for n, k in kstats.items() if n != "sgemm")
-    mb_ns = sum(k["total_ns"] for n, k in kstats.items() if n != "sgemm")
-    hbm_gbs = mb_bytes / mb_ns if mb_ns else None
-    per_kernel = {}
-    for n, k in kstats.items():
-        if not k["launches"]:
-            continue
-        avg = k["total_ns"] / k["launches"]
-        if n == "sgemm":
-            per_kernel[n] = {"avg_launch_ms": avg / 1e6, "tflops": k["flops"] / k["total_ns"] / 1e3,
-                             "share_of_kernel_time": None}
-        else:
-            per_kernel[n] = {"avg_launch_ms": avg / 1e6, "gbs": k["bytes"] / k["total_ns"]}
-    tot_k = sum(k["total_ns"] for k in kstats.values())
-    for n in per_kernel:
-        per_kernel[n]["share_of_kernel_time"] = kstats[n]["total_ns"] / tot_k if tot_k else None
-    peaks, peak_src = measured_peaks()
     dom = max(kstats, key=lambda n: kstats[n]["total_ns"])
     dk = kstats[dom]
     if dom == "sgemm" and impl == svp.SGEMM_3XTF32:
@@ -411,14 +421,10 @@ def run_svp(args, rank, ws, local):
                      "then runs the SGEMM's partial last wave as the K-split tail and Black-Scholes in dynamic "
                      "tile order); in the interleaved timed step the launches co-run (timed_kernel_ms_per_step)")
     if roof["bound"] == "tensor":
-        # context: the same accounting against the guide's nominal 2.25 PFLOP/s dense bf16
-        # (the measured cuBLAS burst figure is power-limited and can be exceeded)
         nominal = 2250.0 * roof["peak"] / float(peaks.get("bf16_tflops", 1590.0))
         roof["peak_nominal"] = nominal
         roof["frac_of_nominal"] = roof["achieved"] / nominal
         if "bf16_tflops_sustained" in peaks:
-            # context: the driver's sustained (power-capped, 4 s back to back) bf16 figure,
-            # scaled the same way; the step runs at the 1000 W cap (profiles/r01 power probe)
             sus = float(peaks["bf16_tflops_sustained"]) * roof["peak"] / float(peaks.get("bf16_tflops", 1590.0))
             roof["peak_sustained"] = sus
             roof["frac_of_sustained"] = roof["achieved"] / sus
@@ -430,117 +436,220 @@ def run_svp(args, rank, ws, local):
                          if dom == "sgemm" else "")
             if key in tr:
                 roof["traffic"] = tr[key]
+                roof["traffic_source"] = "profiles/traffic_r01.json (ncu --set full, cfg5 launch)"
         except Exception:
             pass
+    return dom, roof
 
-    trace("one-stream pass done")
-    # ---------------- the other implementation of the fp32 "sgemm" kernel, same jobs
+
+def run_svp(args, rank, ws, local):
+    import torch
+    from paper_conf_dac_jungc15_b200 import svp
+
+    ords, mode = gpu_plan(args, ws, local)
+    N = args.gpus
+    scaling = args.scaling if args.scaling != "auto" else ("strong" if N > 1 else "weak")
+    torch.cuda.set_device(ords[0])
+    streams = [torch.cuda.current_stream(d) for d in ords]
+    impl = IMPLS[args.sgemm_impl]
+    trace(f"mode {mode}, devices {ords}, scaling {scaling}")
+    # the workload: BASELINE config k; strong scaling = its VPs split over the N GPUs (the
+    # config's definition for cfg5 at 2/4/8 GPUs), weak = N x its VPs
+    per_gpu = args.vps or len(W.config_specs(args.config))
+    all_specs = W.config_specs(args.config, nvps=per_gpu * (N if scaling == "weak" else 1))
+    specs = my_specs(all_specs, rank, ws) if mode == "process" else list(all_specs)
+    t_gen = time.perf_counter()
+    inputs = W.make_inputs_many(specs)
+    t_gen = time.perf_counter() - t_gen
+    nsets = n_buffer_sets(all_specs)
+    f4 = dict(hetero=bool(args.hetero), graph=bool(args.graph), table_mode=args.table_mode)
+
+    # ---------------- device-resident run (value)
+    arm = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, validate_ptrs=True,
+              sgemm_impl=impl, **f4)
+    kids = arm.kids
+    assert arm.ctx.flush_stats is not None
+    arm.step()
+    for d in set(ords):
+        torch.cuda.synchronize(d)
+    clocks = Clocks(sorted(set(ords)))  # sampling starts before the warm-up (nvidia-smi start-up)
+    arm.steps(max(0, args.warmup - 1))
+    arm.ctx.reset_profile()
+    barrier(ws)
+    clocks.mark_start()
+    dt, dt_per_gpu = arm.timed(args.steps)
+    clocks.mark_end()
+    clk = clocks.stop()
+    barrier(ws)
+    dt_max = max_over_ranks(dt, ws)
+    n_jobs_total = sum_over_ranks(len(specs), ws)
+    value = n_jobs_total * args.steps / dt_max
+    st = arm.ctx.flush_stats()
+    launches = launches_per_flush(arm.ctx) * args.steps
+    main_kstats = {name: arm.ctx.kernel_stats(kid) for name, kid in kids.items()}
+    if args.hetero:
+        main_kstats["ew_mix"] = arm.ctx.kernel_stats(svp.KERNEL_EW_MIX)
+    dstats = arm.device_stats()
+    gpus_driven = sum(1 for d in dstats if d["flushes"] > 0)
+    per_gpu_rows = []
+    for g, (d, t) in enumerate(zip(dstats, dt_per_gpu)):
+        per_gpu_rows.append({"gpu": g, "ordinal": d["ordinal"], "vps": d["vps"],
+                             "lpt_est_load_ms": d["est_load_ns"] / 1e6,
+                             "device_ms_per_step": d["device_ns"] / args.steps / 1e6,
+                             "kernel_ms_per_step": d["kernel_ns"] / args.steps / 1e6,
+                             "event_ms_per_step": t / args.steps * 1e3})
+    spans = [r["device_ms_per_step"] for r in per_gpu_rows]
+    loads = [r["lpt_est_load_ms"] for r in per_gpu_rows]
+    multi = {"mode": mode, "devices": ords, "gpus_driven": gpus_driven if mode == "single" else ws,
+             "logical_gpus": len(set(ords)) < len(ords),
+             "per_gpu": per_gpu_rows,
+             "imbalance_max_over_mean": (max(spans) / (sum(spans) / len(spans))) if spans and sum(spans) else None,
+             "lpt_predicted_makespan_ms": max(loads) if loads else None,
+             "lpt_predicted_imbalance": (max(loads) / (sum(loads) / len(loads))) if loads and sum(loads) else None}
+    if mode == "single":
+        assert gpus_driven == N, f"--gpus {N} but the flush ran on {gpus_driven} GPUs"
+    trace("timed region done")
+
+    # ---------------- one stream per GPU: per-kernel roofline numbers (launches do not overlap)
+    iso = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, interleave=False, sgemm_impl=impl)
+    iso.step()
+    iso.ctx.reset_profile()
+    iso_steps = max(3, args.steps // 5)
+    iso_dt, _ = iso.timed(iso_steps)
+    kstats = {name: iso.ctx.kernel_stats(kid) for name, kid in iso.kids.items()}
+    iso.close()
+    iso_value = n_jobs_total * iso_steps / max_over_ranks(iso_dt, ws)
+    mb_bytes = sum(k["bytes"] for n, k in kstats.items() if n != "sgemm")
+    mb_ns = sum(k["total_ns"] for n, k in kstats.items() if n != "sgemm")
+    hbm_gbs = mb_bytes / mb_ns if mb_ns else None
+    per_kernel = {}
+    tot_k = sum(k["total_ns"] for k in kstats.values())
+    for n, k in kstats.items():
+        if not k["launches"]:
+            continue
+        avg = k["total_ns"] / k["launches"]
+        row = {"avg_launch_ms": avg / 1e6, "share_of_kernel_time": k["total_ns"] / tot_k if tot_k else None}
+        if n == "sgemm":
+            row["tflops"] = k["flops"] / k["total_ns"] / 1e3
+        else:
+            row["gbs"] = k["bytes"] / k["total_ns"]
+        per_kernel[n] = row
+    peaks, peak_src = measured_peaks()
+    dom, roof = roofline_of(kstats, impl, peaks, peak_src)
+    if args.config != 5:
+        roof["traffic"] = None  # the committed ncu traffic figure is cfg5's launch
+        roof.pop("traffic_source", None)
+
+    # ---------------- the other implementations of the fp32 "sgemm" kernel, same jobs
     alt = []
-    if not args.no_alt:
-        alts = [a for a in args.alt_impl.split(",") if a and IMPLS[a] != impl]
-        for alt_name in alts:
-            alt_impl = IMPLS[alt_name]
-            actx = svp.Context(num_gpus=1, device_ids=[local], profile_level=1,
-                               external_streams=[stream.cuda_stream], sgemm_impl=alt_impl)
-            for k in vs.kids:
-                actx.register_kernel(k)
-            actx.submit_batch(jobs)
-            actx.flush()
-            actx.reset_profile()
+    if not args.no_alt and "sgemm" in kids:
+        for alt_name in [a for a in args.alt_impl.split(",") if a and IMPLS[a] != impl]:
+            a = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, sgemm_impl=IMPLS[alt_name])
+            a.step()
+            a.ctx.reset_profile()
             ks = max(3, args.steps // 5)
-            adt = max_over_ranks(timed_steps(actx, jobs, ks, stream), ws)
-            sk = actx.kernel_stats(vs.kids["sgemm"]) if "sgemm" in vs.kids else None
-            alt.append({"sgemm_impl": alt_name, "value": n_jobs_total * ks / adt, "unit": "jobs/s",
-                        "ms_per_step": adt / ks * 1e3,
-                        "sgemm_tflops_interleaved": (sk["flops"] / sk["total_ns"] / 1e3) if sk and sk["total_ns"]
-                        else None})
-            actx.close()
-
+            adt = max_over_ranks(a.timed(ks)[0], ws)
+            sk = a.ctx.kernel_stats(a.kids["sgemm"])
+            alt.append({"sgemm_impl": alt_name, "dtype": DTYPE_LABEL[alt_name], "value": n_jobs_total * ks / adt,
+                        "unit": "jobs/s", "ms_per_step": adt / ks * 1e3,
+                        "sgemm_tflops_interleaved": (sk["flops"] / sk["total_ns"] / 1e3) if sk["total_ns"] else None})
+            a.close()
     trace("alt pass done")
-    # ---------------- serial baselines on the same GPU, same buffers, same kernels
-    serial = {}
-    by_kernel = {}
+
+    # ---------------- serial baselines on the same GPUs, same buffers, same kernels
+    serial, by_kernel = {}, {}
     if not args.no_serial:
         for name, kw in (("B1_serial_sync", dict(coalesce=False, interleave=False, sync_each_job=True)),
                          ("B2_serial_async", dict(coalesce=False, interleave=False)),
                          ("B3_serial_graph", dict(coalesce=False, interleave=False, graph=True)),
                          ("B2_profiled", dict(coalesce=False, interleave=False, profile_level=1))):
-            sctx = svp.Context(num_gpus=1, device_ids=[local], external_streams=[stream.cuda_stream],
-                               sgemm_impl=impl, **kw)
-            for k in vs.kids:
-                sctx.register_kernel(k)
-            ks = max(2, args.steps // 5)
-            # warm-up as for the main arm (>= 3 flushes): B3's first flush plans, its second
-            # captures + instantiates the graph; only replays may fall in the timed region
-            for _ in range(max(3, args.warmup)):
-                sctx.submit_batch(jobs)
-                sctx.flush()
-            sctx.reset_profile()
+            # B3 replays one captured graph, so it needs the same buffers every step: one set
+            b = Arm(specs, inputs, "device", ords, streams, 1 if name == "B3_serial_graph" else nsets,
+                    sgemm_impl=impl, **kw)
+            b.steps(max(3, args.warmup))  # B3: plan, capture + instantiate, then replays only
+            b.ctx.reset_profile()
             barrier(ws)
-            sdt = max_over_ranks(timed_steps(sctx, jobs, ks, stream), ws)
+            ks = max(2, args.steps // 5)
+            sdt = max_over_ranks(b.timed(ks)[0], ws)
             if name != "B2_profiled":
                 serial[name] = {"value": n_jobs_total * ks / sdt, "unit": "jobs/s", "steps": ks,
                                 "ms_per_step": sdt / ks * 1e3}
+                if name == "B3_serial_graph" and nsets > 1:
+                    serial[name]["l2"] = "one buffer set (a replayed graph reads the same buffers): L2-resident"
             else:
                 # Eq 9's alignment gain per kernel class: per-job launches vs one coalesced
                 # launch of the same jobs (event-timed kernel time per step, 1 stream each)
-                for kname, kid in vs.kids.items():
-                    st_ser = sctx.kernel_stats(kid)
+                for kname, kid in b.kids.items():
+                    st_ser = b.ctx.kernel_stats(kid)
                     st_coal = kstats[kname]
                     if st_ser["launches"] and st_coal["launches"]:
                         ser_ms = st_ser["total_ns"] / ks / 1e6
-                        coal_ms = st_coal["total_ns"] / st_coal["launches"] / 1e6
+                        coal_ms = st_coal["total_ns"] / iso_steps / 1e6
                         by_kernel[kname] = {"serial_kernel_ms": ser_ms, "coalesced_kernel_ms": coal_ms,
                                             "speedup": ser_ms / coal_ms}
-            sctx.close()
-    ctx.close()
-    del vs
+            b.close()
+    arm.close()
     torch.cuda.empty_cache()
-
     trace("serial passes done")
+
     # ---------------- e2e: pinned host buffers, copies inside the timed region
     e2e = None
     if not args.no_e2e:
-        hctx = svp.Context(num_gpus=1, device_ids=[local], external_streams=[stream.cuda_stream],
-                           arena_bytes=args.arena_gb << 30, sgemm_impl=impl,
-                           max_chunks=int(os.environ.get("SVP_BENCH_MAXCH", "8")), **f4)
-        hvs = VPSet(hctx, specs, inputs, "host")
-        hjobs = svp.JobBatch(hvs.job_list())
-        for _ in range(2):
-            hctx.submit_batch(hjobs)
-            hctx.flush()
-        hst = hctx.flush_stats()
+        h = Arm(specs, inputs, "host", ords, streams, 1, arena_bytes=args.arena_gb << 30, sgemm_impl=impl,
+                max_chunks=int(os.environ.get("SVP_BENCH_MAXCH", "8")), **f4)
+        h.steps(2)
+        hst = h.ctx.flush_stats()
         barrier(ws)
         ks = args.e2e_steps or max(2, min(args.steps, 5))
-        edt = max_over_ranks(timed_steps(hctx, hjobs, ks, stream), ws)
+        edt = max_over_ranks(h.timed(ks)[0], ws)
         e2e = {"value": n_jobs_total * ks / edt, "unit": "jobs/s",
                "h2d_bytes_per_step": int(sum_over_ranks(hst["h2d_bytes"], ws)),
                "d2h_bytes_per_step": int(sum_over_ranks(hst["d2h_bytes"], ws)),
                "steps": ks, "ms_per_step": edt / ks * 1e3, "chunks": int(hst["chunks"]),
                "api": "svp_submit_batch + svp_flush, HOST_PINNED buffers (H2D/D2H staged + interleaved)"}
-        hctx.close()
-        del hvs
+        h.close()
+
+    # ---------------- weak scaling beside the strong number (N > 1)
+    weak = None
+    if N > 1 and scaling == "strong" and not args.no_weak:
+        wspecs_all = W.config_specs(args.config, nvps=per_gpu * N)
+        wspecs = my_specs(wspecs_all, rank, ws) if mode == "process" else wspecs_all
+        winputs = W.make_inputs_many(wspecs)
+        w = Arm(wspecs, winputs, "device", ords, streams, n_buffer_sets(wspecs_all), sgemm_impl=impl, **f4)
+        w.steps(args.warmup)
+        barrier(ws)
+        ks = max(3, args.steps // 3)
+        wdt = max_over_ranks(w.timed(ks)[0], ws)
+        weak = {"value": sum_over_ranks(len(wspecs), ws) * ks / wdt, "unit": "jobs/s", "vps": len(wspecs_all),
+                "steps": ks, "ms_per_step": wdt / ks * 1e3, "scaling": "weak"}
+        w.close()
+        del winputs
 
     cpu = None
-    if rank == 0 and ws == 1 and not args.no_cpu:
+    if rank == 0 and N == 1 and not args.no_cpu:
         cpu = cpu_baseline(specs, inputs, CONFIG_NAMES[args.config])
 
     total_launches = int(sum_over_ranks(launches, ws))  # collective: every rank calls it
     if rank == 0:
         line = {
-            "metric": METRIC, "value": value, "unit": "jobs/s", "n_gpus": ws, "steps": args.steps,
+            "metric": METRIC, "value": value, "unit": "jobs/s", "n_gpus": N, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": dt_max / args.steps * 1e3, "higher_is_better": True,
-            "scaling": args.scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": CONFIG_NAMES[args.config], "vps": len(all_specs), "vps_this_rank0": len(specs),
-                       "residency": "device (HBM)", "parallelism": f"dp{ws}: VPs sharded by the Job Dispatcher (LPT)",
-                       "l2": "inputs > L2: %.1f GB of VP buffers touched per step" %
-                             (sum(s.algorithmic_bytes() for s in all_specs) / 1e9)},
+            "scaling": scaling, "vs_baseline": None, "dtype": DTYPE_LABEL[args.sgemm_impl],
+            "data": "synthetic",
+            "config": {"workload": CONFIG_NAMES[args.config], "config_index": args.config, "vps": len(all_specs),
+                       "residency": "device (HBM)",
+                       "parallelism": (f"dp{N}: VPs sharded by the Job Dispatcher's kernel-stratified LPT, "
+                                       + ("one process driving all GPUs (per-GPU worker threads)" if mode == "single"
+                                          else "one rank per GPU")),
+                       "l2": l2_note(all_specs, nsets)},
             "clocks": clk, "e2e": e2e, "gpu_launches": total_launches,
             "roofline": roof, "cpu_baseline": cpu,
+            "multi_gpu": multi, "weak_scaling": weak,
             "hbm_gbs_membound": hbm_gbs,
             "hbm_frac_membound": (hbm_gbs / float(peaks["hbm_gbs"])) if hbm_gbs else None,
             "elements_per_s": sum(s.n for s in all_specs) * args.steps / dt_max,
-            "sgemm_impl": args.sgemm_impl, "alt_sgemm_impls": alt, "hetero": args.hetero, "graph": args.graph, "table_mode": args.table_mode,
+            "sgemm_impl": args.sgemm_impl, "alt_sgemm_impls": alt, "hetero": args.hetero, "graph": args.graph,
+            "table_mode": args.table_mode,
             "graph_replays_last_step": int(st["graph_replays"]),
             "timed_kernel_ms_per_step": {n: k["total_ns"] / args.steps / 1e6 for n, k in main_kstats.items()
                                          if k["launches"]},
@@ -551,7 +660,8 @@ def run_svp(args, rank, ws, local):
             "flush": {"host_plan_us": st["host_plan_ns"] / 1e3, "host_issue_us": st["host_issue_ns"] / 1e3,
                       "host_total_us": st["host_total_ns"] / 1e3, "device_ms": st["device_ns"] / 1e6,
                       "groups": int(st["groups"]), "launch_ops": int(st["launches"])},
-            "parity": "tests/test_gpu_parity.py (full-size configs vs oracle; not re-run here)",
+            "parity": "tests/test_gpu_parity.py, test_gpu_sgemm_*.py (full-size configs vs oracle; not re-run here)",
+            "profiler_split": "per-VP attribution inside a coalesced launch: parity unpinned (DESIGN.md §3)",
             "setup_s": {"input_generation": t_gen},
         }
         print(json.dumps(line), flush=True)
@@ -571,8 +681,10 @@ def main():
                     help="implementation of the fp32 'sgemm' kernel (all meet its 1e-5 contract)")
     ap.add_argument("--alt-impl", default="3xtf32,ffma",
                     help="comma list of the other sgemm implementations timed beside the main one")
-    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
-                    help="weak: N x the config's VPs over N GPUs (fixed work per GPU); strong: the config's VPs split")
+    ap.add_argument("--scaling", default="auto", choices=["auto", "weak", "strong"],
+                    help="auto: strong at N > 1 (the config's VPs split over N GPUs, as BASELINE cfg5 states), "
+                         "weak at N = 1; weak: N x the config's VPs (fixed work per GPU)")
+    ap.add_argument("--no-weak", action="store_true", help="N > 1: skip the extra weak-scaling measurement")
     ap.add_argument("--hetero", type=int, default=0, choices=[0, 1],
                     help="heterogeneous coalescing of vecadd/SAXPY/Black-Scholes (NEXT f4)")
     ap.add_argument("--graph", type=int, default=0, choices=[0, 1],

@@ -34,7 +34,7 @@
 extern "C" {
 #endif
 
-#define SVP_ABI_VERSION 4
+#define SVP_ABI_VERSION 5
 
 typedef int32_t svp_status;
 enum {
@@ -143,8 +143,18 @@ int32_t svp_abi_version(void);
  *   "hist256"       counts[b] = #{i: d[i]==b}        args svp_args_hist256  bufs [d IN u8, counts OUT u32[256]]
  *                   (counts are overwritten)
  *   "blackscholes"  call/put per option              args svp_args_bs       bufs [S IN, X IN, T IN, call OUT, put OUT] f32
- *   "sgemm"         C = alpha A B + beta C, fp32 FFMA args svp_args_sgemm   bufs [A IN, B IN, C OUT (INOUT if beta != 0)]
- *   "sgemm_tf32"    same, tcgen05 TF32 tensor cores  (own tolerance 2e-3)
+ *   "sgemm"         C = alpha A B + beta C, fp32     args svp_args_sgemm   bufs [A IN, B IN, C OUT (INOUT if beta != 0)]
+ *                   contract (R10/R20): |c - exact| <= 1e-5 (|alpha||A||B| + |beta C|)_ij
+ *                   + (K+1) 2^-149, Inf/NaN propagated as in IEEE fp32.  cfg.sgemm_impl picks
+ *                   the implementation: SVP_SGEMM_TF32BF16 (default; tcgen05 TF32 + 2 BF16
+ *                   MMAs on a hi/lo operand split), SVP_SGEMM_3XTF32 (3 TF32 MMAs) or
+ *                   SVP_SGEMM_FFMA (fp32 FFMA on the CUDA cores).  The two tensor-core splits
+ *                   add 2^-134 |other operand| per product whose operand is below 2^-115 in
+ *                   magnitude (TF32 / BF16 subnormal granularity); an output their tensor-core
+ *                   accumulation leaves NaN (an Inf / NaN operand, or one near FLT_MAX) is
+ *                   recomputed exactly from A and B (fp64 products and sum, one rounding)
+ *   "sgemm_tf32"    same, tcgen05 TF32 tensor cores  (own tolerance 2e-3; raw operands, so a
+ *                   NaN whose payload is only in the low 13 mantissa bits reads as Inf)
  *   "dgemm"         C = alpha A B + beta C, fp64     args svp_args_dgemm   bufs [A IN, B IN, C OUT (INOUT if beta != 0)] f64
  *                   (the paper's Table 1 guest: 320x320 fp64 matmul)
  * GEMM jobs of different shapes are "identical kernels" too: one grouped launch covers
@@ -328,6 +338,25 @@ typedef struct svp_flush_stats {
 } svp_flush_stats;
 svp_status svp_flush_stats_get(svp_ctx* ctx, svp_flush_stats* out);
 
+/* (ABI 5) Per-GPU view of the Job Dispatcher and the Profiler, for GPU index g
+ * (0..num_gpus-1): how many VPs the Dispatcher has placed there and their summed cost
+ * estimate (ns, the LPT load), and -- accumulated since svp_reset_profile, profile_level
+ * >= 1 -- flushes and jobs that ran there, the summed per-flush device span (first op
+ * start to last op end on that GPU) and the summed event-timed kernel op durations
+ * (ops that overlap on different streams each count in full).  Imbalance across GPUs =
+ * max / mean of device_ns.  Errors: SVP_E_INVAL (null, g out of range). */
+typedef struct svp_device_stats {
+    int32_t ordinal;        /* CUDA device ordinal of GPU index g                       */
+    int32_t vps;            /* VPs placed on it (sticky)                               */
+    double est_load_ns;     /* Dispatcher's summed cost estimate of those VPs           */
+    uint64_t flushes;       /* flushes with work on this GPU                            */
+    uint64_t jobs;          /* jobs run on this GPU                                     */
+    double device_ns;       /* summed per-flush device span                             */
+    double kernel_ns;       /* summed event-timed kernel op durations                   */
+    double last_device_ns;  /* the last flush's span on this GPU                        */
+} svp_device_stats;
+svp_status svp_device_stats_get(svp_ctx* ctx, int32_t g, svp_device_stats* out);
+
 /* ------------------------------------------------------------------ plan introspection */
 /* The last flush's plan, one entry per issued op in issue order (tests, tooling). */
 enum { SVP_OP_H2D = 0, SVP_OP_KERNEL = 1, SVP_OP_D2H = 2 };
@@ -349,6 +378,13 @@ typedef struct svp_plan_op {
 svp_status svp_plan_size(svp_ctx* ctx, int32_t* n_ops);
 /* vps_out (optional, capacity cap) receives the op's member VPs in segment order. */
 svp_status svp_plan_get(svp_ctx* ctx, int32_t i, svp_plan_op* op, int32_t* vps_out, int32_t cap);
+/* (ABI 5) Ordering detail of plan op i: *arena_off / *arena_len = the staging-arena byte
+ * range its chunk uses (len 0: nothing staged), *nwaits = how many earlier ops it waits on
+ * through events (cross-stream waits; ops on the same (device, stream) are ordered by
+ * issue order and are not listed), and waits_out[0 .. min(nwaits, cap)) their plan indices.
+ * Any pointer may be NULL.  Errors: SVP_E_INVAL (null ctx, index out of range). */
+svp_status svp_plan_op_detail(svp_ctx* ctx, int32_t i, uint64_t* arena_off, uint64_t* arena_len,
+                              int32_t* waits_out, int32_t cap, int32_t* nwaits);
 
 #ifdef __cplusplus
 }

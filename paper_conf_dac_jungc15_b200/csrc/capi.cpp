@@ -70,8 +70,8 @@ static svp_status check_ctx(svp_ctx* h) {
         return SVP_E_INVAL;
     }
     Ctx* c = reinterpret_cast<Ctx*>(h);
-    if (c->sticky != SVP_OK) {
-        set_error("context is sticky-errored: " + c->sticky_msg);
+    if (c->sticky.load() != SVP_OK) {
+        set_error("context is sticky-errored: " + c->sticky_message());
         return SVP_E_STATE;
     }
     return SVP_OK;
@@ -142,6 +142,7 @@ svp_status svp_init(const svp_config* cfg, svp_ctx** out) {
         }
     }
     c->dev_load.assign(c->ngpu, 0.0);
+    c->dstats.assign(c->ngpu, DevStats{});
     *out = reinterpret_cast<svp_ctx*>(c);
     return SVP_OK;
     SVP_TRY_END
@@ -297,8 +298,8 @@ static bool same_requests(const std::vector<Job>& a, const std::vector<Job>& b) 
 
 static svp_status do_flush(Ctx* c) {
     std::lock_guard<std::mutex> flk(c->flush_mu);
-    if (c->sticky != SVP_OK) {
-        set_error("context is sticky-errored: " + c->sticky_msg);
+    if (c->sticky.load() != SVP_OK) {
+        set_error("context is sticky-errored: " + c->sticky_message());
         return SVP_E_STATE;
     }
     auto t0 = std::chrono::steady_clock::now();
@@ -340,9 +341,13 @@ static svp_status do_flush(Ctx* c) {
         if (c->exec && !f.ops.empty()) {
             st = executor_run(c->exec, &f);
             if (st == SVP_E_CUDA || st == SVP_E_TIMEOUT) {
-                c->sticky = st;
-                c->sticky_msg = executor_error(c->exec);
-                set_error(c->sticky_msg);
+                const std::string msg = executor_error(c->exec);
+                {
+                    std::lock_guard<std::mutex> lk(c->done_mu);
+                    c->sticky_msg = msg;
+                    c->sticky.store(st);
+                }
+                set_error(msg);
             } else if (st) {
                 set_error(executor_error(c->exec));
             }
@@ -409,7 +414,7 @@ svp_status svp_wait(svp_ctx* h, uint64_t job, int32_t timeout_ms) {
         c->done_cv.wait(lk, done);
     }
     if (c->completed_upto < job) {
-        set_error("svp_wait: context errored before the job ran: " + c->sticky_msg);
+        set_error("svp_wait: context errored before the job ran: " + c->sticky_msg);  // under done_mu
         return SVP_E_STATE;
     }
     lk.unlock();
@@ -598,6 +603,7 @@ svp_status svp_reset_profile(svp_ctx* h) {
     c->prof_total = VpProfile{};
     c->prof_launches = 0;
     for (auto& k : c->kstats) k = KStats{};
+    for (auto& d : c->dstats) d = DevStats{};
     return SVP_OK;
     SVP_TRY_END
 }
@@ -620,6 +626,36 @@ svp_status svp_kernel_stats_get(svp_ctx* h, int32_t kernel, svp_kernel_stats* ou
     out->bytes = k.bytes;
     out->flops = k.flops;
     out->max_ns = k.max_ns;
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+svp_status svp_device_stats_get(svp_ctx* h, int32_t g, svp_device_stats* out) {
+    SVP_TRY_BEGIN
+    if (!h || !out) {
+        set_error("null argument");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    if (g < 0 || g >= c->ngpu) {
+        set_error("svp_device_stats_get: GPU index out of range");
+        return SVP_E_INVAL;
+    }
+    memset(out, 0, sizeof(*out));
+    out->ordinal = g < (int32_t)c->device_ids.size() ? c->device_ids[g] : g;
+    {
+        std::lock_guard<std::mutex> lk(c->dmu);
+        for (const auto& kv : c->vp_dev)
+            if (kv.second == g) out->vps += 1;
+        out->est_load_ns = c->dev_load[g];
+    }
+    std::lock_guard<std::mutex> lk(c->pmu);
+    const DevStats& d = c->dstats[g];
+    out->flushes = d.flushes;
+    out->jobs = d.jobs;
+    out->device_ns = d.device_ns;
+    out->kernel_ns = d.kernel_ns;
+    out->last_device_ns = d.last_device_ns;
     return SVP_OK;
     SVP_TRY_END
 }
@@ -671,6 +707,27 @@ svp_status svp_plan_get(svp_ctx* h, int32_t i, svp_plan_op* op, int32_t* vps_out
     op->measured_ns = o.measured_ns;
     if (vps_out)
         for (int k = 0; k < (int)ch.jobs.size() && k < cap; ++k) vps_out[k] = f.jobs[ch.jobs[k]].vp;
+    return SVP_OK;
+}
+
+svp_status svp_plan_op_detail(svp_ctx* h, int32_t i, uint64_t* arena_off, uint64_t* arena_len, int32_t* waits_out,
+                              int32_t cap, int32_t* nwaits) {
+    if (!h) {
+        set_error("null context");
+        return SVP_E_INVAL;
+    }
+    const Flush& f = reinterpret_cast<Ctx*>(h)->last;
+    if (i < 0 || i >= (int32_t)f.ops.size()) {
+        set_error("svp_plan_op_detail: index out of range");
+        return SVP_E_INVAL;
+    }
+    const Op& o = f.ops[i];
+    const Chunk& ch = f.chunks[o.chunk];
+    if (arena_off) *arena_off = ch.arena_off;
+    if (arena_len) *arena_len = ch.arena_len;
+    if (nwaits) *nwaits = (int32_t)o.wait_ops.size();
+    if (waits_out)
+        for (int k = 0; k < (int)o.wait_ops.size() && k < cap; ++k) waits_out[k] = o.wait_ops[k];
     return SVP_OK;
 }
 

@@ -21,9 +21,10 @@
 #include <string.h>
 
 #include <algorithm>
+#include <chrono>
+#include <condition_variable>
 #include <map>
 #include <mutex>
-#include <chrono>
 #include <thread>
 
 #include "internal.h"
@@ -104,9 +105,26 @@ struct PtrRange {
     int device = -1;
 };
 
+// Persistent per-GPU workers (multi-GPU contexts): GPU g > 0 is driven by worker thread g,
+// created once at svp_init and parked on a condition variable between flushes (SURVEY §3.1
+// step 4); the flushing thread drives GPU 0 itself.  A flush posts its plan with a new
+// generation number and waits until every worker has finished its GPU's part.
+struct Workers {
+    std::mutex mu;
+    std::condition_variable go, done;
+    uint64_t gen = 0;
+    int pending = 0;
+    bool stop = false;
+    Flush* f = nullptr;
+    std::vector<std::thread> th;
+    std::vector<svp_status> st;
+    std::vector<double> issue;
+};
+
 struct Executor {
     Ctx* c = nullptr;
     std::vector<Dev> devs;
+    Workers w;
     std::string err;
     std::mutex rmu;                          // submits validate from many threads
     std::map<uintptr_t, PtrRange> ranges;    // allocation start -> range (validate_ptrs 1)
@@ -117,6 +135,9 @@ struct Executor {
     };
     Hot hot[256];
 };
+
+static void start_workers(Executor* e);
+static void stop_workers(Executor* e);
 
 // the calling thread holds e->rmu through a RangeBatchLock
 static thread_local Executor* t_range_locked = nullptr;
@@ -213,12 +234,54 @@ Executor* executor_create(Ctx* c, svp_status* st) {
             return nullptr;
         }
     }
+    start_workers(e);
     *st = SVP_OK;
     return e;
 }
 
+static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns);
+
+static void worker_loop(Executor* e, int g) {
+    Workers& w = e->w;
+    uint64_t seen = 0;
+    for (;;) {
+        Flush* f = nullptr;
+        {
+            std::unique_lock<std::mutex> lk(w.mu);
+            w.go.wait(lk, [&] { return w.stop || w.gen != seen; });
+            if (w.stop) return;
+            seen = w.gen;
+            f = w.f;
+        }
+        double issue = 0;
+        const svp_status st = run_device(e, e->devs[g], *f, &issue);
+        std::lock_guard<std::mutex> lk(w.mu);
+        w.st[g] = st;
+        w.issue[g] = issue;
+        if (--w.pending == 0) w.done.notify_one();
+    }
+}
+
+static void start_workers(Executor* e) {
+    const int G = (int)e->devs.size();
+    e->w.st.assign(G, SVP_OK);
+    e->w.issue.assign(G, 0.0);
+    for (int g = 1; g < G; ++g) e->w.th.emplace_back(worker_loop, e, g);
+}
+
+static void stop_workers(Executor* e) {
+    {
+        std::lock_guard<std::mutex> lk(e->w.mu);
+        e->w.stop = true;
+    }
+    e->w.go.notify_all();
+    for (auto& t : e->w.th) t.join();
+    e->w.th.clear();
+}
+
 void executor_destroy(Executor* e) {
     if (!e) return;
+    stop_workers(e);
     for (auto& d : e->devs) dev_teardown(d);
     delete e;
 }
@@ -489,6 +552,10 @@ static svp_status plan_sgemm_tail(Executor* e, Dev& d, Flush& f, Chunk& ch, std:
             g.beta = 0.f;
             g.tile_begin = (uint32_t)pd.size();
             g.tiles_n = 1;
+            g.A = A + (size_t)sb.m0 * j.K + k0;  // the slice's operand views (exact-recompute path)
+            g.B = B + (size_t)k0 * j.N + sb.n0;
+            g.lda = j.K;
+            g.ldb = j.N;
             pd.push_back(g);
             alignas(64) uint8_t m[256];  // CUtensorMap is 64-B aligned
             if (encode_gemm_maps_view(m, m + 128, A + (size_t)sb.m0 * j.K + k0, B + (size_t)k0 * j.N + sb.n0, sb.rows,
@@ -634,6 +701,10 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
                 g.beta = j.f1;
                 g.tile_begin = tiles;
                 g.tiles_n = (uint32_t)((j.N + BN - 1) / BN);
+                g.A = A;
+                g.B = B;
+                g.lda = j.K;
+                g.ldb = j.N;
                 uint64_t nt = (uint64_t)((j.M + BM - 1) / BM) * g.tiles_n;
                 if ((int64_t)j.M * j.N == 0) nt = 0;
                 tiles += (uint32_t)nt;
@@ -1129,6 +1200,9 @@ static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool u
         (void)lastop;
         std::lock_guard<std::mutex> lk(c->pmu);
         c->fstats.device_ns = std::max(c->fstats.device_ns, (double)span * 1e6);
+        DevStats& ds = c->dstats[d.idx];
+        ds.last_device_ns = (double)span * 1e6;
+        ds.device_ns += (double)span * 1e6;
     }
     // ---- profile_level 2: measured busy cycles per segment (the kernels are done)
     size_t nbusy = 0;
@@ -1148,12 +1222,26 @@ static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool u
 // in the op -- or, with profile_level 2, the SM cycles measured on the VP's tiles of a
 // segment launch; T_v = T_op * w_v / sum w.  Conservation (sum_v T_v = T_op) holds exactly up
 // to fp64 rounding.
+static void count_device_work(Ctx* c, const Flush& f) {  // under pmu
+    std::vector<char> used(c->dstats.size(), 0);
+    for (const auto& j : f.jobs) {
+        if (j.device < 0 || j.device >= (int32_t)c->dstats.size()) continue;
+        c->dstats[j.device].jobs += 1;
+        used[j.device] = 1;
+    }
+    for (size_t g = 0; g < used.size(); ++g) c->dstats[g].flushes += used[g];
+}
+
 static void attribute(Ctx* c, const Flush& f) {
     std::lock_guard<std::mutex> lk(c->pmu);
+    count_device_work(c, f);
     for (const auto& j : f.jobs) {
         c->prof[j.vp].jobs += 1;
         c->prof_total.jobs += 1;
     }
+    for (const auto& o : f.ops)
+        if (o.kind == SVP_OP_KERNEL && o.measured_ns >= 0 && o.device < (int32_t)c->dstats.size())
+            c->dstats[o.device].kernel_ns += o.measured_ns;
     for (const auto& o : f.ops) {
         const Chunk& ch = f.chunks[o.chunk];
         if (o.kind == SVP_OP_KERNEL && o.measured_ns >= 0) {
@@ -1224,14 +1312,29 @@ svp_status executor_run(Executor* e, Flush* f) {
     std::vector<double> issue(G, 0.0);
     // pre-size the dependency-event pools (event creation is not thread-safe per device
     // pool vector growth, but each worker owns its Dev)
-    if (G == 1) {
-        st[0] = run_device(e, e->devs[0], *f, &issue[0]);
-    } else {
-        std::vector<std::thread> th;
-        for (int g = 0; g < G; ++g)
-            th.emplace_back([&, g] { st[g] = run_device(e, e->devs[g], *f, &issue[g]); });
-        for (auto& t : th) t.join();
+    // the flushing thread drives GPU 0 and gets its current device back afterwards
+    int caller_dev = -1;
+    if (cudaGetDevice(&caller_dev) != cudaSuccess) {
+        cudaGetLastError();
+        caller_dev = -1;
     }
+    if (G > 1) {
+        std::lock_guard<std::mutex> lk(e->w.mu);
+        e->w.f = f;
+        e->w.pending = G - 1;
+        e->w.gen += 1;
+    }
+    if (G > 1) e->w.go.notify_all();
+    st[0] = run_device(e, e->devs[0], *f, &issue[0]);
+    if (G > 1) {
+        std::unique_lock<std::mutex> lk(e->w.mu);
+        e->w.done.wait(lk, [&] { return e->w.pending == 0; });
+        for (int g = 1; g < G; ++g) {
+            st[g] = e->w.st[g];
+            issue[g] = e->w.issue[g];
+        }
+    }
+    if (caller_dev >= 0) cudaSetDevice(caller_dev);
     c->fstats.host_issue_ns = *std::max_element(issue.begin(), issue.end());
     for (int g = 0; g < G; ++g) {
         if (st[g] != SVP_OK) {
@@ -1242,6 +1345,7 @@ svp_status executor_run(Executor* e, Flush* f) {
     if (c->cfg.profile_level >= 1) attribute(c, *f);
     else {
         std::lock_guard<std::mutex> lk(c->pmu);
+        count_device_work(c, *f);
         for (const auto& j : f->jobs) {
             c->prof[j.vp].jobs += 1;
             c->prof_total.jobs += 1;

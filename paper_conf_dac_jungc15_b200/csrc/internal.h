@@ -164,6 +164,12 @@ struct KStats {
     double total_ns = 0, bytes = 0, flops = 0, max_ns = 0;
 };
 
+// per-GPU Profiler accumulators (svp_device_stats_get), under Ctx::pmu
+struct DevStats {
+    uint64_t flushes = 0, jobs = 0;
+    double device_ns = 0, kernel_ns = 0, last_device_ns = 0;
+};
+
 // ------------------------------------------------------------------ cost model (D8)
 struct CostModel {
     double hbm_Bps = 6552e9;
@@ -215,8 +221,15 @@ struct Ctx {
     bool disp_stop = false;
     int64_t disp_window_us = 0;
     int32_t disp_max_jobs = 0;
-    int32_t sticky = 0;              // SVP_OK or first fatal status
+    // SVP_OK or the first fatal status.  Read lock-free by every entry point; written once
+    // (with sticky_msg) under done_mu before waiters are notified.  sticky_msg is read
+    // only through sticky_message() (done_mu), never while it is being assigned.
+    std::atomic<int32_t> sticky{0};
     std::string sticky_msg;
+    std::string sticky_message() {
+        std::lock_guard<std::mutex> lk(done_mu);
+        return sticky_msg;
+    }
     bool registered[K_COUNT] = {};
 
     // last flush
@@ -232,6 +245,7 @@ struct Ctx {
     VpProfile prof_total;
     uint64_t prof_launches = 0;
     KStats kstats[K_COUNT];
+    std::vector<DevStats> dstats;    // [ngpu]
 
     Executor* exec = nullptr;        // null in dry_run
     bool coschedule = false;         // SVP_COSCHEDULE=1: memory-first small-grid co-residency

@@ -280,10 +280,13 @@ __device__ __forceinline__ float4 lo_part4(float4 x) {
     return make_float4(lo_part(x.x), lo_part(x.y), lo_part(x.z), lo_part(x.w));
 }
 
-// bf16x2 of (a -> low half, b -> high half), round to nearest even
+// bf16x2 of (a -> low half, b -> high half), round to nearest even; .satfinite (free in
+// SASS: F2FP.SATFINITE): a finite TF32 head beyond the bf16 range (|h| >= (2 - 2^-8) 2^127)
+// becomes +-max_bf16 instead of +-Inf, so a finite operand near FLT_MAX cannot turn a cross
+// term into an infinity (R20)
 __device__ __forceinline__ uint32_t bf2(float a, float b) {
     uint32_t r;
-    asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
+    asm("cvt.rn.satfinite.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
     return r;
 }
 
@@ -291,7 +294,8 @@ __device__ __forceinline__ uint32_t bf2(float a, float b) {
 // back over the raw tile the TF32 MMA reads; the cross terms get bf16(h) and bf16(x - h).
 // (A truncated head -- what the tensor core reads from an untouched tile -- leaves |l| up to
 // 2^-10 |x| and a worst-case product error of 2^-16 + 2^-20 > 1e-5: tests/split_emulation.py.)
-// |x| within 2^-12 of FLT_MAX would round to inf; the guest data never gets there.
+// |x| within 2^-12 of FLT_MAX rounds to inf (then l = -inf): the epilogue's exact recompute
+// of NaN outputs covers it (R20).
 __device__ __forceinline__ float rna_tf32(float x) {
     return __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
 }
@@ -313,6 +317,23 @@ __device__ __forceinline__ void split8_given(const float4& p, const float4& q, c
 }
 
 }  // namespace tc
+
+// One output of C = alpha A B + beta C_old exactly as the definition reads it (PAPER.md
+// Table 1's matmul at BASELINE.json's fp32; R20): products in fp64 (exact for fp32
+// operands), summed in ascending k in fp64 with IEEE +/x (no contraction), alpha * acc +
+// beta * c_old in fp64, one rounding.  The rare path of the tensor-core epilogue for outputs
+// whose accumulator came out NaN -- an Inf or NaN operand, or a finite one at the top of the
+// fp32 range -- so their Inf / NaN / finite value is the IEEE one.
+__device__ __noinline__ float exact_element(const GemmDesc& g, int i, int j, float c_old) {
+    const float* a = g.A + (size_t)i * g.lda;
+    const float* b = g.B + j;
+    double acc = 0.0;
+    for (int k = 0; k < g.K; ++k)
+        acc = __dadd_rn(acc, __dmul_rn((double)__ldg(a + k), (double)__ldg(b + (size_t)k * g.ldb)));
+    double r = __dmul_rn((double)g.alpha, acc);
+    if (g.beta != 0.f) r = __dadd_rn(r, __dmul_rn((double)g.beta, (double)c_old));
+    return (float)r;
+}
 
 template <int SPLIT, int CG, int NH>
 __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
@@ -646,6 +667,7 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                 tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0), r);
                 const int col0 = tn * TN + eh * BN + c0;
                 if (!row_ok) continue;
+                uint32_t nan_mask = 0;  // outputs of this chunk whose accumulator is NaN
 #pragma unroll
                 for (int j = 0; j < 32; j += 4) {
                     const int c = col0 + j;
@@ -656,14 +678,33 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     o.z = kzero ? 0.f : alpha * __uint_as_float(r[j + 2]);
                     o.w = kzero ? 0.f : alpha * __uint_as_float(r[j + 3]);
                     float4* dst = reinterpret_cast<float4*>(crow + c);
+                    float4 old = make_float4(0.f, 0.f, 0.f, 0.f);
                     if (beta != 0.f) {
-                        const float4 old = __ldcs(dst);
+                        old = __ldcs(dst);
                         o.x = __fmaf_rn(beta, old.x, o.x);
                         o.y = __fmaf_rn(beta, old.y, o.y);
                         o.z = __fmaf_rn(beta, old.z, o.z);
                         o.w = __fmaf_rn(beta, old.w, o.w);
                     }
+                    // IEEE special values (R20): an Inf / NaN operand (its low part x - h is NaN),
+                    // or a finite one whose TF32 head rounds past FLT_MAX, leaves NaN in every
+                    // accumulator it reaches.  Those outputs keep C_old for now and are
+                    // recomputed exactly below (rare path, after r[] is dead).
+                    const float acc4 = __uint_as_float(r[j]) + __uint_as_float(r[j + 1]) +
+                                       __uint_as_float(r[j + 2]) + __uint_as_float(r[j + 3]);
+                    if (!kzero && acc4 != acc4) {
+                        if (isnan(__uint_as_float(r[j + 0]))) { nan_mask |= 1u << (j + 0); o.x = old.x; }
+                        if (isnan(__uint_as_float(r[j + 1]))) { nan_mask |= 1u << (j + 1); o.y = old.y; }
+                        if (isnan(__uint_as_float(r[j + 2]))) { nan_mask |= 1u << (j + 2); o.z = old.z; }
+                        if (isnan(__uint_as_float(r[j + 3]))) { nan_mask |= 1u << (j + 3); o.w = old.w; }
+                    }
                     __stcs(dst, o);  // st.global.cs: C is written once
+                }
+                while (nan_mask) {
+                    const int e = __ffs(nan_mask) - 1;
+                    nan_mask &= nan_mask - 1;
+                    float* cp = crow + col0 + e;
+                    *cp = exact_element(g, row, col0 + e, beta != 0.f ? *cp : 0.f);
                 }
             }
             tc_fence_before();

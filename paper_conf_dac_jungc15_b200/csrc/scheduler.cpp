@@ -507,21 +507,33 @@ svp_status plan_flush(Ctx* c, Flush* f) {
             const int32_t lo = vp_last_op[f->jobs[ji].vp];
             if (lo >= 0) prev.push_back(lo);
         }
-        // arena slot (ring) -- waits for the ops that release overlapped regions
+        // arena slot (ring) -- the chunk's first arena op waits for the release (last op) of
+        // every in-flight slot overlapping [off, off + len).  The part of an old slot this
+        // chunk covers is then guarded by this chunk's own release (which follows its first
+        // op, which waited); the parts it does NOT cover keep the old slot's release, so a
+        // later chunk placed there still waits for it (dropping the whole slot here let such
+        // a chunk -- e.g. one whose first op is its kernel, not an H2D on the shared copy
+        // stream -- overwrite staging another chunk was still using).
         std::vector<int32_t> arena_waits;
         if (ch.arena_len) {
             uint64_t off = arena_head[dev];
             if (off + ch.arena_len > arena) off = 0;
+            const uint64_t lo = off, hi = off + ch.arena_len;
             auto& fl = inflight[dev];
-            for (size_t k = 0; k < fl.size();) {
-                bool overlap = fl[k].off < off + ch.arena_len && off < fl[k].off + fl[k].len;
-                if (overlap) {
-                    arena_waits.push_back(fl[k].release_op);
-                    fl.erase(fl.begin() + k);
+            std::vector<Slot> keep;
+            keep.reserve(fl.size() + 2);
+            for (const Slot& s : fl) {
+                const uint64_t se = s.off + s.len;
+                if (s.off < hi && lo < se) {
+                    if (std::find(arena_waits.begin(), arena_waits.end(), s.release_op) == arena_waits.end())
+                        arena_waits.push_back(s.release_op);
+                    if (s.off < lo) keep.push_back(Slot{s.off, lo - s.off, s.release_op});
+                    if (se > hi) keep.push_back(Slot{hi, se - hi, s.release_op});
                 } else {
-                    ++k;
+                    keep.push_back(s);
                 }
             }
+            fl.swap(keep);
             ch.arena_off = off;
             arena_head[dev] = off + ch.arena_len;
         }

@@ -81,7 +81,12 @@ struct GemmDesc {
     float alpha, beta;
     uint32_t tile_begin;  // first output tile of this VP
     uint32_t tiles_n;     // tiles along N
-    uint32_t _pad[7];
+    uint32_t _pad0;
+    // plain operand pointers + row pitches (elements): the tensor-core kernels stream A and B
+    // through TMA maps and read these only on the rare exact-recompute path (R20)
+    const float* A;
+    const float* B;
+    int32_t lda, ldb;
 };
 static_assert(sizeof(GemmDesc) == 64, "GemmDesc must be 64 B");
 

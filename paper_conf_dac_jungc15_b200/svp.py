@@ -36,7 +36,8 @@ EXPORTS = ("svp_config_default", "svp_init", "svp_finalize", "svp_last_error", "
            "svp_assign_vps", "svp_lpt_partition", "svp_profile", "svp_reset_profile", "svp_kernel_stats_get",
            "svp_flush_stats_get", "svp_plan_size", "svp_plan_get", "svp_wait", "svp_start_dispatcher",
            "svp_stop_dispatcher", "svp_ipc_serve", "svp_ipc_server_stats", "svp_ipc_shutdown", "svp_ipc_connect",
-           "svp_ipc_disconnect", "svp_ipc_alloc", "svp_ipc_submit", "svp_ipc_wait", "svp_kernel_lookup")
+           "svp_ipc_disconnect", "svp_ipc_alloc", "svp_ipc_submit", "svp_ipc_wait", "svp_kernel_lookup",
+           "svp_plan_op_detail", "svp_device_stats_get")
 
 
 class svp_config(C.Structure):
@@ -80,6 +81,12 @@ class svp_flush_stats(C.Structure):
                [(n, C.c_double) for n in ("host_plan_ns", "host_issue_ns", "host_total_ns", "device_ns",
                                           "sim_makespan_ns", "sim_serial_ns")] + \
                [(n, C.c_uint64) for n in ("plan_reused", "graph_replays", "kernel_launches")]
+
+
+class svp_device_stats(C.Structure):
+    _fields_ = [("ordinal", C.c_int32), ("vps", C.c_int32), ("est_load_ns", C.c_double), ("flushes", C.c_uint64),
+                ("jobs", C.c_uint64), ("device_ns", C.c_double), ("kernel_ns", C.c_double),
+                ("last_device_ns", C.c_double)]
 
 
 class svp_plan_op(C.Structure):
@@ -150,6 +157,9 @@ def load(build_if_stale: bool = True):
                                      P(C.c_uint64)]
         L.svp_ipc_wait.argtypes = [vp, C.c_uint64, C.c_int32]
         L.svp_kernel_lookup.argtypes = [C.c_char_p, P(C.c_int32)]
+        L.svp_device_stats_get.argtypes = [vp, C.c_int32, P(svp_device_stats)]
+        L.svp_plan_op_detail.argtypes = [vp, C.c_int32, P(C.c_uint64), P(C.c_uint64), P(C.c_int32), C.c_int32,
+                                         P(C.c_int32)]
         for name in EXPORTS:
             f = getattr(L, name)
             if name not in ("svp_config_default", "svp_last_error", "svp_abi_version"):
@@ -353,6 +363,11 @@ class Context:
         _check(self._L.svp_kernel_stats_get(self._h, kernel, C.byref(s)))
         return {k: getattr(s, k) for k, _ in svp_kernel_stats._fields_}
 
+    def device_stats(self, g: int) -> Dict[str, float]:
+        s = svp_device_stats()
+        _check(self._L.svp_device_stats_get(self._h, g, C.byref(s)))
+        return {k: getattr(s, k) for k, _ in svp_device_stats._fields_}
+
     def flush_stats(self) -> Dict[str, float]:
         s = svp_flush_stats()
         _check(self._L.svp_flush_stats_get(self._h, C.byref(s)))
@@ -368,6 +383,11 @@ class Context:
             _check(self._L.svp_plan_get(self._h, i, C.byref(op), vps, 4096))
             d = {k: getattr(op, k) for k, _ in svp_plan_op._fields_}
             d["vps"] = list(vps[: min(op.nvps, 4096)])
+            aoff, alen, nw = C.c_uint64(), C.c_uint64(), C.c_int32()
+            waits = (C.c_int32 * 256)()
+            _check(self._L.svp_plan_op_detail(self._h, i, C.byref(aoff), C.byref(alen), waits, 256, C.byref(nw)))
+            d["arena_off"], d["arena_len"] = aoff.value, alen.value
+            d["waits"] = list(waits[: min(nw.value, 256)])
             out.append(d)
         return out
 

@@ -84,7 +84,8 @@ def check_job(spec, inp, got, want=None, sgemm_tol=SGEMM_TOL, sample=None):
             scale += np.abs(spec.beta * inp["C"].astype(np.float64))
         err = np.abs(G - O)
         assert (err <= sgemm_tol * scale + 1e-30).all(), (spec.vp, float((err / (scale + 1e-30)).max()))
-        assert np.linalg.norm(G - O) <= sgemm_tol * np.linalg.norm(O) + 1e-30
+        fro = np.linalg.norm(G - O) / (np.linalg.norm(O) + 1e-30)
+        assert fro <= sgemm_tol, (spec.vp, "relative Frobenius error", fro)
     else:
         raise ValueError(k)
 

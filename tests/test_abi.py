@@ -23,7 +23,7 @@ def test_library_exports_every_declared_symbol():
     assert set(declared) == set(svp.EXPORTS), (set(declared) ^ set(svp.EXPORTS))
     for name in declared:
         assert hasattr(L, name), name
-    assert L.svp_abi_version() == 4
+    assert L.svp_abi_version() == 5
 
 
 @pytest.mark.skipif(bool(os.environ.get("SVP_LIB")), reason="SVP_LIB selects a sanitizer build on purpose")

@@ -23,6 +23,18 @@ MODES = {
 
 
 @pytest.fixture(scope="module")
+def cfg5_sgemm_oracle():
+    """cfg5 inputs and the oracle's full products of 4 of its 51 SGEMM 2048^3 VPs (first,
+    last, two middle; one VP per host thread, ~10 s)."""
+    specs = W.config_specs(5)
+    inputs = W.make_inputs_many(specs)
+    sg = [i for i, s in enumerate(specs) if s.kernel == "sgemm"]
+    pick = [sg[0], sg[len(sg) // 3], sg[2 * len(sg) // 3], sg[-1]]
+    want = oracle.run_jobs([specs[i] for i in pick], [inputs[i] for i in pick], threads=4)
+    return specs, inputs, pick, want
+
+
+@pytest.fixture(scope="module")
 def small():
     specs = W.mixed_small(nvps=30, max_n=70000)
     return specs, inputs_for(specs)
@@ -520,6 +532,35 @@ def test_config5_bench_launch_config():
             for i, s in enumerate(specs):  # the next step's SAXPY reads this step's y
                 if s.kernel == "saxpy":
                     prev[i] = dict(prev[i], y=outs[i]["y"].copy())
+        assert vs.guards_intact()
+    finally:
+        ctx.close()
+
+
+@pytest.mark.parametrize("impl", [svp.SGEMM_TF32BF16, svp.SGEMM_FFMA, svp.SGEMM_3XTF32])
+def test_config5_sgemm_full_elementwise(impl, cfg5_sgemm_oracle):
+    """the SGEMM bench.py times, at its benched shape and launch
+    configuration (cfg5's 256 VPs in one interleaved flush, 51 SGEMM 2048^3 VPs in one
+    coalesced launch -- wide 256 x 512 CTA-pair tiles for the default TF32+2xBF16 split;
+    the FFMA and 3xTF32 implementations are the ones bench.py times beside it), compared
+    ELEMENT BY ELEMENT against oracle.sgemm for the first, last and two middle SGEMM VPs
+    (4 x 4.2 M outputs), on the second (steady-state) step."""
+    specs, inputs, pick, want = cfg5_sgemm_oracle
+    stream = torch.cuda.current_stream()
+    ctx = svp.Context(num_gpus=1, device_ids=[0], profile_level=1, external_streams=[stream.cuda_stream],
+                      validate_ptrs=True, sgemm_impl=impl, table_mode=svp.TABLE_PARAM)
+    try:
+        vs = VPSet(ctx, specs, inputs, "device", device_ordinals=[0])
+        jobs = svp.JobBatch(vs.job_list())
+        for _ in range(2):
+            ctx.submit_batch(jobs)
+            ctx.flush()
+        torch.cuda.synchronize()
+        st = ctx.flush_stats()
+        assert st["groups"] == 5, st
+        for i, w in zip(pick, want):
+            got = vs.output(i)
+            check_job(specs[i], inputs[i], got, w)
         assert vs.guards_intact()
     finally:
         ctx.close()

@@ -58,12 +58,17 @@ def test_tc_ragged_alpha_beta(kernel, impl, tol, residency):
 
 @pytest.mark.parametrize("impl", TC_FP32)
 def test_3xtf32_2048_sampled(impl):
-    """Full BASELINE cfg5 SGEMM shape (2048^3), 4 VPs coalesced, 64 sampled outputs each."""
+    """Full BASELINE cfg5 SGEMM shape (2048^3), 4 VPs coalesced: VPs 0 and 3 compared element
+    by element with the oracle's full product, VPs 1 and 2 on 64 sampled outputs each."""
     specs = [W.JobSpec(v, "sgemm", M=2048, N=2048, K=2048) for v in range(4)]
     inputs = inputs_for(specs)
     outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl)
+    full = oracle.run_jobs([specs[0], specs[3]], [inputs[0], inputs[3]], threads=2)
     g = np.random.default_rng(1)
     for s, inp, got in zip(specs, inputs, outs):
+        if s.vp in (0, 3):
+            check_job(s, inp, got, full[0 if s.vp == 0 else 1])
+            continue
         sample = [(int(g.integers(0, 2048)), int(g.integers(0, 2048))) for _ in range(64)]
         sample += [(0, 0), (2047, 2047), (127, 255), (128, 256)]
         check_job(s, inp, got, sample=sample)
@@ -98,7 +103,9 @@ def test_kernel_variants_in_subprocess(env):
     import sys
     here = os.path.dirname(os.path.abspath(__file__))
     cmd = [sys.executable, "-m", "pytest", os.path.join(here, "test_gpu_sgemm_tc.py"), "-q", "-m", "gpu",
-           "-p", "no:cacheprovider", "-k", "(fp32_tolerance or ragged_alpha_beta or wide_dynamic or 2048_sampled) and not variants"]
+           "-p", "no:cacheprovider", "-k", "(fp32_tolerance or ragged_alpha_beta or wide_dynamic or 2048_sampled or ieee) and not variants"]
+    if env.get("SVP_TC_WIDE") == "2" or env.get("SVP_TC_TMEM_A") == "1" or env.get("SVP_TC_CTA_PAIR") == "0":
+        cmd += [os.path.join(here, "test_gpu_sgemm_ieee.py")]  # the IEEE edge values on this variant too
     r = subprocess.run(cmd, env={**os.environ, **env}, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
 

@@ -175,6 +175,42 @@ def test_sgemm_random_near_exact():
         assert oracle.sgemm_element(A, B, i, j) == C[i, j]
 
 
+def test_sgemm_element_alpha_beta_against_int64_closed_form():
+    """oracle_sgemm_element's beta / c_old branch (the checker of every full-size sampled
+    GEMM output) against the int64 closed form alpha * sum_k a_ik b_kj + beta * c_old, with
+    integer operands small enough that every value is exact in fp32 -- a dropped beta term,
+    a sign slip or a transposed index fails it.  beta == 0 must not read c_old (BLAS: C is
+    not an input then), so a NaN c_old is ignored."""
+    g = np.random.default_rng(17)
+    M, N, K = 37, 53, 61
+    A = g.integers(-8, 9, (M, K)).astype(np.float32)
+    B = g.integers(-8, 9, (K, N)).astype(np.float32)
+    Cold = g.integers(-100, 101, (M, N)).astype(np.float32)
+    exact = A.astype(np.int64) @ B.astype(np.int64)
+    for alpha, beta in [(1.0, 0.0), (2.0, -3.0), (-1.0, 0.5), (0.0, 1.0), (3.0, 2.0)]:
+        for (i, j) in [(0, 0), (M - 1, N - 1), (5, 17), (36, 0), (0, 52)]:
+            want = alpha * float(exact[i, j]) + (beta * float(Cold[i, j]) if beta else 0.0)
+            got = oracle.sgemm_element(A, B, i, j, alpha, beta, float(Cold[i, j]))
+            assert got == want, (alpha, beta, i, j, got, want)
+            assert oracle.sgemm_element(A, B, i, j, alpha, beta, float(Cold[i, j])) == \
+                oracle.sgemm(A, B, Cold, alpha, beta)[i, j]
+    assert oracle.sgemm_element(A, B, 3, 4, 1.0, 0.0, float("nan")) == float(exact[3, 4])
+
+
+def test_sgemm_ieee_special_values():
+    """The oracle's own IEEE behaviour (R20): Inf*0 = NaN, Inf*x = +-Inf, Inf*Inf = Inf,
+    Inf + -Inf = NaN, a NaN operand poisons its row, subnormal operands are exact (fp64)."""
+    A = np.array([[np.inf, 1.0], [np.inf, -1.0], [np.nan, 0.0], [2.0 ** -140, 0.0]], np.float32)
+    B = np.array([[0.0, 2.0, np.inf], [1.0, 1.0, np.inf]], np.float32)
+    C = oracle.sgemm(A, B)
+    assert np.isnan(C[0, 0])                      # Inf*0 + 1*1
+    assert C[0, 1] == np.inf                      # Inf*2 + 1
+    assert C[0, 2] == np.inf                      # Inf*Inf + Inf
+    assert np.isnan(C[1, 2])                      # Inf*Inf + (-1)*Inf
+    assert np.isnan(C[2]).all()                   # NaN row
+    assert C[3, 1] == np.float32(2.0 ** -139)     # subnormal * 2, exact
+
+
 # ------------------------------------------------------------------ job runner
 def test_run_jobs_independent_per_vp():
     specs = W.mixed_small(nvps=10, max_n=5000)
