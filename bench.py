@@ -494,7 +494,7 @@ def run_svp(args, rank, ws, local):
     per_gpu_rows = []
     for g, (d, t) in enumerate(zip(dstats, dt_per_gpu)):
         per_gpu_rows.append({"gpu": g, "ordinal": d["ordinal"], "vps": d["vps"],
-                             "lpt_est_load_ms": d["est_load_ns"] / 1e6,
+                             "lpt_est_load_ms": d["est_load_ns"] / 1e6,  # VPSet's estimated kernel ns
                              "device_ms_per_step": d["device_ns"] / args.steps / 1e6,
                              "kernel_ms_per_step": d["kernel_ns"] / args.steps / 1e6,
                              "event_ms_per_step": t / args.steps * 1e3})

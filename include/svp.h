@@ -381,10 +381,13 @@ svp_status svp_plan_get(svp_ctx* ctx, int32_t i, svp_plan_op* op, int32_t* vps_o
 /* (ABI 5) Ordering detail of plan op i: *arena_off / *arena_len = the staging-arena byte
  * range its chunk uses (len 0: nothing staged), *nwaits = how many earlier ops it waits on
  * through events (cross-stream waits; ops on the same (device, stream) are ordered by
- * issue order and are not listed), and waits_out[0 .. min(nwaits, cap)) their plan indices.
- * Any pointer may be NULL.  Errors: SVP_E_INVAL (null ctx, index out of range). */
+ * issue order and are not listed), waits_out[0 .. min(nwaits, cap)) their plan indices, and
+ * *measured_start_ns = when the op started on its GPU, event-timed from the start of that
+ * GPU's first op of the flush (profile_level >= 1; -1 otherwise) -- with measured_ns of
+ * svp_plan_get, the flush's measured timeline.  Any pointer may be NULL.
+ * Errors: SVP_E_INVAL (null ctx, index out of range). */
 svp_status svp_plan_op_detail(svp_ctx* ctx, int32_t i, uint64_t* arena_off, uint64_t* arena_len,
-                              int32_t* waits_out, int32_t cap, int32_t* nwaits);
+                              int32_t* waits_out, int32_t cap, int32_t* nwaits, double* measured_start_ns);
 
 #ifdef __cplusplus
 }

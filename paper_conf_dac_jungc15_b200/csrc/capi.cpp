@@ -320,7 +320,7 @@ static svp_status do_flush(Ctx* c) {
         f.groups = c->last.groups;
         f.chunks = c->last.chunks;
         f.ops = c->last.ops;
-        for (auto& o : f.ops) o.measured_ns = -1;
+        for (auto& o : f.ops) o.measured_ns = o.measured_start_ns = -1;
         f.levels = c->last.levels;
         f.plan_gen = c->last.plan_gen;
         f.reused = true;
@@ -711,7 +711,7 @@ svp_status svp_plan_get(svp_ctx* h, int32_t i, svp_plan_op* op, int32_t* vps_out
 }
 
 svp_status svp_plan_op_detail(svp_ctx* h, int32_t i, uint64_t* arena_off, uint64_t* arena_len, int32_t* waits_out,
-                              int32_t cap, int32_t* nwaits) {
+                              int32_t cap, int32_t* nwaits, double* measured_start_ns) {
     if (!h) {
         set_error("null context");
         return SVP_E_INVAL;
@@ -726,6 +726,7 @@ svp_status svp_plan_op_detail(svp_ctx* h, int32_t i, uint64_t* arena_off, uint64
     if (arena_off) *arena_off = ch.arena_off;
     if (arena_len) *arena_len = ch.arena_len;
     if (nwaits) *nwaits = (int32_t)o.wait_ops.size();
+    if (measured_start_ns) *measured_start_ns = o.measured_start_ns;
     if (waits_out)
         for (int k = 0; k < (int)o.wait_ops.size() && k < cap; ++k) waits_out[k] = o.wait_ops[k];
     return SVP_OK;

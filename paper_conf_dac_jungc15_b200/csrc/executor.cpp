@@ -664,12 +664,13 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             ch.kernel_launches = ch.kernel == K_HIST256 && !hist_single_launch() && tiles > 0 ? 2 : 1;
         } else {
             // tcgen05 tiles for sgemm_tf32 and for sgemm with the 3xTF32 implementation
-            const int variant = (ch.kernel == K_SGEMM_TF32 || e->c->cfg.sgemm_impl != SVP_SGEMM_FFMA) ? 1 : 0;
+            const bool plain = ch.sgemm_impl == kSgemmPlain;
+            const int variant = !plain && (ch.kernel == K_SGEMM_TF32 || ch.sgemm_impl != SVP_SGEMM_FFMA) ? 1 : 0;
             const bool pair = variant && ch.kernel == K_SGEMM && sgemm_tc_cta_pair();
             // wide (256 x 512) pair tiles halve the A-side conversion and L2 traffic per flop
             // but halve the tile count: used when they still fill >= 2 waves of CTA pairs
             bool wide = false;
-            if (pair && e->c->cfg.sgemm_impl == SVP_SGEMM_TF32BF16) {
+            if (pair && ch.sgemm_impl == SVP_SGEMM_TF32BF16) {
                 const int mode = sgemm_tc_wide_mode();
                 uint64_t tw = 0;
                 for (int32_t ji : ch.jobs) {
@@ -680,8 +681,8 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
                 wide = mode == 2 || (mode == 1 && tw >= 2ull * (uint64_t)(d.lim.num_sms / 2));
             }
             ch.wide = wide;
-            const int BM = variant ? (pair ? 2 * kTf32BM : kTf32BM) : kGemmBM;
-            const int BN = variant ? (wide ? 2 * kTf32BN : kTf32BN) : kGemmBN;
+            const int BM = plain ? kSgemmPlainTile : variant ? (pair ? 2 * kTf32BM : kTf32BM) : kGemmBM;
+            const int BN = plain ? kSgemmPlainTile : variant ? (wide ? 2 * kTf32BN : kTf32BN) : kGemmBN;
             ch.maps_off = align_up(tbl.size(), 128);
             size_t nj = ch.jobs.size();
             ch.table_off = ch.maps_off + nj * 256;
@@ -709,7 +710,7 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
                 if ((int64_t)j.M * j.N == 0) nt = 0;
                 tiles += (uint32_t)nt;
                 uint8_t* mp = tbl.data() + ch.maps_off + k * 256;
-                if (nt && j.K > 0) {
+                if (nt && j.K > 0 && !plain) {
                     MapKey key{(uint64_t)A, (uint64_t)B, j.M, j.N, j.K, variant};
                     auto it = d.map_cache.find(key);
                     if (it == d.map_cache.end()) {
@@ -738,7 +739,7 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             // not idle GPU time, and the power-capped step measured 0.7-2 % slower with the
             // extra slice pass (profiles/r01/sgemm_tail/)
             const bool alone = !e->c->cfg.interleave || chunks_in_level[ch.level] == 1;
-            if (alone && ch.kernel == K_SGEMM && e->c->cfg.sgemm_impl == SVP_SGEMM_TF32BF16) {
+            if (alone && ch.kernel == K_SGEMM && ch.sgemm_impl == SVP_SGEMM_TF32BF16) {
                 const int P = (int)std::min<uint64_t>(tiles, (uint64_t)d.lim.num_sms / 2);
                 svp_status st = plan_sgemm_tail(e, d, f, ch, tbl, P);
                 if (st) return st;
@@ -759,7 +760,8 @@ static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bo
     return pool[i];
 }
 
-static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStream_t s) {
+static cudaError_t launch_chunk(Dev& d, const Chunk& ch, cudaStream_t s) {
+    const int sgemm_impl = ch.sgemm_impl;
     if (ch.total_tiles == 0 && ch.kernel != K_HIST256) return cudaSuccess;
     const uint8_t* base = d.tbl_dev;
     uint64_t* busy = ch.busy_off >= 0 ? d.busy_dev + ch.busy_off : nullptr;
@@ -805,6 +807,9 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
             return launch_hist256((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
                                   grid_of(d.lim.hist_blocks_per_sm), s, busy, hscr);
         case K_SGEMM:
+            if (sgemm_impl == kSgemmPlain)
+                return launch_sgemm_plain((const GemmDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
+                                          grid_of(d.lim.gemm_plain_blocks_per_sm), s);
             if (sgemm_impl == SVP_SGEMM_TF32BF16) {
                 cudaError_t e = launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.table_off), ch.nsegs,
                                                       base + ch.maps_off, ch.main_tiles, grid_of(1), ch.wide, s);
@@ -826,6 +831,9 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int sgemm_impl, cudaStr
                                 grid_of(ch.small_tiles ? d.lim.dgemm_small_blocks_per_sm : d.lim.dgemm_blocks_per_sm),
                                 ch.small_tiles, s);
         case K_SGEMM_TF32:
+            if (sgemm_impl == kSgemmPlain)
+                return launch_sgemm_plain((const GemmDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
+                                          grid_of(d.lim.gemm_plain_blocks_per_sm), s);
             return launch_sgemm_tf32((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
                                      ch.total_tiles, grid_of(1), s);
     }
@@ -1121,7 +1129,7 @@ static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool captu
                 }
             }
         } else if (chunk_needs_launch(f, ch)) {
-            CK(launch_chunk(d, ch, c->cfg.sgemm_impl, s));
+            CK(launch_chunk(d, ch, s));
         }
         if (prof) {
             CK(rec(d.t_ev[2 * nt + 1], s));
@@ -1191,8 +1199,10 @@ static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool u
             float mx = 0;
             for (size_t i = 0; i < f.ops.size(); ++i) {
                 if (tstart[i] < 0) continue;
-                float ms = 0;
+                float ms = 0, ms0 = 0;
                 CK(cudaEventElapsedTime(&ms, d.t_ev[2 * tstart[first]], d.t_ev[2 * tstart[i] + 1]));
+                CK(cudaEventElapsedTime(&ms0, d.t_ev[2 * tstart[first]], d.t_ev[2 * tstart[i]]));
+                f.ops[i].measured_start_ns = (double)ms0 * 1e6;
                 mx = std::max(mx, ms);
             }
             span = mx;
@@ -1300,8 +1310,9 @@ static void attribute(Ctx* c, const Flush& f) {
         const Chunk& ch = f.chunks[o.chunk];
         double pred = o.est_ns - c->cost.launch_ns;
         double meas = std::max(1.0, o.measured_ns - c->cost.launch_ns);
-        double ratio = c->cost.kscale[ch.kernel] * meas / pred;
-        c->cost.kscale[ch.kernel] = 0.8 * c->cost.kscale[ch.kernel] + 0.2 * std::min(8.0, std::max(0.125, ratio));
+        double& ks = c->cost.kscale[ch.kernel][CostModel::bucket(ch.alg_bytes, ch.flops)];
+        const double ratio = ks * meas / pred;
+        ks = 0.8 * ks + 0.2 * std::min(8.0, std::max(0.125, ratio));
     }
 }
 

@@ -4,6 +4,7 @@
 // Kernel Match, Job Dispatcher, Re-scheduler, cost model) -> executor.cpp (L2: per-GPU
 // streams/events/arena/tables, Profiler) -> kernels/*.cu (L0: sm_100a guest kernels).
 #pragma once
+#include <math.h>
 #include <stdint.h>
 
 #include <atomic>
@@ -42,6 +43,16 @@ struct KernelDesc {
 };
 const KernelDesc* kernel_desc(int32_t id);
 inline bool is_gemm(int32_t k) { return k == K_SGEMM || k == K_SGEMM_TF32 || k == K_DGEMM; }
+// Largest K an "sgemm" job runs with on the tensor-core split implementations (R23):
+// the tcgen05 fp32 accumulation loses magnitude (measured -1.66e-8 relative per accumulating
+// MMA, profiles/r02/accuracy_k.jsonl), so the output's relative error grows with K; up to
+// these K every measured output keeps the 1e-5 fp32 contract.  Jobs with larger K match as a
+// separate group that runs the FFMA kernel.
+// internal "sgemm_impl" of a group whose jobs TMA cannot address (k_sgemm_plain)
+constexpr int32_t kSgemmPlain = 3;
+inline int32_t sgemm_tc_kmax(int32_t impl) {
+    return impl == SVP_SGEMM_TF32BF16 ? 2048 : impl == SVP_SGEMM_3XTF32 ? 1024 : (1 << 30);
+}
 // kernels the heterogeneous launch can carry: same CTA shape (256 threads, no shared
 // memory) and the same SegDesc tile mapping
 inline bool is_ew(int32_t k) { return k == K_VECADD || k == K_SAXPY || k == K_BLACKSCHOLES; }
@@ -114,6 +125,7 @@ struct Chunk {
     uint64_t tail_maps_off = 0, tail_table_off = 0, tail_red_off = 0;
     // kernel launches this op issues (hist256 zeroing kernel, tail split: 3)
     int32_t kernel_launches = 1;
+    int32_t sgemm_impl = -1;        // K_SGEMM: the implementation this launch runs (R23)
 };
 
 struct Op {
@@ -126,6 +138,7 @@ struct Op {
     double est_ns = 0;
     double sim_start = 0, sim_end = 0;
     double measured_ns = -1;
+    double measured_start_ns = -1;  // from the start of this GPU's first op of the flush
     uint64_t bytes = 0;
     double flops = 0;
     bool last_of_job = false;       // serial baseline: sync after this op
@@ -180,10 +193,25 @@ struct CostModel {
     int sgemm_tc_units = 0;          // "sgemm" on tensor cores: TF32-MMA-equivalents per
                                      // product (3xTF32: 3, TF32+2xBF16: 2); 0 = FFMA
     double copy_ns = 2000;           // per-copy fixed overhead
-    // EMA of measured/predicted ratio per kernel (learned from the profiler)
     double fp64_flops = 30e12;
-    double kscale[K_COUNT] = {1, 1, 1, 1, 1, 1, 1, 1, 1};
+    // EMA of measured / predicted kernel time per (kernel, size bucket), learned
+    // from the Profiler: a 64 Ki-element launch and a 16 Mi-element one of the same kernel sit
+    // at different points of Eq 9's T_o + T_e ceil(xi / lambda), so one factor per kernel
+    // would mix them.  Bucket = floor(log4(work)), work = FLOPs (GEMMs) or algorithmic bytes.
+    static constexpr int kBuckets = 32;
+    double kscale[K_COUNT][kBuckets];
+    CostModel() {
+        for (auto& row : kscale)
+            for (double& x : row) x = 1.0;
+    }
+    static int bucket(double alg_bytes, double flops) {
+        const double w = flops > 0 ? flops : alg_bytes;
+        const int b = w >= 1.0 ? (int)(0.5 * log2(w)) : 0;
+        return b < 0 ? 0 : (b >= kBuckets ? kBuckets - 1 : b);
+    }
     double kernel_ns(int32_t kernel, double alg_bytes, double flops) const;
+    // K_SGEMM on an explicit implementation (a group routed to FFMA, R23)
+    double sgemm_ns(int32_t impl, double alg_bytes, double flops) const;
     double h2d_ns(uint64_t bytes, int ncopies) const;
     double d2h_ns(uint64_t bytes, int ncopies) const;
 };

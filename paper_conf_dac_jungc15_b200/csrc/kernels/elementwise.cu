@@ -387,6 +387,9 @@ cudaError_t query_limits(LaunchLimits* out) {
     if (out->mix_blocks_per_sm < 1) out->mix_blocks_per_sm = 1;
     e = query_limits_hist(&out->hist_blocks_per_sm);
     if (e) return e;
+    e = query_limits_gemm_plain(&out->gemm_plain_blocks_per_sm);
+    if (e) return e;
+    if (out->gemm_plain_blocks_per_sm < 1) out->gemm_plain_blocks_per_sm = 1;
     e = query_limits_gemm(&out->gemm_blocks_per_sm);
     if (e) return e;
     e = query_limits_dgemm(&out->dgemm_blocks_per_sm, &out->dgemm_small_blocks_per_sm);

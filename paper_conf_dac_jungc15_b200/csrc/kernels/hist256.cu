@@ -11,9 +11,14 @@
 //    behind the consumers' atomics;
 //  * 8 consumer warps read the staged tile (LDS.128, conflict-free) and increment a CTA
 //    histogram replicated per lane -- h[bin][lane], 256 x 32 u32 = 32 KiB -- so the 32
-//    addresses of every warp ATOMS sit in 32 distinct banks whatever the data (uniform
-//    or 90 % one value): one smem wavefront per instruction.  (Packing two 16-bit bins
-//    per word halves the table but costs instructions: 2.5 vs 3.7 Tlanes/s measured.)
+//    addresses of every warp ATOMS sit in 32 distinct banks whatever the data: one smem
+//    wavefront per instruction.  (Packing two 16-bit bins per word halves the table but
+//    costs instructions: 2.5 vs 3.7 Tlanes/s measured.)  A warp whose batch is skewed
+//    (>= 12 of its 32 lanes start on lane 0's byte) counts that batch into one shared
+//    256-bin table instead, where same-byte lanes hit one word and ATOMS aggregates them:
+//    5.06 vs 3.78 TB/s on 90 %-one-value data, 2.5 vs 3.78 on uniform data
+//    (tools/hist_schemes.py, profiles/r02/hist_schemes.json -- the ceiling table of the
+//    counting schemes, incl. __match_any_sync aggregation and private LDS/STS counters).
 //  * CTAs walk contiguous (blocked) tile ranges, so a CTA stays in one VP for many tiles
 //    (segment lookups are cached) and flushes its replicas to the VP's global counts
 //    (one atomicAdd per non-zero bin) only at VP boundaries.
@@ -37,7 +42,10 @@ constexpr int kHistConsumers = kHistThreads;          // 256 = 8 warps
 constexpr int kHistBlock = kHistConsumers + 32;       // + producer warp
 constexpr int kHistStages = 3;
 constexpr int kHistBins = 256;
-constexpr int kHistSmem = kHistStages * kHistTile + kHistBins * 32 * 4 + 2 * kHistStages * 8 + 128;
+constexpr int kHistSmem = kHistStages * kHistTile + kHistBins * 33 * 4 + 2 * kHistStages * 8 + 128;
+// a warp whose 32 lanes' first bytes agree with lane 0's in at least this many lanes counts
+// its batch into the shared (non-replicated) table h1
+constexpr int kHistSkewLanes = 12;
 
 __device__ __forceinline__ void hist_zero_body(const SegDesc* __restrict__ segs, int nsegs) {
     for (int s = blockIdx.x; s < nsegs; s += gridDim.x) {
@@ -71,6 +79,17 @@ __device__ __forceinline__ void hist_add_word(uint32_t* hl, uint32_t w) {
     hist_add_byte(hl, (w >> 16) & 0xFFu);
     hist_add_byte(hl, w >> 24);
 }
+// Skewed batches (round 2, profiles/r02/hist_schemes.json): ONE shared 256-bin table h1.
+// Lanes holding the same byte hit the same word, which ATOMS.POPC.INC aggregates into one
+// update -- on 90 %-one-value data this ran at 5.06 TB/s against 3.78 for the per-lane
+// replicas (on uniform data the shared table's bank conflicts make it 2.5 TB/s, so each
+// warp picks per batch).
+__device__ __forceinline__ void hist_add_word_shared(uint32_t* h1, uint32_t w) {
+    atomicAdd(h1 + (w & 0xFFu), 1u);
+    atomicAdd(h1 + ((w >> 8) & 0xFFu), 1u);
+    atomicAdd(h1 + ((w >> 16) & 0xFFu), 1u);
+    atomicAdd(h1 + (w >> 24), 1u);
+}
 
 // Sum the 32 lane replicas of each bin (thread t owns bin t; the column walk is rotated
 // by t so a warp's 32 reads hit 32 banks), zero them, and add to the VP's counts.
@@ -79,7 +98,9 @@ __device__ __forceinline__ void hist_flush(uint32_t* h, uint32_t* counts) {
     static_assert(kHistConsumers == kHistBins, "one flush thread per bin");
     consumers_sync();
     const int b = threadIdx.x;
-    uint32_t sum = 0;
+    uint32_t* h1 = h + kHistBins * 32;  // the shared table follows the replicas
+    uint32_t sum = h1[b];
+    h1[b] = 0;
 #pragma unroll 8
     for (int j = 0; j < 32; ++j) {
         const int c = (j + b) & 31;
@@ -105,7 +126,9 @@ __device__ __forceinline__ void hist_flush_fused(uint32_t* h, uint32_t* counts, 
                                                  uint32_t expected, uint32_t* last_flag) {
     consumers_sync();
     const int b = threadIdx.x;
-    uint32_t sum = 0;
+    uint32_t* h1 = h + kHistBins * 32;
+    uint32_t sum = h1[b];
+    h1[b] = 0;
 #pragma unroll 8
     for (int j = 0; j < 32; ++j) {
         const int c = (j + b) & 31;
@@ -151,8 +174,9 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
                                           unsigned long long* __restrict__ busy, uint32_t* __restrict__ scratch) {
     extern __shared__ __align__(128) uint8_t hsm[];
     uint8_t* ring = hsm;                                                         // [stages][tile]
-    uint32_t* h = reinterpret_cast<uint32_t*>(hsm + kHistStages * kHistTile);     // [256][32]
-    uint64_t* full = reinterpret_cast<uint64_t*>(h + kHistBins * 32);
+    uint32_t* h = reinterpret_cast<uint32_t*>(hsm + kHistStages * kHistTile);     // [256][32] + h1[256]
+    uint32_t* h1 = h + kHistBins * 32;
+    uint64_t* full = reinterpret_cast<uint64_t*>(h + kHistBins * 33);
     uint64_t* empty = full + kHistStages;
     __shared__ uint32_t last_flag;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -163,7 +187,7 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
             if (segs[si].n == 0 && threadIdx.x < kHistBins) reinterpret_cast<uint32_t*>(segs[si].ptr[1])[threadIdx.x] = 0u;
     }
 
-    for (int i = threadIdx.x; i < kHistBins * 32; i += kHistBlock) h[i] = 0;
+    for (int i = threadIdx.x; i < kHistBins * 33; i += kHistBlock) h[i] = 0;
     if (threadIdx.x == 0) {
         for (int s = 0; s < kHistStages; ++s) {
             mbar_init(&full[s], 1);
@@ -245,12 +269,25 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
             uint4 r[kHistVec];
 #pragma unroll
             for (int i = 0; i < kHistVec; ++i) r[i] = st[i * kHistConsumers];
+            // per-warp choice of table for this batch (warp-uniform: no divergence)
+            const uint32_t b0 = r[0].x & 0xFFu;
+            const uint32_t hot = __shfl_sync(0xFFFFFFFFu, b0, 0);
+            if (__popc(__ballot_sync(0xFFFFFFFFu, b0 == hot)) >= kHistSkewLanes) {
 #pragma unroll
-            for (int i = 0; i < kHistVec; ++i) {
-                hist_add_word(hl, r[i].x);
-                hist_add_word(hl, r[i].y);
-                hist_add_word(hl, r[i].z);
-                hist_add_word(hl, r[i].w);
+                for (int i = 0; i < kHistVec; ++i) {
+                    hist_add_word_shared(h1, r[i].x);
+                    hist_add_word_shared(h1, r[i].y);
+                    hist_add_word_shared(h1, r[i].z);
+                    hist_add_word_shared(h1, r[i].w);
+                }
+            } else {
+#pragma unroll
+                for (int i = 0; i < kHistVec; ++i) {
+                    hist_add_word(hl, r[i].x);
+                    hist_add_word(hl, r[i].y);
+                    hist_add_word(hl, r[i].z);
+                    hist_add_word(hl, r[i].w);
+                }
             }
             // Release the stage only after every loaded word was consumed: the mbarrier
             // arrive (SYNCS unit) does not wait for this warp's outstanding LDS, so an

@@ -199,6 +199,77 @@ cudaError_t launch_sgemm_ffma(const GemmDesc* descs, int n, const void* maps, ui
     return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------ plain-load SGEMM
+// "sgemm" jobs TMA cannot address -- a row pitch (K or N floats) not a multiple of 16 B, or
+// a device buffer not 16-B aligned (these used to be SVP_E_UNSUPPORTED)
+// -- match as their own group and run here: the same grouped tile walk over the GemmDesc
+// table (A, B, lda, ldb), 64 x 64 tiles, 16-deep k blocks staged through shared memory with
+// guarded scalar loads, 4 x 4 fp32 FFMA register tiles (ascending k, like the FFMA kernel),
+// alpha * acc (+ beta * C) with guarded scalar stores.  No alignment or shape requirement.
+constexpr int PT = 64, PK = 16, kPlainThreads = 256;
+
+__global__ void __launch_bounds__(kPlainThreads)
+    k_sgemm_plain(const GemmDesc* __restrict__ descs, int n, uint32_t total) {
+    __shared__ float As[PK][PT + 4];  // k-major (transposed): As[k][m]
+    __shared__ float Bs[PK][PT];
+    const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+        const GemmDesc& g = descs[find_gemm(descs, n, t)];
+        const uint32_t lt = t - g.tile_begin;
+        const int m0 = (int)(lt / g.tiles_n) * PT, n0 = (int)(lt % g.tiles_n) * PT;
+        float acc[4][4] = {};
+        for (int k0 = 0; k0 < g.K; k0 += PK) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const int e = threadIdx.x + kPlainThreads * i;
+                const int ar = e >> 4, ak = e & 15;           // A: 64 rows x 16 k
+                const int gm = m0 + ar, gk = k0 + ak;
+                As[ak][ar] = (gm < g.M && gk < g.K) ? __ldg(g.A + (size_t)gm * g.lda + gk) : 0.f;
+                const int bk = e >> 6, bn = e & 63;           // B: 16 k x 64 cols
+                const int gk2 = k0 + bk, gn = n0 + bn;
+                Bs[bk][bn] = (gk2 < g.K && gn < g.N) ? __ldg(g.B + (size_t)gk2 * g.ldb + gn) : 0.f;
+            }
+            __syncthreads();
+#pragma unroll
+            for (int k = 0; k < PK; ++k) {
+                float a[4], b[4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) a[i] = As[k][ty * 4 + i];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) b[j] = Bs[k][tx * 4 + j];
+#pragma unroll
+                for (int i = 0; i < 4; ++i)
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) acc[i][j] = __fmaf_rn(a[i], b[j], acc[i][j]);
+            }
+            __syncthreads();
+        }
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            const int gm = m0 + ty * 4 + i;
+            if (gm >= g.M) continue;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const int gn = n0 + tx * 4 + j;
+                if (gn >= g.N) continue;
+                float* c = g.C + (size_t)gm * g.N + gn;
+                float o = g.K == 0 ? 0.f : g.alpha * acc[i][j];
+                if (g.beta != 0.f) o = __fmaf_rn(g.beta, *c, o);
+                *c = o;
+            }
+        }
+    }
+}
+
+cudaError_t launch_sgemm_plain(const GemmDesc* descs, int n, uint32_t total, int grid, cudaStream_t s) {
+    k_sgemm_plain<<<grid, kPlainThreads, 0, s>>>(descs, n, total);
+    return cudaGetLastError();
+}
+
+cudaError_t query_limits_gemm_plain(int* per_sm) {
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k_sgemm_plain, kPlainThreads, 0);
+}
+
 cudaError_t query_limits_gemm(int* per_sm) {
     cudaError_t e = cudaFuncSetAttribute(k_sgemm_ffma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kGemmSmem);
     if (e) return e;

@@ -82,6 +82,7 @@
 
 #include <atomic>
 
+#include "../../../include/svp.h"
 #include "../launch.h"
 #include "common.cuh"
 
@@ -265,6 +266,17 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
         : "memory");
 }
 
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
+        "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n\t"
+        "tcgen05.wait::ld.sync.aligned;"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+        : "r"(taddr)
+        : "memory");
+}
+
 __device__ __forceinline__ int find_tile_owner(const GemmDesc* __restrict__ d, int n, uint32_t t) {
     int lo = 0, hi = n;
     while (lo < hi) {
@@ -280,11 +292,18 @@ __device__ __forceinline__ float4 lo_part4(float4 x) {
     return make_float4(lo_part(x.x), lo_part(x.y), lo_part(x.z), lo_part(x.w));
 }
 
-// bf16x2 of (a -> low half, b -> high half), round to nearest even; .satfinite (free in
-// SASS: F2FP.SATFINITE): a finite TF32 head beyond the bf16 range (|h| >= (2 - 2^-8) 2^127)
-// becomes +-max_bf16 instead of +-Inf, so a finite operand near FLT_MAX cannot turn a cross
-// term into an infinity (R20)
+// bf16x2 of (a -> low half, b -> high half), round to nearest even (the low parts: a NaN or
+// infinite l -- from an Inf / NaN operand, or a head that rounded past FLT_MAX -- must stay
+// non-finite so the output's accumulator turns NaN and the epilogue recomputes it, R20)
 __device__ __forceinline__ uint32_t bf2(float a, float b) {
+    uint32_t r;
+    asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
+    return r;
+}
+// the heads: .satfinite (free in SASS: F2FP.SATFINITE) -- a finite TF32 head beyond the bf16
+// range (|h| >= (2 - 2^-8) 2^127) becomes +-max_bf16 instead of +-Inf, so a finite operand
+// near FLT_MAX cannot turn a cross term into an infinity with a finite accumulator
+__device__ __forceinline__ uint32_t bf2s(float a, float b) {
     uint32_t r;
     asm("cvt.rn.satfinite.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(b), "f"(a));
     return r;
@@ -309,7 +328,7 @@ __device__ __forceinline__ void split8_given(const float4& p, const float4& q, c
     uint32_t hh[4], ll[4];
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
-        hh[i] = bf2(h[2 * i], h[2 * i + 1]);
+        hh[i] = bf2s(h[2 * i], h[2 * i + 1]);
         ll[i] = bf2(x[2 * i] - h[2 * i], x[2 * i + 1] - h[2 * i + 1]);
     }
     hb = make_uint4(hh[0], hh[1], hh[2], hh[3]);
@@ -324,20 +343,35 @@ __device__ __forceinline__ void split8_given(const float4& p, const float4& q, c
 // beta * c_old in fp64, one rounding.  The rare path of the tensor-core epilogue for outputs
 // whose accumulator came out NaN -- an Inf or NaN operand, or a finite one at the top of the
 // fp32 range -- so their Inf / NaN / finite value is the IEEE one.
-__device__ __noinline__ float exact_element(const GemmDesc& g, int i, int j, float c_old) {
+__device__ __forceinline__ float exact_element(const GemmDesc& g, int i, int j, float c_old) {
     const float* a = g.A + (size_t)i * g.lda;
     const float* b = g.B + j;
+    const size_t ldb = (size_t)g.ldb;
     double acc = 0.0;
-    for (int k = 0; k < g.K; ++k)
-        acc = __dadd_rn(acc, __dmul_rn((double)__ldg(a + k), (double)__ldg(b + (size_t)k * g.ldb)));
+#pragma unroll 1
+    for (int k = g.K; k > 0; --k, ++a, b += ldb) acc = __dadd_rn(acc, __dmul_rn((double)__ldg(a), (double)__ldg(b)));
     double r = __dmul_rn((double)g.alpha, acc);
     if (g.beta != 0.f) r = __dadd_rn(r, __dmul_rn((double)g.beta, (double)c_old));
     return (float)r;
 }
 
+// K-chunked accumulation (R23): the tcgen05 fp32 accumulation loses magnitude
+// (measured -1.66e-8 relative per accumulating MMA), so a tile's K range is cut into chunks
+// of `kchunk` 16-k blocks, each accumulated from zero in its own TMEM accumulator (the two
+// accumulators ping-pong between chunks as they do between tiles) and folded into C by the
+// epilogue with IEEE fp32 adds (chunk 0 stores alpha * acc, later chunks C += alpha * acc):
+// the output's relative bias is then that of ONE chunk, whatever K is.  Only for beta == 0
+// (a beta != 0 job keeps C_old for its exact NaN path; the executor routes those with
+// K > the chunk to the FFMA kernel).  Producer, MMA issuer and epilogue all walk the same
+// (tile, chunk) units.
+__device__ __forceinline__ int tc_chunks(const GemmDesc& g, int KB, int kchunk) {
+    return (kchunk > 0 && g.beta == 0.f && KB > kchunk) ? (KB + kchunk - 1) / kchunk : 1;
+}
+
 template <int SPLIT, int CG, int NH>
 __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
-    k_sgemm_tc(const GemmDesc* __restrict__ descs, int n, const uint8_t* __restrict__ maps, uint32_t total) {
+    k_sgemm_tc(const GemmDesc* __restrict__ descs, int n, const uint8_t* __restrict__ maps, uint32_t total,
+               int kchunk) {
     using namespace tc;
     using C = Cfg<SPLIT, CG, NH>;
     constexpr int TN = BN * NH;  // tile width in N per CTA pair (or CTA)
@@ -443,17 +477,20 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
     } else if (warp == 1) {
         // ------------------------------------------------------------ MMA issuer
         if (leader) {
-            uint32_t it = 0, tile_i = 0;
-            for (uint32_t t = cl; t < total; t += ncl, ++tile_i) {
-                const int v = find_tile_owner(descs, n, t);
-                const int KB = (descs[v].K + BK - 1) / BK;
+            uint32_t it = 0, tile_i = 0;  // tile_i counts (tile, chunk) units
+            for (uint32_t t = cl; t < total; t += ncl) {
+              const int v = find_tile_owner(descs, n, t);
+              const int KB = (descs[v].K + BK - 1) / BK;
+              const int nch = tc_chunks(descs[v], KB, kchunk);
+              for (int ck = 0; ck < nch; ++ck, ++tile_i) {
+                const int kb0 = nch == 1 ? 0 : ck * kchunk, kb1 = nch == 1 ? KB : min(KB, kb0 + kchunk);
                 const int a = tile_i % C::kAcc;
                 const uint32_t aph = (tile_i / C::kAcc) & 1;
                 if constexpr (CG == 2) mbar_wait_cluster(&acc_empty[a], aph ^ 1);
                 else mbar_wait(&acc_empty[a], aph ^ 1);
                 tc_fence_after();
                 const uint32_t tmem_d = tmem_base + (uint32_t)(a * BN);
-                for (int kb = 0; kb < KB; ++kb, ++it) {
+                for (int kb = kb0; kb < kb1; ++kb, ++it) {
                     const int s = it % ST;
                     const uint32_t ph = (it / ST) & 1;
                     if constexpr (CG == 2) {
@@ -474,7 +511,7 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                             // 64-n atoms 2h, 2h+1 (bf16); its accumulator is free once the
                             // previous tile's half-h epilogue drained it
                             const int ab = NH == 1 ? a : h;
-                            if (NH == 2 && h == 1 && kb == 0) {
+                            if (NH == 2 && h == 1 && kb == kb0) {
                                 mbar_wait_cluster(&acc_empty[1], aph ^ 1);
                                 tc_fence_after();
                             }
@@ -484,7 +521,7 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                             for (int kk = 0; kk < BK / 8; ++kk) {
                                 const uint64_t ah = desc_a(s_ah + kk * 32);         // +8 k in a 64-B row
                                 const uint64_t bh = desc_b(s_bh + bo + kk * 1024);  // +8 k rows of 128 B
-                                const uint32_t acc0 = (kb > 0 || kk > 0) ? 1u : 0u;
+                                const uint32_t acc0 = (kb > kb0 || kk > 0) ? 1u : 0u;
                                 if (SPLIT == 3) {
                                     mma_tf32<CG>(td, ah, desc_b(s_bl + kk * 1024), acc0);
                                     mma_tf32<CG>(td, desc_a(s_al + kk * 32), bh, 1u);
@@ -505,13 +542,13 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                                 mma_bf16_ta<CG>(td, ta, desc_b16(b16l), 1u);      // bf(A_hi) bf(B_lo)
                                 mma_bf16_ta<CG>(td, ta + 8, desc_b16(b16h), 1u);  // bf(A_lo) bf(B_hi)
                             }
-                            if (kb == KB - 1) mma_commit<CG>(&acc_full[ab]);
+                            if (kb == kb1 - 1) mma_commit<CG>(&acc_full[ab]);
                         }
                         mma_commit<CG>(&empty[s]);
                     }
                     __syncwarp();
                 }
-                if (KB == 0 && lane == 0) {  // K == 0: nothing accumulated
+                if (kb1 == kb0 && lane == 0) {  // K == 0: nothing accumulated
                     for (int h = 0; h < NH; ++h) {
                         const int ab = NH == 1 ? a : h;
                         if (NH == 2 && h == 1) mbar_wait_cluster(&acc_empty[1], aph ^ 1);
@@ -524,6 +561,7 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     }
                 }
                 __syncwarp();
+              }
             }
         }
     } else if (warp < 4 || (warp >= 8 && warp < 14)) {
@@ -646,10 +684,12 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
         const int q = warp & 3;  // TMEM lane quarter
         const int eh = (NH == 2 && warp >= 14) ? 1 : 0;
         const uint32_t acc_empty_leader = CG == 2 ? map_to(&acc_empty[0], 0) : 0;
-        uint32_t tile_i = 0;
-        for (uint32_t t = cl; t < total; t += ncl, ++tile_i) {
-            const int v = find_tile_owner(descs, n, t);
-            const GemmDesc& g = descs[v];
+        uint32_t tile_i = 0;  // (tile, chunk) units, as the MMA issuer counts them
+        for (uint32_t t = cl; t < total; t += ncl) {
+          const int v = find_tile_owner(descs, n, t);
+          const GemmDesc& g = descs[v];
+          const int nch = tc_chunks(g, (g.K + BK - 1) / BK, kchunk);
+          for (int ck = 0; ck < nch; ++ck, ++tile_i) {
             const uint32_t lt = t - g.tile_begin;
             const int tm = lt / g.tiles_n, tn = lt % g.tiles_n;
             const int a = NH == 1 ? (int)(tile_i % C::kAcc) : eh;
@@ -661,16 +701,27 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
             float* crow = g.C + (size_t)(row_ok ? row : 0) * g.N;
             const float alpha = g.alpha, beta = g.beta;
             const bool kzero = g.K == 0;
+            const bool first = ck == 0, last = ck == nch - 1;
 #pragma unroll 1
-            for (int c0 = 0; c0 < BN; c0 += 32) {
-                uint32_t r[32];
-                tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0), r);
+            for (int c0 = 0; c0 < BN; c0 += 16) {
                 const int col0 = tn * TN + eh * BN + c0;
-                if (!row_ok) continue;
-                uint32_t nan_mask = 0;  // outputs of this chunk whose accumulator is NaN
+                // later K chunk: the partial sum the previous chunk stored (this thread wrote
+                // it: program order; in L2) -- loads issued before the TMEM read so their
+                // latency overlaps it
+                float4 prev[4];
+                if (!first && row_ok) {
 #pragma unroll
-                for (int j = 0; j < 32; j += 4) {
-                    const int c = col0 + j;
+                    for (int jj = 0; jj < 4; ++jj)
+                        prev[jj] = col0 + 4 * jj < g.N ? *reinterpret_cast<const float4*>(crow + col0 + 4 * jj)
+                                                       : make_float4(0.f, 0.f, 0.f, 0.f);
+                }
+                uint32_t r[16];
+                tmem_ld16(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0), r);
+                if (!row_ok) continue;
+                uint32_t nan_mask = 0;  // outputs of this slab whose final value came out NaN
+#pragma unroll
+                for (int jj = 0; jj < 4; ++jj) {
+                    const int j = 4 * jj, c = col0 + j;
                     if (c >= g.N) break;
                     float4 o;
                     o.x = kzero ? 0.f : alpha * __uint_as_float(r[j + 0]);
@@ -679,7 +730,13 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     o.w = kzero ? 0.f : alpha * __uint_as_float(r[j + 3]);
                     float4* dst = reinterpret_cast<float4*>(crow + c);
                     float4 old = make_float4(0.f, 0.f, 0.f, 0.f);
-                    if (beta != 0.f) {
+                    if (!first) {
+                        old = prev[jj];
+                        o.x += old.x;
+                        o.y += old.y;
+                        o.z += old.z;
+                        o.w += old.w;
+                    } else if (beta != 0.f) {
                         old = __ldcs(dst);
                         o.x = __fmaf_rn(beta, old.x, o.x);
                         o.y = __fmaf_rn(beta, old.y, o.y);
@@ -688,23 +745,27 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     }
                     // IEEE special values (R20): an Inf / NaN operand (its low part x - h is NaN),
                     // or a finite one whose TF32 head rounds past FLT_MAX, leaves NaN in every
-                    // accumulator it reaches.  Those outputs keep C_old for now and are
-                    // recomputed exactly below (rare path, after r[] is dead).
-                    const float acc4 = __uint_as_float(r[j]) + __uint_as_float(r[j + 1]) +
-                                       __uint_as_float(r[j + 2]) + __uint_as_float(r[j + 3]);
-                    if (!kzero && acc4 != acc4) {
-                        if (isnan(__uint_as_float(r[j + 0]))) { nan_mask |= 1u << (j + 0); o.x = old.x; }
-                        if (isnan(__uint_as_float(r[j + 1]))) { nan_mask |= 1u << (j + 1); o.y = old.y; }
-                        if (isnan(__uint_as_float(r[j + 2]))) { nan_mask |= 1u << (j + 2); o.z = old.z; }
-                        if (isnan(__uint_as_float(r[j + 3]))) { nan_mask |= 1u << (j + 3); o.w = old.w; }
+                    // accumulator it reaches (and, across K chunks, in the partial sum).  In the
+                    // last chunk those outputs keep C_old (chunked: beta == 0, C_old unused) and
+                    // are recomputed exactly below (rare path, after r[] is dead).
+                    if (last) {
+                        const float o4 = o.x + o.y + o.z + o.w;
+                        if (!kzero && o4 != o4) {
+                            if (isnan(o.x)) { nan_mask |= 1u << (j + 0); o.x = old.x; }
+                            if (isnan(o.y)) { nan_mask |= 1u << (j + 1); o.y = old.y; }
+                            if (isnan(o.z)) { nan_mask |= 1u << (j + 2); o.z = old.z; }
+                            if (isnan(o.w)) { nan_mask |= 1u << (j + 3); o.w = old.w; }
+                        }
+                        __stcs(dst, o);  // st.global.cs: C's final value
+                    } else {
+                        *dst = o;  // a partial sum, re-read by the next chunk: keep it in L2
                     }
-                    __stcs(dst, o);  // st.global.cs: C is written once
                 }
                 while (nan_mask) {
                     const int e = __ffs(nan_mask) - 1;
                     nan_mask &= nan_mask - 1;
                     float* cp = crow + col0 + e;
-                    *cp = exact_element(g, row, col0 + e, beta != 0.f ? *cp : 0.f);
+                    *cp = exact_element(g, row, col0 + e, (beta != 0.f && nch == 1) ? *cp : 0.f);
                 }
             }
             tc_fence_before();
@@ -713,6 +774,7 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                 if constexpr (CG == 2) mbar_arrive_cluster(acc_empty_leader + (uint32_t)a * 8u);
                 else mbar_arrive(&acc_empty[a]);
             }
+          }
         }
     }
     // ---------------------------------------------------------------- teardown
@@ -760,7 +822,24 @@ static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uin
         lc.attrs = attr;
         lc.numAttrs = 1;
     }
-    return cudaLaunchKernelEx(&lc, kern, descs, n, reinterpret_cast<const uint8_t*>(maps), total);
+    // the plain-TF32 "sgemm_tf32" (own 2e-3 tolerance) accumulates the whole K in one chunk
+    const int kchunk = SPLIT == 1 ? 0 : sgemm_tc_kchunk(SPLIT == 3 ? SVP_SGEMM_3XTF32 : SVP_SGEMM_TF32BF16) / tc::BK;
+    return cudaLaunchKernelEx(&lc, kern, descs, n, reinterpret_cast<const uint8_t*>(maps), total, kchunk);
+}
+
+// K chunk of the fp32 tensor-core splits in k (a multiple of 16; 0 = off): SVP_SGEMM_KCHUNK
+// for TF32+2xBF16, default 512 (R23: 4 accumulating MMAs per 16 k -> ~ -2.1e-6 relative per
+// chunk on random-sign data, ~ -4.1e-6 on same-sign data); 3xTF32 (6 MMAs per 16 k, larger
+// bias per MMA) uses half of it
+int sgemm_tc_kchunk(int impl) {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("SVP_SGEMM_KCHUNK");
+        int k = e ? atoi(e) : 512;
+        v = k <= 0 ? 0 : (k + 15) / 16 * 16;
+    }
+    if (impl == SVP_SGEMM_3XTF32) return v >= 32 ? v / 32 * 16 : v;
+    return impl == SVP_SGEMM_TF32BF16 ? v : 0;
 }
 
 // CTA-pair kernels for the fp32-accurate splits unless SVP_TC_CTA_PAIR=0 (A/B switch)

@@ -16,6 +16,7 @@ struct LaunchLimits {
     int mix_blocks_per_sm = 4;
     int hist_blocks_per_sm = 4;
     int gemm_blocks_per_sm = 1;
+    int gemm_plain_blocks_per_sm = 1;
     int dgemm_blocks_per_sm = 1;
     int dgemm_small_blocks_per_sm = 1;
 };
@@ -55,6 +56,11 @@ cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total_tiles,
 // Grouped SGEMM (fp32 FFMA, TMA-staged).  maps = 2*n CUtensorMap (A_i, B_i), 64-B aligned.
 cudaError_t launch_sgemm_ffma(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
                               int grid, cudaStream_t s);
+// Grouped SGEMM with plain guarded loads (64 x 64 tiles, FFMA): jobs whose pitches / buffers
+// TMA cannot address (K or N not a multiple of 4, device buffers not 16-B aligned).
+constexpr int kSgemmPlainTile = 64;
+cudaError_t launch_sgemm_plain(const GemmDesc* descs, int n, uint32_t total_tiles, int grid, cudaStream_t s);
+cudaError_t query_limits_gemm_plain(int* per_sm);
 // Grouped SGEMM on tcgen05 TF32 tensor cores (TMEM accumulators).
 cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
                               int grid, cudaStream_t s);
@@ -71,6 +77,8 @@ cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps
 // true: the fp32-accurate tcgen05 SGEMMs run as CTA pairs (cta_group::2, 256 x 256 tiles);
 // SVP_TC_CTA_PAIR=0 selects the single-CTA kernels (128 x 256 tiles)
 bool sgemm_tc_cta_pair();
+// K chunk (in k, multiple of 16; 0 = off) of an fp32 tensor-core split's accumulation (R23)
+int sgemm_tc_kchunk(int sgemm_impl);
 // 256 x 512 tiles for the TF32+2xBF16 pair kernel (two 256-column accumulator halves sharing
 // each A tile): SVP_TC_WIDE=0 never, 1 (default) when a launch has >= 2 waves of them, 2 always
 int sgemm_tc_wide_mode();

@@ -27,6 +27,7 @@
 #include <tuple>
 
 #include "internal.h"
+#include "launch.h"
 #include "tables.h"
 
 namespace svp {
@@ -38,7 +39,12 @@ double CostModel::kernel_ns(int32_t kernel, double alg_bytes, double flops) cons
     else if (kernel == K_DGEMM) body = flops / fp64_flops * 1e9;
     else if (kernel == K_SGEMM_TF32) body = flops / tf32_flops * 1e9;
     else body = alg_bytes / hbm_Bps * 1e9;
-    return launch_ns + body * kscale[kernel];
+    return launch_ns + body * kscale[kernel][bucket(alg_bytes, flops)];
+}
+double CostModel::sgemm_ns(int32_t impl, double alg_bytes, double flops) const {
+    const int units = impl == SVP_SGEMM_3XTF32 ? 3 : impl == SVP_SGEMM_TF32BF16 ? 2 : 0;
+    const double body = flops / (units ? tf32_flops / units : ffma_flops) * 1e9;
+    return launch_ns + body * kscale[K_SGEMM][bucket(alg_bytes, flops)];
 }
 double CostModel::h2d_ns(uint64_t bytes, int ncopies) const {
     return bytes ? copy_ns * ncopies + (double)bytes / pcie_Bps * 1e9 : 0.0;
@@ -102,8 +108,6 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
             j->K = a.K;
             j->f0 = a.alpha;
             j->f1 = a.beta;
-            if ((int64_t)a.M * a.N * a.K > 0 && (a.K % 4 != 0 || a.N % 4 != 0))
-                return fail(SVP_E_UNSUPPORTED, "svp_submit: sgemm needs K % 4 == 0 and N % 4 == 0 (TMA row pitch)");
             break;
         }
         case K_DGEMM: {
@@ -147,9 +151,6 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
         if (bf.bytes < need)
             return fail(SVP_E_INVAL, "svp_submit: buffer " + std::to_string(b) + " has " + std::to_string(bf.bytes) +
                                          " bytes, kernel touches " + std::to_string(need));
-        if ((j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32) && bf.mem == SVP_MEM_DEVICE &&
-            ((uintptr_t)bf.ptr & 15))
-            return fail(SVP_E_UNSUPPORTED, "svp_submit: sgemm device buffers must be 16-B aligned (TMA)");
         if (j->kernel == K_DGEMM && ((uintptr_t)bf.ptr & 7))
             return fail(SVP_E_INVAL, "svp_submit: dgemm buffers must be 8-B aligned");
         bool rd = bf.dir & SVP_DIR_IN, wr = bf.dir & SVP_DIR_OUT;
@@ -177,7 +178,26 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
     // Reading R1 (revised with f2): every job of a kernel is "identical" -- ragged element
     // counts AND ragged GEMM shapes share one coalesced launch (per-VP M, N, K live in
     // the tile table).
+    // Jobs TMA cannot address (a row pitch of K or N floats not a multiple of 16 B, or a
+    // device buffer not 16-B aligned; staged host buffers are 256-B aligned in the arena)
+    // match as their own group on the plain-load kernel (shape key 2); R23: "sgemm" jobs past
+    // the tensor-core split's K limit match apart and run on FFMA (shape key 1).
     j->shape_key = 0;
+    if (j->kernel == K_SGEMM || j->kernel == K_SGEMM_TF32) {
+        bool plain = (j->K % 4) != 0 || (j->N % 4) != 0;
+        for (int b = 0; b < j->nbufs; ++b)
+            if (j->bufs[b].mem == SVP_MEM_DEVICE && ((uintptr_t)j->bufs[b].ptr & 15)) plain = true;
+        if (plain) {
+            j->shape_key = 2;
+        } else if (j->kernel == K_SGEMM && c->cfg.sgemm_impl != SVP_SGEMM_FFMA) {
+            // with K-chunked accumulation (sgemm_tc_kchunk) a beta == 0 job keeps the
+            // tensor cores at any K; a beta != 0 job is not chunked (its exact NaN path needs
+            // C_old), so it keeps them up to one chunk
+            const int kc = sgemm_tc_kchunk(c->cfg.sgemm_impl);
+            const int32_t kmax = kc > 0 ? (j->f1 != 0.f ? kc : (1 << 30)) : sgemm_tc_kmax(c->cfg.sgemm_impl);
+            if (j->K > kmax) j->shape_key = 1;
+        }
+    }
     double cost = c->cost.kernel_ns(j->kernel, j->alg_bytes, j->flops);
     j->device = dispatch_vp(c, j->vp, cost);
     if (c->exec && c->cfg.validate_ptrs && !empty) {
@@ -277,7 +297,8 @@ static void estimate_chunk(const Ctx* c, const Flush& f, Chunk& ch) {
         }
     }
     ch.t_in = c->cost.h2d_ns(ch.in_bytes, nin);
-    ch.t_k = c->cost.kernel_ns(ch.kernel, ch.alg_bytes, ch.flops);
+    ch.t_k = (ch.kernel == K_SGEMM || ch.sgemm_impl == kSgemmPlain) ? c->cost.sgemm_ns(ch.sgemm_impl, ch.alg_bytes, ch.flops)
+                                  : c->cost.kernel_ns(ch.kernel, ch.alg_bytes, ch.flops);
     ch.t_out = c->cost.d2h_ns(ch.out_bytes, nout);
 }
 
@@ -387,8 +408,13 @@ svp_status plan_flush(Ctx* c, Flush* f) {
     const uint64_t arena = c->cfg.arena_bytes;
     for (int32_t gi = 0; gi < (int32_t)f->groups.size(); ++gi) {
         const Group& g = f->groups[gi];
+        const int32_t impl = g.shape_key == 2          ? kSgemmPlain
+                             : g.kernel != K_SGEMM      ? -1
+                             : g.shape_key == 1         ? (int32_t)SVP_SGEMM_FFMA
+                                                        : c->cfg.sgemm_impl;
         Chunk whole;
         whole.kernel = g.kernel;
+        whole.sgemm_impl = impl;
         whole.jobs = g.jobs;
         estimate_chunk(c, *f, whole);
         int nch = 1;
@@ -434,6 +460,7 @@ svp_status plan_flush(Ctx* c, Flush* f) {
             ch.device = g.device;
             ch.level = g.level;
             ch.kernel = g.kernel;
+            ch.sgemm_impl = impl;
             ch.jobs = parts[p];
             estimate_chunk(c, *f, ch);
             ch.arena_len = staged_bytes(*f, ch.jobs);
@@ -458,8 +485,9 @@ svp_status plan_flush(Ctx* c, Flush* f) {
     // (cfg5: 44.1k jobs/s vs 42.7k on one stream).  SVP_COSCHEDULE=1 instead launches the
     // memory-bound kernels first on a small grid (co_grid CTAs/SM) -- measured slower
     // (41.3k), kept as an option for other mixes.
-    auto tensor_kernel = [&](int32_t k) {
-        return k == K_SGEMM_TF32 || (k == K_SGEMM && c->cost.sgemm_tc_units > 0);
+    auto tensor_chunk = [&](const Chunk& ch) {
+        return (ch.kernel == K_SGEMM_TF32 || ch.kernel == K_SGEMM) && ch.sgemm_impl != SVP_SGEMM_FFMA &&
+               ch.sgemm_impl != kSgemmPlain;
     };
     auto device_only = [&](const Chunk& ch) { return ch.t_in == 0 && ch.t_out == 0; };
     std::stable_sort(corder.begin(), corder.end(), [&](int32_t x, int32_t y) {
@@ -469,7 +497,7 @@ svp_status plan_flush(Ctx* c, Flush* f) {
         const bool da = device_only(a), db = device_only(b);
         if (da != db) return da;  // device-only chunks first; copies are on their own streams
         if (da && c->coschedule) {
-            const bool ta = tensor_kernel(a.kernel), tb = tensor_kernel(b.kernel);
+            const bool ta = tensor_chunk(a), tb = tensor_chunk(b);
             if (ta != tb) return !ta;
             return std::make_tuple(-a.t_k, a.group, a.index) < std::make_tuple(-b.t_k, b.group, b.index);
         }
@@ -480,7 +508,7 @@ svp_status plan_flush(Ctx* c, Flush* f) {
         // tensor-core SGEMM chunk (hist256 keeps its default grid: it needs shared memory)
         std::map<std::pair<int32_t, int32_t>, bool> has_tensor;
         for (const auto& ch : f->chunks)
-            if (device_only(ch) && tensor_kernel(ch.kernel)) has_tensor[{ch.level, ch.device}] = true;
+            if (device_only(ch) && tensor_chunk(ch)) has_tensor[{ch.level, ch.device}] = true;
         for (auto& ch : f->chunks) {
             if (!device_only(ch) || !has_tensor.count({ch.level, ch.device})) continue;
             if (ch.kernel == K_VECADD || ch.kernel == K_SAXPY || ch.kernel == K_EW_MIX) ch.co_grid = 2;
@@ -498,6 +526,9 @@ svp_status plan_flush(Ctx* c, Flush* f) {
     // (list scheduling; ties -> lowest index).  Round-robin put cfg5's 5th launch (hist256)
     // behind the SGEMM on stream 0, so it ran alone after it.  SVP_STREAM_RR=1: round-robin.
     static const bool stream_rr = getenv("SVP_STREAM_RR") && atoi(getenv("SVP_STREAM_RR")) != 0;
+    // diagnostic (mode-H timeline study): first compute stream the list scheduler may use
+    static const int first_cs_env = getenv("SVP_FIRST_COMPUTE_STREAM") ? atoi(getenv("SVP_FIRST_COMPUTE_STREAM")) : 0;
+    const int first_cs = std::max(0, std::min(first_cs_env, S - 1));
     std::vector<std::vector<double>> sload(c->ngpu, std::vector<double>(S, 0.0));
     for (int32_t ci : corder) {
         Chunk& ch = f->chunks[ci];
@@ -542,7 +573,8 @@ svp_status plan_flush(Ctx* c, Flush* f) {
             if (stream_rr) {
                 cs = rr[dev]++ % S;
             } else {
-                for (int k = 1; k < S; ++k)
+                cs = first_cs;
+                for (int k = first_cs + 1; k < S; ++k)
                     if (sload[dev][k] < sload[dev][cs]) cs = k;
                 sload[dev][cs] += std::max(ch.t_k, 1.0);
             }

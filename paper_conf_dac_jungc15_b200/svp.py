@@ -159,7 +159,7 @@ def load(build_if_stale: bool = True):
         L.svp_kernel_lookup.argtypes = [C.c_char_p, P(C.c_int32)]
         L.svp_device_stats_get.argtypes = [vp, C.c_int32, P(svp_device_stats)]
         L.svp_plan_op_detail.argtypes = [vp, C.c_int32, P(C.c_uint64), P(C.c_uint64), P(C.c_int32), C.c_int32,
-                                         P(C.c_int32)]
+                                         P(C.c_int32), P(C.c_double)]
         for name in EXPORTS:
             f = getattr(L, name)
             if name not in ("svp_config_default", "svp_last_error", "svp_abi_version"):
@@ -383,10 +383,11 @@ class Context:
             _check(self._L.svp_plan_get(self._h, i, C.byref(op), vps, 4096))
             d = {k: getattr(op, k) for k, _ in svp_plan_op._fields_}
             d["vps"] = list(vps[: min(op.nvps, 4096)])
-            aoff, alen, nw = C.c_uint64(), C.c_uint64(), C.c_int32()
+            aoff, alen, nw, t0 = C.c_uint64(), C.c_uint64(), C.c_int32(), C.c_double()
             waits = (C.c_int32 * 256)()
-            _check(self._L.svp_plan_op_detail(self._h, i, C.byref(aoff), C.byref(alen), waits, 256, C.byref(nw)))
-            d["arena_off"], d["arena_len"] = aoff.value, alen.value
+            _check(self._L.svp_plan_op_detail(self._h, i, C.byref(aoff), C.byref(alen), waits, 256, C.byref(nw),
+                                              C.byref(t0)))
+            d["arena_off"], d["arena_len"], d["measured_start_ns"] = aoff.value, alen.value, t0.value
             d["waits"] = list(waits[: min(nw.value, 256)])
             out.append(d)
         return out

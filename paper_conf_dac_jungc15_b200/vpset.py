@@ -71,7 +71,9 @@ class VPSet:
             if s.kernel not in self.kids:
                 self.kids[s.kernel] = ctx.kernel(s.kernel)
         if assign and residency == "device":
-            costs = [float(getattr(s, "n", 0) * 12 + 2 * s.M * s.N * s.K / 10.0) for s in self.specs]
+            # estimated kernel ns (the Dispatcher's LPT costs): algorithmic bytes at the measured
+            # 6.55 TB/s + FLOPs at ~400 TFLOP/s (the fp32 tensor-core split)
+            costs = [float(s.algorithmic_bytes()) / 6.55 + float(s.flops()) / 4.0e5 for s in self.specs]
             ctx.assign_vps([s.vp for s in self.specs], [self.kids[s.kernel] for s in self.specs], costs)
         self.bufs: List[Dict[str, torch.Tensor]] = []   # views (what the kernel sees)
         self.raw: List[Dict[str, torch.Tensor]] = []    # allocations incl. misalign + guard
@@ -90,7 +92,9 @@ class VPSet:
                 # misalign 1: every buffer shifted by one element (co-aligned -> vector path
                 # with a head shift); misalign 2: only the first buffer (scalar path)
                 mis = m if (m == 1 or bi == 0) else 0
-                if s.kernel in GEMMS or (s.kernel == "hist256" and name == "counts"):
+                if s.kernel in GEMMS:
+                    mis = m  # every matrix shifted by m elements (m = 1: 4-B offset, not 16-B aligned)
+                elif s.kernel == "hist256" and name == "counts":
                     mis = 0
                 elif s.kernel == "hist256":
                     mis = 7 * m

@@ -76,8 +76,7 @@ def _vecadd_bufs(n, mem=svp.MEM_DEVICE, bytes_=None):
 @pytest.mark.parametrize("case,status", [
     ("wrong_nbufs", svp.SVP_E_INVAL), ("wrong_dir", svp.SVP_E_INVAL), ("too_small", svp.SVP_E_INVAL),
     ("bad_vp", svp.SVP_E_INVAL), ("unregistered", svp.SVP_E_NOKERNEL), ("short_args", svp.SVP_E_INVAL),
-    ("null_ptr", svp.SVP_E_INVAL), ("bad_mem", svp.SVP_E_INVAL), ("sgemm_k", svp.SVP_E_UNSUPPORTED),
-    ("sgemm_beta_out", svp.SVP_E_INVAL), ("sgemm_misaligned", svp.SVP_E_UNSUPPORTED),
+    ("null_ptr", svp.SVP_E_INVAL), ("bad_mem", svp.SVP_E_INVAL), ("sgemm_beta_out", svp.SVP_E_INVAL),
 ])
 def test_submit_validation(case, status):
     with svp.Context(dry_run=True) as c:
@@ -120,6 +119,23 @@ def test_submit_validation(case, status):
             c.submit(vp, kid, args, bufs)
         assert e.value.status == status, svp.last_error()
         assert svp.last_error()
+
+
+def test_sgemm_any_shape_and_alignment_is_accepted_and_routed():
+    """K or N not a multiple of 4 (a TMA row pitch must be a multiple
+    of 16 B) and device buffers not 16-B aligned used to be SVP_E_UNSUPPORTED; they are now
+    accepted and match as their own group (the plain-load kernel)."""
+    with svp.Context(dry_run=True) as c:
+        sg = c.register_kernel("sgemm")
+        shapes = [(64, 64, 64, 0), (64, 130, 64, 0), (64, 64, 30, 0), (64, 64, 64, 4), (33, 17, 5, 0)]
+        for vp, (M, N, K, off) in enumerate(shapes):
+            base = FAKE + vp * 2**34
+            c.submit(vp, sg, svp.args_sgemm(M, N, K), [(base + off, 4 * M * K, svp.DIR_IN, 0),
+                                                       (base + 2**30, 4 * K * N, svp.DIR_IN, 0),
+                                                       (base + 2**31, 4 * M * N, svp.DIR_OUT, 0)])
+        c.flush()
+        ops = [op for op in c.plan() if op["kind"] == svp.OP_KERNEL]
+        assert sorted(sorted(op["vps"]) for op in ops) == [[0], [1, 2, 3, 4]]
 
 
 def test_zero_sized_jobs_are_legal():

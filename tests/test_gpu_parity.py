@@ -397,7 +397,7 @@ def test_hist256_single_launch_in_subprocess():
     here = os.path.dirname(os.path.abspath(__file__))
     cmd = [sys.executable, "-m", "pytest", os.path.join(here, "test_gpu_parity.py"), "-q", "-m", "gpu",
            "-p", "no:cacheprovider", "-k",
-           "(hist256_ragged or config4 or mixed_small or repeated_flushes or config5) and not subprocess"]
+           "(hist256_ragged or config4 or mixed_small or repeated_flushes or config5) and not subprocess and not sgemm_full"]
     r = subprocess.run(cmd, env={**os.environ, "SVP_HIST_FUSED": "1"}, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
 

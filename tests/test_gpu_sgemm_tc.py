@@ -138,7 +138,8 @@ def test_tail_split_last_wave(int_inputs, residency, interleave):
     resident on one stream (one chunk, so the launch is alone): the slices read the
     staging arena."""
     specs = [W.JobSpec(v, "sgemm", M=1024, N=1024, K=1024, int_inputs=int_inputs) for v in range(18)]
-    specs.append(W.JobSpec(18, "sgemm", M=1000, N=1012, K=1000, alpha=1.5, beta=0.5, int_inputs=int_inputs))
+    # K <= 512: a beta != 0 job keeps the tensor cores only up to one K chunk (R23)
+    specs.append(W.JobSpec(18, "sgemm", M=1000, N=1012, K=500, alpha=1.5, beta=0.5, int_inputs=int_inputs))
     inputs = inputs_for(specs)
     ctx = svp.Context(num_gpus=1, sgemm_impl=svp.SGEMM_TF32BF16, interleave=interleave, arena_bytes=1 << 31)
     try:
@@ -161,3 +162,54 @@ def test_tail_split_last_wave(int_inputs, residency, interleave):
         ctx.close()
     for s, inp, got in zip(specs, inputs, outs):
         check_job(s, inp, got)
+
+
+@pytest.mark.parametrize("impl", [svp.SGEMM_TF32BF16, svp.SGEMM_3XTF32])
+def test_long_k_keeps_fp32_contract(impl):
+    """DESIGN R23: the tcgen05 fp32 accumulation loses ~1.7e-8 relative per accumulating MMA,
+    so long K runs in 512-k chunks folded into C with fp32 adds (beta == 0, VPs 0 and 1 on
+    the tensor cores) and a beta != 0 job past one chunk runs on FFMA (VP 2): the 1e-5
+    contract (componentwise and Frobenius) holds at K = 4096."""
+    specs = [W.JobSpec(0, "sgemm", M=384, N=256, K=4096), W.JobSpec(1, "sgemm", M=256, N=256, K=512),
+             W.JobSpec(2, "sgemm", M=256, N=384, K=4096, alpha=0.5, beta=2.0)]
+    inputs = inputs_for(specs)
+    outs, _, st = run_svp(specs, inputs, "device", sgemm_impl=impl)
+    assert st["groups"] == 2, st
+    want = oracle.run_jobs(specs, inputs)
+    for s, inp, got, w in zip(specs, inputs, outs, want):
+        check_job(s, inp, got, w)
+
+
+@pytest.mark.parametrize("impl", [svp.SGEMM_TF32BF16, svp.SGEMM_FFMA])
+@pytest.mark.parametrize("residency", ["device", "host"])
+def test_unaligned_shapes_and_buffers(impl, residency):
+    """K or N not a multiple of 4 and device buffers at a 4-B offset
+    (not 16-B aligned) -- the plain-load kernel's group -- next to aligned jobs of the same
+    flush (tensor-core / FFMA group), with alpha / beta and ragged tile edges, against the
+    oracle; integer inputs bit-exact."""
+    dims = [(130, 130, 66), (64, 68, 30), (1, 1, 1), (200, 136, 40), (97, 250, 333), (256, 256, 64)]
+    specs = [W.JobSpec(v, "sgemm", M=M, N=N, K=K, alpha=1.5, beta=-0.5 if v % 2 else 0.0,
+                       int_inputs=(v == 5), misalign=1 if (v == 3 and residency == "device") else 0)
+             for v, (M, N, K) in enumerate(dims)]
+    inputs = inputs_for(specs)
+    outs, _, st = run_svp(specs, inputs, residency, sgemm_impl=impl)
+    assert st["groups"] == 2, st
+    want = oracle.run_jobs(specs, inputs)
+    for s, inp, got, w in zip(specs, inputs, outs, want):
+        check_job(s, inp, got, w)
+
+
+@pytest.mark.parametrize("impl", [svp.SGEMM_TF32BF16, svp.SGEMM_3XTF32])
+@pytest.mark.parametrize("K", [2048, 4096])
+def test_same_sign_operands_keep_fp32_contract(impl, K):
+    """The accumulation bias (R23) is largest relative to the output when nothing cancels:
+    A, B ~ U[0, 1) make |C| = (|A||B|) so the componentwise bound IS a 1e-5 relative bound.
+    Without the K chunks the default split measured 2.04e-5 here at K = 2048
+    (profiles/r02/accuracy/); with them it must hold at the benched K and beyond."""
+    g = np.random.default_rng(3)
+    specs = [W.JobSpec(v, "sgemm", M=256, N=512, K=K) for v in range(2)]
+    inputs = [{"A": g.random((256, K), dtype=np.float32), "B": g.random((K, 512), dtype=np.float32)} for _ in specs]
+    outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl)
+    want = oracle.run_jobs(specs, inputs)
+    for s, inp, got, w in zip(specs, inputs, outs, want):
+        check_job(s, inp, got, w)

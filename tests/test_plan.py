@@ -76,6 +76,33 @@ def test_ragged_gemm_shapes_share_one_launch():
         assert ops[0]["flops"] == sum(2.0 * s * (s + 64) * (s // 2) for s in [128] * 4 + [256] * 2)
 
 
+@pytest.mark.parametrize("impl", [svp.SGEMM_TF32BF16, svp.SGEMM_3XTF32, svp.SGEMM_FFMA])
+def test_sgemm_accuracy_routing(impl):
+    """DESIGN R23: with the tensor-core splits' K-chunked accumulation (default 512 k per
+    chunk) a beta == 0 "sgemm" job stays on the tensor cores at any K; a beta != 0 job (not
+    chunked) past one chunk matches apart and runs on FFMA.  With FFMA every job coalesces
+    into one launch."""
+    with svp.Context(dry_run=True, sgemm_impl=impl) as c:
+        # the beta != 0 chunk limit: 512 k for TF32+2xBF16, 256 k for 3xTF32
+        lim = 256 if impl == svp.SGEMM_3XTF32 else 512
+        jobs = [(512, 0.0), (4096, 0.0), (lim, 1.0), (lim + 4, 1.0), (8192, 0.5)]
+        kid = c.kernel("sgemm")
+        for vp, (K, beta) in enumerate(jobs):
+            bufs = fake_bufs("sgemm", M=256, N=256, K=K, vp=vp)
+            bufs[0] = (bufs[0][0], 4 * 256 * 8192, bufs[0][2], bufs[0][3])  # room for every K
+            bufs[1] = (bufs[1][0], 4 * 256 * 8192, bufs[1][2], bufs[1][3])
+            if beta:
+                bufs[2] = (bufs[2][0], bufs[2][1], svp.DIR_INOUT, bufs[2][3])
+            c.submit(vp, kid, svp.args_sgemm(256, 256, K, 1.0, beta), bufs)
+        c.flush()
+        sg = [op for op in c.plan() if op["kind"] == svp.OP_KERNEL]
+        groups = sorted(sorted(op["vps"]) for op in sg)
+        if impl == svp.SGEMM_FFMA:
+            assert groups == [[0, 1, 2, 3, 4]]
+        else:
+            assert groups == [[0, 1, 2], [3, 4]]
+
+
 def test_no_coalescing_is_one_launch_per_job_in_submission_order():
     with svp.Context(dry_run=True, coalesce=False, interleave=False) as c:
         order = [5, 3, 9, 1]
@@ -194,18 +221,22 @@ def test_simulated_makespan_is_flowshop_of_plan_order():
 
 @pytest.mark.parametrize("seed", range(6))
 def test_johnson_plan_optimal_when_copy_bound(seed):
-    """Small host-resident mixes (PCIe-bound: Tk << Tin, Tout) -- Johnson's 3-machine
-    condition holds, so the planned order is optimal (brute force over all orders)."""
+    """Small host-resident mixes built to be PCIe-bound (Tk << Tin, Tout: vecadd / SAXPY /
+    Black-Scholes of >= 1 Mi elements, whose copies are ~8-16 B/elem at PCIe speed against
+    12-20 B/elem at HBM speed) -- Johnson's 3-machine condition holds on every seed (asserted,
+    so the test is never vacuous), and then the planned order is optimal (brute force over
+    all orders)."""
     g = np.random.default_rng(seed)
+    kinds = ("vecadd", "saxpy", "blackscholes")
     with svp.Context(dry_run=True, max_chunks=1) as c:
-        for vp in range(int(g.integers(2, 6))):
-            submit(c, vp, MIX[int(g.integers(0, 4))], n=int(g.integers(1, 40)) * 100000, mem=svp.MEM_HOST_PINNED)
+        for vp in range(int(g.integers(2, 7))):
+            submit(c, vp, kinds[int(g.integers(0, 3))], n=int(g.integers(10, 40)) * 100000, mem=svp.MEM_HOST_PINNED)
         c.flush()
         ops = c.plan()
         trip = _chunk_triples(ops)
         jobs = [tuple(v) for v in trip.values()]
-        if min(j[0] for j in jobs) >= max(j[1] for j in jobs) or min(j[2] for j in jobs) >= max(j[1] for j in jobs):
-            assert c.flush_stats()["sim_makespan_ns"] == pytest.approx(sched.best_makespan(jobs), rel=1e-9)
+        assert min(j[0] for j in jobs) >= max(j[1] for j in jobs) or min(j[2] for j in jobs) >= max(j[1] for j in jobs)
+        assert c.flush_stats()["sim_makespan_ns"] == pytest.approx(sched.best_makespan(jobs), rel=1e-9)
 
 
 def test_dispatcher_shards_vps_across_gpus():
