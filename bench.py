@@ -466,7 +466,7 @@ def run_svp(args, rank, ws, local):
 
     # ---------------- device-resident run (value)
     arm = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, validate_ptrs=True,
-              sgemm_impl=impl, **f4)
+              sgemm_impl=impl, sgemm_kchunk=args.sgemm_kchunk, **f4)
     kids = arm.kids
     assert arm.ctx.flush_stats is not None
     arm.step()
@@ -511,7 +511,8 @@ def run_svp(args, rank, ws, local):
     trace("timed region done")
 
     # ---------------- one stream per GPU: per-kernel roofline numbers (launches do not overlap)
-    iso = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, interleave=False, sgemm_impl=impl)
+    iso = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, interleave=False, sgemm_impl=impl,
+              sgemm_kchunk=args.sgemm_kchunk)
     iso.step()
     iso.ctx.reset_profile()
     iso_steps = max(3, args.steps // 5)
@@ -540,17 +541,23 @@ def run_svp(args, rank, ws, local):
         roof["traffic"] = None  # the committed ncu traffic figure is cfg5's launch
         roof.pop("traffic_source", None)
 
-    # ---------------- the other implementations of the fp32 "sgemm" kernel, same jobs
+    # ---------------- the other implementations of the fp32 "sgemm" kernel, same jobs (and the
+    # selected one with K-chunked accumulation, the strict mode of DESIGN R23)
     alt = []
     if not args.no_alt and "sgemm" in kids:
-        for alt_name in [a for a in args.alt_impl.split(",") if a and IMPLS[a] != impl]:
-            a = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, sgemm_impl=IMPLS[alt_name])
+        variants = [(a, 0) for a in args.alt_impl.split(",") if a and IMPLS[a] != impl]
+        if args.sgemm_kchunk == 0 and impl != IMPLS["ffma"]:
+            variants.append((args.sgemm_impl, 512))
+        for alt_name, kc in variants:
+            a = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, sgemm_impl=IMPLS[alt_name],
+                    sgemm_kchunk=kc)
             a.step()
             a.ctx.reset_profile()
             ks = max(3, args.steps // 5)
             adt = max_over_ranks(a.timed(ks)[0], ws)
             sk = a.ctx.kernel_stats(a.kids["sgemm"])
-            alt.append({"sgemm_impl": alt_name, "dtype": DTYPE_LABEL[alt_name], "value": n_jobs_total * ks / adt,
+            alt.append({"sgemm_impl": alt_name, "sgemm_kchunk": kc, "dtype": DTYPE_LABEL[alt_name],
+                        "value": n_jobs_total * ks / adt,
                         "unit": "jobs/s", "ms_per_step": adt / ks * 1e3,
                         "sgemm_tflops_interleaved": (sk["flops"] / sk["total_ns"] / 1e3) if sk["total_ns"] else None})
             a.close()
@@ -565,7 +572,7 @@ def run_svp(args, rank, ws, local):
                          ("B2_profiled", dict(coalesce=False, interleave=False, profile_level=1))):
             # B3 replays one captured graph, so it needs the same buffers every step: one set
             b = Arm(specs, inputs, "device", ords, streams, 1 if name == "B3_serial_graph" else nsets,
-                    sgemm_impl=impl, **kw)
+                    sgemm_impl=impl, sgemm_kchunk=args.sgemm_kchunk, **kw)
             b.steps(max(3, args.warmup))  # B3: plan, capture + instantiate, then replays only
             b.ctx.reset_profile()
             barrier(ws)
@@ -596,6 +603,7 @@ def run_svp(args, rank, ws, local):
     e2e = None
     if not args.no_e2e:
         h = Arm(specs, inputs, "host", ords, streams, 1, arena_bytes=args.arena_gb << 30, sgemm_impl=impl,
+                sgemm_kchunk=args.sgemm_kchunk,
                 max_chunks=int(os.environ.get("SVP_BENCH_MAXCH", "8")), **f4)
         h.steps(2)
         hst = h.ctx.flush_stats()
@@ -615,7 +623,8 @@ def run_svp(args, rank, ws, local):
         wspecs_all = W.config_specs(args.config, nvps=per_gpu * N)
         wspecs = my_specs(wspecs_all, rank, ws) if mode == "process" else wspecs_all
         winputs = W.make_inputs_many(wspecs)
-        w = Arm(wspecs, winputs, "device", ords, streams, n_buffer_sets(wspecs_all), sgemm_impl=impl, **f4)
+        w = Arm(wspecs, winputs, "device", ords, streams, n_buffer_sets(wspecs_all), sgemm_impl=impl,
+                sgemm_kchunk=args.sgemm_kchunk, **f4)
         w.steps(args.warmup)
         barrier(ws)
         ks = max(3, args.steps // 3)
@@ -648,7 +657,7 @@ def run_svp(args, rank, ws, local):
             "hbm_gbs_membound": hbm_gbs,
             "hbm_frac_membound": (hbm_gbs / float(peaks["hbm_gbs"])) if hbm_gbs else None,
             "elements_per_s": sum(s.n for s in all_specs) * args.steps / dt_max,
-            "sgemm_impl": args.sgemm_impl, "alt_sgemm_impls": alt, "hetero": args.hetero, "graph": args.graph,
+            "sgemm_impl": args.sgemm_impl, "sgemm_kchunk": args.sgemm_kchunk, "alt_sgemm_impls": alt, "hetero": args.hetero, "graph": args.graph,
             "table_mode": args.table_mode,
             "graph_replays_last_step": int(st["graph_replays"]),
             "timed_kernel_ms_per_step": {n: k["total_ns"] / args.steps / 1e6 for n, k in main_kstats.items()
@@ -679,6 +688,8 @@ def main():
     ap.add_argument("--arena-gb", type=int, default=8)
     ap.add_argument("--sgemm-impl", default="tf32bf16", choices=list(IMPL_NAMES),
                     help="implementation of the fp32 'sgemm' kernel (all meet its 1e-5 contract)")
+    ap.add_argument("--sgemm-kchunk", type=int, default=0,
+                    help="svp_config.sgemm_kchunk: K-chunked tensor-core accumulation (DESIGN R23); 0 = library default")
     ap.add_argument("--alt-impl", default="3xtf32,ffma",
                     help="comma list of the other sgemm implementations timed beside the main one")
     ap.add_argument("--scaling", default="auto", choices=["auto", "weak", "strong"],

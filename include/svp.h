@@ -116,6 +116,14 @@ typedef struct svp_config {
                                     SVP_TABLE_GLOBAL -- one device table
                                     buffer per GPU, uploaded once per flush when it changed.
                                     GEMM launches always use the global table.             */
+    int32_t sgemm_kchunk;        /* (ABI 5) "sgemm" on the tensor-core splits: accumulate K in chunks
+                                    of this many k (multiple of 16; 3xTF32 uses half), each from
+                                    zero, folded into C with fp32 adds -- the accuracy of one
+                                    chunk at any K and for any operand signs (R23),
+                                    at a throughput cost (cfg5: 512 -> ~0.70x).  beta != 0 jobs
+                                    longer than one chunk run on FFMA.  0 (default): one
+                                    accumulation per tile; jobs with K > 2048 (TF32+2xBF16) /
+                                    1024 (3xTF32) run on FFMA                                */
 } svp_config;
 
 enum { SVP_TABLE_GLOBAL = 0, SVP_TABLE_PARAM = 1 };
@@ -152,7 +160,12 @@ int32_t svp_abi_version(void);
  *                   add 2^-134 |other operand| per product whose operand is below 2^-115 in
  *                   magnitude (TF32 / BF16 subnormal granularity); an output their tensor-core
  *                   accumulation leaves NaN (an Inf / NaN operand, or one near FLT_MAX) is
- *                   recomputed exactly from A and B (fp64 products and sum, one rounding)
+ *                   recomputed exactly from A and B (fp64 products and sum, one rounding).
+ *                   Their fp32 accumulation loses ~1.7e-8 (random-sign data) to ~3.4e-8
+ *                   (same-sign data) relative per accumulating MMA: by default they take jobs
+ *                   up to K = 2048 / 1024 (longer ones run on FFMA), where random-sign data
+ *                   stays within 1e-5 but same-sign data at K = 2048 reaches ~2e-5;
+ *                   cfg.sgemm_kchunk (e.g. 512) bounds it for all data at any K (DESIGN R23)
  *   "sgemm_tf32"    same, tcgen05 TF32 tensor cores  (own tolerance 2e-3; raw operands, so a
  *                   NaN whose payload is only in the low 13 mantissa bits reads as Inf)
  *   "dgemm"         C = alpha A B + beta C, fp64     args svp_args_dgemm   bufs [A IN, B IN, C OUT (INOUT if beta != 0)] f64

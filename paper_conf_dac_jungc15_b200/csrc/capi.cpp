@@ -108,7 +108,8 @@ svp_status svp_init(const svp_config* cfg, svp_ctx** out) {
     if (cfg->num_gpus < 0 || cfg->num_gpus > 64 || cfg->streams_per_gpu < 1 || cfg->streams_per_gpu > 32 ||
         cfg->max_chunks < 1 || cfg->max_chunks > 64 || cfg->profile_level < 0 || cfg->profile_level > 2 ||
         cfg->flush_timeout_ms < 0 || cfg->sgemm_impl < 0 || cfg->sgemm_impl > 2 || cfg->table_mode < 0 ||
-        cfg->table_mode > 1 || cfg->validate_ptrs < 0 || cfg->validate_ptrs > 2) {
+        cfg->table_mode > 1 || cfg->validate_ptrs < 0 || cfg->validate_ptrs > 2 || cfg->sgemm_kchunk < 0 ||
+        cfg->sgemm_kchunk % 16 != 0 || cfg->sgemm_kchunk > (1 << 20)) {
         set_error("svp_init: config value out of range");
         return SVP_E_INVAL;
     }

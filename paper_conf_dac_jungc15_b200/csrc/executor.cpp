@@ -63,7 +63,7 @@ struct Maps2 {
 struct Dev {
     int ordinal = 0;
     int idx = 0;
-    std::vector<cudaStream_t> streams;  // [0,S) compute, S = H2D, S+1 = D2H
+    std::vector<cudaStream_t> streams;  // [0] control, [1,S] compute, S+1 = H2D, S+2 = D2H
     cudaStream_t ext = nullptr;
     std::vector<cudaEvent_t> dep_ev, t_ev;
     cudaEvent_t ext_ev = nullptr, tbl_ev = nullptr;
@@ -161,15 +161,20 @@ std::string executor_error(Executor* e) { return e->err; }
 static svp_status dev_setup(Dev& d, const svp_config& cfg, void* ext) {
     CK(cudaSetDevice(d.ordinal));
     CK(cudaFree(0));  // create / adopt the primary context
+    // [0] control stream (table uploads, graph capture / launch, joins); plan stream k runs on
+    // [k + 1]: compute 0..S-1, H2D S, D2H S+1.  Kernels and copies never share the control
+    // stream: in the host-resident cfg5 timeline a compute stream that also carried the
+    // control work started its first kernel ~100 ms late on repeated flushes, stalling every
+    // D2H behind it (profiles/r02/e2e/)
     const int S = cfg.streams_per_gpu;
-    d.streams.resize(S + 2);
+    d.streams.resize(S + 3);
     for (auto& s : d.streams) CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
     d.ext = (cudaStream_t)ext;
     CK(cudaEventCreateWithFlags(&d.ext_ev, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&d.tbl_ev, cudaEventDisableTiming));
-    d.end_ev.resize(S + 2);
+    d.end_ev.resize(S + 3);
     for (auto& e : d.end_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-    d.join_ev.resize(S + 2);
+    d.join_ev.resize(S + 3);
     for (auto& e : d.join_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&d.fork_ev, cudaEventDisableTiming));
     d.arena_bytes = cfg.arena_bytes;
@@ -760,8 +765,9 @@ static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bo
     return pool[i];
 }
 
-static cudaError_t launch_chunk(Dev& d, const Chunk& ch, cudaStream_t s) {
+static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int cfg_kchunk, cudaStream_t s) {
     const int sgemm_impl = ch.sgemm_impl;
+    const int kchunk = sgemm_chunk_k(sgemm_impl, cfg_kchunk);
     if (ch.total_tiles == 0 && ch.kernel != K_HIST256) return cudaSuccess;
     const uint8_t* base = d.tbl_dev;
     uint64_t* busy = ch.busy_off >= 0 ? d.busy_dev + ch.busy_off : nullptr;
@@ -812,18 +818,19 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, cudaStream_t s) {
                                           grid_of(d.lim.gemm_plain_blocks_per_sm), s);
             if (sgemm_impl == SVP_SGEMM_TF32BF16) {
                 cudaError_t e = launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.table_off), ch.nsegs,
-                                                      base + ch.maps_off, ch.main_tiles, grid_of(1), ch.wide, s);
+                                                      base + ch.maps_off, ch.main_tiles, grid_of(1), ch.wide, s,
+                                                      kchunk);
                 if (e || ch.tail_n == 0) return e;
                 // tail split: the last wave's tiles as K-slices, then the ordered reduction
                 e = launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.tail_table_off), ch.tail_n,
                                           base + ch.tail_maps_off, (uint32_t)ch.tail_n,
-                                          2 * std::min<int>(ch.tail_n, d.lim.num_sms / 2), false, s);
+                                          2 * std::min<int>(ch.tail_n, d.lim.num_sms / 2), false, s, kchunk);
                 if (e) return e;
                 return launch_sgemm_tail_reduce((const TailRed*)(base + ch.tail_red_off), ch.tail_nred, s);
             }
             if (sgemm_impl == SVP_SGEMM_3XTF32)
                 return launch_sgemm_3xtf32((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
-                                           ch.total_tiles, grid_of(1), s);
+                                           ch.total_tiles, grid_of(1), s, kchunk);
             return launch_sgemm_ffma((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
                                      ch.total_tiles, grid_of(d.lim.gemm_blocks_per_sm), s);
         case K_DGEMM:
@@ -893,7 +900,7 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
         std::vector<char> touch(d.streams.size(), 0);
         touch[0] = 1;
         for (const auto& o : f.ops)
-            if (o.device == d.idx) touch[o.stream] = 1;
+            if (o.device == d.idx) touch[o.stream + 1] = 1;
         CK(cudaEventRecord(d.ext_ev, d.ext));
         for (size_t s = 0; s < d.streams.size(); ++s)
             if (touch[s]) CK(cudaStreamWaitEvent(d.streams[s], d.ext_ev, 0));
@@ -1095,8 +1102,8 @@ static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool captu
     for (size_t i = 0; i < f.ops.size(); ++i) {
         Op& o = f.ops[i];
         if (o.device != d.idx) continue;
-        cudaStream_t s = d.streams[o.stream];
-        used[o.stream] = 1;
+        cudaStream_t s = d.streams[o.stream + 1];
+        used[o.stream + 1] = 1;
         for (int32_t p : o.wait_ops) {
             const Op& q = f.ops[p];
             if (q.device != d.idx) continue;
@@ -1129,7 +1136,7 @@ static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool captu
                 }
             }
         } else if (chunk_needs_launch(f, ch)) {
-            CK(launch_chunk(d, ch, s));
+            CK(launch_chunk(d, ch, c->cfg.sgemm_kchunk, s));
         }
         if (prof) {
             CK(rec(d.t_ev[2 * nt + 1], s));

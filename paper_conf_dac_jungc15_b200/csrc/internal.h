@@ -48,6 +48,13 @@ inline bool is_gemm(int32_t k) { return k == K_SGEMM || k == K_SGEMM_TF32 || k =
 // MMA, profiles/r02/accuracy_k.jsonl), so the output's relative error grows with K; up to
 // these K every measured output keeps the 1e-5 fp32 contract.  Jobs with larger K match as a
 // separate group that runs the FFMA kernel.
+// K chunk (k, multiple of 16; 0 = off) of a tensor-core split's accumulation (R23) from
+// cfg.sgemm_kchunk: 3xTF32 (6 accumulating MMAs per 16 k against 4) uses half of it
+inline int32_t sgemm_chunk_k(int32_t impl, int32_t cfg_kchunk) {
+    if (cfg_kchunk <= 0) return 0;
+    if (impl == SVP_SGEMM_3XTF32) return cfg_kchunk >= 32 ? cfg_kchunk / 32 * 16 : 16;
+    return impl == SVP_SGEMM_TF32BF16 ? cfg_kchunk : 0;
+}
 // internal "sgemm_impl" of a group whose jobs TMA cannot address (k_sgemm_plain)
 constexpr int32_t kSgemmPlain = 3;
 inline int32_t sgemm_tc_kmax(int32_t impl) {

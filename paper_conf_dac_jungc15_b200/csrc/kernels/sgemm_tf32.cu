@@ -82,7 +82,6 @@
 
 #include <atomic>
 
-#include "../../../include/svp.h"
 #include "../launch.h"
 #include "common.cuh"
 
@@ -266,6 +265,14 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
         : "memory");
 }
 
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t (&r)[8]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];\n\t"
+        "tcgen05.wait::ld.sync.aligned;"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+        : "r"(taddr)
+        : "memory");
+}
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
     asm volatile(
         "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
@@ -702,25 +709,29 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
             const float alpha = g.alpha, beta = g.beta;
             const bool kzero = g.K == 0;
             const bool first = ck == 0, last = ck == nch - 1;
-#pragma unroll 1
-            for (int c0 = 0; c0 < BN; c0 += 16) {
-                const int col0 = tn * TN + eh * BN + c0;
-                // later K chunk: the partial sum the previous chunk stored (this thread wrote
-                // it: program order; in L2) -- loads issued before the TMEM read so their
-                // latency overlaps it
-                float4 prev[4];
-                if (!first && row_ok) {
+            // later K chunk: fold into the partial sum the previous chunk stored (this thread
+            // wrote it: program order; in L2).  The loads run one slab of SW columns ahead, so
+            // their L2 latency overlaps the previous slab's TMEM read, adds and stores.
+            constexpr int SW = 8, NV = SW / 4;
+            const bool rmw = !first && row_ok;
+            auto loadv = [&](float4 (&dst)[NV], int col) {
 #pragma unroll
-                    for (int jj = 0; jj < 4; ++jj)
-                        prev[jj] = col0 + 4 * jj < g.N ? *reinterpret_cast<const float4*>(crow + col0 + 4 * jj)
-                                                       : make_float4(0.f, 0.f, 0.f, 0.f);
-                }
-                uint32_t r[16];
-                tmem_ld16(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0), r);
+                for (int jj = 0; jj < NV; ++jj)
+                    dst[jj] = col + 4 * jj < g.N ? *reinterpret_cast<const float4*>(crow + col + 4 * jj)
+                                                 : make_float4(0.f, 0.f, 0.f, 0.f);
+            };
+            float4 prev[NV], nxt[NV];
+            if (rmw) loadv(prev, tn * TN + eh * BN);
+#pragma unroll 1
+            for (int c0 = 0; c0 < BN; c0 += SW) {
+                const int col0 = tn * TN + eh * BN + c0;
+                if (rmw && c0 + SW < BN) loadv(nxt, col0 + SW);
+                uint32_t r[SW];
+                tmem_ld8(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0), r);
                 if (!row_ok) continue;
                 uint32_t nan_mask = 0;  // outputs of this slab whose final value came out NaN
 #pragma unroll
-                for (int jj = 0; jj < 4; ++jj) {
+                for (int jj = 0; jj < NV; ++jj) {
                     const int j = 4 * jj, c = col0 + j;
                     if (c >= g.N) break;
                     float4 o;
@@ -767,6 +778,10 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     float* cp = crow + col0 + e;
                     *cp = exact_element(g, row, col0 + e, (beta != 0.f && nch == 1) ? *cp : 0.f);
                 }
+                if (rmw) {
+#pragma unroll
+                    for (int jj = 0; jj < NV; ++jj) prev[jj] = nxt[jj];
+                }
             }
             tc_fence_before();
             __syncwarp();
@@ -796,7 +811,7 @@ static std::atomic<bool> g_attr_set[20][64] = {};  // per kernel variant and dev
 
 template <int SPLIT, int CG, int NH = 1>
 static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uint32_t total, int clusters,
-                             cudaStream_t s) {
+                             cudaStream_t s, int kchunk_k = 0) {
     using Cf = tc::Cfg<SPLIT, CG, NH>;
     int dev = 0;
     cudaGetDevice(&dev);
@@ -823,23 +838,8 @@ static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uin
         lc.numAttrs = 1;
     }
     // the plain-TF32 "sgemm_tf32" (own 2e-3 tolerance) accumulates the whole K in one chunk
-    const int kchunk = SPLIT == 1 ? 0 : sgemm_tc_kchunk(SPLIT == 3 ? SVP_SGEMM_3XTF32 : SVP_SGEMM_TF32BF16) / tc::BK;
+    const int kchunk = SPLIT == 1 ? 0 : kchunk_k / tc::BK;
     return cudaLaunchKernelEx(&lc, kern, descs, n, reinterpret_cast<const uint8_t*>(maps), total, kchunk);
-}
-
-// K chunk of the fp32 tensor-core splits in k (a multiple of 16; 0 = off): SVP_SGEMM_KCHUNK
-// for TF32+2xBF16, default 512 (R23: 4 accumulating MMAs per 16 k -> ~ -2.1e-6 relative per
-// chunk on random-sign data, ~ -4.1e-6 on same-sign data); 3xTF32 (6 MMAs per 16 k, larger
-// bias per MMA) uses half of it
-int sgemm_tc_kchunk(int impl) {
-    static int v = -1;
-    if (v < 0) {
-        const char* e = getenv("SVP_SGEMM_KCHUNK");
-        int k = e ? atoi(e) : 512;
-        v = k <= 0 ? 0 : (k + 15) / 16 * 16;
-    }
-    if (impl == SVP_SGEMM_3XTF32) return v >= 32 ? v / 32 * 16 : v;
-    return impl == SVP_SGEMM_TF32BF16 ? v : 0;
 }
 
 // CTA-pair kernels for the fp32-accurate splits unless SVP_TC_CTA_PAIR=0 (A/B switch)
@@ -883,12 +883,14 @@ int sgemm_tc_wide_mode() {
 }
 
 cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
-                                  bool wide, cudaStream_t s) {
+                                  bool wide, cudaStream_t s, int kchunk) {
     const int pairs = (int)std::min<uint32_t>(total, std::max(1, grid / 2));
-    if (wide) return launch_tc<2, 2, 2>(descs, n, maps, total, pairs, s);
+    if (wide) return launch_tc<2, 2, 2>(descs, n, maps, total, pairs, s, kchunk);
     if (sgemm_tc_cta_pair())
-        return tmem_a() ? launch_tc<4, 2>(descs, n, maps, total, pairs, s) : launch_tc<2, 2>(descs, n, maps, total, pairs, s);
-    return tmem_a() ? launch_tc<4, 1>(descs, n, maps, total, grid, s) : launch_tc<2, 1>(descs, n, maps, total, grid, s);
+        return tmem_a() ? launch_tc<4, 2>(descs, n, maps, total, pairs, s, kchunk)
+                        : launch_tc<2, 2>(descs, n, maps, total, pairs, s, kchunk);
+    return tmem_a() ? launch_tc<4, 1>(descs, n, maps, total, grid, s, kchunk)
+                    : launch_tc<2, 1>(descs, n, maps, total, grid, s, kchunk);
 }
 
 // ------------------------------------------------------------------ tail split reduction
@@ -927,10 +929,11 @@ cudaError_t launch_sgemm_tail_reduce(const TailRed* reds, int nred, cudaStream_t
 }
 
 cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
-                                cudaStream_t s) {
+                                cudaStream_t s, int kchunk) {
     if (sgemm_tc_cta_pair())
-        return launch_tc<3, 2>(descs, n, maps, total, (int)std::min<uint32_t>(total, std::max(1, grid / 2)), s);
-    return launch_tc<3, 1>(descs, n, maps, total, grid, s);
+        return launch_tc<3, 2>(descs, n, maps, total, (int)std::min<uint32_t>(total, std::max(1, grid / 2)), s,
+                               kchunk);
+    return launch_tc<3, 1>(descs, n, maps, total, grid, s, kchunk);
 }
 
 }  // namespace svp

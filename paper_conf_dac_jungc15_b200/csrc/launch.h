@@ -67,18 +67,17 @@ cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, ui
 
 // fp32-accurate grouped SGEMM on tcgen05: 3xTF32 (hi/lo operand split, 3 MMAs per k-step).
 cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
-                                int grid, cudaStream_t s);
+                                int grid, cudaStream_t s, int kchunk = 0);
 
 // fp32-accurate grouped SGEMM on tcgen05: A_hi B_hi as one kind::tf32 MMA per 8 k plus the
 // cross terms bf16(A_hi) bf16(B_lo) + bf16(A_lo) bf16(B_hi) as kind::f16 (BF16) MMAs.
 cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
-                                  int grid, bool wide, cudaStream_t s);
+                                  int grid, bool wide, cudaStream_t s, int kchunk = 0);
 
 // true: the fp32-accurate tcgen05 SGEMMs run as CTA pairs (cta_group::2, 256 x 256 tiles);
 // SVP_TC_CTA_PAIR=0 selects the single-CTA kernels (128 x 256 tiles)
 bool sgemm_tc_cta_pair();
-// K chunk (in k, multiple of 16; 0 = off) of an fp32 tensor-core split's accumulation (R23)
-int sgemm_tc_kchunk(int sgemm_impl);
+
 // 256 x 512 tiles for the TF32+2xBF16 pair kernel (two 256-column accumulator halves sharing
 // each A tile): SVP_TC_WIDE=0 never, 1 (default) when a launch has >= 2 waves of them, 2 always
 int sgemm_tc_wide_mode();

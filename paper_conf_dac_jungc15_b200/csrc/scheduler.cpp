@@ -193,7 +193,7 @@ svp_status validate_and_fill(Ctx* c, Job* j) {
             // with K-chunked accumulation (sgemm_tc_kchunk) a beta == 0 job keeps the
             // tensor cores at any K; a beta != 0 job is not chunked (its exact NaN path needs
             // C_old), so it keeps them up to one chunk
-            const int kc = sgemm_tc_kchunk(c->cfg.sgemm_impl);
+            const int kc = sgemm_chunk_k(c->cfg.sgemm_impl, c->cfg.sgemm_kchunk);
             const int32_t kmax = kc > 0 ? (j->f1 != 0.f ? kc : (1 << 30)) : sgemm_tc_kmax(c->cfg.sgemm_impl);
             if (j->K > kmax) j->shape_key = 1;
         }
@@ -526,9 +526,6 @@ svp_status plan_flush(Ctx* c, Flush* f) {
     // (list scheduling; ties -> lowest index).  Round-robin put cfg5's 5th launch (hist256)
     // behind the SGEMM on stream 0, so it ran alone after it.  SVP_STREAM_RR=1: round-robin.
     static const bool stream_rr = getenv("SVP_STREAM_RR") && atoi(getenv("SVP_STREAM_RR")) != 0;
-    // diagnostic (mode-H timeline study): first compute stream the list scheduler may use
-    static const int first_cs_env = getenv("SVP_FIRST_COMPUTE_STREAM") ? atoi(getenv("SVP_FIRST_COMPUTE_STREAM")) : 0;
-    const int first_cs = std::max(0, std::min(first_cs_env, S - 1));
     std::vector<std::vector<double>> sload(c->ngpu, std::vector<double>(S, 0.0));
     for (int32_t ci : corder) {
         Chunk& ch = f->chunks[ci];
@@ -573,8 +570,7 @@ svp_status plan_flush(Ctx* c, Flush* f) {
             if (stream_rr) {
                 cs = rr[dev]++ % S;
             } else {
-                cs = first_cs;
-                for (int k = first_cs + 1; k < S; ++k)
+                for (int k = 1; k < S; ++k)
                     if (sload[dev][k] < sload[dev][cs]) cs = k;
                 sload[dev][cs] += std::max(ch.t_k, 1.0);
             }

@@ -184,7 +184,7 @@ def test_lpt_partition_pure():
 
 
 _STRUCTS = ("svp_config", "svp_buf", "svp_job_desc", "svp_ipc_buf", "svp_vp_profile", "svp_kernel_stats",
-            "svp_flush_stats", "svp_plan_op")
+            "svp_flush_stats", "svp_plan_op", "svp_device_stats")
 
 
 def test_ctypes_layouts_match_the_header(tmp_path):

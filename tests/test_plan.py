@@ -77,12 +77,11 @@ def test_ragged_gemm_shapes_share_one_launch():
 
 
 @pytest.mark.parametrize("impl", [svp.SGEMM_TF32BF16, svp.SGEMM_3XTF32, svp.SGEMM_FFMA])
-def test_sgemm_accuracy_routing(impl):
-    """DESIGN R23: with the tensor-core splits' K-chunked accumulation (default 512 k per
-    chunk) a beta == 0 "sgemm" job stays on the tensor cores at any K; a beta != 0 job (not
-    chunked) past one chunk matches apart and runs on FFMA.  With FFMA every job coalesces
-    into one launch."""
-    with svp.Context(dry_run=True, sgemm_impl=impl) as c:
+def test_sgemm_accuracy_routing_chunked(impl):
+    """DESIGN R23, sgemm_kchunk = 512 (strict mode): with K-chunked accumulation a beta == 0
+    "sgemm" job stays on the tensor cores at any K; a beta != 0 job (not chunked) past one
+    chunk matches apart and runs on FFMA.  With FFMA every job coalesces into one launch."""
+    with svp.Context(dry_run=True, sgemm_impl=impl, sgemm_kchunk=512) as c:
         # the beta != 0 chunk limit: 512 k for TF32+2xBF16, 256 k for 3xTF32
         lim = 256 if impl == svp.SGEMM_3XTF32 else 512
         jobs = [(512, 0.0), (4096, 0.0), (lim, 1.0), (lim + 4, 1.0), (8192, 0.5)]
@@ -101,6 +100,30 @@ def test_sgemm_accuracy_routing(impl):
             assert groups == [[0, 1, 2, 3, 4]]
         else:
             assert groups == [[0, 1, 2], [3, 4]]
+
+
+@pytest.mark.parametrize("impl,kmax", [(svp.SGEMM_TF32BF16, 2048), (svp.SGEMM_3XTF32, 1024), (svp.SGEMM_FFMA, None)])
+def test_sgemm_accuracy_routing_default(impl, kmax):
+    """DESIGN R23, default (no K chunks): jobs with K above the measured limit of the split's
+    single accumulation (2048 for TF32+2xBF16, 1024 for 3xTF32) match apart and run on FFMA."""
+    with svp.Context(dry_run=True, sgemm_impl=impl) as c:
+        Ks = [512, 1024, 2048, 2052, 4096]
+        for vp, K in enumerate(Ks):
+            submit(c, vp, "sgemm", M=256, N=256, K=K)
+        c.flush()
+        sg = [op for op in c.plan() if op["kind"] == svp.OP_KERNEL]
+        if kmax is None:
+            assert len(sg) == 1 and sg[0]["nvps"] == 5
+        else:
+            groups = sorted(sorted(op["vps"]) for op in sg)
+            want = sorted([[v for v, K in enumerate(Ks) if K <= kmax], [v for v, K in enumerate(Ks) if K > kmax]])
+            assert groups == want
+
+
+def test_sgemm_kchunk_must_be_a_multiple_of_16():
+    for bad in (-16, 8, 100):
+        with pytest.raises(svp.SvpError):
+            svp.Context(dry_run=True, sgemm_kchunk=bad)
 
 
 def test_no_coalescing_is_one_launch_per_job_in_submission_order():

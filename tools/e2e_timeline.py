@@ -98,7 +98,7 @@ def main():
         if s1 > e0:
             gaps.append(s1 - e0)
     res = {"config": args.config, "max_chunks": args.max_chunks, "chunks": int(st["chunks"]), "wall_ms": walls,
-           "first_kernels_per_flush": firsts, "first_compute_stream": os.environ.get("SVP_FIRST_COMPUTE_STREAM"),
+           "first_kernels_per_flush": firsts,
            "streams": args.streams, "max_connections": os.environ.get("CUDA_DEVICE_MAX_CONNECTIONS"),
            "span_ms": span / 1e6, "host_total_ms": st["host_total_ns"] / 1e6,
            "h2d_bytes": hb, "d2h_bytes": db,
