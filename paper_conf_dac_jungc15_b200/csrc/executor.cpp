@@ -463,6 +463,12 @@ static bool ew_dynamic_order() {
     return on;
 }
 
+// SVP_HIST_DYN=0: hist256 with the static blocked tile ranges instead of dynamic chunks.
+static bool hist_dynamic_order() {
+    static const bool on = !(getenv("SVP_HIST_DYN") && atoi(getenv("SVP_HIST_DYN")) == 0);
+    return on;
+}
+
 // SVP_HIST_FUSED=1: hist256 as ONE launch with a self-resetting per-launch scratch (the
 // last CTA of each VP writes its counts) instead of a zeroing kernel + the accumulating
 // launch.  Off by default: alone it was 2 us (4 %) faster per cfg5 hist launch, but the
@@ -792,7 +798,8 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int cfg_kchunk, cudaStr
             case K_EW_MIX:
                 return launch_ew_param(ch.kernel, p, ch.nsegs, ch.total_tiles, grid_of(d.lim.mix_blocks_per_sm), s, busy, sched);
             case K_HIST256:
-                return launch_hist256_param(p, ch.nsegs, ch.total_tiles, grid_of(d.lim.hist_blocks_per_sm), s, busy, hscr);
+                return launch_hist256_param(p, ch.nsegs, ch.total_tiles, grid_of(d.lim.hist_blocks_per_sm), s, busy, hscr,
+                                            sched);
         }
         return cudaErrorInvalidValue;
     }
@@ -811,7 +818,7 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int cfg_kchunk, cudaStr
                                  grid_of(d.lim.mix_blocks_per_sm), s, busy, sched);
         case K_HIST256:
             return launch_hist256((const SegDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
-                                  grid_of(d.lim.hist_blocks_per_sm), s, busy, hscr);
+                                  grid_of(d.lim.hist_blocks_per_sm), s, busy, hscr, sched);
         case K_SGEMM:
             if (sgemm_impl == kSgemmPlain)
                 return launch_sgemm_plain((const GemmDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
@@ -979,6 +986,10 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             const bool alone = !c->cfg.interleave || kernels_in_level[ch.level] == 1;
             if (ew_dynamic_order() && alone && (ch.kernel == K_BLACKSCHOLES || ch.kernel == K_EW_MIX) &&
                 ch.total_tiles > 0)
+                ch.sched_slot = (int32_t)nslot++;
+            // hist256: dynamic chunk order whenever it is not the single-launch form (its CTAs
+            // run at data-dependent speeds: replicated vs shared-table counting)
+            if (hist_dynamic_order() && ch.kernel == K_HIST256 && !hist_single_launch() && ch.total_tiles > 0)
                 ch.sched_slot = (int32_t)nslot++;
         }
         // single-launch hist256 scratch (SVP_HIST_FUSED=0: zeroing kernel + launch)

@@ -170,8 +170,18 @@ struct SegCache {
     }
 };
 
+// Dynamic tile order (sched != null; not with the single-launch scratch form): the producer
+// claims chunks of kHistChunk consecutive tiles from the launch's self-resetting counter pair
+// sched[0..1] and tells the consumers each staged tile's id through stile[stage]; a CTA whose
+// data runs slower (uniform bytes: one ATOMS per byte into the replicas) takes fewer chunks
+// than one whose data is skewed (the aggregated shared table is ~1.3x faster), instead of
+// every CTA owning a fixed 1/grid of the tiles.
+constexpr uint32_t kHistChunk = 8;
+constexpr uint32_t kHistEnd = 0xFFFFFFFFu;
+
 __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int nsegs, uint32_t total,
-                                          unsigned long long* __restrict__ busy, uint32_t* __restrict__ scratch) {
+                                          unsigned long long* __restrict__ busy, uint32_t* __restrict__ scratch,
+                                          uint32_t* __restrict__ sched) {
     extern __shared__ __align__(128) uint8_t hsm[];
     uint8_t* ring = hsm;                                                         // [stages][tile]
     uint32_t* h = reinterpret_cast<uint32_t*>(hsm + kHistStages * kHistTile);     // [256][32] + h1[256]
@@ -179,6 +189,8 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
     uint64_t* full = reinterpret_cast<uint64_t*>(h + kHistBins * 33);
     uint64_t* empty = full + kHistStages;
     __shared__ uint32_t last_flag;
+    __shared__ uint32_t stile[kHistStages];  // dynamic order: tile id of each stage
+    const bool dyn = sched != nullptr && scratch == nullptr;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     uint32_t* arrive = scratch ? scratch + (size_t)nsegs * kHistBins : nullptr;
     if (scratch) {
@@ -206,7 +218,20 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
         if (lane == 0) {
             uint32_t it = 0;
             SegCache sc;
-            for (uint32_t t = t0; t < t1; ++t, ++it) {
+            uint32_t t = t0, tend = t1;
+            if (dyn) {
+                const uint32_t c = atomicAdd(sched, 1u);
+                t = min(total, c * kHistChunk);
+                tend = min(total, t + kHistChunk);
+            }
+            for (;; ++t, ++it) {
+                if (t >= tend) {
+                    if (!dyn || t >= total) break;
+                    const uint32_t c = atomicAdd(sched, 1u);
+                    t = min(total, c * kHistChunk);
+                    tend = min(total, t + kHistChunk);
+                    if (t >= tend) break;
+                }
                 const int s = it % kHistStages;
                 const uint32_t ph = (it / kHistStages) & 1;
                 const SegDesc& sd = segs[sc.get(segs, nsegs, total, t)];
@@ -214,6 +239,7 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
                 bool vec;
                 tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, kHistTile, e0, e1, vec);
                 mbar_wait(&empty[s], ph ^ 1);
+                stile[s] = t;  // published by the arrive below (release) to the consumers' wait
                 if (vec) {
                     mbar_expect_tx(&full[s], kHistTile);
                     bulk_g2s(ring + s * kHistTile, reinterpret_cast<const uint8_t*>(sd.ptr[0]) + e0, kHistTile, &full[s]);
@@ -231,6 +257,13 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
                     }
                 }
             }
+            if (dyn) {  // end marker: one more stage carrying no tile
+                const int s = it % kHistStages;
+                const uint32_t ph = (it / kHistStages) & 1;
+                mbar_wait(&empty[s], ph ^ 1);
+                stile[s] = kHistEnd;
+                mbar_arrive(&full[s]);
+            }
         }
         return;  // no CTA-wide barrier after this point
     }
@@ -241,7 +274,20 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
     uint32_t* cur_counts = nullptr;
     uint32_t it = 0;
     SegCache sc;
-    for (uint32_t t = t0; t < t1; ++t, ++it) {
+    for (uint32_t t = t0;; ++t, ++it) {
+        const int s = it % kHistStages;
+        const uint32_t ph = (it / kHistStages) & 1;
+        // profile_level 2: thread 0's cycles per tile (from the wait for the stage to the
+        // release) -> busy[segment]
+        const long long c0 = (busy && threadIdx.x == 0) ? clock64() : 0;
+        if (dyn) {
+            mbar_wait(&full[s], ph);
+            t = stile[s];
+            if (t == kHistEnd) break;
+        } else {
+            if (t >= t1) break;
+            mbar_wait(&full[s], ph);
+        }
         const int si = sc.get(segs, nsegs, total, t);
         const SegDesc& sd = segs[si];
         if (si != cur) {
@@ -258,12 +304,6 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
         int64_t e0, e1;
         bool vec;
         tile_range(sd.n, sd.shift, sd.flags, t - sd.tile_begin, kHistTile, e0, e1, vec);
-        const int s = it % kHistStages;
-        const uint32_t ph = (it / kHistStages) & 1;
-        // profile_level 2: thread 0's cycles per tile (from the wait for the stage to the
-        // release) -> busy[segment]
-        const long long c0 = (busy && threadIdx.x == 0) ? clock64() : 0;
-        mbar_wait(&full[s], ph);
         if (vec) {
             const uint4* st = reinterpret_cast<const uint4*>(ring + s * kHistTile) + threadIdx.x;
             uint4 r[kHistVec];
@@ -333,17 +373,23 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
         else
             hist_flush(h, cur_counts);
     }
+    // dynamic order: the last CTA out (every producer has claimed past the end by then)
+    // leaves the counter pair zeroed for the next launch on this slot
+    if (dyn && threadIdx.x == 0 && atomicAdd(sched + 1, 1u) == gridDim.x - 1) {
+        sched[0] = 0;
+        sched[1] = 0;
+    }
 }
 
 __global__ void __launch_bounds__(kHistBlock) k_hist256(const SegDesc* __restrict__ segs, int nsegs, uint32_t total,
-                                                        unsigned long long* busy, uint32_t* scratch) {
-    hist_body(segs, nsegs, total, busy, scratch);
+                                                        unsigned long long* busy, uint32_t* scratch, uint32_t* sched) {
+    hist_body(segs, nsegs, total, busy, scratch, sched);
 }
 template <int CAP>
 __global__ void __launch_bounds__(kHistBlock) k_hist256_p(const __grid_constant__ SegParamT<CAP> p, int nsegs,
                                                           uint32_t total, unsigned long long* busy,
-                                                          uint32_t* scratch) {
-    hist_body(p.s, nsegs, total, busy, scratch);
+                                                          uint32_t* scratch, uint32_t* sched) {
+    hist_body(p.s, nsegs, total, busy, scratch, sched);
 }
 
 template <int CAP>
@@ -372,7 +418,7 @@ static cudaError_t hist_attr() {
 }
 
 cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s, uint64_t* busy,
-                           uint32_t* scratch) {
+                           uint32_t* scratch, uint32_t* sched) {
     if (nsegs <= 0) return cudaSuccess;
     cudaError_t e;
     if (!scratch) {
@@ -382,13 +428,13 @@ cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total, int g
     }
     if ((e = hist_attr())) return e;
     k_hist256<<<grid, kHistBlock, kHistSmem, s>>>(segs, nsegs, total, reinterpret_cast<unsigned long long*>(busy),
-                                                  scratch);
+                                                  scratch, sched);
     return cudaGetLastError();
 }
 
 template <int CAP>
 static cudaError_t launch_hist256_param_cap(const SegDesc* segs, int nsegs, uint32_t total, int grid,
-                                            cudaStream_t s, uint64_t* busy, uint32_t* scratch) {
+                                            cudaStream_t s, uint64_t* busy, uint32_t* scratch, uint32_t* sched) {
     SegParamT<CAP> p;
     memcpy(p.s, segs, (size_t)nsegs * sizeof(SegDesc));
     cudaError_t e;
@@ -399,17 +445,18 @@ static cudaError_t launch_hist256_param_cap(const SegDesc* segs, int nsegs, uint
     }
     if ((e = hist_attr_p<CAP>())) return e;
     k_hist256_p<CAP><<<grid, kHistBlock, kHistSmem, s>>>(p, nsegs, total, reinterpret_cast<unsigned long long*>(busy),
-                                                         scratch);
+                                                         scratch, sched);
     return cudaGetLastError();
 }
 
 cudaError_t launch_hist256_param(const SegDesc* segs, int nsegs, uint32_t total, int grid, cudaStream_t s,
-                                 uint64_t* busy, uint32_t* scratch) {
+                                 uint64_t* busy, uint32_t* scratch, uint32_t* sched) {
     if (nsegs <= 0) return cudaSuccess;
     if (param_full_block() && nsegs <= kParamSegs)
-        return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s, busy, scratch);
-    if (nsegs <= 16) return launch_hist256_param_cap<16>(segs, nsegs, total, grid, s, busy, scratch);
-    if (nsegs <= kParamSegs) return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s, busy, scratch);
+        return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s, busy, scratch, sched);
+    if (nsegs <= 16) return launch_hist256_param_cap<16>(segs, nsegs, total, grid, s, busy, scratch, sched);
+    if (nsegs <= kParamSegs)
+        return launch_hist256_param_cap<kParamSegs>(segs, nsegs, total, grid, s, busy, scratch, sched);
     return cudaErrorInvalidValue;
 }
 

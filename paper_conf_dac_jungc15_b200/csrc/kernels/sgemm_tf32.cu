@@ -366,11 +366,11 @@ __device__ __forceinline__ float exact_element(const GemmDesc& g, int i, int j, 
 // (measured -1.66e-8 relative per accumulating MMA), so a tile's K range is cut into chunks
 // of `kchunk` 16-k blocks, each accumulated from zero in its own TMEM accumulator (the two
 // accumulators ping-pong between chunks as they do between tiles) and folded into C by the
-// epilogue with IEEE fp32 adds (chunk 0 stores alpha * acc, later chunks C += alpha * acc):
-// the output's relative bias is then that of ONE chunk, whatever K is.  Only for beta == 0
-// (a beta != 0 job keeps C_old for its exact NaN path; the executor routes those with
-// K > the chunk to the FFMA kernel).  Producer, MMA issuer and epilogue all walk the same
-// (tile, chunk) units.
+// epilogue with IEEE fp32 adds (chunk 0 stores alpha * acc, later chunks add alpha * acc with
+// red.global.add.v4.f32): the output's relative bias is then that of ONE chunk, whatever K
+// is.  Only for beta == 0 (a beta != 0 job keeps C_old for its exact NaN path; the executor
+// routes those with K > the chunk to the FFMA kernel).  Producer, MMA issuer and epilogue all
+// walk the same (tile, chunk) units.
 __device__ __forceinline__ int tc_chunks(const GemmDesc& g, int KB, int kchunk) {
     return (kchunk > 0 && g.beta == 0.f && KB > kchunk) ? (KB + kchunk - 1) / kchunk : 1;
 }
@@ -692,6 +692,7 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
         const int eh = (NH == 2 && warp >= 14) ? 1 : 0;
         const uint32_t acc_empty_leader = CG == 2 ? map_to(&acc_empty[0], 0) : 0;
         uint32_t tile_i = 0;  // (tile, chunk) units, as the MMA issuer counts them
+        uint32_t nan_slabs = 0;  // K chunks: 8-column slabs of this row whose partial had a NaN
         for (uint32_t t = cl; t < total; t += ncl) {
           const int v = find_tile_owner(descs, n, t);
           const GemmDesc& g = descs[v];
@@ -709,27 +710,22 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
             const float alpha = g.alpha, beta = g.beta;
             const bool kzero = g.K == 0;
             const bool first = ck == 0, last = ck == nch - 1;
-            // later K chunk: fold into the partial sum the previous chunk stored (this thread
-            // wrote it: program order; in L2).  The loads run one slab of SW columns ahead, so
-            // their L2 latency overlaps the previous slab's TMEM read, adds and stores.
+            // K chunks (nch > 1, beta == 0): chunk 0 stores alpha * acc, later chunks fold their
+            // alpha * acc into C with fire-and-forget vector reductions (red.global.add.v4.f32:
+            // IEEE round-to-nearest in L2, applied in program order per address), so no chunk
+            // boundary waits on a read of the partial sum.  A chunk whose accumulator holds a NaN
+            // (an Inf / NaN operand, or one near FLT_MAX, in its k range) marks the 8-column slab;
+            // after the last chunk those slabs are read back and their NaN outputs recomputed
+            // exactly (rare path).
             constexpr int SW = 8, NV = SW / 4;
-            const bool rmw = !first && row_ok;
-            auto loadv = [&](float4 (&dst)[NV], int col) {
-#pragma unroll
-                for (int jj = 0; jj < NV; ++jj)
-                    dst[jj] = col + 4 * jj < g.N ? *reinterpret_cast<const float4*>(crow + col + 4 * jj)
-                                                 : make_float4(0.f, 0.f, 0.f, 0.f);
-            };
-            float4 prev[NV], nxt[NV];
-            if (rmw) loadv(prev, tn * TN + eh * BN);
+            if (first) nan_slabs = 0;
 #pragma unroll 1
             for (int c0 = 0; c0 < BN; c0 += SW) {
                 const int col0 = tn * TN + eh * BN + c0;
-                if (rmw && c0 + SW < BN) loadv(nxt, col0 + SW);
                 uint32_t r[SW];
                 tmem_ld8(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0), r);
                 if (!row_ok) continue;
-                uint32_t nan_mask = 0;  // outputs of this slab whose final value came out NaN
+                uint32_t nan_mask = 0;  // single-chunk tiles: outputs whose value came out NaN
 #pragma unroll
                 for (int jj = 0; jj < NV; ++jj) {
                     const int j = 4 * jj, c = col0 + j;
@@ -740,14 +736,20 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     o.z = kzero ? 0.f : alpha * __uint_as_float(r[j + 2]);
                     o.w = kzero ? 0.f : alpha * __uint_as_float(r[j + 3]);
                     float4* dst = reinterpret_cast<float4*>(crow + c);
+                    if (nch > 1) {
+                        const float o4 = o.x + o.y + o.z + o.w;
+                        if (o4 != o4) nan_slabs |= 1u << (c0 / SW);
+                        if (first) {
+                            *dst = o;  // a partial sum, folded into by the next chunks: keep it in L2
+                        } else {
+                            asm volatile("red.global.add.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(dst), "f"(o.x),
+                                         "f"(o.y), "f"(o.z), "f"(o.w)
+                                         : "memory");
+                        }
+                        continue;
+                    }
                     float4 old = make_float4(0.f, 0.f, 0.f, 0.f);
-                    if (!first) {
-                        old = prev[jj];
-                        o.x += old.x;
-                        o.y += old.y;
-                        o.z += old.z;
-                        o.w += old.w;
-                    } else if (beta != 0.f) {
+                    if (beta != 0.f) {
                         old = __ldcs(dst);
                         o.x = __fmaf_rn(beta, old.x, o.x);
                         o.y = __fmaf_rn(beta, old.y, o.y);
@@ -756,31 +758,36 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     }
                     // IEEE special values (R20): an Inf / NaN operand (its low part x - h is NaN),
                     // or a finite one whose TF32 head rounds past FLT_MAX, leaves NaN in every
-                    // accumulator it reaches (and, across K chunks, in the partial sum).  In the
-                    // last chunk those outputs keep C_old (chunked: beta == 0, C_old unused) and
-                    // are recomputed exactly below (rare path, after r[] is dead).
-                    if (last) {
-                        const float o4 = o.x + o.y + o.z + o.w;
-                        if (!kzero && o4 != o4) {
-                            if (isnan(o.x)) { nan_mask |= 1u << (j + 0); o.x = old.x; }
-                            if (isnan(o.y)) { nan_mask |= 1u << (j + 1); o.y = old.y; }
-                            if (isnan(o.z)) { nan_mask |= 1u << (j + 2); o.z = old.z; }
-                            if (isnan(o.w)) { nan_mask |= 1u << (j + 3); o.w = old.w; }
-                        }
-                        __stcs(dst, o);  // st.global.cs: C's final value
-                    } else {
-                        *dst = o;  // a partial sum, re-read by the next chunk: keep it in L2
+                    // accumulator it reaches.  Those outputs keep C_old for now and are recomputed
+                    // exactly below (rare path, after r[] is dead).
+                    const float o4 = o.x + o.y + o.z + o.w;
+                    if (!kzero && o4 != o4) {
+                        if (isnan(o.x)) { nan_mask |= 1u << (j + 0); o.x = old.x; }
+                        if (isnan(o.y)) { nan_mask |= 1u << (j + 1); o.y = old.y; }
+                        if (isnan(o.z)) { nan_mask |= 1u << (j + 2); o.z = old.z; }
+                        if (isnan(o.w)) { nan_mask |= 1u << (j + 3); o.w = old.w; }
                     }
+                    __stcs(dst, o);  // st.global.cs: C is written once
                 }
                 while (nan_mask) {
                     const int e = __ffs(nan_mask) - 1;
                     nan_mask &= nan_mask - 1;
                     float* cp = crow + col0 + e;
-                    *cp = exact_element(g, row, col0 + e, (beta != 0.f && nch == 1) ? *cp : 0.f);
+                    *cp = exact_element(g, row, col0 + e, beta != 0.f ? *cp : 0.f);
                 }
-                if (rmw) {
-#pragma unroll
-                    for (int jj = 0; jj < NV; ++jj) prev[jj] = nxt[jj];
+            }
+            if (last && nch > 1 && nan_slabs && row_ok) {
+                // this thread's reductions to these addresses precede the loads (same thread,
+                // same address: program order)
+                while (nan_slabs) {
+                    const int sl = __ffs(nan_slabs) - 1;
+                    nan_slabs &= nan_slabs - 1;
+                    const int col0 = tn * TN + eh * BN + sl * SW;
+#pragma unroll 1
+                    for (int e = 0; e < SW && col0 + e < g.N; ++e) {
+                        float* cp = crow + col0 + e;
+                        if (isnan(*(volatile float*)cp)) *cp = exact_element(g, row, col0 + e, 0.f);
+                    }
                 }
             }
             tc_fence_before();

@@ -46,12 +46,14 @@ cudaError_t launch_ew_param(int kind, const SegDesc* segs, int nsegs, uint32_t t
                             uint64_t* busy = nullptr, uint32_t* sched = nullptr);
 bool param_full_block();  // SVP_PARAM_FULL=1: always the kParamSegs block (A/B knob)
 cudaError_t launch_hist256_param(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s,
-                                 uint64_t* busy = nullptr, uint32_t* scratch = nullptr);
+                                 uint64_t* busy = nullptr, uint32_t* scratch = nullptr, uint32_t* sched = nullptr);
 // hist256: without `scratch`, a zeroing kernel then the accumulating launch; with
 // `scratch` (nsegs * 257 zeroed u32, left zeroed) one launch whose last CTA per VP writes
 // the VP's counts.
+// `sched` (2 zeroed u32, left zeroed): dynamic tile order (chunks of 8 tiles claimed by each
+// CTA's producer), ignored with `scratch`.
 cudaError_t launch_hist256(const SegDesc* segs, int nsegs, uint32_t total_tiles, int grid, cudaStream_t s,
-                        uint64_t* busy = nullptr, uint32_t* scratch = nullptr);
+                        uint64_t* busy = nullptr, uint32_t* scratch = nullptr, uint32_t* sched = nullptr);
 
 // Grouped SGEMM (fp32 FFMA, TMA-staged).  maps = 2*n CUtensorMap (A_i, B_i), 64-B aligned.
 cudaError_t launch_sgemm_ffma(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
