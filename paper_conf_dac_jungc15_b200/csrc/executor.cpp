@@ -516,6 +516,9 @@ static svp_status plan_sgemm_tail(Executor* e, Dev& d, Flush& f, Chunk& ch, std:
     for (const auto& sb : subs) K = std::max(K, f.jobs[ch.jobs[sb.k]].K);
     int S = std::min<int>(P / (int)subs.size(), K / 64);
     if (S < 2) return SVP_OK;
+    // K-chunked mode (R23): the slices run as single accumulations, so each must fit in a chunk
+    const int kc = sgemm_chunk_k(ch.sgemm_impl, e->c->cfg.sgemm_kchunk);
+    if (kc > 0 && (K + S - 1) / S > kc) return SVP_OK;
     size_t ws_need = 0;
     for (const auto& sb : subs) ws_need += (size_t)S * sb.rows * sb.cols;
     if (ws_need > kTailWsFloats) return SVP_OK;
@@ -589,7 +592,6 @@ static svp_status plan_sgemm_tail(Executor* e, Dev& d, Flush& f, Chunk& ch, std:
     ch.tail_n = (int32_t)pd.size();
     ch.tail_nred = (int32_t)rd.size();
     ch.kernel_launches = 3;
-    (void)e;
     return SVP_OK;
 }
 
@@ -745,6 +747,35 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
             ch.kernel_launches = 1;
             ch.main_tiles = tiles;
             ch.tail_n = ch.tail_nred = 0;
+            ch.cmaps_off = -1;
+            if (variant && ch.kernel == K_SGEMM) {
+                // one TMA map of C per VP: the epilogue of beta == 0 tiles writes C by TMA (and
+                // folds K chunks with TMA reduce-add, R23); cached per (C, M, N)
+                const size_t coff = align_up(tbl.size(), 128);
+                tbl.resize(coff + nj * 128);
+                for (size_t k = 0; k < nj; ++k) {
+                    const Job& j = f.jobs[ch.jobs[k]];
+                    uint8_t* mp = tbl.data() + coff + k * 128;
+                    float* Cp = (float*)ch.staged[k * SVP_MAX_BUFS + 2];
+                    if ((int64_t)j.M * j.N > 0 && j.K > 0) {
+                        MapKey key{(uint64_t)Cp, 0, j.M, j.N, 0, 7};
+                        auto it = d.map_cache.find(key);
+                        if (it == d.map_cache.end()) {
+                            Maps2 m;
+                            if (encode_c_map(m.a, Cp, j.M, j.N) != 0) {
+                                d.err = "cuTensorMapEncodeTiled failed for an sgemm C map";
+                                return SVP_E_CUDA;
+                            }
+                            if (d.map_cache.size() > 4096) d.map_cache.clear();
+                            it = d.map_cache.emplace(key, m).first;
+                        }
+                        memcpy(mp, it->second.a, 128);
+                    } else {
+                        memset(mp, 0, 128);
+                    }
+                }
+                ch.cmaps_off = (int64_t)coff;
+            }
             // tail split only for a launch that has the GPU to itself: co-running with the
             // memory-bound launches of an interleaved level, the last wave's idle pairs are
             // not idle GPU time, and the power-capped step measured 0.7-2 % slower with the
@@ -824,20 +855,22 @@ static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int cfg_kchunk, cudaStr
                 return launch_sgemm_plain((const GemmDesc*)(base + ch.table_off), ch.nsegs, ch.total_tiles,
                                           grid_of(d.lim.gemm_plain_blocks_per_sm), s);
             if (sgemm_impl == SVP_SGEMM_TF32BF16) {
+                const void* cmaps = ch.cmaps_off >= 0 ? (const void*)(base + ch.cmaps_off) : nullptr;
                 cudaError_t e = launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.table_off), ch.nsegs,
                                                       base + ch.maps_off, ch.main_tiles, grid_of(1), ch.wide, s,
-                                                      kchunk);
+                                                      kchunk, cmaps);
                 if (e || ch.tail_n == 0) return e;
                 // tail split: the last wave's tiles as K-slices, then the ordered reduction
                 e = launch_sgemm_tf32bf16((const GemmDesc*)(base + ch.tail_table_off), ch.tail_n,
                                           base + ch.tail_maps_off, (uint32_t)ch.tail_n,
-                                          2 * std::min<int>(ch.tail_n, d.lim.num_sms / 2), false, s, kchunk);
+                                          2 * std::min<int>(ch.tail_n, d.lim.num_sms / 2), false, s);
                 if (e) return e;
                 return launch_sgemm_tail_reduce((const TailRed*)(base + ch.tail_red_off), ch.tail_nred, s);
             }
             if (sgemm_impl == SVP_SGEMM_3XTF32)
                 return launch_sgemm_3xtf32((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
-                                           ch.total_tiles, grid_of(1), s, kchunk);
+                                           ch.total_tiles, grid_of(1), s, kchunk,
+                                           ch.cmaps_off >= 0 ? (const void*)(base + ch.cmaps_off) : nullptr);
             return launch_sgemm_ffma((const GemmDesc*)(base + ch.table_off), ch.nsegs, base + ch.maps_off,
                                      ch.total_tiles, grid_of(d.lim.gemm_blocks_per_sm), s);
         case K_DGEMM:

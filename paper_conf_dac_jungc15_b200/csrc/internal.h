@@ -113,6 +113,7 @@ struct Chunk {
     uint32_t total_tiles = 0;
     int32_t nsegs = 0;
     uint64_t maps_off = 0;          // sgemm: tensor maps offset
+    int64_t cmaps_off = -1;         // tensor-core sgemm with K chunks: C tensor maps (R23), else -1
     bool small_tiles = false;       // dgemm: 32x32 tile variant (launch under 2 waves of 64x64)
     bool wide = false;              // sgemm TF32+2xBF16: 256x512 pair tiles (>= 2 waves of them)
     bool param = false;             // table_mode param: the SegDesc table goes by value

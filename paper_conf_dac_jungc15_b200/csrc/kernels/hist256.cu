@@ -218,19 +218,20 @@ __device__ __forceinline__ void hist_body(const SegDesc* __restrict__ segs, int 
         if (lane == 0) {
             uint32_t it = 0;
             SegCache sc;
-            uint32_t t = t0, tend = t1;
+            uint32_t t = t0, tend = t1, next = 0;
             if (dyn) {
                 const uint32_t c = atomicAdd(sched, 1u);
+                next = atomicAdd(sched, 1u);  // claimed one chunk ahead: its latency hides
                 t = min(total, c * kHistChunk);
                 tend = min(total, t + kHistChunk);
             }
             for (;; ++t, ++it) {
                 if (t >= tend) {
                     if (!dyn || t >= total) break;
-                    const uint32_t c = atomicAdd(sched, 1u);
-                    t = min(total, c * kHistChunk);
+                    t = min(total, next * kHistChunk);
                     tend = min(total, t + kHistChunk);
                     if (t >= tend) break;
+                    next = atomicAdd(sched, 1u);
                 }
                 const int s = it % kHistStages;
                 const uint32_t ph = (it / kHistStages) & 1;

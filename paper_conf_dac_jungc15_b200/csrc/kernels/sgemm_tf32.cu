@@ -123,7 +123,11 @@ struct Cfg {
     static constexpr int kAcc = (SPLIT == 4 || NH == 2) ? 1 : 2;  // accumulator sets (NH x 256 cols each)
     static constexpr int kTaCol = 256;                     // SPLIT 4: A ring, 16 cols per stage
     static_assert(SPLIT != 4 || kTaCol + 16 * kStages <= kTmemCols, "TMEM");
-    static constexpr size_t kBarOff = (size_t)kStages * kStageBytes;
+    // K-chunk folds (R23): a 32 x 32 fp32 staging slab (128-B swizzled) per epilogue warp,
+    // written back into C by TMA store (first chunk) / TMA reduce-add (later chunks)
+    static constexpr int kEpiWarps = 4 * NH;
+    static constexpr size_t kStagingOff = (size_t)kStages * kStageBytes;  // 1024-B aligned
+    static constexpr size_t kBarOff = kStagingOff + (size_t)kEpiWarps * 4096;
     static constexpr size_t kSmem = 1024 + kBarOff + 256;
     static constexpr int kMmaM = BM * CG;
     static_assert(kSmem <= 227 * 1024, "shared memory");
@@ -371,6 +375,20 @@ __device__ __forceinline__ float exact_element(const GemmDesc& g, int i, int j, 
 // is.  Only for beta == 0 (a beta != 0 job keeps C_old for its exact NaN path; the executor
 // routes those with K > the chunk to the FFMA kernel).  Producer, MMA issuer and epilogue all
 // walk the same (tile, chunk) units.
+__device__ __forceinline__ void tma_store_2d(const void* tmap, int32_t c0, int32_t c1, const void* smem_src) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(tmap), "r"(c0),
+                 "r"(c1), "r"(smem_u32(smem_src))
+                 : "memory");
+}
+__device__ __forceinline__ void tma_reduce_add_2d(const void* tmap, int32_t c0, int32_t c1, const void* smem_src) {
+    asm volatile("cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.bulk_group [%0, {%1, %2}], [%3];" ::"l"(tmap),
+                 "r"(c0), "r"(c1), "r"(smem_u32(smem_src))
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
 __device__ __forceinline__ int tc_chunks(const GemmDesc& g, int KB, int kchunk) {
     return (kchunk > 0 && g.beta == 0.f && KB > kchunk) ? (KB + kchunk - 1) / kchunk : 1;
 }
@@ -378,7 +396,7 @@ __device__ __forceinline__ int tc_chunks(const GemmDesc& g, int KB, int kchunk) 
 template <int SPLIT, int CG, int NH>
 __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
     k_sgemm_tc(const GemmDesc* __restrict__ descs, int n, const uint8_t* __restrict__ maps, uint32_t total,
-               int kchunk) {
+               int kchunk, const uint8_t* __restrict__ cmaps) {
     using namespace tc;
     using C = Cfg<SPLIT, CG, NH>;
     constexpr int TN = BN * NH;  // tile width in N per CTA pair (or CTA)
@@ -710,22 +728,65 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
             const float alpha = g.alpha, beta = g.beta;
             const bool kzero = g.K == 0;
             const bool first = ck == 0, last = ck == nch - 1;
-            // K chunks (nch > 1, beta == 0): chunk 0 stores alpha * acc, later chunks fold their
-            // alpha * acc into C with fire-and-forget vector reductions (red.global.add.v4.f32:
-            // IEEE round-to-nearest in L2, applied in program order per address), so no chunk
-            // boundary waits on a read of the partial sum.  A chunk whose accumulator holds a NaN
-            // (an Inf / NaN operand, or one near FLT_MAX, in its k range) marks the 8-column slab;
-            // after the last chunk those slabs are read back and their NaN outputs recomputed
-            // exactly (rare path).
+            // beta == 0 tiles (with C maps) leave through TMA: full 128-B rows per store instead
+            // of 16-B pieces of 32 different rows per warp store instruction
+            const bool tma_epi = cmaps != nullptr && beta == 0.f && !kzero;
+            // TMA epilogue (beta == 0): each 32 x 32 block of alpha * acc goes through this
+            // warp's swizzled smem slab to C by TMA -- a store for chunk 0, a reduce-add (IEEE
+            // round-to-nearest, performed by L2) for later chunks -- so a chunk boundary costs
+            // the TMEM read and the slab writes, never a read of the partial sum.  The issuing
+            // lane waits for its previous chunk's bulk group to complete before reducing into
+            // the same addresses.  A chunk whose accumulator holds a NaN (an Inf / NaN operand,
+            // or one near FLT_MAX, in its k range) marks the 8-column slab; after the last
+            // chunk those slabs are read back and their NaN outputs recomputed exactly.
             constexpr int SW = 8, NV = SW / 4;
             if (first) nan_slabs = 0;
+            if (tma_epi) {
+                uint8_t* slab = smem + C::kStagingOff + (size_t)(warp < 8 ? warp - 4 : warp - 10) * 4096;
+                const void* cmap = cmaps + (size_t)v * 128;
+                const int row0 = tm * C::kMmaM + (int)rank * BM + q * 32;
+                if (lane == 0) bulk_wait0();  // the previous (tile, chunk) unit's writes landed
+#pragma unroll 1
+                for (int c0 = 0; c0 < BN; c0 += 32) {
+                    if (lane == 0) bulk_wait_read0();  // the slab is free again
+                    __syncwarp();
+#pragma unroll 1
+                    for (int sl = 0; sl < 4; ++sl) {
+                        uint32_t r[SW];
+                        tmem_ld8(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0 + sl * SW), r);
+#pragma unroll
+                        for (int jj = 0; jj < NV; ++jj) {
+                            const int j = 4 * jj;
+                            float4 o;
+                            o.x = alpha * __uint_as_float(r[j + 0]);
+                            o.y = alpha * __uint_as_float(r[j + 1]);
+                            o.z = alpha * __uint_as_float(r[j + 2]);
+                            o.w = alpha * __uint_as_float(r[j + 3]);
+                            const float o4 = o.x + o.y + o.z + o.w;
+                            if (o4 != o4) nan_slabs |= 1u << ((c0 + sl * SW) / SW);
+                            const int ck16 = 2 * sl + jj;  // 16-B chunk of this lane's 128-B row
+                            *reinterpret_cast<float4*>(slab + lane * 128 + ((ck16 ^ (lane & 7)) << 4)) = o;
+                        }
+                    }
+                    fence_proxy_async();
+                    __syncwarp();
+                    if (lane == 0) {
+                        const int col = tn * TN + eh * BN + c0;
+                        if (first) tma_store_2d(cmap, col, row0, slab);
+                        else tma_reduce_add_2d(cmap, col, row0, slab);
+                        bulk_commit();
+                    }
+                }
+                if (lane == 0) bulk_wait_read0();
+                __syncwarp();
+            } else {
 #pragma unroll 1
             for (int c0 = 0; c0 < BN; c0 += SW) {
                 const int col0 = tn * TN + eh * BN + c0;
                 uint32_t r[SW];
                 tmem_ld8(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0), r);
                 if (!row_ok) continue;
-                uint32_t nan_mask = 0;  // single-chunk tiles: outputs whose value came out NaN
+                uint32_t nan_mask = 0;  // outputs whose value came out NaN
 #pragma unroll
                 for (int jj = 0; jj < NV; ++jj) {
                     const int j = 4 * jj, c = col0 + j;
@@ -736,18 +797,6 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     o.z = kzero ? 0.f : alpha * __uint_as_float(r[j + 2]);
                     o.w = kzero ? 0.f : alpha * __uint_as_float(r[j + 3]);
                     float4* dst = reinterpret_cast<float4*>(crow + c);
-                    if (nch > 1) {
-                        const float o4 = o.x + o.y + o.z + o.w;
-                        if (o4 != o4) nan_slabs |= 1u << (c0 / SW);
-                        if (first) {
-                            *dst = o;  // a partial sum, folded into by the next chunks: keep it in L2
-                        } else {
-                            asm volatile("red.global.add.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(dst), "f"(o.x),
-                                         "f"(o.y), "f"(o.z), "f"(o.w)
-                                         : "memory");
-                        }
-                        continue;
-                    }
                     float4 old = make_float4(0.f, 0.f, 0.f, 0.f);
                     if (beta != 0.f) {
                         old = __ldcs(dst);
@@ -776,9 +825,15 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     *cp = exact_element(g, row, col0 + e, beta != 0.f ? *cp : 0.f);
                 }
             }
-            if (last && nch > 1 && nan_slabs && row_ok) {
-                // this thread's reductions to these addresses precede the loads (same thread,
-                // same address: program order)
+            }
+            if (last && tma_epi && __any_sync(0xFFFFFFFFu, nan_slabs != 0)) {
+                // the warp's bulk writes of every chunk have landed (wait_group 0) and are made
+                // visible to this proxy's loads before the read-back
+                if (lane == 0) bulk_wait0();
+                __syncwarp();
+                asm volatile("fence.proxy.async.global;" ::: "memory");
+            }
+            if (last && tma_epi && nan_slabs && row_ok) {
                 while (nan_slabs) {
                     const int sl = __ffs(nan_slabs) - 1;
                     nan_slabs &= nan_slabs - 1;
@@ -800,6 +855,7 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
         }
     }
     // ---------------------------------------------------------------- teardown
+    if (warp >= 4 && ((warp < 8) || (NH == 2 && warp >= 14)) && lane == 0) bulk_wait0();  // epilogue TMA writes
     tc_fence_before();
     __syncthreads();
     if constexpr (CG == 2) cluster_sync_all();  // neither CTA frees TMEM / exits under the peer
@@ -818,7 +874,7 @@ static std::atomic<bool> g_attr_set[20][64] = {};  // per kernel variant and dev
 
 template <int SPLIT, int CG, int NH = 1>
 static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uint32_t total, int clusters,
-                             cudaStream_t s, int kchunk_k = 0) {
+                             cudaStream_t s, int kchunk_k = 0, const void* cmaps = nullptr) {
     using Cf = tc::Cfg<SPLIT, CG, NH>;
     int dev = 0;
     cudaGetDevice(&dev);
@@ -845,8 +901,9 @@ static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uin
         lc.numAttrs = 1;
     }
     // the plain-TF32 "sgemm_tf32" (own 2e-3 tolerance) accumulates the whole K in one chunk
-    const int kchunk = SPLIT == 1 ? 0 : kchunk_k / tc::BK;
-    return cudaLaunchKernelEx(&lc, kern, descs, n, reinterpret_cast<const uint8_t*>(maps), total, kchunk);
+    const int kchunk = (SPLIT == 1 || !cmaps) ? 0 : kchunk_k / tc::BK;
+    return cudaLaunchKernelEx(&lc, kern, descs, n, reinterpret_cast<const uint8_t*>(maps), total, kchunk,
+                              reinterpret_cast<const uint8_t*>(cmaps));
 }
 
 // CTA-pair kernels for the fp32-accurate splits unless SVP_TC_CTA_PAIR=0 (A/B switch)
@@ -890,14 +947,14 @@ int sgemm_tc_wide_mode() {
 }
 
 cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
-                                  bool wide, cudaStream_t s, int kchunk) {
+                                  bool wide, cudaStream_t s, int kchunk, const void* cmaps) {
     const int pairs = (int)std::min<uint32_t>(total, std::max(1, grid / 2));
-    if (wide) return launch_tc<2, 2, 2>(descs, n, maps, total, pairs, s, kchunk);
+    if (wide) return launch_tc<2, 2, 2>(descs, n, maps, total, pairs, s, kchunk, cmaps);
     if (sgemm_tc_cta_pair())
-        return tmem_a() ? launch_tc<4, 2>(descs, n, maps, total, pairs, s, kchunk)
-                        : launch_tc<2, 2>(descs, n, maps, total, pairs, s, kchunk);
-    return tmem_a() ? launch_tc<4, 1>(descs, n, maps, total, grid, s, kchunk)
-                    : launch_tc<2, 1>(descs, n, maps, total, grid, s, kchunk);
+        return tmem_a() ? launch_tc<4, 2>(descs, n, maps, total, pairs, s, kchunk, cmaps)
+                        : launch_tc<2, 2>(descs, n, maps, total, pairs, s, kchunk, cmaps);
+    return tmem_a() ? launch_tc<4, 1>(descs, n, maps, total, grid, s, kchunk, cmaps)
+                    : launch_tc<2, 1>(descs, n, maps, total, grid, s, kchunk, cmaps);
 }
 
 // ------------------------------------------------------------------ tail split reduction
@@ -936,11 +993,11 @@ cudaError_t launch_sgemm_tail_reduce(const TailRed* reds, int nred, cudaStream_t
 }
 
 cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total, int grid,
-                                cudaStream_t s, int kchunk) {
+                                cudaStream_t s, int kchunk, const void* cmaps) {
     if (sgemm_tc_cta_pair())
         return launch_tc<3, 2>(descs, n, maps, total, (int)std::min<uint32_t>(total, std::max(1, grid / 2)), s,
-                               kchunk);
-    return launch_tc<3, 1>(descs, n, maps, total, grid, s, kchunk);
+                               kchunk, cmaps);
+    return launch_tc<3, 1>(descs, n, maps, total, grid, s, kchunk, cmaps);
 }
 
 }  // namespace svp

@@ -69,12 +69,15 @@ cudaError_t launch_sgemm_tf32(const GemmDesc* descs, int n, const void* maps, ui
 
 // fp32-accurate grouped SGEMM on tcgen05: 3xTF32 (hi/lo operand split, 3 MMAs per k-step).
 cudaError_t launch_sgemm_3xtf32(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
-                                int grid, cudaStream_t s, int kchunk = 0);
+                                int grid, cudaStream_t s, int kchunk = 0, const void* cmaps = nullptr);
 
 // fp32-accurate grouped SGEMM on tcgen05: A_hi B_hi as one kind::tf32 MMA per 8 k plus the
 // cross terms bf16(A_hi) bf16(B_lo) + bf16(A_lo) bf16(B_hi) as kind::f16 (BF16) MMAs.
+// kchunk (k) > 0 with cmaps (one 128-B CUtensorMap of C per VP, box 32 x 32, 128-B swizzle):
+// K-chunked accumulation folded into C by TMA store / reduce-add (R23)
 cudaError_t launch_sgemm_tf32bf16(const GemmDesc* descs, int n, const void* maps, uint32_t total_tiles,
-                                  int grid, bool wide, cudaStream_t s, int kchunk = 0);
+                                  int grid, bool wide, cudaStream_t s, int kchunk = 0, const void* cmaps = nullptr);
+int encode_c_map(void* mapC, const float* C, int M, int N);
 
 // true: the fp32-accurate tcgen05 SGEMMs run as CTA pairs (cta_group::2, 256 x 256 tiles);
 // SVP_TC_CTA_PAIR=0 selects the single-CTA kernels (128 x 256 tiles)

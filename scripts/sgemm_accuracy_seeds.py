@@ -17,6 +17,7 @@ from gpu_common import run_svp  # noqa: E402
 from paper_conf_dac_jungc15_b200 import svp  # noqa: E402
 
 K = int(os.environ.get("ACC_K", "2048"))
+KCHUNK = int(os.environ.get("ACC_KCHUNK", "0"))  # svp_config.sgemm_kchunk (strict mode, R23)
 MN = 512
 for dist in ("u11", "u01", "normal"):
     for seed in range(4):
@@ -31,13 +32,13 @@ for dist in ("u11", "u01", "normal"):
         inputs = [{"A": mk(MN, K), "B": mk(K, MN)} for _ in specs]
         want = oracle.run_jobs(specs, inputs, threads=2)
         for name, impl in (("tf32bf16", svp.SGEMM_TF32BF16), ("ffma", svp.SGEMM_FFMA)):
-            outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl)
+            outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl, sgemm_kchunk=KCHUNK)
             for i in range(2):
                 G = outs[i]["C"].astype(np.float64)
                 O = want[i]["C"].astype(np.float64)
                 A, B = inputs[i]["A"].astype(np.float64), inputs[i]["B"].astype(np.float64)
                 d = G - O
-                print(json.dumps({"impl": name, "dist": dist, "seed": seed, "vp": i, "K": K,
+                print(json.dumps({"impl": name, "dist": dist, "seed": seed, "vp": i, "K": K, "kchunk": KCHUNK,
                                   "frob_rel": float(np.linalg.norm(d) / np.linalg.norm(O)),
                                   "bias_beta": float((d * O).sum() / (O * O).sum()),
                                   "max_comp_ratio": float((np.abs(d) / (np.abs(A) @ np.abs(B))).max())}), flush=True)
