@@ -545,9 +545,9 @@ def run_svp(args, rank, ws, local):
     # selected one with K-chunked accumulation, the strict mode of DESIGN R23)
     alt = []
     if not args.no_alt and "sgemm" in kids:
-        variants = [(a, 0) for a in args.alt_impl.split(",") if a and IMPLS[a] != impl]
-        if args.sgemm_kchunk == 0 and impl != IMPLS["ffma"]:
-            variants.append((args.sgemm_impl, 512))
+        variants = [(a, None) for a in args.alt_impl.split(",") if a and IMPLS[a] != impl]
+        if args.sgemm_kchunk != 0 and impl != IMPLS["ffma"]:
+            variants.append((args.sgemm_impl, 0))  # one accumulation per tile: the cost of R23's chunks
         for alt_name, kc in variants:
             a = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, sgemm_impl=IMPLS[alt_name],
                     sgemm_kchunk=kc)
@@ -688,8 +688,9 @@ def main():
     ap.add_argument("--arena-gb", type=int, default=8)
     ap.add_argument("--sgemm-impl", default="tf32bf16", choices=list(IMPL_NAMES),
                     help="implementation of the fp32 'sgemm' kernel (all meet its 1e-5 contract)")
-    ap.add_argument("--sgemm-kchunk", type=int, default=0,
-                    help="svp_config.sgemm_kchunk: K-chunked tensor-core accumulation (DESIGN R23); 0 = library default")
+    ap.add_argument("--sgemm-kchunk", type=int, default=None,
+                    help="svp_config.sgemm_kchunk: K chunk of the tensor-core accumulation (DESIGN R23); "
+                         "default: the library's (768); 0 = one accumulation per tile")
     ap.add_argument("--alt-impl", default="3xtf32,ffma",
                     help="comma list of the other sgemm implementations timed beside the main one")
     ap.add_argument("--scaling", default="auto", choices=["auto", "weak", "strong"],

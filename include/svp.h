@@ -118,19 +118,20 @@ typedef struct svp_config {
                                     GEMM launches always use the global table.             */
     int32_t sgemm_kchunk;        /* (ABI 5) "sgemm" on the tensor-core splits: accumulate K in chunks
                                     of this many k (multiple of 16; 3xTF32 uses half), each from
-                                    zero, folded into C with fp32 adds -- the accuracy of one
-                                    chunk at any K and for any operand signs (R23),
-                                    at a throughput cost (cfg5: 512 -> ~0.70x).  beta != 0 jobs
-                                    longer than one chunk run on FFMA.  0 (default): one
-                                    accumulation per tile; jobs with K > 2048 (TF32+2xBF16) /
-                                    1024 (3xTF32) run on FFMA                                */
+                                    zero in TMEM, folded into C by TMA reduce-add (IEEE fp32) --
+                                    the error of one chunk at any K and for any operand signs
+                                    (R23).  Default 768 (cfg5: ~0.92x of 0).  beta != 0
+                                    jobs longer than one chunk run on FFMA.  0: one accumulation
+                                    per tile, jobs with K > 2048 (TF32+2xBF16) / 1024 (3xTF32)
+                                    run on FFMA; same-sign operands then err up to ~2e-5 at
+                                    K = 2048                                                  */
 } svp_config;
 
 enum { SVP_TABLE_GLOBAL = 0, SVP_TABLE_PARAM = 1 };
 
 /* Fill *cfg with defaults: num_gpus 0, 4 compute streams, coalesce 1, interleave 1,
    max_chunks 8, profile_level 0, validate_ptrs 1, sgemm_impl SVP_SGEMM_TF32BF16,
-   table_mode SVP_TABLE_PARAM, rest 0 (hetero 0, graph 0). */
+   table_mode SVP_TABLE_PARAM, sgemm_kchunk 768, rest 0 (hetero 0, graph 0). */
 void svp_config_default(svp_config* cfg);
 
 /* Create a context.  On success *out owns streams/events/threads for every GPU.
@@ -162,10 +163,9 @@ int32_t svp_abi_version(void);
  *                   accumulation leaves NaN (an Inf / NaN operand, or one near FLT_MAX) is
  *                   recomputed exactly from A and B (fp64 products and sum, one rounding).
  *                   Their fp32 accumulation loses ~1.7e-8 (random-sign data) to ~3.4e-8
- *                   (same-sign data) relative per accumulating MMA: by default they take jobs
- *                   up to K = 2048 / 1024 (longer ones run on FFMA), where random-sign data
- *                   stays within 1e-5 but same-sign data at K = 2048 reaches ~2e-5;
- *                   cfg.sgemm_kchunk (e.g. 512) bounds it for all data at any K (DESIGN R23)
+ *                   (same-sign data) relative per accumulating MMA, so K is accumulated in
+ *                   chunks of cfg.sgemm_kchunk (default 768) folded into C with fp32 adds:
+ *                   measured <= 7.4e-6 componentwise on same-sign data at any K (DESIGN R23)
  *   "sgemm_tf32"    same, tcgen05 TF32 tensor cores  (own tolerance 2e-3; raw operands, so a
  *                   NaN whose payload is only in the low 13 mantissa bits reads as Inf)
  *   "dgemm"         C = alpha A B + beta C, fp64     args svp_args_dgemm   bufs [A IN, B IN, C OUT (INOUT if beta != 0)] f64

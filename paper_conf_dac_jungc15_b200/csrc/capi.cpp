@@ -96,6 +96,7 @@ void svp_config_default(svp_config* cfg) {
     cfg->validate_ptrs = 1;
     cfg->sgemm_impl = SVP_SGEMM_TF32BF16;
     cfg->table_mode = SVP_TABLE_PARAM;
+    cfg->sgemm_kchunk = 768;  // R23: the tensor-core splits' fp32 contract for any K and operand signs
 }
 
 svp_status svp_init(const svp_config* cfg, svp_ctx** out) {

@@ -463,9 +463,13 @@ static bool ew_dynamic_order() {
     return on;
 }
 
-// SVP_HIST_DYN=0: hist256 with the static blocked tile ranges instead of dynamic chunks.
+// SVP_HIST_DYN=1: hist256 in dynamic chunk order instead of the static blocked tile ranges.
+// Measured (profiles/r02/hist_dyn/): the dynamic order makes a CTA visit more VPs, and each
+// VP switch costs a flush of the replicated table (256 column sums of 32 replicas + 256
+// global atomics), which outweighed the balance gain (cfg5 hist launch 3.09 -> 2.82 TB/s):
+// off by default, SVP_HIST_DYN=1 enables it.
 static bool hist_dynamic_order() {
-    static const bool on = !(getenv("SVP_HIST_DYN") && atoi(getenv("SVP_HIST_DYN")) == 0);
+    static const bool on = getenv("SVP_HIST_DYN") && atoi(getenv("SVP_HIST_DYN")) == 1;
     return on;
 }
 

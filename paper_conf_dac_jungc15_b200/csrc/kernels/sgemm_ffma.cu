@@ -309,10 +309,10 @@ static int encode2d(void* out, const float* base, uint64_t inner, uint64_t outer
     return r == CUDA_SUCCESS ? 0 : (int)r;
 }
 
-// C (M x N row-major fp32) as 32-column x 32-row boxes with the 128-B swizzle: the epilogue's
-// staging slab layout for the K-chunk folds of the tensor-core SGEMM (TMA store / reduce-add)
+// C (M x N row-major fp32) as 16-column x 32-row boxes with the 64-B swizzle: the layout of
+// the tensor-core SGEMM epilogue's staging half-slabs (TMA store / reduce-add)
 int encode_c_map(void* mapC, const float* C, int M, int N) {
-    return encode2d(mapC, C, (uint64_t)N, (uint64_t)M, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B);
+    return encode2d(mapC, C, (uint64_t)N, (uint64_t)M, 16, 32, CU_TENSOR_MAP_SWIZZLE_64B);
 }
 
 int encode_gemm_maps(void* mapA, void* mapB, const float* A, const float* B, int M, int N, int K, int variant) {

@@ -123,8 +123,8 @@ struct Cfg {
     static constexpr int kAcc = (SPLIT == 4 || NH == 2) ? 1 : 2;  // accumulator sets (NH x 256 cols each)
     static constexpr int kTaCol = 256;                     // SPLIT 4: A ring, 16 cols per stage
     static_assert(SPLIT != 4 || kTaCol + 16 * kStages <= kTmemCols, "TMEM");
-    // K-chunk folds (R23): a 32 x 32 fp32 staging slab (128-B swizzled) per epilogue warp,
-    // written back into C by TMA store (first chunk) / TMA reduce-add (later chunks)
+    // TMA epilogue (beta == 0) and K-chunk folds (R23): 4 KiB of staging per epilogue warp (two
+    // 32 x 16 fp32 half-slabs, 64-B swizzled), written into C by TMA store / reduce-add
     static constexpr int kEpiWarps = 4 * NH;
     static constexpr size_t kStagingOff = (size_t)kStages * kStageBytes;  // 1024-B aligned
     static constexpr size_t kBarOff = kStagingOff + (size_t)kEpiWarps * 4096;
@@ -375,15 +375,29 @@ __device__ __forceinline__ float exact_element(const GemmDesc& g, int i, int j, 
 // is.  Only for beta == 0 (a beta != 0 job keeps C_old for its exact NaN path; the executor
 // routes those with K > the chunk to the FFMA kernel).  Producer, MMA issuer and epilogue all
 // walk the same (tile, chunk) units.
-__device__ __forceinline__ void tma_store_2d(const void* tmap, int32_t c0, int32_t c1, const void* smem_src) {
-    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(tmap), "r"(c0),
-                 "r"(c1), "r"(smem_u32(smem_src))
+// L2 policy of the epilogue's C writes: a partial sum another K chunk will fold into stays in
+// L2 (evict_last -- the 74 pairs' in-flight tiles are ~39 MB), a final value streams out
+// (evict_first)
+__device__ __forceinline__ uint64_t l2_policy(bool keep) {
+    uint64_t pol;
+    if (keep) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    else asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ void tma_store_2d(const void* tmap, int32_t c0, int32_t c1, const void* smem_src,
+                                             uint64_t pol) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%1, %2}], [%3], %4;" ::"l"(
+                     tmap),
+                 "r"(c0), "r"(c1), "r"(smem_u32(smem_src)), "l"(pol)
                  : "memory");
 }
-__device__ __forceinline__ void tma_reduce_add_2d(const void* tmap, int32_t c0, int32_t c1, const void* smem_src) {
-    asm volatile("cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.bulk_group [%0, {%1, %2}], [%3];" ::"l"(tmap),
-                 "r"(c0), "r"(c1), "r"(smem_u32(smem_src))
-                 : "memory");
+__device__ __forceinline__ void tma_reduce_add_2d(const void* tmap, int32_t c0, int32_t c1, const void* smem_src,
+                                                  uint64_t pol) {
+    asm volatile(
+        "cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.bulk_group.L2::cache_hint [%0, {%1, %2}], [%3], %4;" ::"l"(
+            tmap),
+        "r"(c0), "r"(c1), "r"(smem_u32(smem_src)), "l"(pol)
+        : "memory");
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
@@ -742,16 +756,19 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
             constexpr int SW = 8, NV = SW / 4;
             if (first) nan_slabs = 0;
             if (tma_epi) {
+                // two 32-row x 16-column half-slabs (64-B rows, 64-B swizzle) per epilogue warp,
+                // alternating: the TMA op of one is in flight while the other is refilled
                 uint8_t* slab = smem + C::kStagingOff + (size_t)(warp < 8 ? warp - 4 : warp - 10) * 4096;
                 const void* cmap = cmaps + (size_t)v * 128;
                 const int row0 = tm * C::kMmaM + (int)rank * BM + q * 32;
                 if (lane == 0) bulk_wait0();  // the previous (tile, chunk) unit's writes landed
 #pragma unroll 1
-                for (int c0 = 0; c0 < BN; c0 += 32) {
-                    if (lane == 0) bulk_wait_read0();  // the slab is free again
+                for (int c0 = 0; c0 < BN; c0 += 16) {
+                    uint8_t* hs = slab + ((c0 >> 4) & 1) * 2048;
+                    if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");  // hs is free
                     __syncwarp();
-#pragma unroll 1
-                    for (int sl = 0; sl < 4; ++sl) {
+#pragma unroll
+                    for (int sl = 0; sl < 2; ++sl) {
                         uint32_t r[SW];
                         tmem_ld8(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0 + sl * SW), r);
 #pragma unroll
@@ -764,16 +781,17 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                             o.w = alpha * __uint_as_float(r[j + 3]);
                             const float o4 = o.x + o.y + o.z + o.w;
                             if (o4 != o4) nan_slabs |= 1u << ((c0 + sl * SW) / SW);
-                            const int ck16 = 2 * sl + jj;  // 16-B chunk of this lane's 128-B row
-                            *reinterpret_cast<float4*>(slab + lane * 128 + ((ck16 ^ (lane & 7)) << 4)) = o;
+                            const int ck16 = 2 * sl + jj;  // 16-B chunk of this lane's 64-B row
+                            *reinterpret_cast<float4*>(hs + lane * 64 + ((ck16 ^ ((lane >> 1) & 3)) << 4)) = o;
                         }
                     }
                     fence_proxy_async();
                     __syncwarp();
                     if (lane == 0) {
                         const int col = tn * TN + eh * BN + c0;
-                        if (first) tma_store_2d(cmap, col, row0, slab);
-                        else tma_reduce_add_2d(cmap, col, row0, slab);
+                        const uint64_t pol = l2_policy(!last);
+                        if (first) tma_store_2d(cmap, col, row0, hs, pol);
+                        else tma_reduce_add_2d(cmap, col, row0, hs, pol);
                         bulk_commit();
                     }
                 }

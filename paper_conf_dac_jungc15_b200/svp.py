@@ -240,7 +240,7 @@ class Context:
                  flush_timeout_ms: int = 0, validate_ptrs: int = 1, sgemm_impl: int = SGEMM_TF32BF16,
                  external_streams: Optional[Sequence[int]] = None, hbm_gbps: float = 0.0, pcie_gbps: float = 0.0,
                  ffma_tflops: float = 0.0, launch_us: float = 0.0, hetero: bool = False, graph: bool = False,
-                 table_mode: int = TABLE_PARAM, sgemm_kchunk: int = 0):
+                 table_mode: int = TABLE_PARAM, sgemm_kchunk: Optional[int] = None):
         L = load()
         cfg = svp_config()
         L.svp_config_default(C.byref(cfg))
@@ -267,7 +267,8 @@ class Context:
             cfg.external_streams = C.cast(self._ext, C.POINTER(C.c_void_p))
         cfg.hbm_gbps, cfg.pcie_gbps, cfg.ffma_tflops, cfg.launch_us = hbm_gbps, pcie_gbps, ffma_tflops, launch_us
         cfg.hetero, cfg.graph, cfg.table_mode = int(hetero), int(graph), int(table_mode)
-        cfg.sgemm_kchunk = int(sgemm_kchunk)
+        if sgemm_kchunk is not None:  # else the library default (svp_config_default)
+            cfg.sgemm_kchunk = int(sgemm_kchunk)
         h = C.c_void_p()
         _check(L.svp_init(C.byref(cfg), C.byref(h)))
         self._h = h

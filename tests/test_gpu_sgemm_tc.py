@@ -165,14 +165,14 @@ def test_tail_split_last_wave(int_inputs, residency, interleave):
 
 
 @pytest.mark.parametrize("impl", [svp.SGEMM_TF32BF16, svp.SGEMM_3XTF32])
-@pytest.mark.parametrize("kchunk", [0, 512])
+@pytest.mark.parametrize("kchunk", [0, 512, None])
 def test_long_k_keeps_fp32_contract(impl, kchunk):
     """DESIGN R23: the tcgen05 fp32 accumulation loses ~1.7e-8 relative per accumulating MMA.
-    Default: K = 4096 is past the single accumulation's limit, so those jobs match apart and
-    run on FFMA (VP 1, K = 512, stays on the tensor cores).  sgemm_kchunk = 512: long K runs
-    in chunks folded into C with fp32 adds (beta == 0: VPs 0 and 1 on the tensor cores) and
-    a beta != 0 job past one chunk runs on FFMA (VP 2).  Either way the 1e-5 contract
-    (componentwise and Frobenius) holds at K = 4096."""
+    sgemm_kchunk = 0: K = 4096 is past the single accumulation's limit, so those jobs match
+    apart and run on FFMA (VP 1, K = 512, stays on the tensor cores).  sgemm_kchunk = 512 and
+    the default (768): long K runs in chunks folded into C with fp32 adds (beta == 0: VPs 0
+    and 1 on the tensor cores) and a beta != 0 job past one chunk runs on FFMA (VP 2).  Either
+    way the 1e-5 contract (componentwise and Frobenius) holds at K = 4096."""
     specs = [W.JobSpec(0, "sgemm", M=384, N=256, K=4096), W.JobSpec(1, "sgemm", M=256, N=256, K=512),
              W.JobSpec(2, "sgemm", M=256, N=384, K=4096, alpha=0.5, beta=2.0)]
     inputs = inputs_for(specs)
@@ -204,15 +204,16 @@ def test_unaligned_shapes_and_buffers(impl, residency):
 
 @pytest.mark.parametrize("impl", [svp.SGEMM_TF32BF16, svp.SGEMM_3XTF32])
 @pytest.mark.parametrize("K", [2048, 4096])
-def test_same_sign_operands_keep_fp32_contract_chunked(impl, K):
+@pytest.mark.parametrize("kchunk", [None, 512])
+def test_same_sign_operands_keep_fp32_contract_chunked(impl, K, kchunk):
     """The accumulation bias (R23) is largest relative to the output when nothing cancels:
     A, B ~ U[0, 1) make |C| = (|A||B|) so the componentwise bound IS a 1e-5 relative bound.
-    A single accumulation measured 2.04e-5 here at K = 2048 (profiles/r02/accuracy/); with
-    sgemm_kchunk = 512 (strict mode) it must hold at the benched K and beyond."""
+    A single accumulation measured 2.04e-5 here at K = 2048 (profiles/r02/accuracy/); with the
+    default K chunks (768) and with 512 it must hold at the benched K and beyond."""
     g = np.random.default_rng(3)
     specs = [W.JobSpec(v, "sgemm", M=256, N=512, K=K) for v in range(2)]
     inputs = [{"A": g.random((256, K), dtype=np.float32), "B": g.random((K, 512), dtype=np.float32)} for _ in specs]
-    outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl, sgemm_kchunk=512)
+    outs, _, _ = run_svp(specs, inputs, "device", sgemm_impl=impl, sgemm_kchunk=kchunk)
     want = oracle.run_jobs(specs, inputs)
     for s, inp, got, w in zip(specs, inputs, outs, want):
         check_job(s, inp, got, w)

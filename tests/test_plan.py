@@ -103,10 +103,11 @@ def test_sgemm_accuracy_routing_chunked(impl):
 
 
 @pytest.mark.parametrize("impl,kmax", [(svp.SGEMM_TF32BF16, 2048), (svp.SGEMM_3XTF32, 1024), (svp.SGEMM_FFMA, None)])
-def test_sgemm_accuracy_routing_default(impl, kmax):
-    """DESIGN R23, default (no K chunks): jobs with K above the measured limit of the split's
-    single accumulation (2048 for TF32+2xBF16, 1024 for 3xTF32) match apart and run on FFMA."""
-    with svp.Context(dry_run=True, sgemm_impl=impl) as c:
+def test_sgemm_accuracy_routing_unchunked(impl, kmax):
+    """DESIGN R23, sgemm_kchunk = 0 (one accumulation per tile): jobs with K above the measured
+    limit of the split's single accumulation (2048 for TF32+2xBF16, 1024 for 3xTF32) match
+    apart and run on FFMA."""
+    with svp.Context(dry_run=True, sgemm_impl=impl, sgemm_kchunk=0) as c:
         Ks = [512, 1024, 2048, 2052, 4096]
         for vp, K in enumerate(Ks):
             submit(c, vp, "sgemm", M=256, N=256, K=K)
