@@ -383,7 +383,7 @@ def gpu_plan(args, ws, local):
     return ords, "single"
 
 
-def roofline_of(kstats, impl, peaks, peak_src):
+def roofline_of(kstats, impl, peaks, peak_src, kchunk=None):
     from paper_conf_dac_jungc15_b200 import svp
     dom = max(kstats, key=lambda n: kstats[n]["total_ns"])
     dk = kstats[dom]
@@ -428,17 +428,21 @@ def roofline_of(kstats, impl, peaks, peak_src):
             sus = float(peaks["bf16_tflops_sustained"]) * roof["peak"] / float(peaks.get("bf16_tflops", 1590.0))
             roof["peak_sustained"] = sus
             roof["frac_of_sustained"] = roof["achieved"] / sus
-    prof_path = os.path.join(ROOT, "profiles", "traffic_r01.json")
-    if os.path.exists(prof_path):
+    # DRAM bytes per launch of the dominant kernel from one committed ncu --set full capture
+    # (round 2 first, round-1 figures for kernels not re-captured)
+    key = dom + ({svp.SGEMM_3XTF32: "_3xtf32", svp.SGEMM_TF32BF16: "_tf32bf16"}.get(impl, "") if dom == "sgemm" else "")
+    if dom == "sgemm" and impl == svp.SGEMM_TF32BF16 and kchunk == 0:
+        key += "_kchunk0"
+    for name in ("traffic_r02.json", "traffic_r01.json"):
+        prof_path = os.path.join(ROOT, "profiles", name)
         try:
             tr = json.load(open(prof_path))
-            key = dom + ({svp.SGEMM_3XTF32: "_3xtf32", svp.SGEMM_TF32BF16: "_tf32bf16"}.get(impl, "")
-                         if dom == "sgemm" else "")
-            if key in tr:
-                roof["traffic"] = tr[key]
-                roof["traffic_source"] = "profiles/traffic_r01.json (ncu --set full, cfg5 launch)"
         except Exception:
-            pass
+            continue
+        if key in tr:
+            roof["traffic"] = tr[key]
+            roof["traffic_source"] = f"profiles/{name} (ncu --set full of the cfg5 launch)"
+            break
     return dom, roof
 
 
@@ -536,7 +540,7 @@ def run_svp(args, rank, ws, local):
             row["gbs"] = k["bytes"] / k["total_ns"]
         per_kernel[n] = row
     peaks, peak_src = measured_peaks()
-    dom, roof = roofline_of(kstats, impl, peaks, peak_src)
+    dom, roof = roofline_of(kstats, impl, peaks, peak_src, args.sgemm_kchunk)
     if args.config != 5:
         roof["traffic"] = None  # the committed ncu traffic figure is cfg5's launch
         roof.pop("traffic_source", None)

@@ -72,8 +72,8 @@ class VPSet:
                 self.kids[s.kernel] = ctx.kernel(s.kernel)
         if assign and residency == "device":
             # estimated kernel ns (the Dispatcher's LPT costs): algorithmic bytes at the measured
-            # 6.55 TB/s + FLOPs at ~400 TFLOP/s (the fp32 tensor-core split)
-            costs = [float(s.algorithmic_bytes()) / 6.55 + float(s.flops()) / 4.0e5 for s in self.specs]
+            # 6.55 TB/s (6550 B/ns) + FLOPs at ~400 TFLOP/s (4e5 flop/ns, the fp32 tensor-core split)
+            costs = [float(s.algorithmic_bytes()) / 6550.0 + float(s.flops()) / 4.0e5 for s in self.specs]
             ctx.assign_vps([s.vp for s in self.specs], [self.kids[s.kernel] for s in self.specs], costs)
         self.bufs: List[Dict[str, torch.Tensor]] = []   # views (what the kernel sees)
         self.raw: List[Dict[str, torch.Tensor]] = []    # allocations incl. misalign + guard

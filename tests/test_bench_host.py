@@ -56,7 +56,7 @@ def test_cfg5_dispatcher_split(G):
     specs = W.config_specs(5)
     with svp.Context(dry_run=True, num_gpus=G) as c:
         kids = {k: c.kernel(k) for k in W.KERNELS}
-        costs = [float(s.algorithmic_bytes()) / 6.55 + float(s.flops()) / 4.0e5 for s in specs]
+        costs = [float(s.algorithmic_bytes()) / 6550.0 + float(s.flops()) / 4.0e5 for s in specs]
         dev = c.assign_vps([s.vp for s in specs], [kids[s.kernel] for s in specs], costs)
         ds = [c.device_stats(g) for g in range(G)]
     assert sum(d["vps"] for d in ds) == 256
