@@ -437,6 +437,23 @@ def test_two_logical_gpus_one_process(small, residency):
     for i, (s, inp) in enumerate(zip(specs, inputs)):
         check_job(s, inp, vs.output(i))
     assert vs.guards_intact()
+    # per-GPU Profiler view (svp_device_stats_get): every job counted once on its VP's GPU,
+    # each GPU's span and kernel time measured, placement matching the plan
+    ds = [ctx.device_stats(g) for g in range(2)]
+    assert sum(d["jobs"] for d in ds) == len(specs)
+    assert all(d["flushes"] == 1 and d["device_ns"] > 0 and d["kernel_ns"] > 0 for d in ds), ds
+    assert sum(d["vps"] for d in ds) == len({s.vp for s in specs})
+    for g in range(2):
+        assert ds[g]["jobs"] == sum(1 for s in specs if owner.get(s.vp) == g)
+    # measured timeline: every op started after the ops it waits on ended (same GPU)
+    for op in ops:
+        assert op["measured_start_ns"] >= 0 and op["measured_ns"] >= 0
+        for w in op["waits"]:
+            q = ops[w]
+            if q["device"] == op["device"]:
+                assert op["measured_start_ns"] + 1e3 >= q["measured_start_ns"] + q["measured_ns"], (op, q)
+    ctx.reset_profile()
+    assert all(ctx.device_stats(g)["jobs"] == 0 for g in range(2))
     ctx.close()
 
 
