@@ -1254,11 +1254,11 @@ static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool u
             float mx = 0;
             for (size_t i = 0; i < f.ops.size(); ++i) {
                 if (tstart[i] < 0) continue;
-                float ms = 0, ms0 = 0;
-                CK(cudaEventElapsedTime(&ms, d.t_ev[2 * tstart[first]], d.t_ev[2 * tstart[i] + 1]));
-                CK(cudaEventElapsedTime(&ms0, d.t_ev[2 * tstart[first]], d.t_ev[2 * tstart[i]]));
+                // one query per op: its start offset; its end = start + the duration above
+                float ms0 = 0;
+                if (i != (size_t)first) CK(cudaEventElapsedTime(&ms0, d.t_ev[2 * tstart[first]], d.t_ev[2 * tstart[i]]));
                 f.ops[i].measured_start_ns = (double)ms0 * 1e6;
-                mx = std::max(mx, ms);
+                mx = std::max(mx, ms0 + (float)(f.ops[i].measured_ns * 1e-6));
             }
             span = mx;
         }

@@ -5,6 +5,7 @@
 // streams/events/arena/tables, Profiler) -> kernels/*.cu (L0: sm_100a guest kernels).
 #pragma once
 #include <math.h>
+#include <string.h>
 #include <stdint.h>
 
 #include <atomic>
@@ -213,9 +214,13 @@ struct CostModel {
             for (double& x : row) x = 1.0;
     }
     static int bucket(double alg_bytes, double flops) {
+        // floor(log2 w) / 2 from the exponent bits: this runs once per submitted job
         const double w = flops > 0 ? flops : alg_bytes;
-        const int b = w >= 1.0 ? (int)(0.5 * log2(w)) : 0;
-        return b < 0 ? 0 : (b >= kBuckets ? kBuckets - 1 : b);
+        if (!(w >= 1.0)) return 0;
+        uint64_t bits;
+        memcpy(&bits, &w, sizeof bits);
+        const int b = ((int)((bits >> 52) & 0x7ff) - 1023) >> 1;
+        return b >= kBuckets ? kBuckets - 1 : b;
     }
     double kernel_ns(int32_t kernel, double alg_bytes, double flops) const;
     // K_SGEMM on an explicit implementation (a group routed to FFMA, R23)
