@@ -301,7 +301,7 @@ class Arm:
     """One svp.Context driving this process's GPUs, and the workload's VP buffers (one or
     more rotating buffer sets) pre-marshalled as JobBatches."""
 
-    def __init__(self, specs, inputs, residency, ordinals, streams, nsets=1, kids=None, **cfg):
+    def __init__(self, specs, inputs, residency, ordinals, streams, nsets=1, kids=None, host_numa=False, **cfg):
         from paper_conf_dac_jungc15_b200 import svp
         from paper_conf_dac_jungc15_b200.vpset import VPSet
         self.svp = svp
@@ -310,7 +310,8 @@ class Arm:
         self.ctx = svp.Context(num_gpus=len(self.ordinals), device_ids=self.ordinals,
                                external_streams=[st.cuda_stream for st in streams], **cfg)
         self.sets = [VPSet(self.ctx, specs, inputs, residency,
-                           device_ordinals=self.ordinals if residency == "device" else None)
+                           device_ordinals=self.ordinals if residency == "device" else None,
+                           host_numa=host_numa)
                      for _ in range(nsets)]
         self.kids = self.sets[0].kids
         self.batches = [svp.JobBatch(vs.job_list()) for vs in self.sets]
@@ -607,7 +608,7 @@ def run_svp(args, rank, ws, local):
     e2e = None
     if not args.no_e2e:
         h = Arm(specs, inputs, "host", ords, streams, 1, arena_bytes=args.arena_gb << 30, sgemm_impl=impl,
-                sgemm_kchunk=args.sgemm_kchunk,
+                sgemm_kchunk=args.sgemm_kchunk, host_numa=bool(args.host_numa),
                 max_chunks=int(os.environ.get("SVP_BENCH_MAXCH", "8")), **f4)
         h.steps(2)
         hst = h.ctx.flush_stats()
@@ -618,7 +619,10 @@ def run_svp(args, rank, ws, local):
                "h2d_bytes_per_step": int(sum_over_ranks(hst["h2d_bytes"], ws)),
                "d2h_bytes_per_step": int(sum_over_ranks(hst["d2h_bytes"], ws)),
                "steps": ks, "ms_per_step": edt / ks * 1e3, "chunks": int(hst["chunks"]),
-               "api": "svp_submit_batch + svp_flush, HOST_PINNED buffers (H2D/D2H staged + interleaved)"}
+               "api": "svp_submit_batch + svp_flush, HOST_PINNED buffers (H2D/D2H staged + interleaved)",
+               "host_buffers": ("svp_host_alloc on each VP's GPU's NUMA node (node %s)"
+                                % sorted({h.ctx.device_stats(g)["numa_node"] for g in range(len(ords))})
+                                if args.host_numa else "torch pinned (cudaHostAlloc, first-touch placement)")}
         h.close()
 
     # ---------------- weak scaling beside the strong number (N > 1)
@@ -707,6 +711,8 @@ def main():
                     help="steady-state plan reuse + CUDA graph replay (NEXT f4)")
     ap.add_argument("--table-mode", type=int, default=1, choices=[0, 1],
                     help="segment tables: 0 global device buffer, 1 by-value kernel parameter")
+    ap.add_argument("--host-numa", type=int, default=1, choices=[0, 1],
+                    help="e2e: host buffers from svp_host_alloc on the VP's GPU's NUMA node (0: torch pinned)")
     ap.add_argument("--no-serial", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other sgemm implementation")
     ap.add_argument("--no-e2e", action="store_true")

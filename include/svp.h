@@ -34,7 +34,7 @@
 extern "C" {
 #endif
 
-#define SVP_ABI_VERSION 5
+#define SVP_ABI_VERSION 6
 
 typedef int32_t svp_status;
 enum {
@@ -367,8 +367,31 @@ typedef struct svp_device_stats {
     double device_ns;       /* summed per-flush device span                             */
     double kernel_ns;       /* summed event-timed kernel op durations                   */
     double last_device_ns;  /* the last flush's span on this GPU                        */
+    int32_t numa_node;      /* (ABI 6) the GPU's NUMA node (sysfs of its PCI function),
+                               -1 unknown (single-socket hosts, hidden sysfs)           */
+    int32_t worker_cpu_pinned; /* (ABI 6) 1 if the worker thread driving this GPU runs on
+                               the GPU's local CPUs (GPU indices >= 1 of a multi-GPU
+                               context; GPU 0 is driven by the flushing thread, never
+                               pinned).  SVP_NUMA_AFFINITY=0 turns the pinning off.     */
 } svp_device_stats;
 svp_status svp_device_stats_get(svp_ctx* ctx, int32_t g, svp_device_stats* out);
+
+/* (ABI 6) NUMA-local page-locked host memory for host-resident VP buffers (PAPER.md
+ * L266-286: the H2D / D2H copies of a VP's data are its job's first and last steps; on a
+ * multi-socket B200 node, pages on the far socket cross the inter-socket link before PCIe).
+ * Allocates `bytes` (rounded up to whole pages) of anonymous host memory, binds it
+ * (mbind MPOL_PREFERRED) to the NUMA node of GPU index `gpu` of this context, and
+ * page-locks it with cudaHostRegister(Portable), so any GPU of the process can DMA it and
+ * svp_submit accepts it as SVP_MEM_HOST_PINNED.  *ptr_out receives the address (page
+ * aligned); *numa_node_out (optional) the node the pages were bound to, or -1 when the
+ * GPU's node is unknown (the memory is then page-locked but not placed).  The memory is
+ * the caller's until svp_host_free(ctx, ptr) or svp_finalize(ctx), which releases every
+ * block still allocated; freeing a block with jobs in flight on it is undefined.
+ * Errors: SVP_E_INVAL (null, bytes == 0, gpu out of range), SVP_E_UNSUPPORTED (dry-run
+ * context), SVP_E_NOMEM (mmap / pinning failed), SVP_E_CUDA. */
+svp_status svp_host_alloc(svp_ctx* ctx, int32_t gpu, uint64_t bytes, void** ptr_out, int32_t* numa_node_out);
+/* Releases a block from svp_host_alloc.  SVP_E_INVAL if ptr is not one (or already freed). */
+svp_status svp_host_free(svp_ctx* ctx, void* ptr);
 
 /* ------------------------------------------------------------------ plan introspection */
 /* The last flush's plan, one entry per issued op in issue order (tests, tooling). */

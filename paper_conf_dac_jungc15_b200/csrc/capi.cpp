@@ -8,6 +8,7 @@
 #include <stdio.h>
 #include <stdlib.h>
 #include <string.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <chrono>
@@ -158,7 +159,9 @@ svp_status svp_finalize(svp_ctx* h) {
     }
     Ctx* c = reinterpret_cast<Ctx*>(h);
     stop_dispatcher(c);
-    if (c->exec) executor_destroy(c->exec);
+    if (c->exec) executor_destroy(c->exec);  // synchronizes every stream first
+    for (auto& kv : c->host_blocks) host_free_near(kv.first, kv.second);
+    c->host_blocks.clear();
     delete c;
     return SVP_OK;
     SVP_TRY_END
@@ -658,6 +661,8 @@ svp_status svp_device_stats_get(svp_ctx* h, int32_t g, svp_device_stats* out) {
     out->device_ns = d.device_ns;
     out->kernel_ns = d.kernel_ns;
     out->last_device_ns = d.last_device_ns;
+    out->numa_node = -1;
+    if (c->exec) executor_numa_info(c->exec, g, &out->numa_node, &out->worker_cpu_pinned);
     return SVP_OK;
     SVP_TRY_END
 }
@@ -735,3 +740,67 @@ svp_status svp_plan_op_detail(svp_ctx* h, int32_t i, uint64_t* arena_off, uint64
 }
 
 }  // extern "C"
+
+svp_status svp_host_alloc(svp_ctx* h, int32_t gpu, uint64_t bytes, void** ptr_out, int32_t* numa_node_out) {
+    SVP_TRY_BEGIN
+    svp_status st = check_ctx(h);
+    if (st) return st;
+    if (!ptr_out || bytes == 0) {
+        set_error("svp_host_alloc: null ptr_out or bytes == 0");
+        return SVP_E_INVAL;
+    }
+    *ptr_out = nullptr;
+    if (numa_node_out) *numa_node_out = -1;
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    if (gpu < 0 || gpu >= c->ngpu) {
+        set_error("svp_host_alloc: GPU index out of range");
+        return SVP_E_INVAL;
+    }
+    if (!c->exec) {
+        set_error("svp_host_alloc: a dry-run context has no CUDA devices");
+        return SVP_E_UNSUPPORTED;
+    }
+    const long pg = sysconf(_SC_PAGESIZE) > 0 ? sysconf(_SC_PAGESIZE) : 4096;
+    const size_t len = (size_t)((bytes + (uint64_t)pg - 1) / (uint64_t)pg * (uint64_t)pg);
+    const int ordinal = gpu < (int32_t)c->device_ids.size() ? c->device_ids[gpu] : gpu;
+    void* p = nullptr;
+    int node = -1;
+    std::string err;
+    st = host_alloc_near(ordinal, len, &p, &node, &err);
+    if (st) {
+        set_error(err);
+        return st;
+    }
+    {
+        std::lock_guard<std::mutex> lk(c->hmu);
+        c->host_blocks[p] = len;
+    }
+    *ptr_out = p;
+    if (numa_node_out) *numa_node_out = node;
+    return SVP_OK;
+    SVP_TRY_END
+}
+
+svp_status svp_host_free(svp_ctx* h, void* ptr) {
+    SVP_TRY_BEGIN
+    if (!h) {
+        set_error("null context");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    size_t len = 0;
+    {
+        std::lock_guard<std::mutex> lk(c->hmu);
+        auto it = c->host_blocks.find(ptr);
+        if (it == c->host_blocks.end()) {
+            set_error("svp_host_free: not a block from svp_host_alloc (or already freed)");
+            return SVP_E_INVAL;
+        }
+        len = it->second;
+        c->host_blocks.erase(it);
+    }
+    if (c->exec) executor_forget_range(c->exec, (uintptr_t)ptr, (uintptr_t)ptr + len);
+    host_free_near(ptr, len);
+    return SVP_OK;
+    SVP_TRY_END
+}

@@ -70,6 +70,8 @@ struct Dev {
     std::vector<cudaEvent_t> end_ev;
     uint8_t* arena = nullptr;
     uint64_t arena_bytes = 0;
+    int numa_node = -1;       // the GPU's NUMA node (sysfs), -1 unknown
+    bool cpu_pinned = false;  // its worker thread runs on the GPU's local CPUs
     // profile_level 2: per-segment busy-cycle counters of this flush's segment launches
     uint64_t* busy_dev = nullptr;
     size_t busy_cap = 0;  // counters
@@ -158,6 +160,11 @@ RangeBatchLock::~RangeBatchLock() {
 
 std::string executor_error(Executor* e) { return e->err; }
 
+void executor_numa_info(Executor* e, int g, int32_t* node, int32_t* pinned) {
+    *node = e->devs[g].numa_node;
+    *pinned = e->devs[g].cpu_pinned ? 1 : 0;
+}
+
 static svp_status dev_setup(Dev& d, const svp_config& cfg, void* ext) {
     CK(cudaSetDevice(d.ordinal));
     CK(cudaFree(0));  // create / adopt the primary context
@@ -178,6 +185,7 @@ static svp_status dev_setup(Dev& d, const svp_config& cfg, void* ext) {
     for (auto& e : d.join_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&d.fork_ev, cudaEventDisableTiming));
     d.arena_bytes = cfg.arena_bytes;
+    d.numa_node = gpu_numa_node(d.ordinal);
     CK(query_limits(&d.lim));
     return SVP_OK;
 }
@@ -271,7 +279,11 @@ static void start_workers(Executor* e) {
     const int G = (int)e->devs.size();
     e->w.st.assign(G, SVP_OK);
     e->w.issue.assign(G, 0.0);
-    for (int g = 1; g < G; ++g) e->w.th.emplace_back(worker_loop, e, g);
+    for (int g = 1; g < G; ++g) {
+        e->w.th.emplace_back(worker_loop, e, g);
+        // worker g runs on the CPUs next to its GPU (numa.cpp; SVP_NUMA_AFFINITY=0 disables)
+        e->devs[g].cpu_pinned = pin_thread_near_gpu(e->devs[g].ordinal, e->w.th.back().native_handle());
+    }
 }
 
 static void stop_workers(Executor* e) {
@@ -339,6 +351,16 @@ static bool alloc_range(const void* p, uintptr_t* start, uintptr_t* end) {
     *start = (uintptr_t)base;
     *end = (uintptr_t)base + size;
     return true;
+}
+
+// An allocation [start, end) was released (svp_host_free): drop its cached ranges so an
+// address reused later is resolved afresh.
+void executor_forget_range(Executor* e, uintptr_t start, uintptr_t end) {
+    std::lock_guard<std::mutex> lk(e->rmu);
+    for (auto it = e->ranges.lower_bound(start); it != e->ranges.end() && it->first < end;)
+        it = e->ranges.erase(it);
+    for (auto& h : e->hot)
+        if (h.start < end && start < h.end) h = Executor::Hot{};
 }
 
 svp_status executor_check_ptr(Executor* e, const void* p, uint64_t bytes, int32_t mem, int32_t device,

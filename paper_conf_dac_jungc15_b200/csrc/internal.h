@@ -5,6 +5,8 @@
 // streams/events/arena/tables, Profiler) -> kernels/*.cu (L0: sm_100a guest kernels).
 #pragma once
 #include <math.h>
+#include <pthread.h>
+#include <sched.h>
 #include <string.h>
 #include <stdint.h>
 
@@ -288,6 +290,10 @@ struct Ctx {
     KStats kstats[K_COUNT];
     std::vector<DevStats> dstats;    // [ngpu]
 
+    // svp_host_alloc blocks (NUMA-placed, page-locked), released by svp_host_free / finalize
+    std::mutex hmu;
+    std::unordered_map<void*, size_t> host_blocks;
+
     Executor* exec = nullptr;        // null in dry_run
     bool coschedule = false;         // SVP_COSCHEDULE=1: memory-first small-grid co-residency
                                      // (measured slower than longest-first)
@@ -306,6 +312,16 @@ Executor* executor_create(Ctx* c, svp_status* st);
 void executor_destroy(Executor* e);
 svp_status executor_run(Executor* e, Flush* f);      // tables, staging, issue, wait, profile
 std::string executor_error(Executor* e);
+
+// numa.cpp: NUMA placement near a GPU (sysfs of its PCI function; -1 / false = unknown)
+int gpu_numa_node(int ordinal);
+bool parse_cpulist(const char* s, cpu_set_t* set);
+bool gpu_local_cpus(int ordinal, cpu_set_t* set);
+bool pin_thread_near_gpu(int ordinal, pthread_t th);
+void executor_numa_info(Executor* e, int g, int32_t* node, int32_t* pinned);
+void executor_forget_range(Executor* e, uintptr_t start, uintptr_t end);
+svp_status host_alloc_near(int ordinal, size_t len, void** out, int* node_out, std::string* err);
+void host_free_near(void* p, size_t len);
 // residency check for svp_submit (validate_ptrs): returns SVP_OK or SVP_E_INVAL
 // Residency check of one buffer [p, p + bytes) (cfg.validate_ptrs): declared DEVICE ->
 // device (or managed) memory on the VP's GPU; HOST_PINNED -> page-locked host memory; and

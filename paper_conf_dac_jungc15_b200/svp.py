@@ -37,7 +37,7 @@ EXPORTS = ("svp_config_default", "svp_init", "svp_finalize", "svp_last_error", "
            "svp_flush_stats_get", "svp_plan_size", "svp_plan_get", "svp_wait", "svp_start_dispatcher",
            "svp_stop_dispatcher", "svp_ipc_serve", "svp_ipc_server_stats", "svp_ipc_shutdown", "svp_ipc_connect",
            "svp_ipc_disconnect", "svp_ipc_alloc", "svp_ipc_submit", "svp_ipc_wait", "svp_kernel_lookup",
-           "svp_plan_op_detail", "svp_device_stats_get")
+           "svp_plan_op_detail", "svp_device_stats_get", "svp_host_alloc", "svp_host_free")
 
 
 class svp_config(C.Structure):
@@ -86,7 +86,7 @@ class svp_flush_stats(C.Structure):
 class svp_device_stats(C.Structure):
     _fields_ = [("ordinal", C.c_int32), ("vps", C.c_int32), ("est_load_ns", C.c_double), ("flushes", C.c_uint64),
                 ("jobs", C.c_uint64), ("device_ns", C.c_double), ("kernel_ns", C.c_double),
-                ("last_device_ns", C.c_double)]
+                ("last_device_ns", C.c_double), ("numa_node", C.c_int32), ("worker_cpu_pinned", C.c_int32)]
 
 
 class svp_plan_op(C.Structure):
@@ -158,6 +158,8 @@ def load(build_if_stale: bool = True):
         L.svp_ipc_wait.argtypes = [vp, C.c_uint64, C.c_int32]
         L.svp_kernel_lookup.argtypes = [C.c_char_p, P(C.c_int32)]
         L.svp_device_stats_get.argtypes = [vp, C.c_int32, P(svp_device_stats)]
+        L.svp_host_alloc.argtypes = [vp, C.c_int32, C.c_uint64, P(C.c_void_p), P(C.c_int32)]
+        L.svp_host_free.argtypes = [vp, C.c_void_p]
         L.svp_plan_op_detail.argtypes = [vp, C.c_int32, P(C.c_uint64), P(C.c_uint64), P(C.c_int32), C.c_int32,
                                          P(C.c_int32), P(C.c_double)]
         for name in EXPORTS:
@@ -369,6 +371,16 @@ class Context:
         s = svp_device_stats()
         _check(self._L.svp_device_stats_get(self._h, g, C.byref(s)))
         return {k: getattr(s, k) for k, _ in svp_device_stats._fields_}
+
+    def host_alloc(self, gpu: int, nbytes: int):
+        """svp_host_alloc: page-locked host memory on GPU index `gpu`'s NUMA node.
+        Returns (address, numa node or -1)."""
+        p, node = C.c_void_p(), C.c_int32()
+        _check(self._L.svp_host_alloc(self._h, gpu, nbytes, C.byref(p), C.byref(node)))
+        return p.value, node.value
+
+    def host_free(self, addr: int):
+        _check(self._L.svp_host_free(self._h, addr))
 
     def flush_stats(self) -> Dict[str, float]:
         s = svp_flush_stats()

@@ -9,6 +9,7 @@ that no kernel wrote past a VP's extent (the segment table needs no padding).
 """
 from __future__ import annotations
 
+import ctypes
 from typing import Dict, List, Optional, Sequence
 
 import numpy as np
@@ -62,7 +63,9 @@ class VPSet:
 
     def __init__(self, ctx: svp.Context, specs: Sequence, inputs: Optional[Sequence[Dict[str, np.ndarray]]] = None,
                  residency: str = "device", device_ordinals: Optional[Sequence[int]] = None,
-                 assign: bool = True):
+                 assign: bool = True, host_numa: bool = False):
+        """host_numa (residency "host"): allocate every VP's buffers with svp_host_alloc on the
+        NUMA node of the GPU the Dispatcher placed the VP on (the VPs are assigned first)."""
         self.ctx = ctx
         self.specs = list(specs)
         self.residency = residency
@@ -70,7 +73,8 @@ class VPSet:
         for s in self.specs:
             if s.kernel not in self.kids:
                 self.kids[s.kernel] = ctx.kernel(s.kernel)
-        if assign and residency == "device":
+        self.host_blocks: List[int] = []
+        if assign and (residency == "device" or host_numa):
             # estimated kernel ns (the Dispatcher's LPT costs): algorithmic bytes at the measured
             # 6.55 TB/s (6550 B/ns) + FLOPs at ~400 TFLOP/s (4e5 flop/ns, the fp32 tensor-core split)
             costs = [float(s.algorithmic_bytes()) / 6550.0 + float(s.flops()) / 4.0e5 for s in self.specs]
@@ -99,7 +103,11 @@ class VPSet:
                 elif s.kernel == "hist256":
                     mis = 7 * m
                 nbytes = (ne + mis) * es + GUARD
-                if dev.type == "cpu":
+                if dev.type == "cpu" and host_numa:
+                    addr, _node = ctx.host_alloc(ctx.vp_device(s.vp), nbytes)
+                    self.host_blocks.append(addr)
+                    raw = torch.frombuffer((ctypes.c_uint8 * nbytes).from_address(addr), dtype=torch.uint8)
+                elif dev.type == "cpu":
                     raw = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
                 else:
                     raw = torch.empty(nbytes, dtype=torch.uint8, device=dev)
@@ -112,6 +120,14 @@ class VPSet:
         self.inputs = inputs
         if inputs is not None:
             self.load_inputs()
+
+    def release_host(self):
+        """svp_host_free every host_numa block (else the context frees them at close).  The
+        buffer views must not be used afterwards."""
+        for a in self.host_blocks:
+            self.ctx.host_free(a)
+        self.host_blocks = []
+        self.bufs, self.raw = [], []
 
     def load_inputs(self):
         for i, s in enumerate(self.specs):

@@ -23,7 +23,7 @@ def test_library_exports_every_declared_symbol():
     assert set(declared) == set(svp.EXPORTS), (set(declared) ^ set(svp.EXPORTS))
     for name in declared:
         assert hasattr(L, name), name
-    assert L.svp_abi_version() == 5
+    assert L.svp_abi_version() == 6
 
 
 @pytest.mark.skipif(bool(os.environ.get("SVP_LIB")), reason="SVP_LIB selects a sanitizer build on purpose")
@@ -246,3 +246,21 @@ def test_use_after_finalize_and_null_context():
     L = svp.load()
     assert L.svp_flush(None) == svp.SVP_E_INVAL
     assert L.svp_finalize(None) in (svp.SVP_OK, svp.SVP_E_INVAL)
+
+
+def test_host_alloc_rejects_dry_run_and_bad_args():
+    """svp_host_alloc needs CUDA (page-locking); a dry-run context answers UNSUPPORTED, and
+    argument errors / unknown pointers answer INVAL without touching the allocator."""
+    with svp.Context(dry_run=True) as c:
+        with pytest.raises(svp.SvpError) as e:
+            c.host_alloc(0, 4096)
+        assert e.value.status == svp.SVP_E_UNSUPPORTED
+        with pytest.raises(svp.SvpError) as e:
+            c.host_alloc(0, 0)
+        assert e.value.status == svp.SVP_E_INVAL
+        with pytest.raises(svp.SvpError) as e:
+            c.host_alloc(5, 4096)
+        assert e.value.status == svp.SVP_E_INVAL
+        with pytest.raises(svp.SvpError) as e:
+            c.host_free(0x1000)
+        assert e.value.status == svp.SVP_E_INVAL

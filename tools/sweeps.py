@@ -10,6 +10,9 @@ S2 (Fig 10b + Eq 9): one vecadd VP of n = k tiles; kernel t
 S3 (Fig 9 + Eq 7/8): N host-resident SGEMM jobs (H2D A,B -> kernel ->
     D2H C) with Tk ~ Tm, interleaved on separate copy/compute streams vs one stream;
     measured speedup next to Eq 7's prediction from the measured Tm, Tk.
+S3a (Fig 9a): two interleaved host-resident programs, input size fixed,
+    kernel length varied (tensor-core SGEMM K-chunk count, FFMA); speedup vs Tk / Tm.  Run
+    with --only a (not in the default set).
 S4 (BASELINE metric): jobs/s of the cfg5 mix vs #VPs (1 GPU).
 S5 (Table 1): N VPs each running the paper's program -- 300
     multiplications of two 320x320 fp64 matrices -- coalesced per program-order level vs
@@ -140,6 +143,51 @@ def s3_interleaving(quick):
                      "interleaved_ms": res["interleaved"] * 1e3, "speedup": res["serial"] / res["interleaved"],
                      "eq7_pred_ms": eq7, "eq8_speedup_if_equal": 3 * N / (2 + N)})
     return {"sgemm_n": n, "rows": rows}
+
+
+def s3a_kernel_length(quick):
+    """Fig 9(a): two interleaved programs (H2D -> kernel -> D2H), the input
+    size fixed and the kernel's length varied.  Every point is the same 3072^3 host-resident
+    SGEMM per program (so Tm is the same), and the kernel length is set by the tensor-core
+    SGEMM's K-chunk count (sgemm_kchunk: each chunk's partial sums are folded into C, so
+    more chunks = a longer kernel computing the same product), the FFMA kernel and the
+    plain-load kernel.  Serial vs interleaved with the measured Tm, Tk; Eq 7's prediction
+    2 Tm + N max(Tm, Tk), and the three-engine flow-shop bound."""
+    n, N = 3072, 2
+    variants = [("tf32bf16", svp.SGEMM_TF32BF16, kc, n) for kc in
+                ([1536, 256, 64, 16] if quick else [1536, 1024, 512, 256, 128, 64, 32, 16])]
+    variants.append(("ffma", svp.SGEMM_FFMA, None, n))
+    # K = n - 1: a row pitch TMA cannot address -> the plain-load kernel (shape key 2), the
+    # slowest of the four; its copies are 1/n (0.03 %) shorter than the others'
+    variants.append(("plain_load", svp.SGEMM_FFMA, None, n - 1))
+    rows = []
+    for label, impl, kc, K in variants:
+        specs = [W.JobSpec(v, "sgemm", M=n, N=n, K=K) for v in range(N)]
+        inputs = [W.make_inputs(s) for s in specs]
+        res = {}
+        for name, kw in (("interleaved", dict(coalesce=False, interleave=True)),
+                         ("serial", dict(coalesce=False, interleave=False))):
+            c = ctx_for(sgemm_impl=impl, sgemm_kchunk=kc, profile_level=1, arena_bytes=4 << 30, **kw)
+            vs = VPSet(c, specs, inputs, "host")
+            res[name] = flush_time(c, vs.job_list(), reps=3, warm=1)
+            if name == "serial":
+                ops = c.plan()
+                tin = statistics.median([o["measured_ns"] for o in ops if o["kind"] == svp.OP_H2D]) / 1e6
+                tk = statistics.median([o["measured_ns"] for o in ops if o["kind"] == svp.OP_KERNEL]) / 1e6
+                tout = statistics.median([o["measured_ns"] for o in ops if o["kind"] == svp.OP_D2H]) / 1e6
+            c.close()
+            del vs
+            torch.cuda.empty_cache()
+        rows.append({"kernel": label, "sgemm_kchunk": kc, "K": K, "Tin_ms": tin, "Tk_ms": tk, "Tout_ms": tout,
+                     "Tk_over_Tm": tk / tin, "serial_ms": res["serial"] * 1e3,
+                     "interleaved_ms": res["interleaved"] * 1e3, "speedup": res["serial"] / res["interleaved"],
+                     "eq7_pred_ms": 2 * tin + N * max(tin, tk),
+                     "eq7_pred_speedup": res["serial"] * 1e3 / (2 * tin + N * max(tin, tk)),
+                     # three engines (H2D copy, compute, D2H copy) as a flow shop of N identical
+                     # programs: the first program's three stages + (N - 1) x the slowest stage
+                     "flowshop_pred_ms": tin + tk + tout + (N - 1) * max(tin, tk, tout)})
+    rows.sort(key=lambda r: r["Tk_ms"])
+    return {"sgemm_n": n, "programs": N, "rows": rows}
 
 
 def s4_vps(quick):
@@ -279,6 +327,8 @@ def main():
         res["S2_staircase_fig10b"] = s2_staircase(args.quick)
     if "3" in args.only:
         res["S3_interleaving_fig9"] = s3_interleaving(args.quick)
+    if "a" in args.only:
+        res["S3a_kernel_length_fig9a"] = s3a_kernel_length(args.quick)
     if "4" in args.only:
         res["S4_jobs_vs_vps"] = s4_vps(args.quick)
     if "5" in args.only:
