@@ -301,7 +301,10 @@ class Arm:
     """One svp.Context driving this process's GPUs, and the workload's VP buffers (one or
     more rotating buffer sets) pre-marshalled as JobBatches."""
 
-    def __init__(self, specs, inputs, residency, ordinals, streams, nsets=1, kids=None, host_numa=False, **cfg):
+    def __init__(self, specs, inputs, residency, ordinals, streams, nsets=1, kids=None, host_numa=False,
+                 share=None, **cfg):
+        """share: another device-resident Arm whose buffer sets (and job batches) this one
+        reuses -- its VPs are placed on the same GPUs by the same deterministic LPT."""
         from paper_conf_dac_jungc15_b200 import svp
         from paper_conf_dac_jungc15_b200.vpset import VPSet
         self.svp = svp
@@ -309,12 +312,16 @@ class Arm:
         self.streams = streams
         self.ctx = svp.Context(num_gpus=len(self.ordinals), device_ids=self.ordinals,
                                external_streams=[st.cuda_stream for st in streams], **cfg)
-        self.sets = [VPSet(self.ctx, specs, inputs, residency,
-                           device_ordinals=self.ordinals if residency == "device" else None,
-                           host_numa=host_numa)
-                     for _ in range(nsets)]
+        if share is not None:
+            share.sets[0].assign_to(self.ctx)
+            self.sets, self.batches = share.sets, share.batches
+        else:
+            self.sets = [VPSet(self.ctx, specs, inputs, residency,
+                               device_ordinals=self.ordinals if residency == "device" else None,
+                               host_numa=host_numa)
+                         for _ in range(nsets)]
+            self.batches = [svp.JobBatch(vs.job_list()) for vs in self.sets]
         self.kids = self.sets[0].kids
-        self.batches = [svp.JobBatch(vs.job_list()) for vs in self.sets]
         self.i = 0
 
     def step(self):
@@ -470,11 +477,17 @@ def run_svp(args, rank, ws, local):
     f4 = dict(hetero=bool(args.hetero), graph=bool(args.graph), table_mode=args.table_mode)
 
     # ---------------- device-resident run (value)
-    arm = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, validate_ptrs=True,
-              sgemm_impl=impl, sgemm_kchunk=args.sgemm_kchunk, **f4)
+    # timed at the library's default profile_level 0 (no per-op events); the per-GPU
+    # Profiler numbers come from a profiled pass over the same buffers right after
+    arm = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=args.timed_profile_level,
+              validate_ptrs=True, sgemm_impl=impl, sgemm_kchunk=args.sgemm_kchunk, **f4)
     kids = arm.kids
     assert arm.ctx.flush_stats is not None
     arm.step()
+    if args.graph:
+        # steady state of the plan cache: every buffer set's plan seen twice (planned, then
+        # captured), so the timed steps replay graphs (setup, before the W warm-up steps)
+        arm.steps(2 * len(arm.batches))
     for d in set(ords):
         torch.cuda.synchronize(d)
     clocks = Clocks(sorted(set(ords)))  # sampling starts before the warm-up (nvidia-smi start-up)
@@ -491,17 +504,31 @@ def run_svp(args, rank, ws, local):
     value = n_jobs_total * args.steps / dt_max
     st = arm.ctx.flush_stats()
     launches = launches_per_flush(arm.ctx) * args.steps
-    main_kstats = {name: arm.ctx.kernel_stats(kid) for name, kid in kids.items()}
+    # profiled pass (profile_level 1, same buffers, same options): per-GPU spans, kernel
+    # times and the interleaved step's per-kernel times
+    if args.timed_profile_level >= 1:
+        pa, prof_steps = arm, args.steps
+    else:
+        pa = Arm(specs, inputs, "device", ords, streams, share=arm, profile_level=1, sgemm_impl=impl,
+                 sgemm_kchunk=args.sgemm_kchunk, **f4)
+        prof_steps = max(3, min(args.steps, 20))
+        pa.steps((2 if args.graph else 1) * len(pa.batches) + 1)
+        pa.ctx.reset_profile()
+        pa.timed(prof_steps)
+    pst = pa.ctx.flush_stats()
+    main_kstats = {name: pa.ctx.kernel_stats(kid) for name, kid in kids.items()}
     if args.hetero:
-        main_kstats["ew_mix"] = arm.ctx.kernel_stats(svp.KERNEL_EW_MIX)
-    dstats = arm.device_stats()
+        main_kstats["ew_mix"] = pa.ctx.kernel_stats(svp.KERNEL_EW_MIX)
+    dstats = pa.device_stats()
+    if pa is not arm:
+        pa.close()
     gpus_driven = sum(1 for d in dstats if d["flushes"] > 0)
     per_gpu_rows = []
     for g, (d, t) in enumerate(zip(dstats, dt_per_gpu)):
         per_gpu_rows.append({"gpu": g, "ordinal": d["ordinal"], "vps": d["vps"],
                              "lpt_est_load_ms": d["est_load_ns"] / 1e6,  # VPSet's estimated kernel ns
-                             "device_ms_per_step": d["device_ns"] / args.steps / 1e6,
-                             "kernel_ms_per_step": d["kernel_ns"] / args.steps / 1e6,
+                             "device_ms_per_step": d["device_ns"] / prof_steps / 1e6,
+                             "kernel_ms_per_step": d["kernel_ns"] / prof_steps / 1e6,
                              "event_ms_per_step": t / args.steps * 1e3})
     spans = [r["device_ms_per_step"] for r in per_gpu_rows]
     loads = [r["lpt_est_load_ms"] for r in per_gpu_rows]
@@ -516,7 +543,7 @@ def run_svp(args, rank, ws, local):
     trace("timed region done")
 
     # ---------------- one stream per GPU: per-kernel roofline numbers (launches do not overlap)
-    iso = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, interleave=False, sgemm_impl=impl,
+    iso = Arm(specs, inputs, "device", ords, streams, share=arm, profile_level=1, interleave=False, sgemm_impl=impl,
               sgemm_kchunk=args.sgemm_kchunk)
     iso.step()
     iso.ctx.reset_profile()
@@ -554,7 +581,7 @@ def run_svp(args, rank, ws, local):
         if args.sgemm_kchunk != 0 and impl != IMPLS["ffma"]:
             variants.append((args.sgemm_impl, 0))  # one accumulation per tile: the cost of R23's chunks
         for alt_name, kc in variants:
-            a = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=1, sgemm_impl=IMPLS[alt_name],
+            a = Arm(specs, inputs, "device", ords, streams, share=arm, profile_level=1, sgemm_impl=IMPLS[alt_name],
                     sgemm_kchunk=kc)
             a.step()
             a.ctx.reset_profile()
@@ -575,10 +602,11 @@ def run_svp(args, rank, ws, local):
                          ("B2_serial_async", dict(coalesce=False, interleave=False)),
                          ("B3_serial_graph", dict(coalesce=False, interleave=False, graph=True)),
                          ("B2_profiled", dict(coalesce=False, interleave=False, profile_level=1))):
-            # B3 replays one captured graph, so it needs the same buffers every step: one set
-            b = Arm(specs, inputs, "device", ords, streams, 1 if name == "B3_serial_graph" else nsets,
-                    sgemm_impl=impl, sgemm_kchunk=args.sgemm_kchunk, **kw)
-            b.steps(max(3, args.warmup))  # B3: plan, capture + instantiate, then replays only
+            # same buffer sets as the coalesced arm; B3 replays one captured graph per set
+            b = Arm(specs, inputs, "device", ords, streams, share=arm, sgemm_impl=impl,
+                    sgemm_kchunk=args.sgemm_kchunk, **kw)
+            # B3: each set's plan, then its capture + instantiate, then replays only
+            b.steps(max(3, args.warmup) + (2 * len(b.batches) if kw.get("graph") else 0))
             b.ctx.reset_profile()
             barrier(ws)
             ks = max(2, args.steps // 5)
@@ -586,8 +614,6 @@ def run_svp(args, rank, ws, local):
             if name != "B2_profiled":
                 serial[name] = {"value": n_jobs_total * ks / sdt, "unit": "jobs/s", "steps": ks,
                                 "ms_per_step": sdt / ks * 1e3}
-                if name == "B3_serial_graph" and nsets > 1:
-                    serial[name]["l2"] = "one buffer set (a replayed graph reads the same buffers): L2-resident"
             else:
                 # Eq 9's alignment gain per kernel class: per-job launches vs one coalesced
                 # launch of the same jobs (event-timed kernel time per step, 1 stream each)
@@ -668,14 +694,15 @@ def run_svp(args, rank, ws, local):
             "sgemm_impl": args.sgemm_impl, "sgemm_kchunk": args.sgemm_kchunk, "alt_sgemm_impls": alt, "hetero": args.hetero, "graph": args.graph,
             "table_mode": args.table_mode,
             "graph_replays_last_step": int(st["graph_replays"]),
-            "timed_kernel_ms_per_step": {n: k["total_ns"] / args.steps / 1e6 for n, k in main_kstats.items()
+            "timed_kernel_ms_per_step": {n: k["total_ns"] / prof_steps / 1e6 for n, k in main_kstats.items()
                                          if k["launches"]},
             "speedup_vs_serial": {k: value / v["value"] for k, v in serial.items()},
             "serial": serial, "speedup_by_kernel_class": by_kernel, "per_kernel": per_kernel,
             "one_stream": {"value": iso_value, "unit": "jobs/s",
                            "note": "coalesced, 1 compute stream (no interleaving); per_kernel/roofline timed here"},
             "flush": {"host_plan_us": st["host_plan_ns"] / 1e3, "host_issue_us": st["host_issue_ns"] / 1e3,
-                      "host_total_us": st["host_total_ns"] / 1e3, "device_ms": st["device_ns"] / 1e6,
+                      "host_total_us": st["host_total_ns"] / 1e3, "device_ms": pst["device_ns"] / 1e6,
+                      "timed_profile_level": args.timed_profile_level,
                       "groups": int(st["groups"]), "launch_ops": int(st["launches"])},
             "parity": "tests/test_gpu_parity.py, test_gpu_sgemm_*.py (full-size configs vs oracle; not re-run here)",
             "profiler_split": "per-VP attribution inside a coalesced launch: parity unpinned (DESIGN.md §3)",
@@ -707,12 +734,15 @@ def main():
     ap.add_argument("--no-weak", action="store_true", help="N > 1: skip the extra weak-scaling measurement")
     ap.add_argument("--hetero", type=int, default=0, choices=[0, 1],
                     help="heterogeneous coalescing of vecadd/SAXPY/Black-Scholes (NEXT f4)")
-    ap.add_argument("--graph", type=int, default=0, choices=[0, 1],
-                    help="steady-state plan reuse + CUDA graph replay (NEXT f4)")
+    ap.add_argument("--graph", type=int, default=1, choices=[0, 1],
+                    help="plan cache + CUDA graph replay (NEXT f4; the library default since ABI 6)")
     ap.add_argument("--table-mode", type=int, default=1, choices=[0, 1],
                     help="segment tables: 0 global device buffer, 1 by-value kernel parameter")
     ap.add_argument("--host-numa", type=int, default=1, choices=[0, 1],
                     help="e2e: host buffers from svp_host_alloc on the VP's GPU's NUMA node (0: torch pinned)")
+    ap.add_argument("--timed-profile-level", type=int, default=0, choices=[0, 1, 2],
+                    help="profile_level of the timed context (default 0, the library default: no per-op events; "
+                         "per-GPU / per-kernel numbers then come from a profiled pass over the same buffers)")
     ap.add_argument("--no-serial", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other sgemm implementation")
     ap.add_argument("--no-e2e", action="store_true")

@@ -103,11 +103,15 @@ typedef struct svp_config {
     int32_t hetero;              /* 1: heterogeneous coalescing -- the vecadd, SAXPY and
                                     Black-Scholes groups of one (level, GPU) share ONE launch
                                     whose segment table names each segment's kernel          */
-    int32_t graph;               /* 1: steady-state replay -- a flush whose requests (VP,
-                                    kernel, args, buffers, in order) equal the previous
-                                    flush's reuses its plan and tables, and from the second
-                                    repeat on replays the flush's device work as one CUDA
-                                    graph per GPU.  Ignored with sync_each_job.              */
+    int32_t graph;               /* 1 (default since ABI 6): steady-state replay -- a flush
+                                    whose requests (VP, kernel, args, buffers, in order)
+                                    equal those of one of the last 32 successful flushes
+                                    reuses that plan, and on its second sighting captures the
+                                    flush's device work as one CUDA graph per GPU (with a
+                                    private copy of its device tables), replayed on every
+                                    later sighting.  A loop that rotates input buffer sets
+                                    therefore replays one graph per set.  Results are the
+                                    same with 0.  Ignored with sync_each_job.               */
     int32_t table_mode;          /* where a coalesced launch finds its segment table (SURVEY
                                     §8(b)): SVP_TABLE_PARAM (default) -- launches of
                                     elementwise / hist256 groups with <= 64 VPs receive it
@@ -131,7 +135,7 @@ enum { SVP_TABLE_GLOBAL = 0, SVP_TABLE_PARAM = 1 };
 
 /* Fill *cfg with defaults: num_gpus 0, 4 compute streams, coalesce 1, interleave 1,
    max_chunks 8, profile_level 0, validate_ptrs 1, sgemm_impl SVP_SGEMM_TF32BF16,
-   table_mode SVP_TABLE_PARAM, sgemm_kchunk 768, rest 0 (hetero 0, graph 0). */
+   table_mode SVP_TABLE_PARAM, sgemm_kchunk 768, graph 1, rest 0 (hetero 0). */
 void svp_config_default(svp_config* cfg);
 
 /* Create a context.  On success *out owns streams/events/threads for every GPU.
@@ -343,7 +347,7 @@ typedef struct svp_flush_stats {
     double device_ns;        /* first-op start to last-op end (profile_level >= 1) */
     double sim_makespan_ns;  /* cost-model makespan of the plan (always)           */
     double sim_serial_ns;    /* cost-model time of the same ops run one at a time  */
-    uint64_t plan_reused;    /* cfg.graph: 1 if the previous flush's plan was reused */
+    uint64_t plan_reused;    /* cfg.graph: 1 if a recent flush's plan was reused     */
     uint64_t graph_replays;  /* cfg.graph: GPUs whose work ran as a replayed CUDA graph */
     uint64_t kernel_launches; /* kernels actually launched (`launches` counts coalesced
                                  launch ops; hist256's zeroing kernel and the SGEMM tail

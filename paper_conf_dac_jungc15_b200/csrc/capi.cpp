@@ -97,6 +97,7 @@ void svp_config_default(svp_config* cfg) {
     cfg->validate_ptrs = 1;
     cfg->sgemm_impl = SVP_SGEMM_TF32BF16;
     cfg->table_mode = SVP_TABLE_PARAM;
+    cfg->graph = 1;           // plan cache + graph replay (every BASELINE config gains, profiles/r02/graph/)
     cfg->sgemm_kchunk = 768;  // R23: the tensor-core splits' fp32 contract for any K and operand signs
 }
 
@@ -317,17 +318,25 @@ static svp_status do_flush(Ctx* c) {
     }
     memset(&c->fstats, 0, sizeof(c->fstats));
     svp_status st = SVP_OK;
-    // Steady-state replay (cfg.graph, NEXT f4): the same requests as the previous flush
-    // get the same plan, so copy it (and, in the executor, its tables and CUDA graph).
-    const bool reuse = c->cfg.graph && !c->cfg.sync_each_job && c->last_ok && same_requests(f.jobs, c->last.jobs);
+    // Steady-state replay (cfg.graph, NEXT f4): the same requests as a recent flush (the
+    // previous one, or one of the Ctx::kPlanCache before it -- a serving loop that alternates
+    // input buffer sets alternates plans) get the same plan, so copy it (and, in the
+    // executor, replay its CUDA graph).  A mismatch is found at the first differing job.
+    const Flush* hit = nullptr;
+    if (c->cfg.graph && !c->cfg.sync_each_job) {
+        if (c->last_ok && same_requests(f.jobs, c->last.jobs)) hit = &c->last;
+        for (size_t k = 0; !hit && k < c->plan_cache.size(); ++k)
+            if (same_requests(f.jobs, c->plan_cache[k].jobs)) hit = &c->plan_cache[k];
+    }
+    const bool reuse = hit != nullptr;
     if (reuse) {
-        for (size_t i = 0; i < f.jobs.size(); ++i) f.jobs[i].level = c->last.jobs[i].level;
-        f.groups = c->last.groups;
-        f.chunks = c->last.chunks;
-        f.ops = c->last.ops;
+        for (size_t i = 0; i < f.jobs.size(); ++i) f.jobs[i].level = hit->jobs[i].level;
+        f.groups = hit->groups;
+        f.chunks = hit->chunks;
+        f.ops = hit->ops;
         for (auto& o : f.ops) o.measured_ns = o.measured_start_ns = -1;
-        f.levels = c->last.levels;
-        f.plan_gen = c->last.plan_gen;
+        f.levels = hit->levels;
+        f.plan_gen = hit->plan_gen;
         f.reused = true;
         c->fstats.plan_reused = 1;
     } else {
@@ -374,6 +383,19 @@ static svp_status do_flush(Ctx* c) {
             if (op.kind == SVP_OP_D2H) c->fstats.d2h_bytes += op.bytes;
         }
         c->fstats.launches = launches;
+    }
+    if (c->cfg.graph && c->last_ok && !c->last.jobs.empty()) {
+        // the previous flush joins the plan cache (most recent first, one entry per plan)
+        const uint64_t gen = c->last.plan_gen;
+        for (size_t k = 0; k < c->plan_cache.size();)
+            if (c->plan_cache[k].plan_gen == gen || c->plan_cache[k].plan_gen == f.plan_gen)
+                c->plan_cache.erase(c->plan_cache.begin() + (long)k);
+            else
+                ++k;
+        if (gen != f.plan_gen) {
+            c->plan_cache.insert(c->plan_cache.begin(), std::move(c->last));
+            if (c->plan_cache.size() > Ctx::kPlanCache) c->plan_cache.pop_back();
+        }
     }
     c->last = std::move(f);
     c->last_ok = st == SVP_OK;

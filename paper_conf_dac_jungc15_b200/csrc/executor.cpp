@@ -92,10 +92,19 @@ struct Dev {
     std::unordered_map<MapKey, Maps2, MapKeyHash> map_cache;
     std::string err;
     uint64_t table_uploads = 0;
-    // steady-state replay (cfg.graph): the device work of plan `gexec_gen` as one graph
-    cudaGraphExec_t gexec = nullptr;
-    uint64_t gexec_gen = 0;
-    std::vector<int32_t> g_tstart;      // profiling event slots of each op inside the graph
+    // steady-state replay (cfg.graph): the device work of each recently seen plan as one
+    // graph, keyed by plan generation (a serving loop that alternates input buffer sets
+    // alternates plans).  Each graph owns a copy of its plan's device tables: the shared
+    // tbl_dev holds whatever plan ran last.
+    struct GraphEntry {
+        cudaGraphExec_t gexec = nullptr;
+        std::vector<int32_t> tstart;    // profiling event slots of each op inside the graph
+        uint8_t* tbl = nullptr;         // the plan's device tables (device-table launches)
+        size_t tbl_cap = 0;
+        uint64_t last_use = 0;
+    };
+    std::unordered_map<uint64_t, GraphEntry> graphs;
+    uint64_t graph_clock = 0;
     cudaEvent_t fork_ev = nullptr;
     std::vector<cudaEvent_t> join_ev;
 };
@@ -199,7 +208,11 @@ static void dev_teardown(Dev& d) {
     for (auto e : d.end_ev) cudaEventDestroy(e);
     for (auto e : d.join_ev) cudaEventDestroy(e);
     if (d.fork_ev) cudaEventDestroy(d.fork_ev);
-    if (d.gexec) cudaGraphExecDestroy(d.gexec);
+    for (auto& kv : d.graphs) {
+        if (kv.second.gexec) cudaGraphExecDestroy(kv.second.gexec);
+        if (kv.second.tbl) cudaFree(kv.second.tbl);
+    }
+    d.graphs.clear();
     if (d.ext_ev) cudaEventDestroy(d.ext_ev);
     if (d.tbl_ev) cudaEventDestroy(d.tbl_ev);
     if (d.arena) cudaFree(d.arena);
@@ -828,11 +841,24 @@ static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bo
     return pool[i];
 }
 
-static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int cfg_kchunk, cudaStream_t s) {
+// Captured graphs hold the addresses of the per-device scratch buffers: a reallocation
+// drops every one of them (they are re-captured on the plans' next sightings).
+static svp_status drop_graphs(Dev& d) {
+    for (auto& kv : d.graphs) {
+        if (kv.second.gexec) CK(cudaGraphExecDestroy(kv.second.gexec));
+        if (kv.second.tbl) CK(cudaFree(kv.second.tbl));
+    }
+    d.graphs.clear();
+    return SVP_OK;
+}
+
+static constexpr size_t kGraphsPerDevice = 32;
+
+// base: the device table buffer the launch reads (d.tbl_dev, or a captured plan's own copy)
+static cudaError_t launch_chunk(Dev& d, const Chunk& ch, int cfg_kchunk, cudaStream_t s, const uint8_t* base) {
     const int sgemm_impl = ch.sgemm_impl;
     const int kchunk = sgemm_chunk_k(sgemm_impl, cfg_kchunk);
     if (ch.total_tiles == 0 && ch.kernel != K_HIST256) return cudaSuccess;
-    const uint8_t* base = d.tbl_dev;
     uint64_t* busy = ch.busy_off >= 0 ? d.busy_dev + ch.busy_off : nullptr;
     uint32_t* sched = ch.sched_slot >= 0 ? d.sched_dev + 2 * ch.sched_slot : nullptr;
     uint32_t* hscr = ch.hscr_off >= 0 ? d.hscr_dev + ch.hscr_off : nullptr;
@@ -927,10 +953,10 @@ static bool chunk_needs_launch(const Flush& f, const Chunk& ch) {
 
 bool executor_chunk_launches(const Flush& f, const Chunk& ch) { return chunk_needs_launch(f, ch); }
 
-static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool capturing, std::vector<int>& used,
-                            std::vector<int32_t>& tstart);
-static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool upload, const std::vector<int>& used,
-                                const std::vector<int32_t>& tstart,
+static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool capturing, const uint8_t* base,
+                            cudaStream_t direct, std::vector<int>& used, std::vector<int32_t>& tstart);
+static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool upload, bool direct,
+                                const std::vector<int>& used, const std::vector<int32_t>& tstart,
                                 std::chrono::steady_clock::time_point t_issue0, double* issue_ns);
 
 static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
@@ -954,14 +980,49 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             return SVP_E_NOMEM;
         }
     }
-    // ---- tables (a reused plan's chunks already carry theirs, resident since last flush)
+    // ---- steady-state replay: a reused plan replays its graph if this GPU captured one,
+    // else it is captured now (second sighting of the plan)
+    const bool graph = c->cfg.graph && f.reused && !c->cfg.sync_each_job;
+    Dev::GraphEntry* ge = nullptr;
+    if (graph) {
+        auto it = d.graphs.find(f.plan_gen);
+        if (it != d.graphs.end()) ge = &it->second;
+    }
+    bool replay = ge && ge->gexec;
+    // ---- tables (a replayed graph carries its own; everything else builds them)
     std::vector<uint8_t> tbl;
-    if (!f.reused) {
+    if (!replay) {
         svp_status st = build_tables(e, d, f, tbl);
         if (st) return st;
     }
     auto t_issue0 = std::chrono::steady_clock::now();
-    if (d.ext) {
+    // tables changed -> new host copy; the device copy is refreshed only if some launch on
+    // this GPU reads the global table (param-mode launches carry theirs by value)
+    if (!replay && !tbl.empty() &&
+        (tbl.size() != d.tbl_last.size() || memcmp(tbl.data(), d.tbl_last.data(), tbl.size()))) {
+        d.tbl_last.swap(tbl);
+        d.tbl_dev_valid = false;
+    }
+    bool need_dev = false;
+    for (const auto& ch : f.chunks)
+        if (ch.device == d.idx && !ch.param && chunk_needs_launch(f, ch)) need_dev = true;
+    const bool capture = graph && !replay;
+    // a capture reads its own table copy (below), not the shared buffer
+    const bool upload = !replay && !capture && need_dev && !d.tbl_dev_valid && !d.tbl_last.empty();
+    // direct issue: when every op of this GPU is on one plan stream and nothing needs the
+    // control stream (no upload, no graph), the ops go straight onto the caller's stream --
+    // no fork / join events (a launch-bound flush: 7 -> 3 stream calls)
+    bool direct = d.ext != nullptr && !graph && !upload;
+    {
+        int one = -1;
+        for (const auto& o : f.ops) {
+            if (!direct) break;
+            if (o.device != d.idx) continue;
+            if (one < 0) one = o.stream;
+            else if (o.stream != one) direct = false;
+        }
+    }
+    if (d.ext && !direct) {
         // only the streams this flush uses on this GPU (and stream 0: table upload, capture)
         std::vector<char> touch(d.streams.size(), 0);
         touch[0] = 1;
@@ -971,17 +1032,6 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
         for (size_t s = 0; s < d.streams.size(); ++s)
             if (touch[s]) CK(cudaStreamWaitEvent(d.streams[s], d.ext_ev, 0));
     }
-    // tables changed -> new host copy; the device copy is refreshed only if some launch on
-    // this GPU reads the global table (param-mode launches carry theirs by value)
-    if (!f.reused && !tbl.empty() &&
-        (tbl.size() != d.tbl_last.size() || memcmp(tbl.data(), d.tbl_last.data(), tbl.size()))) {
-        d.tbl_last.swap(tbl);
-        d.tbl_dev_valid = false;
-    }
-    bool need_dev = false;
-    for (const auto& ch : f.chunks)
-        if (ch.device == d.idx && !ch.param && chunk_needs_launch(f, ch)) need_dev = true;
-    const bool upload = need_dev && !d.tbl_dev_valid && !d.tbl_last.empty();
     if (upload) {
         const size_t bytes = d.tbl_last.size();
         if (bytes > d.tbl_cap) {
@@ -1019,9 +1069,9 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             }
         }
         if (nbusy > d.busy_cap) {
-            if (d.gexec) {  // a captured graph holds the old counter addresses
-                CK(cudaGraphExecDestroy(d.gexec));
-                d.gexec = nullptr;
+            {
+                svp_status gs = drop_graphs(d);  // captured graphs hold the old counter addresses
+                if (gs) return gs;
             }
             if (d.busy_dev) CK(cudaFree(d.busy_dev));
             d.busy_dev = nullptr;
@@ -1062,9 +1112,9 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             }
         }
         if (nh > d.hscr_cap) {
-            if (d.gexec) {
-                CK(cudaGraphExecDestroy(d.gexec));
-                d.gexec = nullptr;
+            {
+                svp_status gs = drop_graphs(d);
+                if (gs) return gs;
             }
             if (d.hscr_dev) CK(cudaFree(d.hscr_dev));
             d.hscr_dev = nullptr;
@@ -1075,9 +1125,9 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             d.hscr_cap = cap;
         }
         if (nslot > d.sched_cap) {
-            if (d.gexec) {  // a captured graph holds the old counter addresses
-                CK(cudaGraphExecDestroy(d.gexec));
-                d.gexec = nullptr;
+            {
+                svp_status gs = drop_graphs(d);  // captured graphs hold the old counter addresses
+                if (gs) return gs;
             }
             // the previous flush's launches have finished (svp_flush is synchronous)
             if (d.sched_dev) CK(cudaFree(d.sched_dev));
@@ -1089,16 +1139,39 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             d.sched_cap = cap;
         }
     }
+    if (replay && d.graphs.find(f.plan_gen) == d.graphs.end()) {
+        // cannot happen: a replayed plan needs no more scratch than when it was captured,
+        // and any growth since then dropped its graph before this flush
+        d.err = "internal: the graph of a replayed plan was dropped during its flush";
+        return SVP_E_STATE;
+    }
     // ---- steady-state replay: second sighting of a plan -> capture, later -> replay
     std::vector<int> used(d.streams.size(), 0);
     std::vector<int32_t> tstart(f.ops.size(), -1);
-    const bool graph = c->cfg.graph && f.reused && !c->cfg.sync_each_job;
-    bool replay = graph && d.gexec && d.gexec_gen == f.plan_gen;
+    const uint8_t* base = d.tbl_dev;
     bool capturing = false;
-    if (graph && !replay) {
-        if (d.gexec) {
-            CK(cudaGraphExecDestroy(d.gexec));
-            d.gexec = nullptr;
+    if (capture) {
+        // the entry for this plan (evicting the least recently used one past the cap); its
+        // device tables are a private copy, uploaded before the capture begins
+        if (d.graphs.size() >= kGraphsPerDevice) {
+            auto lru = d.graphs.begin();
+            for (auto it = d.graphs.begin(); it != d.graphs.end(); ++it)
+                if (it->second.last_use < lru->second.last_use) lru = it;
+            if (lru->second.gexec) CK(cudaGraphExecDestroy(lru->second.gexec));
+            if (lru->second.tbl) CK(cudaFree(lru->second.tbl));
+            d.graphs.erase(lru);
+        }
+        ge = &d.graphs[f.plan_gen];
+        if (need_dev && !d.tbl_last.empty()) {
+            const size_t bytes = d.tbl_last.size();
+            if (bytes > ge->tbl_cap) {
+                if (ge->tbl) CK(cudaFree(ge->tbl));
+                ge->tbl = nullptr;
+                CK(cudaMalloc(&ge->tbl, bytes));
+                ge->tbl_cap = bytes;
+            }
+            CK(cudaMemcpy(ge->tbl, d.tbl_last.data(), bytes, cudaMemcpyHostToDevice));
+            base = ge->tbl;
         }
         CK(cudaStreamBeginCapture(d.streams[0], cudaStreamCaptureModeThreadLocal));
         capturing = true;
@@ -1114,7 +1187,7 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             return cs;
         }
     }
-    svp_status ist = replay ? SVP_OK : issue_ops(e, d, f, prof, capturing, used, tstart);
+    svp_status ist = replay ? SVP_OK : issue_ops(e, d, f, prof, capturing, base, direct ? d.ext : nullptr, used, tstart);
     if (capturing) {
         // join every stream back into stream 0, close the capture, instantiate
         svp_status js = ist;
@@ -1136,33 +1209,33 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             d.err = std::string("cudaStreamEndCapture: ") + cudaGetErrorString(ce);
             return SVP_E_CUDA;
         }
-        ce = cudaGraphInstantiate(&d.gexec, g, 0);
+        ce = cudaGraphInstantiate(&ge->gexec, g, 0);
         cudaGraphDestroy(g);
         if (ce != cudaSuccess) {
-            d.gexec = nullptr;
+            ge->gexec = nullptr;
             d.err = std::string("cudaGraphInstantiate: ") + cudaGetErrorString(ce);
             return SVP_E_CUDA;
         }
-        d.gexec_gen = f.plan_gen;
-        d.g_tstart = tstart;
+        ge->tstart = tstart;
         replay = true;
     } else if (ist) {
         return ist;
     }
     if (replay) {
-        CK(cudaGraphLaunch(d.gexec, d.streams[0]));
-        tstart = d.g_tstart;
+        ge->last_use = ++d.graph_clock;
+        CK(cudaGraphLaunch(ge->gexec, d.streams[0]));
+        tstart = ge->tstart;
         std::fill(used.begin(), used.end(), 0);
         used[0] = 1;
         std::lock_guard<std::mutex> lk(c->pmu);
         c->fstats.graph_replays += 1;
     }
-    return finish_device(e, d, f, prof, upload, used, tstart, t_issue0, issue_ns);
+    return finish_device(e, d, f, prof, upload, direct, used, tstart, t_issue0, issue_ns);
 }
 
 // Enqueue the device's ops in plan order (directly, or into an open stream capture).
-static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool capturing, std::vector<int>& used,
-                            std::vector<int32_t>& tstart) {
+static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool capturing, const uint8_t* base,
+                            cudaStream_t direct, std::vector<int>& used, std::vector<int32_t>& tstart) {
     Ctx* c = e->c;
     size_t nt = 0;
     // inside a capture, timing events become event-record nodes of the graph
@@ -1172,11 +1245,11 @@ static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool captu
     for (size_t i = 0; i < f.ops.size(); ++i) {
         Op& o = f.ops[i];
         if (o.device != d.idx) continue;
-        cudaStream_t s = d.streams[o.stream + 1];
-        used[o.stream + 1] = 1;
-        for (int32_t p : o.wait_ops) {
+        cudaStream_t s = direct ? direct : d.streams[o.stream + 1];
+        if (!direct) used[o.stream + 1] = 1;
+        for (int32_t p : o.wait_ops) {  // (direct: one stream, already in order)
             const Op& q = f.ops[p];
-            if (q.device != d.idx) continue;
+            if (q.device != d.idx || direct) continue;
             CK(cudaStreamWaitEvent(s, d.dep_ev[p], 0));
         }
         if (prof) {
@@ -1206,13 +1279,13 @@ static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool captu
                 }
             }
         } else if (chunk_needs_launch(f, ch)) {
-            CK(launch_chunk(d, ch, c->cfg.sgemm_kchunk, s));
+            CK(launch_chunk(d, ch, c->cfg.sgemm_kchunk, s, base));
         }
         if (prof) {
             CK(rec(d.t_ev[2 * nt + 1], s));
             ++nt;
         }
-        if (o.needs_event) {
+        if (o.needs_event && !direct) {
             cudaEvent_t ev = pool_get(d, d.dep_ev, i, false);
             if (!ev) {
                 d.err = "event allocation failed";
@@ -1225,13 +1298,17 @@ static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool captu
     return SVP_OK;
 }
 
-static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool upload, const std::vector<int>& used,
-                                const std::vector<int32_t>& tstart,
+static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool upload, bool direct,
+                                const std::vector<int>& used, const std::vector<int32_t>& tstart,
                                 std::chrono::steady_clock::time_point t_issue0, double* issue_ns) {
     Ctx* c = e->c;
     // ---- join into the external stream, then wait (watchdog)
     std::vector<cudaEvent_t> finals;
-    for (size_t s = 0; s < d.streams.size(); ++s) {
+    if (direct) {  // the ops ran on the external stream itself
+        CK(cudaEventRecord(d.end_ev[0], d.ext));
+        finals.push_back(d.end_ev[0]);
+    }
+    for (size_t s = 0; s < d.streams.size() && !direct; ++s) {
         if (!used[s] && !(upload && s == 0)) continue;
         CK(cudaEventRecord(d.end_ev[s], d.streams[s]));
         finals.push_back(d.end_ev[s]);

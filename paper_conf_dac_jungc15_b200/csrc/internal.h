@@ -275,7 +275,9 @@ struct Ctx {
     }
     bool registered[K_COUNT] = {};
 
-    // last flush
+    // last flush, and (cfg.graph) the plans of the kPlanCache successful flushes before it
+    static constexpr size_t kPlanCache = 32;
+    std::vector<Flush> plan_cache;
     Flush last;
     bool last_ok = false;            // the last flush completed with SVP_OK
     uint64_t plan_gen = 0;           // bumped for every freshly planned flush

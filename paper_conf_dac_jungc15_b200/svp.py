@@ -241,7 +241,7 @@ class Context:
                  profile_level: int = 0, sync_each_job: bool = False, dry_run: bool = False,
                  flush_timeout_ms: int = 0, validate_ptrs: int = 1, sgemm_impl: int = SGEMM_TF32BF16,
                  external_streams: Optional[Sequence[int]] = None, hbm_gbps: float = 0.0, pcie_gbps: float = 0.0,
-                 ffma_tflops: float = 0.0, launch_us: float = 0.0, hetero: bool = False, graph: bool = False,
+                 ffma_tflops: float = 0.0, launch_us: float = 0.0, hetero: bool = False, graph: bool = True,
                  table_mode: int = TABLE_PARAM, sgemm_kchunk: Optional[int] = None):
         L = load()
         cfg = svp_config()

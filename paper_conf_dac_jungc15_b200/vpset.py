@@ -75,10 +75,7 @@ class VPSet:
                 self.kids[s.kernel] = ctx.kernel(s.kernel)
         self.host_blocks: List[int] = []
         if assign and (residency == "device" or host_numa):
-            # estimated kernel ns (the Dispatcher's LPT costs): algorithmic bytes at the measured
-            # 6.55 TB/s (6550 B/ns) + FLOPs at ~400 TFLOP/s (4e5 flop/ns, the fp32 tensor-core split)
-            costs = [float(s.algorithmic_bytes()) / 6550.0 + float(s.flops()) / 4.0e5 for s in self.specs]
-            ctx.assign_vps([s.vp for s in self.specs], [self.kids[s.kernel] for s in self.specs], costs)
+            self.assign_to(ctx)
         self.bufs: List[Dict[str, torch.Tensor]] = []   # views (what the kernel sees)
         self.raw: List[Dict[str, torch.Tensor]] = []    # allocations incl. misalign + guard
         self.offsets: List[Dict[str, int]] = []
@@ -120,6 +117,17 @@ class VPSet:
         self.inputs = inputs
         if inputs is not None:
             self.load_inputs()
+
+    def assign_to(self, ctx: svp.Context):
+        """Register this set's kernels in ctx and pin its VPs to GPUs with the Dispatcher's
+        kernel-stratified LPT (deterministic: a second context sharing these buffers gets
+        the same placement)."""
+        for name in self.kids:
+            ctx.kernel(name)
+        # estimated kernel ns (the Dispatcher's LPT costs): algorithmic bytes at the measured
+        # 6.55 TB/s (6550 B/ns) + FLOPs at ~400 TFLOP/s (4e5 flop/ns, the fp32 tensor-core split)
+        costs = [float(s.algorithmic_bytes()) / 6550.0 + float(s.flops()) / 4.0e5 for s in self.specs]
+        ctx.assign_vps([s.vp for s in self.specs], [self.kids[s.kernel] for s in self.specs], costs)
 
     def release_host(self):
         """svp_host_free every host_numa block (else the context frees them at close).  The

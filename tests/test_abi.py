@@ -37,7 +37,7 @@ def test_config_default():
     svp.load().svp_config_default(cfg)
     assert cfg.streams_per_gpu == 4 and cfg.coalesce == 1 and cfg.interleave == 1 and cfg.max_chunks == 8
     assert cfg.validate_ptrs == 1 and cfg.dry_run == 0 and cfg.sgemm_impl == svp.SGEMM_TF32BF16
-    assert cfg.table_mode == svp.TABLE_PARAM and cfg.hetero == 0 and cfg.graph == 0 and cfg.sgemm_kchunk == 768
+    assert cfg.table_mode == svp.TABLE_PARAM and cfg.hetero == 0 and cfg.graph == 1 and cfg.sgemm_kchunk == 768
 
 
 @pytest.mark.skipif(torch.cuda.is_available(), reason="needs a host without GPUs")

@@ -106,6 +106,39 @@ def test_graph_replans_when_requests_change(small):
         ctx.close()
 
 
+@pytest.mark.parametrize("table_mode", [svp.TABLE_GLOBAL, svp.TABLE_PARAM])
+def test_graph_alternating_buffer_sets(small, table_mode):
+    """A serving loop that rotates input buffer sets (ping-pong, or bench.py's sets that keep
+    the working set out of L2) alternates between plans.  Each set's plan is cached and its
+    graph replayed with that plan's OWN copy of the device tables (segment tables, SGEMM
+    tensor maps): a replay must never read the tables another set's flush uploaded.  Fresh
+    inputs every round, every output against the oracle."""
+    specs, _ = small
+    ctx = svp.Context(num_gpus=1, graph=True, profile_level=1, table_mode=table_mode)
+    try:
+        sets = [VPSet(ctx, specs, None, "device") for _ in range(3)]
+        jbs = [svp.JobBatch(vs.job_list()) for vs in sets]
+        seen = []
+        for r in range(9):
+            k = r % 3
+            inputs = inputs_for(specs, seed=W.BASE_SEED + 31 * r)
+            sets[k].inputs = inputs
+            sets[k].load_inputs()
+            ctx.submit_batch(jbs[k])
+            ctx.flush()
+            torch.cuda.synchronize()
+            st = ctx.flush_stats()
+            seen.append((st["plan_reused"], st["graph_replays"]))
+            for i, (s, inp) in enumerate(zip(specs, inputs)):
+                check_job(s, inp, sets[k].output(i))
+        # round 0-2: three fresh plans; 3-5: second sightings (reused plan, captured graph
+        # replayed once); 6-8: replays
+        assert seen == [(0, 0)] * 3 + [(1, 1)] * 6, seen
+        assert all(vs.guards_intact() for vs in sets)
+    finally:
+        ctx.close()
+
+
 def test_serial_graph_baseline_b3(small):
     """B3: the serial per-job launches captured in a graph are still
     per-VP correct."""

@@ -165,7 +165,7 @@ def test_tail_split_last_wave(int_inputs, residency, interleave):
 
 
 @pytest.mark.parametrize("impl", [svp.SGEMM_TF32BF16, svp.SGEMM_3XTF32])
-@pytest.mark.parametrize("kchunk", [0, 512, None])
+@pytest.mark.parametrize("kchunk", [0, 16, 512, None])
 def test_long_k_keeps_fp32_contract(impl, kchunk):
     """DESIGN R23: the tcgen05 fp32 accumulation loses ~1.7e-8 relative per accumulating MMA.
     sgemm_kchunk = 0: K = 4096 is past the single accumulation's limit, so those jobs match

@@ -469,8 +469,29 @@ def test_graph_mode_reuses_identical_plans():
         assert strip(p3) != strip(p1)
 
 
-def test_graph_mode_off_never_reuses():
+def test_plan_cache_alternating_request_sets():
+    """cfg graph (the default): the plans of the last 32 flushes before the previous one are
+    cached too, so a loop that rotates buffer sets reuses one plan per set; a set not seen
+    within the last 33 flushes is planned afresh.  A reused plan equals the original."""
     with svp.Context(dry_run=True) as c:
+        def flush_set(k):
+            for vp in range(6):
+                submit(c, vp, MIX[vp % 4], n=50000 + 1000 * k + vp, mem=svp.MEM_DEVICE)
+            c.flush()
+            strip = [{kk: v for kk, v in op.items() if kk != "measured_ns"} for op in c.plan()]
+            return c.flush_stats()["plan_reused"], strip
+        first = {k: flush_set(k)[1] for k in range(3)}
+        for k in (0, 1, 2, 0, 2, 1):
+            reused, plan = flush_set(k)
+            assert reused == 1 and plan == first[k], k
+        for k in range(3, 37):  # 34 new sets: 0, 1, 2 fall out of the cache
+            assert flush_set(k)[0] == 0
+        assert flush_set(0)[0] == 0
+        assert flush_set(10)[0] == 1
+
+
+def test_graph_mode_off_never_reuses():
+    with svp.Context(dry_run=True, graph=False) as c:
         for _ in range(2):
             submit(c, 0, "vecadd", n=1000)
             c.flush()
