@@ -360,6 +360,17 @@ class Arm:
         self.sets = []
 
 
+def rest(ords, seconds):
+    """Let the GPUs idle before a measurement pass. The power limiter reacts to the previous
+    pass's load within a fraction of a second: a pass that follows ~0.2 s of full load ran
+    every kernel 9-30 % slower (profiles/r02/bench_order/). Each pass then starts in the
+    same (burst) state as the timed region."""
+    import torch
+    for d in set(ords):
+        torch.cuda.synchronize(d)
+    time.sleep(seconds)
+
+
 def launches_per_flush(ctx):
     """Kernels launched by the last flush (svp_flush_stats.kernel_launches: every coalesced
     launch op, plus hist256's zeroing kernel and the SGEMM tail split's slice launch and
@@ -512,6 +523,7 @@ def run_svp(args, rank, ws, local):
         pa = Arm(specs, inputs, "device", ords, streams, share=arm, profile_level=1, sgemm_impl=impl,
                  sgemm_kchunk=args.sgemm_kchunk, **f4)
         prof_steps = max(3, min(args.steps, 20))
+        rest(ords, args.rest_s)
         pa.steps((2 if args.graph else 1) * len(pa.batches) + 1)
         pa.ctx.reset_profile()
         pa.timed(prof_steps)
@@ -545,7 +557,8 @@ def run_svp(args, rank, ws, local):
     # ---------------- one stream per GPU: per-kernel roofline numbers (launches do not overlap)
     iso = Arm(specs, inputs, "device", ords, streams, share=arm, profile_level=1, interleave=False, sgemm_impl=impl,
               sgemm_kchunk=args.sgemm_kchunk)
-    iso.step()
+    rest(ords, args.rest_s)
+    iso.steps(2 * len(iso.batches) + 1)  # (graph replay: every set planned, then captured)
     iso.ctx.reset_profile()
     iso_steps = max(3, args.steps // 5)
     iso_dt, _ = iso.timed(iso_steps)
@@ -583,7 +596,8 @@ def run_svp(args, rank, ws, local):
         for alt_name, kc in variants:
             a = Arm(specs, inputs, "device", ords, streams, share=arm, profile_level=1, sgemm_impl=IMPLS[alt_name],
                     sgemm_kchunk=kc)
-            a.step()
+            rest(ords, args.rest_s)
+            a.steps(2 * len(a.batches) + 1)
             a.ctx.reset_profile()
             ks = max(3, args.steps // 5)
             adt = max_over_ranks(a.timed(ks)[0], ws)
@@ -598,14 +612,15 @@ def run_svp(args, rank, ws, local):
     # ---------------- serial baselines on the same GPUs, same buffers, same kernels
     serial, by_kernel = {}, {}
     if not args.no_serial:
-        for name, kw in (("B1_serial_sync", dict(coalesce=False, interleave=False, sync_each_job=True)),
-                         ("B2_serial_async", dict(coalesce=False, interleave=False)),
+        for name, kw in (("B1_serial_sync", dict(coalesce=False, interleave=False, sync_each_job=True, graph=False)),
+                         ("B2_serial_async", dict(coalesce=False, interleave=False, graph=False)),
                          ("B3_serial_graph", dict(coalesce=False, interleave=False, graph=True)),
-                         ("B2_profiled", dict(coalesce=False, interleave=False, profile_level=1))):
+                         ("B2_profiled", dict(coalesce=False, interleave=False, profile_level=1, graph=False))):
             # same buffer sets as the coalesced arm; B3 replays one captured graph per set
             b = Arm(specs, inputs, "device", ords, streams, share=arm, sgemm_impl=impl,
                     sgemm_kchunk=args.sgemm_kchunk, **kw)
             # B3: each set's plan, then its capture + instantiate, then replays only
+            rest(ords, args.rest_s)
             b.steps(max(3, args.warmup) + (2 * len(b.batches) if kw.get("graph") else 0))
             b.ctx.reset_profile()
             barrier(ws)
@@ -743,6 +758,8 @@ def main():
     ap.add_argument("--timed-profile-level", type=int, default=0, choices=[0, 1, 2],
                     help="profile_level of the timed context (default 0, the library default: no per-op events; "
                          "per-GPU / per-kernel numbers then come from a profiled pass over the same buffers)")
+    ap.add_argument("--rest-s", type=float, default=1.0,
+                    help="idle seconds before each measurement pass after the timed region (power-limiter reset)")
     ap.add_argument("--no-serial", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other sgemm implementation")
     ap.add_argument("--no-e2e", action="store_true")
