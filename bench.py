@@ -302,12 +302,14 @@ class Arm:
     more rotating buffer sets) pre-marshalled as JobBatches."""
 
     def __init__(self, specs, inputs, residency, ordinals, streams, nsets=1, kids=None, host_numa=False,
-                 share=None, **cfg):
+                 share=None, async_flush=False, **cfg):
         """share: another device-resident Arm whose buffer sets (and job batches) this one
         reuses -- its VPs are placed on the same GPUs by the same deterministic LPT."""
         from paper_conf_dac_jungc15_b200 import svp
         from paper_conf_dac_jungc15_b200.vpset import VPSet
         self.svp = svp
+        self.async_flush = async_flush
+        self.ticket = 0
         self.ordinals = list(ordinals)
         self.streams = streams
         self.ctx = svp.Context(num_gpus=len(self.ordinals), device_ids=self.ordinals,
@@ -326,12 +328,20 @@ class Arm:
 
     def step(self):
         self.ctx.submit_batch(self.batches[self.i % len(self.batches)])
-        self.ctx.flush()
+        if self.async_flush:
+            self.ticket = self.ctx.flush_async()
+        else:
+            self.ctx.flush()
         self.i += 1
 
     def steps(self, k):
+        """k steps; with async flushes (svp_flush_async) step i's device work overlaps step
+        i+1's submit / plan / issue, and the last step is completed (svp_flush_wait) before
+        returning, so k steps means k completed flushes."""
         for _ in range(k):
             self.step()
+        if self.async_flush and self.ticket:
+            self.ctx.flush_wait(self.ticket)
 
     def timed(self, k):
         """k steps bracketed by CUDA events on every GPU's stream (the stream the library
@@ -491,7 +501,8 @@ def run_svp(args, rank, ws, local):
     # timed at the library's default profile_level 0 (no per-op events); the per-GPU
     # Profiler numbers come from a profiled pass over the same buffers right after
     arm = Arm(specs, inputs, "device", ords, streams, nsets, profile_level=args.timed_profile_level,
-              validate_ptrs=True, sgemm_impl=impl, sgemm_kchunk=args.sgemm_kchunk, **f4)
+              validate_ptrs=True, sgemm_impl=impl, sgemm_kchunk=args.sgemm_kchunk,
+              async_flush=bool(args.async_flush), **f4)
     kids = arm.kids
     assert arm.ctx.flush_stats is not None
     arm.step()
@@ -649,7 +660,7 @@ def run_svp(args, rank, ws, local):
     e2e = None
     if not args.no_e2e:
         h = Arm(specs, inputs, "host", ords, streams, 1, arena_bytes=args.arena_gb << 30, sgemm_impl=impl,
-                sgemm_kchunk=args.sgemm_kchunk, host_numa=bool(args.host_numa),
+                sgemm_kchunk=args.sgemm_kchunk, host_numa=bool(args.host_numa), async_flush=bool(args.async_flush),
                 max_chunks=int(os.environ.get("SVP_BENCH_MAXCH", "8")), **f4)
         h.steps(2)
         hst = h.ctx.flush_stats()
@@ -707,6 +718,7 @@ def run_svp(args, rank, ws, local):
             "hbm_frac_membound": (hbm_gbs / float(peaks["hbm_gbs"])) if hbm_gbs else None,
             "elements_per_s": sum(s.n for s in all_specs) * args.steps / dt_max,
             "sgemm_impl": args.sgemm_impl, "sgemm_kchunk": args.sgemm_kchunk, "alt_sgemm_impls": alt, "hetero": args.hetero, "graph": args.graph,
+            "async_flush": args.async_flush,
             "table_mode": args.table_mode,
             "graph_replays_last_step": int(st["graph_replays"]),
             "timed_kernel_ms_per_step": {n: k["total_ns"] / prof_steps / 1e6 for n, k in main_kstats.items()
@@ -760,6 +772,8 @@ def main():
                          "per-GPU / per-kernel numbers then come from a profiled pass over the same buffers)")
     ap.add_argument("--rest-s", type=float, default=1.0,
                     help="idle seconds before each measurement pass after the timed region (power-limiter reset)")
+    ap.add_argument("--async-flush", type=int, default=1, choices=[0, 1],
+                    help="timed and e2e loops use svp_flush_async (step i's device work overlaps step i+1's host work)")
     ap.add_argument("--no-serial", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other sgemm implementation")
     ap.add_argument("--no-e2e", action="store_true")

@@ -235,6 +235,28 @@ svp_status svp_submit_batch(svp_ctx* ctx, int32_t n, const svp_job_desc* jobs, u
  * Errors: SVP_E_CUDA (sticky), SVP_E_TIMEOUT, SVP_E_NOMEM, SVP_E_STATE. */
 svp_status svp_flush(svp_ctx* ctx);
 
+/* (ABI 6) Pipelined flush: the same flush as svp_flush, but it returns once the device
+ * work is enqueued.  The flush stays pending until the NEXT flush (async or not) has been
+ * planned and issued, so the host's submit / plan / issue of flush i+1 overlaps the device
+ * work of flush i.  A launch-bound loop of small flushes then runs at the pace of the
+ * slower of host and GPU, not their sum.  At most one flush is pending: each flush
+ * completes the previous pending one (waits for it, runs the Profiler, marks its jobs done
+ * for svp_wait) after issuing its own work.
+ * *ticket_out = the flush's sequence number.  Its outputs are in place after
+ * svp_flush_wait(ctx, ticket), a later svp_flush, svp_wait on one of its jobs, or
+ * svp_finalize.  Until then, the caller must not modify that flush's input buffers or read
+ * its outputs.  The GPUs run consecutive flushes in order (each forks from the previous
+ * one's join on the caller's stream); only host work overlaps.  With profile_level >= 1 or
+ * sync_each_job there is no overlap: the previous flush completes before the next is
+ * issued, because per-op timing events are reused from flush to flush.
+ * svp_flush_stats_get reports the last COMPLETED flush.  Errors: as svp_flush (an error of
+ * the completed previous flush is returned here if the new one succeeded). */
+svp_status svp_flush_async(svp_ctx* ctx, uint64_t* ticket_out);
+/* Complete every flush up to `ticket` (a no-op for completed ones).  Returns the status of
+ * flush `ticket`.  Errors: SVP_E_INVAL (null ctx, ticket never issued), or that flush's
+ * error. */
+svp_status svp_flush_wait(svp_ctx* ctx, uint64_t ticket);
+
 /* ------------------------------------------------------------------ VP Control */
 /* Block the calling VP until job `job` (an id returned by svp_submit*) has run and its
  * outputs are in place -- the synchronous-call path of PAPER.md L276-286 / Fig 4(b):

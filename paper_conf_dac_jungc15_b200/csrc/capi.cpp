@@ -152,6 +152,8 @@ svp_status svp_init(const svp_config* cfg, svp_ctx** out) {
     SVP_TRY_END
 }
 
+static svp_status complete_pending(Ctx* c);
+
 svp_status svp_finalize(svp_ctx* h) {
     SVP_TRY_BEGIN
     if (!h) {
@@ -160,6 +162,10 @@ svp_status svp_finalize(svp_ctx* h) {
     }
     Ctx* c = reinterpret_cast<Ctx*>(h);
     stop_dispatcher(c);
+    {
+        std::lock_guard<std::mutex> flk(c->flush_mu);
+        complete_pending(c);
+    }
     if (c->exec) executor_destroy(c->exec);  // synchronizes every stream first
     for (auto& kv : c->host_blocks) host_free_near(kv.first, kv.second);
     c->host_blocks.clear();
@@ -302,21 +308,89 @@ static bool same_requests(const std::vector<Job>& a, const std::vector<Job>& b) 
     return true;
 }
 
-static svp_status do_flush(Ctx* c) {
+// The wait half of a flush (under flush_mu): its device work, the Profiler, the flush
+// statistics, the plan cache, and job completion (svp_wait).
+static svp_status complete_flush(Ctx* c, Ctx::PendingFlush& p) {
+    Flush& f = p.f;
+    svp_status st = p.st;
+    if (st == SVP_OK && c->exec && !f.ops.empty()) {
+        st = executor_complete(c->exec, &f);
+        if (st == SVP_E_CUDA || st == SVP_E_TIMEOUT) {
+            const std::string msg = executor_error(c->exec);
+            {
+                std::lock_guard<std::mutex> lk(c->done_mu);
+                c->sticky_msg = msg;
+                c->sticky.store(st);
+            }
+            set_error(msg);
+        } else if (st) {
+            set_error(executor_error(c->exec));
+        }
+    }
+    auto t2 = std::chrono::steady_clock::now();
+    f.stats.host_total_ns = std::chrono::duration<double, std::nano>(t2 - p.t0).count();
+    c->fstats = f.stats;
+    if (c->cfg.graph && c->last_ok && !c->last.jobs.empty()) {
+        // the previous flush joins the plan cache (most recent first, one entry per plan)
+        const uint64_t gen = c->last.plan_gen;
+        for (size_t k = 0; k < c->plan_cache.size();)
+            if (c->plan_cache[k].plan_gen == gen || c->plan_cache[k].plan_gen == f.plan_gen)
+                c->plan_cache.erase(c->plan_cache.begin() + (long)k);
+            else
+                ++k;
+        if (gen != f.plan_gen) {
+            c->plan_cache.insert(c->plan_cache.begin(), std::move(c->last));
+            if (c->plan_cache.size() > Ctx::kPlanCache) c->plan_cache.pop_back();
+        }
+    }
+    const uint64_t seq = f.seq;
+    c->last = std::move(f);
+    c->last_ok = st == SVP_OK;
+    {
+        std::lock_guard<std::mutex> lk(c->done_mu);
+        if (st != SVP_OK && p.upto > c->completed_upto) c->failed.emplace_back(p.upto, st);
+        if (st != SVP_OK) c->failed_flushes.emplace_back(seq, st);
+        if (p.upto > c->completed_upto) c->completed_upto = p.upto;
+    }
+    c->done_cv.notify_all();
+    return st;
+}
+
+// Complete the pending async flush, if any (under flush_mu).
+static svp_status complete_pending(Ctx* c) {
+    if (!c->pending) return SVP_OK;
+    std::unique_ptr<Ctx::PendingFlush> p = std::move(c->pending);
+    return complete_flush(c, *p);
+}
+
+// One flush of everything queued so far (serialized by flush_mu): plan (or reuse a cached
+// plan), issue every GPU's work, then -- after completing the previous async flush, whose
+// device work ran meanwhile -- either wait for it (svp_flush) or leave it pending
+// (svp_flush_async; *ticket = its sequence number).  Marks every job id below the
+// snapshot's next id as completed (or failed with the flush's status) and wakes svp_wait
+// callers when the flush completes.
+static svp_status do_flush(Ctx* c, bool async, uint64_t* ticket) {
     std::lock_guard<std::mutex> flk(c->flush_mu);
     if (c->sticky.load() != SVP_OK) {
         set_error("context is sticky-errored: " + c->sticky_message());
         return SVP_E_STATE;
     }
-    auto t0 = std::chrono::steady_clock::now();
-    Flush f;
-    uint64_t upto = 0;
+    // overlap needs per-op profiling off (its events are reused flush to flush) and no
+    // per-job synchronization; otherwise the previous flush completes first
+    const bool overlap = c->cfg.profile_level == 0 && !c->cfg.sync_each_job;
+    if (!overlap) {
+        svp_status ps = complete_pending(c);
+        if (ps == SVP_E_CUDA || ps == SVP_E_TIMEOUT) return ps;
+    }
+    auto p = std::make_unique<Ctx::PendingFlush>();
+    p->t0 = std::chrono::steady_clock::now();
+    Flush& f = p->f;
     {
         std::lock_guard<std::mutex> lk(c->qmu);
         f.jobs.swap(c->queue);
-        upto = c->next_job_id - 1;
+        p->upto = c->next_job_id - 1;
     }
-    memset(&c->fstats, 0, sizeof(c->fstats));
+    f.seq = ++c->flush_seq;
     svp_status st = SVP_OK;
     // Steady-state replay (cfg.graph, NEXT f4): the same requests as a recent flush (the
     // previous one, or one of the Ctx::kPlanCache before it -- a serving loop that alternates
@@ -338,7 +412,7 @@ static svp_status do_flush(Ctx* c) {
         f.levels = hit->levels;
         f.plan_gen = hit->plan_gen;
         f.reused = true;
-        c->fstats.plan_reused = 1;
+        f.stats.plan_reused = 1;
     } else {
         st = plan_flush(c, &f);
         f.plan_gen = ++c->plan_gen;
@@ -349,70 +423,98 @@ static svp_status do_flush(Ctx* c) {
         if (!reuse) simulate(c, &f, &makespan, &serial);
         c->last_sim_makespan = makespan;
         c->last_sim_serial = serial;
-        c->fstats.sim_makespan_ns = makespan;
-        c->fstats.sim_serial_ns = serial;
-        c->fstats.host_plan_ns = std::chrono::duration<double, std::nano>(t1 - t0).count();
+        f.stats.sim_makespan_ns = makespan;
+        f.stats.sim_serial_ns = serial;
+        f.stats.host_plan_ns = std::chrono::duration<double, std::nano>(t1 - p->t0).count();
+        f.stats.jobs = f.jobs.size();
+        f.stats.groups = f.groups.size();
+        f.stats.chunks = f.chunks.size();
+        f.stats.levels = f.levels;
         if (c->exec && !f.ops.empty()) {
-            st = executor_run(c->exec, &f);
-            if (st == SVP_E_CUDA || st == SVP_E_TIMEOUT) {
-                const std::string msg = executor_error(c->exec);
-                {
-                    std::lock_guard<std::mutex> lk(c->done_mu);
-                    c->sticky_msg = msg;
-                    c->sticky.store(st);
+            st = executor_issue(c->exec, &f);
+            if (st) {
+                executor_abandon(c->exec, &f);
+                if (st == SVP_E_CUDA || st == SVP_E_TIMEOUT) {
+                    const std::string msg = executor_error(c->exec);
+                    {
+                        std::lock_guard<std::mutex> lk(c->done_mu);
+                        c->sticky_msg = msg;
+                        c->sticky.store(st);
+                    }
+                    set_error(msg);
+                } else {
+                    set_error(executor_error(c->exec));
                 }
-                set_error(msg);
-            } else if (st) {
-                set_error(executor_error(c->exec));
             }
         }
-        auto t2 = std::chrono::steady_clock::now();
-        c->fstats.host_total_ns = std::chrono::duration<double, std::nano>(t2 - t0).count();
-        c->fstats.jobs = f.jobs.size();
-        c->fstats.groups = f.groups.size();
-        c->fstats.chunks = f.chunks.size();
-        c->fstats.levels = f.levels;
+    }
+    if (st == SVP_OK) {
+        // (after the issue half: the tables decide each chunk's kernel_launches)
         uint64_t launches = 0;
         for (auto& op : f.ops) {
             if (op.kind == SVP_OP_KERNEL) {
                 ++launches;
                 if (executor_chunk_launches(f, f.chunks[op.chunk]))
-                    c->fstats.kernel_launches += (uint64_t)f.chunks[op.chunk].kernel_launches;
+                    f.stats.kernel_launches += (uint64_t)f.chunks[op.chunk].kernel_launches;
             }
-            if (op.kind == SVP_OP_H2D) c->fstats.h2d_bytes += op.bytes;
-            if (op.kind == SVP_OP_D2H) c->fstats.d2h_bytes += op.bytes;
+            if (op.kind == SVP_OP_H2D) f.stats.h2d_bytes += op.bytes;
+            if (op.kind == SVP_OP_D2H) f.stats.d2h_bytes += op.bytes;
         }
-        c->fstats.launches = launches;
+        f.stats.launches = launches;
     }
-    if (c->cfg.graph && c->last_ok && !c->last.jobs.empty()) {
-        // the previous flush joins the plan cache (most recent first, one entry per plan)
-        const uint64_t gen = c->last.plan_gen;
-        for (size_t k = 0; k < c->plan_cache.size();)
-            if (c->plan_cache[k].plan_gen == gen || c->plan_cache[k].plan_gen == f.plan_gen)
-                c->plan_cache.erase(c->plan_cache.begin() + (long)k);
-            else
-                ++k;
-        if (gen != f.plan_gen) {
-            c->plan_cache.insert(c->plan_cache.begin(), std::move(c->last));
-            if (c->plan_cache.size() > Ctx::kPlanCache) c->plan_cache.pop_back();
-        }
+    p->st = st;
+    // the previous async flush's device work ran while this one was planned and issued
+    svp_status prev = complete_pending(c);
+    if (async && st == SVP_OK && prev == SVP_OK && c->exec && !f.ops.empty()) {
+        if (ticket) *ticket = f.seq;
+        c->pending = std::move(p);
+        return SVP_OK;
     }
-    c->last = std::move(f);
-    c->last_ok = st == SVP_OK;
-    {
-        std::lock_guard<std::mutex> lk(c->done_mu);
-        if (st != SVP_OK && upto > c->completed_upto) c->failed.emplace_back(upto, st);
-        if (upto > c->completed_upto) c->completed_upto = upto;
-    }
-    c->done_cv.notify_all();
-    return st;
+    if (ticket) *ticket = f.seq;
+    st = complete_flush(c, *p);
+    return st != SVP_OK ? st : prev;
 }
 
 svp_status svp_flush(svp_ctx* h) {
     SVP_TRY_BEGIN
     svp_status st = check_ctx(h);
     if (st) return st;
-    return do_flush(reinterpret_cast<Ctx*>(h));
+    return do_flush(reinterpret_cast<Ctx*>(h), false, nullptr);
+    SVP_TRY_END
+}
+
+svp_status svp_flush_async(svp_ctx* h, uint64_t* ticket_out) {
+    SVP_TRY_BEGIN
+    svp_status st = check_ctx(h);
+    if (st) return st;
+    if (ticket_out) *ticket_out = 0;
+    return do_flush(reinterpret_cast<Ctx*>(h), true, ticket_out);
+    SVP_TRY_END
+}
+
+svp_status svp_flush_wait(svp_ctx* h, uint64_t ticket) {
+    SVP_TRY_BEGIN
+    if (!h) {
+        set_error("null context");
+        return SVP_E_INVAL;
+    }
+    Ctx* c = reinterpret_cast<Ctx*>(h);
+    std::lock_guard<std::mutex> flk(c->flush_mu);
+    if (ticket > c->flush_seq) {
+        set_error("svp_flush_wait: unknown ticket");
+        return SVP_E_INVAL;
+    }
+    if (c->pending && c->pending->f.seq <= ticket) {
+        svp_status st = complete_pending(c);
+        if (st) return st;
+    }
+    std::lock_guard<std::mutex> lk(c->done_mu);
+    for (const auto& fs : c->failed_flushes)
+        if (fs.first == ticket) {
+            set_error("svp_flush_wait: that flush failed");
+            return fs.second;
+        }
+    return SVP_OK;
     SVP_TRY_END
 }
 
@@ -429,6 +531,11 @@ svp_status svp_wait(svp_ctx* h, uint64_t job, int32_t timeout_ms) {
             set_error("svp_wait: unknown job id");
             return SVP_E_INVAL;
         }
+    }
+    {
+        // a job of the pending async flush: complete that flush here
+        std::lock_guard<std::mutex> flk(c->flush_mu);
+        if (c->pending && job <= c->pending->upto) complete_pending(c);
     }
     std::unique_lock<std::mutex> lk(c->done_mu);
     auto done = [&] { return c->completed_upto >= job || c->sticky != SVP_OK; };
@@ -465,7 +572,7 @@ static void dispatcher_loop(Ctx* c) {
                 });
             }
         }
-        if (do_flush(c) == SVP_E_STATE && c->sticky != SVP_OK) {
+        if (do_flush(c, false, nullptr) == SVP_E_STATE && c->sticky != SVP_OK) {
             c->done_cv.notify_all();
             return;
         }

@@ -65,9 +65,21 @@ struct Dev {
     int idx = 0;
     std::vector<cudaStream_t> streams;  // [0] control, [1,S] compute, S+1 = H2D, S+2 = D2H
     cudaStream_t ext = nullptr;
+    cudaStream_t own_ext = nullptr;     // created when the caller gave no external stream
     std::vector<cudaEvent_t> dep_ev, t_ev;
     cudaEvent_t ext_ev = nullptr, tbl_ev = nullptr;
-    std::vector<cudaEvent_t> end_ev;
+    // join events per flush parity: an async flush (svp_flush_async) may still be in flight
+    // while the next one is issued
+    std::vector<cudaEvent_t> end_ev[2];
+    // what the wait half of a flush needs from its issue half (per parity)
+    struct Pending {
+        bool active = false;
+        bool prof = false;
+        std::vector<cudaEvent_t> finals;
+        std::vector<int32_t> tstart;
+    };
+    Pending pend[2];
+    bool tbl_upload_inflight = false;  // tbl_host is the source of an enqueued upload
     uint8_t* arena = nullptr;
     uint64_t arena_bytes = 0;
     int numa_node = -1;       // the GPU's NUMA node (sysfs), -1 unknown
@@ -127,6 +139,7 @@ struct Workers {
     int pending = 0;
     bool stop = false;
     Flush* f = nullptr;
+    bool complete = false;   // this round: the issue half (false) or the wait half (true)
     std::vector<std::thread> th;
     std::vector<svp_status> st;
     std::vector<double> issue;
@@ -185,11 +198,19 @@ static svp_status dev_setup(Dev& d, const svp_config& cfg, void* ext) {
     const int S = cfg.streams_per_gpu;
     d.streams.resize(S + 3);
     for (auto& s : d.streams) CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    // the stream a flush forks from and joins into: the caller's, else one of our own, so
+    // consecutive flushes (svp_flush_async keeps one in flight) always run in order
     d.ext = (cudaStream_t)ext;
+    if (!d.ext) {
+        CK(cudaStreamCreateWithFlags(&d.own_ext, cudaStreamNonBlocking));
+        d.ext = d.own_ext;
+    }
     CK(cudaEventCreateWithFlags(&d.ext_ev, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&d.tbl_ev, cudaEventDisableTiming));
-    d.end_ev.resize(S + 3);
-    for (auto& e : d.end_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    for (auto& set : d.end_ev) {
+        set.resize(S + 3);
+        for (auto& e : set) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    }
     d.join_ev.resize(S + 3);
     for (auto& e : d.join_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&d.fork_ev, cudaEventDisableTiming));
@@ -203,9 +224,14 @@ static void dev_teardown(Dev& d) {
     cudaSetDevice(d.ordinal);
     for (auto& s : d.streams) if (s) cudaStreamSynchronize(s);
     for (auto& s : d.streams) if (s) cudaStreamDestroy(s);
+    if (d.own_ext) {
+        cudaStreamSynchronize(d.own_ext);
+        cudaStreamDestroy(d.own_ext);
+    }
     for (auto e : d.dep_ev) cudaEventDestroy(e);
     for (auto e : d.t_ev) cudaEventDestroy(e);
-    for (auto e : d.end_ev) cudaEventDestroy(e);
+    for (auto& set : d.end_ev)
+        for (auto e : set) cudaEventDestroy(e);
     for (auto e : d.join_ev) cudaEventDestroy(e);
     if (d.fork_ev) cudaEventDestroy(d.fork_ev);
     for (auto& kv : d.graphs) {
@@ -266,24 +292,27 @@ Executor* executor_create(Ctx* c, svp_status* st) {
 }
 
 static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns);
+static svp_status complete_device(Executor* e, Dev& d, Flush& f);
 
 static void worker_loop(Executor* e, int g) {
     Workers& w = e->w;
     uint64_t seen = 0;
     for (;;) {
         Flush* f = nullptr;
+        bool complete = false;
         {
             std::unique_lock<std::mutex> lk(w.mu);
             w.go.wait(lk, [&] { return w.stop || w.gen != seen; });
             if (w.stop) return;
             seen = w.gen;
             f = w.f;
+            complete = w.complete;
         }
         double issue = 0;
-        const svp_status st = run_device(e, e->devs[g], *f, &issue);
+        const svp_status st = complete ? complete_device(e, e->devs[g], *f) : run_device(e, e->devs[g], *f, &issue);
         std::lock_guard<std::mutex> lk(w.mu);
         w.st[g] = st;
-        w.issue[g] = issue;
+        if (!complete) w.issue[g] = issue;
         if (--w.pending == 0) w.done.notify_one();
     }
 }
@@ -843,7 +872,15 @@ static cudaEvent_t pool_get(Dev& d, std::vector<cudaEvent_t>& pool, size_t i, bo
 
 // Captured graphs hold the addresses of the per-device scratch buffers: a reallocation
 // drops every one of them (they are re-captured on the plans' next sightings).
+// Before freeing or replacing anything the device work of a still-pending async flush may
+// use (scratch buffers, captured graphs, the table buffers): let that work finish.
+static svp_status quiesce(Dev& d) {
+    if (d.pend[0].active || d.pend[1].active) CK(cudaDeviceSynchronize());
+    return SVP_OK;
+}
+
 static svp_status drop_graphs(Dev& d) {
+    if (svp_status q = quiesce(d)) return q;
     for (auto& kv : d.graphs) {
         if (kv.second.gexec) CK(cudaGraphExecDestroy(kv.second.gexec));
         if (kv.second.tbl) CK(cudaFree(kv.second.tbl));
@@ -1035,6 +1072,8 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
     if (upload) {
         const size_t bytes = d.tbl_last.size();
         if (bytes > d.tbl_cap) {
+            if (svp_status q = quiesce(d)) return q;
+            if (d.tbl_upload_inflight) CK(cudaEventSynchronize(d.tbl_ev));
             if (d.tbl_dev) CK(cudaFree(d.tbl_dev));
             if (d.tbl_host) CK(cudaFreeHost(d.tbl_host));
             d.tbl_dev = nullptr;
@@ -1044,16 +1083,18 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
             CK(cudaHostAlloc(&d.tbl_host, cap, cudaHostAllocDefault));
             d.tbl_cap = cap;
         }
+        if (d.tbl_upload_inflight) CK(cudaEventSynchronize(d.tbl_ev));  // (async flushes)
         memcpy(d.tbl_host, d.tbl_last.data(), bytes);
         CK(cudaMemcpyAsync(d.tbl_dev, d.tbl_host, bytes, cudaMemcpyHostToDevice, d.streams[0]));
         CK(cudaEventRecord(d.tbl_ev, d.streams[0]));
+        d.tbl_upload_inflight = true;
         for (size_t s = 1; s < d.streams.size(); ++s) CK(cudaStreamWaitEvent(d.streams[s], d.tbl_ev, 0));
         d.tbl_dev_valid = true;
         ++d.table_uploads;
         {
-            std::lock_guard<std::mutex> lk(c->pmu);  // one worker thread per GPU updates fstats
-            c->fstats.table_uploads += 1;
-            c->fstats.table_bytes += bytes;
+            std::lock_guard<std::mutex> lk(c->pmu);  // one worker thread per GPU updates the stats
+            f.stats.table_uploads += 1;
+            f.stats.table_bytes += bytes;
         }
     }
     // ---- profile_level 2: busy-cycle counters for every segment launch on this GPU
@@ -1154,6 +1195,7 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
         // the entry for this plan (evicting the least recently used one past the cap); its
         // device tables are a private copy, uploaded before the capture begins
         if (d.graphs.size() >= kGraphsPerDevice) {
+            if (svp_status q = quiesce(d)) return q;
             auto lru = d.graphs.begin();
             for (auto it = d.graphs.begin(); it != d.graphs.end(); ++it)
                 if (it->second.last_use < lru->second.last_use) lru = it;
@@ -1228,7 +1270,7 @@ static svp_status run_device(Executor* e, Dev& d, Flush& f, double* issue_ns) {
         std::fill(used.begin(), used.end(), 0);
         used[0] = 1;
         std::lock_guard<std::mutex> lk(c->pmu);
-        c->fstats.graph_replays += 1;
+        f.stats.graph_replays += 1;
     }
     return finish_device(e, d, f, prof, upload, direct, used, tstart, t_issue0, issue_ns);
 }
@@ -1301,20 +1343,38 @@ static svp_status issue_ops(Executor* e, Dev& d, Flush& f, bool prof, bool captu
 static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool upload, bool direct,
                                 const std::vector<int>& used, const std::vector<int32_t>& tstart,
                                 std::chrono::steady_clock::time_point t_issue0, double* issue_ns) {
-    Ctx* c = e->c;
-    // ---- join into the external stream, then wait (watchdog)
-    std::vector<cudaEvent_t> finals;
+    // ---- join into the external stream (the wait is complete_device, possibly later)
+    auto& ev = d.end_ev[f.seq & 1];
+    Dev::Pending& pd = d.pend[f.seq & 1];
+    pd.finals.clear();
     if (direct) {  // the ops ran on the external stream itself
-        CK(cudaEventRecord(d.end_ev[0], d.ext));
-        finals.push_back(d.end_ev[0]);
+        CK(cudaEventRecord(ev[0], d.ext));
+        pd.finals.push_back(ev[0]);
     }
     for (size_t s = 0; s < d.streams.size() && !direct; ++s) {
         if (!used[s] && !(upload && s == 0)) continue;
-        CK(cudaEventRecord(d.end_ev[s], d.streams[s]));
-        finals.push_back(d.end_ev[s]);
-        if (d.ext) CK(cudaStreamWaitEvent(d.ext, d.end_ev[s], 0));
+        CK(cudaEventRecord(ev[s], d.streams[s]));
+        pd.finals.push_back(ev[s]);
+        if (d.ext) CK(cudaStreamWaitEvent(d.ext, ev[s], 0));
     }
     *issue_ns = std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t_issue0).count();
+    pd.prof = prof;
+    pd.tstart = tstart;
+    pd.active = true;
+    return SVP_OK;
+}
+
+// The wait half of a flush on one GPU: its join events (watchdog), then the measured op
+// durations and busy counters.
+static svp_status complete_device(Executor* e, Dev& d, Flush& f) {
+    Ctx* c = e->c;
+    Dev::Pending& pd = d.pend[f.seq & 1];
+    if (!pd.active) return SVP_OK;
+    pd.active = false;
+    CK(cudaSetDevice(d.ordinal));
+    const bool prof = pd.prof;
+    const std::vector<int32_t>& tstart = pd.tstart;
+    const std::vector<cudaEvent_t>& finals = pd.finals;
     if (c->cfg.flush_timeout_ms > 0) {
         auto deadline = std::chrono::steady_clock::now() + std::chrono::milliseconds(c->cfg.flush_timeout_ms);
         for (auto ev : finals) {
@@ -1363,7 +1423,7 @@ static svp_status finish_device(Executor* e, Dev& d, Flush& f, bool prof, bool u
         }
         (void)lastop;
         std::lock_guard<std::mutex> lk(c->pmu);
-        c->fstats.device_ns = std::max(c->fstats.device_ns, (double)span * 1e6);
+        f.stats.device_ns = std::max(f.stats.device_ns, (double)span * 1e6);
         DevStats& ds = c->dstats[d.idx];
         ds.last_device_ns = (double)span * 1e6;
         ds.device_ns += (double)span * 1e6;
@@ -1470,13 +1530,12 @@ static void attribute(Ctx* c, const Flush& f) {
     }
 }
 
-svp_status executor_run(Executor* e, Flush* f) {
-    Ctx* c = e->c;
+// One half of a flush on every GPU: GPU 0 on the calling thread, GPUs 1.. on their
+// workers.  Returns the first GPU's error.
+static svp_status run_half(Executor* e, Flush* f, bool complete) {
     const int G = (int)e->devs.size();
     std::vector<svp_status> st(G, SVP_OK);
     std::vector<double> issue(G, 0.0);
-    // pre-size the dependency-event pools (event creation is not thread-safe per device
-    // pool vector growth, but each worker owns its Dev)
     // the flushing thread drives GPU 0 and gets its current device back afterwards
     int caller_dev = -1;
     if (cudaGetDevice(&caller_dev) != cudaSuccess) {
@@ -1484,29 +1543,43 @@ svp_status executor_run(Executor* e, Flush* f) {
         caller_dev = -1;
     }
     if (G > 1) {
-        std::lock_guard<std::mutex> lk(e->w.mu);
-        e->w.f = f;
-        e->w.pending = G - 1;
-        e->w.gen += 1;
+        {
+            std::lock_guard<std::mutex> lk(e->w.mu);
+            e->w.f = f;
+            e->w.complete = complete;
+            e->w.pending = G - 1;
+            e->w.gen += 1;
+        }
+        e->w.go.notify_all();
     }
-    if (G > 1) e->w.go.notify_all();
-    st[0] = run_device(e, e->devs[0], *f, &issue[0]);
+    st[0] = complete ? complete_device(e, e->devs[0], *f) : run_device(e, e->devs[0], *f, &issue[0]);
     if (G > 1) {
         std::unique_lock<std::mutex> lk(e->w.mu);
         e->w.done.wait(lk, [&] { return e->w.pending == 0; });
         for (int g = 1; g < G; ++g) {
             st[g] = e->w.st[g];
-            issue[g] = e->w.issue[g];
+            if (!complete) issue[g] = e->w.issue[g];
         }
     }
     if (caller_dev >= 0) cudaSetDevice(caller_dev);
-    c->fstats.host_issue_ns = *std::max_element(issue.begin(), issue.end());
+    if (!complete) f->stats.host_issue_ns = *std::max_element(issue.begin(), issue.end());
     for (int g = 0; g < G; ++g) {
         if (st[g] != SVP_OK) {
             e->err = "GPU " + std::to_string(g) + ": " + e->devs[g].err;
             return st[g];
         }
     }
+    return SVP_OK;
+}
+
+// Issue half: every GPU's ops enqueued and joined into its external stream (no waiting).
+svp_status executor_issue(Executor* e, Flush* f) { return run_half(e, f, false); }
+
+// Wait half: every GPU's join events, measured durations, then the Profiler.
+svp_status executor_complete(Executor* e, Flush* f) {
+    Ctx* c = e->c;
+    svp_status st = run_half(e, f, true);
+    if (st) return st;
     if (c->cfg.profile_level >= 1) attribute(c, *f);
     else {
         std::lock_guard<std::mutex> lk(c->pmu);
@@ -1519,6 +1592,19 @@ svp_status executor_run(Executor* e, Flush* f) {
             if (o.kind == SVP_OP_KERNEL && chunk_needs_launch(*f, f->chunks[o.chunk])) c->prof_launches += 1;
     }
     return SVP_OK;
+}
+
+// After a failed issue half: wait for whatever the GPUs that did issue enqueued (no
+// profiling), so nothing of this flush is left running when the error is returned.
+void executor_abandon(Executor* e, Flush* f) {
+    for (auto& d : e->devs) {
+        Dev::Pending& pd = d.pend[f->seq & 1];
+        if (!pd.active) continue;
+        pd.active = false;
+        cudaSetDevice(d.ordinal);
+        for (auto ev : pd.finals) cudaEventSynchronize(ev);
+        cudaGetLastError();
+    }
 }
 
 }  // namespace svp

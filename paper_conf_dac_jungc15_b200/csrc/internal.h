@@ -11,8 +11,10 @@
 #include <stdint.h>
 
 #include <atomic>
+#include <chrono>
 #include <condition_variable>
 #include <functional>
+#include <memory>
 #include <mutex>
 #include <string>
 #include <thread>
@@ -173,6 +175,8 @@ struct Flush {
     // requests equal the previous flush's, so plan, chunks and tables were copied from it
     uint64_t plan_gen = 0;
     bool reused = false;
+    uint64_t seq = 0;             // flush sequence number (svp_flush_async tickets)
+    svp_flush_stats stats{};      // this flush's statistics (svp_flush_stats_get: the last completed)
 };
 
 // ------------------------------------------------------------------ per-VP profile
@@ -279,6 +283,18 @@ struct Ctx {
     static constexpr size_t kPlanCache = 32;
     std::vector<Flush> plan_cache;
     Flush last;
+    // svp_flush_async: the flush whose device work may still run (its wait half pending),
+    // under flush_mu.  Completed when the next flush has been issued, by svp_flush_wait,
+    // by svp_wait on one of its jobs, or at svp_finalize.
+    struct PendingFlush {
+        Flush f;
+        uint64_t upto = 0;  // last job id of the flush
+        svp_status st = SVP_OK;
+        std::chrono::steady_clock::time_point t0;
+    };
+    std::unique_ptr<PendingFlush> pending;
+    uint64_t flush_seq = 0;       // last issued flush
+    std::vector<std::pair<uint64_t, int32_t>> failed_flushes;  // (seq, status), ascending
     bool last_ok = false;            // the last flush completed with SVP_OK
     uint64_t plan_gen = 0;           // bumped for every freshly planned flush
     double last_sim_makespan = 0, last_sim_serial = 0;
@@ -312,7 +328,13 @@ void simulate(Ctx* c, Flush* f, double* makespan, double* serial);
 // executor.cpp
 Executor* executor_create(Ctx* c, svp_status* st);
 void executor_destroy(Executor* e);
-svp_status executor_run(Executor* e, Flush* f);      // tables, staging, issue, wait, profile
+// A flush in two halves (svp_flush_async overlaps the next flush's planning and issue with
+// the device work between them): issue = tables, staging, enqueue, join into the external
+// streams; complete = wait (watchdog), measured durations, Profiler.  abandon = after a
+// failed issue, wait quietly for what was enqueued.
+svp_status executor_issue(Executor* e, Flush* f);
+svp_status executor_complete(Executor* e, Flush* f);
+void executor_abandon(Executor* e, Flush* f);
 std::string executor_error(Executor* e);
 
 // numa.cpp: NUMA placement near a GPU (sysfs of its PCI function; -1 / false = unknown)

@@ -37,7 +37,8 @@ EXPORTS = ("svp_config_default", "svp_init", "svp_finalize", "svp_last_error", "
            "svp_flush_stats_get", "svp_plan_size", "svp_plan_get", "svp_wait", "svp_start_dispatcher",
            "svp_stop_dispatcher", "svp_ipc_serve", "svp_ipc_server_stats", "svp_ipc_shutdown", "svp_ipc_connect",
            "svp_ipc_disconnect", "svp_ipc_alloc", "svp_ipc_submit", "svp_ipc_wait", "svp_kernel_lookup",
-           "svp_plan_op_detail", "svp_device_stats_get", "svp_host_alloc", "svp_host_free")
+           "svp_plan_op_detail", "svp_device_stats_get", "svp_host_alloc", "svp_host_free",
+           "svp_flush_async", "svp_flush_wait")
 
 
 class svp_config(C.Structure):
@@ -160,6 +161,8 @@ def load(build_if_stale: bool = True):
         L.svp_device_stats_get.argtypes = [vp, C.c_int32, P(svp_device_stats)]
         L.svp_host_alloc.argtypes = [vp, C.c_int32, C.c_uint64, P(C.c_void_p), P(C.c_int32)]
         L.svp_host_free.argtypes = [vp, C.c_void_p]
+        L.svp_flush_async.argtypes = [vp, P(C.c_uint64)]
+        L.svp_flush_wait.argtypes = [vp, C.c_uint64]
         L.svp_plan_op_detail.argtypes = [vp, C.c_int32, P(C.c_uint64), P(C.c_uint64), P(C.c_int32), C.c_int32,
                                          P(C.c_int32), P(C.c_double)]
         for name in EXPORTS:
@@ -331,6 +334,16 @@ class Context:
 
     def flush(self):
         _check(self._L.svp_flush(self._h))
+
+    def flush_async(self) -> int:
+        """svp_flush_async: enqueue the flush and return its ticket; it completes when the
+        next flush has been issued, or at flush_wait(ticket)."""
+        t = C.c_uint64()
+        _check(self._L.svp_flush_async(self._h, C.byref(t)))
+        return t.value
+
+    def flush_wait(self, ticket: int):
+        _check(self._L.svp_flush_wait(self._h, ticket))
 
     def wait(self, job: int, timeout_ms: int = 0):
         """VP Control: block until `job` has run (svp_wait).  Releases the GIL."""

@@ -264,3 +264,24 @@ def test_host_alloc_rejects_dry_run_and_bad_args():
         with pytest.raises(svp.SvpError) as e:
             c.host_free(0x1000)
         assert e.value.status == svp.SVP_E_INVAL
+
+
+def test_flush_async_tickets_dry_run():
+    """svp_flush_async / svp_flush_wait bookkeeping without a GPU: tickets count flushes,
+    a dry-run flush completes at once, svp_wait sees its jobs done, unknown tickets are
+    rejected."""
+    with svp.Context(dry_run=True) as c:
+        k = c.register_kernel("vecadd")
+        buf = [(0x10000, 4096, svp.DIR_IN, svp.MEM_DEVICE), (0x20000, 4096, svp.DIR_IN, svp.MEM_DEVICE),
+               (0x30000, 4096, svp.DIR_OUT, svp.MEM_DEVICE)]
+        tickets = []
+        for r in range(3):
+            ids = c.submit_batch([(0, k, svp.args_vecadd(1024), buf)])
+            tickets.append(c.flush_async())
+            c.wait(ids[0])
+        assert tickets == [tickets[0], tickets[0] + 1, tickets[0] + 2]
+        c.flush_wait(tickets[-1])
+        c.flush()  # a synchronous flush takes the next ticket
+        with pytest.raises(svp.SvpError) as e:
+            c.flush_wait(tickets[-1] + 10)
+        assert e.value.status == svp.SVP_E_INVAL
