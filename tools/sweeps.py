@@ -19,8 +19,9 @@ S5 (Table 1): N VPs each running the paper's progra
     serial per-VP launches; DGEMM TFLOP/s; the same program with steady-state graph replay.
 S6 (NEXT f4, launch-bound mixes): N VPs with small vecadd / SAXPY / Black-Scholes jobs
     (16Ki-64Ki elements); wall time of submit + flush per round for the default path,
-    hetero (one mixed launch), graph (plan reuse + CUDA-graph replay), both, and the
-    serial baselines B2 / B3 (B2 as a graph).
+    hetero (one mixed launch), graph (plan reuse + CUDA-graph replay), graph with pipelined
+    flushes (svp_flush_async, rounds back to back), both, and the serial baselines B2 / B3
+    (B2 as a graph).
 Times are CUDA-event device times around whole flushes (median of reps).
 """
 import argparse
@@ -62,6 +63,7 @@ def flush_time(ctx, jobs, reps=5, warm=2):
 def ctx_for(**kw):
     # SVP_SWEEP_VALIDATE: validate_ptrs level of every context (A/B of the range cache)
     kw.setdefault("validate_ptrs", int(os.environ.get("SVP_SWEEP_VALIDATE", "1")))
+    kw.setdefault("graph", False)  # the paper's experiments: plain flushes unless a row asks for replay
     return svp.Context(num_gpus=1, external_streams=[torch.cuda.current_stream().cuda_stream], **kw)
 
 
@@ -282,6 +284,24 @@ def wall_time(ctx, jobs, reps=50, warm=5):
     return statistics.median(ts)
 
 
+def pipelined_time(ctx, jobs, reps=200, warm=10):
+    """Host wall time per round of submit + svp_flush_async, rounds back to back (each
+    round's device work overlaps the next round's host work); the last is waited for."""
+    import time
+    jobs = svp.JobBatch(jobs)
+    for _ in range(warm):
+        ctx.submit_batch(jobs)
+        t = ctx.flush_async()
+    ctx.flush_wait(t)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        ctx.submit_batch(jobs)
+        t = ctx.flush_async()
+    ctx.flush_wait(t)
+    return (time.perf_counter() - t0) / reps
+
+
 def s6_f4(quick):
     kinds = ("vecadd", "saxpy", "blackscholes")
     rows = []
@@ -299,6 +319,8 @@ def s6_f4(quick):
             vs = VPSet(c, specs, inputs, "device")
             t = wall_time(c, vs.job_list())
             st = c.flush_stats()
+            if name == "graph":  # the same rounds pipelined (svp_flush_async)
+                row["graph_async_us"] = pipelined_time(c, vs.job_list()) * 1e6
             row[name + "_us"] = t * 1e6
             row[name + "_launches"] = int(st["launches"])
             row[name + "_host_plan_us"] = st["host_plan_ns"] / 1e3
@@ -306,6 +328,8 @@ def s6_f4(quick):
             c.close()
             del vs
         row["speedup_graph_vs_default"] = row["default_us"] / row["graph_us"]
+        row["speedup_graph_async_vs_default"] = row["default_us"] / row["graph_async_us"]
+        row["speedup_graph_async_vs_B2"] = row["B2_serial_async_us"] / row["graph_async_us"]
         row["speedup_hetero_graph_vs_default"] = row["default_us"] / row["hetero_graph_us"]
         row["speedup_default_vs_B2"] = row["B2_serial_async_us"] / row["default_us"]
         rows.append(row)
