@@ -406,12 +406,17 @@ __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_
 __device__ __forceinline__ int tc_chunks(const GemmDesc& g, int KB, int kchunk) {
     return (kchunk > 0 && g.beta == 0.f && KB > kchunk) ? (KB + kchunk - 1) / kchunk : 1;
 }
+// flag in the kernel's kchunk argument above the 16-bit block count: the TMA epilogue frees the
+// accumulator right after its last tcgen05.ld instead of after its last slab write
+constexpr int kEpiEarlyRelease = 1 << 16;
 
 template <int SPLIT, int CG, int NH>
 __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
     k_sgemm_tc(const GemmDesc* __restrict__ descs, int n, const uint8_t* __restrict__ maps, uint32_t total,
-               int kchunk, const uint8_t* __restrict__ cmaps) {
+               int kchunk_flags, const uint8_t* __restrict__ cmaps) {
     using namespace tc;
+    const int kchunk = kchunk_flags & 0xFFFF;
+    const bool early_release = (kchunk_flags & kEpiEarlyRelease) != 0;
     using C = Cfg<SPLIT, CG, NH>;
     constexpr int TN = BN * NH;  // tile width in N per CTA pair (or CTA)
     constexpr int ST = C::kStages, SB = C::kStageBytes, TB = C::kTileB, TB16 = C::kTileB16;
@@ -755,6 +760,18 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
             // chunk those slabs are read back and their NaN outputs recomputed exactly.
             constexpr int SW = 8, NV = SW / 4;
             if (first) nan_slabs = 0;
+            // the accumulator is free for the next (tile, chunk) unit's MMAs once this warp's
+            // last tcgen05.ld returned (early release), else after its last write
+            bool released = false;
+            auto release = [&]() {
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) {
+                    if constexpr (CG == 2) mbar_arrive_cluster(acc_empty_leader + (uint32_t)a * 8u);
+                    else mbar_arrive(&acc_empty[a]);
+                }
+                released = true;
+            };
             if (tma_epi) {
                 // two 32-row x 16-column half-slabs (64-B rows, 64-B swizzle) per epilogue warp,
                 // alternating: the TMA op of one is in flight while the other is refilled
@@ -771,6 +788,7 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     for (int sl = 0; sl < 2; ++sl) {
                         uint32_t r[SW];
                         tmem_ld8(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * BN + c0 + sl * SW), r);
+                        if (early_release && c0 == BN - 16 && sl == 1) release();  // TMEM fully read
 #pragma unroll
                         for (int jj = 0; jj < NV; ++jj) {
                             const int j = 4 * jj;
@@ -863,12 +881,7 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
                     }
                 }
             }
-            tc_fence_before();
-            __syncwarp();
-            if (lane == 0) {
-                if constexpr (CG == 2) mbar_arrive_cluster(acc_empty_leader + (uint32_t)a * 8u);
-                else mbar_arrive(&acc_empty[a]);
-            }
+            if (!released) release();
           }
         }
     }
@@ -889,6 +902,17 @@ __global__ void __launch_bounds__(tc::Cfg<SPLIT, CG, NH>::kThreads, 1)
 }
 
 static std::atomic<bool> g_attr_set[20][64] = {};  // per kernel variant and device
+
+// SVP_TC_EARLY=0: the TMA epilogue frees the accumulator only after its last write (A/B switch;
+// early release measured +0.9 % one-stream SGEMM, profiles/r02/epi_ab/)
+static bool sgemm_tc_early_release() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("SVP_TC_EARLY");
+        v = (e && atoi(e) == 0) ? 0 : 1;
+    }
+    return v == 1;
+}
 
 template <int SPLIT, int CG, int NH = 1>
 static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uint32_t total, int clusters,
@@ -920,7 +944,8 @@ static cudaError_t launch_tc(const GemmDesc* descs, int n, const void* maps, uin
     }
     // the plain-TF32 "sgemm_tf32" (own 2e-3 tolerance) accumulates the whole K in one chunk
     const int kchunk = (SPLIT == 1 || !cmaps) ? 0 : kchunk_k / tc::BK;
-    return cudaLaunchKernelEx(&lc, kern, descs, n, reinterpret_cast<const uint8_t*>(maps), total, kchunk,
+    const int flags = sgemm_tc_early_release() ? kEpiEarlyRelease : 0;
+    return cudaLaunchKernelEx(&lc, kern, descs, n, reinterpret_cast<const uint8_t*>(maps), total, kchunk | flags,
                               reinterpret_cast<const uint8_t*>(cmaps));
 }
 
