@@ -495,7 +495,8 @@ def run_svp(args, rank, ws, local):
     inputs = W.make_inputs_many(specs)
     t_gen = time.perf_counter() - t_gen
     nsets = n_buffer_sets(all_specs)
-    f4 = dict(hetero=bool(args.hetero), graph=bool(args.graph), table_mode=args.table_mode)
+    f4 = dict(hetero=bool(args.hetero), graph=bool(args.graph), table_mode=args.table_mode,
+              streams_per_gpu=args.streams)
 
     # ---------------- device-resident run (value)
     # timed at the library's default profile_level 0 (no per-op events); the per-GPU
@@ -774,6 +775,7 @@ def main():
                     help="idle seconds before each measurement pass after the timed region (power-limiter reset)")
     ap.add_argument("--async-flush", type=int, default=1, choices=[0, 1],
                     help="timed and e2e loops use svp_flush_async (step i's device work overlaps step i+1's host work)")
+    ap.add_argument("--streams", type=int, default=4, help="compute streams per GPU (svp_config.streams_per_gpu)")
     ap.add_argument("--no-serial", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other sgemm implementation")
     ap.add_argument("--no-e2e", action="store_true")
