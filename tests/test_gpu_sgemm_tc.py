@@ -92,10 +92,11 @@ def test_split_wide_dynamic_range(impl):
 
 @pytest.mark.parametrize("env", [{"SVP_TC_CTA_PAIR": "0"}, {"SVP_TC_TMEM_A": "1"},
                                  {"SVP_TC_CTA_PAIR": "0", "SVP_TC_TMEM_A": "1"}, {"SVP_TC_WIDE": "0"},
-                                 {"SVP_TC_WIDE": "2"}])
+                                 {"SVP_TC_WIDE": "2"}, {"SVP_TC_EARLY": "0"}])
 def test_kernel_variants_in_subprocess(env):
     """The non-default tcgen05 variants (single-CTA kernels; A-side bf16 operands in TMEM;
-    256 x 512 pair tiles never / always instead of per launch)
+    256 x 512 pair tiles never / always instead of per launch; the accumulator released after
+    the epilogue's last write instead of its last tcgen05.ld)
     are chosen once per process from the environment: run this file's fp32 parity tests
     in a child process with the switch set."""
     import os
