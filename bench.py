@@ -131,7 +131,7 @@ class Clocks:
     # mostly shows the idle time before a ~0.1-s timed region
     Q = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw.instant,clocks_event_reasons.active,"
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap,enforced.power.limit")
 
     def __init__(self, device_indices):
         self.p = None
@@ -190,7 +190,11 @@ class Clocks:
                 continue
             try:
                 pw = float(parts[4]) if parts[4] not in ("", "[N/A]") else float("nan")
-                rows.append((self._ts(parts[0]), float(parts[2]), float(parts[3]), parts[6:10], pw))
+                try:
+                    lim = float(parts[10]) if len(parts) > 10 else float("nan")
+                except ValueError:
+                    lim = float("nan")
+                rows.append((self._ts(parts[0]), float(parts[2]), float(parts[3]), parts[6:10], pw, lim))
             except ValueError:
                 continue
         os.unlink(self.f.name)
@@ -208,10 +212,12 @@ class Clocks:
                 if val.lower().startswith("active"):
                     reasons.add(nm)
         pws = [r[4] for r in sel if r[4] == r[4]]
+        lims = [r[5] for r in sel if r[5] == r[5]]
         return {"sm_mhz": statistics.median(r[1] for r in sel), "sm_max_mhz": max(r[2] for r in sel),
                 "samples": len(sel), "in_window": len(inside), "window_ms": (self.t1 - self.t0) * 1e3,
                 "reasons": sorted(reasons), "power_w": statistics.median(pws) if pws else None,
-                "power_field": "power.draw.instant (median of the samples)"}
+                "power_field": "power.draw.instant (median of the samples)",
+                "power_limit_w": statistics.median(lims) if lims else None}
 
 
 def measured_peaks():
