@@ -12,7 +12,14 @@
 //    the paper's program spread over the SMs instead of leaving 80 % of them idle;
 //  * A staged transposed in shared memory (k-major rows padded to 65 doubles: the 16
 //    k-rows of a warp's stores fall in distinct banks), B staged as is; two smem buffers
-//    with the next k block's global loads issued before the current block's DFMAs.
+//    with the next k block's global loads issued before the current block's DFMAs;
+//  * split K (session 3): when even the 32x32 tiles leave most CTA slots empty (the Table 1
+//    program with 1-2 VPs: 100 tiles per VP), each tile runs on a cluster of S = 2 or 4
+//    CTAs, CTA r accumulating k blocks [r*ceil(KB/S), ...); ranks 1..S-1 leave their 4x4
+//    partials in shared memory and rank 0 adds them through DSMEM in rank order (a fixed
+//    order: the result does not depend on timing) before the epilogue.
+#include <stdlib.h>
+
 #include "../launch.h"
 #include "common.cuh"
 
@@ -30,16 +37,22 @@ __device__ __forceinline__ int find_dgemm(const DgemmDesc* __restrict__ d, int n
 }
 
 // TM x TN output tile, (TM/4) x (TN/4) threads with 4x4 accumulators each, DK-deep k blocks
-template <int TM, int TN, int DK>
+template <int TM, int TN, int DK, int S = 1>
 __global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* __restrict__ descs, int n,
                                                                uint32_t total) {
     constexpr int NT = (TM / 4) * (TN / 4);
+    __shared__ double red[S > 1 ? 16 * NT : 1];  // split K: this CTA's partials, [i*4+j][tid]
+    uint32_t rank = 0;
+    if constexpr (S > 1) asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+    auto cluster_sync = [] {
+        asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    };
     constexpr int LA = TM * DK / NT, LB = DK * TN / NT;  // elements per thread per k block
     constexpr int kApad = TM + 1;
     __shared__ double As[2][DK][kApad];
     __shared__ __align__(16) double Bs[2][DK][TN];
     const int tid = threadIdx.x, tx = tid % (TN / 4), ty = tid / (TN / 4);
-    for (uint32_t t = blockIdx.x; t < total; t += gridDim.x) {
+    for (uint32_t t = blockIdx.x / S; t < total; t += gridDim.x / S) {
         const DgemmDesc& g = descs[find_dgemm(descs, n, t)];
         const uint32_t lt = t - g.tile_begin;
         const int m0 = (lt / g.tiles_n) * TM, n0 = (lt % g.tiles_n) * TN;
@@ -81,14 +94,16 @@ __global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* 
                 Bs[buf][idx / TN][idx % TN] = rb[i];
             }
         };
-        const int KB = (K + DK - 1) / DK;
-        if (KB > 0) {
-            load(0);
+        // this CTA's k blocks [kb0, KB) (split K: rank r of the cluster takes a contiguous share)
+        const int KBall = (K + DK - 1) / DK, per = (KBall + S - 1) / S;
+        const int kb0 = min(KBall, (int)rank * per), KB = min(KBall, kb0 + per);
+        if (KB > kb0) {
+            load(kb0 * DK);
             store(0);
         }
         __syncthreads();
-        for (int kb = 0; kb < KB; ++kb) {
-            const int cur = kb & 1;
+        for (int kb = kb0; kb < KB; ++kb) {
+            const int cur = (kb - kb0) & 1;
             if (kb + 1 < KB) load((kb + 1) * DK);
 #pragma unroll
             for (int k = 0; k < DK; ++k) {
@@ -108,6 +123,37 @@ __global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* 
             }
             if (kb + 1 < KB) store(cur ^ 1);
             __syncthreads();
+        }
+        if constexpr (S > 1) {
+            // ranks 1..S-1 publish their partials; rank 0 adds them in rank order
+            if (rank != 0) {
+#pragma unroll
+                for (int i = 0; i < 4; ++i)
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) red[(i * 4 + j) * NT + tid] = acc[i][j];
+            }
+            cluster_sync();
+            if (rank == 0) {
+#pragma unroll 1
+                for (uint32_t r = 1; r < (uint32_t)S; ++r) {
+                    uint32_t base;
+                    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;"
+                                 : "=r"(base)
+                                 : "r"((uint32_t)__cvta_generic_to_shared(red)), "r"(r));
+#pragma unroll
+                    for (int i = 0; i < 4; ++i)
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) {
+                            double v;
+                            asm volatile("ld.shared::cluster.f64 %0, [%1];"
+                                         : "=d"(v)
+                                         : "r"(base + (uint32_t)(((i * 4 + j) * NT + tid) * 8)));
+                            acc[i][j] += v;
+                        }
+                }
+            }
+            cluster_sync();  // the peers' partials are read before they are overwritten
+            if (rank != 0) continue;
         }
         // epilogue
 #pragma unroll
@@ -141,6 +187,34 @@ cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total, int grid
         cudaGetLastError();
         return sms * per;
     }();
+    // split K when S times the tiles still fit in one wave of the deep small variant
+    static const bool split_on = !(getenv("SVP_DGEMM_SPLIT") && atoi(getenv("SVP_DGEMM_SPLIT")) == 0);
+    static const int split_cap = [] {
+        int dev = 0, sms = 0, per = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_dgemm<kDgemmSmall, kDgemmSmall, kDgemmSmallDeepBK, 4>,
+                                                      (kDgemmSmall / 4) * (kDgemmSmall / 4), 0);
+        cudaGetLastError();
+        return sms * per;
+    }();
+    const int S = !small || !split_on ? 1 : total * 4 <= (uint32_t)split_cap ? 4 : total * 2 <= (uint32_t)split_cap ? 2 : 1;
+    if (S > 1) {
+        cudaLaunchConfig_t lc = {};
+        cudaLaunchAttribute attr[1];
+        lc.gridDim = dim3(total * S);
+        lc.blockDim = dim3((kDgemmSmall / 4) * (kDgemmSmall / 4));
+        lc.stream = s;
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = S;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        lc.attrs = attr;
+        lc.numAttrs = 1;
+        if (S == 4)
+            return cudaLaunchKernelEx(&lc, k_dgemm<kDgemmSmall, kDgemmSmall, kDgemmSmallDeepBK, 4>, descs, n, total);
+        return cudaLaunchKernelEx(&lc, k_dgemm<kDgemmSmall, kDgemmSmall, kDgemmSmallDeepBK, 2>, descs, n, total);
+    }
     if (small && total <= (uint32_t)deep_cap)
         k_dgemm<kDgemmSmall, kDgemmSmall, kDgemmSmallDeepBK>
             <<<grid, (kDgemmSmall / 4) * (kDgemmSmall / 4), 0, s>>>(descs, n, total);
