@@ -14,7 +14,7 @@
 //    k-rows of a warp's stores fall in distinct banks), B staged as is; two smem buffers
 //    with the next k block's global loads issued before the current block's DFMAs;
 //  * split K (session 3): when even the 32x32 tiles leave most CTA slots empty (the Table 1
-//    program with 1-2 VPs: 100 tiles per VP), each tile runs on a cluster of S = 2 or 4
+//    program with 1-4 VPs: 100 tiles per VP), each tile runs on a cluster of S = 2 or 4
 //    CTAs, CTA r accumulating k blocks [r*ceil(KB/S), ...); ranks 1..S-1 leave their 4x4
 //    partials in shared memory and rank 0 adds them through DSMEM in rank order (a fixed
 //    order: the result does not depend on timing) before the epilogue.
@@ -38,10 +38,9 @@ __device__ __forceinline__ int find_dgemm(const DgemmDesc* __restrict__ d, int n
 
 // TM x TN output tile, (TM/4) x (TN/4) threads with 4x4 accumulators each, DK-deep k blocks
 template <int TM, int TN, int DK, int S = 1>
-__global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* __restrict__ descs, int n,
+__global__ void __launch_bounds__((TM / 4) * (TN / 4), S > 1 ? 6 : 0) k_dgemm(const DgemmDesc* __restrict__ descs, int n,
                                                                uint32_t total) {
     constexpr int NT = (TM / 4) * (TN / 4);
-    __shared__ double red[S > 1 ? 16 * NT : 1];  // split K: this CTA's partials, [i*4+j][tid]
     uint32_t rank = 0;
     if constexpr (S > 1) asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
     auto cluster_sync = [] {
@@ -51,6 +50,9 @@ __global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* 
     constexpr int kApad = TM + 1;
     __shared__ double As[2][DK][kApad];
     __shared__ __align__(16) double Bs[2][DK][TN];
+    // split K: this CTA's partials, [i*4+j][tid], in the A staging buffers (free after the k loop)
+    double* red = &As[0][0][0];
+    static_assert(S == 1 || 2 * DK * kApad >= 16 * NT, "partials fit in the A staging buffers");
     const int tid = threadIdx.x, tx = tid % (TN / 4), ty = tid / (TN / 4);
     for (uint32_t t = blockIdx.x / S; t < total; t += gridDim.x / S) {
         const DgemmDesc& g = descs[find_dgemm(descs, n, t)];
@@ -96,14 +98,14 @@ __global__ void __launch_bounds__((TM / 4) * (TN / 4)) k_dgemm(const DgemmDesc* 
         };
         // this CTA's k blocks [kb0, KB) (split K: rank r of the cluster takes a contiguous share)
         const int KBall = (K + DK - 1) / DK, per = (KBall + S - 1) / S;
-        const int kb0 = min(KBall, (int)rank * per), KB = min(KBall, kb0 + per);
+        const int kb0 = S == 1 ? 0 : min(KBall, (int)rank * per), KB = S == 1 ? KBall : min(KBall, kb0 + per);
         if (KB > kb0) {
             load(kb0 * DK);
             store(0);
         }
         __syncthreads();
         for (int kb = kb0; kb < KB; ++kb) {
-            const int cur = (kb - kb0) & 1;
+            const int cur = S == 1 ? (kb & 1) : ((kb - kb0) & 1);
             if (kb + 1 < KB) load((kb + 1) * DK);
 #pragma unroll
             for (int k = 0; k < DK; ++k) {
@@ -198,7 +200,12 @@ cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total, int grid
         cudaGetLastError();
         return sms * per;
     }();
-    const int S = !small || !split_on ? 1 : total * 4 <= (uint32_t)split_cap ? 4 : total * 2 <= (uint32_t)split_cap ? 2 : 1;
+    // S = 4 only while the split launch would use at most half the CTA slots (S5: 2 VPs, 200
+    // tiles, ran 5.5 ms at S = 2 and 7.3 ms at S = 4), S = 2 while it fits in one wave
+    const int S = !small || !split_on                         ? 1
+                  : total * 4 <= (uint32_t)split_cap / 2 ? 4
+                  : total * 2 <= (uint32_t)split_cap     ? 2
+                                                         : 1;
     if (S > 1) {
         cudaLaunchConfig_t lc = {};
         cudaLaunchAttribute attr[1];
