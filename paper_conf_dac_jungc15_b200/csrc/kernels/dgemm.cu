@@ -20,6 +20,8 @@
 //    order: the result does not depend on timing) before the epilogue.
 #include <stdlib.h>
 
+#include <algorithm>
+
 #include "../launch.h"
 #include "common.cuh"
 
@@ -176,6 +178,164 @@ __global__ void __launch_bounds__((TM / 4) * (TN / 4), S > 1 ? 6 : 0) k_dgemm(co
     }
 }
 
+// Small tiles on the FP64 tensor cores (session 3): the SIMT 32x32 kernel is bound by shared-
+// memory loads (ncu: 0.5 LDS per DFMA, 40 % bank conflicts, FP64 pipe 25 % busy).  Here a
+// 32x32 tile is 4 warps of 16x16, each 2x2 mma.sync.m8n8k4.f64 tiles (DMMA): per 4 k a thread
+// loads 4 doubles for 32 FMAs.  A is staged m-major and B k-major with rows of TT + 4 / DK + 4
+// doubles, so the fragment loads (lane -> (lane >> 2, lane & 3)) and the staging stores are
+// both conflict-free.  The same split-K clusters as k_dgemm (rank-order DSMEM reduction).
+constexpr int kMmaT = 32, kMmaDK = 32, kMmaThreads = 128;
+
+__device__ __forceinline__ void dmma(double (&d)[2], double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                 : "+d"(d[0]), "+d"(d[1])
+                 : "d"(a), "d"(b));
+}
+
+template <int S>
+__global__ void __launch_bounds__(kMmaThreads, S > 1 ? 6 : 0) k_dgemm_mma(const DgemmDesc* __restrict__ descs, int n,
+                                                                        uint32_t total) {
+    constexpr int T = kMmaT, DK = kMmaDK, NT = kMmaThreads;
+    constexpr int PA = DK + 4, PB = T + 4;   // row strides (doubles): 4 mod 16 -> conflict-free
+    constexpr int LA = T * DK / NT, LB = DK * T / NT;
+    __shared__ __align__(16) double As[2][T][PA];   // A tile, m-major (k fastest)
+    __shared__ __align__(16) double Bs[2][DK][PB];  // B tile, k-major (n fastest)
+    double* red = &As[0][0][0];                     // split K: partials [e][tid] after the k loop
+    static_assert(S == 1 || 2 * T * PA >= 8 * NT, "partials fit in the A staging buffers");
+    uint32_t rank = 0;
+    if constexpr (S > 1) asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+    auto cluster_sync = [] {
+        asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    };
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int wm = (warp >> 1) * 16, wn = (warp & 1) * 16;
+    const int fr = lane >> 2, fk = lane & 3;  // fragment row / k (A), col / k (B)
+    for (uint32_t t = blockIdx.x / S; t < total; t += gridDim.x / S) {
+        const DgemmDesc& g = descs[find_dgemm(descs, n, t)];
+        const uint32_t lt = t - g.tile_begin;
+        const int m0 = (lt / g.tiles_n) * T, n0 = (lt % g.tiles_n) * T;
+        const int M = g.M, N = g.N, K = g.K;
+        const double* __restrict__ A = g.A;
+        const double* __restrict__ B = g.B;
+        double acc[2][2][2];
+#pragma unroll
+        for (int i = 0; i < 2; ++i)
+#pragma unroll
+            for (int j = 0; j < 2; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+        double ra[LA], rb[LB];
+        auto load = [&](int k0) {
+#pragma unroll
+            for (int i = 0; i < LA; ++i) {
+                const int idx = tid + i * NT, r = idx / DK, c = idx % DK;
+                const int gm = m0 + r, gk = k0 + c;
+                ra[i] = (gm < M && gk < K) ? A[(size_t)gm * K + gk] : 0.0;
+            }
+#pragma unroll
+            for (int i = 0; i < LB; ++i) {
+                const int idx = tid + i * NT, rr = idx / T, cc = idx % T;
+                const int bk = k0 + rr, bn = n0 + cc;
+                rb[i] = (bk < K && bn < N) ? B[(size_t)bk * N + bn] : 0.0;
+            }
+        };
+        auto store = [&](int buf) {
+#pragma unroll
+            for (int i = 0; i < LA; ++i) {
+                const int idx = tid + i * NT;
+                As[buf][idx / DK][idx % DK] = ra[i];
+            }
+#pragma unroll
+            for (int i = 0; i < LB; ++i) {
+                const int idx = tid + i * NT;
+                Bs[buf][idx / T][idx % T] = rb[i];
+            }
+        };
+        const int KBall = (K + DK - 1) / DK, per = (KBall + S - 1) / S;
+        const int kb0 = S == 1 ? 0 : min(KBall, (int)rank * per), KB = S == 1 ? KBall : min(KBall, kb0 + per);
+        if (KB > kb0) {
+            load(kb0 * DK);
+            store(0);
+        }
+        __syncthreads();
+        for (int kb = kb0; kb < KB; ++kb) {
+            const int cur = S == 1 ? (kb & 1) : ((kb - kb0) & 1);
+            if (kb + 1 < KB) load((kb + 1) * DK);
+#pragma unroll
+            for (int ks = 0; ks < DK; ks += 4) {
+                double a[2], b[2];
+#pragma unroll
+                for (int i = 0; i < 2; ++i) a[i] = As[cur][wm + i * 8 + fr][ks + fk];
+#pragma unroll
+                for (int j = 0; j < 2; ++j) b[j] = Bs[cur][ks + fk][wn + j * 8 + fr];
+#pragma unroll
+                for (int i = 0; i < 2; ++i)
+#pragma unroll
+                    for (int j = 0; j < 2; ++j) dmma(acc[i][j], a[i], b[j]);
+            }
+            if (kb + 1 < KB) store(cur ^ 1);
+            __syncthreads();
+        }
+        if constexpr (S > 1) {
+            if (rank != 0) {
+#pragma unroll
+                for (int e = 0; e < 8; ++e) red[e * NT + tid] = (&acc[0][0][0])[e];
+            }
+            cluster_sync();
+            if (rank == 0) {
+#pragma unroll 1
+                for (uint32_t r = 1; r < (uint32_t)S; ++r) {
+                    uint32_t base;
+                    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;"
+                                 : "=r"(base)
+                                 : "r"((uint32_t)__cvta_generic_to_shared(red)), "r"(r));
+#pragma unroll
+                    for (int e = 0; e < 8; ++e) {
+                        double v;
+                        asm volatile("ld.shared::cluster.f64 %0, [%1];" : "=d"(v) : "r"(base + (uint32_t)((e * NT + tid) * 8)));
+                        (&acc[0][0][0])[e] += v;
+                    }
+                }
+            }
+            cluster_sync();
+            if (rank != 0) continue;
+        }
+        // epilogue: D fragment (row lane / 4, cols 2 (lane % 4) + {0, 1}) of each 8x8 tile
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+            const int r = m0 + wm + i * 8 + fr;
+            if (r >= M) continue;
+#pragma unroll
+            for (int j = 0; j < 2; ++j)
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    const int c = n0 + wn + j * 8 + 2 * fk + h;
+                    if (c >= N) continue;
+                    double* dst = g.C + (size_t)r * N + c;
+                    double o = g.alpha * acc[i][j][h];
+                    if (g.beta != 0.0) o = __fma_rn(g.beta, *dst, o);
+                    *dst = o;
+                }
+        }
+        __syncthreads();  // smem reuse by the next tile
+    }
+}
+
+static cudaError_t launch_cluster(const void* kern, int S, uint32_t grid, int threads, cudaStream_t s,
+                                  const DgemmDesc* descs, int n, uint32_t total) {
+    cudaLaunchConfig_t lc = {};
+    cudaLaunchAttribute attr[1];
+    lc.gridDim = dim3(grid);
+    lc.blockDim = dim3(threads);
+    lc.stream = s;
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = S;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    lc.attrs = attr;
+    lc.numAttrs = S > 1 ? 1 : 0;
+    void* args[] = {(void*)&descs, (void*)&n, (void*)&total};
+    return cudaLaunchKernelExC(&lc, kern, args);
+}
+
 cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total, int grid, bool small, cudaStream_t s) {
     // small tiles: 32-deep k stages (fewer barriers per tile, 255 registers) when all tiles
     // are resident at once at that occupancy -- the Table 1 program with 1-4 VPs (S5: 1 VP
@@ -189,6 +349,38 @@ cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total, int grid
         cudaGetLastError();
         return sms * per;
     }();
+    static const bool dmma_on = !(getenv("SVP_DGEMM_DMMA") && atoi(getenv("SVP_DGEMM_DMMA")) == 0);
+    if (small && dmma_on) {
+        // the DMMA small-tile kernel (32 x 32 tiles like the SIMT small variant), split K on
+        // clusters under the same rule
+        static const int mma_cap = [] {
+            int dev = 0, sms = 0, per = 0;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_dgemm_mma<4>, kMmaThreads, 0);
+            cudaGetLastError();
+            return sms * per;
+        }();
+        static const int mma_per_sm = [] {
+            int per = 0;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_dgemm_mma<1>, kMmaThreads, 0);
+            cudaGetLastError();
+            return std::max(1, per);
+        }();
+        static const bool split_ok = !(getenv("SVP_DGEMM_SPLIT") && atoi(getenv("SVP_DGEMM_SPLIT")) == 0);
+        const int Sm = !split_ok                             ? 1
+                       : total * 4 <= (uint32_t)mma_cap / 2 ? 4
+                       : total * 2 <= (uint32_t)mma_cap     ? 2
+                                                            : 1;
+        if (Sm == 4) return launch_cluster((const void*)k_dgemm_mma<4>, 4, total * 4, kMmaThreads, s, descs, n, total);
+        if (Sm == 2) return launch_cluster((const void*)k_dgemm_mma<2>, 2, total * 2, kMmaThreads, s, descs, n, total);
+        int dev = 0, sms = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        const uint32_t g1 = std::min<uint32_t>(total, (uint32_t)(sms * mma_per_sm));
+        k_dgemm_mma<1><<<g1, kMmaThreads, 0, s>>>(descs, n, total);
+        return cudaGetLastError();
+    }
     // split K when S times the tiles still fit in one wave of the deep small variant
     static const bool split_on = !(getenv("SVP_DGEMM_SPLIT") && atoi(getenv("SVP_DGEMM_SPLIT")) == 0);
     static const int split_cap = [] {
