@@ -683,7 +683,7 @@ static svp_status build_tables(Executor* e, Dev& d, Flush& f, std::vector<uint8_
                 if ((int64_t)j.M * j.N > 0)
                     big += (uint64_t)((j.M + kDgemmBM - 1) / kDgemmBM) * ((j.N + kDgemmBN - 1) / kDgemmBN);
             }
-            ch.small_tiles = big < 2ull * d.lim.num_sms * d.lim.dgemm_blocks_per_sm;
+            ch.small_tiles = dgemm_dmma_enabled() || big < 2ull * d.lim.num_sms * d.lim.dgemm_blocks_per_sm;
             const int TM = ch.small_tiles ? kDgemmSmall : kDgemmBM, TN = ch.small_tiles ? kDgemmSmall : kDgemmBN;
             uint32_t tiles = 0;
             for (size_t k = 0; k < ch.jobs.size(); ++k) {

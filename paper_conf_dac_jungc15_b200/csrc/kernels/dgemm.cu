@@ -336,6 +336,11 @@ static cudaError_t launch_cluster(const void* kern, int S, uint32_t grid, int th
     return cudaLaunchKernelExC(&lc, kern, args);
 }
 
+bool dgemm_dmma_enabled() {
+    static const bool on = !(getenv("SVP_DGEMM_DMMA") && atoi(getenv("SVP_DGEMM_DMMA")) == 0);
+    return on;
+}
+
 cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total, int grid, bool small, cudaStream_t s) {
     // small tiles: 32-deep k stages (fewer barriers per tile, 255 registers) when all tiles
     // are resident at once at that occupancy -- the Table 1 program with 1-4 VPs (S5: 1 VP
@@ -349,8 +354,7 @@ cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total, int grid
         cudaGetLastError();
         return sms * per;
     }();
-    static const bool dmma_on = !(getenv("SVP_DGEMM_DMMA") && atoi(getenv("SVP_DGEMM_DMMA")) == 0);
-    if (small && dmma_on) {
+    if (small && dgemm_dmma_enabled()) {
         // the DMMA small-tile kernel (32 x 32 tiles like the SIMT small variant), split K on
         // clusters under the same rule
         static const int mma_cap = [] {

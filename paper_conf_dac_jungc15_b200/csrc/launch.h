@@ -90,6 +90,9 @@ int sgemm_tc_wide_mode();
 // Grouped fp64 GEMM (the paper's Table 1 matmul), FP64 DFMA with smem tiles; `small`:
 // 32x32 tiles (the table was built with kDgemmSmall tiles).
 cudaError_t launch_dgemm(const DgemmDesc* descs, int n, uint32_t total_tiles, int grid, bool small, cudaStream_t s);
+// the small-tile DGEMM runs on the FP64 tensor cores (DMMA) unless SVP_DGEMM_DMMA=0; the executor
+// then uses the 32 x 32 tiles for every DGEMM launch
+bool dgemm_dmma_enabled();
 cudaError_t query_limits_dgemm(int* per_sm, int* per_sm_small);
 
 // Host: encode the TMA descriptors an SGEMM entry needs (driver entry point fetched at

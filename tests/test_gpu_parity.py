@@ -581,3 +581,17 @@ def test_config5_sgemm_full_elementwise(impl, cfg5_sgemm_oracle):
         assert vs.guards_intact()
     finally:
         ctx.close()
+
+
+def test_dgemm_simt_kernels_in_subprocess():
+    """SVP_DGEMM_DMMA=0 (read once per process): the SIMT DGEMM kernels -- 64 x 64 tiles for big
+    launches, 32 x 32 ones (with split K) for small -- still meet the fp64 contract on the
+    DGEMM parity cases and the Table 1 program."""
+    import os
+    import subprocess
+    import sys
+    here = os.path.dirname(os.path.abspath(__file__))
+    cmd = [sys.executable, "-m", "pytest", os.path.join(here, "test_gpu_parity.py"), "-q", "-m", "gpu",
+           "-p", "no:cacheprovider", "-k", "(dgemm or table1) and not subprocess"]
+    r = subprocess.run(cmd, env={**os.environ, "SVP_DGEMM_DMMA": "0"}, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
