@@ -11,7 +11,7 @@ import re
 import subprocess
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-KEYS = ["UTCHMMA", "UTCQMMA", "UTCBAR", "LDTM", "STTM", "UTMALDG", "UBLKCP", "SYNCS", "FFMA2", "FFMA", "DFMA",
+KEYS = ["UTCHMMA", "UTCQMMA", "UTCBAR", "LDTM", "STTM", "UTMALDG", "UBLKCP", "SYNCS", "FFMA2", "FFMA", "DMMA", "DFMA",
         "ATOMS", "MATCH", "LDG", "STG", "LDS", "STS", "MUFU", "F2FP", "BAR"]
 
 
